@@ -1,0 +1,288 @@
+"""Pins of the CPU oracle against things other than itself (CPU only).
+
+* Fig. 4 message-passing verdicts and Fig. 1's worked trace (tests/golden/).
+* The C1 litmus config: its race set follows from the rules by hand.
+* The §3.2 definition: a brute-force transitive closure (oracle/bf.py).
+  Theorem 1 + Lemmas 1-2 give: every reported pair is unordered
+  (soundness, always), and on granules where the printed atomic rules agree
+  with §3.2 (SURVEY §8(c.4) amb. 3) the first racy access per granule — and
+  so the per-granule verdict — is the same.  Checked on an exhaustive family
+  of tiny traces and on random feasible traces.
+* The FastTrack invariant of §3.4, asserted after every record.
+* 66 re-authored litmus traces (§6.1 categories), expected multisets by hand.
+* Closed forms: race-free-by-construction configs (C2, C3 at reduced size)
+  report nothing; C4 reports exactly its injected races.
+* Infeasible traces are rejected.
+"""
+import itertools
+import json
+import os
+
+import numpy as np
+import pytest
+
+import bcgen
+import oracle
+from bcgen import TraceBuilder, GLOBAL_BASE
+from bcgen.configs import ConfigPlan
+from bcgen.fuzz import random_trace
+from oracle.bf import brute_force, valid_granules
+
+import litmus
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+KIND = {n: i for i, n in enumerate(bcgen.KIND_NAMES)}
+CLS = {n: i for i, n in enumerate(bcgen.CLS_NAMES)}
+
+
+def run(recs, geom, flags=0):
+    st, races, stats = oracle.detect_geom(recs, geom, flags)
+    assert st == 0, st
+    return races
+
+
+def loc_of(r, G=2):
+    sp = int(r["space"])
+    return (sp, int(r["block"]) if sp == 1 else 0, int(r["addr"]) >> G)
+
+
+def check_against_bf(recs, geom, races, strict=True):
+    """Soundness always; first racy event + verdict per valid granule."""
+    G = geom["granule_log2"]
+    bf = brute_force(recs, geom["grid"], geom["block"], G)
+    bfset = bf.race_set()
+    orset = {(loc_of(r, G), int(r["prior_event"]), int(r["cur_event"])) for r in races if r["cls"] != 4}
+    assert orset <= bfset, sorted(orset - bfset)[:5]
+    if not strict:
+        return bf
+    valid = valid_granules(bf)
+    first_bf, first_or = {}, {}
+    for (l, p, c) in bfset:
+        first_bf[l] = min(c, first_bf.get(l, c))
+    for (l, p, c) in orset:
+        first_or[l] = min(c, first_or.get(l, c))
+    for l in valid:
+        assert first_bf.get(l) == first_or.get(l), (l, first_bf.get(l), first_or.get(l))
+    return bf
+
+
+# --------------------------------------------------------------- golden pins
+def test_fig4_message_passing():
+    cases = json.load(open(os.path.join(GOLDEN, "fig4_mp.json")))["cases"]
+    x, y = GLOBAL_BASE, GLOBAL_BASE + 0x100000
+    for c in cases:
+        tb = TraceBuilder(grid=(2,), block=(1,))
+        st_rec = tb.st(0, x)
+        tb.rel(0, y, scope=c["rel"])
+        tb.acq(1, y, scope=c["acq"])
+        ld_rec = tb.ld(1, x)
+        races = run(tb.records(), tb.geom.as_dict())
+        assert len(races) == len(c["races"]), c
+        for r, e in zip(races, c["races"]):
+            assert r["kind"] == KIND[e["kind"]] and r["cls"] == CLS[e["cls"]] and r["space"] == 0
+            assert r["addr"] == x and r["prior_event"] == st_rec << 5 and r["cur_event"] == ld_rec << 5
+        check_against_bf(tb.records(), tb.geom.as_dict(), races)
+
+
+def test_fig1_translation():
+    g = json.load(open(os.path.join(GOLDEN, "fig1.json")))
+    a, b, d = GLOBAL_BASE, GLOBAL_BASE + 0x100, GLOBAL_BASE + 0x200
+    tb = TraceBuilder(block=(2,))
+    tb.ld(0, a); tb.if_(0, [0]); tb.st(0, b); tb.else_(0); tb.fi(0); tb.rel(0, d, scope="blk")
+    recs = tb.records()
+    assert [bcgen.OP_NAMES[o] for o in recs["op"]] == [r["op"] for r in g["records"]]
+    assert list(recs["mask"]) == [3, 3, 1, 1, 2, 3]
+    st, races, stats = oracle.detect_geom(recs, tb.geom.as_dict())
+    assert st == 0 and len(races) == len(g["races"]) == 0
+    # thread ops in Fig. 1(b): 2 rd + 1 wr + 2 relBlk lane events; if/else/fi control
+    assert stats["lane_events"] == 5 and stats["control_events"] == 3
+    check_against_bf(recs, tb.geom.as_dict(), races)
+
+
+def test_c1_litmus():
+    recs, tb = bcgen.configs.make_c1()
+    races = run(recs, tb.geom.as_dict())
+    assert len(races) == 1
+    r = races[0]
+    assert (r["kind"], r["cls"], r["space"]) == (KIND["WW"], CLS["INTER_BLOCK"], 0)
+    assert r["addr"] == GLOBAL_BASE + 0x200000
+    # prior = block 0 lane 5's store, cur = block 1 lane 5's store
+    assert recs[int(r["prior_event"]) >> 5]["warp"] == 0 and int(r["prior_event"]) & 31 == 5
+    assert recs[int(r["cur_event"]) >> 5]["warp"] == 1 and int(r["cur_event"]) & 31 == 5
+    check_against_bf(recs, tb.geom.as_dict(), races)
+    recs2, tb2 = bcgen.configs.make_c1(with_sync=False)
+    races2 = run(recs2, tb2.geom.as_dict())
+    kinds = sorted(int(x["kind"]) for x in races2)
+    assert kinds == [KIND["WW"]] + [KIND["WR"]] * 32
+    check_against_bf(recs2, tb2.geom.as_dict(), races2)
+
+
+# ------------------------------------------------------------- litmus suite
+@pytest.mark.parametrize("entry", litmus.SUITE, ids=[e[0] for e in litmus.SUITE])
+def test_litmus(entry):
+    name, fn, expected, opts = entry
+    tb = fn()
+    recs, geom = tb.records(), tb.geom.as_dict()
+    races = run(recs, geom, oracle.F_CHECK_INVARIANT)
+    got = sorted((int(r["kind"]), int(r["cls"]), int(r["space"])) for r in races)
+    assert got == expected, (name, got, expected)
+    bf = check_against_bf(recs, geom, races, strict=not opts.get("atomic_gap"))
+    if opts.get("atomic_gap"):
+        assert len(bf.race_set()) == 1  # §3.2 has the race the printed rules miss
+    if "overwrite_expected" in opts:
+        races_o = run(recs, geom, oracle.F_RELEASE_OVERWRITE)
+        got_o = sorted((int(r["kind"]), int(r["cls"]), int(r["space"])) for r in races_o)
+        assert got_o == sorted(opts["overwrite_expected"])
+
+
+def test_same_value_filter_flag():
+    tb = TraceBuilder(block=(32,))
+    tb.st(0, lambda l: GLOBAL_BASE if l < 3 else GLOBAL_BASE + 4 * l, same_value=True)
+    assert len(run(tb.records(), tb.geom.as_dict())) == 0
+    races = run(tb.records(), tb.geom.as_dict(), oracle.F_NO_SAME_VALUE_FILTER)
+    assert len(races) == 2 and all(r["cls"] == CLS["SAME_INSN"] for r in races)
+
+
+# ----------------------------------------------------- brute-force property
+@pytest.mark.parametrize("chunk", range(8))
+def test_random_traces_vs_bruteforce(chunk):
+    for seed in range(chunk * 60, chunk * 60 + 60):
+        recs, tb = random_trace(seed)
+        geom = tb.geom.as_dict()
+        st, races, _ = oracle.detect_geom(recs, geom, oracle.F_CHECK_INVARIANT)
+        assert st == 0, (seed, st)
+        check_against_bf(recs, geom, races)
+
+
+def test_random_traces_vector_and_granule():
+    for seed in range(1000, 1060):
+        for G in (0, 3):
+            recs, tb = random_trace(seed, granule_log2=G)
+            geom = tb.geom.as_dict()
+            st, races, _ = oracle.detect_geom(recs, geom, oracle.F_CHECK_INVARIANT)
+            assert st == 0
+            check_against_bf(recs, geom, races)
+
+
+def _alphabet():
+    g0, g1, s = GLOBAL_BASE, GLOBAL_BASE + 4, GLOBAL_BASE + 0x1000
+
+    def addr(pat):
+        return {0: lambda l: g0 if l == 0 else g1, 1: lambda l: g1 if l == 0 else g0,
+                2: lambda l: g0}[pat]
+    ops = [("ld", 0), ("st", 0), ("st", 2), ("atom", 2), ("ld", 1), ("rel", None), ("acq", None),
+           ("br", None)]
+    return ops, addr, s
+
+
+def test_exhaustive_two_warps_two_lanes():
+    """Every program of 2 ops per warp over an 8-op alphabet, for two 2-lane
+    warps in different blocks, under every interleaving of the 4 ops."""
+    ops, addr, s = _alphabet()
+    orders = [o for o in itertools.product([0, 1], repeat=4) if sum(o) == 2]
+    n = 0
+    for p0 in itertools.product(range(len(ops)), repeat=2):
+        for p1 in itertools.product(range(len(ops)), repeat=2):
+            for order in orders:
+                tb = TraceBuilder(grid=(2,), block=(2,))
+                pcs = [0, 0]
+                progs = [p0, p1]
+                for w in order:
+                    kind, pat = ops[progs[w][pcs[w]]]
+                    pcs[w] += 1
+                    if kind == "rel":
+                        tb.rel(w, s)
+                    elif kind == "acq":
+                        tb.acq(w, s)
+                    elif kind == "br":
+                        tb.if_(w, [0]); tb.st(w, addr(0)); tb.else_(w); tb.ld(w, addr(0)); tb.fi(w)
+                    else:
+                        getattr(tb, kind)(w, addr(pat))
+                recs, geom = tb.records(), tb.geom.as_dict()
+                races = run(recs, geom)
+                check_against_bf(recs, geom, races)
+                n += 1
+    assert n == 8 ** 4 * 6
+
+
+# ------------------------------------------------------------ closed forms
+def test_c2_reduced_race_free():
+    plan = ConfigPlan(2, n_blocks=3, iters=3)
+    races = run(plan.records(), plan.geometry)
+    assert len(races) == 0
+
+
+def test_c3_reduced_race_free():
+    plan = ConfigPlan(3, n_blocks=8, iters=2, tpb=64)
+    races = run(plan.records(), plan.geometry)
+    assert len(races) == 0
+
+
+def test_c3_small_vs_bruteforce():
+    plan = ConfigPlan(3, n_blocks=3, iters=1, tpb=32)
+    recs = plan.records()
+    races = run(recs, plan.geometry)
+    assert len(races) == 0
+    bf = brute_force(recs, plan.geometry["grid"], plan.geometry["block"], 2)
+    assert len(bf.race_set()) == 0
+
+
+def test_c4_reduced_exactly_injected():
+    plan = ConfigPlan(4, n_blocks=12, log2_nodes=14, nodes_per_thread=2, inj_scale=4)
+    recs = plan.records()
+    races = run(recs, plan.geometry)
+    truth = plan.truth()
+    assert len(truth) > 0
+    assert np.array_equal(np.sort(races.view("V32")), np.sort(truth.view("V32")))
+
+
+# ---------------------------------------------------------------- infeasible
+def _infeasible_traces():
+    X = GLOBAL_BASE
+    out = []
+    tb = TraceBuilder(block=(32,)); tb.raw(0, 0xFFFF, bcgen.OP_LD, addrs=lambda l: X)  # mask != top
+    out.append(("mask_mismatch", tb))
+    tb = TraceBuilder(block=(32,)); tb.raw(0, 0xFFFFFFFF, bcgen.OP_ELSE)
+    out.append(("else_without_if", tb))
+    tb = TraceBuilder(block=(32,)); tb.if_(0, [0]); tb.raw(0, 1, bcgen.OP_FI)
+    out.append(("fi_without_else", tb))
+    tb = TraceBuilder(block=(64,)); tb.bar(0); tb.ld(0, X)
+    out.append(("record_while_waiting", tb))
+    tb = TraceBuilder(block=(64,)); tb.bar(0)
+    out.append(("incomplete_barrier", tb))
+    tb = TraceBuilder(block=(32,)); tb.ld(0, X + 2)
+    out.append(("misaligned", tb))
+    tb = TraceBuilder(block=(32,), smem_bytes=64); tb.ld(0, lambda l: 4 * l, space=1)
+    out.append(("shared_oob", tb))
+    tb = TraceBuilder(block=(32,)); tb.raw(0, 0xFFFFFFFF, bcgen.OP_IF, aux=0x1_0000_0000 - 1)
+    tb.if_(0, [0]); tb.raw(0, 1, bcgen.OP_IF, aux=2)
+    out.append(("if_aux_outside_mask", tb))
+    tb = TraceBuilder(block=(32,)); tb.if_(0, 0); tb.raw(0, 0, bcgen.OP_LD)
+    out.append(("empty_mask_memory", tb))
+    tb = TraceBuilder(block=(32,))
+    for _ in range(33):
+        tb.if_(0, 0xFFFFFFFF)
+    out.append(("depth_33", tb))
+    tb = TraceBuilder(block=(40,)); tb.raw(1, 0x1FF, bcgen.OP_LD, addrs=lambda l: X)
+    out.append(("lane_beyond_partial_warp", tb))
+    tb = TraceBuilder(block=(32,)); tb.raw(1, 0xFFFFFFFF, bcgen.OP_LD, addrs=lambda l: X)
+    out.append(("warp_out_of_range", tb))
+    return out
+
+
+@pytest.mark.parametrize("case", _infeasible_traces(), ids=lambda c: c[0])
+def test_infeasible_rejected(case):
+    name, tb = case
+    st, races, _ = oracle.detect_geom(tb.records(), tb.geom.as_dict())
+    assert st == oracle.INFEASIBLE, name
+
+
+def test_depth_32_accepted():
+    tb = TraceBuilder(block=(32,))
+    for _ in range(32):
+        tb.if_(0, 0xFFFFFFFF)
+    tb.st(0, lambda l: GLOBAL_BASE + 4 * l)
+    for _ in range(32):
+        tb.else_(0); tb.fi(0)
+    st, races, _ = oracle.detect_geom(tb.records(), tb.geom.as_dict())
+    assert st == 0 and len(races) == 0
