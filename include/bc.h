@@ -1,0 +1,154 @@
+/* bc.h — C ABI of the B200-native BARRACUDA race check.
+ *
+ * What this library computes (PAPER.md = /root/reference/PAPER.md, cited as P:Lnnn):
+ *
+ *   Input  — a *feasible* warp-granular trace of one kernel launch (§3.1) in the
+ *            paper's fixed 272-byte queue record format (§4.2, Fig. 6), in
+ *            global trace order, plus the traced launch geometry.
+ *   Output — the race set the happens-before rules of Fig. 2 / Fig. 3 (§3.3)
+ *            report on that trace: every failed epoch / vector-clock check is one race
+ *            (prior event, current event) on a shadow granule, classified as in P:L1345-1347,
+ *            plus barrier-divergence findings.  The set is bit-identical to the
+ *            plain CPU oracle (oracle/oracle.cpp, test infrastructure) that interprets the
+ *            same rules on uncompressed vector clocks.  Readings of garbled passages are
+ *            listed in DESIGN.md §"Readings" (R1-R15) and are the same on both sides.
+ *
+ * Calls:
+ *   bc_init -> bc_load_trace -> bc_detect -> bc_races -> bc_destroy
+ *
+ * Conventions:
+ *   - One context per process / GPU.  Not thread-safe.  Every call is stream-ordered on
+ *     cfg.stream and returns only after the work it needs has completed.
+ *   - Errors are negative bc_status values; detail text via bc_last_error(ctx).
+ *     Races and barrier-divergence findings are RESULTS, never errors.
+ *   - There is no CPU fallback: bc_init fails with BC_ERR_CUDA if no sm_100 device is usable.
+ */
+#ifndef BC_H_
+#define BC_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---------------------------------------------------------------- status codes */
+typedef enum {
+  BC_OK = 0,
+  BC_ERR_INVALID_ARG = -1,      /* bad geometry / pointer / flag                                */
+  BC_ERR_INFEASIBLE_TRACE = -2, /* trace violates P:L360-366 feasibility or R10 barrier rules   */
+  BC_ERR_OOM = -3,              /* device allocation failed                                     */
+  BC_ERR_CUDA = -4,             /* CUDA runtime error (no device, launch failure, ...)          */
+  BC_ERR_NCCL = -5,             /* multi-GPU communicator error                                 */
+  BC_ERR_STATE = -6,            /* call out of order (e.g. bc_detect before bc_load_trace)      */
+  BC_ERR_TRUNCATED = -7,        /* bc_races: cap < number of races (cap entries were copied)    */
+  BC_ERR_OVERFLOW = -8          /* a 32-bit index space overflowed (records >= 2^27, keys >= 2^30,
+                                   sync-lookup step cap)                 */
+} bc_status;
+
+/* ------------------------------------------------------------- the trace record */
+/* One warp-level instruction ("fields identifying the warp, the operation, a
+ * 32-bit mask of active threads, and 32 entries for the addresses accessed by each thread
+ * in the warp ... a fixed 16 + 8 x 32 = 272 bytes").  Little endian, 8-byte aligned. */
+enum {
+  BC_OP_LD = 0, BC_OP_ST = 1, BC_OP_ATOM = 2,                   /* rd / wr / atm   */
+  BC_OP_ACQ_BLK = 3, BC_OP_ACQ_GLB = 4,                         /* acqBlk / acqGlb               */
+  BC_OP_REL_BLK = 5, BC_OP_REL_GLB = 6,                         /* relBlk / relGlb               */
+  BC_OP_AR_BLK = 7, BC_OP_AR_GLB = 8,                           /* arBlk  / arGlb                */
+  BC_OP_FENCE = 9,                                              /* standalone fence: no-op (R14) */
+  BC_OP_BAR = 10,                                               /* one warp's bar.sync arrival   */
+  BC_OP_IF = 11, BC_OP_ELSE = 12, BC_OP_FI = 13                 /* if(w) else(w) fi(w) P:L290-306 */
+};
+enum { BC_SPACE_GLOBAL = 0, BC_SPACE_SHARED = 1, BC_SPACE_NONE = 2 };
+enum { BC_REC_SAME_VALUE = 1 }; /* all active lanes store one value (reading R6) */
+
+typedef struct bc_record {
+  uint32_t warp;      /* global warp id = block_linear * warps_per_block + warp_in_block        */
+  uint32_t mask;      /* bit i = lane i active; must equal the warp's SIMT-stack top */
+  uint8_t op;         /* BC_OP_*                                                                */
+  uint8_t space;      /* BC_SPACE_GLOBAL | BC_SPACE_SHARED (shared: byte offset in block smem)  */
+  uint8_t size_log2;  /* access width 2^k bytes, k in 0..4; addresses naturally aligned        */
+  uint8_t flags;      /* BC_REC_SAME_VALUE                                                      */
+  uint32_t aux;       /* IF: then-lane mask (else = top & ~aux); otherwise 0                   */
+  uint64_t addr[32];  /* per-lane byte address; inactive lanes ignored                          */
+} bc_record;          /* 272 bytes */
+
+/* ------------------------------------------------------------------ race record */
+enum { BC_KIND_WW = 0, BC_KIND_WR, BC_KIND_RW, BC_KIND_WA, BC_KIND_AW, BC_KIND_RA, BC_KIND_AR,
+       BC_KIND_NONE = 0xFF };                                   /* (prior, current) access type */
+enum { BC_CLS_SAME_INSN = 0,          /* two lanes of one warp instruction         */
+       BC_CLS_BRANCH = 1,             /* same warp, different instruction: branch ordering P:L591-630 */
+       BC_CLS_INTRA_BLOCK = 2, BC_CLS_INTER_BLOCK = 3,
+       BC_CLS_BARRIER_DIVERGENCE = 4 };                         /* finding          */
+
+typedef struct bc_race {
+  uint64_t addr;         /* granule start: global byte address, or byte offset in the block's smem */
+  uint64_t prior_event;  /* (record_index << 5) | lane; ~0 for findings                         */
+  uint64_t cur_event;    /* (record_index << 5) | lane                                          */
+  uint8_t kind, cls, space, pad;
+  uint32_t block;        /* shared: owning block; global: block of the current event; finding: block */
+} bc_race;               /* 32 bytes.  Canonical order: findings, then global races by address,
+                            then shared races by (block, offset); ties by (cur_event, prior_event) */
+
+/* ------------------------------------------------------------------ configuration */
+enum {
+  BC_F_RELEASE_OVERWRITE = 1u,    /* printed S_x := C_t release (reading R1 uses join); not yet
+                                     supported on the GPU path -> BC_ERR_INVALID_ARG            */
+  BC_F_NO_SAME_VALUE_FILTER = 2u  /* report intra-warp same-value WW races too (R6)           */
+};
+
+typedef struct bc_config {
+  uint32_t grid_dim[3], block_dim[3]; /* traced launch geometry; x fastest          */
+  uint32_t warp_size;                 /* must be 32                                 */
+  uint32_t granule_log2;              /* shadow granularity 2^G bytes, G in 0..4  */
+  uint32_t smem_bytes_per_block;      /* shared-memory shadow size per block      */
+  uint32_t flags;                     /* BC_F_*                                                  */
+  int32_t device;                     /* CUDA device ordinal                                     */
+  int32_t rank, world;                /* world = 1 single GPU (multi-GPU: DESIGN.md §"Multi-GPU")*/
+  void* stream;                       /* cudaStream_t (NULL = a stream owned by the context)     */
+} bc_config;
+
+typedef struct bc_stats {
+  uint64_t records, lane_events, control_events; /* SURVEY §8(d.1) units                         */
+  uint64_t items;            /* (granule, lane event) pairs checked after the write-page filter   */
+  uint64_t segments;         /* distinct shadow granules checked                                  */
+  uint64_t races, findings;  /* race records / barrier-divergence findings                       */
+  uint64_t sync_ops;         /* acquire / release lane operations                                 */
+  uint64_t written_pages;    /* 1-MB global pages with at least one write          */
+  float ms_total;            /* device time of bc_detect (cudaEvents on the stream)               */
+  float ms_kernel[12];       /* per phase, see bc_phase_name()                                   */
+} bc_stats;
+
+/* ------------------------------------------------------------------------- calls */
+/* Create a context for one traced launch geometry. */
+bc_status bc_init(const bc_config* cfg, struct bc_ctx** out);
+
+/* Hand the trace to the context.  recs_on_device = 0: `recs` is host memory and is copied
+ * (stream-ordered; the caller keeps ownership).  recs_on_device = 1: `recs` is device memory
+ * on cfg.device, borrowed (not copied) until the next bc_load_trace / bc_destroy; the caller
+ * must keep it alive and unmodified.  n_recs may be 0.  n_recs >= 2^27 -> BC_ERR_OVERFLOW. */
+bc_status bc_load_trace(struct bc_ctx* ctx, const bc_record* recs, uint64_t n_recs, int recs_on_device);
+
+/* Run the race check on the loaded trace (all kernels on cfg.stream) and synchronize.
+ * Infeasible trace -> BC_ERR_INFEASIBLE_TRACE (no races are kept).  `out` may be NULL.
+ * Repeated calls on the same trace are idempotent. */
+bc_status bc_detect(struct bc_ctx* ctx, bc_stats* out);
+
+/* Copy the canonical race list (findings first) into host memory.  out == NULL: only
+ * *n_total is written.  cap < *n_total: cap records are copied and BC_ERR_TRUNCATED returned. */
+bc_status bc_races(struct bc_ctx* ctx, bc_race* out, uint64_t cap, uint64_t* n_total);
+
+/* Same, into device memory (`out` is a device pointer on cfg.device). */
+bc_status bc_races_device(struct bc_ctx* ctx, bc_race* out_dev, uint64_t cap, uint64_t* n_total);
+
+void bc_destroy(struct bc_ctx* ctx);
+
+const char* bc_status_string(bc_status s);
+const char* bc_last_error(const struct bc_ctx* ctx);
+const char* bc_phase_name(int i); /* names of bc_stats.ms_kernel[i]; NULL past the end */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BC_H_ */

@@ -1,0 +1,225 @@
+"""paper_conf_pldi_eizenbergppmd17_b200 — B200-native BARRACUDA race check (PLDI'17).
+
+Thin Python binding over the C ABI in include/bc.h (lib/libbc.so, sm_100a kernels).
+Argument marshalling only: every step of the race check runs in the CUDA kernels of
+csrc/.  There is no CPU fallback: if the extension is missing, importing the binding
+functions raises.  PyTorch provides device memory (borrowed device traces, device race
+buffers) and streams.
+
+Calls mirror the boundary:
+
+    ctx = Context(geometry, device=0)      # bc_init
+    ctx.load_trace(records)                # bc_load_trace  (numpy host array or torch CUDA uint8 tensor)
+    stats = ctx.detect()                   # bc_detect
+    races = ctx.races()                    # bc_races  -> numpy array of RACE_DTYPE
+    ctx.close()                            # bc_destroy
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "lib", "libbc.so")
+
+RECORD_BYTES = 272
+RACE_DTYPE = np.dtype([
+    ("addr", "<u8"), ("prior_event", "<u8"), ("cur_event", "<u8"),
+    ("kind", "u1"), ("cls", "u1"), ("space", "u1"), ("pad", "u1"), ("block", "<u4"),
+])
+
+OK = 0
+STATUS = {0: "OK", -1: "INVALID_ARG", -2: "INFEASIBLE_TRACE", -3: "OOM", -4: "CUDA", -5: "NCCL",
+          -6: "STATE", -7: "TRUNCATED", -8: "OVERFLOW"}
+F_RELEASE_OVERWRITE = 1
+F_NO_SAME_VALUE_FILTER = 2
+
+EXPORTS = ["bc_init", "bc_load_trace", "bc_detect", "bc_races", "bc_races_device", "bc_destroy",
+           "bc_status_string", "bc_last_error", "bc_phase_name"]
+
+
+class BcError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class _Config(ctypes.Structure):
+    _fields_ = [("grid_dim", ctypes.c_uint32 * 3), ("block_dim", ctypes.c_uint32 * 3),
+                ("warp_size", ctypes.c_uint32), ("granule_log2", ctypes.c_uint32),
+                ("smem_bytes_per_block", ctypes.c_uint32), ("flags", ctypes.c_uint32),
+                ("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("stream", ctypes.c_void_p)]
+
+
+class _Stats(ctypes.Structure):
+    _fields_ = [("records", ctypes.c_uint64), ("lane_events", ctypes.c_uint64),
+                ("control_events", ctypes.c_uint64), ("items", ctypes.c_uint64),
+                ("segments", ctypes.c_uint64), ("races", ctypes.c_uint64), ("findings", ctypes.c_uint64),
+                ("sync_ops", ctypes.c_uint64), ("written_pages", ctypes.c_uint64),
+                ("ms_total", ctypes.c_float), ("ms_kernel", ctypes.c_float * 12)]
+
+
+_lib = None
+
+
+def lib():
+    """Load lib/libbc.so (fails loudly when the CUDA extension has not been built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} missing: build it with `python __graft_entry__.py` "
+                              "(there is no CPU fallback)")
+        L = ctypes.CDLL(LIB_PATH)
+        L.bc_init.restype = ctypes.c_int
+        L.bc_init.argtypes = [ctypes.POINTER(_Config), ctypes.POINTER(ctypes.c_void_p)]
+        L.bc_load_trace.restype = ctypes.c_int
+        L.bc_load_trace.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int]
+        L.bc_detect.restype = ctypes.c_int
+        L.bc_detect.argtypes = [ctypes.c_void_p, ctypes.POINTER(_Stats)]
+        L.bc_races.restype = ctypes.c_int
+        L.bc_races.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64)]
+        L.bc_races_device.restype = ctypes.c_int
+        L.bc_races_device.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                      ctypes.POINTER(ctypes.c_uint64)]
+        L.bc_destroy.argtypes = [ctypes.c_void_p]
+        L.bc_status_string.restype = ctypes.c_char_p
+        L.bc_status_string.argtypes = [ctypes.c_int]
+        L.bc_last_error.restype = ctypes.c_char_p
+        L.bc_last_error.argtypes = [ctypes.c_void_p]
+        L.bc_phase_name.restype = ctypes.c_char_p
+        L.bc_phase_name.argtypes = [ctypes.c_int]
+        _lib = L
+    return _lib
+
+
+def phase_names():
+    L = lib()
+    out, i = [], 0
+    while True:
+        p = L.bc_phase_name(i)
+        if not p:
+            return out
+        out.append(p.decode())
+        i += 1
+
+
+def _stats_dict(s: _Stats):
+    d = {k: getattr(s, k) for k, _ in _Stats._fields_ if k != "ms_kernel"}
+    d["ms_kernel"] = dict(zip(phase_names(), list(s.ms_kernel)))
+    return d
+
+
+class Context:
+    """One traced launch geometry on one GPU (bc_init ... bc_destroy)."""
+
+    def __init__(self, geometry: dict, device: int = 0, flags: int = 0, stream=None):
+        L = lib()
+        grid = tuple(geometry["grid"]) + (1,) * (3 - len(geometry["grid"]))
+        block = tuple(geometry["block"]) + (1,) * (3 - len(geometry["block"]))
+        c = _Config()
+        for i in range(3):
+            c.grid_dim[i], c.block_dim[i] = grid[i], block[i]
+        c.warp_size = 32
+        c.granule_log2 = geometry.get("granule_log2", 2)
+        c.smem_bytes_per_block = geometry.get("smem_bytes", 0)
+        c.flags = flags
+        c.device = device
+        c.rank, c.world = 0, 1
+        c.stream = stream
+        h = ctypes.c_void_p()
+        st = L.bc_init(ctypes.byref(c), ctypes.byref(h))
+        if st != OK:
+            raise BcError(st, L.bc_status_string(st).decode())
+        self._h = h
+        self._keep = None
+        self.device = device
+
+    def _check(self, st, allow=()):
+        if st != OK and st not in allow:
+            L = lib()
+            raise BcError(st, f"{L.bc_status_string(st).decode()} ({L.bc_last_error(self._h).decode()})")
+        return st
+
+    def load_trace(self, records):
+        """records: numpy RECORD_DTYPE array / bytes-like on the host (copied), or a CUDA tensor
+        of n*272 bytes (borrowed until the next load_trace / close)."""
+        L = lib()
+        if hasattr(records, "is_cuda") and records.is_cuda:
+            n = records.numel() * records.element_size() // RECORD_BYTES
+            self._keep = records
+            return self._check(L.bc_load_trace(self._h, ctypes.c_void_p(records.data_ptr()), n, 1))
+        if hasattr(records, "data_ptr"):  # pinned / host torch tensor
+            n = records.numel() * records.element_size() // RECORD_BYTES
+            self._keep = records
+            return self._check(L.bc_load_trace(self._h, ctypes.c_void_p(records.data_ptr()), n, 0))
+        a = np.ascontiguousarray(records)
+        n = a.nbytes // RECORD_BYTES
+        self._keep = a
+        return self._check(L.bc_load_trace(self._h, ctypes.c_void_p(a.ctypes.data if n else 0), n, 0))
+
+    def detect(self, allow=()):
+        """bc_detect; returns (status, stats dict)."""
+        s = _Stats()
+        st = self._check(lib().bc_detect(self._h, ctypes.byref(s)), allow)
+        return st, _stats_dict(s)
+
+    def num_races(self):
+        n = ctypes.c_uint64()
+        self._check(lib().bc_races(self._h, None, 0, ctypes.byref(n)))
+        return int(n.value)
+
+    def races(self):
+        n = self.num_races()
+        out = np.zeros(n, dtype=RACE_DTYPE)
+        if n:
+            tot = ctypes.c_uint64()
+            self._check(lib().bc_races(self._h, ctypes.c_void_p(out.ctypes.data), n, ctypes.byref(tot)))
+        return out
+
+    def races_device(self, out_tensor):
+        """Copy races into a CUDA uint8 tensor of >= n*32 bytes; returns n."""
+        n = self.num_races()
+        tot = ctypes.c_uint64()
+        cap = out_tensor.numel() * out_tensor.element_size() // 32
+        self._check(lib().bc_races_device(self._h, ctypes.c_void_p(out_tensor.data_ptr()), cap,
+                                          ctypes.byref(tot)), allow=(-7,))
+        return n
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().bc_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+@dataclass
+class Result:
+    status: int
+    races: np.ndarray
+    stats: dict
+
+
+def detect(records, geometry: dict, device="cuda:0", flags: int = 0, stream=None) -> Result:
+    """One-shot bc_init/bc_load_trace/bc_detect/bc_races.  Infeasible traces return
+    status -2 with no races (as the oracle does)."""
+    dev = int(str(device).split(":")[-1]) if str(device).startswith("cuda") else int(device)
+    with Context(geometry, device=dev, flags=flags, stream=stream) as ctx:
+        ctx.load_trace(records)
+        st, stats = ctx.detect(allow=(-2,))
+        races = ctx.races() if st == OK else np.zeros(0, dtype=RACE_DTYPE)
+        return Result(st, races, stats)

@@ -1,0 +1,410 @@
+// api.cu — the C ABI of include/bc.h: context, trace ownership and the bc_detect pipeline.
+//
+//   bc_detect = header (a1/a2) -> K1 warp partition (radix sort) -> K2 replay (a3) -> barrier
+//               labels -> K3 sync skeleton (a4) -> K4 expansion (a5) -> K5 radix sort (a6)
+//               -> K7 shadow check (a7) -> K8 finalize (a8/a9)
+// all on cfg.stream; every phase is bracketed by cudaEvents for bc_stats.ms_kernel.
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "common.cuh"
+#include "kernels.cuh"
+
+using namespace bc;
+
+struct bc_ctx {
+  bc_config cfg;
+  Geo g;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  const bc_record* trace = nullptr;  // device
+  bc_record* owned = nullptr;
+  size_t owned_cap = 0;
+  u64 n_recs = 0;
+  bool loaded = false;
+  bool detected = false;
+  bc_race* races = nullptr;  // device, findings first
+  size_t races_cap = 0;
+  u64 n_races = 0;
+  bc_stats stats{};
+  std::string err;
+  cudaEvent_t ev[16] = {};
+};
+
+static const char* kPhase[] = {"header", "partition", "replay", "sync", "expand", "sort", "check", "finalize",
+                               nullptr};
+enum { PH_HEADER = 0, PH_PARTITION, PH_REPLAY, PH_SYNC, PH_EXPAND, PH_SORT, PH_CHECK, PH_FINALIZE, PH_N };
+
+static bc_status fail(bc_ctx* c, bc_status s, const std::string& msg) {
+  if (c) c->err = msg;
+  return s;
+}
+
+static bc_status cuda_check(bc_ctx* c, const char* where) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(c, BC_ERR_CUDA, std::string(where) + ": " + cudaGetErrorString(e));
+  return BC_OK;
+}
+
+static int bits_for(u64 maxval) {
+  int b = 0;
+  while (b < 64 && (maxval >> b)) ++b;
+  return b;
+}
+
+extern "C" {
+
+const char* bc_status_string(bc_status s) {
+  switch (s) {
+    case BC_OK: return "ok";
+    case BC_ERR_INVALID_ARG: return "invalid argument";
+    case BC_ERR_INFEASIBLE_TRACE: return "infeasible trace";
+    case BC_ERR_OOM: return "out of device memory";
+    case BC_ERR_CUDA: return "CUDA error";
+    case BC_ERR_NCCL: return "NCCL error";
+    case BC_ERR_STATE: return "call out of order";
+    case BC_ERR_TRUNCATED: return "output truncated";
+    case BC_ERR_OVERFLOW: return "32-bit index overflow";
+  }
+  return "unknown status";
+}
+
+const char* bc_last_error(const bc_ctx* c) { return c ? c->err.c_str() : "null context"; }
+
+const char* bc_phase_name(int i) { return (i >= 0 && i < PH_N) ? kPhase[i] : nullptr; }
+
+bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
+  if (!cfg || !out) return BC_ERR_INVALID_ARG;
+  *out = nullptr;
+  if (cfg->warp_size != 32 || cfg->granule_log2 > 4) return BC_ERR_INVALID_ARG;
+  if (cfg->flags & ~(u32)(BC_F_NO_SAME_VALUE_FILTER)) return BC_ERR_INVALID_ARG;  // overwrite: not on GPU yet
+  if (cfg->world != 1 && cfg->world != 0) return BC_ERR_INVALID_ARG;
+  u64 nb = (u64)cfg->grid_dim[0] * cfg->grid_dim[1] * cfg->grid_dim[2];
+  u64 tpb = (u64)cfg->block_dim[0] * cfg->block_dim[1] * cfg->block_dim[2];
+  if (nb == 0 || tpb == 0 || tpb > 1024 || nb * tpb > 0xFFFFFFFFull) return BC_ERR_INVALID_ARG;
+  u64 wpb = (tpb + 31) / 32;
+  if (nb * wpb >= (1ull << 30)) return BC_ERR_INVALID_ARG;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return BC_ERR_CUDA;
+  }
+  if (cfg->device < 0 || cfg->device >= ndev) return BC_ERR_INVALID_ARG;
+  if (cudaSetDevice(cfg->device) != cudaSuccess) return BC_ERR_CUDA;
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, cfg->device) != cudaSuccess || prop.major < 10) return BC_ERR_CUDA;
+  bc_ctx* c = new bc_ctx();
+  c->cfg = *cfg;
+  Geo& g = c->g;
+  g.n_blocks = (u32)nb;
+  g.tpb = (u32)tpb;
+  g.wpb = (u32)wpb;
+  g.n_warps = (u32)(nb * wpb);
+  g.G = cfg->granule_log2;
+  g.smem = cfg->smem_bytes_per_block;
+  g.smem_gran = (u32)(((u64)g.smem + (1u << g.G) - 1) >> g.G);
+  g.flags = cfg->flags;
+  g.n_recs = 0;
+  if (cfg->stream) {
+    c->stream = (cudaStream_t)cfg->stream;
+  } else {
+    cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking);
+    c->own_stream = true;
+  }
+  // keep pooled scratch memory cached between bc_detect calls
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, cfg->device) == cudaSuccess) {
+    uint64_t thr = ~0ull;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  for (int i = 0; i < 16; ++i) cudaEventCreate(&c->ev[i]);
+  if (cudaGetLastError() != cudaSuccess) {
+    bc_destroy(c);
+    return BC_ERR_CUDA;
+  }
+  *out = c;
+  return BC_OK;
+}
+
+void bc_destroy(bc_ctx* c) {
+  if (!c) return;
+  cudaSetDevice(c->cfg.device);
+  if (c->stream) cudaStreamSynchronize(c->stream);
+  if (c->owned) cudaFree(c->owned);
+  if (c->races) cudaFree(c->races);
+  for (int i = 0; i < 16; ++i)
+    if (c->ev[i]) cudaEventDestroy(c->ev[i]);
+  if (c->own_stream) cudaStreamDestroy(c->stream);
+  delete c;
+}
+
+bc_status bc_load_trace(bc_ctx* c, const bc_record* recs, uint64_t n, int on_device) {
+  if (!c) return BC_ERR_INVALID_ARG;
+  if (n && !recs) return fail(c, BC_ERR_INVALID_ARG, "null trace");
+  if (n >= (1ull << 27)) return fail(c, BC_ERR_OVERFLOW, "more than 2^27 records (event id = rec << 5 | lane)");
+  cudaSetDevice(c->cfg.device);
+  c->loaded = false;
+  c->detected = false;
+  c->n_recs = n;
+  c->g.n_recs = n;
+  bool aligned = ((uintptr_t)recs & 15) == 0;
+  if (n == 0) {
+    c->trace = nullptr;
+  } else if (on_device && aligned) {
+    c->trace = recs;
+  } else {
+    size_t bytes = n * sizeof(bc_record);
+    if (bytes > c->owned_cap) {
+      if (c->owned) cudaFree(c->owned);
+      c->owned = nullptr;
+      c->owned_cap = 0;
+      if (cudaMalloc(&c->owned, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(c, BC_ERR_OOM, "trace buffer");
+      }
+      c->owned_cap = bytes;
+    }
+    cudaMemcpyAsync(c->owned, recs, bytes, on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
+                    c->stream);
+    if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_check(c, "trace copy");
+    c->trace = c->owned;
+  }
+  c->loaded = true;
+  return BC_OK;
+}
+
+static bc_status detect_impl(bc_ctx* c, Scratch& S) {
+  cudaStream_t st = c->stream;
+  Geo g = c->g;
+  const u64 n = g.n_recs;
+  const bc_record* recs = c->trace;
+  bc_stats& sx = c->stats;
+  memset(&sx, 0, sizeof(sx));
+  sx.records = n;
+  c->n_races = 0;
+  cudaEventRecord(c->ev[0], st);
+  if (n == 0) {
+    cudaEventRecord(c->ev[PH_N], st);
+    cudaEventSynchronize(c->ev[PH_N]);
+    cudaEventElapsedTime(&sx.ms_total, c->ev[0], c->ev[PH_N]);
+    return BC_OK;
+  }
+  const u64 nwords = 1ull << 23;  // page bitmap: 2^28 1-MB pages (48-bit addresses)
+  u32* err = S.alloc<u32>(1);
+  u64* cnt = S.alloc<u64>(C_N);
+  u32* wkey = S.alloc<u32>(n);
+  u32* wval = S.alloc<u32>(n);
+  u32* if_cnt = S.alloc<u32>(g.n_warps + 1);
+  u32* bar_cnt = S.alloc<u32>(g.n_warps + 1);
+  u32* sync_list = S.alloc<u32>(n);
+  u32* page_bits = S.alloc<u32>(nwords);
+  cudaMemsetAsync(err, 0, 4, st);
+  cudaMemsetAsync(cnt, 0, C_N * 8, st);
+  cudaMemsetAsync(if_cnt, 0, (g.n_warps + 1) * 4, st);
+  cudaMemsetAsync(bar_cnt, 0, (g.n_warps + 1) * 4, st);
+  cudaMemsetAsync(page_bits, 0, nwords * 4, st);
+  // ---- header pass
+  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt, err, st);
+  u32* page_rank = S.alloc<u32>(nwords);
+  u64* tot = S.alloc<u64>(4);
+  launch_popc(page_bits, page_rank, nwords, st);
+  exclusive_scan_u32(page_rank, page_rank, nwords, S.alloc<char>(scan_temp_bytes(nwords)), tot + 0, st);
+  cudaEventRecord(c->ev[1], st);
+  u64 hc_cnt[C_N];
+  u32 herr = 0;
+  u64 n_pages = 0;
+  cudaMemcpyAsync(hc_cnt, cnt, sizeof(hc_cnt), cudaMemcpyDeviceToHost, st);
+  cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
+  cudaMemcpyAsync(&n_pages, tot, 8, cudaMemcpyDeviceToHost, st);
+  if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "header");
+  sx.lane_events = hc_cnt[C_LANE_EVENTS];
+  sx.control_events = hc_cnt[C_CONTROL_EVENTS];
+  sx.sync_ops = hc_cnt[C_SYNC_LANEOPS];
+  sx.written_pages = n_pages;
+  if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "record header violates feasibility");
+  if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "global address >= 2^48");
+  const u32 shared_base = (u32)std::min<u64>(n_pages << (20 - g.G), 0xFFFFFFFFull);
+  const u64 n_keys = (n_pages << (20 - g.G)) + (u64)g.n_blocks * g.smem_gran;
+  if (n_keys >= (1ull << 30)) return fail(c, BC_ERR_OVERFLOW, "shadow key space >= 2^30 granules");
+
+  // ---- K1: records grouped by warp (stable -> trace order within a warp)
+  u32* wk2 = S.alloc<u32>(n);
+  u32* wv2 = S.alloc<u32>(n);
+  bool alt = radix_sort_pairs(wkey, wval, wk2, wv2, n, 0, bits_for(g.n_warps - 1), S.alloc<char>(rs_temp_bytes(n)), st);
+  u32* skeys = alt ? wk2 : wkey;
+  u32* wrec = alt ? wv2 : wval;
+  u32* warp_start = S.alloc<u32>(g.n_warps + 1);
+  launch_warp_start(skeys, n, g.n_warps, warp_start, st);
+  const u64 n_if = hc_cnt[C_IFS], n_bar = hc_cnt[C_BARS];
+  u32* node_base = S.alloc<u32>(g.n_warps + 1);
+  u32* bar_base = S.alloc<u32>(g.n_warps + 1);
+  exclusive_scan_u32(if_cnt, node_base, g.n_warps, S.alloc<char>(scan_temp_bytes(g.n_warps)), nullptr, st);
+  launch_node_base(node_base, g.n_warps, node_base, st);
+  exclusive_scan_u32(bar_cnt, bar_base, g.n_warps, S.alloc<char>(scan_temp_bytes(g.n_warps)), nullptr, st);
+  cudaEventRecord(c->ev[2], st);
+  // ---- K2: clock replay
+  const u64 n_nodes = g.n_warps + 2 * n_if;
+  uint4* snap = S.alloc<uint4>(n);
+  uint4* nodes = S.alloc<uint4>(n_nodes);
+  u32* bar_rec = S.alloc<u32>(n_bar + 1);
+  u32* bar_next = S.alloc<u32>(n_bar + 1);
+  u32* blockR = S.alloc<u32>(n_bar + 1);
+  u32* find_blk = S.alloc<u32>(n_bar + 1);
+  u32* find_rec = S.alloc<u32>(n_bar + 1);
+  u32* find_cnt = S.alloc<u32>(1);
+  cudaMemsetAsync(find_cnt, 0, 4, st);
+  launch_replay(recs, wrec, warp_start, g, node_base, bar_base, snap, nodes, bar_rec, bar_next, find_blk, find_rec,
+                find_cnt, err, st);
+  launch_barriers(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err, st);
+  cudaEventRecord(c->ev[3], st);
+  bc_status cs = cuda_check(c, "replay");
+  if (cs) return cs;
+
+  HbCtx hc{};
+  hc.g = g;
+  hc.snap = snap;
+  hc.nodes = nodes;
+  hc.bar_base = bar_base;
+  hc.blockR = blockR;
+  hc.err = err;
+  hc.n_acq = 0;
+  hc.n_idx = 0;
+  // ---- K3: sync skeleton
+  if (hc_cnt[C_SYNC_RECS]) {
+    u64 ne = 0;
+    int rs = run_sync_skeleton(recs, sync_list, (u32)hc_cnt[C_SYNC_RECS], (u32)hc_cnt[C_SYNC_LANEOPS], hc, S, st, &ne);
+    if (rs) return fail(c, (bc_status)rs, "sync skeleton");
+  }
+  cudaEventRecord(c->ev[4], st);
+  // ---- K4: expansion
+  const u64 bound = hc_cnt[C_ITEM_BOUND];
+  u32* ikeys = S.alloc<u32>(bound + 1);
+  u32* ievs = S.alloc<u32>(bound + 1);
+  u64 tiles = expand_tiles(n);
+  u64* estatus = S.alloc<u64>(tiles + 1);
+  u32* ecounter = S.alloc<u32>(1);
+  cudaMemsetAsync(estatus, 0, (tiles + 1) * 8, st);
+  cudaMemsetAsync(ecounter, 0, 4, st);
+  launch_expand(recs, g, page_bits, page_rank, shared_base, ikeys, ievs, estatus, ecounter, cnt, err, st);
+  u64 n_items = 0;
+  u32 nfind = 0;
+  cudaMemcpyAsync(&n_items, cnt + C_ITEMS, 8, cudaMemcpyDeviceToHost, st);
+  cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
+  cudaMemcpyAsync(&nfind, find_cnt, 4, cudaMemcpyDeviceToHost, st);
+  cudaEventRecord(c->ev[5], st);
+  if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "expand");
+  if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "infeasible trace");
+  if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "index overflow");
+  sx.items = n_items;
+  // ---- K5: stable radix sort by granule key
+  u32* ik2 = S.alloc<u32>(n_items + 1);
+  u32* iv2 = S.alloc<u32>(n_items + 1);
+  int kbits = bits_for(n_keys ? n_keys - 1 : 0);
+  alt = radix_sort_pairs(ikeys, ievs, ik2, iv2, n_items, 2, 2 + kbits, S.alloc<char>(rs_temp_bytes(n_items)), st);
+  u32* skey = alt ? ik2 : ikeys;
+  u32* sev = alt ? iv2 : ievs;
+  cudaEventRecord(c->ev[6], st);
+  // ---- K7: shadow check
+  u32 race_cap = (u32)std::min<u64>(std::max<u64>(1u << 16, n_items / 16), 1u << 30);
+  uint4* rbuf = nullptr;
+  u32* rcnt = S.alloc<u32>(1);
+  u64* segc = S.alloc<u64>(1);
+  void* cstatus = S.alloc<char>(check_status_bytes(n_items));
+  u32* ccounter = S.alloc<u32>(1);
+  u32 n_r = 0;
+  for (int attempt = 0; attempt < 2; ++attempt) {
+    rbuf = S.alloc<uint4>(race_cap);
+    cudaMemsetAsync(rcnt, 0, 4, st);
+    cudaMemsetAsync(segc, 0, 8, st);
+    cudaMemsetAsync(err, 0, 4, st);
+    launch_check(hc, skey, sev, n_items, cstatus, ccounter, rbuf, rcnt, race_cap, segc, st);
+    cudaMemcpyAsync(&n_r, rcnt, 4, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(&sx.segments, segc, 8, cudaMemcpyDeviceToHost, st);
+    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "check");
+    if (n_r <= race_cap) break;
+    race_cap = n_r;
+  }
+  if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "sync lookup step cap");
+  cudaEventRecord(c->ev[7], st);
+  // ---- K8: finalize
+  u64 total = (u64)n_r + nfind;
+  if (total > c->races_cap) {
+    if (c->races) cudaFree(c->races);
+    c->races = nullptr;
+    c->races_cap = 0;
+    if (cudaMalloc(&c->races, std::max<u64>(total, 1) * sizeof(bc_race)) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(c, BC_ERR_OOM, "race buffer");
+    }
+    c->races_cap = std::max<u64>(total, 1);
+  }
+  u32* page_num = S.alloc<u32>(n_pages + 1);
+  if (n_r) launch_page_list(page_bits, page_rank, nwords, page_num, st);
+  finalize_races(rbuf, n_r, find_blk, find_rec, nfind, g, snap, page_num, shared_base, (u32)n_keys, c->races, S, st);
+  cudaEventRecord(c->ev[PH_N], st);
+  if (cudaEventSynchronize(c->ev[PH_N]) != cudaSuccess) return cuda_check(c, "finalize");
+  cs = cuda_check(c, "detect");
+  if (cs) return cs;
+  c->n_races = total;
+  sx.races = n_r;
+  sx.findings = nfind;
+  cudaEventElapsedTime(&sx.ms_total, c->ev[0], c->ev[PH_N]);
+  for (int i = 0; i < PH_N; ++i) {
+    cudaEvent_t e1 = i + 1 < PH_N ? c->ev[i + 1] : c->ev[PH_N];
+    cudaEventElapsedTime(&sx.ms_kernel[i], c->ev[i], e1);
+  }
+  return BC_OK;
+}
+
+bc_status bc_detect(bc_ctx* c, bc_stats* out) {
+  if (!c) return BC_ERR_INVALID_ARG;
+  if (!c->loaded) return fail(c, BC_ERR_STATE, "bc_detect before bc_load_trace");
+  cudaSetDevice(c->cfg.device);
+  c->detected = false;
+  c->err.clear();
+  bc_status s;
+  {
+    Scratch S(c->stream);
+    try {
+      s = detect_impl(c, S);
+    } catch (const std::bad_alloc&) {
+      s = fail(c, BC_ERR_OOM, "scratch allocation");
+    }
+    S.release();
+  }
+  cudaStreamSynchronize(c->stream);
+  if (s == BC_OK) {
+    c->detected = true;
+  } else {
+    c->n_races = 0;
+  }
+  if (out) *out = c->stats;
+  return s;
+}
+
+static bc_status races_copy(bc_ctx* c, bc_race* out, uint64_t cap, uint64_t* n_total, cudaMemcpyKind kind) {
+  if (!c || !n_total) return BC_ERR_INVALID_ARG;
+  if (!c->detected) return fail(c, BC_ERR_STATE, "bc_races before a successful bc_detect");
+  *n_total = c->n_races;
+  if (!out) return BC_OK;
+  u64 k = std::min<u64>(cap, c->n_races);
+  if (k) {
+    cudaSetDevice(c->cfg.device);
+    cudaMemcpyAsync(out, c->races, k * sizeof(bc_race), kind, c->stream);
+    if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_check(c, "race copy");
+  }
+  return k < c->n_races ? BC_ERR_TRUNCATED : BC_OK;
+}
+
+bc_status bc_races(bc_ctx* c, bc_race* out, uint64_t cap, uint64_t* n_total) {
+  return races_copy(c, out, cap, n_total, cudaMemcpyDeviceToHost);
+}
+
+bc_status bc_races_device(bc_ctx* c, bc_race* out, uint64_t cap, uint64_t* n_total) {
+  return races_copy(c, out, cap, n_total, cudaMemcpyDeviceToDevice);
+}
+
+}  // extern "C"

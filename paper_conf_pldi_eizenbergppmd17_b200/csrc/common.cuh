@@ -1,0 +1,287 @@
+// common.cuh — device-side types and helpers shared by the sm_100a kernels of libbc.
+//
+// Nothing here is shared with the oracle (oracle/oracle.cpp); see DESIGN.md "Parity".
+//
+// Clock representation (DESIGN.md §"Record-index clocks"): every step of a thread (an
+// endi / if / else / fi / bar join-fork) is labelled with
+// (trace record index + 1).  The labels along one thread's timeline are strictly increasing,
+// so "t knows u's step labelled L" is a lossless stand-in for the paper's epoch comparison
+// c@u ⪯ C_t: the access of u in record r1 happened before t's current point iff
+// know_t(u) >= r1 + 1.  know_t(u) is never materialised as a vector; it is evaluated from
+//   - the barrier label of t's block phase (§4.3.2 block max),
+//   - the warp's SIMT-stack node chain (the PTVC warp part, Fig. 7),
+//   - foreign knowledge through acquire/release views (the SPARSEVC part).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "bc.h"
+
+namespace bc {
+
+typedef uint32_t u32;
+typedef uint64_t u64;
+
+constexpr u32 NONE = 0xFFFFFFFFu;
+constexpr int WARP = 32;
+
+// error flags (device word) -> bc_status
+constexpr u32 ERR_INFEASIBLE = 1u;
+constexpr u32 ERR_OVERFLOW = 2u;
+
+// item op codes (2 low bits of an item's key word)
+constexpr u32 IOP_LD = 0, IOP_ST = 1, IOP_ST_SV = 2, IOP_ATOM = 3;
+
+// sync-index key space (K3)
+constexpr u32 KEY_BLOCK = 0x80000000u;  // block-level entry: key = KEY_BLOCK | block
+constexpr u32 KEY_LINK = 0xC0000000u;   // link entry:        key = KEY_LINK | target array
+constexpr u32 SYNC_LOOKUP_CAP = 4096;   // step cap of one foreign lookup
+
+struct Geo {
+  u32 n_blocks, tpb, wpb, n_warps;
+  u32 G;           // granule_log2
+  u32 smem;        // bytes per block
+  u32 smem_gran;   // granules per block
+  u32 flags;
+  u64 n_recs;
+};
+
+__host__ __device__ inline u32 init_mask(const Geo& g, u32 w) {
+  u32 wib = w % g.wpb;
+  u32 lanes = g.tpb - wib * 32u;
+  return lanes >= 32u ? 0xFFFFFFFFu : ((1u << lanes) - 1u);
+}
+
+// 16-byte record header as loaded from the 272-byte record
+struct Hdr {
+  u32 warp, mask, aux;
+  u32 op, space, size_log2, flags;
+};
+__device__ __forceinline__ Hdr load_hdr(const bc_record* recs, u64 r) {
+  uint4 v = __ldg(reinterpret_cast<const uint4*>(recs + r));
+  Hdr h;
+  h.warp = v.x;
+  h.mask = v.y;
+  h.op = v.z & 0xFFu;
+  h.space = (v.z >> 8) & 0xFFu;
+  h.size_log2 = (v.z >> 16) & 0xFFu;
+  h.flags = (v.z >> 24) & 0xFFu;
+  h.aux = v.w;
+  return h;
+}
+
+__device__ __forceinline__ void set_err(u32* err, u32 bits) { atomicOr(err, bits); }
+
+__device__ __forceinline__ u32 lanemask_lt() {
+  u32 m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+// ---------------------------------------------------------------- per-record snapshot
+// K2 output, one per record (16 B): the compressed clock of the record's active lanes.
+//   warp  : traced warp id
+//   ps    : label of the warp's last step before this record (0 = none)
+//   node  : SIMT-stack node the record executes in (its mask == the record's mask)
+//   phase : number of BAR records of the warp before this record
+struct Snap {
+  u32 warp, ps, node, phase;
+};
+__device__ __forceinline__ Snap load_snap(const uint4* snap, u32 r) {
+  uint4 v = snap[r];
+  return Snap{v.x, v.y, v.z, v.w};
+}
+
+// SIMT-stack node (16 B): mask, parent node, popen = label of the warp's last step before the
+// IF that opened this node's branch (what the lanes outside it last shared with it).
+struct Node {
+  u32 mask, parent, popen, pad;
+};
+
+// ------------------------------------------------------------ read-only analysis state
+// Everything the happens-before query needs; passed by value to K3/K7/K8.
+struct HbCtx {
+  Geo g;
+  const uint4* snap;      // [n_recs]
+  const uint4* nodes;     // [n_nodes]
+  const u32* bar_base;    // [n_warps] first slot of the warp's barrier list
+  const u32* blockR;      // [n_bar_slots] completion label of barrier k of block b at bar_base[b*wpb]+k
+  // foreign knowledge (K3); n_acq == 0 => none
+  u32 n_acq;
+  const u32* acq_block_start;  // [n_blocks + 1] ranges into acq_*
+  const u32* acq_rec;          // acquire records sorted by (block, rec)
+  const u32* acq_warp;
+  const u32* acq_lane;         // a lane active in the acquire record
+  const u32* acq_arr;          // its arrF array id
+  u32 n_idx;
+  const u64* idx_ak;           // (arr << 32 | key), sorted with idx_pos
+  const u32* idx_pos;
+  const u32* idx_mask;
+  const u32* idx_clk;
+  u32* err;
+};
+
+__device__ __forceinline__ u32 barrier_label(const HbCtx& c, u32 warp, u32 phase) {
+  if (phase == 0) return 0;
+  u32 w0 = (warp / c.g.wpb) * c.g.wpb;
+  return c.blockR[c.bar_base[w0] + phase - 1];
+}
+
+// know_t(u) for u = lane `ul` of t's own warp, t executing record with snapshot s (intra-warp
+// part only; the PTVC DIVERGED / NESTEDDIVERGED lookup of Fig. 7).
+__device__ __forceinline__ u32 intra_know(const HbCtx& c, const Snap& s, u32 ul) {
+  u32 n = s.node;
+  uint4 nd = c.nodes[n];
+  if ((nd.x >> ul) & 1u) return s.ps;
+  // walk up the branch tree to the lowest ancestor whose mask holds ul
+  for (int d = 0; d < 40; ++d) {
+    u32 p = nd.y;
+    if (p == NONE) return 0;  // cannot happen for a valid lane (root mask = init mask)
+    uint4 pd = c.nodes[p];
+    if ((pd.x >> ul) & 1u) return nd.z;
+    nd = pd;
+  }
+  return 0;
+}
+
+// structural happens-before: does t (executing record r2 with snapshot s2) know the step of
+// (warp w1, lane l1) at record r1?  Same block only; no same-thread shortcut (callers do it).
+__device__ __forceinline__ bool struct_knows(const HbCtx& c, u32 w1, u32 l1, u32 r1, const Snap& s2) {
+  if (w1 / c.g.wpb != s2.warp / c.g.wpb) return false;
+  if (r1 + 1u <= barrier_label(c, s2.warp, s2.phase)) return true;
+  if (w1 == s2.warp && intra_know(c, s2, l1) >= r1 + 1u) return true;
+  return false;
+}
+
+// ------------------------------------------------------- foreign knowledge (K3 output)
+// The sync index holds, per array (S_x global part, S_x[b] block part, or an acquire record's
+// view), entries sorted by (arr, key, pos):
+//   key = KEY_BLOCK|b : the releaser knew all of block b up to label clk
+//   key = warp w      : the releaser knew lanes `mask` of warp w up to label clk
+//   key = KEY_LINK|a  : the releaser / acquirer also knew array a's entries with pos < clk
+// pos = (record << 5 | lane) of the release that appended the entry; a view (arr, bound)
+// sees the entries with pos < bound (S_x as it stood when the acquire ran, Fig. 3).
+__device__ __forceinline__ u32 idx_lower_bound(const HbCtx& c, u64 ak) {
+  u32 lo = 0, hi = c.n_idx;
+  while (lo < hi) {
+    u32 mid = (lo + hi) >> 1;
+    if (c.idx_ak[mid] < ak) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+// does view (arr, bound) know the step of (warp uw, lane ul) at record r1?
+static __device__ __noinline__ bool view_knows(const HbCtx& c, u32 uw, u32 ul, u32 r1, u32 arr, u32 bound) {
+  u32 st_arr[48], st_bd[48];
+  int sp = 0;
+  st_arr[sp] = arr;
+  st_bd[sp++] = bound;
+  u32 steps = 0;
+  const u32 need = r1 + 1u;
+  const u32 ub = uw / c.g.wpb;
+  while (sp > 0) {
+    --sp;
+    u32 a = st_arr[sp], bd = st_bd[sp];
+    if (++steps > SYNC_LOOKUP_CAP) {
+      set_err(c.err, ERR_OVERFLOW);
+      return false;
+    }
+    // block-level entries
+    u64 ak = ((u64)a << 32) | (KEY_BLOCK | ub);
+    for (u32 i = idx_lower_bound(c, ak); i < c.n_idx && c.idx_ak[i] == ak && c.idx_pos[i] < bd; ++i)
+      if (c.idx_clk[i] >= need) return true;
+    // warp-level entries
+    ak = ((u64)a << 32) | uw;
+    for (u32 i = idx_lower_bound(c, ak); i < c.n_idx && c.idx_ak[i] == ak && c.idx_pos[i] < bd; ++i)
+      if (((c.idx_mask[i] >> ul) & 1u) && c.idx_clk[i] >= need) return true;
+    // links: per target, the last entry with pos < bd carries the largest bound
+    u64 lk = ((u64)a << 32) | KEY_LINK;
+    u64 end = ((u64)a << 32) | 0xFFFFFFFFull;
+    u32 i = idx_lower_bound(c, lk);
+    while (i < c.n_idx && c.idx_ak[i] <= end) {
+      u64 key = c.idx_ak[i];
+      u32 best = 0;
+      bool any = false;
+      for (; i < c.n_idx && c.idx_ak[i] == key; ++i)
+        if (c.idx_pos[i] < bd) {
+          u32 b2 = c.idx_clk[i] < bd ? c.idx_clk[i] : bd;
+          if (!any || b2 > best) best = b2;
+          any = true;
+        }
+      if (any) {
+        if (sp >= 48) {
+          set_err(c.err, ERR_OVERFLOW);
+          return false;
+        }
+        st_arr[sp] = (u32)(key & 0x3FFFFFFFull);
+        st_bd[sp++] = best;
+      }
+    }
+  }
+  return false;
+}
+
+// foreign part of know_t(u) >= r1+1 for t executing record r2 (snapshot s2): through the
+// views of the acquires of t's block that t structurally knows (every release->acquire path
+// into t's block ends at one of them).
+static __device__ __noinline__ bool foreign_knows(const HbCtx& c, u32 w1, u32 l1, u32 r1, u32 r2, const Snap& s2) {
+  u32 b2 = s2.warp / c.g.wpb;
+  u32 lo = c.acq_block_start[b2], hi = c.acq_block_start[b2 + 1];
+  for (u32 i = lo; i < hi; ++i) {
+    u32 ra = c.acq_rec[i];
+    if (ra >= r2) break;
+    if (!struct_knows(c, c.acq_warp[i], c.acq_lane[i], ra, s2)) continue;
+    if (view_knows(c, w1, l1, r1, c.acq_arr[i], NONE)) return true;
+  }
+  return false;
+}
+
+// e1 = (record r1, lane l1) happened before e2 = (record r2, lane l2)?  r1 <= r2 in trace order.
+// s2 = snapshot of r2; w1 = warp of r1.
+__device__ __forceinline__ bool hb(const HbCtx& c, u32 r1, u32 l1, u32 w1, u32 r2, u32 l2, const Snap& s2) {
+  if (w1 == s2.warp && l1 == l2) return true;  // same thread: program order
+  if (r1 == r2) return false;                  // lanes of one instruction are concurrent
+  if (struct_knows(c, w1, l1, r1, s2)) return true;
+  if (c.n_acq == 0 || c.acq_block_start[s2.warp / c.g.wpb] == c.acq_block_start[s2.warp / c.g.wpb + 1])
+    return false;
+  return foreign_knows(c, w1, l1, r1, r2, s2);
+}
+
+// ------------------------------------------------------------------ warp primitives
+template <typename T>
+__device__ __forceinline__ T warp_incl_sum(T v) {
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    T n = __shfl_up_sync(0xFFFFFFFFu, v, o);
+    if ((threadIdx.x & 31) >= o) v += n;
+  }
+  return v;
+}
+
+// decoupled look-back status words (u64): [63:62] flag, [61:0] value
+constexpr u64 LB_AGG = 1ull << 62, LB_INC = 2ull << 62, LB_MASK = (1ull << 62) - 1;
+
+// exclusive prefix of `agg` for tile `tile` over u64 status words (single value per tile).
+// Called by one thread.
+__device__ __forceinline__ u64 lookback_u64(volatile u64* status, u32 tile, u64 agg) {
+  if (tile == 0) {
+    status[0] = LB_INC | agg;
+    return 0;
+  }
+  status[tile] = LB_AGG | agg;
+  u64 excl = 0;
+  int t = (int)tile - 1;
+  while (true) {
+    u64 s = status[t];
+    u64 f = s & ~LB_MASK;
+    if (f == 0) continue;
+    excl += s & LB_MASK;
+    if (f == LB_INC) break;
+    --t;
+  }
+  __threadfence();
+  status[tile] = LB_INC | (excl + agg);
+  return excl;
+}
+
+}  // namespace bc

@@ -1,0 +1,125 @@
+// finalize.cu — K8 race finalize: canonical order and classification.
+//
+// Races leave K7 as (granule key, current event, prior event, kind) in arbitrary order.  The
+// dense key order is the canonical location order (global granules by address, then shared
+// granules by (block, offset)), so a stable LSD sort by prior, then current, then key gives
+// the canonical (location, current, prior) order.  Classification from the two events
+// (reading R9): same record -> SAME_INSN; same warp -> BRANCH (branch ordering,
+// P:L591-630); same block -> INTRA_BLOCK; else INTER_BLOCK.  Barrier-divergence findings
+// come first, ordered by (block, record).
+#include "common.cuh"
+#include "kernels.cuh"
+
+namespace bc {
+
+namespace {
+
+inline unsigned nb(u64 n) { return (unsigned)((n + 255) / 256); }
+
+__global__ void k_field(const uint4* __restrict__ r, u32 n, int f, u32* __restrict__ out) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint4 v = r[i];
+  out[i] = f == 0 ? v.x : f == 1 ? v.y : v.z;
+}
+
+__global__ void k_page_list(const u32* __restrict__ bits, const u32* __restrict__ rank, u64 nwords,
+                            u32* __restrict__ page_num) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= nwords) return;
+  u32 b = bits[i];
+  u32 k = rank[i];
+  while (b) {
+    int j = __ffs(b) - 1;
+    b &= b - 1;
+    page_num[k++] = (u32)(i * 32 + j);
+  }
+}
+
+__global__ void k_emit_races(const uint4* __restrict__ r, const u32* __restrict__ perm, u32 n, Geo g,
+                             const uint4* __restrict__ snap, const u32* __restrict__ page_num, u32 shared_base,
+                             bc_race* __restrict__ out) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint4 v = r[perm[i]];
+  u32 key = v.x, cur = v.y, prior = v.z, kind = v.w;
+  bc_race o;
+  u32 cw = snap[cur >> 5].x, pw = snap[prior >> 5].x;
+  if (key < shared_base) {
+    u32 sh = 20 - g.G;
+    u64 page = page_num[key >> sh];
+    o.addr = (page << 20) | ((u64)(key & ((1u << sh) - 1u)) << g.G);
+    o.space = BC_SPACE_GLOBAL;
+    o.block = cw / g.wpb;
+  } else {
+    u32 k = key - shared_base;
+    o.addr = (u64)(k % g.smem_gran) << g.G;
+    o.space = BC_SPACE_SHARED;
+    o.block = k / g.smem_gran;
+  }
+  o.prior_event = (u64)prior;
+  o.cur_event = (u64)cur;
+  o.kind = (uint8_t)kind;
+  if ((cur >> 5) == (prior >> 5)) o.cls = BC_CLS_SAME_INSN;
+  else if (cw == pw) o.cls = BC_CLS_BRANCH;
+  else if (cw / g.wpb == pw / g.wpb) o.cls = BC_CLS_INTRA_BLOCK;
+  else o.cls = BC_CLS_INTER_BLOCK;
+  o.pad = 0;
+  out[i] = o;
+}
+
+__global__ void k_emit_findings(const u32* __restrict__ fblk, const u32* __restrict__ frec,
+                                const u32* __restrict__ perm, u32 n, bc_race* __restrict__ out) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  u32 p = perm[i];
+  bc_race o;
+  o.addr = 0;
+  o.prior_event = ~0ull;
+  o.cur_event = (u64)frec[p] << 5;
+  o.kind = BC_KIND_NONE;
+  o.cls = BC_CLS_BARRIER_DIVERGENCE;
+  o.space = BC_SPACE_NONE;
+  o.pad = 0;
+  o.block = fblk[p];
+  out[i] = o;
+}
+
+int bits_for(u64 maxval) {
+  int b = 0;
+  while (b < 32 && (maxval >> b)) ++b;
+  return b;
+}
+
+}  // namespace
+
+void launch_page_list(const u32* bits, const u32* rank, u64 nwords, u32* page_num, cudaStream_t st) {
+  k_page_list<<<nb(nwords), 256, 0, st>>>(bits, rank, nwords, page_num);
+}
+
+// races[n_r] (key, cur, prior, kind) + findings -> out[n_f + n_r] in canonical order
+void finalize_races(const uint4* races, u32 n_r, const u32* fblk, const u32* frec, u32 n_f, const Geo& g,
+                    const uint4* snap, const u32* page_num, u32 shared_base, u32 n_keys, bc_race* out, Scratch& S,
+                    cudaStream_t st) {
+  if (n_f) {
+    u32* p = S.alloc<u32>(n_f);
+    launch_iota(p, n_f, st);
+    sort_perm_by(p, frec, n_f, 32, S, st);
+    sort_perm_by(p, fblk, n_f, bits_for(g.n_blocks), S, st);
+    k_emit_findings<<<nb(n_f), 256, 0, st>>>(fblk, frec, p, n_f, out);
+  }
+  if (n_r) {
+    u32* p = S.alloc<u32>(n_r);
+    u32* f = S.alloc<u32>(n_r);
+    launch_iota(p, n_r, st);
+    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 2, f);
+    sort_perm_by(p, f, n_r, 32, S, st);
+    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 1, f);
+    sort_perm_by(p, f, n_r, 32, S, st);
+    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 0, f);
+    sort_perm_by(p, f, n_r, bits_for(n_keys), S, st);
+    k_emit_races<<<nb(n_r), 256, 0, st>>>(races, p, n_r, g, snap, page_num, shared_base, out + n_f);
+  }
+}
+
+}  // namespace bc

@@ -1,0 +1,85 @@
+// kernels.cuh — host-side launchers of the libbc kernels and the scratch allocator.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <new>
+#include <vector>
+
+#include "common.cuh"
+
+namespace bc {
+
+// counters written by the kernels (u64 device array)
+enum { C_LANE_EVENTS = 0, C_CONTROL_EVENTS, C_SYNC_RECS, C_ACQ_RECS, C_MEM_RECS, C_IFS, C_BARS, C_SYNC_LANEOPS,
+       C_ITEMS, C_ITEM_BOUND, C_SEGMENTS, C_N };
+
+// Stream-ordered scratch memory for one bc_detect: cudaMallocAsync from the device's memory
+// pool (kept cached between calls), all freed at release().
+class Scratch {
+ public:
+  explicit Scratch(cudaStream_t st) : st_(st) {}
+  ~Scratch() { release(); }
+  template <typename T>
+  T* alloc(size_t n) {
+    void* p = nullptr;
+    size_t bytes = n * sizeof(T);
+    if (bytes == 0) bytes = 16;
+    bytes = (bytes + 255) & ~(size_t)255;
+    if (cudaMallocAsync(&p, bytes, st_) != cudaSuccess || !p) {
+      cudaGetLastError();
+      throw std::bad_alloc();
+    }
+    ptrs_.push_back(p);
+    return (T*)p;
+  }
+  void release() {
+    for (void* p : ptrs_) cudaFreeAsync(p, st_);
+    ptrs_.clear();
+  }
+
+ private:
+  cudaStream_t st_;
+  std::vector<void*> ptrs_;
+};
+
+// sort.cu
+size_t rs_temp_bytes(u64 n);
+bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi, void* temp,
+                      cudaStream_t st);
+size_t scan_temp_bytes(u64 n);
+void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_dev, cudaStream_t st);
+
+// trace.cu
+void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
+                   u32* sync_list, u32* page_bits, u64* cnt, u32* err, cudaStream_t st);
+void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st);
+void launch_replay(const bc_record* recs, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
+                   const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next, u32* find_blk,
+                   u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st);
+void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, const u32* bar_rec, const u32* bar_next,
+                     u32* blockR, u32* err, cudaStream_t st);
+void launch_popc(const u32* bits, u32* out, u64 n, cudaStream_t st);
+u64 expand_tiles(u64 n_recs);
+void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
+                   u32* keys, u32* evs, u64* status, u32* tile_counter, u64* cnt, u32* err, cudaStream_t st);
+void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st);
+
+// sync.cu
+void sort_perm_by(u32* perm, const u32* f, u32 n, int bits, Scratch& S, cudaStream_t st);
+void launch_iota(u32* p, u32 n, cudaStream_t st);
+void launch_gather_u32(const u32* src, const u32* perm, u32 n, u32* dst, cudaStream_t st);
+int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_lo, HbCtx& hc, Scratch& S,
+                      cudaStream_t st, u64* n_entries_out);
+
+// check.cu
+size_t check_status_bytes(u64 n);
+void launch_check(const HbCtx& c, const u32* keys, const u32* evs, u64 n, void* status, u32* tile_counter,
+                  uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, cudaStream_t st);
+
+// finalize.cu
+void launch_page_list(const u32* bits, const u32* rank, u64 nwords, u32* page_num, cudaStream_t st);
+void finalize_races(const uint4* races, u32 n_r, const u32* fblk, const u32* frec, u32 n_f, const Geo& g,
+                    const uint4* snap, const u32* page_num, u32 shared_base, u32 n_keys, bc_race* out, Scratch& S,
+                    cudaStream_t st);
+
+}  // namespace bc

@@ -1,0 +1,478 @@
+// sync.cu — K3 sync skeleton: the ACQ / REL / ACQREL x BLOCK / GLOBAL
+// rules of Fig. 3 and their scope semantics (§3.3.4) over the
+// sync-location map S_x, reading R1 (release joins into S_x).
+//
+// S_x is kept as append-only arrays of entries instead of materialised vector clocks:
+//   array G_x          (id = xid)            : what global-scope releases put in every S_x[b]
+//   array B_{x,b}      (id = nx + bid)       : what block-scope releases of block b put in S_x[b]
+//   array F_a          (id = nx + nB + a)    : the view acquire record a took
+// A release lane-op at event e appends, at pos e, the releaser's structural clock (block-level
+// barrier label, the warp's SIMT-stack levels) plus LINKs to the views of the acquires of its
+// block it structurally knows (its foreign knowledge).  An acquire lane-op at event e records
+// LINKs (G_x, bound e) and the block arrays it may read: S_x[b] = G_x ⊔ B_{x,b} (ACQ_BLK) or
+// ⊔_b S_x[b] = G_x ⊔ ⊔_b B_{x,b} (ACQ_GLB).  Because a view is "entries with pos < bound",
+// nothing has to be processed in trace order: every lane-op is independent (one thread each),
+// and an AR chain (threadFenceReduction's atomicInc ticket) costs O(1) entries per op instead of
+// the O(n) vector-clock copy of the printed rules.
+#include "common.cuh"
+#include "kernels.cuh"
+
+namespace bc {
+
+namespace {
+
+__device__ __forceinline__ bool is_acq_op(u32 op) {
+  return op == BC_OP_ACQ_BLK || op == BC_OP_ACQ_GLB || op == BC_OP_AR_BLK || op == BC_OP_AR_GLB;
+}
+__device__ __forceinline__ bool is_rel_op(u32 op) {
+  return op == BC_OP_REL_BLK || op == BC_OP_REL_GLB || op == BC_OP_AR_BLK || op == BC_OP_AR_GLB;
+}
+__device__ __forceinline__ bool is_glb_op(u32 op) {
+  return op == BC_OP_ACQ_GLB || op == BC_OP_REL_GLB || op == BC_OP_AR_GLB;
+}
+
+__global__ void k_popc_recs(const bc_record* __restrict__ recs, const u32* __restrict__ srec, u32 n,
+                            u32* __restrict__ out) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) out[i] = __popc(__ldg(&recs[srec[i]].mask));
+}
+
+// lane-ops: rec, lane, 64-bit location key (split), index
+__global__ void k_laneops(const bc_record* __restrict__ recs, const u32* __restrict__ srec, u32 n,
+                          const u32* __restrict__ off, Geo g, u32* __restrict__ lo_rec, u32* __restrict__ lo_lane,
+                          u32* __restrict__ xk_lo, u32* __restrict__ xk_hi, u32* __restrict__ lo_idx,
+                          u32* __restrict__ err) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  u32 r = srec[i];
+  const bc_record& rc = recs[r];
+  u32 m = rc.mask, o = off[i];
+  u32 w = rc.warp;
+  while (m) {
+    int l = __ffs(m) - 1;
+    m &= m - 1;
+    u64 a = rc.addr[l];
+    u64 xk;
+    if (rc.space == BC_SPACE_SHARED) {
+      xk = (1ull << 63) | ((u64)(w / g.wpb) << 32) | (u64)(a >> g.G);
+    } else {
+      xk = a >> g.G;
+      if (xk >> 63) set_err(err, ERR_OVERFLOW);
+    }
+    lo_rec[o] = r;
+    lo_lane[o] = (u32)l;
+    xk_lo[o] = (u32)xk;
+    xk_hi[o] = (u32)(xk >> 32);
+    lo_idx[o] = o;
+    ++o;
+  }
+}
+
+// flags of the first occurrence of each distinct (hi, lo) in sorted order
+__global__ void k_uniq_flags2(const u32* __restrict__ hi, const u32* __restrict__ lo, const u32* __restrict__ perm,
+                              u32 n, u32* __restrict__ flag) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  u32 p = perm[i];
+  u32 f = 1;
+  if (i > 0) {
+    u32 q = perm[i - 1];
+    f = (hi[p] != hi[q] || lo[p] != lo[q]) ? 1u : 0u;
+  }
+  flag[i] = f;
+}
+
+// xid[perm[i]] = (inclusive flag scan)[i] - 1 ; here `ex` is the exclusive scan of flags
+__global__ void k_assign_ids(const u32* __restrict__ perm, const u32* __restrict__ flag, const u32* __restrict__ ex,
+                             u32 n, u32* __restrict__ id) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  id[perm[i]] = ex[i] + flag[i] - 1;
+}
+
+// candidate (xid, block) pairs of block-scope releases
+__global__ void k_bpairs(const bc_record* __restrict__ recs, const u32* __restrict__ lo_rec, const u32* __restrict__ xid,
+                         u32 n, Geo g, u32* __restrict__ pk_hi, u32* __restrict__ pk_lo, u32* __restrict__ cnt) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  u32 r = lo_rec[i];
+  u32 op = recs[r].op;
+  if (op == BC_OP_REL_BLK || op == BC_OP_AR_BLK) {
+    u32 at = atomicAdd(cnt, 1u);
+    pk_hi[at] = xid[i];
+    pk_lo[at] = recs[r].warp / g.wpb;
+  }
+}
+
+// compact unique sorted pairs
+__global__ void k_compact_pairs(const u32* __restrict__ hi, const u32* __restrict__ lo, const u32* __restrict__ perm,
+                                const u32* __restrict__ flag, const u32* __restrict__ ex, u32 n,
+                                u32* __restrict__ ohi, u32* __restrict__ olo) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n || !flag[i]) return;
+  u32 p = perm[i];
+  ohi[ex[i]] = hi[p];
+  olo[ex[i]] = lo[p];
+}
+
+struct K3In {
+  HbCtx hc;
+  const bc_record* recs;
+  u32 n_lo;
+  const u32 *lo_rec, *lo_lane, *xid;
+  u32 nx, nB;
+  const u32 *bp_x, *bp_b;  // unique sorted (xid, block) pairs, bid = index
+  const u32* acq_idx_of_rec_sorted;  // unused
+};
+
+__device__ __forceinline__ u32 pair_lower(const K3In& k, u32 x, u32 b) {
+  u32 lo = 0, hi = k.nB;
+  while (lo < hi) {
+    u32 m = (lo + hi) >> 1;
+    if (k.bp_x[m] < x || (k.bp_x[m] == x && k.bp_b[m] < b)) lo = m + 1; else hi = m;
+  }
+  return lo;
+}
+__device__ __forceinline__ u32 find_bid(const K3In& k, u32 x, u32 b) {
+  u32 i = pair_lower(k, x, b);
+  return (i < k.nB && k.bp_x[i] == x && k.bp_b[i] == b) ? i : NONE;
+}
+
+// index of acquire record r in the (block, rec)-sorted acquire list
+__device__ __forceinline__ u32 acq_index(const HbCtx& c, u32 b, u32 r) {
+  u32 lo = c.acq_block_start[b], hi = c.acq_block_start[b + 1];
+  while (lo < hi) {
+    u32 m = (lo + hi) >> 1;
+    if (c.acq_rec[m] < r) lo = m + 1; else hi = m;
+  }
+  return lo;
+}
+
+// Emit (or count, when out == nullptr) the entries of lane-op i.
+struct EntOut {
+  u32 *arr, *key, *pos, *mask, *clk;
+};
+
+__device__ __forceinline__ void put(const EntOut* o, u32& n, u32 arr, u32 key, u32 pos, u32 mask, u32 clk) {
+  if (o) {
+    o->arr[n] = arr;
+    o->key[n] = key;
+    o->pos[n] = pos;
+    o->mask[n] = mask;
+    o->clk[n] = clk;
+  }
+  ++n;
+}
+
+__device__ u32 laneop_entries(const K3In& k, u32 i, const EntOut* o, u32 base) {
+  const HbCtx& c = k.hc;
+  u32 r = k.lo_rec[i], lane = k.lo_lane[i];
+  u32 op = k.recs[r].op;
+  u32 w = k.recs[r].warp;
+  u32 b = w / c.g.wpb;
+  u32 x = k.xid[i];
+  u32 ev = (r << 5) | lane;
+  u32 n = base;
+  // range of block arrays of x
+  u32 blo = pair_lower(k, x, 0), bhi = pair_lower(k, x + 1, 0);
+  u32 my_bid = find_bid(k, x, b);
+  if (is_acq_op(op)) {
+    u32 ai = acq_index(c, b, r);
+    u32 farr = k.nx + k.nB + ai;
+    put(o, n, farr, KEY_LINK | x, ev, 0u, ev);  // S_x global part
+    if (is_glb_op(op)) {
+      for (u32 j = blo; j < bhi; ++j) put(o, n, farr, KEY_LINK | (k.nx + j), ev, 0u, ev);
+    } else if (my_bid != NONE) {
+      put(o, n, farr, KEY_LINK | (k.nx + my_bid), ev, 0u, ev);
+    }
+  }
+  if (is_rel_op(op)) {
+    u32 tarr = is_glb_op(op) ? x : (k.nx + my_bid);
+    Snap s = load_snap(c.snap, r);
+    // structural clock of the releaser (its block only)
+    u32 bl = barrier_label(c, w, s.phase);
+    if (bl) put(o, n, tarr, KEY_BLOCK | b, ev, 0xFFFFFFFFu, bl);
+    {
+      uint4 nd = c.nodes[s.node];
+      if (s.ps) put(o, n, tarr, w, ev, nd.x, s.ps);
+      for (int d = 0; d < 40 && nd.y != NONE; ++d) {
+        uint4 pd = c.nodes[nd.y];
+        if (nd.z) put(o, n, tarr, w, ev, pd.x, nd.z);
+        nd = pd;
+      }
+    }
+    // foreign knowledge: the acquires of this block it structurally knows
+    for (u32 j = c.acq_block_start[b]; j < c.acq_block_start[b + 1]; ++j) {
+      u32 ra = c.acq_rec[j];
+      if (ra >= r) break;
+      if (struct_knows(c, c.acq_warp[j], c.acq_lane[j], ra, s)) put(o, n, tarr, KEY_LINK | (k.nx + k.nB + j), ev, 0u, ev);
+    }
+    // ACQREL: the part of S_x it acquired that lives in another array
+    if (op == BC_OP_AR_BLK) {
+      put(o, n, tarr, KEY_LINK | x, ev, 0u, ev);
+    } else if (op == BC_OP_AR_GLB) {
+      for (u32 j = blo; j < bhi; ++j) put(o, n, tarr, KEY_LINK | (k.nx + j), ev, 0u, ev);
+    }
+  }
+  return n - base;
+}
+
+__global__ void k_ent_count(K3In k, u32* __restrict__ out) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < k.n_lo) out[i] = laneop_entries(k, i, nullptr, 0);
+}
+
+__global__ void k_ent_fill(K3In k, const u32* __restrict__ off, EntOut o) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < k.n_lo) laneop_entries(k, i, &o, off[i]);
+}
+
+// acquire list: sync records (sorted by rec) that acquire -> keys = block, vals = rec
+__global__ void k_acq_collect(const bc_record* __restrict__ recs, const u32* __restrict__ srec, u32 n, Geo g,
+                              u32* __restrict__ akey, u32* __restrict__ aval, u32* __restrict__ cnt) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  u32 r = srec[i];
+  u32 op = recs[r].op;
+  // keep trace order: the slot is the rank among acquires, computed by a flag scan on the host side
+  if (is_acq_op(op)) {
+    u32 at = cnt[i];
+    akey[at] = recs[r].warp / g.wpb;
+    aval[at] = r;
+  }
+}
+__global__ void k_acq_flags(const bc_record* __restrict__ recs, const u32* __restrict__ srec, u32 n,
+                            u32* __restrict__ flag) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) flag[i] = is_acq_op(recs[srec[i]].op) ? 1u : 0u;
+}
+__global__ void k_acq_info(const bc_record* __restrict__ recs, const u32* __restrict__ arec, u32 n,
+                           u32* __restrict__ awarp, u32* __restrict__ alane) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  u32 r = arec[i];
+  awarp[i] = recs[r].warp;
+  alane[i] = __ffs(recs[r].mask) - 1;
+}
+__global__ void k_block_start(const u32* __restrict__ sorted_blocks, u32 n, u32 n_blocks, u32* __restrict__ start) {
+  u32 b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b > n_blocks) return;
+  u32 lo = 0, hi = n;
+  while (lo < hi) {
+    u32 m = (lo + hi) >> 1;
+    if (sorted_blocks[m] < b) lo = m + 1; else hi = m;
+  }
+  start[b] = lo;
+}
+
+__global__ void k_gather_u32(const u32* __restrict__ src, const u32* __restrict__ perm, u32 n, u32* __restrict__ dst) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) dst[i] = src[perm[i]];
+}
+__global__ void k_iota_add(u32* __restrict__ p, u32 n, u32 add) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = i + add;
+}
+__global__ void k_iota(u32* __restrict__ p, u32 n) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = i;
+}
+__global__ void k_make_ak(const u32* __restrict__ arr, const u32* __restrict__ key, const u32* __restrict__ pos,
+                          const u32* __restrict__ mask, const u32* __restrict__ clk, const u32* __restrict__ perm,
+                          u32 n, u64* __restrict__ ak, u32* __restrict__ opos, u32* __restrict__ omask,
+                          u32* __restrict__ oclk) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  u32 p = perm[i];
+  ak[i] = ((u64)arr[p] << 32) | key[p];
+  opos[i] = pos[p];
+  omask[i] = mask[p];
+  oclk[i] = clk[p];
+}
+
+inline unsigned nb(u64 n) { return (unsigned)((n + 255) / 256); }
+
+}  // namespace
+
+// Sort a permutation `perm` (initially any order) stably by the 32-bit field `f` (bits [0, bits)).
+void sort_perm_by(u32* perm, const u32* f, u32 n, int bits, Scratch& S, cudaStream_t st) {
+  if (n <= 1) return;
+  u32* k = S.alloc<u32>(n);
+  u32* k2 = S.alloc<u32>(n);
+  u32* p2 = S.alloc<u32>(n);
+  void* tmp = S.alloc<char>(rs_temp_bytes(n));
+  k_gather_u32<<<nb(n), 256, 0, st>>>(f, perm, n, k);
+  bool alt = radix_sort_pairs(k, perm, k2, p2, n, 0, bits, tmp, st);
+  if (alt) cudaMemcpyAsync(perm, p2, n * sizeof(u32), cudaMemcpyDeviceToDevice, st);
+}
+
+void launch_iota(u32* p, u32 n, cudaStream_t st) {
+  if (n) k_iota<<<nb(n), 256, 0, st>>>(p, n);
+}
+void launch_gather_u32(const u32* src, const u32* perm, u32 n, u32* dst, cudaStream_t st) {
+  if (n) k_gather_u32<<<nb(n), 256, 0, st>>>(src, perm, n, dst);
+}
+
+static int bits_for(u64 maxval) {
+  int b = 0;
+  while (b < 32 && (maxval >> b)) ++b;
+  return b;
+}
+
+// Runs K3.  Fills the foreign-knowledge fields of `hc` (acq_*, idx_*).  Returns 0 or a bc_status.
+int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_lo, HbCtx& hc, Scratch& S,
+                      cudaStream_t st, u64* n_entries_out) {
+  const Geo& g = hc.g;
+  *n_entries_out = 0;
+  if (n_srec == 0) return 0;
+  // 1. sync records in trace order
+  {
+    u32* k2 = S.alloc<u32>(n_srec);
+    u32* v = S.alloc<u32>(n_srec);
+    u32* v2 = S.alloc<u32>(n_srec);
+    void* tmp = S.alloc<char>(rs_temp_bytes(n_srec));
+    launch_iota(v, n_srec, st);
+    bool alt = radix_sort_pairs(sync_list, v, k2, v2, n_srec, 0, bits_for(g.n_recs), tmp, st);
+    if (alt) cudaMemcpyAsync(sync_list, k2, n_srec * sizeof(u32), cudaMemcpyDeviceToDevice, st);
+  }
+  // 2. acquire list sorted by (block, rec)
+  u32* aflag = S.alloc<u32>(n_srec);
+  u32* aex = S.alloc<u32>(n_srec);
+  u64* tot = S.alloc<u64>(1);
+  k_acq_flags<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, aflag);
+  exclusive_scan_u32(aflag, aex, n_srec, S.alloc<char>(scan_temp_bytes(n_srec)), tot, st);
+  u64 n_acq64 = 0;
+  cudaMemcpyAsync(&n_acq64, tot, 8, cudaMemcpyDeviceToHost, st);
+  if (cudaStreamSynchronize(st) != cudaSuccess) return BC_ERR_CUDA;
+  u32 n_acq = (u32)n_acq64;
+  u32* acq_blk = S.alloc<u32>(n_acq + 1);
+  u32* acq_rec = S.alloc<u32>(n_acq + 1);
+  u32* acq_warp = S.alloc<u32>(n_acq + 1);
+  u32* acq_lane = S.alloc<u32>(n_acq + 1);
+  u32* acq_bstart = S.alloc<u32>(g.n_blocks + 1);
+  if (n_acq) {
+    k_acq_collect<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, g, acq_blk, acq_rec, aex);
+    u32* k2 = S.alloc<u32>(n_acq);
+    u32* v2 = S.alloc<u32>(n_acq);
+    void* tmp = S.alloc<char>(rs_temp_bytes(n_acq));
+    bool alt = radix_sort_pairs(acq_blk, acq_rec, k2, v2, n_acq, 0, bits_for(g.n_blocks), tmp, st);
+    if (alt) {
+      cudaMemcpyAsync(acq_blk, k2, n_acq * 4, cudaMemcpyDeviceToDevice, st);
+      cudaMemcpyAsync(acq_rec, v2, n_acq * 4, cudaMemcpyDeviceToDevice, st);
+    }
+    k_acq_info<<<nb(n_acq), 256, 0, st>>>(recs, acq_rec, n_acq, acq_warp, acq_lane);
+  }
+  k_block_start<<<nb(g.n_blocks + 1), 256, 0, st>>>(acq_blk, n_acq, g.n_blocks, acq_bstart);
+  hc.n_acq = n_acq;
+  hc.acq_block_start = acq_bstart;
+  hc.acq_rec = acq_rec;
+  hc.acq_warp = acq_warp;
+  hc.acq_lane = acq_lane;
+
+  // 3. lane-ops and dense sync-location ids
+  u32* cnt = S.alloc<u32>(n_srec);
+  u32* off = S.alloc<u32>(n_srec);
+  k_popc_recs<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, cnt);
+  exclusive_scan_u32(cnt, off, n_srec, S.alloc<char>(scan_temp_bytes(n_srec)), nullptr, st);
+  u32* lo_rec = S.alloc<u32>(n_lo);
+  u32* lo_lane = S.alloc<u32>(n_lo);
+  u32* xk_lo = S.alloc<u32>(n_lo);
+  u32* xk_hi = S.alloc<u32>(n_lo);
+  u32* perm = S.alloc<u32>(n_lo);
+  k_laneops<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, off, g, lo_rec, lo_lane, xk_lo, xk_hi, perm, hc.err);
+  sort_perm_by(perm, xk_lo, n_lo, 32, S, st);
+  sort_perm_by(perm, xk_hi, n_lo, 32, S, st);
+  u32* flag = S.alloc<u32>(n_lo);
+  u32* ex = S.alloc<u32>(n_lo);
+  u32* xid = S.alloc<u32>(n_lo);
+  k_uniq_flags2<<<nb(n_lo), 256, 0, st>>>(xk_hi, xk_lo, perm, n_lo, flag);
+  exclusive_scan_u32(flag, ex, n_lo, S.alloc<char>(scan_temp_bytes(n_lo)), tot, st);
+  k_assign_ids<<<nb(n_lo), 256, 0, st>>>(perm, flag, ex, n_lo, xid);
+  u64 nx64 = 0;
+  cudaMemcpyAsync(&nx64, tot, 8, cudaMemcpyDeviceToHost, st);
+  // 4. block arrays B_{x,b}
+  u32* pk_hi = S.alloc<u32>(n_lo);
+  u32* pk_lo = S.alloc<u32>(n_lo);
+  u32* pcnt = S.alloc<u32>(1);
+  cudaMemsetAsync(pcnt, 0, 4, st);
+  k_bpairs<<<nb(n_lo), 256, 0, st>>>(recs, lo_rec, xid, n_lo, g, pk_hi, pk_lo, pcnt);
+  u32 np = 0;
+  cudaMemcpyAsync(&np, pcnt, 4, cudaMemcpyDeviceToHost, st);
+  if (cudaStreamSynchronize(st) != cudaSuccess) return BC_ERR_CUDA;
+  u32 nx = (u32)nx64;
+  u32 nB = 0;
+  u32* bp_x = S.alloc<u32>(np + 1);
+  u32* bp_b = S.alloc<u32>(np + 1);
+  if (np) {
+    u32* pp = S.alloc<u32>(np);
+    launch_iota(pp, np, st);
+    sort_perm_by(pp, pk_lo, np, 32, S, st);
+    sort_perm_by(pp, pk_hi, np, 32, S, st);
+    u32* pf = S.alloc<u32>(np);
+    u32* pe = S.alloc<u32>(np);
+    k_uniq_flags2<<<nb(np), 256, 0, st>>>(pk_hi, pk_lo, pp, np, pf);
+    exclusive_scan_u32(pf, pe, np, S.alloc<char>(scan_temp_bytes(np)), tot, st);
+    k_compact_pairs<<<nb(np), 256, 0, st>>>(pk_hi, pk_lo, pp, pf, pe, np, bp_x, bp_b);
+    u64 nb64 = 0;
+    cudaMemcpyAsync(&nb64, tot, 8, cudaMemcpyDeviceToHost, st);
+    if (cudaStreamSynchronize(st) != cudaSuccess) return BC_ERR_CUDA;
+    nB = (u32)nb64;
+  }
+  if ((u64)nx + nB + n_acq >= (1ull << 30)) return BC_ERR_OVERFLOW;
+  hc.acq_arr = nullptr;
+  // arrF ids are nx + nB + acquire index; expose them for K7
+  {
+    u32* acq_arr = S.alloc<u32>(n_acq + 1);
+    if (n_acq) k_iota_add<<<nb(n_acq), 256, 0, st>>>(acq_arr, n_acq, nx + nB);
+    hc.acq_arr = acq_arr;
+  }
+  // 5. entries
+  K3In k;
+  k.hc = hc;
+  k.recs = recs;
+  k.n_lo = n_lo;
+  k.lo_rec = lo_rec;
+  k.lo_lane = lo_lane;
+  k.xid = xid;
+  k.nx = nx;
+  k.nB = nB;
+  k.bp_x = bp_x;
+  k.bp_b = bp_b;
+  k.acq_idx_of_rec_sorted = nullptr;
+  u32* ecnt = S.alloc<u32>(n_lo);
+  u32* eoff = S.alloc<u32>(n_lo);
+  k_ent_count<<<nb(n_lo), 128, 0, st>>>(k, ecnt);
+  exclusive_scan_u32(ecnt, eoff, n_lo, S.alloc<char>(scan_temp_bytes(n_lo)), tot, st);
+  u64 ne64 = 0;
+  cudaMemcpyAsync(&ne64, tot, 8, cudaMemcpyDeviceToHost, st);
+  if (cudaStreamSynchronize(st) != cudaSuccess) return BC_ERR_CUDA;
+  if (ne64 >= (1ull << 31)) return BC_ERR_OVERFLOW;
+  u32 ne = (u32)ne64;
+  *n_entries_out = ne;
+  EntOut eo;
+  eo.arr = S.alloc<u32>(ne + 1);
+  eo.key = S.alloc<u32>(ne + 1);
+  eo.pos = S.alloc<u32>(ne + 1);
+  eo.mask = S.alloc<u32>(ne + 1);
+  eo.clk = S.alloc<u32>(ne + 1);
+  k_ent_fill<<<nb(n_lo), 128, 0, st>>>(k, eoff, eo);
+  // 6. index sorted by (arr, key, pos)
+  u32* ep = S.alloc<u32>(ne + 1);
+  launch_iota(ep, ne, st);
+  sort_perm_by(ep, eo.pos, ne, 32, S, st);
+  sort_perm_by(ep, eo.key, ne, 32, S, st);
+  sort_perm_by(ep, eo.arr, ne, bits_for((u64)nx + nB + n_acq), S, st);
+  u64* ak = S.alloc<u64>(ne + 1);
+  u32* ipos = S.alloc<u32>(ne + 1);
+  u32* imask = S.alloc<u32>(ne + 1);
+  u32* iclk = S.alloc<u32>(ne + 1);
+  if (ne) k_make_ak<<<nb(ne), 256, 0, st>>>(eo.arr, eo.key, eo.pos, eo.mask, eo.clk, ep, ne, ak, ipos, imask, iclk);
+  hc.n_idx = ne;
+  hc.idx_ak = ak;
+  hc.idx_pos = ipos;
+  hc.idx_mask = imask;
+  hc.idx_clk = iclk;
+  return 0;
+}
+
+}  // namespace bc

@@ -1,0 +1,404 @@
+// trace.cu — the record-level passes of the hot path:
+//   k_header   (a1/a2) header validation, event counts, K1 partition keys, write-page marking
+//   k_replay   (a3)    K2 compressed clock replay: one thread per traced warp walks its records
+//   k_barriers (a3)    block barrier completion labels (§4.3.2 block max)
+//   k_expand   (a5)    K4 lane expansion into (granule key | op, event) items in trace order
+#include "common.cuh"
+#include "kernels.cuh"
+
+namespace bc {
+
+// counters in `cnt` (u64)
+
+// ---------------------------------------------------------------------------- k_header
+// One warp per 32 consecutive records.  Lane l validates record base+l's header (the checks of
+// P:L360-366 that need no state; stack / barrier checks are in k_replay / k_barriers), then the
+// warp marks the 1-MB pages written by the ST / ATOM global records among the 32 (the paper's
+// on-demand global shadow page table, used here to skip never-written memory).
+__global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ recs, Geo g, u32* __restrict__ wkey,
+                                                u32* __restrict__ wval, u32* __restrict__ if_cnt,
+                                                u32* __restrict__ bar_cnt, u32* __restrict__ sync_list,
+                                                u32* __restrict__ page_bits, u64* __restrict__ cnt,
+                                                u32* __restrict__ err) {
+  const u32 lane = threadIdx.x & 31;
+  const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const u64 r = gw * 32 + lane;
+  bool valid = r < g.n_recs;
+  Hdr h{};
+  u32 bad = 0;
+  u32 lane_ev = 0, ctl_ev = 0, is_sync = 0, is_acq = 0, is_mem = 0, is_if = 0, is_bar = 0, ibound = 0;
+  if (valid) {
+    h = load_hdr(recs, r);
+    if (h.op > BC_OP_FI || h.warp >= g.n_warps) {
+      bad = 1;
+    } else {
+      if (h.mask & ~init_mask(g, h.warp)) bad = 1;
+      if (h.op <= BC_OP_AR_GLB) {
+        if (h.mask == 0 || h.size_log2 > 4 || h.space > BC_SPACE_SHARED) bad = 1;
+        lane_ev = __popc(h.mask);
+        if (h.op <= BC_OP_ATOM) {
+          is_mem = 1;
+          u32 ng = (1u << (h.size_log2 & 7)) >> g.G;
+          ibound = lane_ev * (ng ? ng : 1u);
+        } else {
+          is_sync = 1;
+        }
+        if (h.op == BC_OP_ACQ_BLK || h.op == BC_OP_ACQ_GLB || h.op == BC_OP_AR_BLK || h.op == BC_OP_AR_GLB)
+          is_acq = 1;
+      } else {
+        ctl_ev = 1;
+        if ((h.op == BC_OP_FENCE || h.op == BC_OP_BAR) && h.mask == 0) bad = 1;
+        if (h.op == BC_OP_IF) {
+          if (h.mask == 0 || (h.aux & ~h.mask)) bad = 1;
+          is_if = 1;
+        }
+        if (h.op == BC_OP_BAR) is_bar = 1;
+      }
+    }
+    wkey[r] = bad ? 0u : h.warp;
+    wval[r] = (u32)r;
+    if (!bad) {
+      if (is_if) atomicAdd(&if_cnt[h.warp], 1u);
+      if (is_bar) atomicAdd(&bar_cnt[h.warp], 1u);
+      if (is_sync) {
+        u64 at = atomicAdd((unsigned long long*)&cnt[C_SYNC_RECS], 1ull);
+        sync_list[at] = (u32)r;
+      }
+    }
+  }
+  if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
+  // warp-reduced counters
+  if (bad) ibound = 0;
+  u32 v[8] = {lane_ev, ctl_ev, is_acq, is_mem, is_if, is_bar, is_sync ? lane_ev : 0u, ibound};
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v[i] += __shfl_down_sync(0xFFFFFFFFu, v[i], o);
+  }
+  if (lane == 0) {
+    if (v[0]) atomicAdd((unsigned long long*)&cnt[C_LANE_EVENTS], (unsigned long long)v[0]);
+    if (v[1]) atomicAdd((unsigned long long*)&cnt[C_CONTROL_EVENTS], (unsigned long long)v[1]);
+    if (v[2]) atomicAdd((unsigned long long*)&cnt[C_ACQ_RECS], (unsigned long long)v[2]);
+    if (v[3]) atomicAdd((unsigned long long*)&cnt[C_MEM_RECS], (unsigned long long)v[3]);
+    if (v[4]) atomicAdd((unsigned long long*)&cnt[C_IFS], (unsigned long long)v[4]);
+    if (v[5]) atomicAdd((unsigned long long*)&cnt[C_BARS], (unsigned long long)v[5]);
+    if (v[6]) atomicAdd((unsigned long long*)&cnt[C_SYNC_LANEOPS], (unsigned long long)v[6]);
+    if (v[7]) atomicAdd((unsigned long long*)&cnt[C_ITEM_BOUND], (unsigned long long)v[7]);
+  }
+  // page marking: ST / ATOM on global memory
+  u32 wr = __ballot_sync(0xFFFFFFFFu, valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) &&
+                                          h.space == BC_SPACE_GLOBAL);
+  while (wr) {
+    int j = __ffs(wr) - 1;
+    wr &= wr - 1;
+    u32 m = __shfl_sync(0xFFFFFFFFu, h.mask, j);
+    u64 rj = gw * 32 + j;
+    if ((m >> lane) & 1u) {
+      u64 a = recs[rj].addr[lane];
+      u64 p = a >> 20;
+      if (p >= (1ull << 28)) {
+        set_err(err, ERR_OVERFLOW);
+      } else {
+        u32 bit = 1u << (p & 31);
+        u32* wp = &page_bits[p >> 5];
+        if (!(*(volatile u32*)wp & bit)) atomicOr(wp, bit);
+      }
+    }
+  }
+}
+
+// warp_start[w] = first index of warp w in the warp-sorted record list (lower bound)
+__global__ void k_warp_start(const u32* __restrict__ skeys, u64 n, u32 n_warps, u32* __restrict__ warp_start) {
+  u32 w = blockIdx.x * blockDim.x + threadIdx.x;
+  if (w > n_warps) return;
+  u64 lo = 0, hi = n;
+  while (lo < hi) {
+    u64 mid = (lo + hi) >> 1;
+    if (skeys[mid] < w) lo = mid + 1; else hi = mid;
+  }
+  warp_start[w] = (u32)lo;
+}
+
+// ---------------------------------------------------------------------------- k_replay
+// K2: compressed clock replay (Fig. 7, §4.3.1-4.3.2).  One thread per traced
+// warp walks the warp's records in trace order with the SIMT stack of Fig. 2 (K_w, P:L430-432,
+// P:L591-609).  Stack levels are branch-tree nodes: IF pushes the then-node (else-node is its
+// sibling, id+1, entered at ELSE); FI pops.  Every join-fork step (endi, if, else, fi, bar) is
+// labelled rec+1.  Per record it emits the snapshot {warp, ps, node, phase}; per IF the two
+// nodes {mask, parent, popen}; per BAR its record and the warp's next record (for the barrier
+// feasibility check) and a BARRIER_DIVERGENCE finding when the mask is not the full warp
+// (P:L639-644).
+__global__ void __launch_bounds__(128) k_replay(const bc_record* __restrict__ recs, const u32* __restrict__ wrec,
+                                                const u32* __restrict__ warp_start, Geo g,
+                                                const u32* __restrict__ node_base, const u32* __restrict__ bar_base,
+                                                uint4* __restrict__ snap, uint4* __restrict__ nodes,
+                                                u32* __restrict__ bar_rec, u32* __restrict__ bar_next,
+                                                u32* __restrict__ find_blk, u32* __restrict__ find_rec,
+                                                u32* __restrict__ find_cnt, u32* __restrict__ err) {
+  const u32 w = blockIdx.x * blockDim.x + threadIdx.x;
+  if (w >= g.n_warps) return;
+  const u32 imask = init_mask(g, w);
+  u32 st_node[33], st_mask[33];
+  u64 then_bits = 0;  // bit d set: level d is a then-node
+  int depth = 0;
+  st_node[0] = w;
+  st_mask[0] = imask;
+  nodes[w] = make_uint4(imask, NONE, 0u, 0u);
+  u32 ps = 0, phase = 0, nif = 0, nbar = 0;
+  bool need_next = false;
+  bool bad = false;
+  const u32 nb0 = node_base[w], bb0 = bar_base[w];
+  const u32 i0 = warp_start[w], i1 = warp_start[w + 1];
+  u32 rn = i0 < i1 ? wrec[i0] : 0;
+  uint4 hn = i0 < i1 ? __ldg(reinterpret_cast<const uint4*>(recs + rn)) : make_uint4(0, 0, 0, 0);
+  for (u32 i = i0; i < i1 && !bad; ++i) {
+    const u32 r = rn;
+    const uint4 hv = hn;
+    if (i + 1 < i1) {  // prefetch the next header
+      rn = wrec[i + 1];
+      hn = __ldg(reinterpret_cast<const uint4*>(recs + rn));
+    }
+    const u32 mask = hv.y, op = hv.z & 0xFFu, aux = hv.w;
+    if (need_next) {
+      bar_next[bb0 + nbar - 1] = r;
+      need_next = false;
+    }
+    snap[r] = make_uint4(w, ps, st_node[depth], phase);
+    if (mask != st_mask[depth]) {  // feasibility: record mask == K_w.peek()
+      bad = true;
+      break;
+    }
+    switch (op) {
+      case BC_OP_FENCE:
+        break;  // standalone fence: no trace operation (R14)
+      case BC_OP_IF: {
+        if (depth >= 32) { bad = true; break; }
+        u32 then = mask & aux;
+        u32 nid = nb0 + 2 * nif;
+        ++nif;
+        nodes[nid] = make_uint4(then, st_node[depth], ps, 0u);
+        nodes[nid + 1] = make_uint4(mask & ~then, st_node[depth], ps, 0u);
+        ++depth;
+        st_node[depth] = nid;
+        st_mask[depth] = then;
+        then_bits |= 1ull << depth;
+        ps = r + 1;
+        break;
+      }
+      case BC_OP_ELSE: {
+        if (depth == 0 || !((then_bits >> depth) & 1ull)) { bad = true; break; }
+        st_node[depth] += 1;
+        st_mask[depth] = st_mask[depth - 1] & ~st_mask[depth];
+        then_bits &= ~(1ull << depth);
+        ps = r + 1;
+        break;
+      }
+      case BC_OP_FI: {
+        if (depth == 0 || ((then_bits >> depth) & 1ull)) { bad = true; break; }
+        --depth;
+        ps = r + 1;
+        break;
+      }
+      case BC_OP_BAR: {
+        if (mask != imask) {  // barrier divergence; the barrier still completes (R10)
+          u32 at = atomicAdd(find_cnt, 1u);
+          find_blk[at] = w / g.wpb;
+          find_rec[at] = r;
+        }
+        bar_rec[bb0 + nbar] = r;
+        bar_next[bb0 + nbar] = NONE;
+        ++nbar;
+        ++phase;
+        need_next = true;
+        ps = r + 1;
+        break;
+      }
+      default:  // LD/ST/ATOM and ACQ/REL/AR: the record's endi(w) step
+        ps = r + 1;
+        break;
+    }
+  }
+  if (bad) set_err(err, ERR_INFEASIBLE);
+}
+
+// ---------------------------------------------------------------------------- k_barriers
+// Per block: every warp must arrive at every barrier exactly once (R10).  Barrier k completes
+// at the last arrival R_k = max over the block's warps of their k-th BAR record; its step is
+// labelled R_k + 1 for every thread of the block.  A warp whose next record after its k-th
+// BAR precedes R_k issued a record while waiting -> infeasible.
+__global__ void k_barriers(Geo g, const u32* __restrict__ bar_cnt, const u32* __restrict__ bar_base,
+                           const u32* __restrict__ bar_rec, const u32* __restrict__ bar_next,
+                           u32* __restrict__ blockR, u32* __restrict__ err) {
+  u32 b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b >= g.n_blocks) return;
+  u32 w0 = b * g.wpb;
+  u32 nb = bar_cnt[w0];
+  for (u32 i = 1; i < g.wpb; ++i)
+    if (bar_cnt[w0 + i] != nb) {
+      set_err(err, ERR_INFEASIBLE);
+      return;
+    }
+  for (u32 k = 0; k < nb; ++k) {
+    u32 R = 0, mn = NONE;
+    for (u32 i = 0; i < g.wpb; ++i) {
+      u32 bi = bar_base[w0 + i] + k;
+      R = max(R, bar_rec[bi]);
+      mn = min(mn, bar_next[bi]);
+    }
+    if (mn != NONE && mn < R) set_err(err, ERR_INFEASIBLE);
+    blockR[bar_base[w0] + k] = R + 1;
+  }
+}
+
+// ---------------------------------------------------------------------------- k_expand
+// K4: lowering of each LD / ST / ATOM warp record into one thread operation per active lane
+// and per shadow granule (R7), emitted as 8-byte items
+//   x = (dense granule key << 2) | op,   y = event = (record << 5) | lane
+// in trace order (the radix sort that follows is stable).  Dense keys: global granules of
+// written 1-MB pages first (page rank from the write bitmap, so keys follow address order),
+// then shared granules (block, offset).  Accesses to never-written global
+// pages cannot take part in a race (every race needs a write) and are dropped.
+// Also validates per-lane alignment / shared bounds for every op <= AR_GLB.
+// One warp per record, 8 warps x EXP_RPW records per tile, tile offsets by decoupled look-back.
+constexpr int EXP_RPW = 4;
+constexpr int EXP_TILE = 8 * EXP_RPW;
+
+__global__ void __launch_bounds__(256) k_expand(const bc_record* __restrict__ recs, Geo g,
+                                                const u32* __restrict__ page_bits,
+                                                const u32* __restrict__ page_rank, u32 shared_base,
+                                                u32* __restrict__ okeys, u32* __restrict__ oevs, u64* status,
+                                                u32* tile_counter,
+                                                u64* __restrict__ cnt, u32* __restrict__ err) {
+  __shared__ u32 s_tile;
+  __shared__ u32 s_rcnt[EXP_TILE];
+  __shared__ u64 s_base;
+  const int t = threadIdx.x, w = t >> 5, lane = t & 31;
+  if (t == 0) s_tile = atomicAdd(tile_counter, 1u);
+  __syncthreads();
+  const u64 tile = s_tile;
+  u32 key0[EXP_RPW], ngr[EXP_RPW], opc[EXP_RPW], incl[EXP_RPW];
+  bool bad = false;
+#pragma unroll
+  for (int j = 0; j < EXP_RPW; ++j) {
+    const u64 r = tile * EXP_TILE + w * EXP_RPW + j;
+    key0[j] = 0;
+    ngr[j] = 0;
+    opc[j] = 0;
+    if (r < g.n_recs) {
+      uint4 hv = __ldg(reinterpret_cast<const uint4*>(recs + r));
+      const u32 mask = hv.y, op = hv.z & 0xFFu, space = (hv.z >> 8) & 0xFFu, sl = (hv.z >> 16) & 0xFFu,
+                fl = (hv.z >> 24) & 0xFFu;
+      if (op <= BC_OP_AR_GLB && ((mask >> lane) & 1u) && sl <= 4 && space <= 1 && hv.x < g.n_warps) {
+        const u64 a = __ldg(&recs[r].addr[lane]);
+        const u64 size = 1ull << sl;
+        if (a & (size - 1)) bad = true;  // natural alignment
+        if (space == BC_SPACE_SHARED && a + size > g.smem) bad = true;
+        if (op <= BC_OP_ATOM && !bad) {
+          u32 n = (u32)(size >> g.G);
+          if (n == 0) n = 1;
+          opc[j] = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM : ((fl & BC_REC_SAME_VALUE) ? IOP_ST_SV : IOP_ST);
+          if (space == BC_SPACE_SHARED) {
+            u32 blk = hv.x / g.wpb;
+            key0[j] = shared_base + blk * g.smem_gran + (u32)(a >> g.G);
+            ngr[j] = n;
+          } else {
+            u64 p = a >> 20;
+            if (p < (1ull << 28)) {
+              u32 word = page_bits[p >> 5];
+              u32 bit = (u32)(p & 31);
+              if ((word >> bit) & 1u) {
+                u32 dense = page_rank[p >> 5] + __popc(word & ((1u << bit) - 1u));
+                key0[j] = (dense << (20 - g.G)) | (u32)((a & 0xFFFFFull) >> g.G);
+                ngr[j] = n;
+              }
+            } else {
+              set_err(err, ERR_OVERFLOW);
+            }
+          }
+        }
+      }
+    }
+    incl[j] = warp_incl_sum(ngr[j]);
+    if (lane == 31) s_rcnt[w * EXP_RPW + j] = incl[j];
+  }
+  if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
+  __syncthreads();
+  if (w == 0) {
+    u32 v = s_rcnt[lane];  // EXP_TILE == 32
+    u32 x = warp_incl_sum(v);
+    s_rcnt[lane] = x - v;
+    u32 total = __shfl_sync(0xFFFFFFFFu, x, 31);
+    if (lane == 0) s_base = lookback_u64(status, (u32)tile, total);
+    if (lane == 0 && (tile + 1) * EXP_TILE >= g.n_recs) {
+      // last tile: publish the item total
+      cnt[C_ITEMS] = s_base + total;
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < EXP_RPW; ++j) {
+    if (ngr[j] == 0) continue;
+    const u64 r = tile * EXP_TILE + w * EXP_RPW + j;
+    u64 o = s_base + s_rcnt[w * EXP_RPW + j] + incl[j] - ngr[j];
+    const u32 ev = (u32)(r << 5) | lane;
+    for (u32 k = 0; k < ngr[j]; ++k) {
+      okeys[o + k] = ((key0[j] + k) << 2) | opc[j];
+      oevs[o + k] = ev;
+    }
+  }
+}
+
+// page_rank[i] = number of set bits in page_bits[0..i)  (exclusive popcount scan input)
+__global__ void k_popc(const u32* __restrict__ bits, u32* __restrict__ out, u64 n) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) out[i] = __popc(bits[i]);
+}
+
+// --------------------------------------------------------------------- host launchers
+void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
+                   u32* sync_list, u32* page_bits, u64* cnt, u32* err, cudaStream_t st) {
+  u64 warps = (g.n_recs + 31) / 32;
+  if (warps == 0) return;
+  u64 blocks = (warps + 7) / 8;
+  k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt, err);
+}
+
+void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st) {
+  k_warp_start<<<(n_warps + 1 + 255) / 256, 256, 0, st>>>(skeys, n, n_warps, warp_start);
+}
+
+void launch_replay(const bc_record* recs, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
+                   const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next, u32* find_blk,
+                   u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st) {
+  k_replay<<<(g.n_warps + 127) / 128, 128, 0, st>>>(recs, wrec, warp_start, g, node_base, bar_base, snap, nodes,
+                                                     bar_rec, bar_next, find_blk, find_rec, find_cnt, err);
+}
+
+void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, const u32* bar_rec, const u32* bar_next,
+                     u32* blockR, u32* err, cudaStream_t st) {
+  k_barriers<<<(g.n_blocks + 127) / 128, 128, 0, st>>>(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err);
+}
+
+void launch_popc(const u32* bits, u32* out, u64 n, cudaStream_t st) {
+  k_popc<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(bits, out, n);
+}
+
+u64 expand_tiles(u64 n_recs) { return (n_recs + EXP_TILE - 1) / EXP_TILE; }
+
+void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
+                   u32* keys, u32* evs, u64* status, u32* tile_counter, u64* cnt, u32* err, cudaStream_t st) {
+  u64 tiles = expand_tiles(g.n_recs);
+  if (tiles == 0) return;
+  k_expand<<<(unsigned)tiles, 256, 0, st>>>(recs, g, page_bits, page_rank, shared_base, keys, evs, status,
+                                           tile_counter, cnt, err);
+}
+
+__global__ void k_node_base(const u32* __restrict__ if_excl, u32 n_warps, u32* __restrict__ node_base) {
+  u32 w = blockIdx.x * blockDim.x + threadIdx.x;
+  if (w < n_warps) node_base[w] = n_warps + 2u * if_excl[w];
+}
+void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st) {
+  k_node_base<<<(n_warps + 255) / 256, 256, 0, st>>>(if_excl, n_warps, node_base);
+}
+
+}  // namespace bc

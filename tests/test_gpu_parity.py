@@ -1,0 +1,268 @@
+"""Parity of the CUDA path (through the C ABI) with the CPU oracle — element by element.
+
+Bar (BASELINE.json north_star): the race set is bit-identical — same granule
+addresses, same (prior, current) event pairs, same kind / class / space / block, same
+canonical order — and the status (OK / INFEASIBLE) is the same.  All values are integers.
+Cases: the paper's worked examples (Fig. 1, Fig. 4), the C1 litmus config, the 66-trace
+suite, seeded random feasible traces (nested branches, barrier divergence, block / global
+acquire-release, vector accesses, several granule sizes), an exhaustive tiny family,
+infeasible traces, and C2-C5 at sizes the oracle finishes in seconds (several tiles and a
+ragged tail) plus C2 at full size.
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+import bcgen
+import oracle
+import paper_conf_pldi_eizenbergppmd17_b200 as bc
+from bcgen import GLOBAL_BASE, TraceBuilder
+from bcgen.configs import ConfigPlan
+from bcgen.fuzz import random_trace
+
+import litmus
+
+pytestmark = pytest.mark.gpu
+
+
+def _gpu(recs, geom, flags=0):
+    return bc.detect(recs, geom, device="cuda:0", flags=flags)
+
+
+def assert_parity(recs, geom, flags=0, expect_status=None):
+    st_o, want, stats_o = oracle.detect_geom(recs, geom, flags)
+    res = _gpu(recs, geom, flags)
+    assert res.status == st_o, (res.status, st_o)
+    if expect_status is not None:
+        assert st_o == expect_status
+    if st_o != 0:
+        return want, res
+    got = res.races
+    assert len(got) == len(want), (len(got), len(want), got[:4], want[:4])
+    assert np.array_equal(got.view(np.uint8), want.view(np.uint8)), _first_diff(got, want)
+    assert res.stats["lane_events"] == stats_o["lane_events"]
+    assert res.stats["control_events"] == stats_o["control_events"]
+    return want, res
+
+
+def _first_diff(got, want):
+    for i, (a, b) in enumerate(zip(got, want)):
+        if a.tobytes() != b.tobytes():
+            return i, a, b
+    return None
+
+
+# ------------------------------------------------------------------ paper examples
+def test_c1_litmus():
+    recs, tb = bcgen.configs.make_c1()
+    want, res = assert_parity(recs, tb.geom.as_dict())
+    assert len(want) == 1
+    recs, tb = bcgen.configs.make_c1(with_sync=False)
+    want, res = assert_parity(recs, tb.geom.as_dict())
+    assert len(want) == 33
+
+
+def test_fig4_message_passing():
+    x, y = GLOBAL_BASE, GLOBAL_BASE + 0x100000
+    for rel, acq in itertools.product(("blk", "glb"), repeat=2):
+        tb = TraceBuilder(grid=(2,), block=(1,))
+        tb.st(0, x)
+        tb.rel(0, y, scope=rel)
+        tb.acq(1, y, scope=acq)
+        tb.ld(1, x)
+        want, _ = assert_parity(tb.records(), tb.geom.as_dict())
+        assert len(want) == (1 if (rel, acq) == ("blk", "blk") else 0)
+
+
+def test_fig1_translation():
+    a, b, d = GLOBAL_BASE, GLOBAL_BASE + 0x100, GLOBAL_BASE + 0x200
+    tb = TraceBuilder(block=(2,))
+    tb.ld(0, a); tb.if_(0, [0]); tb.st(0, b); tb.else_(0); tb.fi(0); tb.rel(0, d, scope="blk")
+    assert_parity(tb.records(), tb.geom.as_dict())
+
+
+@pytest.mark.parametrize("entry", litmus.SUITE, ids=[e[0] for e in litmus.SUITE])
+def test_litmus_suite(entry):
+    name, fn, expected, opts = entry
+    tb = fn()
+    want, res = assert_parity(tb.records(), tb.geom.as_dict())
+    got = sorted((int(r["kind"]), int(r["cls"]), int(r["space"])) for r in res.races)
+    assert got == expected
+
+
+def test_same_value_flag():
+    tb = TraceBuilder(block=(32,))
+    tb.st(0, lambda l: GLOBAL_BASE if l < 3 else GLOBAL_BASE + 4 * l, same_value=True)
+    assert_parity(tb.records(), tb.geom.as_dict())
+    want, _ = assert_parity(tb.records(), tb.geom.as_dict(), flags=oracle.F_NO_SAME_VALUE_FILTER)
+    assert len(want) == 2
+
+
+# ------------------------------------------------------------------ random traces
+@pytest.mark.parametrize("chunk", range(6))
+def test_random_traces(chunk):
+    for seed in range(chunk * 50, chunk * 50 + 50):
+        recs, tb = random_trace(seed)
+        assert_parity(recs, tb.geom.as_dict())
+
+
+@pytest.mark.parametrize("G", [0, 1, 3, 4])
+def test_random_traces_granules(G):
+    for seed in range(2000, 2030):
+        recs, tb = random_trace(seed, granule_log2=G)
+        assert_parity(recs, tb.geom.as_dict())
+
+
+def test_random_traces_big_blocks():
+    for seed in range(3000, 3012):
+        recs, tb = random_trace(seed, max_blocks=6, tpb=256, ops_per_warp=(10, 40), n_glob=6, n_sync=3)
+        assert_parity(recs, tb.geom.as_dict())
+
+
+def test_random_traces_same_value():
+    for seed in range(4000, 4030):
+        recs, tb = random_trace(seed, same_value=True)
+        assert_parity(recs, tb.geom.as_dict())
+        assert_parity(recs, tb.geom.as_dict(), flags=oracle.F_NO_SAME_VALUE_FILTER)
+
+
+def test_exhaustive_sample():
+    """Every 5th program of the exhaustive 2-warp x 2-lane family of test_oracle_pins."""
+    from test_oracle_pins import _alphabet
+    ops, addr, s = _alphabet()
+    orders = [o for o in itertools.product([0, 1], repeat=4) if sum(o) == 2]
+    k = 0
+    for p0 in itertools.product(range(len(ops)), repeat=2):
+        for p1 in itertools.product(range(len(ops)), repeat=2):
+            for order in orders:
+                k += 1
+                if k % 5:
+                    continue
+                tb = TraceBuilder(grid=(2,), block=(2,))
+                pcs = [0, 0]
+                progs = [p0, p1]
+                for w in order:
+                    kind, pat = ops[progs[w][pcs[w]]]
+                    pcs[w] += 1
+                    if kind == "rel":
+                        tb.rel(w, s)
+                    elif kind == "acq":
+                        tb.acq(w, s)
+                    elif kind == "br":
+                        tb.if_(w, [0]); tb.st(w, addr(0)); tb.else_(w); tb.ld(w, addr(0)); tb.fi(w)
+                    else:
+                        getattr(tb, kind)(w, addr(pat))
+                assert_parity(tb.records(), tb.geom.as_dict())
+
+
+# ------------------------------------------------------------------ infeasible / edge
+def _infeasible():
+    from test_oracle_pins import _infeasible_traces
+    return _infeasible_traces()
+
+
+@pytest.mark.parametrize("case", _infeasible(), ids=lambda c: c[0])
+def test_infeasible(case):
+    name, tb = case
+    assert_parity(tb.records(), tb.geom.as_dict(), expect_status=oracle.INFEASIBLE)
+
+
+def test_empty_trace():
+    recs = np.zeros(0, dtype=bcgen.RECORD_DTYPE)
+    res = _gpu(recs, dict(grid=(1,), block=(32,), smem_bytes=0))
+    assert res.status == 0 and len(res.races) == 0
+
+
+def test_control_only_trace():
+    tb = TraceBuilder(block=(64,))
+    tb.fence(0); tb.bar(0); tb.bar(1); tb.if_(1, 0); tb.else_(1); tb.fi(1)
+    assert_parity(tb.records(), tb.geom.as_dict())
+
+
+def test_depth_32():
+    tb = TraceBuilder(block=(32,))
+    for _ in range(32):
+        tb.if_(0, 0xFFFFFFFF)
+    tb.st(0, lambda l: GLOBAL_BASE + 4 * (l // 2))
+    for _ in range(32):
+        tb.else_(0); tb.fi(0)
+    tb.ld(0, lambda l: GLOBAL_BASE + 4 * ((l + 1) % 16))
+    assert_parity(tb.records(), tb.geom.as_dict())
+
+
+def test_hot_granule_long_segment():
+    """One granule touched by thousands of reads and writes from many warps / blocks: the
+    segment spans many K7 tiles (look-back carries), with inflated read vectors."""
+    tb = TraceBuilder(grid=(4,), block=(256,))
+    hot = GLOBAL_BASE + 0x40
+    import random
+    rng = random.Random(7)
+    for it in range(60):
+        for b in range(4):
+            for wib in range(8):
+                w = tb.warp(b, wib)
+                r = rng.random()
+                if r < 0.7:
+                    tb.ld(w, hot)
+                elif r < 0.85:
+                    tb.atom(w, hot)
+                else:
+                    tb.st(w, lambda l: hot if l == rng.randrange(32) else GLOBAL_BASE + 0x1000 + 4 * l)
+    want, _ = assert_parity(tb.records(), tb.geom.as_dict())
+    assert len(want) > 100
+
+
+# ------------------------------------------------------------------ configs
+@pytest.mark.parametrize("cfg,kw", [
+    (2, dict(n_blocks=8, iters=6)),
+    (2, dict(n_blocks=5, iters=3, tpb=96)),
+    (3, dict(n_blocks=16, iters=2, tpb=64)),
+    (3, dict(n_blocks=9, iters=3, tpb=256)),
+    (4, dict(n_blocks=12, log2_nodes=14, nodes_per_thread=2, inj_scale=4)),
+    (4, dict(n_blocks=40, log2_nodes=16, nodes_per_thread=3, inj_scale=8)),
+    (5, dict(n_blocks=8, log2_nodes=15, nodes_per_thread=3, inj_scale=4)),
+])
+def test_configs_reduced(cfg, kw):
+    plan = ConfigPlan(cfg, **kw)
+    recs = plan.records()
+    want, res = assert_parity(recs, plan.geometry)
+    if cfg in (4, 5):
+        truth = plan.truth()
+        assert np.array_equal(np.sort(want.view("V32")), np.sort(truth.view("V32")))
+
+
+def test_c3_64_blocks():
+    plan = ConfigPlan(3, n_blocks=64)
+    assert_parity(plan.records(), plan.geometry)
+
+
+def test_c4_64_blocks():
+    plan = ConfigPlan(4, n_blocks=64)
+    assert_parity(plan.records(), plan.geometry)
+
+
+@pytest.mark.slow
+def test_c2_full_size():
+    plan = ConfigPlan(2)
+    want, res = assert_parity(plan.records(), plan.geometry)
+    assert len(want) == 0 and res.stats["lane_events"] > 9_000_000
+
+
+# ------------------------------------------------------------------ API behaviour
+def test_device_borrowed_trace_and_idempotent():
+    import torch
+    recs, tb = bcgen.configs.make_c1(with_sync=False)
+    geom = tb.geom.as_dict()
+    st, want, _ = oracle.detect_geom(recs, geom)
+    dev = torch.from_numpy(recs.view(np.uint8).copy()).cuda()
+    with bc.Context(geom, device=0) as ctx:
+        ctx.load_trace(dev)
+        for _ in range(3):
+            st2, stats = ctx.detect()
+            assert st2 == 0
+            got = ctx.races()
+            assert np.array_equal(got.view(np.uint8), want.view(np.uint8))
+        out = torch.zeros(len(want) * 32, dtype=torch.uint8, device="cuda")
+        assert ctx.races_device(out) == len(want)
+        assert np.array_equal(out.cpu().numpy(), want.view(np.uint8))
