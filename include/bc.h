@@ -116,8 +116,10 @@ typedef struct bc_stats {
   uint64_t races, findings;  /* race records / barrier-divergence findings                       */
   uint64_t sync_ops;         /* acquire / release lane operations                                 */
   uint64_t written_pages;    /* 1-MB global pages with at least one write          */
+  uint64_t kernel_launches;  /* libbc kernels launched by this bc_detect                          */
   float ms_total;            /* device time of bc_detect (cudaEvents on the stream)               */
-  float ms_kernel[12];       /* per phase, see bc_phase_name()                                   */
+  float ms_kernel[12];       /* per phase, then kernel-only k_check / k_sort_items / k_expand;
+                                see bc_phase_name()                                              */
 } bc_stats;
 
 /* ------------------------------------------------------------------------- calls */

@@ -14,6 +14,10 @@
 
 using namespace bc;
 
+namespace bc {
+u64 g_launches = 0;
+}
+
 struct bc_ctx {
   bc_config cfg;
   Geo g;
@@ -34,7 +38,7 @@ struct bc_ctx {
 };
 
 static const char* kPhase[] = {"header", "partition", "replay", "sync", "expand", "sort", "check", "finalize",
-                               nullptr};
+                               "k_check", "k_sort_items", "k_expand", nullptr};
 enum { PH_HEADER = 0, PH_PARTITION, PH_REPLAY, PH_SYNC, PH_EXPAND, PH_SORT, PH_CHECK, PH_FINALIZE, PH_N };
 
 static bc_status fail(bc_ctx* c, bc_status s, const std::string& msg) {
@@ -73,7 +77,7 @@ const char* bc_status_string(bc_status s) {
 
 const char* bc_last_error(const bc_ctx* c) { return c ? c->err.c_str() : "null context"; }
 
-const char* bc_phase_name(int i) { return (i >= 0 && i < PH_N) ? kPhase[i] : nullptr; }
+const char* bc_phase_name(int i) { return (i >= 0 && i < PH_N + 3) ? kPhase[i] : nullptr; }
 
 bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   if (!cfg || !out) return BC_ERR_INVALID_ARG;
@@ -184,6 +188,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   memset(&sx, 0, sizeof(sx));
   sx.records = n;
   c->n_races = 0;
+  const u64 launches0 = g_launches;
   cudaEventRecord(c->ev[0], st);
   if (n == 0) {
     cudaEventRecord(c->ev[PH_N], st);
@@ -258,16 +263,18 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   launch_replay(recs, wrec, warp_start, g, node_base, bar_base, snap, nodes, bar_rec, bar_next, find_blk, find_rec,
                 find_cnt, err, st);
   launch_barriers(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err, st);
+  launch_snap_blab(snap, n, g.wpb, g.n_warps, n_bar, bar_base, blockR, st);
   cudaEventRecord(c->ev[3], st);
   bc_status cs = cuda_check(c, "replay");
   if (cs) return cs;
+  cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
+  if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "replay");
+  if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "SIMT stack / barrier feasibility");
 
   HbCtx hc{};
   hc.g = g;
   hc.snap = snap;
   hc.nodes = nodes;
-  hc.bar_base = bar_base;
-  hc.blockR = blockR;
   hc.err = err;
   hc.n_acq = 0;
   hc.n_idx = 0;
@@ -287,7 +294,9 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* ecounter = S.alloc<u32>(1);
   cudaMemsetAsync(estatus, 0, (tiles + 1) * 8, st);
   cudaMemsetAsync(ecounter, 0, 4, st);
+  cudaEventRecord(c->ev[14], st);
   launch_expand(recs, g, page_bits, page_rank, shared_base, ikeys, ievs, estatus, ecounter, cnt, err, st);
+  cudaEventRecord(c->ev[15], st);
   u64 n_items = 0;
   u32 nfind = 0;
   cudaMemcpyAsync(&n_items, cnt + C_ITEMS, 8, cudaMemcpyDeviceToHost, st);
@@ -302,7 +311,10 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* ik2 = S.alloc<u32>(n_items + 1);
   u32* iv2 = S.alloc<u32>(n_items + 1);
   int kbits = bits_for(n_keys ? n_keys - 1 : 0);
-  alt = radix_sort_pairs(ikeys, ievs, ik2, iv2, n_items, 2, 2 + kbits, S.alloc<char>(rs_temp_bytes(n_items)), st);
+  void* rtmp = S.alloc<char>(rs_temp_bytes(n_items));
+  cudaEventRecord(c->ev[12], st);
+  alt = radix_sort_pairs(ikeys, ievs, ik2, iv2, n_items, 2, 2 + kbits, rtmp, st);
+  cudaEventRecord(c->ev[13], st);
   u32* skey = alt ? ik2 : ikeys;
   u32* sev = alt ? iv2 : ievs;
   cudaEventRecord(c->ev[6], st);
@@ -319,7 +331,9 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     cudaMemsetAsync(rcnt, 0, 4, st);
     cudaMemsetAsync(segc, 0, 8, st);
     cudaMemsetAsync(err, 0, 4, st);
+    cudaEventRecord(c->ev[10], st);
     launch_check(hc, skey, sev, n_items, cstatus, ccounter, rbuf, rcnt, race_cap, segc, st);
+    cudaEventRecord(c->ev[11], st);
     cudaMemcpyAsync(&n_r, rcnt, 4, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&sx.segments, segc, 8, cudaMemcpyDeviceToHost, st);
@@ -356,6 +370,13 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     cudaEvent_t e1 = i + 1 < PH_N ? c->ev[i + 1] : c->ev[PH_N];
     cudaEventElapsedTime(&sx.ms_kernel[i], c->ev[i], e1);
   }
+  // kernel-only timings of the three heavy kernels (no host gaps inside)
+  if (n_items) {
+    cudaEventElapsedTime(&sx.ms_kernel[PH_N + 0], c->ev[10], c->ev[11]);
+    cudaEventElapsedTime(&sx.ms_kernel[PH_N + 1], c->ev[12], c->ev[13]);
+  }
+  cudaEventElapsedTime(&sx.ms_kernel[PH_N + 2], c->ev[14], c->ev[15]);
+  sx.kernel_launches = g_launches - launches0;
   return BC_OK;
 }
 

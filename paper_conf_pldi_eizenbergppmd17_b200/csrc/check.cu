@@ -94,53 +94,114 @@ __device__ __forceinline__ void emit(const CheckArgs& a, u32 key, u32 cur, u32 p
   if (at < a.race_cap) a.races[at] = make_uint4(key, cur, prior, kind);
 }
 
-// lazily loaded snapshot of the current item's record
-struct Cur {
-  u32 ev, rec, lane;
-  bool have;
-  Snap s;
-};
-__device__ __forceinline__ const Snap& cur_snap(const CheckArgs& a, Cur& cu) {
-  if (!cu.have) {
-    cu.s = load_snap(a.c.snap, cu.rec);
-    cu.have = true;
+// the analysis context of the running K7 launch (set by launch_check; one K7 at a time)
+__constant__ HbCtx cHC;
+
+// slow path of the happens-before query: divergent intra-warp walk and foreign knowledge
+static __device__ __noinline__ bool hb_slow(u32 ev1, u32 w1, u32 ev2, u32 s2w, u32 s2ps, u32 s2node, u32 s2blab) {
+  const Snap s2{s2w, s2ps, s2node, s2blab};
+  return hb(cHC, ev1 >> 5, ev1 & 31u, w1, ev2 >> 5, ev2 & 31u, s2);
+}
+
+// happens-before of event ev1 (by warp w1) before event ev2 whose record snapshot is s2.
+// Inline fast path: same record / same thread / barrier label / converged warp.
+__device__ __forceinline__ bool hb_ev(const HbCtx& c, u32 ev1, u32 w1, u32 ev2, const Snap& s2) {
+  const u32 r1 = ev1 >> 5, r2 = ev2 >> 5, l1 = ev1 & 31u, l2 = ev2 & 31u;
+  if (r1 == r2) return l1 == l2;                 // lanes of one instruction are concurrent
+  if (w1 == s2.warp) {
+    if (l1 == l2) return true;                   // program order
+    if (s2.node == s2.warp && s2.ps >= r1 + 1u) return true;  // converged warp, endi join
   }
-  return cu.s;
-}
-__device__ __forceinline__ bool hb_ev(const CheckArgs& a, u32 ev1, Cur& cu) {
-  u32 r1 = ev1 >> 5, l1 = ev1 & 31u;
-  if (r1 == cu.rec) return l1 == cu.lane;
-  const Snap& s2 = cur_snap(a, cu);
-  u32 w1 = __ldg(&a.c.snap[r1].x);
-  return hb(a.c, r1, l1, w1, cu.rec, cu.lane, s2);
+  const bool sameb = (w1 / c.g.wpb) == (s2.warp / c.g.wpb);
+  if (sameb && r1 + 1u <= s2.blab) return true;  // completed barrier (Fig. 3 BAR)
+  if (c.n_acq == 0 && !(w1 == s2.warp && s2.node != s2.warp)) return false;
+  return hb_slow(ev1, w1, ev2, s2.warp, s2.ps, s2.node, s2.blab);
 }
 
-// thread identity of an event (warp << 5 | lane)
-__device__ __forceinline__ u32 ev_tid(const CheckArgs& a, u32 ev) { return (__ldg(&a.c.snap[ev >> 5].x) << 5) | (ev & 31u); }
-
-// R_x is a vector clock at writer `cu` (index i): entries = latest read per thread among items
-// [lo, hi] (all reads of this granule).  Check each entry (Fig. 2 WRITESHARED, Fig. 3 *ATOMSHARED).
-__device__ __noinline__ void vc_check(const CheckArgs& a, u64 lo, u64 hi, Cur& cu, u32 key, u32 kind) {
+// R_x is a vector clock at writer (ev2, s2): its entries are the latest read per thread among
+// items [lo, hi] (all reads of this granule).  Check each (Fig. 2 WRITESHARED, Fig. 3 *ATOMSHARED).
+static __device__ __noinline__ void vc_check(const u32* __restrict__ evs, uint4* races, u32* race_cnt, u32 race_cap,
+                                             u64 lo, u64 hi, u32 ev2, u32 s2w, u32 s2ps, u32 s2node, u32 s2blab,
+                                             u32 key, u32 kind) {
+  const Snap s2{s2w, s2ps, s2node, s2blab};
+  const HbCtx& c = cHC;
   u32 seen[32];
   int ns = 0;
   for (u64 j = hi + 1; j-- > lo;) {
-    u32 ev = a.evs[j];
-    u32 tid = ev_tid(a, ev);
+    u32 ev = evs[j];
+    u32 w1 = __ldg(&c.snap[ev >> 5].x);
+    u32 tid = (w1 << 5) | (ev & 31u);
     bool dup = false;
     for (int q = 0; q < ns; ++q)
       if (seen[q] == tid) { dup = true; break; }
     if (!dup && ns == 32) {
       // overflow of the small set: look for a later read of the same thread directly
-      for (u64 q = j + 1; q <= hi; ++q)
-        if (ev_tid(a, a.evs[q]) == tid) { dup = true; break; }
+      for (u64 q = j + 1; q <= hi; ++q) {
+        u32 e2 = evs[q];
+        if (((__ldg(&c.snap[e2 >> 5].x) << 5) | (e2 & 31u)) == tid) { dup = true; break; }
+      }
     }
     if (dup) continue;
     if (ns < 32) seen[ns++] = tid;
-    if (!hb_ev(a, ev, cu)) emit(a, key, cu.ev, ev, kind);
+    if (!hb(c, ev >> 5, ev & 31u, w1, ev2 >> 5, ev2 & 31u, s2)) {
+      u32 at = atomicAdd(race_cnt, 1u);
+      if (at < race_cap) races[at] = make_uint4(key, ev2, ev, kind);
+    }
   }
 }
 
+// warp 0: exclusive prefix of this tile from its predecessors' published summaries,
+// 32 predecessors per round (decoupled look-back, non-commutative combine in tile order).
+__device__ __forceinline__ Sum warp_lookback(TileStatus* status, u32 tile, const Sum& agg, int lane) {
+  if (tile == 0) {
+    if (lane == 0) publish(&status[0], agg, 2u);
+    return sum_ident();
+  }
+  if (lane == 0) publish(&status[tile], agg, 1u);
+  Sum P = sum_ident();
+  int hi = (int)tile - 1;
+  while (true) {
+    int idx = hi - lane;  // lane 0 = nearest predecessor
+    u32 f = 2u;
+    Sum s = sum_ident();
+    if (idx >= 0) {
+      f = ((volatile TileStatus*)&status[idx])->flag;
+    }
+    // all lanes spin together until every inspected predecessor has published
+    while (__any_sync(0xFFFFFFFFu, f == 0u)) {
+      if (f == 0u) f = ((volatile TileStatus*)&status[idx])->flag;
+    }
+    __threadfence();
+    if (idx >= 0) {
+      volatile TileStatus* v = &status[idx];
+      s = Sum{v->fk, v->lk, v->lw, v->fi, v->bits};
+    }
+    u32 incm = __ballot_sync(0xFFFFFFFFu, idx >= 0 && f == 2u);
+    int last = incm ? (__ffs(incm) - 1) : 31;  // nearest inclusive predecessor ends this round
+    if (hi - last < 0) last = hi;                // fewer than 32 tiles left (tile 0 is inclusive)
+    // P = combine(s[last], ..., s[1], s[0], P)
+    Sum acc = sum_ident();
+    for (int k = last; k >= 0; --k) {
+      Sum sk;
+      sk.fk = __shfl_sync(0xFFFFFFFFu, s.fk, k);
+      sk.lk = __shfl_sync(0xFFFFFFFFu, s.lk, k);
+      sk.lw = __shfl_sync(0xFFFFFFFFu, s.lw, k);
+      sk.fi = __shfl_sync(0xFFFFFFFFu, s.fi, k);
+      sk.bits = __shfl_sync(0xFFFFFFFFu, s.bits, k);
+      acc = combine(acc, sk);
+    }
+    P = combine(acc, P);
+    if (incm) break;
+    hi -= 32;
+  }
+  if (lane == 0) publish(&status[tile], combine(P, agg), 2u);
+  return P;
+}
+
 __global__ void __launch_bounds__(CK_THREADS) k_check(CheckArgs a) {
+  __shared__ u32 s_kx[CK_TILE];
+  __shared__ u32 s_ev[CK_TILE];
+  __shared__ u32 s_w[CK_TILE];
   __shared__ u32 s_tile;
   __shared__ Sum s_wt[CK_THREADS / 32];
   __shared__ Sum s_prefix;
@@ -152,52 +213,66 @@ __global__ void __launch_bounds__(CK_THREADS) k_check(CheckArgs a) {
   }
   __syncthreads();
   const u32 tile = s_tile;
-  const u64 base = (u64)tile * CK_TILE + (u64)t * CK_IPT;
+  const u64 tbase = (u64)tile * CK_TILE;
+  const u64 base = tbase + (u64)t * CK_IPT;
+  const HbCtx& c = a.c;
 
+  // ---- A: items + their records' snapshots (all gathers in flight together)
   u32 kx[CK_IPT], ev[CK_IPT];
-  u32 infl = 0;  // bit j: item j is a read that found its predecessor read unordered (READINFLATE)
-  u32 segs = 0;
-  u32 pk = NONE, pop = 0, pev = 0;  // previous item
-  if (base > 0 && base - 1 < a.n) {
-    pk = a.keys[base - 1];
-    pev = a.evs[base - 1];
-    pop = pk & 3u;
-    pk >>= 2;
-  }
+  uint4 sn[CK_IPT];
 #pragma unroll
   for (int j = 0; j < CK_IPT; ++j) {
     u64 i = base + j;
-    if (i < a.n) {
-      kx[j] = a.keys[i];
-      ev[j] = a.evs[i];
+    kx[j] = i < a.n ? a.keys[i] : NONE;
+    ev[j] = i < a.n ? a.evs[i] : 0u;
+  }
+#pragma unroll
+  for (int j = 0; j < CK_IPT; ++j) sn[j] = base + j < a.n ? __ldg(c.snap + (ev[j] >> 5)) : make_uint4(0, 0, 0, 0);
+  // previous item (the last item of thread t-1, or the item before the tile)
+  u32 pkx = __shfl_up_sync(0xFFFFFFFFu, kx[CK_IPT - 1], 1);
+  u32 pev = __shfl_up_sync(0xFFFFFFFFu, ev[CK_IPT - 1], 1);
+  u32 pw = __shfl_up_sync(0xFFFFFFFFu, sn[CK_IPT - 1].x, 1);
+  if (lane == 0) {
+    if (base > 0 && base - 1 < a.n) {
+      pkx = a.keys[base - 1];
+      pev = a.evs[base - 1];
+      pw = __ldg(&c.snap[pev >> 5].x);
     } else {
-      kx[j] = NONE;
-      ev[j] = 0;
+      pkx = NONE;
     }
   }
+#pragma unroll
+  for (int j = 0; j < CK_IPT; ++j) {
+    s_kx[t * CK_IPT + j] = kx[j];
+    s_ev[t * CK_IPT + j] = ev[j];
+    s_w[t * CK_IPT + j] = sn[j].x;
+  }
+
+  // ---- B: READINFLATE flags (a read whose predecessor read of the granule is unordered)
+  u32 infl = 0, segs = 0;
   Sum mine = sum_ident();
 #pragma unroll
   for (int j = 0; j < CK_IPT; ++j) {
-    u64 i = base + j;
-    if (i >= a.n) break;
-    u32 key = kx[j] >> 2, op = kx[j] & 3u;
-    if (key != pk) ++segs;
-    if (op == IOP_LD && key == pk && pop == IOP_LD) {
-      Cur cu{ev[j], ev[j] >> 5, ev[j] & 31u, false, Snap{}};
-      if (!hb_ev(a, pev, cu)) infl |= 1u << j;
+    const u64 i = base + j;
+    const u32 qkx = j ? kx[j - 1] : pkx;
+    const u32 qev = j ? ev[j - 1] : pev;
+    const u32 qw = j ? sn[j - 1].x : pw;
+    if (i < a.n) {
+      const u32 key = kx[j] >> 2, op = kx[j] & 3u;
+      const bool same = qkx != NONE && (qkx >> 2) == key;
+      if (!same) ++segs;
+      if (op == IOP_LD && same && (qkx & 3u) == IOP_LD && !hb_ev(c, qev, qw, ev[j], to_snap(sn[j]))) infl |= 1u << j;
+      Sum it;
+      it.fk = key;
+      it.lk = key;
+      it.lw = op != IOP_LD ? (u32)i + 1u : 0u;
+      it.fi = ((infl >> j) & 1u) ? (u32)i : NONE;
+      it.bits = 1u | (op != IOP_LD ? 2u : 0u);
+      mine = combine(mine, it);
     }
-    Sum it;
-    it.fk = key;
-    it.lk = key;
-    it.lw = op != IOP_LD ? (u32)i + 1u : 0u;
-    it.fi = ((infl >> j) & 1u) ? (u32)i : NONE;
-    it.bits = 1u | (op != IOP_LD ? 2u : 0u);
-    mine = combine(mine, it);
-    pk = key;
-    pop = op;
-    pev = ev[j];
   }
-  // block scan of thread summaries
+
+  // ---- C: block scan of thread summaries + look-back across tiles
   Sum incl = mine;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
@@ -209,91 +284,77 @@ __global__ void __launch_bounds__(CK_THREADS) k_check(CheckArgs a) {
   if (lane == 31) s_wt[w] = incl;
   if (segs) atomicAdd(&s_segs, segs);
   __syncthreads();
-  Sum wp = sum_ident();
-  for (int ww = 0; ww < w; ++ww) wp = combine(wp, s_wt[ww]);
-  if (t == 0) {
+  if (w == 0) {
     Sum agg = sum_ident();
     for (int ww = 0; ww < CK_THREADS / 32; ++ww) agg = combine(agg, s_wt[ww]);
-    Sum P = sum_ident();
-    if (tile == 0) {
-      publish(&a.status[0], agg, 2u);
-    } else {
-      publish(&a.status[tile], agg, 1u);
-      int pt = (int)tile - 1;
-      while (true) {
-        volatile TileStatus* v = &a.status[pt];
-        u32 f = v->flag;
-        if (f == 0) continue;
-        __threadfence();
-        Sum s{v->fk, v->lk, v->lw, v->fi, v->bits};
-        P = combine(s, P);
-        if (f == 2u) break;
-        --pt;
-      }
-      publish(&a.status[tile], combine(P, agg), 2u);
+    Sum P = warp_lookback(a.status, tile, agg, lane);
+    if (lane == 0) {
+      s_prefix = P;
+      if (s_segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)s_segs);
     }
-    s_prefix = P;
-    if (s_segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)s_segs);
   }
+  Sum wp = sum_ident();
+  for (int ww = 0; ww < w; ++ww) wp = combine(wp, s_wt[ww]);
   __syncthreads();
-  Sum st = combine(s_prefix, combine(wp, excl));
+  const Sum st = combine(s_prefix, combine(wp, excl));
 
-  // per-item checks with the exact incoming state
-  const u32 no_sv = a.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
+  // ---- D: per-item checks with the exact incoming state
+  const u32 no_sv = c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   u32 lk = st.lk, lw = st.lw, fi = st.fi;
-  if (base > 0 && base - 1 < a.n) {
-    pk = a.keys[base - 1];
-    pev = a.evs[base - 1];
-    pop = pk & 3u;
-    pk >>= 2;
-  } else {
-    pk = NONE;
-  }
-#pragma unroll 1
+#pragma unroll
   for (int j = 0; j < CK_IPT; ++j) {
-    u64 i = base + j;
-    if (i >= a.n) break;
-    u32 key = kx[j] >> 2, op = kx[j] & 3u;
-    if (key != lk) {
-      lk = key;
-      lw = 0;
-      fi = NONE;
-    }
-    Cur cu{ev[j], ev[j] >> 5, ev[j] & 31u, false, Snap{}};
-    // W_x check (every rule of Fig. 2; atomics only against a plain last write)
-    if (lw) {
-      u32 pk2 = a.keys[lw - 1], pev2 = a.evs[lw - 1];
-      bool patm = (pk2 & 3u) == IOP_ATOM;
-      if (op == IOP_LD) {
-        if (!hb_ev(a, pev2, cu)) emit(a, key, cu.ev, pev2, patm ? BC_KIND_AR : BC_KIND_WR);
-      } else if (op == IOP_ATOM) {
-        if (!patm && !hb_ev(a, pev2, cu)) emit(a, key, cu.ev, pev2, BC_KIND_WA);
-      } else {
-        if (!hb_ev(a, pev2, cu)) {
-          bool filtered = !patm && op == IOP_ST_SV && !no_sv && (pev2 >> 5) == cu.rec;
-          if (!filtered) emit(a, key, cu.ev, pev2, patm ? BC_KIND_AW : BC_KIND_WW);
+    const u64 i = base + j;
+    if (i < a.n) {
+      const u32 key = kx[j] >> 2, op = kx[j] & 3u;
+      const Snap s2 = to_snap(sn[j]);
+      const u32 qkx = j ? kx[j - 1] : pkx;
+      const u32 qev = j ? ev[j - 1] : pev;
+      const u32 qw = j ? sn[j - 1].x : pw;
+      if (key != lk) {
+        lk = key;
+        lw = 0;
+        fi = NONE;
+      }
+      // W_x check (every rule of Fig. 2; atomics only against a plain last write)
+      if (lw) {
+        const u64 li = (u64)lw - 1;
+        u32 pkx2, pev2, pw2;
+        if (li >= tbase) {
+          pkx2 = s_kx[li - tbase];
+          pev2 = s_ev[li - tbase];
+          pw2 = s_w[li - tbase];
+        } else {
+          pkx2 = a.keys[li];
+          pev2 = a.evs[li];
+          pw2 = __ldg(&c.snap[pev2 >> 5].x);
+        }
+        const bool patm = (pkx2 & 3u) == IOP_ATOM;
+        if (op == IOP_LD) {
+          if (!hb_ev(c, pev2, pw2, ev[j], s2)) emit(a, key, ev[j], pev2, patm ? BC_KIND_AR : BC_KIND_WR);
+        } else if (op == IOP_ATOM) {
+          if (!patm && !hb_ev(c, pev2, pw2, ev[j], s2)) emit(a, key, ev[j], pev2, BC_KIND_WA);
+        } else if (!hb_ev(c, pev2, pw2, ev[j], s2)) {
+          const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (pev2 >> 5) == (ev[j] >> 5);
+          if (!filtered) emit(a, key, ev[j], pev2, patm ? BC_KIND_AW : BC_KIND_WW);
         }
       }
-    }
-    // R_x check at writers (WRITE*/ATOM*: R_x ⪯ C_t or R_x ⊑ C_t)
-    if (op != IOP_LD && key == pk && pop == IOP_LD) {
-      u32 kind = op == IOP_ATOM ? BC_KIND_RA : BC_KIND_RW;
-      if (fi == NONE) {
-        if (!hb_ev(a, pev, cu)) emit(a, key, cu.ev, pev, kind);
-      } else {
-        vc_check(a, (u64)fi - 1, i - 1, cu, key, kind);
+      // R_x check at writers (WRITE* / *ATOM*: R_x ⪯ C_t as an epoch, R_x ⊑ C_t as a vector)
+      if (op != IOP_LD && qkx != NONE && (qkx >> 2) == key && (qkx & 3u) == IOP_LD) {
+        const u32 kind = op == IOP_ATOM ? BC_KIND_RA : BC_KIND_RW;
+        if (fi == NONE) {
+          if (!hb_ev(c, qev, qw, ev[j], s2)) emit(a, key, ev[j], qev, kind);
+        } else {
+          vc_check(a.evs, a.races, a.race_cnt, a.race_cap, (u64)fi - 1, i - 1, ev[j], s2.warp, s2.ps, s2.node,
+                   s2.blab, key, kind);
+        }
+      }
+      if (op != IOP_LD) {
+        lw = (u32)i + 1u;
+        fi = NONE;
+      } else if (((infl >> j) & 1u) && fi == NONE) {
+        fi = (u32)i;
       }
     }
-    // state update
-    if (op != IOP_LD) {
-      lw = (u32)i + 1u;
-      fi = NONE;
-    } else if (((infl >> j) & 1u) && fi == NONE) {
-      fi = (u32)i;
-    }
-    pk = key;
-    pop = op;
-    pev = ev[j];
   }
 }
 
@@ -307,6 +368,7 @@ void launch_check(const HbCtx& c, const u32* keys, const u32* evs, u64 n, void* 
   u64 tiles = (n + CK_TILE - 1) / CK_TILE;
   cudaMemsetAsync(status, 0, tiles * sizeof(TileStatus), st);
   cudaMemsetAsync(tile_counter, 0, sizeof(u32), st);
+  cudaMemcpyToSymbolAsync(cHC, &c, sizeof(HbCtx), 0, cudaMemcpyHostToDevice, st);
   CheckArgs a;
   a.c = c;
   a.keys = keys;
@@ -318,7 +380,7 @@ void launch_check(const HbCtx& c, const u32* keys, const u32* evs, u64 n, void* 
   a.race_cnt = race_cnt;
   a.race_cap = race_cap;
   a.seg_cnt = seg_cnt;
-  k_check<<<(unsigned)tiles, CK_THREADS, 0, st>>>(a);
+  k_check<<<(unsigned)tiles, CK_THREADS, 0, st>>>(a); ++g_launches;
 }
 
 }  // namespace bc

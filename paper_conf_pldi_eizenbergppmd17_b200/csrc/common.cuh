@@ -35,7 +35,7 @@ constexpr u32 IOP_LD = 0, IOP_ST = 1, IOP_ST_SV = 2, IOP_ATOM = 3;
 // sync-index key space (K3)
 constexpr u32 KEY_BLOCK = 0x80000000u;  // block-level entry: key = KEY_BLOCK | block
 constexpr u32 KEY_LINK = 0xC0000000u;   // link entry:        key = KEY_LINK | target array
-constexpr u32 SYNC_LOOKUP_CAP = 4096;   // step cap of one foreign lookup
+constexpr u32 SYNC_LOOKUP_CAP = 1u << 16;  // step cap of one foreign lookup
 
 struct Geo {
   u32 n_blocks, tpb, wpb, n_warps;
@@ -80,17 +80,20 @@ __device__ __forceinline__ u32 lanemask_lt() {
 
 // ---------------------------------------------------------------- per-record snapshot
 // K2 output, one per record (16 B): the compressed clock of the record's active lanes.
-//   warp  : traced warp id
-//   ps    : label of the warp's last step before this record (0 = none)
-//   node  : SIMT-stack node the record executes in (its mask == the record's mask)
-//   phase : number of BAR records of the warp before this record
+//   warp : traced warp id
+//   ps   : label of the warp's last step before this record (0 = none)
+//   node : SIMT-stack node the record executes in (its mask == the record's mask); node == warp
+//          is the warp's root (converged) node
+//   blab : label of the last completed barrier of the block (0 = none); K2 writes the barrier
+//          phase here and k_snap_blab replaces it by the label once all warps are replayed
 struct Snap {
-  u32 warp, ps, node, phase;
+  u32 warp, ps, node, blab;
 };
 __device__ __forceinline__ Snap load_snap(const uint4* snap, u32 r) {
-  uint4 v = snap[r];
+  uint4 v = __ldg(snap + r);
   return Snap{v.x, v.y, v.z, v.w};
 }
+__device__ __forceinline__ Snap to_snap(uint4 v) { return Snap{v.x, v.y, v.z, v.w}; }
 
 // SIMT-stack node (16 B): mask, parent node, popen = label of the warp's last step before the
 // IF that opened this node's branch (what the lanes outside it last shared with it).
@@ -104,8 +107,6 @@ struct HbCtx {
   Geo g;
   const uint4* snap;      // [n_recs]
   const uint4* nodes;     // [n_nodes]
-  const u32* bar_base;    // [n_warps] first slot of the warp's barrier list
-  const u32* blockR;      // [n_bar_slots] completion label of barrier k of block b at bar_base[b*wpb]+k
   // foreign knowledge (K3); n_acq == 0 => none
   u32 n_acq;
   const u32* acq_block_start;  // [n_blocks + 1] ranges into acq_*
@@ -121,34 +122,31 @@ struct HbCtx {
   u32* err;
 };
 
-__device__ __forceinline__ u32 barrier_label(const HbCtx& c, u32 warp, u32 phase) {
-  if (phase == 0) return 0;
-  u32 w0 = (warp / c.g.wpb) * c.g.wpb;
-  return c.blockR[c.bar_base[w0] + phase - 1];
-}
-
-// know_t(u) for u = lane `ul` of t's own warp, t executing record with snapshot s (intra-warp
-// part only; the PTVC DIVERGED / NESTEDDIVERGED lookup of Fig. 7).
-__device__ __forceinline__ u32 intra_know(const HbCtx& c, const Snap& s, u32 ul) {
-  u32 n = s.node;
-  uint4 nd = c.nodes[n];
-  if ((nd.x >> ul) & 1u) return s.ps;
+// know_t(u) for u = lane `ul` of t's own warp, t executing a record with snapshot s (intra-warp
+// part only; the PTVC CONVERGED / DIVERGED / NESTEDDIVERGED lookup of Fig. 7).
+static __device__ __noinline__ u32 intra_walk(const uint4* __restrict__ nodes, u32 node, u32 ps, u32 ul) {
+  uint4 nd = __ldg(nodes + node);
+  if ((nd.x >> ul) & 1u) return ps;
   // walk up the branch tree to the lowest ancestor whose mask holds ul
   for (int d = 0; d < 40; ++d) {
     u32 p = nd.y;
     if (p == NONE) return 0;  // cannot happen for a valid lane (root mask = init mask)
-    uint4 pd = c.nodes[p];
+    uint4 pd = __ldg(nodes + p);
     if ((pd.x >> ul) & 1u) return nd.z;
     nd = pd;
   }
   return 0;
+}
+__device__ __forceinline__ u32 intra_know(const HbCtx& c, const Snap& s, u32 ul) {
+  if (s.node == s.warp) return s.ps;  // converged: every lane of the warp is in the root node
+  return intra_walk(c.nodes, s.node, s.ps, ul);
 }
 
 // structural happens-before: does t (executing record r2 with snapshot s2) know the step of
 // (warp w1, lane l1) at record r1?  Same block only; no same-thread shortcut (callers do it).
 __device__ __forceinline__ bool struct_knows(const HbCtx& c, u32 w1, u32 l1, u32 r1, const Snap& s2) {
   if (w1 / c.g.wpb != s2.warp / c.g.wpb) return false;
-  if (r1 + 1u <= barrier_label(c, s2.warp, s2.phase)) return true;
+  if (r1 + 1u <= s2.blab) return true;
   if (w1 == s2.warp && intra_know(c, s2, l1) >= r1 + 1u) return true;
   return false;
 }
@@ -170,10 +168,14 @@ __device__ __forceinline__ u32 idx_lower_bound(const HbCtx& c, u64 ak) {
   return lo;
 }
 
-// does view (arr, bound) know the step of (warp uw, lane ul) at record r1?
-static __device__ __noinline__ bool view_knows(const HbCtx& c, u32 uw, u32 ul, u32 r1, u32 arr, u32 bound) {
-  u32 st_arr[48], st_bd[48];
-  int sp = 0;
+// does view (arr, bound) know the step of (warp uw, lane ul) at record r1?  Depth-first over
+// the link DAG; an array already visited with a bound >= the new one is skipped (its entries
+// are a superset), which keeps chains of releases linear.
+static __device__ __noinline__ bool view_knows(const HbCtx c, u32 uw, u32 ul, u32 r1, u32 arr, u32 bound) {
+  constexpr int STK = 96, VIS = 160;
+  u32 st_arr[STK], st_bd[STK];
+  u32 vis_arr[VIS], vis_bd[VIS];
+  int sp = 0, nv = 0;
   st_arr[sp] = arr;
   st_bd[sp++] = bound;
   u32 steps = 0;
@@ -181,7 +183,19 @@ static __device__ __noinline__ bool view_knows(const HbCtx& c, u32 uw, u32 ul, u
   const u32 ub = uw / c.g.wpb;
   while (sp > 0) {
     --sp;
-    u32 a = st_arr[sp], bd = st_bd[sp];
+    const u32 a = st_arr[sp], bd = st_bd[sp];
+    bool skip = false;
+    for (int q = 0; q < nv; ++q)
+      if (vis_arr[q] == a) {
+        if (vis_bd[q] >= bd) skip = true; else vis_bd[q] = bd;
+        break;
+      }
+    if (skip) continue;
+    if (nv < VIS) {
+      bool found = false;
+      for (int q = 0; q < nv; ++q) found |= vis_arr[q] == a;
+      if (!found) { vis_arr[nv] = a; vis_bd[nv++] = bd; }
+    }
     if (++steps > SYNC_LOOKUP_CAP) {
       set_err(c.err, ERR_OVERFLOW);
       return false;
@@ -209,11 +223,16 @@ static __device__ __noinline__ bool view_knows(const HbCtx& c, u32 uw, u32 ul, u
           any = true;
         }
       if (any) {
-        if (sp >= 48) {
+        u32 tgt = (u32)(key & 0x3FFFFFFFull);
+        bool seen = false;
+        for (int q = 0; q < nv; ++q)
+          if (vis_arr[q] == tgt && vis_bd[q] >= best) seen = true;
+        if (seen) continue;
+        if (sp >= STK) {
           set_err(c.err, ERR_OVERFLOW);
           return false;
         }
-        st_arr[sp] = (u32)(key & 0x3FFFFFFFull);
+        st_arr[sp] = tgt;
         st_bd[sp++] = best;
       }
     }
@@ -224,7 +243,7 @@ static __device__ __noinline__ bool view_knows(const HbCtx& c, u32 uw, u32 ul, u
 // foreign part of know_t(u) >= r1+1 for t executing record r2 (snapshot s2): through the
 // views of the acquires of t's block that t structurally knows (every release->acquire path
 // into t's block ends at one of them).
-static __device__ __noinline__ bool foreign_knows(const HbCtx& c, u32 w1, u32 l1, u32 r1, u32 r2, const Snap& s2) {
+static __device__ __noinline__ bool foreign_knows(const HbCtx c, u32 w1, u32 l1, u32 r1, u32 r2, const Snap s2) {
   u32 b2 = s2.warp / c.g.wpb;
   u32 lo = c.acq_block_start[b2], hi = c.acq_block_start[b2 + 1];
   for (u32 i = lo; i < hi; ++i) {
@@ -236,14 +255,15 @@ static __device__ __noinline__ bool foreign_knows(const HbCtx& c, u32 w1, u32 l1
   return false;
 }
 
-// e1 = (record r1, lane l1) happened before e2 = (record r2, lane l2)?  r1 <= r2 in trace order.
-// s2 = snapshot of r2; w1 = warp of r1.
+// e1 = (record r1, lane l1, warp w1) happened before e2 = (record r2, lane l2, snapshot s2)?
+// r1 <= r2 in trace order.
 __device__ __forceinline__ bool hb(const HbCtx& c, u32 r1, u32 l1, u32 w1, u32 r2, u32 l2, const Snap& s2) {
+  if (r1 == r2) return l1 == l2;               // lanes of one instruction are concurrent
   if (w1 == s2.warp && l1 == l2) return true;  // same thread: program order
-  if (r1 == r2) return false;                  // lanes of one instruction are concurrent
   if (struct_knows(c, w1, l1, r1, s2)) return true;
-  if (c.n_acq == 0 || c.acq_block_start[s2.warp / c.g.wpb] == c.acq_block_start[s2.warp / c.g.wpb + 1])
-    return false;
+  if (c.n_acq == 0) return false;
+  u32 b2 = s2.warp / c.g.wpb;
+  if (c.acq_block_start[b2] == c.acq_block_start[b2 + 1]) return false;
   return foreign_knows(c, w1, l1, r1, r2, s2);
 }
 
@@ -260,6 +280,35 @@ __device__ __forceinline__ T warp_incl_sum(T v) {
 
 // decoupled look-back status words (u64): [63:62] flag, [61:0] value
 constexpr u64 LB_AGG = 1ull << 62, LB_INC = 2ull << 62, LB_MASK = (1ull << 62) - 1;
+
+// Warp-cooperative version: all 32 lanes call it; 32 predecessors are inspected per round.
+__device__ __forceinline__ u64 lookback_u64_warp(volatile u64* status, u32 tile, u64 agg, int lane) {
+  if (tile == 0) {
+    if (lane == 0) status[0] = LB_INC | agg;
+    return 0;
+  }
+  if (lane == 0) status[tile] = LB_AGG | agg;
+  u64 excl = 0;
+  int hi = (int)tile - 1;
+  while (true) {
+    int idx = hi - lane;
+    u64 s = idx >= 0 ? (u64)status[idx] : (u64)(2ull << 62);
+    while (__any_sync(0xFFFFFFFFu, (s & ~LB_MASK) == 0)) {
+      if ((s & ~LB_MASK) == 0) s = status[idx];
+    }
+    u32 incm = __ballot_sync(0xFFFFFFFFu, (s & ~LB_MASK) == LB_INC);
+    int last = incm ? __ffs(incm) - 1 : 31;  // nearest inclusive predecessor ends the walk
+    u64 v = lane <= last ? (s & LB_MASK) : 0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, o);
+    excl += v;
+    if (incm) break;
+    hi -= 32;
+  }
+  __threadfence();
+  if (lane == 0) status[tile] = LB_INC | (excl + agg);
+  return excl;
+}
 
 // exclusive prefix of `agg` for tile `tile` over u64 status words (single value per tile).
 // Called by one thread.

@@ -94,7 +94,7 @@ int bits_for(u64 maxval) {
 }  // namespace
 
 void launch_page_list(const u32* bits, const u32* rank, u64 nwords, u32* page_num, cudaStream_t st) {
-  k_page_list<<<nb(nwords), 256, 0, st>>>(bits, rank, nwords, page_num);
+  k_page_list<<<nb(nwords), 256, 0, st>>>(bits, rank, nwords, page_num); ++g_launches;
 }
 
 // races[n_r] (key, cur, prior, kind) + findings -> out[n_f + n_r] in canonical order
@@ -106,19 +106,19 @@ void finalize_races(const uint4* races, u32 n_r, const u32* fblk, const u32* fre
     launch_iota(p, n_f, st);
     sort_perm_by(p, frec, n_f, 32, S, st);
     sort_perm_by(p, fblk, n_f, bits_for(g.n_blocks), S, st);
-    k_emit_findings<<<nb(n_f), 256, 0, st>>>(fblk, frec, p, n_f, out);
+    k_emit_findings<<<nb(n_f), 256, 0, st>>>(fblk, frec, p, n_f, out); ++g_launches;
   }
   if (n_r) {
     u32* p = S.alloc<u32>(n_r);
     u32* f = S.alloc<u32>(n_r);
     launch_iota(p, n_r, st);
-    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 2, f);
+    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 2, f); ++g_launches;
     sort_perm_by(p, f, n_r, 32, S, st);
-    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 1, f);
+    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 1, f); ++g_launches;
     sort_perm_by(p, f, n_r, 32, S, st);
-    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 0, f);
+    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 0, f); ++g_launches;
     sort_perm_by(p, f, n_r, bits_for(n_keys), S, st);
-    k_emit_races<<<nb(n_r), 256, 0, st>>>(races, p, n_r, g, snap, page_num, shared_base, out + n_f);
+    k_emit_races<<<nb(n_r), 256, 0, st>>>(races, p, n_r, g, snap, page_num, shared_base, out + n_f); ++g_launches;
   }
 }
 

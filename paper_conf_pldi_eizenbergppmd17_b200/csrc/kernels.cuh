@@ -9,6 +9,9 @@
 
 namespace bc {
 
+// kernels launched by this process (bc_stats.kernel_launches is the delta over one bc_detect)
+extern u64 g_launches;
+
 // counters written by the kernels (u64 device array)
 enum { C_LANE_EVENTS = 0, C_CONTROL_EVENTS, C_SYNC_RECS, C_ACQ_RECS, C_MEM_RECS, C_IFS, C_BARS, C_SYNC_LANEOPS,
        C_ITEMS, C_ITEM_BOUND, C_SEGMENTS, C_N };
@@ -59,6 +62,8 @@ void launch_replay(const bc_record* recs, const u32* wrec, const u32* warp_start
 void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, const u32* bar_rec, const u32* bar_next,
                      u32* blockR, u32* err, cudaStream_t st);
 void launch_popc(const u32* bits, u32* out, u64 n, cudaStream_t st);
+void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, const u32* bar_base, const u32* blockR,
+                      cudaStream_t st);
 u64 expand_tiles(u64 n_recs);
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
                    u32* keys, u32* evs, u64* status, u32* tile_counter, u64* cnt, u32* err, cudaStream_t st);

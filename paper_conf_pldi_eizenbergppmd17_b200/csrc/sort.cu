@@ -222,14 +222,14 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   cudaMemsetAsync(hist, 0, 4 * RS_BINS * sizeof(u32), st);
   int blocks = (int)((n + 255) / 256);
   if (blocks > 148 * 8) blocks = 148 * 8;
-  k_rs_hist<<<blocks, 256, 0, st>>>(keys, n, bit_lo, passes, hist);
-  k_rs_hist_scan<<<1, RS_BINS, 0, st>>>(hist, passes);
+  k_rs_hist<<<blocks, 256, 0, st>>>(keys, n, bit_lo, passes, hist); ++g_launches;
+  k_rs_hist_scan<<<1, RS_BINS, 0, st>>>(hist, passes); ++g_launches;
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
   for (int p = 0; p < passes; ++p) {
     cudaMemsetAsync(counter, 0, sizeof(u32), st);
     cudaMemsetAsync(status, 0, tiles * RS_BINS * sizeof(u64), st);
     k_rs_onesweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, bit_lo + 8 * p, hist + p * RS_BINS,
-                                                           status, counter);
+                                                           status, counter); ++g_launches;
     u32* tk = ki; ki = ko; ko = tk;
     u32* tv = vi; vi = vo; vo = tv;
   }
@@ -245,7 +245,7 @@ void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_d
   u32* counter = (u32*)temp;
   u64* status = (u64*)((char*)temp + 64);
   cudaMemsetAsync(temp, 0, 64 + tiles * sizeof(u64), st);
-  k_scan_u32<<<(unsigned)tiles, SC_THREADS, 0, st>>>(in, out, n, status, counter, total_dev);
+  k_scan_u32<<<(unsigned)tiles, SC_THREADS, 0, st>>>(in, out, n, status, counter, total_dev); ++g_launches;
 }
 
 }  // namespace bc

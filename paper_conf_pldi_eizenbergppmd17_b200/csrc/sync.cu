@@ -14,6 +14,9 @@
 // nothing has to be processed in trace order: every lane-op is independent (one thread each),
 // and an AR chain (threadFenceReduction's atomicInc ticket) costs O(1) entries per op instead of
 // the O(n) vector-clock copy of the printed rules.
+#include <cstdio>
+#include <cstdlib>
+
 #include "common.cuh"
 #include "kernels.cuh"
 
@@ -190,7 +193,7 @@ __device__ u32 laneop_entries(const K3In& k, u32 i, const EntOut* o, u32 base) {
     u32 tarr = is_glb_op(op) ? x : (k.nx + my_bid);
     Snap s = load_snap(c.snap, r);
     // structural clock of the releaser (its block only)
-    u32 bl = barrier_label(c, w, s.phase);
+    u32 bl = s.blab;
     if (bl) put(o, n, tarr, KEY_BLOCK | b, ev, 0xFFFFFFFFu, bl);
     {
       uint4 nd = c.nodes[s.node];
@@ -301,16 +304,16 @@ void sort_perm_by(u32* perm, const u32* f, u32 n, int bits, Scratch& S, cudaStre
   u32* k2 = S.alloc<u32>(n);
   u32* p2 = S.alloc<u32>(n);
   void* tmp = S.alloc<char>(rs_temp_bytes(n));
-  k_gather_u32<<<nb(n), 256, 0, st>>>(f, perm, n, k);
+  k_gather_u32<<<nb(n), 256, 0, st>>>(f, perm, n, k); ++g_launches;
   bool alt = radix_sort_pairs(k, perm, k2, p2, n, 0, bits, tmp, st);
   if (alt) cudaMemcpyAsync(perm, p2, n * sizeof(u32), cudaMemcpyDeviceToDevice, st);
 }
 
 void launch_iota(u32* p, u32 n, cudaStream_t st) {
-  if (n) k_iota<<<nb(n), 256, 0, st>>>(p, n);
+  if (n) k_iota<<<nb(n), 256, 0, st>>>(p, n); ++g_launches;
 }
 void launch_gather_u32(const u32* src, const u32* perm, u32 n, u32* dst, cudaStream_t st) {
-  if (n) k_gather_u32<<<nb(n), 256, 0, st>>>(src, perm, n, dst);
+  if (n) k_gather_u32<<<nb(n), 256, 0, st>>>(src, perm, n, dst); ++g_launches;
 }
 
 static int bits_for(u64 maxval) {
@@ -339,7 +342,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   u32* aflag = S.alloc<u32>(n_srec);
   u32* aex = S.alloc<u32>(n_srec);
   u64* tot = S.alloc<u64>(1);
-  k_acq_flags<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, aflag);
+  k_acq_flags<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, aflag); ++g_launches;
   exclusive_scan_u32(aflag, aex, n_srec, S.alloc<char>(scan_temp_bytes(n_srec)), tot, st);
   u64 n_acq64 = 0;
   cudaMemcpyAsync(&n_acq64, tot, 8, cudaMemcpyDeviceToHost, st);
@@ -351,7 +354,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   u32* acq_lane = S.alloc<u32>(n_acq + 1);
   u32* acq_bstart = S.alloc<u32>(g.n_blocks + 1);
   if (n_acq) {
-    k_acq_collect<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, g, acq_blk, acq_rec, aex);
+    k_acq_collect<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, g, acq_blk, acq_rec, aex); ++g_launches;
     u32* k2 = S.alloc<u32>(n_acq);
     u32* v2 = S.alloc<u32>(n_acq);
     void* tmp = S.alloc<char>(rs_temp_bytes(n_acq));
@@ -360,9 +363,9 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
       cudaMemcpyAsync(acq_blk, k2, n_acq * 4, cudaMemcpyDeviceToDevice, st);
       cudaMemcpyAsync(acq_rec, v2, n_acq * 4, cudaMemcpyDeviceToDevice, st);
     }
-    k_acq_info<<<nb(n_acq), 256, 0, st>>>(recs, acq_rec, n_acq, acq_warp, acq_lane);
+    k_acq_info<<<nb(n_acq), 256, 0, st>>>(recs, acq_rec, n_acq, acq_warp, acq_lane); ++g_launches;
   }
-  k_block_start<<<nb(g.n_blocks + 1), 256, 0, st>>>(acq_blk, n_acq, g.n_blocks, acq_bstart);
+  k_block_start<<<nb(g.n_blocks + 1), 256, 0, st>>>(acq_blk, n_acq, g.n_blocks, acq_bstart); ++g_launches;
   hc.n_acq = n_acq;
   hc.acq_block_start = acq_bstart;
   hc.acq_rec = acq_rec;
@@ -372,22 +375,22 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   // 3. lane-ops and dense sync-location ids
   u32* cnt = S.alloc<u32>(n_srec);
   u32* off = S.alloc<u32>(n_srec);
-  k_popc_recs<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, cnt);
+  k_popc_recs<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, cnt); ++g_launches;
   exclusive_scan_u32(cnt, off, n_srec, S.alloc<char>(scan_temp_bytes(n_srec)), nullptr, st);
   u32* lo_rec = S.alloc<u32>(n_lo);
   u32* lo_lane = S.alloc<u32>(n_lo);
   u32* xk_lo = S.alloc<u32>(n_lo);
   u32* xk_hi = S.alloc<u32>(n_lo);
   u32* perm = S.alloc<u32>(n_lo);
-  k_laneops<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, off, g, lo_rec, lo_lane, xk_lo, xk_hi, perm, hc.err);
+  k_laneops<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, off, g, lo_rec, lo_lane, xk_lo, xk_hi, perm, hc.err); ++g_launches;
   sort_perm_by(perm, xk_lo, n_lo, 32, S, st);
   sort_perm_by(perm, xk_hi, n_lo, 32, S, st);
   u32* flag = S.alloc<u32>(n_lo);
   u32* ex = S.alloc<u32>(n_lo);
   u32* xid = S.alloc<u32>(n_lo);
-  k_uniq_flags2<<<nb(n_lo), 256, 0, st>>>(xk_hi, xk_lo, perm, n_lo, flag);
+  k_uniq_flags2<<<nb(n_lo), 256, 0, st>>>(xk_hi, xk_lo, perm, n_lo, flag); ++g_launches;
   exclusive_scan_u32(flag, ex, n_lo, S.alloc<char>(scan_temp_bytes(n_lo)), tot, st);
-  k_assign_ids<<<nb(n_lo), 256, 0, st>>>(perm, flag, ex, n_lo, xid);
+  k_assign_ids<<<nb(n_lo), 256, 0, st>>>(perm, flag, ex, n_lo, xid); ++g_launches;
   u64 nx64 = 0;
   cudaMemcpyAsync(&nx64, tot, 8, cudaMemcpyDeviceToHost, st);
   // 4. block arrays B_{x,b}
@@ -395,7 +398,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   u32* pk_lo = S.alloc<u32>(n_lo);
   u32* pcnt = S.alloc<u32>(1);
   cudaMemsetAsync(pcnt, 0, 4, st);
-  k_bpairs<<<nb(n_lo), 256, 0, st>>>(recs, lo_rec, xid, n_lo, g, pk_hi, pk_lo, pcnt);
+  k_bpairs<<<nb(n_lo), 256, 0, st>>>(recs, lo_rec, xid, n_lo, g, pk_hi, pk_lo, pcnt); ++g_launches;
   u32 np = 0;
   cudaMemcpyAsync(&np, pcnt, 4, cudaMemcpyDeviceToHost, st);
   if (cudaStreamSynchronize(st) != cudaSuccess) return BC_ERR_CUDA;
@@ -410,20 +413,22 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
     sort_perm_by(pp, pk_hi, np, 32, S, st);
     u32* pf = S.alloc<u32>(np);
     u32* pe = S.alloc<u32>(np);
-    k_uniq_flags2<<<nb(np), 256, 0, st>>>(pk_hi, pk_lo, pp, np, pf);
+    k_uniq_flags2<<<nb(np), 256, 0, st>>>(pk_hi, pk_lo, pp, np, pf); ++g_launches;
     exclusive_scan_u32(pf, pe, np, S.alloc<char>(scan_temp_bytes(np)), tot, st);
-    k_compact_pairs<<<nb(np), 256, 0, st>>>(pk_hi, pk_lo, pp, pf, pe, np, bp_x, bp_b);
+    k_compact_pairs<<<nb(np), 256, 0, st>>>(pk_hi, pk_lo, pp, pf, pe, np, bp_x, bp_b); ++g_launches;
     u64 nb64 = 0;
     cudaMemcpyAsync(&nb64, tot, 8, cudaMemcpyDeviceToHost, st);
     if (cudaStreamSynchronize(st) != cudaSuccess) return BC_ERR_CUDA;
     nB = (u32)nb64;
   }
+  if (getenv("BC_DEBUG"))
+    fprintf(stderr, "[bc] K3: n_srec=%u n_lo=%u n_acq=%u nx=%u np=%u nB=%u\n", n_srec, n_lo, n_acq, nx, np, nB);
   if ((u64)nx + nB + n_acq >= (1ull << 30)) return BC_ERR_OVERFLOW;
   hc.acq_arr = nullptr;
   // arrF ids are nx + nB + acquire index; expose them for K7
   {
     u32* acq_arr = S.alloc<u32>(n_acq + 1);
-    if (n_acq) k_iota_add<<<nb(n_acq), 256, 0, st>>>(acq_arr, n_acq, nx + nB);
+    if (n_acq) k_iota_add<<<nb(n_acq), 256, 0, st>>>(acq_arr, n_acq, nx + nB); ++g_launches;
     hc.acq_arr = acq_arr;
   }
   // 5. entries
@@ -441,11 +446,12 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   k.acq_idx_of_rec_sorted = nullptr;
   u32* ecnt = S.alloc<u32>(n_lo);
   u32* eoff = S.alloc<u32>(n_lo);
-  k_ent_count<<<nb(n_lo), 128, 0, st>>>(k, ecnt);
+  k_ent_count<<<nb(n_lo), 256, 0, st>>>(k, ecnt); ++g_launches;
   exclusive_scan_u32(ecnt, eoff, n_lo, S.alloc<char>(scan_temp_bytes(n_lo)), tot, st);
   u64 ne64 = 0;
   cudaMemcpyAsync(&ne64, tot, 8, cudaMemcpyDeviceToHost, st);
   if (cudaStreamSynchronize(st) != cudaSuccess) return BC_ERR_CUDA;
+  if (getenv("BC_DEBUG")) fprintf(stderr, "[bc] K3: entries=%llu\n", (unsigned long long)ne64);
   if (ne64 >= (1ull << 31)) return BC_ERR_OVERFLOW;
   u32 ne = (u32)ne64;
   *n_entries_out = ne;
@@ -455,7 +461,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   eo.pos = S.alloc<u32>(ne + 1);
   eo.mask = S.alloc<u32>(ne + 1);
   eo.clk = S.alloc<u32>(ne + 1);
-  k_ent_fill<<<nb(n_lo), 128, 0, st>>>(k, eoff, eo);
+  k_ent_fill<<<nb(n_lo), 256, 0, st>>>(k, eoff, eo); ++g_launches;
   // 6. index sorted by (arr, key, pos)
   u32* ep = S.alloc<u32>(ne + 1);
   launch_iota(ep, ne, st);
@@ -466,7 +472,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   u32* ipos = S.alloc<u32>(ne + 1);
   u32* imask = S.alloc<u32>(ne + 1);
   u32* iclk = S.alloc<u32>(ne + 1);
-  if (ne) k_make_ak<<<nb(ne), 256, 0, st>>>(eo.arr, eo.key, eo.pos, eo.mask, eo.clk, ep, ne, ak, ipos, imask, iclk);
+  if (ne) k_make_ak<<<nb(ne), 256, 0, st>>>(eo.arr, eo.key, eo.pos, eo.mask, eo.clk, ep, ne, ak, ipos, imask, iclk); ++g_launches;
   hc.n_idx = ne;
   hc.idx_ak = ak;
   hc.idx_pos = ipos;

@@ -75,15 +75,21 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v[i] += __shfl_down_sync(0xFFFFFFFFu, v[i], o);
   }
-  if (lane == 0) {
-    if (v[0]) atomicAdd((unsigned long long*)&cnt[C_LANE_EVENTS], (unsigned long long)v[0]);
-    if (v[1]) atomicAdd((unsigned long long*)&cnt[C_CONTROL_EVENTS], (unsigned long long)v[1]);
-    if (v[2]) atomicAdd((unsigned long long*)&cnt[C_ACQ_RECS], (unsigned long long)v[2]);
-    if (v[3]) atomicAdd((unsigned long long*)&cnt[C_MEM_RECS], (unsigned long long)v[3]);
-    if (v[4]) atomicAdd((unsigned long long*)&cnt[C_IFS], (unsigned long long)v[4]);
-    if (v[5]) atomicAdd((unsigned long long*)&cnt[C_BARS], (unsigned long long)v[5]);
-    if (v[6]) atomicAdd((unsigned long long*)&cnt[C_SYNC_LANEOPS], (unsigned long long)v[6]);
-    if (v[7]) atomicAdd((unsigned long long*)&cnt[C_ITEM_BOUND], (unsigned long long)v[7]);
+  {
+    __shared__ unsigned long long s_cnt[8];
+    if (threadIdx.x < 8) s_cnt[threadIdx.x] = 0;
+    __syncthreads();
+    if (lane == 0) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        if (v[i]) atomicAdd(&s_cnt[i], (unsigned long long)v[i]);
+    }
+    __syncthreads();
+    if (threadIdx.x < 8) {
+      const int slot[8] = {C_LANE_EVENTS, C_CONTROL_EVENTS, C_ACQ_RECS, C_MEM_RECS, C_IFS, C_BARS, C_SYNC_LANEOPS,
+                           C_ITEM_BOUND};
+      if (s_cnt[threadIdx.x]) atomicAdd((unsigned long long*)&cnt[slot[threadIdx.x]], s_cnt[threadIdx.x]);
+    }
   }
   // page marking: ST / ATOM on global memory
   u32 wr = __ballot_sync(0xFFFFFFFFu, valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) &&
@@ -260,7 +266,7 @@ __global__ void k_barriers(Geo g, const u32* __restrict__ bar_cnt, const u32* __
 // pages cannot take part in a race (every race needs a write) and are dropped.
 // Also validates per-lane alignment / shared bounds for every op <= AR_GLB.
 // One warp per record, 8 warps x EXP_RPW records per tile, tile offsets by decoupled look-back.
-constexpr int EXP_RPW = 4;
+constexpr int EXP_RPW = 16;
 constexpr int EXP_TILE = 8 * EXP_RPW;
 
 __global__ void __launch_bounds__(256) k_expand(const bc_record* __restrict__ recs, Geo g,
@@ -324,14 +330,26 @@ __global__ void __launch_bounds__(256) k_expand(const bc_record* __restrict__ re
   if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
   __syncthreads();
   if (w == 0) {
-    u32 v = s_rcnt[lane];  // EXP_TILE == 32
-    u32 x = warp_incl_sum(v);
-    s_rcnt[lane] = x - v;
+    // exclusive scan of the EXP_TILE record counts (EXP_RPW per lane, in record order)
+    u32 v[EXP_RPW / 2 > 0 ? EXP_TILE / 32 : 1];
+    u32 sum = 0;
+#pragma unroll
+    for (int q = 0; q < EXP_TILE / 32; ++q) {
+      v[q] = s_rcnt[lane * (EXP_TILE / 32) + q];
+      sum += v[q];
+    }
+    u32 x = warp_incl_sum(sum);
+    u32 run = x - sum;
+#pragma unroll
+    for (int q = 0; q < EXP_TILE / 32; ++q) {
+      s_rcnt[lane * (EXP_TILE / 32) + q] = run;
+      run += v[q];
+    }
     u32 total = __shfl_sync(0xFFFFFFFFu, x, 31);
-    if (lane == 0) s_base = lookback_u64(status, (u32)tile, total);
-    if (lane == 0 && (tile + 1) * EXP_TILE >= g.n_recs) {
-      // last tile: publish the item total
-      cnt[C_ITEMS] = s_base + total;
+    u64 b = lookback_u64_warp(status, (u32)tile, total, lane);
+    if (lane == 0) {
+      s_base = b;
+      if ((tile + 1) * EXP_TILE >= g.n_recs) cnt[C_ITEMS] = b + total;  // last tile: item total
     }
   }
   __syncthreads();
@@ -360,27 +378,48 @@ void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u3
   u64 warps = (g.n_recs + 31) / 32;
   if (warps == 0) return;
   u64 blocks = (warps + 7) / 8;
-  k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt, err);
+  k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt, err); ++g_launches;
 }
 
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st) {
-  k_warp_start<<<(n_warps + 1 + 255) / 256, 256, 0, st>>>(skeys, n, n_warps, warp_start);
+  k_warp_start<<<(n_warps + 1 + 255) / 256, 256, 0, st>>>(skeys, n, n_warps, warp_start); ++g_launches;
 }
 
 void launch_replay(const bc_record* recs, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
                    const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next, u32* find_blk,
                    u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st) {
   k_replay<<<(g.n_warps + 127) / 128, 128, 0, st>>>(recs, wrec, warp_start, g, node_base, bar_base, snap, nodes,
-                                                     bar_rec, bar_next, find_blk, find_rec, find_cnt, err);
+                                                     bar_rec, bar_next, find_blk, find_rec, find_cnt, err); ++g_launches;
 }
 
 void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, const u32* bar_rec, const u32* bar_next,
                      u32* blockR, u32* err, cudaStream_t st) {
-  k_barriers<<<(g.n_blocks + 127) / 128, 128, 0, st>>>(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err);
+  k_barriers<<<(g.n_blocks + 127) / 128, 128, 0, st>>>(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err); ++g_launches;
+}
+
+// snapshot .w: barrier phase -> label of the block's last completed barrier (0 = none)
+__global__ void k_snap_blab(uint4* __restrict__ snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars,
+                            const u32* __restrict__ bar_base, const u32* __restrict__ blockR) {
+  u64 r = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= n) return;
+  uint2 v = *reinterpret_cast<const uint2*>(reinterpret_cast<const u32*>(snap + r) + 2);  // (node, phase)
+  u32 w = reinterpret_cast<const u32*>(snap + r)[0];
+  u32 ph = v.y;
+  u32 lab = 0;
+  if (ph && w < n_warps) {  // (records after an infeasibility are garbage; results are discarded)
+    u64 i = (u64)bar_base[(w / wpb) * wpb] + ph - 1;
+    lab = i < n_bars ? blockR[i] : 0u;
+  }
+  reinterpret_cast<u32*>(snap + r)[3] = lab;
+}
+void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, const u32* bar_base, const u32* blockR,
+                      cudaStream_t st) {
+  k_snap_blab<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(snap, n, wpb, n_warps, n_bars, bar_base, blockR);
+  ++g_launches;
 }
 
 void launch_popc(const u32* bits, u32* out, u64 n, cudaStream_t st) {
-  k_popc<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(bits, out, n);
+  k_popc<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(bits, out, n); ++g_launches;
 }
 
 u64 expand_tiles(u64 n_recs) { return (n_recs + EXP_TILE - 1) / EXP_TILE; }
@@ -390,7 +429,7 @@ void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, co
   u64 tiles = expand_tiles(g.n_recs);
   if (tiles == 0) return;
   k_expand<<<(unsigned)tiles, 256, 0, st>>>(recs, g, page_bits, page_rank, shared_base, keys, evs, status,
-                                           tile_counter, cnt, err);
+                                           tile_counter, cnt, err); ++g_launches;
 }
 
 __global__ void k_node_base(const u32* __restrict__ if_excl, u32 n_warps, u32* __restrict__ node_base) {
@@ -398,7 +437,7 @@ __global__ void k_node_base(const u32* __restrict__ if_excl, u32 n_warps, u32* _
   if (w < n_warps) node_base[w] = n_warps + 2u * if_excl[w];
 }
 void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st) {
-  k_node_base<<<(n_warps + 255) / 256, 256, 0, st>>>(if_excl, n_warps, node_base);
+  k_node_base<<<(n_warps + 255) / 256, 256, 0, st>>>(if_excl, n_warps, node_base); ++g_launches;
 }
 
 }  // namespace bc
