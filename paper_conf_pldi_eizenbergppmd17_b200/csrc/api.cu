@@ -287,15 +287,19 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   cudaEventRecord(c->ev[4], st);
   // ---- K4: expansion
   const u64 bound = hc_cnt[C_ITEM_BOUND];
-  u32* ikeys = S.alloc<u32>(bound + 1);
+  u32* skeys0 = S.alloc<u32>(bound + 1);  // staging (tiles in completion order)
+  u32* sevs0 = S.alloc<u32>(bound + 1);
+  u32* ikeys = S.alloc<u32>(bound + 1);   // trace order
   u32* ievs = S.alloc<u32>(bound + 1);
   u64 tiles = expand_tiles(n);
-  u64* estatus = S.alloc<u64>(tiles + 1);
-  u32* ecounter = S.alloc<u32>(1);
-  cudaMemsetAsync(estatus, 0, (tiles + 1) * 8, st);
-  cudaMemsetAsync(ecounter, 0, 4, st);
+  u32* tile_off = S.alloc<u32>(tiles + 1);
+  u32* tile_cnt = S.alloc<u32>(tiles + 1);
+  u32* tile_dst = S.alloc<u32>(tiles + 1);
+  cudaMemsetAsync(cnt + C_ITEMS, 0, 8, st);
   cudaEventRecord(c->ev[14], st);
-  launch_expand(recs, g, page_bits, page_rank, shared_base, ikeys, ievs, estatus, ecounter, cnt, err, st);
+  launch_expand(recs, g, page_bits, page_rank, shared_base, skeys0, sevs0, tile_off, tile_cnt, cnt, err, st);
+  exclusive_scan_u32(tile_cnt, tile_dst, tiles, S.alloc<char>(scan_temp_bytes(tiles)), nullptr, st);
+  launch_expand_place(skeys0, sevs0, tile_off, tile_cnt, tile_dst, tiles, ikeys, ievs, st);
   cudaEventRecord(c->ev[15], st);
   u64 n_items = 0;
   u32 nfind = 0;

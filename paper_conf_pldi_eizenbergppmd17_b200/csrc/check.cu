@@ -150,237 +150,272 @@ static __device__ __noinline__ void vc_check(const u32* __restrict__ evs, uint4*
   }
 }
 
-// warp 0: exclusive prefix of this tile from its predecessors' published summaries,
-// 32 predecessors per round (decoupled look-back, non-commutative combine in tile order).
-__device__ __forceinline__ Sum warp_lookback(TileStatus* status, u32 tile, const Sum& agg, int lane) {
-  if (tile == 0) {
-    if (lane == 0) publish(&status[0], agg, 2u);
-    return sum_ident();
-  }
-  if (lane == 0) publish(&status[tile], agg, 1u);
-  Sum P = sum_ident();
-  int hi = (int)tile - 1;
-  while (true) {
-    int idx = hi - lane;  // lane 0 = nearest predecessor
-    u32 f = 2u;
-    Sum s = sum_ident();
-    if (idx >= 0) {
-      f = ((volatile TileStatus*)&status[idx])->flag;
-    }
-    // all lanes spin together until every inspected predecessor has published
-    while (__any_sync(0xFFFFFFFFu, f == 0u)) {
-      if (f == 0u) f = ((volatile TileStatus*)&status[idx])->flag;
-    }
-    __threadfence();
-    if (idx >= 0) {
-      volatile TileStatus* v = &status[idx];
-      s = Sum{v->fk, v->lk, v->lw, v->fi, v->bits};
-    }
-    u32 incm = __ballot_sync(0xFFFFFFFFu, idx >= 0 && f == 2u);
-    int last = incm ? (__ffs(incm) - 1) : 31;  // nearest inclusive predecessor ends this round
-    if (hi - last < 0) last = hi;                // fewer than 32 tiles left (tile 0 is inclusive)
-    // P = combine(s[last], ..., s[1], s[0], P)
-    Sum acc = sum_ident();
-    for (int k = last; k >= 0; --k) {
-      Sum sk;
-      sk.fk = __shfl_sync(0xFFFFFFFFu, s.fk, k);
-      sk.lk = __shfl_sync(0xFFFFFFFFu, s.lk, k);
-      sk.lw = __shfl_sync(0xFFFFFFFFu, s.lw, k);
-      sk.fi = __shfl_sync(0xFFFFFFFFu, s.fi, k);
-      sk.bits = __shfl_sync(0xFFFFFFFFu, s.bits, k);
-      acc = combine(acc, sk);
-    }
-    P = combine(acc, P);
-    if (incm) break;
-    hi -= 32;
-  }
-  if (lane == 0) publish(&status[tile], combine(P, agg), 2u);
-  return P;
+// ---------------------------------------------------------------------------------------
+// Persistent warp-range formulation.  The grid is sized to be fully co-resident; warp w owns
+// the contiguous item range [beg_w, end_w) and walks it in rounds of 32 (lane i = item r*32+i),
+// carrying the automaton state (LW, FI of the current granule) from round to round; per lane,
+// LW / FI inside a round come from ballots.  The state entering the range depends only on the
+// items of the same granule before beg_w, so the warp recomputes it by walking backwards from
+// beg_w (usually a few items: a writer or the start of the granule ends the walk); only if that
+// walk exceeds K7_WALK_CAP items does the warp wait for warp w-1 to publish its final state.
+// Items are read exactly once (plus the short walk), with a K7_PF-round register prefetch.
+constexpr int K7_WARPS = 8;
+constexpr int K7_PF = 4;
+constexpr u32 K7_WALK_CAP = 1u << 14;
+
+__device__ __forceinline__ u32 hibit(u32 m) { return 31u - __clz(m); }  // m != 0
+
+// summary of one round (standalone), uniform across the warp
+__device__ __forceinline__ Sum round_sum(u32 V, u32 Kin, u32 W, u32 I, u32 key, u64 base_r) {
+  Sum r = sum_ident();
+  if (!V) return r;
+  const u32 last = hibit(V);
+  r.fk = __shfl_sync(0xFFFFFFFFu, key, 0);
+  r.lk = __shfl_sync(0xFFFFFFFFu, key, last);
+  const u32 kc = Kin & ~1u & V;                 // key changes inside the round
+  const u32 ts = kc ? hibit(kc) : 0u;           // start lane of the tail key run
+  const u32 Wt = W & V & (~0u << ts);
+  const bool hasW = Wt != 0;
+  const u32 rs = hasW ? hibit(Wt) + 1u : ts;    // start of the trailing read run
+  const u32 It = rs < 32 ? (I & V & (~0u << rs)) : 0u;
+  r.lw = hasW ? (u32)(base_r + hibit(Wt)) + 1u : 0u;
+  r.fi = It ? (u32)(base_r + __ffs(It) - 1) : NONE;
+  r.bits = (kc ? 0u : 1u) | (hasW ? 2u : 0u);
+  return r;
 }
 
-__global__ void __launch_bounds__(CK_THREADS) k_check(CheckArgs a) {
-  __shared__ u32 s_kx[CK_TILE];
-  __shared__ u32 s_ev[CK_TILE];
-  __shared__ u32 s_w[CK_TILE];
-  __shared__ u32 s_tile;
-  __shared__ Sum s_wt[CK_THREADS / 32];
-  __shared__ Sum s_prefix;
-  __shared__ u32 s_segs;
-  const int t = threadIdx.x, w = t >> 5, lane = t & 31;
-  if (t == 0) {
-    s_tile = atomicAdd(a.tile_counter, 1u);
-    s_segs = 0;
-  }
-  __syncthreads();
-  const u32 tile = s_tile;
-  const u64 tbase = (u64)tile * CK_TILE;
-  const u64 base = tbase + (u64)t * CK_IPT;
+struct WarpEnd {  // final state of a warp's range (for the fallback of warp w+1)
+  u32 flag, lk, lw, fi;
+};
+
+// READINFLATE flag of item i (a read): its predecessor i-1 is a read of the same granule that
+// does not happen before it (Fig. 2, READINFLATE).
+__device__ __forceinline__ bool infl_flag(const HbCtx& c, u32 qev, u32 ev) {
+  const Snap s2 = load_snap(c.snap, ev >> 5);
+  const u32 qw = __ldg(&c.snap[qev >> 5].x);
+  return !hb_ev(c, qev, qw, ev, s2);
+}
+
+// State (lk, lw, fi) after item s-1 restricted to the granule of item s-1, computed from the
+// items before s.  Returns false if the walk exceeded the cap.
+__device__ bool walk_back(const CheckArgs& a, u64 s, Sum& out) {
   const HbCtx& c = a.c;
-
-  // ---- A: items + their records' snapshots (all gathers in flight together)
-  u32 kx[CK_IPT], ev[CK_IPT];
-  uint4 sn[CK_IPT];
-#pragma unroll
-  for (int j = 0; j < CK_IPT; ++j) {
-    u64 i = base + j;
-    kx[j] = i < a.n ? a.keys[i] : NONE;
-    ev[j] = i < a.n ? a.evs[i] : 0u;
+  const int lane = threadIdx.x & 31;
+  const u32 k0 = a.keys[s - 1] >> 2;
+  out = sum_ident();
+  out.fk = k0;
+  out.lk = k0;
+  out.bits = 1u;
+  u32 fi = NONE;
+  u64 hi = s - 1;  // highest item of the current window
+  for (u32 walked = 0;; walked += 32) {
+    if (walked >= K7_WALK_CAP) return false;
+    const u64 lo = hi >= 31 ? hi - 31 : 0;
+    const u64 i = lo + lane;
+    const bool in = i <= hi;
+    const u32 kx = in ? a.keys[i] : NONE, ev = in ? a.evs[i] : 0u;
+    const bool inkey = in && (kx >> 2) == k0;
+    const u32 W = __ballot_sync(0xFFFFFFFFu, inkey && (kx & 3u) != IOP_LD);
+    const u32 B = __ballot_sync(0xFFFFFFFFu, in && !inkey);  // other granules (below, keys sorted)
+    const int hw = W ? (int)hibit(W) : -1, hb_ = B ? (int)hibit(B) : -1;
+    const int bnd = hw > hb_ ? hw : hb_;  // the read run is (bnd, top]
+    // inflation flags of the run's reads (predecessor inside the run)
+    u32 qkx = __shfl_up_sync(0xFFFFFFFFu, kx, 1), qev = __shfl_up_sync(0xFFFFFFFFu, ev, 1);
+    if (lane == 0 && lo > 0) {
+      qkx = a.keys[lo - 1];
+      qev = a.evs[lo - 1];
+    }
+    const bool inrun = in && lane > bnd;
+    const bool e = inrun && (lane > 0 || lo > 0) && qkx != NONE && (qkx >> 2) == k0 && (qkx & 3u) == IOP_LD &&
+                   infl_flag(c, qev, ev);
+    const u32 I = __ballot_sync(0xFFFFFFFFu, e);
+    if (I) fi = (u32)(lo + __ffs(I) - 1);  // earlier windows hold earlier items
+    if (bnd >= 0 || lo == 0) {
+      if (hw >= 0 && hw > hb_) {
+        out.lw = (u32)(lo + hw) + 1u;
+        out.bits |= 2u;
+      }
+      out.fi = fi;
+      return true;
+    }
+    hi = lo - 1;
   }
-#pragma unroll
-  for (int j = 0; j < CK_IPT; ++j) sn[j] = base + j < a.n ? __ldg(c.snap + (ev[j] >> 5)) : make_uint4(0, 0, 0, 0);
-  // previous item (the last item of thread t-1, or the item before the tile)
-  u32 pkx = __shfl_up_sync(0xFFFFFFFFu, kx[CK_IPT - 1], 1);
-  u32 pev = __shfl_up_sync(0xFFFFFFFFu, ev[CK_IPT - 1], 1);
-  u32 pw = __shfl_up_sync(0xFFFFFFFFu, sn[CK_IPT - 1].x, 1);
-  if (lane == 0) {
-    if (base > 0 && base - 1 < a.n) {
-      pkx = a.keys[base - 1];
-      pev = a.evs[base - 1];
-      pw = __ldg(&c.snap[pev >> 5].x);
-    } else {
-      pkx = NONE;
+}
+
+__global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd* wend, u32 nw) {
+  const u32 w = blockIdx.x * K7_WARPS + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  const HbCtx& c = a.c;
+  const u32 lt = lanemask_lt();
+  const u64 nr = (a.n + 31) / 32;  // rounds in total
+  const u64 beg = (nr * w / nw) * 32, end = min(a.n, (nr * (w + 1) / nw) * 32);
+
+  // ---- incoming state
+  Sum carry = sum_ident();
+  u32 pkx = NONE, pev = 0;
+  if (beg > 0 && beg < end) {
+    pkx = a.keys[beg - 1];
+    pev = a.evs[beg - 1];
+    if ((pkx >> 2) == (a.keys[beg] >> 2)) {  // the first granule straddles the boundary
+      if (!walk_back(a, beg, carry)) {
+        // very long read run: take warp w-1's final state (all warps are co-resident)
+        volatile WarpEnd* pe = &wend[w - 1];
+        while (pe->flag == 0) {
+        }
+        __threadfence();
+        carry.fk = carry.lk = pe->lk;
+        carry.lw = pe->lw;
+        carry.fi = pe->fi;
+        carry.bits = 1u | (carry.lw ? 2u : 0u);
+      }
     }
   }
-#pragma unroll
-  for (int j = 0; j < CK_IPT; ++j) {
-    s_kx[t * CK_IPT + j] = kx[j];
-    s_ev[t * CK_IPT + j] = ev[j];
-    s_w[t * CK_IPT + j] = sn[j].x;
-  }
 
-  // ---- B: READINFLATE flags (a read whose predecessor read of the granule is unordered)
-  u32 infl = 0, segs = 0;
-  Sum mine = sum_ident();
-#pragma unroll
-  for (int j = 0; j < CK_IPT; ++j) {
-    const u64 i = base + j;
-    const u32 qkx = j ? kx[j - 1] : pkx;
-    const u32 qev = j ? ev[j - 1] : pev;
-    const u32 qw = j ? sn[j - 1].x : pw;
-    if (i < a.n) {
-      const u32 key = kx[j] >> 2, op = kx[j] & 3u;
-      const bool same = qkx != NONE && (qkx >> 2) == key;
-      if (!same) ++segs;
-      if (op == IOP_LD && same && (qkx & 3u) == IOP_LD && !hb_ev(c, qev, qw, ev[j], to_snap(sn[j]))) infl |= 1u << j;
-      Sum it;
-      it.fk = key;
-      it.lk = key;
-      it.lw = op != IOP_LD ? (u32)i + 1u : 0u;
-      it.fi = ((infl >> j) & 1u) ? (u32)i : NONE;
-      it.bits = 1u | (op != IOP_LD ? 2u : 0u);
-      mine = combine(mine, it);
-    }
-  }
-
-  // ---- C: block scan of thread summaries + look-back across tiles
-  Sum incl = mine;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    Sum left = shfl_up_sum(incl, o);
-    if (lane >= o) incl = combine(left, incl);
-  }
-  Sum excl = shfl_up_sum(incl, 1);
-  if (lane == 0) excl = sum_ident();
-  if (lane == 31) s_wt[w] = incl;
-  if (segs) atomicAdd(&s_segs, segs);
-  __syncthreads();
-  if (w == 0) {
-    Sum agg = sum_ident();
-    for (int ww = 0; ww < CK_THREADS / 32; ++ww) agg = combine(agg, s_wt[ww]);
-    Sum P = warp_lookback(a.status, tile, agg, lane);
-    if (lane == 0) {
-      s_prefix = P;
-      if (s_segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)s_segs);
-    }
-  }
-  Sum wp = sum_ident();
-  for (int ww = 0; ww < w; ++ww) wp = combine(wp, s_wt[ww]);
-  __syncthreads();
-  const Sum st = combine(s_prefix, combine(wp, excl));
-
-  // ---- D: per-item checks with the exact incoming state
+  // ---- the range, round by round
   const u32 no_sv = c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
-  u32 lk = st.lk, lw = st.lw, fi = st.fi;
+  u32 segs = 0;
+  u32 pf_k[K7_PF], pf_e[K7_PF];
 #pragma unroll
-  for (int j = 0; j < CK_IPT; ++j) {
-    const u64 i = base + j;
-    if (i < a.n) {
-      const u32 key = kx[j] >> 2, op = kx[j] & 3u;
-      const Snap s2 = to_snap(sn[j]);
-      const u32 qkx = j ? kx[j - 1] : pkx;
-      const u32 qev = j ? ev[j - 1] : pev;
-      const u32 qw = j ? sn[j - 1].x : pw;
-      if (key != lk) {
-        lk = key;
-        lw = 0;
-        fi = NONE;
+  for (int q = 0; q < K7_PF; ++q) {
+    const u64 i = beg + (u64)q * 32 + lane;
+    pf_k[q] = i < end ? a.keys[i] : NONE;
+    pf_e[q] = i < end ? a.evs[i] : 0u;
+  }
+  for (u64 base_r = beg; base_r < end; base_r += 32) {
+    const u64 i = base_r + lane;
+    const bool valid = i < end;
+    const u32 kx = pf_k[0], ev = pf_e[0];
+#pragma unroll
+    for (int q = 0; q + 1 < K7_PF; ++q) {
+      pf_k[q] = pf_k[q + 1];
+      pf_e[q] = pf_e[q + 1];
+    }
+    {
+      const u64 ip = base_r + (u64)K7_PF * 32 + lane;
+      pf_k[K7_PF - 1] = ip < end ? a.keys[ip] : NONE;
+      pf_e[K7_PF - 1] = ip < end ? a.evs[ip] : 0u;
+    }
+    u32 qkx = __shfl_up_sync(0xFFFFFFFFu, kx, 1);
+    u32 qev = __shfl_up_sync(0xFFFFFFFFu, ev, 1);
+    if (lane == 0) {
+      qkx = pkx;
+      qev = pev;
+    }
+    const u32 key = kx >> 2, op = kx & 3u;
+    const bool same = qkx != NONE && (qkx >> 2) == key;
+    const bool e = valid && op == IOP_LD && same && (qkx & 3u) == IOP_LD && infl_flag(c, qev, ev);
+    const u32 V = __ballot_sync(0xFFFFFFFFu, valid);
+    const u32 I = __ballot_sync(0xFFFFFFFFu, e);
+    const u32 W = __ballot_sync(0xFFFFFFFFu, valid && op != IOP_LD);
+    const u32 K = __ballot_sync(0xFFFFFFFFu, valid && !same);
+    segs += __popc(K);
+    const bool cont_key = carry.fk != NONE && carry.lk == key;
+    // segment start of this lane inside the round (-1: the key run continues from before)
+    const u32 Kle = K & (lt | (1u << lane));
+    const int sstart = Kle ? (int)hibit(Kle) : -1;
+    const u32 segm = sstart >= 0 ? (~0u << sstart) : ~0u;
+    const u32 cand = W & lt & segm;
+    const int lwl = cand ? (int)hibit(cand) : -1;
+    const u32 src = lwl >= 0 ? (u32)lwl : (u32)lane;
+    const u32 wkx = __shfl_sync(0xFFFFFFFFu, kx, src);
+    const u32 wev = __shfl_sync(0xFFFFFFFFu, ev, src);
+    if (valid) {
+      u32 lw = 0, pkx2 = 0, pev2 = 0;
+      if (lwl >= 0) {
+        lw = (u32)(base_r + lwl) + 1u;
+        pkx2 = wkx;
+        pev2 = wev;
+      } else if (sstart < 0 && cont_key && carry.lw) {
+        lw = carry.lw;
+        pkx2 = a.keys[lw - 1];
+        pev2 = a.evs[lw - 1];
       }
-      // W_x check (every rule of Fig. 2; atomics only against a plain last write)
-      if (lw) {
-        const u64 li = (u64)lw - 1;
-        u32 pkx2, pev2, pw2;
-        if (li >= tbase) {
-          pkx2 = s_kx[li - tbase];
-          pev2 = s_ev[li - tbase];
-          pw2 = s_w[li - tbase];
-        } else {
-          pkx2 = a.keys[li];
-          pev2 = a.evs[li];
-          pw2 = __ldg(&c.snap[pev2 >> 5].x);
+      const bool patm = (pkx2 & 3u) == IOP_ATOM;
+      const bool needW = lw && !(op == IOP_ATOM && patm);
+      const bool needR = op != IOP_LD && same && (qkx & 3u) == IOP_LD;
+      if (needW || needR) {
+        const Snap s2 = load_snap(c.snap, ev >> 5);
+        // W_x check (every rule of Fig. 2; atomics only against a plain last write)
+        if (needW) {
+          const u32 pw2 = __ldg(&c.snap[pev2 >> 5].x);
+          if (!hb_ev(c, pev2, pw2, ev, s2)) {
+            if (op == IOP_LD) {
+              emit(a, key, ev, pev2, patm ? BC_KIND_AR : BC_KIND_WR);
+            } else if (op == IOP_ATOM) {
+              emit(a, key, ev, pev2, BC_KIND_WA);
+            } else {
+              const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (pev2 >> 5) == (ev >> 5);
+              if (!filtered) emit(a, key, ev, pev2, patm ? BC_KIND_AW : BC_KIND_WW);
+            }
+          }
         }
-        const bool patm = (pkx2 & 3u) == IOP_ATOM;
-        if (op == IOP_LD) {
-          if (!hb_ev(c, pev2, pw2, ev[j], s2)) emit(a, key, ev[j], pev2, patm ? BC_KIND_AR : BC_KIND_WR);
-        } else if (op == IOP_ATOM) {
-          if (!patm && !hb_ev(c, pev2, pw2, ev[j], s2)) emit(a, key, ev[j], pev2, BC_KIND_WA);
-        } else if (!hb_ev(c, pev2, pw2, ev[j], s2)) {
-          const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (pev2 >> 5) == (ev[j] >> 5);
-          if (!filtered) emit(a, key, ev[j], pev2, patm ? BC_KIND_AW : BC_KIND_WW);
+        // R_x check at writers (WRITE* / *ATOM*: R_x ⪯ C_t as an epoch, R_x ⊑ C_t as a vector)
+        if (needR) {
+          const u32 kind = op == IOP_ATOM ? BC_KIND_RA : BC_KIND_RW;
+          // first READINFLATE in the read run ending at this writer
+          const int rs = lwl >= 0 ? lwl + 1 : sstart;  // -1: the run started before this round
+          const u32 Ir = I & lt & (rs >= 0 ? (~0u << rs) : ~0u);
+          u32 fi = NONE;
+          if (rs < 0 && cont_key && carry.fi != NONE) fi = carry.fi;  // the run's first inflation came earlier
+          else if (Ir) fi = (u32)(base_r + __ffs(Ir) - 1);
+          if (fi == NONE) {
+            const u32 qw = __ldg(&c.snap[qev >> 5].x);
+            if (!hb_ev(c, qev, qw, ev, s2)) emit(a, key, ev, qev, kind);
+          } else {
+            vc_check(a.evs, a.races, a.race_cnt, a.race_cap, (u64)fi - 1, i - 1, ev, s2.warp, s2.ps, s2.node,
+                     s2.blab, key, kind);
+          }
         }
-      }
-      // R_x check at writers (WRITE* / *ATOM*: R_x ⪯ C_t as an epoch, R_x ⊑ C_t as a vector)
-      if (op != IOP_LD && qkx != NONE && (qkx >> 2) == key && (qkx & 3u) == IOP_LD) {
-        const u32 kind = op == IOP_ATOM ? BC_KIND_RA : BC_KIND_RW;
-        if (fi == NONE) {
-          if (!hb_ev(c, qev, qw, ev[j], s2)) emit(a, key, ev[j], qev, kind);
-        } else {
-          vc_check(a.evs, a.races, a.race_cnt, a.race_cap, (u64)fi - 1, i - 1, ev[j], s2.warp, s2.ps, s2.node,
-                   s2.blab, key, kind);
-        }
-      }
-      if (op != IOP_LD) {
-        lw = (u32)i + 1u;
-        fi = NONE;
-      } else if (((infl >> j) & 1u) && fi == NONE) {
-        fi = (u32)i;
       }
     }
+    carry = combine(carry, round_sum(V, K, W, I, key, base_r));
+    const u32 last = hibit(V);
+    pkx = __shfl_sync(0xFFFFFFFFu, kx, last);
+    pev = __shfl_sync(0xFFFFFFFFu, ev, last);
+  }
+  if (lane == 0) {
+    if (segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)segs);
+    volatile WarpEnd* me = &wend[w];
+    me->lk = carry.lk;
+    me->lw = carry.lw;
+    me->fi = carry.fi;
+    __threadfence();
+    me->flag = 1u;
   }
 }
 
 }  // namespace
 
-size_t check_status_bytes(u64 n) { return ((n + CK_TILE - 1) / CK_TILE + 1) * sizeof(TileStatus); }
+size_t check_status_bytes(u64 n) { return (size_t)148 * 64 * sizeof(WarpEnd) + 256; }
 
 void launch_check(const HbCtx& c, const u32* keys, const u32* evs, u64 n, void* status, u32* tile_counter,
                   uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, cudaStream_t st) {
   if (n == 0) return;
-  u64 tiles = (n + CK_TILE - 1) / CK_TILE;
-  cudaMemsetAsync(status, 0, tiles * sizeof(TileStatus), st);
-  cudaMemsetAsync(tile_counter, 0, sizeof(u32), st);
+  static int grid = 0;
+  if (!grid) {
+    int dev = 0, sms = 0, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_check, K7_WARPS * 32, 0);
+    if (per < 1) per = 1;
+    grid = sms * per;
+    if (grid * K7_WARPS > 148 * 64) grid = 148 * 64 / K7_WARPS;
+  }
+  const u32 nw = (u32)grid * K7_WARPS;
+  cudaMemsetAsync(status, 0, (size_t)nw * sizeof(WarpEnd), st);
   cudaMemcpyToSymbolAsync(cHC, &c, sizeof(HbCtx), 0, cudaMemcpyHostToDevice, st);
   CheckArgs a;
   a.c = c;
   a.keys = keys;
   a.evs = evs;
   a.n = n;
-  a.status = (TileStatus*)status;
+  a.status = nullptr;
   a.tile_counter = tile_counter;
   a.races = races;
   a.race_cnt = race_cnt;
   a.race_cap = race_cap;
   a.seg_cnt = seg_cnt;
-  k_check<<<(unsigned)tiles, CK_THREADS, 0, st>>>(a); ++g_launches;
+  k_check<<<grid, K7_WARPS * 32, 0, st>>>(a, (WarpEnd*)status, nw); ++g_launches;
 }
 
 }  // namespace bc

@@ -66,7 +66,9 @@ void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, cons
                       cudaStream_t st);
 u64 expand_tiles(u64 n_recs);
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
-                   u32* keys, u32* evs, u64* status, u32* tile_counter, u64* cnt, u32* err, cudaStream_t st);
+                   u32* keys, u32* evs, u32* tile_off, u32* tile_cnt, u64* cnt, u32* err, cudaStream_t st);
+void launch_expand_place(const u32* skeys, const u32* sevs, const u32* tile_off, const u32* tile_cnt,
+                         const u32* tile_dst, u64 tiles, u32* okeys, u32* oevs, cudaStream_t st);
 void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st);
 
 // sync.cu

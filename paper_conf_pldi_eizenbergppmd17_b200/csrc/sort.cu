@@ -5,7 +5,8 @@
 // entry orders the host threads' accesses) turned into data parallelism: a STABLE sort of
 // (location key, trace position) items groups each location's accesses into one contiguous
 // segment that is still in trace order.  8-bit digits, 4096 keys per tile, one global
-// histogram pass for all digits, then one scatter pass per digit with decoupled look-back.
+// per pass: upsweep (per-tile digit counts), one exclusive scan over (digit, tile), downsweep
+// (stable in-tile rank, scatter through shared memory).
 #include "common.cuh"
 #include "kernels.cuh"
 
@@ -19,70 +20,45 @@ constexpr int RS_TILE = RS_THREADS * RS_ITEMS;  // 4096
 constexpr int RS_WARPS = RS_THREADS / 32;
 constexpr int RS_BINS = 256;
 
-__global__ void __launch_bounds__(256) k_rs_hist(const u32* __restrict__ keys, u64 n, int bit_lo, int passes,
-                                                 u32* __restrict__ hist) {
-  __shared__ u32 sh[4][RS_BINS];
-  for (int i = threadIdx.x; i < 4 * RS_BINS; i += blockDim.x) (&sh[0][0])[i] = 0;
+// upsweep: per-tile digit counts, digit-major (counts[d * tiles + tile]) so that one exclusive
+// scan gives every (digit, tile) its global output offset
+__global__ void __launch_bounds__(RS_THREADS) k_rs_upsweep(const u32* __restrict__ kin, u64 n, int shift, u64 tiles,
+                                                           u32* __restrict__ counts) {
+  __shared__ u32 h[RS_BINS];
+  const int t = threadIdx.x;
+  h[t] = 0;
   __syncthreads();
-  u64 stride = (u64)gridDim.x * blockDim.x;
-  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-    u32 k = keys[i];
-    for (int p = 0; p < passes; ++p) atomicAdd(&sh[p][(k >> (bit_lo + 8 * p)) & 0xFFu], 1u);
+  const u64 base = (u64)blockIdx.x * RS_TILE;
+#pragma unroll 4
+  for (int j = 0; j < RS_ITEMS; ++j) {
+    u64 idx = base + (u64)j * RS_THREADS + t;
+    if (idx < n) atomicAdd(&h[(kin[idx] >> shift) & 0xFFu], 1u);
   }
   __syncthreads();
-  for (int i = threadIdx.x; i < passes * RS_BINS; i += blockDim.x) {
-    u32 v = (&sh[0][0])[i];
-    if (v) atomicAdd(&hist[i], v);
-  }
+  counts[(u64)t * tiles + blockIdx.x] = h[t];
 }
 
-// exclusive scan of each pass's 256-bin histogram (one block of 256 threads)
-__global__ void k_rs_hist_scan(u32* hist, int passes) {
-  __shared__ u32 s[RS_BINS];
-  for (int p = 0; p < passes; ++p) {
-    u32 v = hist[p * RS_BINS + threadIdx.x];
-    s[threadIdx.x] = v;
-    __syncthreads();
-    for (int o = 1; o < RS_BINS; o <<= 1) {
-      u32 t = threadIdx.x >= (u32)o ? s[threadIdx.x - o] : 0;
-      __syncthreads();
-      s[threadIdx.x] += t;
-      __syncthreads();
-    }
-    hist[p * RS_BINS + threadIdx.x] = s[threadIdx.x] - v;
-    __syncthreads();
-  }
-}
-
-__global__ void __launch_bounds__(RS_THREADS) k_rs_onesweep(const u32* __restrict__ kin, const u32* __restrict__ vin,
-                                                            u32* __restrict__ kout, u32* __restrict__ vout, u64 n,
-                                                            int shift, const u32* __restrict__ digit_base,
-                                                            u64* status, u32* tile_counter) {
+// downsweep: stable rank inside the tile, then scatter through shared memory
+__global__ void __launch_bounds__(RS_THREADS, 2) k_rs_downsweep(const u32* __restrict__ kin, const u32* __restrict__ vin,
+                                                               u32* __restrict__ kout, u32* __restrict__ vout, u64 n,
+                                                               int shift, const u32* __restrict__ offs, u64 tiles) {
   __shared__ u32 skeys[RS_TILE];
   __shared__ u32 svals[RS_TILE];
   __shared__ u32 whist[RS_WARPS][RS_BINS];
   __shared__ u32 tofs[RS_BINS];
   __shared__ u32 gstart[RS_BINS];
-  __shared__ u32 s_tile;
 
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
-  if (t == 0) s_tile = atomicAdd(tile_counter, 1u);
   for (int i = t; i < RS_WARPS * RS_BINS; i += RS_THREADS) (&whist[0][0])[i] = 0;
   __syncthreads();
-  const u32 tile = s_tile;
+  const u32 tile = blockIdx.x;
   const u64 base = (u64)tile * RS_TILE;
 
-  u32 k[RS_ITEMS], v[RS_ITEMS], rank[RS_ITEMS];
+  u32 k[RS_ITEMS], rank[RS_ITEMS];
 #pragma unroll
   for (int j = 0; j < RS_ITEMS; ++j) {
     u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-    if (idx < n) {
-      k[j] = kin[idx];
-      v[j] = vin[idx];
-    } else {
-      k[j] = 0;
-      v[j] = 0;
-    }
+    k[j] = idx < n ? kin[idx] : 0u;
   }
   const u32 lt = lanemask_lt();
 #pragma unroll
@@ -105,28 +81,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_onesweep(const u32* __restric
     whist[ww][t] = total;
     total += c;
   }
-  // decoupled look-back per digit
-  {
-    volatile u64* st = status;
-    u64 excl = 0;
-    if (tile == 0) {
-      st[t] = LB_INC | total;
-    } else {
-      st[(u64)tile * RS_BINS + t] = LB_AGG | total;
-      int pt = (int)tile - 1;
-      while (true) {
-        u64 s = st[(u64)pt * RS_BINS + t];
-        u64 f = s & ~LB_MASK;
-        if (f == 0) continue;
-        excl += s & LB_MASK;
-        if (f == LB_INC) break;
-        --pt;
-      }
-      __threadfence();
-      st[(u64)tile * RS_BINS + t] = LB_INC | (excl + total);
-    }
-    gstart[t] = digit_base[t] + (u32)excl;
-  }
+  gstart[t] = offs[(u64)t * tiles + tile];
   // tile-local exclusive scan of totals over digits
   {
     u32 x = warp_incl_sum(total);
@@ -145,7 +100,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_onesweep(const u32* __restric
       u32 d = (k[j] >> shift) & 0xFFu;
       u32 pos = tofs[d] + whist[w][d] + rank[j];
       skeys[pos] = k[j];
-      svals[pos] = v[j];
+      svals[pos] = vin[idx];
     }
   }
   __syncthreads();
@@ -187,7 +142,10 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__
     if (ww < w) off += wsum[ww];
     agg += wsum[ww];
   }
-  if (t == 0) s_excl = lookback_u64(status, tile, agg);
+  if (w == 0) {
+    u64 e = lookback_u64_warp(status, tile, agg, l);
+    if (l == 0) s_excl = e;
+  }
   __syncthreads();
   u64 run = s_excl + off + x - sum;
 #pragma unroll
@@ -202,9 +160,10 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__
 }  // namespace
 
 // ------------------------------------------------------------------ host side
+size_t scan_temp_bytes(u64 n);
 size_t rs_temp_bytes(u64 n) {
   u64 tiles = (n + RS_TILE - 1) / RS_TILE;
-  return 4 * RS_BINS * sizeof(u32) + 64 + tiles * RS_BINS * sizeof(u64) + 256;
+  return ((tiles * RS_BINS * sizeof(u32) + 255) & ~(u64)255) + scan_temp_bytes(tiles * RS_BINS) + 256;
 }
 
 // Stable sort of (keys, vals) by key bits [bit_lo, bit_hi).  Result is in (keys, vals) when
@@ -214,22 +173,15 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   if (n <= 1 || bit_hi <= bit_lo) return false;
   int passes = (bit_hi - bit_lo + 7) / 8;
   if (passes > 4) passes = 4;
-  char* tp = (char*)temp;
-  u32* hist = (u32*)tp;
-  u32* counter = (u32*)(tp + 4 * RS_BINS * sizeof(u32));
-  u64* status = (u64*)(tp + 4 * RS_BINS * sizeof(u32) + 64);
-  u64 tiles = (n + RS_TILE - 1) / RS_TILE;
-  cudaMemsetAsync(hist, 0, 4 * RS_BINS * sizeof(u32), st);
-  int blocks = (int)((n + 255) / 256);
-  if (blocks > 148 * 8) blocks = 148 * 8;
-  k_rs_hist<<<blocks, 256, 0, st>>>(keys, n, bit_lo, passes, hist); ++g_launches;
-  k_rs_hist_scan<<<1, RS_BINS, 0, st>>>(hist, passes); ++g_launches;
+  const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
+  u32* counts = (u32*)temp;
+  void* stemp = (char*)temp + ((tiles * RS_BINS * sizeof(u32) + 255) & ~(u64)255);
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
   for (int p = 0; p < passes; ++p) {
-    cudaMemsetAsync(counter, 0, sizeof(u32), st);
-    cudaMemsetAsync(status, 0, tiles * RS_BINS * sizeof(u64), st);
-    k_rs_onesweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, bit_lo + 8 * p, hist + p * RS_BINS,
-                                                           status, counter); ++g_launches;
+    const int shift = bit_lo + 8 * p;
+    k_rs_upsweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, shift, tiles, counts); ++g_launches;
+    exclusive_scan_u32(counts, counts, tiles * RS_BINS, stemp, nullptr, st);
+    k_rs_downsweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, shift, counts, tiles); ++g_launches;
     u32* tk = ki; ki = ko; ko = tk;
     u32* tv = vi; vi = vo; vo = tv;
   }

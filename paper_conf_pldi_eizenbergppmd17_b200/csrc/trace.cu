@@ -94,14 +94,31 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
   // page marking: ST / ATOM on global memory
   u32 wr = __ballot_sync(0xFFFFFFFFu, valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) &&
                                           h.space == BC_SPACE_GLOBAL);
-  while (wr) {
-    int j = __ffs(wr) - 1;
-    wr &= wr - 1;
-    u32 m = __shfl_sync(0xFFFFFFFFu, h.mask, j);
-    u64 rj = gw * 32 + j;
-    if ((m >> lane) & 1u) {
-      u64 a = recs[rj].addr[lane];
-      u64 p = a >> 20;
+  while (wr) {  // 8 records' address rows in flight at a time
+    int js[8];
+    u64 a[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      js[k] = -1;
+      if (wr) {
+        js[k] = __ffs(wr) - 1;
+        wr &= wr - 1;
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      a[k] = ~0ull;
+      if (js[k] >= 0) {
+        u32 m = __shfl_sync(0xFFFFFFFFu, h.mask, js[k]);
+        if ((m >> lane) & 1u) a[k] = __ldg(&recs[gw * 32 + js[k]].addr[lane]);
+      } else {
+        __shfl_sync(0xFFFFFFFFu, h.mask, 0);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (a[k] == ~0ull) continue;
+      u64 p = a[k] >> 20;
       if (p >= (1ull << 28)) {
         set_err(err, ERR_OVERFLOW);
       } else {
@@ -155,14 +172,25 @@ __global__ void __launch_bounds__(128) k_replay(const bc_record* __restrict__ re
   bool bad = false;
   const u32 nb0 = node_base[w], bb0 = bar_base[w];
   const u32 i0 = warp_start[w], i1 = warp_start[w + 1];
-  u32 rn = i0 < i1 ? wrec[i0] : 0;
-  uint4 hn = i0 < i1 ? __ldg(reinterpret_cast<const uint4*>(recs + rn)) : make_uint4(0, 0, 0, 0);
+  constexpr int PF = 4;  // records whose headers are in flight together
+  u32 rq[PF];
+  uint4 hq[PF];
+#pragma unroll
+  for (int k = 0; k < PF; ++k) {
+    rq[k] = i0 + k < i1 ? wrec[i0 + k] : 0u;
+    hq[k] = i0 + k < i1 ? __ldg(reinterpret_cast<const uint4*>(recs + rq[k])) : make_uint4(0, 0, 0, 0);
+  }
   for (u32 i = i0; i < i1 && !bad; ++i) {
-    const u32 r = rn;
-    const uint4 hv = hn;
-    if (i + 1 < i1) {  // prefetch the next header
-      rn = wrec[i + 1];
-      hn = __ldg(reinterpret_cast<const uint4*>(recs + rn));
+    const u32 r = rq[0];
+    const uint4 hv = hq[0];
+#pragma unroll
+    for (int k = 0; k + 1 < PF; ++k) {
+      rq[k] = rq[k + 1];
+      hq[k] = hq[k + 1];
+    }
+    if (i + PF < i1) {  // prefetch PF records ahead
+      rq[PF - 1] = wrec[i + PF];
+      hq[PF - 1] = __ldg(reinterpret_cast<const uint4*>(recs + rq[PF - 1]));
     }
     const u32 mask = hv.y, op = hv.z & 0xFFu, aux = hv.w;
     if (need_next) {
@@ -265,61 +293,85 @@ __global__ void k_barriers(Geo g, const u32* __restrict__ bar_cnt, const u32* __
 // then shared granules (block, offset).  Accesses to never-written global
 // pages cannot take part in a race (every race needs a write) and are dropped.
 // Also validates per-lane alignment / shared bounds for every op <= AR_GLB.
-// One warp per record, 8 warps x EXP_RPW records per tile, tile offsets by decoupled look-back.
-constexpr int EXP_RPW = 16;
-constexpr int EXP_TILE = 8 * EXP_RPW;
+// One warp per record, EXP_WARPS warps x EXP_RPW records per tile, tile offsets by decoupled
+// look-back.  Loads are issued in three waves so that each warp has all its records' headers,
+// then all their address rows (coalesced 256 B each), then all page-table words in flight.
+constexpr int EXP_RPW = 8;
+constexpr int EXP_WARPS = 16;
+constexpr int EXP_TILE = EXP_WARPS * EXP_RPW;
 
-__global__ void __launch_bounds__(256) k_expand(const bc_record* __restrict__ recs, Geo g,
+__global__ void __launch_bounds__(EXP_WARPS * 32) k_expand(const bc_record* __restrict__ recs, Geo g,
                                                 const u32* __restrict__ page_bits,
                                                 const u32* __restrict__ page_rank, u32 shared_base,
-                                                u32* __restrict__ okeys, u32* __restrict__ oevs, u64* status,
-                                                u32* tile_counter,
+                                                u32* __restrict__ okeys, u32* __restrict__ oevs,
+                                                u32* __restrict__ tile_off, u32* __restrict__ tile_cnt,
                                                 u64* __restrict__ cnt, u32* __restrict__ err) {
-  __shared__ u32 s_tile;
   __shared__ u32 s_rcnt[EXP_TILE];
   __shared__ u64 s_base;
   const int t = threadIdx.x, w = t >> 5, lane = t & 31;
-  if (t == 0) s_tile = atomicAdd(tile_counter, 1u);
-  __syncthreads();
-  const u64 tile = s_tile;
+  const u64 tile = blockIdx.x;
+  const u64 r0 = tile * EXP_TILE + (u64)w * EXP_RPW;
+  // wave 1: headers (lane j < EXP_RPW holds record r0 + j)
+  uint4 hv = make_uint4(0, 0, 0xFFu, 0);  // op 0xFF: past the end
+  if (lane < EXP_RPW && r0 + lane < g.n_recs) hv = __ldg(reinterpret_cast<const uint4*>(recs + r0 + lane));
+  u32 hwarp[EXP_RPW], hmask[EXP_RPW], hz[EXP_RPW];
+#pragma unroll
+  for (int j = 0; j < EXP_RPW; ++j) {
+    hwarp[j] = __shfl_sync(0xFFFFFFFFu, hv.x, j);
+    hmask[j] = __shfl_sync(0xFFFFFFFFu, hv.y, j);
+    hz[j] = __shfl_sync(0xFFFFFFFFu, hv.z, j);
+  }
+  // wave 2: address rows of memory / sync records
+  u64 a[EXP_RPW];
+#pragma unroll
+  for (int j = 0; j < EXP_RPW; ++j) {
+    const u32 op = hz[j] & 0xFFu;
+    a[j] = 0;
+    if (op <= BC_OP_AR_GLB && ((hmask[j] >> lane) & 1u)) a[j] = __ldg(&recs[r0 + j].addr[lane]);
+  }
+  // wave 3: page-table words of global memory accesses
+  u32 pw[EXP_RPW], pr[EXP_RPW];
+#pragma unroll
+  for (int j = 0; j < EXP_RPW; ++j) {
+    const u32 op = hz[j] & 0xFFu, space = (hz[j] >> 8) & 0xFFu;
+    pw[j] = 0;
+    pr[j] = 0;
+    const u64 p = a[j] >> 20;
+    if (op <= BC_OP_ATOM && space == BC_SPACE_GLOBAL && ((hmask[j] >> lane) & 1u) && p < (1ull << 28)) {
+      pw[j] = __ldg(&page_bits[p >> 5]);
+      pr[j] = __ldg(&page_rank[p >> 5]);
+    }
+  }
   u32 key0[EXP_RPW], ngr[EXP_RPW], opc[EXP_RPW], incl[EXP_RPW];
   bool bad = false;
 #pragma unroll
   for (int j = 0; j < EXP_RPW; ++j) {
-    const u64 r = tile * EXP_TILE + w * EXP_RPW + j;
     key0[j] = 0;
     ngr[j] = 0;
     opc[j] = 0;
-    if (r < g.n_recs) {
-      uint4 hv = __ldg(reinterpret_cast<const uint4*>(recs + r));
-      const u32 mask = hv.y, op = hv.z & 0xFFu, space = (hv.z >> 8) & 0xFFu, sl = (hv.z >> 16) & 0xFFu,
-                fl = (hv.z >> 24) & 0xFFu;
-      if (op <= BC_OP_AR_GLB && ((mask >> lane) & 1u) && sl <= 4 && space <= 1 && hv.x < g.n_warps) {
-        const u64 a = __ldg(&recs[r].addr[lane]);
-        const u64 size = 1ull << sl;
-        if (a & (size - 1)) bad = true;  // natural alignment
-        if (space == BC_SPACE_SHARED && a + size > g.smem) bad = true;
-        if (op <= BC_OP_ATOM && !bad) {
-          u32 n = (u32)(size >> g.G);
-          if (n == 0) n = 1;
-          opc[j] = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM : ((fl & BC_REC_SAME_VALUE) ? IOP_ST_SV : IOP_ST);
-          if (space == BC_SPACE_SHARED) {
-            u32 blk = hv.x / g.wpb;
-            key0[j] = shared_base + blk * g.smem_gran + (u32)(a >> g.G);
-            ngr[j] = n;
-          } else {
-            u64 p = a >> 20;
-            if (p < (1ull << 28)) {
-              u32 word = page_bits[p >> 5];
-              u32 bit = (u32)(p & 31);
-              if ((word >> bit) & 1u) {
-                u32 dense = page_rank[p >> 5] + __popc(word & ((1u << bit) - 1u));
-                key0[j] = (dense << (20 - g.G)) | (u32)((a & 0xFFFFFull) >> g.G);
-                ngr[j] = n;
-              }
-            } else {
-              set_err(err, ERR_OVERFLOW);
+    const u32 op = hz[j] & 0xFFu, space = (hz[j] >> 8) & 0xFFu, sl = (hz[j] >> 16) & 0xFFu, fl = (hz[j] >> 24) & 0xFFu;
+    if (op <= BC_OP_AR_GLB && ((hmask[j] >> lane) & 1u) && sl <= 4 && space <= 1 && hwarp[j] < g.n_warps) {
+      const u64 size = 1ull << sl;
+      if (a[j] & (size - 1)) bad = true;  // natural alignment
+      if (space == BC_SPACE_SHARED && a[j] + size > g.smem) bad = true;
+      if (op <= BC_OP_ATOM && !bad) {
+        u32 n = (u32)(size >> g.G);
+        if (n == 0) n = 1;
+        opc[j] = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM : ((fl & BC_REC_SAME_VALUE) ? IOP_ST_SV : IOP_ST);
+        if (space == BC_SPACE_SHARED) {
+          key0[j] = shared_base + (hwarp[j] / g.wpb) * g.smem_gran + (u32)(a[j] >> g.G);
+          ngr[j] = n;
+        } else {
+          const u64 p = a[j] >> 20;
+          if (p < (1ull << 28)) {
+            const u32 bit = (u32)(p & 31);
+            if ((pw[j] >> bit) & 1u) {
+              const u32 dense = pr[j] + __popc(pw[j] & ((1u << bit) - 1u));
+              key0[j] = (dense << (20 - g.G)) | (u32)((a[j] & 0xFFFFFull) >> g.G);
+              ngr[j] = n;
             }
+          } else {
+            set_err(err, ERR_OVERFLOW);
           }
         }
       }
@@ -346,17 +398,18 @@ __global__ void __launch_bounds__(256) k_expand(const bc_record* __restrict__ re
       run += v[q];
     }
     u32 total = __shfl_sync(0xFFFFFFFFu, x, 31);
-    u64 b = lookback_u64_warp(status, (u32)tile, total, lane);
-    if (lane == 0) {
+    if (lane == 0) {  // staging slot (tiles land in any order; k_expand_place restores trace order)
+      u64 b = total ? atomicAdd((unsigned long long*)&cnt[C_ITEMS], (unsigned long long)total) : 0ull;
       s_base = b;
-      if ((tile + 1) * EXP_TILE >= g.n_recs) cnt[C_ITEMS] = b + total;  // last tile: item total
+      tile_off[tile] = (u32)b;
+      tile_cnt[tile] = total;
     }
   }
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < EXP_RPW; ++j) {
     if (ngr[j] == 0) continue;
-    const u64 r = tile * EXP_TILE + w * EXP_RPW + j;
+    const u64 r = r0 + j;
     u64 o = s_base + s_rcnt[w * EXP_RPW + j] + incl[j] - ngr[j];
     const u32 ev = (u32)(r << 5) | lane;
     for (u32 k = 0; k < ngr[j]; ++k) {
@@ -425,11 +478,33 @@ void launch_popc(const u32* bits, u32* out, u64 n, cudaStream_t st) {
 u64 expand_tiles(u64 n_recs) { return (n_recs + EXP_TILE - 1) / EXP_TILE; }
 
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
-                   u32* keys, u32* evs, u64* status, u32* tile_counter, u64* cnt, u32* err, cudaStream_t st) {
+                   u32* keys, u32* evs, u32* tile_off, u32* tile_cnt, u64* cnt, u32* err, cudaStream_t st) {
   u64 tiles = expand_tiles(g.n_recs);
   if (tiles == 0) return;
-  k_expand<<<(unsigned)tiles, 256, 0, st>>>(recs, g, page_bits, page_rank, shared_base, keys, evs, status,
-                                           tile_counter, cnt, err); ++g_launches;
+  k_expand<<<(unsigned)tiles, EXP_WARPS * 32, 0, st>>>(recs, g, page_bits, page_rank, shared_base, keys, evs,
+                                                      tile_off, tile_cnt, cnt, err); ++g_launches;
+}
+
+// staging -> trace order: tile t's items move from tile_off[t] to tile_dst[t] (exclusive scan
+// of the per-tile counts in tile order).  One warp per tile, coalesced.
+__global__ void k_expand_place(const u32* __restrict__ skeys, const u32* __restrict__ sevs,
+                               const u32* __restrict__ tile_off, const u32* __restrict__ tile_cnt,
+                               const u32* __restrict__ tile_dst, u64 tiles, u32* __restrict__ okeys,
+                               u32* __restrict__ oevs) {
+  const u64 tw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (tw >= tiles) return;
+  const u32 n = tile_cnt[tw], so = tile_off[tw], d = tile_dst[tw];
+  for (u32 k = lane; k < n; k += 32) {
+    okeys[d + k] = skeys[so + k];
+    oevs[d + k] = sevs[so + k];
+  }
+}
+void launch_expand_place(const u32* skeys, const u32* sevs, const u32* tile_off, const u32* tile_cnt,
+                         const u32* tile_dst, u64 tiles, u32* okeys, u32* oevs, cudaStream_t st) {
+  if (!tiles) return;
+  k_expand_place<<<(unsigned)((tiles * 32 + 255) / 256), 256, 0, st>>>(skeys, sevs, tile_off, tile_cnt, tile_dst,
+                                                                       tiles, okeys, oevs); ++g_launches;
 }
 
 __global__ void k_node_base(const u32* __restrict__ if_excl, u32 n_warps, u32* __restrict__ node_base) {
