@@ -205,13 +205,14 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* bar_cnt = S.alloc<u32>(g.n_warps + 1);
   u32* sync_list = S.alloc<u32>(n);
   u32* page_bits = S.alloc<u32>(nwords);
+  u32* ub_off = S.alloc<u32>(n + 1);  // per record: upper bound of its items, then its first slot
   cudaMemsetAsync(err, 0, 4, st);
   cudaMemsetAsync(cnt, 0, C_N * 8, st);
   cudaMemsetAsync(if_cnt, 0, (g.n_warps + 1) * 4, st);
   cudaMemsetAsync(bar_cnt, 0, (g.n_warps + 1) * 4, st);
   cudaMemsetAsync(page_bits, 0, nwords * 4, st);
   // ---- header pass
-  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt, err, st);
+  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt, ub_off, err, st);
   u32* page_rank = S.alloc<u32>(nwords);
   u64* tot = S.alloc<u64>(4);
   launch_popc(page_bits, page_rank, nwords, st);
@@ -267,14 +268,17 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   cudaEventRecord(c->ev[3], st);
   bc_status cs = cuda_check(c, "replay");
   if (cs) return cs;
-  cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
-  if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "replay");
-  if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "SIMT stack / barrier feasibility");
+  if (hc_cnt[C_SYNC_RECS]) {  // K3 walks snapshots: make sure the replay accepted the trace
+    cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
+    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "replay");
+    if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "SIMT stack / barrier feasibility");
+  }
 
   HbCtx hc{};
   hc.g = g;
   hc.snap = snap;
   hc.nodes = nodes;
+  hc.n_nodes = (u32)n_nodes;
   hc.err = err;
   hc.n_acq = 0;
   hc.n_idx = 0;
@@ -285,67 +289,55 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     if (rs) return fail(c, (bc_status)rs, "sync skeleton");
   }
   cudaEventRecord(c->ev[4], st);
-  // ---- K4: expansion
+  // ---- K4: expansion (static slots from the header's per-record upper bounds)
   const u64 bound = hc_cnt[C_ITEM_BOUND];
-  u32* skeys0 = S.alloc<u32>(bound + 1);  // staging (tiles in completion order)
-  u32* sevs0 = S.alloc<u32>(bound + 1);
-  u32* ikeys = S.alloc<u32>(bound + 1);   // trace order
+  exclusive_scan_u32(ub_off, ub_off, n, S.alloc<char>(scan_temp_bytes(n)), nullptr, st);
+  u32* ikeys = S.alloc<u32>(bound + 1);
   u32* ievs = S.alloc<u32>(bound + 1);
-  u64 tiles = expand_tiles(n);
-  u32* tile_off = S.alloc<u32>(tiles + 1);
-  u32* tile_cnt = S.alloc<u32>(tiles + 1);
-  u32* tile_dst = S.alloc<u32>(tiles + 1);
-  cudaMemsetAsync(cnt + C_ITEMS, 0, 8, st);
   cudaEventRecord(c->ev[14], st);
-  launch_expand(recs, g, page_bits, page_rank, shared_base, skeys0, sevs0, tile_off, tile_cnt, cnt, err, st);
-  exclusive_scan_u32(tile_cnt, tile_dst, tiles, S.alloc<char>(scan_temp_bytes(tiles)), nullptr, st);
-  launch_expand_place(skeys0, sevs0, tile_off, tile_cnt, tile_dst, tiles, ikeys, ievs, st);
+  launch_expand(recs, g, page_bits, page_rank, shared_base, ub_off, ikeys, ievs, err, st);
   cudaEventRecord(c->ev[15], st);
-  u64 n_items = 0;
-  u32 nfind = 0;
-  cudaMemcpyAsync(&n_items, cnt + C_ITEMS, 8, cudaMemcpyDeviceToHost, st);
-  cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
-  cudaMemcpyAsync(&nfind, find_cnt, 4, cudaMemcpyDeviceToHost, st);
   cudaEventRecord(c->ev[5], st);
-  if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "expand");
-  if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "infeasible trace");
-  if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "index overflow");
-  sx.items = n_items;
-  // ---- K5: stable radix sort by granule key
-  u32* ik2 = S.alloc<u32>(n_items + 1);
-  u32* iv2 = S.alloc<u32>(n_items + 1);
+  // ---- K5: stable radix sort by granule key; the first pass drops the never-written slots
+  u64* n_items_dev = cnt + C_ITEMS;
+  u32* ik2 = S.alloc<u32>(bound + 1);
+  u32* iv2 = S.alloc<u32>(bound + 1);
   int kbits = bits_for(n_keys ? n_keys - 1 : 0);
-  void* rtmp = S.alloc<char>(rs_temp_bytes(n_items));
+  void* rtmp = S.alloc<char>(rs_temp_bytes(bound));
   cudaEventRecord(c->ev[12], st);
-  alt = radix_sort_pairs(ikeys, ievs, ik2, iv2, n_items, 2, 2 + kbits, rtmp, st);
+  alt = radix_sort_pairs(ikeys, ievs, ik2, iv2, bound, 2, 2 + kbits, rtmp, st, nullptr, n_items_dev, true);
   cudaEventRecord(c->ev[13], st);
   u32* skey = alt ? ik2 : ikeys;
   u32* sev = alt ? iv2 : ievs;
   cudaEventRecord(c->ev[6], st);
   // ---- K7: shadow check
-  u32 race_cap = (u32)std::min<u64>(std::max<u64>(1u << 16, n_items / 16), 1u << 30);
+  u32 race_cap = (u32)std::min<u64>(std::max<u64>(1u << 16, bound / 16), 1u << 30);
   uint4* rbuf = nullptr;
   u32* rcnt = S.alloc<u32>(1);
   u64* segc = S.alloc<u64>(1);
-  void* cstatus = S.alloc<char>(check_status_bytes(n_items));
-  u32* ccounter = S.alloc<u32>(1);
-  u32 n_r = 0;
+  void* cstatus = S.alloc<char>(check_status_bytes(bound));
+  u32 n_r = 0, nfind = 0;
+  u64 n_items = 0;
   for (int attempt = 0; attempt < 2; ++attempt) {
     rbuf = S.alloc<uint4>(race_cap);
     cudaMemsetAsync(rcnt, 0, 4, st);
     cudaMemsetAsync(segc, 0, 8, st);
-    cudaMemsetAsync(err, 0, 4, st);
     cudaEventRecord(c->ev[10], st);
-    launch_check(hc, skey, sev, n_items, cstatus, ccounter, rbuf, rcnt, race_cap, segc, st);
+    launch_check(hc, skey, sev, n_items_dev, bound, cstatus, rbuf, rcnt, race_cap, segc, st);
     cudaEventRecord(c->ev[11], st);
     cudaMemcpyAsync(&n_r, rcnt, 4, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&sx.segments, segc, 8, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(&n_items, n_items_dev, 8, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(&nfind, find_cnt, 4, cudaMemcpyDeviceToHost, st);
     if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "check");
+    if (herr) break;
     if (n_r <= race_cap) break;
     race_cap = n_r;
   }
-  if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "sync lookup step cap");
+  if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "infeasible trace");
+  if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "index overflow / sync lookup step cap");
+  sx.items = n_items;
   cudaEventRecord(c->ev[7], st);
   // ---- K8: finalize
   u64 total = (u64)n_r + nfind;

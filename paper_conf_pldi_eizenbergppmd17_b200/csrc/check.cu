@@ -80,9 +80,9 @@ struct CheckArgs {
   HbCtx c;
   const u32* keys;  // (granule key << 2) | op
   const u32* evs;   // (record << 5) | lane
-  u64 n;
+  u64 n;            // set on the device from *n_dev
   TileStatus* status;
-  u32* tile_counter;
+  const u64* n_dev;
   uint4* races;  // (key, cur_ev, prior_ev, kind)
   u32* race_cnt;
   u32 race_cap;
@@ -243,12 +243,13 @@ __device__ bool walk_back(const CheckArgs& a, u64 s, Sum& out) {
 }
 
 __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd* wend, u32 nw) {
+  const u64 n = *a.n_dev;
   const u32 w = blockIdx.x * K7_WARPS + (threadIdx.x >> 5);
   const int lane = threadIdx.x & 31;
   const HbCtx& c = a.c;
   const u32 lt = lanemask_lt();
-  const u64 nr = (a.n + 31) / 32;  // rounds in total
-  const u64 beg = (nr * w / nw) * 32, end = min(a.n, (nr * (w + 1) / nw) * 32);
+  const u64 nr = (n + 31) / 32;  // rounds in total
+  const u64 beg = (nr * w / nw) * 32, end = min(n, (nr * (w + 1) / nw) * 32);
 
   // ---- incoming state
   Sum carry = sum_ident();
@@ -388,9 +389,9 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
 
 size_t check_status_bytes(u64 n) { return (size_t)148 * 64 * sizeof(WarpEnd) + 256; }
 
-void launch_check(const HbCtx& c, const u32* keys, const u32* evs, u64 n, void* status, u32* tile_counter,
+void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_dev, u64 n_max, void* status,
                   uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, cudaStream_t st) {
-  if (n == 0) return;
+  if (n_max == 0) return;
   static int grid = 0;
   if (!grid) {
     int dev = 0, sms = 0, per = 0;
@@ -408,9 +409,9 @@ void launch_check(const HbCtx& c, const u32* keys, const u32* evs, u64 n, void* 
   a.c = c;
   a.keys = keys;
   a.evs = evs;
-  a.n = n;
+  a.n = 0;
   a.status = nullptr;
-  a.tile_counter = tile_counter;
+  a.n_dev = n_dev;
   a.races = races;
   a.race_cnt = race_cnt;
   a.race_cap = race_cap;

@@ -31,6 +31,8 @@ constexpr u32 ERR_OVERFLOW = 2u;
 
 // item op codes (2 low bits of an item's key word)
 constexpr u32 IOP_LD = 0, IOP_ST = 1, IOP_ST_SV = 2, IOP_ATOM = 3;
+// item key of a dropped slot (never-written global page); removed by the first radix pass
+constexpr u32 KEY_DROP = 0xFFFFFFFFu;
 
 // sync-index key space (K3)
 constexpr u32 KEY_BLOCK = 0x80000000u;  // block-level entry: key = KEY_BLOCK | block
@@ -107,6 +109,7 @@ struct HbCtx {
   Geo g;
   const uint4* snap;      // [n_recs]
   const uint4* nodes;     // [n_nodes]
+  u32 n_nodes;
   // foreign knowledge (K3); n_acq == 0 => none
   u32 n_acq;
   const u32* acq_block_start;  // [n_blocks + 1] ranges into acq_*
@@ -124,13 +127,14 @@ struct HbCtx {
 
 // know_t(u) for u = lane `ul` of t's own warp, t executing a record with snapshot s (intra-warp
 // part only; the PTVC CONVERGED / DIVERGED / NESTEDDIVERGED lookup of Fig. 7).
-static __device__ __noinline__ u32 intra_walk(const uint4* __restrict__ nodes, u32 node, u32 ps, u32 ul) {
+static __device__ __noinline__ u32 intra_walk(const uint4* __restrict__ nodes, u32 n_nodes, u32 node, u32 ps, u32 ul) {
+  if (node >= n_nodes) return 0;  // only after an infeasible replay (result discarded)
   uint4 nd = __ldg(nodes + node);
   if ((nd.x >> ul) & 1u) return ps;
   // walk up the branch tree to the lowest ancestor whose mask holds ul
   for (int d = 0; d < 40; ++d) {
     u32 p = nd.y;
-    if (p == NONE) return 0;  // cannot happen for a valid lane (root mask = init mask)
+    if (p >= n_nodes) return 0;  // NONE: cannot happen for a valid lane (root mask = init mask)
     uint4 pd = __ldg(nodes + p);
     if ((pd.x >> ul) & 1u) return nd.z;
     nd = pd;
@@ -139,7 +143,7 @@ static __device__ __noinline__ u32 intra_walk(const uint4* __restrict__ nodes, u
 }
 __device__ __forceinline__ u32 intra_know(const HbCtx& c, const Snap& s, u32 ul) {
   if (s.node == s.warp) return s.ps;  // converged: every lane of the warp is in the root node
-  return intra_walk(c.nodes, s.node, s.ps, ul);
+  return intra_walk(c.nodes, c.n_nodes, s.node, s.ps, ul);
 }
 
 // structural happens-before: does t (executing record r2 with snapshot s2) know the step of

@@ -48,13 +48,13 @@ class Scratch {
 // sort.cu
 size_t rs_temp_bytes(u64 n);
 bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi, void* temp,
-                      cudaStream_t st);
+                      cudaStream_t st, const u64* n_dev = nullptr, u64* n_out_dev = nullptr, bool drop = false);
 size_t scan_temp_bytes(u64 n);
 void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_dev, cudaStream_t st);
 
 // trace.cu
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
-                   u32* sync_list, u32* page_bits, u64* cnt, u32* err, cudaStream_t st);
+                   u32* sync_list, u32* page_bits, u64* cnt, u32* rec_ub, u32* err, cudaStream_t st);
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st);
 void launch_replay(const bc_record* recs, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
                    const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next, u32* find_blk,
@@ -64,11 +64,8 @@ void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, cons
 void launch_popc(const u32* bits, u32* out, u64 n, cudaStream_t st);
 void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, const u32* bar_base, const u32* blockR,
                       cudaStream_t st);
-u64 expand_tiles(u64 n_recs);
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
-                   u32* keys, u32* evs, u32* tile_off, u32* tile_cnt, u64* cnt, u32* err, cudaStream_t st);
-void launch_expand_place(const u32* skeys, const u32* sevs, const u32* tile_off, const u32* tile_cnt,
-                         const u32* tile_dst, u64 tiles, u32* okeys, u32* oevs, cudaStream_t st);
+                   const u32* ub_off, u32* keys, u32* evs, u32* err, cudaStream_t st);
 void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st);
 
 // sync.cu
@@ -80,7 +77,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
 
 // check.cu
 size_t check_status_bytes(u64 n);
-void launch_check(const HbCtx& c, const u32* keys, const u32* evs, u64 n, void* status, u32* tile_counter,
+void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_dev, u64 n_max, void* status,
                   uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, cudaStream_t st);
 
 // finalize.cu

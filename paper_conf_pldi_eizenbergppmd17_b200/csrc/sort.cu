@@ -22,17 +22,24 @@ constexpr int RS_BINS = 256;
 
 // upsweep: per-tile digit counts, digit-major (counts[d * tiles + tile]) so that one exclusive
 // scan gives every (digit, tile) its global output offset
-__global__ void __launch_bounds__(RS_THREADS) k_rs_upsweep(const u32* __restrict__ kin, u64 n, int shift, u64 tiles,
-                                                           u32* __restrict__ counts) {
+// n = *n_dev when n_dev is set (item count known only on the device), else n_max.
+// drop: keys equal to KEY_DROP are not counted (first pass of a compacting sort).
+__global__ void __launch_bounds__(RS_THREADS) k_rs_upsweep(const u32* __restrict__ kin, u64 n_max,
+                                                           const u64* __restrict__ n_dev, int drop, int shift,
+                                                           u64 tiles, u32* __restrict__ counts) {
   __shared__ u32 h[RS_BINS];
   const int t = threadIdx.x;
+  const u64 n = n_dev ? *n_dev : n_max;
   h[t] = 0;
   __syncthreads();
   const u64 base = (u64)blockIdx.x * RS_TILE;
 #pragma unroll 4
   for (int j = 0; j < RS_ITEMS; ++j) {
     u64 idx = base + (u64)j * RS_THREADS + t;
-    if (idx < n) atomicAdd(&h[(kin[idx] >> shift) & 0xFFu], 1u);
+    if (idx < n) {
+      const u32 k = kin[idx];
+      if (!(drop && k == KEY_DROP)) atomicAdd(&h[(k >> shift) & 0xFFu], 1u);
+    }
   }
   __syncthreads();
   counts[(u64)t * tiles + blockIdx.x] = h[t];
@@ -40,19 +47,23 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_upsweep(const u32* __restrict
 
 // downsweep: stable rank inside the tile, then scatter through shared memory
 __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_downsweep(const u32* __restrict__ kin, const u32* __restrict__ vin,
-                                                               u32* __restrict__ kout, u32* __restrict__ vout, u64 n,
-                                                               int shift, const u32* __restrict__ offs, u64 tiles) {
+                                                               u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
+                                                               const u64* __restrict__ n_dev, int drop, int shift,
+                                                               const u32* __restrict__ offs, u64 tiles) {
   __shared__ u32 skeys[RS_TILE];
   __shared__ u32 svals[RS_TILE];
   __shared__ u32 whist[RS_WARPS][RS_BINS];
   __shared__ u32 tofs[RS_BINS];
   __shared__ u32 gstart[RS_BINS];
+  __shared__ u32 s_kept;
 
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
-  for (int i = t; i < RS_WARPS * RS_BINS; i += RS_THREADS) (&whist[0][0])[i] = 0;
-  __syncthreads();
+  const u64 n = n_dev ? *n_dev : n_max;
   const u32 tile = blockIdx.x;
   const u64 base = (u64)tile * RS_TILE;
+  if (base >= n) return;
+  for (int i = t; i < RS_WARPS * RS_BINS; i += RS_THREADS) (&whist[0][0])[i] = 0;
+  __syncthreads();
 
   u32 k[RS_ITEMS], rank[RS_ITEMS];
 #pragma unroll
@@ -64,7 +75,7 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_downsweep(const u32* __res
 #pragma unroll
   for (int j = 0; j < RS_ITEMS; ++j) {
     u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-    u32 d = idx < n ? ((k[j] >> shift) & 0xFFu) : 256u;
+    u32 d = (idx < n && !(drop && k[j] == KEY_DROP)) ? ((k[j] >> shift) & 0xFFu) : 256u;
     u32 peers = __match_any_sync(0xFFFFFFFFu, d);
     u32 old = d < 256u ? whist[w][d] : 0u;
     __syncwarp();
@@ -91,12 +102,13 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_downsweep(const u32* __res
     u32 off = 0;
     for (int ww = 0; ww < w; ++ww) off += wsum[ww];
     tofs[t] = off + x - total;
+    if (t == RS_BINS - 1) s_kept = off + x;  // kept items of the tile
   }
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < RS_ITEMS; ++j) {
     u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-    if (idx < n) {
+    if (idx < n && !(drop && k[j] == KEY_DROP)) {
       u32 d = (k[j] >> shift) & 0xFFu;
       u32 pos = tofs[d] + whist[w][d] + rank[j];
       skeys[pos] = k[j];
@@ -104,7 +116,7 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_downsweep(const u32* __res
     }
   }
   __syncthreads();
-  u32 tile_n = (u32)((n - base) < (u64)RS_TILE ? (n - base) : (u64)RS_TILE);
+  const u32 tile_n = s_kept;
   for (u32 q = t; q < tile_n; q += RS_THREADS) {
     u32 kk = skeys[q];
     u32 d = (kk >> shift) & 0xFFu;
@@ -167,21 +179,32 @@ size_t rs_temp_bytes(u64 n) {
 }
 
 // Stable sort of (keys, vals) by key bits [bit_lo, bit_hi).  Result is in (keys, vals) when
-// the function returns false, else in (keys_alt, vals_alt).
-bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi,
-                      void* temp, cudaStream_t st) {
-  if (n <= 1 || bit_hi <= bit_lo) return false;
+// the function returns false, else in (keys_alt, vals_alt).  n is the (upper bound of the) item
+// count; with n_dev the exact count is read on the device.  drop: the first pass removes items
+// whose key is KEY_DROP and writes the number kept to *n_out_dev (at least one pass is run).
+bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi, void* temp,
+                      cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop) {
+  if (!drop && (n <= 1 || bit_hi <= bit_lo)) return false;
+  if (n == 0) {
+    if (n_out_dev) cudaMemsetAsync(n_out_dev, 0, 8, st);
+    return false;
+  }
   int passes = (bit_hi - bit_lo + 7) / 8;
   if (passes > 4) passes = 4;
+  if (passes < 1) passes = 1;
   const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
   u32* counts = (u32*)temp;
   void* stemp = (char*)temp + ((tiles * RS_BINS * sizeof(u32) + 255) & ~(u64)255);
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
+  const u64* nd = n_dev;
   for (int p = 0; p < passes; ++p) {
     const int shift = bit_lo + 8 * p;
-    k_rs_upsweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, shift, tiles, counts); ++g_launches;
-    exclusive_scan_u32(counts, counts, tiles * RS_BINS, stemp, nullptr, st);
-    k_rs_downsweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, shift, counts, tiles); ++g_launches;
+    const int dr = (drop && p == 0) ? 1 : 0;
+    k_rs_upsweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, tiles, counts); ++g_launches;
+    exclusive_scan_u32(counts, counts, tiles * RS_BINS, stemp, dr ? n_out_dev : nullptr, st);
+    k_rs_downsweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, nd, dr, shift, counts, tiles);
+    ++g_launches;
+    if (dr) nd = n_out_dev;
     u32* tk = ki; ki = ko; ko = tk;
     u32* tv = vi; vi = vo; vo = tv;
   }

@@ -195,10 +195,10 @@ __device__ u32 laneop_entries(const K3In& k, u32 i, const EntOut* o, u32 base) {
     // structural clock of the releaser (its block only)
     u32 bl = s.blab;
     if (bl) put(o, n, tarr, KEY_BLOCK | b, ev, 0xFFFFFFFFu, bl);
-    {
+    if (s.node < c.n_nodes) {
       uint4 nd = c.nodes[s.node];
       if (s.ps) put(o, n, tarr, w, ev, nd.x, s.ps);
-      for (int d = 0; d < 40 && nd.y != NONE; ++d) {
+      for (int d = 0; d < 40 && nd.y < c.n_nodes; ++d) {
         uint4 pd = c.nodes[nd.y];
         if (nd.z) put(o, n, tarr, w, ev, pd.x, nd.z);
         nd = pd;

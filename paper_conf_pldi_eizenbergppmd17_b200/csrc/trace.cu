@@ -19,7 +19,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
                                                 u32* __restrict__ wval, u32* __restrict__ if_cnt,
                                                 u32* __restrict__ bar_cnt, u32* __restrict__ sync_list,
                                                 u32* __restrict__ page_bits, u64* __restrict__ cnt,
-                                                u32* __restrict__ err) {
+                                                u32* __restrict__ rec_ub, u32* __restrict__ err) {
   const u32 lane = threadIdx.x & 31;
   const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const u64 r = gw * 32 + lane;
@@ -69,6 +69,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
   if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
   // warp-reduced counters
   if (bad) ibound = 0;
+  if (valid) rec_ub[r] = ibound;  // upper bound of the record's items (K4 writes at static slots)
   u32 v[8] = {lane_ev, ctl_ev, is_acq, is_mem, is_if, is_bar, is_sync ? lane_ev : 0u, ibound};
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
@@ -287,33 +288,33 @@ __global__ void k_barriers(Geo g, const u32* __restrict__ bar_cnt, const u32* __
 // ---------------------------------------------------------------------------- k_expand
 // K4: lowering of each LD / ST / ATOM warp record into one thread operation per active lane
 // and per shadow granule (R7), emitted as 8-byte items
-//   x = (dense granule key << 2) | op,   y = event = (record << 5) | lane
-// in trace order (the radix sort that follows is stable).  Dense keys: global granules of
-// written 1-MB pages first (page rank from the write bitmap, so keys follow address order),
-// then shared granules (block, offset).  Accesses to never-written global
-// pages cannot take part in a race (every race needs a write) and are dropped.
-// Also validates per-lane alignment / shared bounds for every op <= AR_GLB.
-// One warp per record, EXP_WARPS warps x EXP_RPW records per tile, tile offsets by decoupled
-// look-back.  Loads are issued in three waves so that each warp has all its records' headers,
-// then all their address rows (coalesced 256 B each), then all page-table words in flight.
+//   key = (dense granule key << 2) | op,   ev = event = (record << 5) | lane
+// at static slots: record r owns [ub_off[r], ub_off[r] + popc(mask) * granules) (upper bound
+// from k_header), lane l the popc(mask & lanemask_lt) * granules slots of it -- so items land in
+// trace order with no synchronisation at all.  Dense keys: global granules of written 1-MB
+// pages first (page rank from the write bitmap, so keys follow address order), then shared
+// granules (block, offset).  Accesses to never-written global pages cannot take
+// part in a race (every race needs a write): their slots get the sentinel key
+// KEY_DROP, which the first radix pass removes.  Also validates per-lane alignment / shared
+// bounds for every op <= AR_GLB.  One warp per EXP_RPW consecutive records; loads issued in three
+// waves (headers, address rows, page-table words) so each warp has them all in flight.
 constexpr int EXP_RPW = 8;
-constexpr int EXP_WARPS = 16;
-constexpr int EXP_TILE = EXP_WARPS * EXP_RPW;
 
-__global__ void __launch_bounds__(EXP_WARPS * 32) k_expand(const bc_record* __restrict__ recs, Geo g,
+__global__ void __launch_bounds__(256) k_expand(const bc_record* __restrict__ recs, Geo g,
                                                 const u32* __restrict__ page_bits,
                                                 const u32* __restrict__ page_rank, u32 shared_base,
-                                                u32* __restrict__ okeys, u32* __restrict__ oevs,
-                                                u32* __restrict__ tile_off, u32* __restrict__ tile_cnt,
-                                                u64* __restrict__ cnt, u32* __restrict__ err) {
-  __shared__ u32 s_rcnt[EXP_TILE];
-  __shared__ u64 s_base;
-  const int t = threadIdx.x, w = t >> 5, lane = t & 31;
-  const u64 tile = blockIdx.x;
-  const u64 r0 = tile * EXP_TILE + (u64)w * EXP_RPW;
-  // wave 1: headers (lane j < EXP_RPW holds record r0 + j)
+                                                const u32* __restrict__ ub_off, u32* __restrict__ okeys,
+                                                u32* __restrict__ oevs, u32* __restrict__ err) {
+  const int lane = threadIdx.x & 31;
+  const u64 r0 = (((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * EXP_RPW;
+  if (r0 >= g.n_recs) return;
+  // wave 1: headers and slot offsets (lane j < EXP_RPW holds record r0 + j)
   uint4 hv = make_uint4(0, 0, 0xFFu, 0);  // op 0xFF: past the end
-  if (lane < EXP_RPW && r0 + lane < g.n_recs) hv = __ldg(reinterpret_cast<const uint4*>(recs + r0 + lane));
+  u32 uo = 0;
+  if (lane < EXP_RPW && r0 + lane < g.n_recs) {
+    hv = __ldg(reinterpret_cast<const uint4*>(recs + r0 + lane));
+    uo = __ldg(ub_off + r0 + lane);
+  }
   u32 hwarp[EXP_RPW], hmask[EXP_RPW], hz[EXP_RPW];
 #pragma unroll
   for (int j = 0; j < EXP_RPW; ++j) {
@@ -342,81 +343,46 @@ __global__ void __launch_bounds__(EXP_WARPS * 32) k_expand(const bc_record* __re
       pr[j] = __ldg(&page_rank[p >> 5]);
     }
   }
-  u32 key0[EXP_RPW], ngr[EXP_RPW], opc[EXP_RPW], incl[EXP_RPW];
-  bool bad = false;
+  const u32 lt = lanemask_lt();
+  bool bad = false, ovf = false;
 #pragma unroll
   for (int j = 0; j < EXP_RPW; ++j) {
-    key0[j] = 0;
-    ngr[j] = 0;
-    opc[j] = 0;
     const u32 op = hz[j] & 0xFFu, space = (hz[j] >> 8) & 0xFFu, sl = (hz[j] >> 16) & 0xFFu, fl = (hz[j] >> 24) & 0xFFu;
+    const u32 uoj = __shfl_sync(0xFFFFFFFFu, uo, j);
     if (op <= BC_OP_AR_GLB && ((hmask[j] >> lane) & 1u) && sl <= 4 && space <= 1 && hwarp[j] < g.n_warps) {
       const u64 size = 1ull << sl;
       if (a[j] & (size - 1)) bad = true;  // natural alignment
       if (space == BC_SPACE_SHARED && a[j] + size > g.smem) bad = true;
-      if (op <= BC_OP_ATOM && !bad) {
+      if (op <= BC_OP_ATOM) {
         u32 n = (u32)(size >> g.G);
         if (n == 0) n = 1;
-        opc[j] = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM : ((fl & BC_REC_SAME_VALUE) ? IOP_ST_SV : IOP_ST);
-        if (space == BC_SPACE_SHARED) {
-          key0[j] = shared_base + (hwarp[j] / g.wpb) * g.smem_gran + (u32)(a[j] >> g.G);
-          ngr[j] = n;
+        const u32 opc = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM
+                                                                 : ((fl & BC_REC_SAME_VALUE) ? IOP_ST_SV : IOP_ST);
+        u32 key0 = KEY_DROP;
+        if (bad) {
+        } else if (space == BC_SPACE_SHARED) {
+          key0 = shared_base + (hwarp[j] / g.wpb) * g.smem_gran + (u32)(a[j] >> g.G);
         } else {
           const u64 p = a[j] >> 20;
           if (p < (1ull << 28)) {
             const u32 bit = (u32)(p & 31);
-            if ((pw[j] >> bit) & 1u) {
-              const u32 dense = pr[j] + __popc(pw[j] & ((1u << bit) - 1u));
-              key0[j] = (dense << (20 - g.G)) | (u32)((a[j] & 0xFFFFFull) >> g.G);
-              ngr[j] = n;
-            }
+            if ((pw[j] >> bit) & 1u)
+              key0 = (pr[j] + __popc(pw[j] & ((1u << bit) - 1u))) << (20 - g.G) | (u32)((a[j] & 0xFFFFFull) >> g.G);
           } else {
-            set_err(err, ERR_OVERFLOW);
+            ovf = true;
           }
+        }
+        const u64 o = (u64)uoj + (u64)__popc(hmask[j] & lt) * n;
+        const u32 ev = (u32)((r0 + j) << 5) | lane;
+        for (u32 k = 0; k < n; ++k) {
+          okeys[o + k] = key0 == KEY_DROP ? KEY_DROP : (((key0 + k) << 2) | opc);
+          oevs[o + k] = ev;
         }
       }
     }
-    incl[j] = warp_incl_sum(ngr[j]);
-    if (lane == 31) s_rcnt[w * EXP_RPW + j] = incl[j];
   }
   if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
-  __syncthreads();
-  if (w == 0) {
-    // exclusive scan of the EXP_TILE record counts (EXP_RPW per lane, in record order)
-    u32 v[EXP_RPW / 2 > 0 ? EXP_TILE / 32 : 1];
-    u32 sum = 0;
-#pragma unroll
-    for (int q = 0; q < EXP_TILE / 32; ++q) {
-      v[q] = s_rcnt[lane * (EXP_TILE / 32) + q];
-      sum += v[q];
-    }
-    u32 x = warp_incl_sum(sum);
-    u32 run = x - sum;
-#pragma unroll
-    for (int q = 0; q < EXP_TILE / 32; ++q) {
-      s_rcnt[lane * (EXP_TILE / 32) + q] = run;
-      run += v[q];
-    }
-    u32 total = __shfl_sync(0xFFFFFFFFu, x, 31);
-    if (lane == 0) {  // staging slot (tiles land in any order; k_expand_place restores trace order)
-      u64 b = total ? atomicAdd((unsigned long long*)&cnt[C_ITEMS], (unsigned long long)total) : 0ull;
-      s_base = b;
-      tile_off[tile] = (u32)b;
-      tile_cnt[tile] = total;
-    }
-  }
-  __syncthreads();
-#pragma unroll
-  for (int j = 0; j < EXP_RPW; ++j) {
-    if (ngr[j] == 0) continue;
-    const u64 r = r0 + j;
-    u64 o = s_base + s_rcnt[w * EXP_RPW + j] + incl[j] - ngr[j];
-    const u32 ev = (u32)(r << 5) | lane;
-    for (u32 k = 0; k < ngr[j]; ++k) {
-      okeys[o + k] = ((key0[j] + k) << 2) | opc[j];
-      oevs[o + k] = ev;
-    }
-  }
+  if (__any_sync(0xFFFFFFFFu, ovf) && lane == 0) set_err(err, ERR_OVERFLOW);
 }
 
 // page_rank[i] = number of set bits in page_bits[0..i)  (exclusive popcount scan input)
@@ -427,11 +393,12 @@ __global__ void k_popc(const u32* __restrict__ bits, u32* __restrict__ out, u64 
 
 // --------------------------------------------------------------------- host launchers
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
-                   u32* sync_list, u32* page_bits, u64* cnt, u32* err, cudaStream_t st) {
+                   u32* sync_list, u32* page_bits, u64* cnt, u32* rec_ub, u32* err, cudaStream_t st) {
   u64 warps = (g.n_recs + 31) / 32;
   if (warps == 0) return;
   u64 blocks = (warps + 7) / 8;
-  k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt, err); ++g_launches;
+  k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt,
+                                             rec_ub, err); ++g_launches;
 }
 
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st) {
@@ -475,44 +442,20 @@ void launch_popc(const u32* bits, u32* out, u64 n, cudaStream_t st) {
   k_popc<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(bits, out, n); ++g_launches;
 }
 
-u64 expand_tiles(u64 n_recs) { return (n_recs + EXP_TILE - 1) / EXP_TILE; }
-
-void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
-                   u32* keys, u32* evs, u32* tile_off, u32* tile_cnt, u64* cnt, u32* err, cudaStream_t st) {
-  u64 tiles = expand_tiles(g.n_recs);
-  if (tiles == 0) return;
-  k_expand<<<(unsigned)tiles, EXP_WARPS * 32, 0, st>>>(recs, g, page_bits, page_rank, shared_base, keys, evs,
-                                                      tile_off, tile_cnt, cnt, err); ++g_launches;
-}
-
-// staging -> trace order: tile t's items move from tile_off[t] to tile_dst[t] (exclusive scan
-// of the per-tile counts in tile order).  One warp per tile, coalesced.
-__global__ void k_expand_place(const u32* __restrict__ skeys, const u32* __restrict__ sevs,
-                               const u32* __restrict__ tile_off, const u32* __restrict__ tile_cnt,
-                               const u32* __restrict__ tile_dst, u64 tiles, u32* __restrict__ okeys,
-                               u32* __restrict__ oevs) {
-  const u64 tw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
-  if (tw >= tiles) return;
-  const u32 n = tile_cnt[tw], so = tile_off[tw], d = tile_dst[tw];
-  for (u32 k = lane; k < n; k += 32) {
-    okeys[d + k] = skeys[so + k];
-    oevs[d + k] = sevs[so + k];
-  }
-}
-void launch_expand_place(const u32* skeys, const u32* sevs, const u32* tile_off, const u32* tile_cnt,
-                         const u32* tile_dst, u64 tiles, u32* okeys, u32* oevs, cudaStream_t st) {
-  if (!tiles) return;
-  k_expand_place<<<(unsigned)((tiles * 32 + 255) / 256), 256, 0, st>>>(skeys, sevs, tile_off, tile_cnt, tile_dst,
-                                                                       tiles, okeys, oevs); ++g_launches;
-}
-
 __global__ void k_node_base(const u32* __restrict__ if_excl, u32 n_warps, u32* __restrict__ node_base) {
   u32 w = blockIdx.x * blockDim.x + threadIdx.x;
   if (w < n_warps) node_base[w] = n_warps + 2u * if_excl[w];
 }
 void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st) {
   k_node_base<<<(n_warps + 255) / 256, 256, 0, st>>>(if_excl, n_warps, node_base); ++g_launches;
+}
+
+void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
+                   const u32* ub_off, u32* keys, u32* evs, u32* err, cudaStream_t st) {
+  const u64 warps = (g.n_recs + EXP_RPW - 1) / EXP_RPW;
+  if (!warps) return;
+  k_expand<<<(unsigned)((warps * 32 + 255) / 256), 256, 0, st>>>(recs, g, page_bits, page_rank, shared_base, ub_off,
+                                                                  keys, evs, err); ++g_launches;
 }
 
 }  // namespace bc
