@@ -89,7 +89,7 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   u64 tpb = (u64)cfg->block_dim[0] * cfg->block_dim[1] * cfg->block_dim[2];
   if (nb == 0 || tpb == 0 || tpb > 1024 || nb * tpb > 0xFFFFFFFFull) return BC_ERR_INVALID_ARG;
   u64 wpb = (tpb + 31) / 32;
-  if (nb * wpb >= (1ull << 30)) return BC_ERR_INVALID_ARG;
+  if (nb * wpb >= (1ull << 30) || nb * wpb * wpb >= (1ull << 32)) return BC_ERR_INVALID_ARG;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
     cudaGetLastError();
@@ -106,6 +106,7 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   g.tpb = (u32)tpb;
   g.wpb = (u32)wpb;
   g.n_warps = (u32)(nb * wpb);
+  g.wpb_m = wpb == 1 ? 0u : (u32)(((1ull << 32) + wpb - 1) / wpb);
   g.G = cfg->granule_log2;
   g.smem = cfg->smem_bytes_per_block;
   g.smem_gran = (u32)(((u64)g.smem + (1u << g.G) - 1) >> g.G);
@@ -211,20 +212,34 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   cudaMemsetAsync(if_cnt, 0, (g.n_warps + 1) * 4, st);
   cudaMemsetAsync(bar_cnt, 0, (g.n_warps + 1) * 4, st);
   cudaMemsetAsync(page_bits, 0, nwords * 4, st);
-  // ---- header pass
-  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt, ub_off, err, st);
+  // ---- header pass; written pages ranked in address order from the list of non-zero bitmap words
+  u32* word_list = S.alloc<u32>(nwords);
+  u32* wl2 = S.alloc<u32>(nwords);
+  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, ub_off, err, st);
+  u32* words = word_list;
+  u32* wl_prefix = wl2;
   u32* page_rank = S.alloc<u32>(nwords);
-  u64* tot = S.alloc<u64>(4);
-  launch_popc(page_bits, page_rank, nwords, st);
-  exclusive_scan_u32(page_rank, page_rank, nwords, S.alloc<char>(scan_temp_bytes(nwords)), tot + 0, st);
+  u32* need_sort = S.alloc<u32>(1);
+  cudaMemsetAsync(need_sort, 0, 4, st);
+  launch_page_rank(words, cnt + C_PAGE_WORDS, page_bits, page_rank, wl_prefix, cnt + C_PAGES, need_sort, 0, st);
   cudaEventRecord(c->ev[1], st);
   u64 hc_cnt[C_N];
-  u32 herr = 0;
-  u64 n_pages = 0;
+  u32 herr = 0, h_need_sort = 0;
   cudaMemcpyAsync(hc_cnt, cnt, sizeof(hc_cnt), cudaMemcpyDeviceToHost, st);
   cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
-  cudaMemcpyAsync(&n_pages, tot, 8, cudaMemcpyDeviceToHost, st);
+  cudaMemcpyAsync(&h_need_sort, need_sort, 4, cudaMemcpyDeviceToHost, st);
   if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "header");
+  if (h_need_sort) {  // more non-zero page words than one CTA sorts: radix sort, then rank
+    const u64 nwl = hc_cnt[C_PAGE_WORDS];
+    if (radix_sort_pairs(word_list, nullptr, wl2, nullptr, nwl, 0, 23, S.alloc<char>(rs_temp_bytes(nwl)), st)) {
+      words = wl2;
+      wl_prefix = word_list;
+    }
+    launch_page_rank(words, cnt + C_PAGE_WORDS, page_bits, page_rank, wl_prefix, cnt + C_PAGES, need_sort, 1, st);
+    cudaMemcpyAsync(hc_cnt, cnt, sizeof(hc_cnt), cudaMemcpyDeviceToHost, st);
+    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "page rank");
+  }
+  const u64 n_pages = hc_cnt[C_PAGES], n_words = hc_cnt[C_PAGE_WORDS];
   sx.lane_events = hc_cnt[C_LANE_EVENTS];
   sx.control_events = hc_cnt[C_CONTROL_EVENTS];
   sx.sync_ops = hc_cnt[C_SYNC_LANEOPS];
@@ -352,7 +367,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     c->races_cap = std::max<u64>(total, 1);
   }
   u32* page_num = S.alloc<u32>(n_pages + 1);
-  if (n_r) launch_page_list(page_bits, page_rank, nwords, page_num, st);
+  if (n_r) launch_page_list(words, wl_prefix, page_bits, n_words, page_num, st);
   finalize_races(rbuf, n_r, find_blk, find_rec, nfind, g, snap, page_num, shared_base, (u32)n_keys, c->races, S, st);
   cudaEventRecord(c->ev[PH_N], st);
   if (cudaEventSynchronize(c->ev[PH_N]) != cudaSuccess) return cuda_check(c, "finalize");

@@ -12,19 +12,15 @@
 // the oracle").  So the whole automaton is two segmented scans over the sorted items —
 //   LW(i) = last writer before i in its granule          (segmented max)
 //   FI(i) = first inflating read in the run ending at i  (segmented min, reset at writers)
-// plus independent happens-before queries per item.  One tile = 2048 items; the scan state crosses
-// tiles by decoupled look-back, so arbitrarily long (hot) granule segments cost the same per item
-// as short ones, and the shadow state never has to be materialised in memory within a window.
+// plus independent happens-before queries per item, evaluated with warp ballots over rounds of 32
+// sorted items (below).  Arbitrarily long (hot) granule segments cost the same per item as short
+// ones, and the shadow state never has to be materialised in memory.
 #include "common.cuh"
 #include "kernels.cuh"
 
 namespace bc {
 
 namespace {
-
-constexpr int CK_THREADS = 256;
-constexpr int CK_IPT = 8;
-constexpr int CK_TILE = CK_THREADS * CK_IPT;
 
 struct Sum {
   u32 fk, lk, lw, fi, bits;  // bits: 1 = one key throughout, 2 = tail key run holds a writer
@@ -51,37 +47,10 @@ __device__ __forceinline__ Sum combine(const Sum& L, const Sum& R) {
   return o;
 }
 
-__device__ __forceinline__ Sum shfl_up_sum(const Sum& s, int o) {
-  Sum r;
-  r.fk = __shfl_up_sync(0xFFFFFFFFu, s.fk, o);
-  r.lk = __shfl_up_sync(0xFFFFFFFFu, s.lk, o);
-  r.lw = __shfl_up_sync(0xFFFFFFFFu, s.lw, o);
-  r.fi = __shfl_up_sync(0xFFFFFFFFu, s.fi, o);
-  r.bits = __shfl_up_sync(0xFFFFFFFFu, s.bits, o);
-  return r;
-}
-
-struct TileStatus {  // 32 B
-  u32 flag, fk, lk, lw, fi, bits, pad0, pad1;
-};
-
-__device__ __forceinline__ void publish(TileStatus* ts, const Sum& s, u32 flag) {
-  volatile TileStatus* v = ts;
-  v->fk = s.fk;
-  v->lk = s.lk;
-  v->lw = s.lw;
-  v->fi = s.fi;
-  v->bits = s.bits;
-  __threadfence();
-  v->flag = flag;
-}
-
 struct CheckArgs {
   HbCtx c;
   const u32* keys;  // (granule key << 2) | op
   const u32* evs;   // (record << 5) | lane
-  u64 n;            // set on the device from *n_dev
-  TileStatus* status;
   const u64* n_dev;
   uint4* races;  // (key, cur_ev, prior_ev, kind)
   u32* race_cnt;
@@ -112,7 +81,7 @@ __device__ __forceinline__ bool hb_ev(const HbCtx& c, u32 ev1, u32 w1, u32 ev2, 
     if (l1 == l2) return true;                   // program order
     if (s2.node == s2.warp && s2.ps >= r1 + 1u) return true;  // converged warp, endi join
   }
-  const bool sameb = (w1 / c.g.wpb) == (s2.warp / c.g.wpb);
+  const bool sameb = blk_of(c.g, w1) == blk_of(c.g, s2.warp);
   if (sameb && r1 + 1u <= s2.blab) return true;  // completed barrier (Fig. 3 BAR)
   if (c.n_acq == 0 && !(w1 == s2.warp && s2.node != s2.warp)) return false;
   return hb_slow(ev1, w1, ev2, s2.warp, s2.ps, s2.node, s2.blab);
@@ -242,6 +211,33 @@ __device__ bool walk_back(const CheckArgs& a, u64 s, Sum& out) {
   }
 }
 
+// Software pipeline per warp: items (key, ev) are loaded K7_PF rounds ahead, the 16-B clock
+// snapshot of each item's record K7_PS rounds ahead (its address is the item's ev, which arrived
+// K7_PF - K7_PS rounds earlier), so the happens-before queries of a round touch registers only.
+// The predecessor item's warp (for READINFLATE and the epoch R check) comes from the lane below by
+// a shuffle; the last writer's (key, ev, warp) is carried in registers across rounds.
+// An item's snapshot is gathered only if some query of the round can read it: an item alone in its
+// granule never needs one, nor does an atomic whose same-granule neighbours are atomics (its W check
+// is elided against the atomic before it, it is not a read, and the next item, if atomic, does not
+// check against it).  Every other consumer -- READINFLATE (both reads), the W check
+// (the current item and the last writer, which is followed by a read or by the checking item), the
+// R check at a writer (the writer and the read before it) -- lies inside this set.  On atomic-heavy
+// traces (C4/C5 cost/mask) this removes almost all random 16-B gathers.
+constexpr int K7_PS = 2;
+
+__device__ __forceinline__ uint4 snap_if_needed(const HbCtx& c, u32 k, u32 e, u32 kprev0, u32 knext31) {
+  const int lane = threadIdx.x & 31;
+  u32 kp = __shfl_up_sync(0xFFFFFFFFu, k, 1), kn = __shfl_down_sync(0xFFFFFFFFu, k, 1);
+  if (lane == 0) kp = kprev0;
+  if (lane == 31) kn = knext31;
+  if (k == NONE) return make_uint4(0, 0, 0, 0);
+  const u32 key = k >> 2;
+  const bool sp = kp != NONE && (kp >> 2) == key, sn = kn != NONE && (kn >> 2) == key;
+  const bool atm_only = (k & 3u) == IOP_ATOM && (!sp || (kp & 3u) == IOP_ATOM) && (!sn || (kn & 3u) == IOP_ATOM);
+  if ((!sp && !sn) || atm_only) return make_uint4(0, 0, 0, 0);
+  return __ldg(c.snap + (e >> 5));
+}
+
 __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd* wend, u32 nw) {
   const u64 n = *a.n_dev;
   const u32 w = blockIdx.x * K7_WARPS + (threadIdx.x >> 5);
@@ -253,10 +249,12 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
 
   // ---- incoming state
   Sum carry = sum_ident();
-  u32 pkx = NONE, pev = 0;
+  u32 pkx = NONE, pev = 0, pw = 0;      // item beg-1 (the predecessor of lane 0 in the first round)
+  u32 cwk = 0, cwe = 0, cww = 0;        // carried last writer: key word, event, warp
   if (beg > 0 && beg < end) {
     pkx = a.keys[beg - 1];
     pev = a.evs[beg - 1];
+    pw = __ldg(&c.snap[pev >> 5].x);
     if ((pkx >> 2) == (a.keys[beg] >> 2)) {  // the first granule straddles the boundary
       if (!walk_back(a, beg, carry)) {
         // very long read run: take warp w-1's final state (all warps are co-resident)
@@ -269,6 +267,11 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
         carry.fi = pe->fi;
         carry.bits = 1u | (carry.lw ? 2u : 0u);
       }
+      if (carry.lw) {
+        cwk = a.keys[carry.lw - 1];
+        cwe = a.evs[carry.lw - 1];
+        cww = __ldg(&c.snap[cwe >> 5].x);
+      }
     }
   }
 
@@ -276,35 +279,50 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
   const u32 no_sv = c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   u32 segs = 0;
   u32 pf_k[K7_PF], pf_e[K7_PF];
+  uint4 pf_s[K7_PS];
 #pragma unroll
   for (int q = 0; q < K7_PF; ++q) {
     const u64 i = beg + (u64)q * 32 + lane;
     pf_k[q] = i < end ? a.keys[i] : NONE;
     pf_e[q] = i < end ? a.evs[i] : 0u;
   }
+#pragma unroll
+  for (int q = 0; q < K7_PS; ++q) {
+    const u32 kp0 = q == 0 ? pkx : __shfl_sync(0xFFFFFFFFu, pf_k[q > 0 ? q - 1 : 0], 31);
+    const u32 kn31 = __shfl_sync(0xFFFFFFFFu, pf_k[q + 1], 0);
+    pf_s[q] = snap_if_needed(c, pf_k[q], pf_e[q], kp0, kn31);
+  }
   for (u64 base_r = beg; base_r < end; base_r += 32) {
     const u64 i = base_r + lane;
     const bool valid = i < end;
     const u32 kx = pf_k[0], ev = pf_e[0];
+    const Snap s2 = to_snap(pf_s[0]);
 #pragma unroll
     for (int q = 0; q + 1 < K7_PF; ++q) {
       pf_k[q] = pf_k[q + 1];
       pf_e[q] = pf_e[q + 1];
     }
+#pragma unroll
+    for (int q = 0; q + 1 < K7_PS; ++q) pf_s[q] = pf_s[q + 1];
     {
       const u64 ip = base_r + (u64)K7_PF * 32 + lane;
       pf_k[K7_PF - 1] = ip < end ? a.keys[ip] : NONE;
       pf_e[K7_PF - 1] = ip < end ? a.evs[ip] : 0u;
+      const u32 kp0 = __shfl_sync(0xFFFFFFFFu, K7_PS >= 2 ? pf_k[K7_PS >= 2 ? K7_PS - 2 : 0] : kx, 31);
+      const u32 kn31 = __shfl_sync(0xFFFFFFFFu, pf_k[K7_PS], 0);
+      pf_s[K7_PS - 1] = snap_if_needed(c, pf_k[K7_PS - 1], pf_e[K7_PS - 1], kp0, kn31);
     }
     u32 qkx = __shfl_up_sync(0xFFFFFFFFu, kx, 1);
     u32 qev = __shfl_up_sync(0xFFFFFFFFu, ev, 1);
+    u32 qw = __shfl_up_sync(0xFFFFFFFFu, s2.warp, 1);
     if (lane == 0) {
       qkx = pkx;
       qev = pev;
+      qw = pw;
     }
     const u32 key = kx >> 2, op = kx & 3u;
     const bool same = qkx != NONE && (qkx >> 2) == key;
-    const bool e = valid && op == IOP_LD && same && (qkx & 3u) == IOP_LD && infl_flag(c, qev, ev);
+    const bool e = valid && op == IOP_LD && same && (qkx & 3u) == IOP_LD && !hb_ev(c, qev, qw, ev, s2);
     const u32 V = __ballot_sync(0xFFFFFFFFu, valid);
     const u32 I = __ballot_sync(0xFFFFFFFFu, e);
     const u32 W = __ballot_sync(0xFFFFFFFFu, valid && op != IOP_LD);
@@ -320,59 +338,58 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
     const u32 src = lwl >= 0 ? (u32)lwl : (u32)lane;
     const u32 wkx = __shfl_sync(0xFFFFFFFFu, kx, src);
     const u32 wev = __shfl_sync(0xFFFFFFFFu, ev, src);
+    const u32 wwp = __shfl_sync(0xFFFFFFFFu, s2.warp, src);
     if (valid) {
-      u32 lw = 0, pkx2 = 0, pev2 = 0;
+      u32 pkx2 = 0, pev2 = 0, pw2 = 0;
+      bool haveW = false;
       if (lwl >= 0) {
-        lw = (u32)(base_r + lwl) + 1u;
-        pkx2 = wkx;
-        pev2 = wev;
+        pkx2 = wkx; pev2 = wev; pw2 = wwp; haveW = true;
       } else if (sstart < 0 && cont_key && carry.lw) {
-        lw = carry.lw;
-        pkx2 = a.keys[lw - 1];
-        pev2 = a.evs[lw - 1];
+        pkx2 = cwk; pev2 = cwe; pw2 = cww; haveW = true;
       }
       const bool patm = (pkx2 & 3u) == IOP_ATOM;
-      const bool needW = lw && !(op == IOP_ATOM && patm);
-      const bool needR = op != IOP_LD && same && (qkx & 3u) == IOP_LD;
-      if (needW || needR) {
-        const Snap s2 = load_snap(c.snap, ev >> 5);
-        // W_x check (every rule of Fig. 2; atomics only against a plain last write)
-        if (needW) {
-          const u32 pw2 = __ldg(&c.snap[pev2 >> 5].x);
-          if (!hb_ev(c, pev2, pw2, ev, s2)) {
-            if (op == IOP_LD) {
-              emit(a, key, ev, pev2, patm ? BC_KIND_AR : BC_KIND_WR);
-            } else if (op == IOP_ATOM) {
-              emit(a, key, ev, pev2, BC_KIND_WA);
-            } else {
-              const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (pev2 >> 5) == (ev >> 5);
-              if (!filtered) emit(a, key, ev, pev2, patm ? BC_KIND_AW : BC_KIND_WW);
-            }
-          }
+      const bool needW = valid && haveW && !(op == IOP_ATOM && patm);
+      const bool needR = valid && op != IOP_LD && same && (qkx & 3u) == IOP_LD;
+      // W_x check (every rule of Fig. 2; atomics only against a plain last write)
+      if (needW && !hb_ev(c, pev2, pw2, ev, s2)) {
+        if (op == IOP_LD) {
+          emit(a, key, ev, pev2, patm ? BC_KIND_AR : BC_KIND_WR);
+        } else if (op == IOP_ATOM) {
+          emit(a, key, ev, pev2, BC_KIND_WA);
+        } else {
+          const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (pev2 >> 5) == (ev >> 5);
+          if (!filtered) emit(a, key, ev, pev2, patm ? BC_KIND_AW : BC_KIND_WW);
         }
-        // R_x check at writers (WRITE* / *ATOM*: R_x ⪯ C_t as an epoch, R_x ⊑ C_t as a vector)
-        if (needR) {
-          const u32 kind = op == IOP_ATOM ? BC_KIND_RA : BC_KIND_RW;
-          // first READINFLATE in the read run ending at this writer
-          const int rs = lwl >= 0 ? lwl + 1 : sstart;  // -1: the run started before this round
-          const u32 Ir = I & lt & (rs >= 0 ? (~0u << rs) : ~0u);
-          u32 fi = NONE;
-          if (rs < 0 && cont_key && carry.fi != NONE) fi = carry.fi;  // the run's first inflation came earlier
-          else if (Ir) fi = (u32)(base_r + __ffs(Ir) - 1);
-          if (fi == NONE) {
-            const u32 qw = __ldg(&c.snap[qev >> 5].x);
-            if (!hb_ev(c, qev, qw, ev, s2)) emit(a, key, ev, qev, kind);
-          } else {
-            vc_check(a.evs, a.races, a.race_cnt, a.race_cap, (u64)fi - 1, i - 1, ev, s2.warp, s2.ps, s2.node,
-                     s2.blab, key, kind);
-          }
+      }
+      // R_x check at writers (WRITE* / *ATOM*: R_x ⪯ C_t as an epoch, R_x ⊑ C_t as a vector)
+      if (needR) {
+        const u32 kind = op == IOP_ATOM ? BC_KIND_RA : BC_KIND_RW;
+        // first READINFLATE in the read run ending at this writer
+        const int rs = lwl >= 0 ? lwl + 1 : sstart;  // -1: the run started before this round
+        const u32 Ir = I & lt & (rs >= 0 ? (~0u << rs) : ~0u);
+        u32 fi = NONE;
+        if (rs < 0 && cont_key && carry.fi != NONE) fi = carry.fi;  // the run's first inflation came earlier
+        else if (Ir) fi = (u32)(base_r + __ffs(Ir) - 1);
+        if (fi == NONE) {
+          if (!hb_ev(c, qev, qw, ev, s2)) emit(a, key, ev, qev, kind);
+        } else {
+          vc_check(a.evs, a.races, a.race_cnt, a.race_cap, (u64)fi - 1, i - 1, ev, s2.warp, s2.ps, s2.node,
+                   s2.blab, key, kind);
         }
       }
     }
-    carry = combine(carry, round_sum(V, K, W, I, key, base_r));
+    const Sum rsum = round_sum(V, K, W, I, key, base_r);
+    if (rsum.bits & 2u) {  // the round's tail key run holds a writer: it is the new carried writer
+      const u32 lwln = (u32)(rsum.lw - 1u - (u32)base_r);
+      cwk = __shfl_sync(0xFFFFFFFFu, kx, lwln);
+      cwe = __shfl_sync(0xFFFFFFFFu, ev, lwln);
+      cww = __shfl_sync(0xFFFFFFFFu, s2.warp, lwln);
+    }
+    carry = combine(carry, rsum);
     const u32 last = hibit(V);
     pkx = __shfl_sync(0xFFFFFFFFu, kx, last);
     pev = __shfl_sync(0xFFFFFFFFu, ev, last);
+    pw = __shfl_sync(0xFFFFFFFFu, s2.warp, last);
   }
   if (lane == 0) {
     if (segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)segs);
@@ -409,8 +426,6 @@ void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_
   a.c = c;
   a.keys = keys;
   a.evs = evs;
-  a.n = 0;
-  a.status = nullptr;
   a.n_dev = n_dev;
   a.races = races;
   a.race_cnt = race_cnt;

@@ -41,12 +41,16 @@ constexpr u32 SYNC_LOOKUP_CAP = 1u << 16;  // step cap of one foreign lookup
 
 struct Geo {
   u32 n_blocks, tpb, wpb, n_warps;
+  u32 wpb_m;       // ceil(2^32 / wpb), 0 when wpb == 1: block of warp w = umulhi(w, wpb_m) (exact: n_warps * wpb < 2^32)
   u32 G;           // granule_log2
   u32 smem;        // bytes per block
   u32 smem_gran;   // granules per block
   u32 flags;
   u64 n_recs;
 };
+
+// traced block of traced warp w without an integer division
+__device__ __forceinline__ u32 blk_of(const Geo& g, u32 w) { return g.wpb_m ? __umulhi(w, g.wpb_m) : w; }
 
 __host__ __device__ inline u32 init_mask(const Geo& g, u32 w) {
   u32 wib = w % g.wpb;
@@ -149,7 +153,7 @@ __device__ __forceinline__ u32 intra_know(const HbCtx& c, const Snap& s, u32 ul)
 // structural happens-before: does t (executing record r2 with snapshot s2) know the step of
 // (warp w1, lane l1) at record r1?  Same block only; no same-thread shortcut (callers do it).
 __device__ __forceinline__ bool struct_knows(const HbCtx& c, u32 w1, u32 l1, u32 r1, const Snap& s2) {
-  if (w1 / c.g.wpb != s2.warp / c.g.wpb) return false;
+  if (blk_of(c.g, w1) != blk_of(c.g, s2.warp)) return false;
   if (r1 + 1u <= s2.blab) return true;
   if (w1 == s2.warp && intra_know(c, s2, l1) >= r1 + 1u) return true;
   return false;

@@ -23,16 +23,18 @@ __global__ void k_field(const uint4* __restrict__ r, u32 n, int f, u32* __restri
   out[i] = f == 0 ? v.x : f == 1 ? v.y : v.z;
 }
 
-__global__ void k_page_list(const u32* __restrict__ bits, const u32* __restrict__ rank, u64 nwords,
-                            u32* __restrict__ page_num) {
+// rank -> page number, from the sorted list of non-zero bitmap words (k_page_rank)
+__global__ void k_page_list(const u32* __restrict__ words, const u32* __restrict__ wl_prefix,
+                            const u32* __restrict__ bits, u64 n_words, u32* __restrict__ page_num) {
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= nwords) return;
-  u32 b = bits[i];
-  u32 k = rank[i];
+  if (i >= n_words) return;
+  const u32 wd = words[i];
+  u32 b = bits[wd];
+  u32 k = wl_prefix[i];
   while (b) {
     int j = __ffs(b) - 1;
     b &= b - 1;
-    page_num[k++] = (u32)(i * 32 + j);
+    page_num[k++] = wd * 32u + (u32)j;
   }
 }
 
@@ -93,8 +95,10 @@ int bits_for(u64 maxval) {
 
 }  // namespace
 
-void launch_page_list(const u32* bits, const u32* rank, u64 nwords, u32* page_num, cudaStream_t st) {
-  k_page_list<<<nb(nwords), 256, 0, st>>>(bits, rank, nwords, page_num); ++g_launches;
+void launch_page_list(const u32* words, const u32* wl_prefix, const u32* page_bits, u64 n_words, u32* page_num,
+                      cudaStream_t st) {
+  if (!n_words) return;
+  k_page_list<<<nb(n_words), 256, 0, st>>>(words, wl_prefix, page_bits, n_words, page_num); ++g_launches;
 }
 
 // races[n_r] (key, cur, prior, kind) + findings -> out[n_f + n_r] in canonical order

@@ -14,7 +14,7 @@ extern u64 g_launches;
 
 // counters written by the kernels (u64 device array)
 enum { C_LANE_EVENTS = 0, C_CONTROL_EVENTS, C_SYNC_RECS, C_ACQ_RECS, C_MEM_RECS, C_IFS, C_BARS, C_SYNC_LANEOPS,
-       C_ITEMS, C_ITEM_BOUND, C_SEGMENTS, C_N };
+       C_ITEMS, C_ITEM_BOUND, C_SEGMENTS, C_PAGE_WORDS, C_PAGES, C_N };
 
 // Stream-ordered scratch memory for one bc_detect: cudaMallocAsync from the device's memory
 // pool (kept cached between calls), all freed at release().
@@ -54,14 +54,15 @@ void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_d
 
 // trace.cu
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
-                   u32* sync_list, u32* page_bits, u64* cnt, u32* rec_ub, u32* err, cudaStream_t st);
+                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, u32* err, cudaStream_t st);
+void launch_page_rank(u32* words, const u64* n_words_dev, const u32* page_bits, u32* page_rank, u32* wl_prefix,
+                      u64* n_pages_dev, u32* need_sort, int presorted, cudaStream_t st);
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st);
 void launch_replay(const bc_record* recs, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
                    const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next, u32* find_blk,
                    u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st);
 void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, const u32* bar_rec, const u32* bar_next,
                      u32* blockR, u32* err, cudaStream_t st);
-void launch_popc(const u32* bits, u32* out, u64 n, cudaStream_t st);
 void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, const u32* bar_base, const u32* blockR,
                       cudaStream_t st);
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
@@ -81,7 +82,8 @@ void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_
                   uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, cudaStream_t st);
 
 // finalize.cu
-void launch_page_list(const u32* bits, const u32* rank, u64 nwords, u32* page_num, cudaStream_t st);
+void launch_page_list(const u32* words, const u32* wl_prefix, const u32* page_bits, u64 n_words, u32* page_num,
+                      cudaStream_t st);
 void finalize_races(const uint4* races, u32 n_r, const u32* fblk, const u32* frec, u32 n_f, const Geo& g,
                     const uint4* snap, const u32* page_num, u32 shared_base, u32 n_keys, bc_race* out, Scratch& S,
                     cudaStream_t st);

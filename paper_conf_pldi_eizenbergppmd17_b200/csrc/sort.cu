@@ -1,12 +1,18 @@
-// sort.cu — hand-written stable LSD radix sort (onesweep-style, decoupled look-back) and
-// device-wide exclusive scan for sm_100a.
+// sort.cu — hand-written stable LSD radix sort (onesweep: one histogram pass, then one kernel per
+// 8-bit digit with decoupled look-back) and a device-wide exclusive scan, for sm_100a.
 //
 // The radix sort is the paper's per-location serialisation (a spinlock per shadow
 // entry orders the host threads' accesses) turned into data parallelism: a STABLE sort of
 // (location key, trace position) items groups each location's accesses into one contiguous
-// segment that is still in trace order.  8-bit digits, 4096 keys per tile, one global
-// per pass: upsweep (per-tile digit counts), one exclusive scan over (digit, tile), downsweep
-// (stable in-tile rank, scatter through shared memory).
+// segment that is still in trace order.
+//   k_rs_hist  : one read of the keys -> the global 256-bin histogram of every digit pass
+//   k_rs_bins  : exclusive scan of each pass's histogram (digit start offsets); kept-item count
+//   k_rs_pass  : per 4096-key tile (taken in launch order from an atomic ticket): stable in-tile
+//                rank (warp match + per-warp histograms), per-digit decoupled look-back over the
+//                preceding tiles, scatter through shared memory so that each digit's run is
+//                written contiguously.  Reads 8 B and writes 8 B per item: the pass roofline.
+#include <algorithm>
+
 #include "common.cuh"
 #include "kernels.cuh"
 
@@ -19,110 +25,194 @@ constexpr int RS_ITEMS = 16;
 constexpr int RS_TILE = RS_THREADS * RS_ITEMS;  // 4096
 constexpr int RS_WARPS = RS_THREADS / 32;
 constexpr int RS_BINS = 256;
+constexpr int RS_MAXP = 4;
+// temp header: ghist[RS_MAXP][256], gbase[RS_MAXP][256], tickets[RS_MAXP]; status arrays follow
+constexpr size_t RS_HDR_BYTES = (2 * RS_MAXP * 256 + 64) * sizeof(u32);
+// look-back status word per (tile, digit): [31:30] flag, [29:0] count (items < 2^30 per sort)
+constexpr u32 ST_AGG = 1u << 30, ST_INC = 2u << 30, ST_VAL = (1u << 30) - 1u;
+constexpr int RS_LB = 8;  // predecessors inspected per look-back step
 
-// upsweep: per-tile digit counts, digit-major (counts[d * tiles + tile]) so that one exclusive
-// scan gives every (digit, tile) its global output offset
-// n = *n_dev when n_dev is set (item count known only on the device), else n_max.
-// drop: keys equal to KEY_DROP are not counted (first pass of a compacting sort).
-__global__ void __launch_bounds__(RS_THREADS) k_rs_upsweep(const u32* __restrict__ kin, u64 n_max,
-                                                           const u64* __restrict__ n_dev, int drop, int shift,
-                                                           u64 tiles, u32* __restrict__ counts) {
-  __shared__ u32 h[RS_BINS];
+// Lanes of the warp holding the same 9-bit label (digit, or 256 = no item): 9 ballots, a fixed
+// cost independent of how many distinct digits the warp holds.
+__device__ __forceinline__ u32 match9(u32 d) {
+  u32 m = 0xFFFFFFFFu;
+#pragma unroll
+  for (int b = 0; b < 9; ++b) {
+    const bool bit = (d >> b) & 1u;
+    const u32 bal = __ballot_sync(0xFFFFFFFFu, bit);
+    m &= bit ? bal : ~bal;
+  }
+  return m;
+}
+
+constexpr int RS_HIST_ITEMS = 8;
+
+// Global digit histograms of all passes in one read.  Same-digit keys of a warp are combined
+// (match9) before the shared-memory atomic (sorted-ish inputs hit one bin hard).  Each thread keeps
+// RS_HIST_ITEMS loads in flight.
+__global__ void __launch_bounds__(RS_THREADS) k_rs_hist(const u32* __restrict__ kin, u64 n_max,
+                                                        const u64* __restrict__ n_dev, int drop, int bit_lo,
+                                                        int passes, u32* __restrict__ ghist) {
+  __shared__ u32 h[RS_MAXP][RS_BINS];
   const int t = threadIdx.x;
-  const u64 n = n_dev ? *n_dev : n_max;
-  h[t] = 0;
+  for (int i = t; i < RS_MAXP * RS_BINS; i += RS_THREADS) (&h[0][0])[i] = 0;
   __syncthreads();
-  const u64 base = (u64)blockIdx.x * RS_TILE;
-#pragma unroll 4
-  for (int j = 0; j < RS_ITEMS; ++j) {
-    u64 idx = base + (u64)j * RS_THREADS + t;
-    if (idx < n) {
-      const u32 k = kin[idx];
-      if (!(drop && k == KEY_DROP)) atomicAdd(&h[(k >> shift) & 0xFFu], 1u);
+  const u64 n = n_dev ? *n_dev : n_max;
+  const u32 lt = lanemask_lt();
+  constexpr int CH = RS_THREADS * RS_HIST_ITEMS;
+  const u64 stride = (u64)gridDim.x * CH;
+  for (u64 base = (u64)blockIdx.x * CH; base < n; base += stride) {
+    u32 k[RS_HIST_ITEMS];
+#pragma unroll
+    for (int j = 0; j < RS_HIST_ITEMS; ++j) {
+      const u64 idx = base + (u64)j * RS_THREADS + t;
+      k[j] = idx < n ? kin[idx] : KEY_DROP;
+    }
+#pragma unroll
+    for (int j = 0; j < RS_HIST_ITEMS; ++j) {
+      const u64 idx = base + (u64)j * RS_THREADS + t;
+      const bool ok = idx < n && !(drop && k[j] == KEY_DROP);
+      const u32 vm = __ballot_sync(0xFFFFFFFFu, ok);
+      for (int p = 0; p < passes; ++p) {
+        const u32 d = ok ? (k[j] >> (bit_lo + 8 * p)) & 0xFFu : 0x100u;
+        // one digit across the warp (the common case for the high digits): one atomic
+        const u32 d0 = __shfl_sync(0xFFFFFFFFu, d, vm ? __ffs(vm) - 1 : 0);
+        if (__all_sync(0xFFFFFFFFu, !ok || d == d0)) {
+          if (vm && (lt & vm) == 0 && ok) atomicAdd(&h[p][d], (u32)__popc(vm));
+        } else if (ok) {
+          atomicAdd(&h[p][d], 1u);
+        }
+      }
     }
   }
   __syncthreads();
-  counts[(u64)t * tiles + blockIdx.x] = h[t];
+  for (int i = t; i < passes * RS_BINS; i += RS_THREADS) {
+    const u32 v = (&h[0][0])[i];
+    if (v) atomicAdd(&ghist[i], v);
+  }
 }
 
-// downsweep: stable rank inside the tile, then scatter through shared memory
-__global__ void __launch_bounds__(RS_THREADS, 2) k_rs_downsweep(const u32* __restrict__ kin, const u32* __restrict__ vin,
-                                                               u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
-                                                               const u64* __restrict__ n_dev, int drop, int shift,
-                                                               const u32* __restrict__ offs, u64 tiles) {
+// gbase[p][d] = exclusive prefix of ghist[p][*]; *n_out = kept items (pass 0 total)
+__global__ void __launch_bounds__(RS_BINS) k_rs_bins(const u32* __restrict__ ghist, u32* __restrict__ gbase,
+                                                     u64* __restrict__ n_out) {
+  __shared__ u32 wsum[RS_BINS / 32];
+  const int t = threadIdx.x, w = t >> 5, l = t & 31, p = blockIdx.x;
+  const u32 v = ghist[p * RS_BINS + t];
+  const u32 x = warp_incl_sum(v);
+  if (l == 31) wsum[w] = x;
+  __syncthreads();
+  u32 off = 0, tot = 0;
+  for (int ww = 0; ww < RS_BINS / 32; ++ww) {
+    if (ww < w) off += wsum[ww];
+    tot += wsum[ww];
+  }
+  gbase[p * RS_BINS + t] = off + x - v;
+  if (p == 0 && t == 0 && n_out) *n_out = tot;
+}
+
+__global__ void __launch_bounds__(RS_THREADS, 2) k_rs_pass(const u32* __restrict__ kin, const u32* __restrict__ vin,
+                                                           u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
+                                                           const u64* __restrict__ n_dev, int drop, int shift,
+                                                           const u32* __restrict__ gbase, u32* __restrict__ status,
+                                                           u32* __restrict__ ticket) {
   __shared__ u32 skeys[RS_TILE];
   __shared__ u32 svals[RS_TILE];
   __shared__ u32 whist[RS_WARPS][RS_BINS];
   __shared__ u32 tofs[RS_BINS];
   __shared__ u32 gstart[RS_BINS];
-  __shared__ u32 s_kept;
+  __shared__ u32 wsum[RS_WARPS];
+  __shared__ u32 s_tile, s_kept;
 
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
-  const u64 n = n_dev ? *n_dev : n_max;
-  const u32 tile = blockIdx.x;
-  const u64 base = (u64)tile * RS_TILE;
-  if (base >= n) return;
+  if (t == 0) s_tile = atomicAdd(ticket, 1u);
   for (int i = t; i < RS_WARPS * RS_BINS; i += RS_THREADS) (&whist[0][0])[i] = 0;
   __syncthreads();
+  const u32 tile = s_tile;
+  const u64 n = n_dev ? *n_dev : n_max;
+  const u64 base = (u64)tile * RS_TILE;
+  if (base >= n) return;  // every later ticket is past the end too: nobody looks back at it
 
-  u32 k[RS_ITEMS], rank[RS_ITEMS];
+  u32 k[RS_ITEMS], v[RS_ITEMS], rank[RS_ITEMS];
 #pragma unroll
   for (int j = 0; j < RS_ITEMS; ++j) {
-    u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-    k[j] = idx < n ? kin[idx] : 0u;
+    const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
+    k[j] = idx < n ? kin[idx] : KEY_DROP;
+    v[j] = (vin && idx < n) ? vin[idx] : 0u;
   }
   const u32 lt = lanemask_lt();
 #pragma unroll
   for (int j = 0; j < RS_ITEMS; ++j) {
-    u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-    u32 d = (idx < n && !(drop && k[j] == KEY_DROP)) ? ((k[j] >> shift) & 0xFFu) : 256u;
-    u32 peers = __match_any_sync(0xFFFFFFFFu, d);
-    u32 old = d < 256u ? whist[w][d] : 0u;
+    const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
+    const u32 d = (idx < n && !(drop && k[j] == KEY_DROP)) ? ((k[j] >> shift) & 0xFFu) : 256u;
+    const u32 peers = match9(d);
+    const u32 old = d < 256u ? whist[w][d] : 0u;
     __syncwarp();
     if (d < 256u && (peers & lt) == 0) whist[w][d] = old + __popc(peers);
     __syncwarp();
-    rank[j] = old + __popc(peers & lt);
+    rank[j] = d < 256u ? old + __popc(peers & lt) : NONE;
   }
   __syncthreads();
-  // per digit: exclusive prefix over warps, tile total
+  // per digit (thread t): prefix over warps, tile total
   u32 total = 0;
 #pragma unroll
   for (int ww = 0; ww < RS_WARPS; ++ww) {
-    u32 c = whist[ww][t];
+    const u32 c = whist[ww][t];
     whist[ww][t] = total;
     total += c;
   }
-  gstart[t] = offs[(u64)t * tiles + tile];
-  // tile-local exclusive scan of totals over digits
+  // publish the tile aggregate, then look back for the exclusive prefix of this digit
+  volatile u32* vs = status;
+  u32 excl = 0;
+  if (tile == 0) {
+    vs[t] = ST_INC | total;
+  } else {
+    vs[(u64)tile * RS_BINS + t] = ST_AGG | total;
+    // walk back RS_LB predecessors per step with all their loads in flight (the first wave of
+    // co-resident tiles would otherwise walk up to ~300 tiles one L2 round trip at a time)
+    bool done = false;
+    for (u64 pt = tile; !done; pt = pt > RS_LB ? pt - RS_LB : 0) {
+      u32 s[RS_LB];
+#pragma unroll
+      for (int q = 0; q < RS_LB; ++q) s[q] = pt > (u64)q ? vs[(pt - 1 - q) * RS_BINS + t] : (u32)(2u << 30);
+#pragma unroll
+      for (int q = 0; q < RS_LB; ++q) {
+        if (done) break;
+        while ((s[q] & ~ST_VAL) == 0) s[q] = vs[(pt - 1 - q) * RS_BINS + t];
+        excl += s[q] & ST_VAL;
+        if (s[q] & ST_INC) done = true;
+      }
+    }
+    vs[(u64)tile * RS_BINS + t] = ST_INC | (excl + total);
+  }
+  gstart[t] = gbase[t] + excl;
+  // tile-local exclusive scan of the digit totals
   {
-    u32 x = warp_incl_sum(total);
-    __shared__ u32 wsum[RS_WARPS];
+    const u32 x = warp_incl_sum(total);
     if (l == 31) wsum[w] = x;
     __syncthreads();
     u32 off = 0;
     for (int ww = 0; ww < w; ++ww) off += wsum[ww];
     tofs[t] = off + x - total;
-    if (t == RS_BINS - 1) s_kept = off + x;  // kept items of the tile
+    if (t == RS_BINS - 1) s_kept = off + x;
   }
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < RS_ITEMS; ++j) {
-    u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-    if (idx < n && !(drop && k[j] == KEY_DROP)) {
-      u32 d = (k[j] >> shift) & 0xFFu;
-      u32 pos = tofs[d] + whist[w][d] + rank[j];
+    if (rank[j] != NONE) {
+      const u32 d = (k[j] >> shift) & 0xFFu;
+      const u32 pos = tofs[d] + whist[w][d] + rank[j];
       skeys[pos] = k[j];
-      svals[pos] = vin[idx];
+      svals[pos] = v[j];
     }
   }
   __syncthreads();
   const u32 tile_n = s_kept;
   for (u32 q = t; q < tile_n; q += RS_THREADS) {
-    u32 kk = skeys[q];
-    u32 d = (kk >> shift) & 0xFFu;
-    u64 op = (u64)gstart[d] + (q - tofs[d]);
+    const u32 kk = skeys[q];
+    const u32 d = (kk >> shift) & 0xFFu;
+    const u64 op = (u64)gstart[d] + (q - tofs[d]);
     kout[op] = kk;
-    vout[op] = svals[q];
+    if (vout) vout[op] = svals[q];
   }
 }
 
@@ -174,14 +264,15 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__
 // ------------------------------------------------------------------ host side
 size_t scan_temp_bytes(u64 n);
 size_t rs_temp_bytes(u64 n) {
-  u64 tiles = (n + RS_TILE - 1) / RS_TILE;
-  return ((tiles * RS_BINS * sizeof(u32) + 255) & ~(u64)255) + scan_temp_bytes(tiles * RS_BINS) + 256;
+  const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
+  // histograms + bases + tickets, then one status array per pass
+  return RS_HDR_BYTES + (size_t)RS_MAXP * ((tiles ? tiles : 1) * RS_BINS * sizeof(u32)) + 256;
 }
 
-// Stable sort of (keys, vals) by key bits [bit_lo, bit_hi).  Result is in (keys, vals) when
-// the function returns false, else in (keys_alt, vals_alt).  n is the (upper bound of the) item
-// count; with n_dev the exact count is read on the device.  drop: the first pass removes items
-// whose key is KEY_DROP and writes the number kept to *n_out_dev (at least one pass is run).
+// Stable sort of (keys, vals) by key bits [bit_lo, bit_hi) (vals may be null: keys only).  Result is in (keys, vals) when the
+// function returns false, else in (keys_alt, vals_alt).  n is the (upper bound of the) item count;
+// with n_dev the exact count is read on the device.  drop: the first pass removes items whose key
+// is KEY_DROP and writes the number kept to *n_out_dev (at least one pass is run).
 bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi, void* temp,
                       cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop) {
   if (!drop && (n <= 1 || bit_hi <= bit_lo)) return false;
@@ -190,19 +281,28 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
     return false;
   }
   int passes = (bit_hi - bit_lo + 7) / 8;
-  if (passes > 4) passes = 4;
+  if (passes > RS_MAXP) passes = RS_MAXP;
   if (passes < 1) passes = 1;
   const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
-  u32* counts = (u32*)temp;
-  void* stemp = (char*)temp + ((tiles * RS_BINS * sizeof(u32) + 255) & ~(u64)255);
+  u32* ghist = (u32*)temp;                          // [RS_MAXP][256]
+  u32* gbase = ghist + RS_MAXP * RS_BINS;           // [RS_MAXP][256]
+  u32* tickets = gbase + RS_MAXP * RS_BINS;         // [RS_MAXP]
+  u32* status = (u32*)((char*)temp + RS_HDR_BYTES);         // [passes][tiles][256]
+  const size_t st_bytes = (size_t)tiles * RS_BINS * sizeof(u32);
+  cudaMemsetAsync(temp, 0, RS_HDR_BYTES + passes * st_bytes, st);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const unsigned hgrid = (unsigned)std::min<u64>((n + RS_THREADS * RS_HIST_ITEMS - 1) / (RS_THREADS * RS_HIST_ITEMS), (u64)sms * 8);
+  k_rs_hist<<<hgrid, RS_THREADS, 0, st>>>(keys, n, n_dev, drop ? 1 : 0, bit_lo, passes, ghist); ++g_launches;
+  k_rs_bins<<<passes, RS_BINS, 0, st>>>(ghist, gbase, drop ? n_out_dev : nullptr); ++g_launches;
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
   const u64* nd = n_dev;
   for (int p = 0; p < passes; ++p) {
     const int shift = bit_lo + 8 * p;
     const int dr = (drop && p == 0) ? 1 : 0;
-    k_rs_upsweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, tiles, counts); ++g_launches;
-    exclusive_scan_u32(counts, counts, tiles * RS_BINS, stemp, dr ? n_out_dev : nullptr, st);
-    k_rs_downsweep<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, nd, dr, shift, counts, tiles);
+    k_rs_pass<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, nd, dr, shift, gbase + p * RS_BINS,
+                                                       (u32*)((char*)status + p * st_bytes), tickets + p);
     ++g_launches;
     if (dr) nd = n_out_dev;
     u32* tk = ki; ki = ko; ko = tk;

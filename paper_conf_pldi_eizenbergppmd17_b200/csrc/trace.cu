@@ -1,6 +1,6 @@
 // trace.cu — the record-level passes of the hot path:
 //   k_header   (a1/a2) header validation, event counts, K1 partition keys, write-page marking
-//   k_replay   (a3)    K2 compressed clock replay: one thread per traced warp walks its records
+//   k_replay   (a3)    K2 compressed clock replay: one analysis warp per traced warp walks its records
 //   k_barriers (a3)    block barrier completion labels (§4.3.2 block max)
 //   k_expand   (a5)    K4 lane expansion into (granule key | op, event) items in trace order
 #include "common.cuh"
@@ -18,8 +18,9 @@ namespace bc {
 __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ recs, Geo g, u32* __restrict__ wkey,
                                                 u32* __restrict__ wval, u32* __restrict__ if_cnt,
                                                 u32* __restrict__ bar_cnt, u32* __restrict__ sync_list,
-                                                u32* __restrict__ page_bits, u64* __restrict__ cnt,
-                                                u32* __restrict__ rec_ub, u32* __restrict__ err) {
+                                                u32* __restrict__ page_bits, u32* __restrict__ word_list,
+                                                u64* __restrict__ cnt, u32* __restrict__ rec_ub,
+                                                u32* __restrict__ err) {
   const u32 lane = threadIdx.x & 31;
   const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const u64 r = gw * 32 + lane;
@@ -125,7 +126,13 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
       } else {
         u32 bit = 1u << (p & 31);
         u32* wp = &page_bits[p >> 5];
-        if (!(*(volatile u32*)wp & bit)) atomicOr(wp, bit);
+        if (!(*(volatile u32*)wp & bit)) {
+          // the thread that turns a bitmap word non-zero lists it (ranked by k_page_rank)
+          if (atomicOr(wp, bit) == 0u) {
+            const u64 at = atomicAdd((unsigned long long*)&cnt[C_PAGE_WORDS], 1ull);
+            word_list[at] = (u32)(p >> 5);
+          }
+        }
       }
     }
   }
@@ -144,136 +151,154 @@ __global__ void k_warp_start(const u32* __restrict__ skeys, u64 n, u32 n_warps, 
 }
 
 // ---------------------------------------------------------------------------- k_replay
-// K2: compressed clock replay (Fig. 7, §4.3.1-4.3.2).  One thread per traced
-// warp walks the warp's records in trace order with the SIMT stack of Fig. 2 (K_w, P:L430-432,
-// P:L591-609).  Stack levels are branch-tree nodes: IF pushes the then-node (else-node is its
-// sibling, id+1, entered at ELSE); FI pops.  Every join-fork step (endi, if, else, fi, bar) is
-// labelled rec+1.  Per record it emits the snapshot {warp, ps, node, phase}; per IF the two
-// nodes {mask, parent, popen}; per BAR its record and the warp's next record (for the barrier
-// feasibility check) and a BARRIER_DIVERGENCE finding when the mask is not the full warp
-// (P:L639-644).
-__global__ void __launch_bounds__(128) k_replay(const bc_record* __restrict__ recs, const u32* __restrict__ wrec,
+// K2: compressed clock replay (Fig. 7, §4.3.1-4.3.2).  One analysis warp per traced
+// warp walks the traced warp's records in trace order with the SIMT stack of Fig. 2 (K_w,
+// P:L430-432).  Stack levels are branch-tree nodes: IF pushes the then-node (else-node
+// is its sibling, id+1, entered at ELSE); FI pops.  Every join-fork step (endi, if, else, fi, bar)
+// is labelled rec+1.  The 32 lanes load 32 consecutive records (index + header) at once, one chunk
+// ahead, and then step through them together: the stack update is uniform (every lane computes it,
+// operands broadcast by shuffles), and lane j keeps the state record j saw, so the per-record
+// snapshot {warp, ps, node, phase} is written by 32 lanes in parallel.  Per IF it writes the two
+// nodes {mask, parent, popen}; per BAR its record and the warp's next record (barrier feasibility)
+// and a BARRIER_DIVERGENCE finding when the mask is not the warp's initial mask.
+__global__ void __launch_bounds__(256) k_replay(const bc_record* __restrict__ recs, const u32* __restrict__ wrec,
                                                 const u32* __restrict__ warp_start, Geo g,
                                                 const u32* __restrict__ node_base, const u32* __restrict__ bar_base,
                                                 uint4* __restrict__ snap, uint4* __restrict__ nodes,
                                                 u32* __restrict__ bar_rec, u32* __restrict__ bar_next,
                                                 u32* __restrict__ find_blk, u32* __restrict__ find_rec,
                                                 u32* __restrict__ find_cnt, u32* __restrict__ err) {
-  const u32 w = blockIdx.x * blockDim.x + threadIdx.x;
-  if (w >= g.n_warps) return;
+  const u32 w = (u32)(((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+  const u32 lane = threadIdx.x & 31;
+  if (w >= g.n_warps) return;  // warp-uniform
   const u32 imask = init_mask(g, w);
   u32 st_node[33], st_mask[33];
   u64 then_bits = 0;  // bit d set: level d is a then-node
   int depth = 0;
   st_node[0] = w;
   st_mask[0] = imask;
-  nodes[w] = make_uint4(imask, NONE, 0u, 0u);
+  if (lane == 0) nodes[w] = make_uint4(imask, NONE, 0u, 0u);
   u32 ps = 0, phase = 0, nif = 0, nbar = 0;
   bool need_next = false;
   bool bad = false;
   const u32 nb0 = node_base[w], bb0 = bar_base[w];
   const u32 i0 = warp_start[w], i1 = warp_start[w + 1];
-  constexpr int PF = 4;  // records whose headers are in flight together
-  u32 rq[PF];
-  uint4 hq[PF];
-#pragma unroll
-  for (int k = 0; k < PF; ++k) {
-    rq[k] = i0 + k < i1 ? wrec[i0 + k] : 0u;
-    hq[k] = i0 + k < i1 ? __ldg(reinterpret_cast<const uint4*>(recs + rq[k])) : make_uint4(0, 0, 0, 0);
+  u32 nr = 0;
+  uint4 nh = make_uint4(0, 0, 0, 0);
+  if (i0 + lane < i1) {
+    nr = wrec[i0 + lane];
+    nh = __ldg(reinterpret_cast<const uint4*>(recs + nr));
   }
-  for (u32 i = i0; i < i1 && !bad; ++i) {
-    const u32 r = rq[0];
-    const uint4 hv = hq[0];
-#pragma unroll
-    for (int k = 0; k + 1 < PF; ++k) {
-      rq[k] = rq[k + 1];
-      hq[k] = hq[k + 1];
+  for (u32 c0 = i0; c0 < i1 && !bad; c0 += 32) {
+    const u32 r = nr;
+    const uint4 hv = nh;
+    const u32 cnt = min(32u, i1 - c0);
+    if (c0 + 32 + lane < i1) {  // next chunk in flight while this one is stepped through
+      nr = wrec[c0 + 32 + lane];
+      nh = __ldg(reinterpret_cast<const uint4*>(recs + nr));
     }
-    if (i + PF < i1) {  // prefetch PF records ahead
-      rq[PF - 1] = wrec[i + PF];
-      hq[PF - 1] = __ldg(reinterpret_cast<const uint4*>(recs + rq[PF - 1]));
-    }
-    const u32 mask = hv.y, op = hv.z & 0xFFu, aux = hv.w;
-    if (need_next) {
-      bar_next[bb0 + nbar - 1] = r;
-      need_next = false;
-    }
-    snap[r] = make_uint4(w, ps, st_node[depth], phase);
-    if (mask != st_mask[depth]) {  // feasibility: record mask == K_w.peek()
-      bad = true;
-      break;
-    }
-    switch (op) {
-      case BC_OP_FENCE:
-        break;  // standalone fence: no trace operation (R14)
-      case BC_OP_IF: {
-        if (depth >= 32) { bad = true; break; }
-        u32 then = mask & aux;
-        u32 nid = nb0 + 2 * nif;
-        ++nif;
-        nodes[nid] = make_uint4(then, st_node[depth], ps, 0u);
-        nodes[nid + 1] = make_uint4(mask & ~then, st_node[depth], ps, 0u);
-        ++depth;
-        st_node[depth] = nid;
-        st_mask[depth] = then;
-        then_bits |= 1ull << depth;
-        ps = r + 1;
+    u32 my_ps = 0, my_node = 0, my_phase = 0;
+    u32 done = 0;
+    for (u32 j = 0; j < cnt; ++j) {
+      const u32 rj = __shfl_sync(0xFFFFFFFFu, r, j);
+      const u32 mask = __shfl_sync(0xFFFFFFFFu, hv.y, j);
+      const u32 op = __shfl_sync(0xFFFFFFFFu, hv.z, j) & 0xFFu;
+      const u32 aux = __shfl_sync(0xFFFFFFFFu, hv.w, j);
+      if (need_next) {
+        if (lane == 0) bar_next[bb0 + nbar - 1] = rj;
+        need_next = false;
+      }
+      if (lane == j) {
+        my_ps = ps;
+        my_node = st_node[depth];
+        my_phase = phase;
+      }
+      done = j + 1;
+      if (mask != st_mask[depth]) {  // feasibility: record mask == K_w.peek()
+        bad = true;
         break;
       }
-      case BC_OP_ELSE: {
-        if (depth == 0 || !((then_bits >> depth) & 1ull)) { bad = true; break; }
-        st_node[depth] += 1;
-        st_mask[depth] = st_mask[depth - 1] & ~st_mask[depth];
-        then_bits &= ~(1ull << depth);
-        ps = r + 1;
-        break;
-      }
-      case BC_OP_FI: {
-        if (depth == 0 || ((then_bits >> depth) & 1ull)) { bad = true; break; }
-        --depth;
-        ps = r + 1;
-        break;
-      }
-      case BC_OP_BAR: {
-        if (mask != imask) {  // barrier divergence; the barrier still completes (R10)
-          u32 at = atomicAdd(find_cnt, 1u);
-          find_blk[at] = w / g.wpb;
-          find_rec[at] = r;
+      switch (op) {
+        case BC_OP_FENCE:
+          break;  // standalone fence: no trace operation (R14)
+        case BC_OP_IF: {
+          if (depth >= 32) { bad = true; break; }
+          const u32 then = mask & aux;
+          const u32 nid = nb0 + 2 * nif;
+          ++nif;
+          if (lane == 0) {
+            nodes[nid] = make_uint4(then, st_node[depth], ps, 0u);
+            nodes[nid + 1] = make_uint4(mask & ~then, st_node[depth], ps, 0u);
+          }
+          ++depth;
+          st_node[depth] = nid;
+          st_mask[depth] = then;
+          then_bits |= 1ull << depth;
+          ps = rj + 1;
+          break;
         }
-        bar_rec[bb0 + nbar] = r;
-        bar_next[bb0 + nbar] = NONE;
-        ++nbar;
-        ++phase;
-        need_next = true;
-        ps = r + 1;
-        break;
+        case BC_OP_ELSE: {
+          if (depth == 0 || !((then_bits >> depth) & 1ull)) { bad = true; break; }
+          st_node[depth] += 1;
+          st_mask[depth] = st_mask[depth - 1] & ~st_mask[depth];
+          then_bits &= ~(1ull << depth);
+          ps = rj + 1;
+          break;
+        }
+        case BC_OP_FI: {
+          if (depth == 0 || ((then_bits >> depth) & 1ull)) { bad = true; break; }
+          --depth;
+          ps = rj + 1;
+          break;
+        }
+        case BC_OP_BAR: {
+          if (lane == 0) {
+            if (mask != imask) {  // barrier divergence; the barrier still completes (R10)
+              const u32 at = atomicAdd(find_cnt, 1u);
+              find_blk[at] = blk_of(g, w);
+              find_rec[at] = rj;
+            }
+            bar_rec[bb0 + nbar] = rj;
+            bar_next[bb0 + nbar] = NONE;
+          }
+          ++nbar;
+          ++phase;
+          need_next = true;
+          ps = rj + 1;
+          break;
+        }
+        default:  // LD/ST/ATOM and ACQ/REL/AR: the record's endi(w) step
+          ps = rj + 1;
+          break;
       }
-      default:  // LD/ST/ATOM and ACQ/REL/AR: the record's endi(w) step
-        ps = r + 1;
-        break;
+      if (bad) break;
     }
+    if (lane < done) snap[r] = make_uint4(w, my_ps, my_node, my_phase);
   }
-  if (bad) set_err(err, ERR_INFEASIBLE);
+  if (bad && lane == 0) set_err(err, ERR_INFEASIBLE);
 }
 
 // ---------------------------------------------------------------------------- k_barriers
 // Per block: every warp must arrive at every barrier exactly once (R10).  Barrier k completes
 // at the last arrival R_k = max over the block's warps of their k-th BAR record; its step is
 // labelled R_k + 1 for every thread of the block.  A warp whose next record after its k-th
-// BAR precedes R_k issued a record while waiting -> infeasible.
-__global__ void k_barriers(Geo g, const u32* __restrict__ bar_cnt, const u32* __restrict__ bar_base,
-                           const u32* __restrict__ bar_rec, const u32* __restrict__ bar_next,
-                           u32* __restrict__ blockR, u32* __restrict__ err) {
-  u32 b = blockIdx.x * blockDim.x + threadIdx.x;
-  if (b >= g.n_blocks) return;
-  u32 w0 = b * g.wpb;
-  u32 nb = bar_cnt[w0];
-  for (u32 i = 1; i < g.wpb; ++i)
-    if (bar_cnt[w0 + i] != nb) {
-      set_err(err, ERR_INFEASIBLE);
-      return;
-    }
-  for (u32 k = 0; k < nb; ++k) {
+// BAR precedes R_k issued a record while waiting -> infeasible.  One warp per traced block; lane l
+// handles barriers l, l+32, ... (warps per block <= 32, so lane i also checks warp i's count).
+__global__ void __launch_bounds__(256) k_barriers(Geo g, const u32* __restrict__ bar_cnt,
+                                                  const u32* __restrict__ bar_base, const u32* __restrict__ bar_rec,
+                                                  const u32* __restrict__ bar_next, u32* __restrict__ blockR,
+                                                  u32* __restrict__ err) {
+  const u32 b = (u32)(((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+  const u32 lane = threadIdx.x & 31;
+  if (b >= g.n_blocks) return;  // warp-uniform
+  const u32 w0 = b * g.wpb;
+  const u32 nb = bar_cnt[w0];
+  const bool diff = lane < g.wpb && bar_cnt[w0 + lane] != nb;
+  if (__any_sync(0xFFFFFFFFu, diff)) {
+    if (lane == 0) set_err(err, ERR_INFEASIBLE);
+    return;
+  }
+  for (u32 k = lane; k < nb; k += 32) {
     u32 R = 0, mn = NONE;
     for (u32 i = 0; i < g.wpb; ++i) {
       u32 bi = bar_base[w0 + i] + k;
@@ -385,19 +410,83 @@ __global__ void __launch_bounds__(256) k_expand(const bc_record* __restrict__ re
   if (__any_sync(0xFFFFFFFFu, ovf) && lane == 0) set_err(err, ERR_OVERFLOW);
 }
 
-// page_rank[i] = number of set bits in page_bits[0..i)  (exclusive popcount scan input)
-__global__ void k_popc(const u32* __restrict__ bits, u32* __restrict__ out, u64 n) {
-  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < n) out[i] = __popc(bits[i]);
+// Ranks of the written 1-MB pages in address order (the dense global key space):
+// `words` = the non-zero bitmap words; unless `presorted`, the CTA first sorts them in shared memory
+// (bitonic, up to PR_MAX words; a longer list sets *need_sort and returns, and the host sorts it with
+// the radix sort and calls again with presorted = 1).  page_rank[word] = set bits in all lower words;
+// wl_prefix[i] = page_rank[words[i]]; *n_pages_dev = written pages.  The CTA walks the list in
+// chunks of 1024 with a running carry; only listed words of page_rank are ever read.
+constexpr u32 PR_MAX = 8192;
+__global__ void __launch_bounds__(1024) k_page_rank(u32* __restrict__ words, const u64* __restrict__ n_words_dev,
+                                                    const u32* __restrict__ page_bits, u32* __restrict__ page_rank,
+                                                    u32* __restrict__ wl_prefix, u64* __restrict__ n_pages_dev,
+                                                    u32* __restrict__ need_sort, int presorted) {
+  __shared__ u32 wsum[32];
+  __shared__ u32 s_carry;
+  __shared__ u32 sw[PR_MAX];
+  const u32 t = threadIdx.x, w = t >> 5, l = t & 31;
+  const u64 nw = *n_words_dev;
+  if (!presorted) {
+    if (nw > PR_MAX) {
+      if (t == 0) *need_sort = 1u;
+      return;
+    }
+    u32 P = 1;
+    while (P < nw) P <<= 1;
+    for (u32 i = t; i < P; i += 1024) sw[i] = i < nw ? words[i] : 0xFFFFFFFFu;
+    __syncthreads();
+    for (u32 k = 2; k <= P; k <<= 1) {
+      for (u32 j = k >> 1; j > 0; j >>= 1) {
+        for (u32 i = t; i < P; i += 1024) {
+          const u32 ij = i ^ j;
+          if (ij > i) {
+            const u32 a = sw[i], b = sw[ij];
+            if (((i & k) == 0) == (a > b)) {
+              sw[i] = b;
+              sw[ij] = a;
+            }
+          }
+        }
+        __syncthreads();
+      }
+    }
+    for (u32 i = t; i < nw; i += 1024) words[i] = sw[i];
+  }
+  if (t == 0) s_carry = 0;
+  __syncthreads();
+  for (u64 c0 = 0; c0 < nw; c0 += 1024) {
+    const u64 i = c0 + t;
+    const u32 wd = i < nw ? words[i] : 0u;
+    const u32 v = i < nw ? (u32)__popc(page_bits[wd]) : 0u;
+    const u32 x = warp_incl_sum(v);
+    if (l == 31) wsum[w] = x;
+    __syncthreads();
+    u32 off = 0, tot = 0;
+    for (u32 ww = 0; ww < 32; ++ww) {
+      if (ww < w) off += wsum[ww];
+      tot += wsum[ww];
+    }
+    const u32 carry = s_carry;
+    if (i < nw) {
+      const u32 r = carry + off + x - v;
+      page_rank[wd] = r;
+      wl_prefix[i] = r;
+    }
+    __syncthreads();
+    if (t == 0) s_carry = carry + tot;
+    __syncthreads();
+  }
+  if (t == 0) *n_pages_dev = s_carry;
 }
 
 // --------------------------------------------------------------------- host launchers
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
-                   u32* sync_list, u32* page_bits, u64* cnt, u32* rec_ub, u32* err, cudaStream_t st) {
+                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, u32* err,
+                   cudaStream_t st) {
   u64 warps = (g.n_recs + 31) / 32;
   if (warps == 0) return;
   u64 blocks = (warps + 7) / 8;
-  k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, cnt,
+  k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt,
                                              rec_ub, err); ++g_launches;
 }
 
@@ -408,13 +497,13 @@ void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cu
 void launch_replay(const bc_record* recs, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
                    const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next, u32* find_blk,
                    u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st) {
-  k_replay<<<(g.n_warps + 127) / 128, 128, 0, st>>>(recs, wrec, warp_start, g, node_base, bar_base, snap, nodes,
+  k_replay<<<(unsigned)(((u64)g.n_warps * 32 + 255) / 256), 256, 0, st>>>(recs, wrec, warp_start, g, node_base, bar_base, snap, nodes,
                                                      bar_rec, bar_next, find_blk, find_rec, find_cnt, err); ++g_launches;
 }
 
 void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, const u32* bar_rec, const u32* bar_next,
                      u32* blockR, u32* err, cudaStream_t st) {
-  k_barriers<<<(g.n_blocks + 127) / 128, 128, 0, st>>>(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err); ++g_launches;
+  k_barriers<<<(unsigned)(((u64)g.n_blocks * 32 + 255) / 256), 256, 0, st>>>(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err); ++g_launches;
 }
 
 // snapshot .w: barrier phase -> label of the block's last completed barrier (0 = none)
@@ -438,8 +527,11 @@ void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, cons
   ++g_launches;
 }
 
-void launch_popc(const u32* bits, u32* out, u64 n, cudaStream_t st) {
-  k_popc<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(bits, out, n); ++g_launches;
+void launch_page_rank(u32* words, const u64* n_words_dev, const u32* page_bits, u32* page_rank, u32* wl_prefix,
+                      u64* n_pages_dev, u32* need_sort, int presorted, cudaStream_t st) {
+  k_page_rank<<<1, 1024, 0, st>>>(words, n_words_dev, page_bits, page_rank, wl_prefix, n_pages_dev, need_sort,
+                                  presorted);
+  ++g_launches;
 }
 
 __global__ void k_node_base(const u32* __restrict__ if_excl, u32 n_warps, u32* __restrict__ node_base) {
