@@ -1,5 +1,5 @@
-// sort.cu — hand-written stable LSD radix sort (onesweep: one histogram pass, then one kernel per
-// 8-bit digit with decoupled look-back) and a device-wide exclusive scan, for sm_100a.
+// sort.cu — hand-written stable LSD radix sort (8-bit digits, reduce-then-scan per pass) and a
+// device-wide exclusive scan, for sm_100a.
 //
 // The radix sort is the paper's per-location serialisation (a spinlock per shadow
 // entry orders the host threads' accesses) turned into data parallelism: a STABLE sort of
@@ -7,10 +7,12 @@
 // segment that is still in trace order.
 //   k_rs_hist  : one read of the keys -> the global 256-bin histogram of every digit pass
 //   k_rs_bins  : exclusive scan of each pass's histogram (digit start offsets); kept-item count
-//   k_rs_pass  : per 4096-key tile (taken in launch order from an atomic ticket): stable in-tile
-//                rank (warp match + per-warp histograms), per-digit decoupled look-back over the
-//                preceding tiles, scatter through shared memory so that each digit's run is
-//                written contiguously.  Reads 8 B and writes 8 B per item: the pass roofline.
+//   k_rs_up    : per 4096-key tile, the digit counts (reads 4 B / item)
+//   k_rs_rows  : one CTA per digit scans that digit's counts over all tiles (256 independent rows:
+//                no serial chain across tiles, unlike a decoupled look-back whose first wave of
+//                ~450 co-resident tiles walks back one L2 round trip per step)
+//   k_rs_down  : per tile: stable in-tile rank (ballot match + per-warp histograms), scatter through
+//                shared memory so that each digit's run is written contiguously (8 B in, 8 B out).
 #include <algorithm>
 
 #include "common.cuh"
@@ -26,11 +28,8 @@ constexpr int RS_TILE = RS_THREADS * RS_ITEMS;  // 4096
 constexpr int RS_WARPS = RS_THREADS / 32;
 constexpr int RS_BINS = 256;
 constexpr int RS_MAXP = 4;
-// temp header: ghist[RS_MAXP][256], gbase[RS_MAXP][256], tickets[RS_MAXP]; status arrays follow
+// temp header: ghist[RS_MAXP][256], gbase[RS_MAXP][256]; the (digit, tile) table follows
 constexpr size_t RS_HDR_BYTES = (2 * RS_MAXP * 256 + 64) * sizeof(u32);
-// look-back status word per (tile, digit): [31:30] flag, [29:0] count (items < 2^30 per sort)
-constexpr u32 ST_AGG = 1u << 30, ST_INC = 2u << 30, ST_VAL = (1u << 30) - 1u;
-constexpr int RS_LB = 8;  // predecessors inspected per look-back step
 
 // Lanes of the warp holding the same 9-bit label (digit, or 256 = no item): 9 ballots, a fixed
 // cost independent of how many distinct digits the warp holds.
@@ -110,46 +109,134 @@ __global__ void __launch_bounds__(RS_BINS) k_rs_bins(const u32* __restrict__ ghi
   if (p == 0 && t == 0 && n_out) *n_out = tot;
 }
 
-__global__ void __launch_bounds__(RS_THREADS, 2) k_rs_pass(const u32* __restrict__ kin, const u32* __restrict__ vin,
+// Upsweep of one pass: the digit counts of every tile, digit-major (counts[d * tiles + tile]);
+// tiles past the (device-side) item count write zeros.
+__global__ void __launch_bounds__(RS_THREADS) k_rs_up(const u32* __restrict__ kin, u64 n_max,
+                                                      const u64* __restrict__ n_dev, int drop, int shift,
+                                                      u32* __restrict__ counts, u64 tiles) {
+  __shared__ u32 h[RS_BINS];
+  const int t = threadIdx.x;
+  h[t] = 0;
+  __syncthreads();
+  const u64 n = n_dev ? *n_dev : n_max;
+  const u64 base = (u64)blockIdx.x * RS_TILE;
+  const u32 lt = lanemask_lt();
+  if (base < n) {
+    u32 k[RS_ITEMS];
+#pragma unroll
+    for (int j = 0; j < RS_ITEMS; ++j) {
+      const u64 idx = base + (u64)j * RS_THREADS + t;
+      k[j] = idx < n ? kin[idx] : KEY_DROP;
+    }
+#pragma unroll
+    for (int j = 0; j < RS_ITEMS; ++j) {
+      const u64 idx = base + (u64)j * RS_THREADS + t;
+      const bool ok = idx < n && !(drop && k[j] == KEY_DROP);
+      const u32 d = ok ? (k[j] >> shift) & 0xFFu : 0x100u;
+      const u32 vm = __ballot_sync(0xFFFFFFFFu, ok);
+      const u32 d0 = __shfl_sync(0xFFFFFFFFu, d, vm ? __ffs(vm) - 1 : 0);
+      if (__all_sync(0xFFFFFFFFu, !ok || d == d0)) {
+        if (vm && (lt & vm) == 0 && ok) atomicAdd(&h[d], (u32)__popc(vm));
+      } else if (ok) {
+        atomicAdd(&h[d], 1u);
+      }
+    }
+  }
+  __syncthreads();
+  counts[(u64)t * tiles + blockIdx.x] = h[t];
+}
+
+// One CTA per digit d: offs[d * tiles + tile] = gbase[d] + (items of digit d in tiles < tile).
+// The 256 rows are independent, so there is no serial chain across tiles.
+__global__ void __launch_bounds__(RS_THREADS) k_rs_rows(u32* __restrict__ counts, u64 tiles,
+                                                        const u32* __restrict__ gbase) {
+  __shared__ u32 wsum[RS_WARPS];
+  __shared__ u32 s_carry;
+  const int t = threadIdx.x, w = t >> 5, l = t & 31, d = blockIdx.x;
+  u32* row = counts + (u64)d * tiles;
+  if (t == 0) s_carry = gbase[d];
+  __syncthreads();
+  constexpr int PER = 8;
+  for (u64 c0 = 0; c0 < tiles; c0 += RS_THREADS * PER) {
+    u32 v[PER], sum = 0;
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const u64 i = c0 + (u64)t * PER + q;
+      v[q] = i < tiles ? row[i] : 0u;
+      sum += v[q];
+    }
+    const u32 x = warp_incl_sum(sum);
+    if (l == 31) wsum[w] = x;
+    __syncthreads();
+    u32 off = 0, tot = 0;
+    for (int ww = 0; ww < RS_WARPS; ++ww) {
+      if (ww < w) off += wsum[ww];
+      tot += wsum[ww];
+    }
+    u32 run = s_carry + off + x - sum;
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const u64 i = c0 + (u64)t * PER + q;
+      if (i < tiles) row[i] = run;
+      run += v[q];
+    }
+    __syncthreads();
+    if (t == 0) s_carry += tot;
+    __syncthreads();
+  }
+}
+
+// Downsweep of one pass (stable in-tile rank, scatter through shared memory so that each digit's
+// run is written contiguously).  Register diet for occupancy (3 CTAs / SM): keys are staged in
+// shared memory in input order while they are ranked, each item keeps only (digit << 16 | rank),
+// and values are loaded after ranking.
+__global__ void __launch_bounds__(RS_THREADS, 3) k_rs_down(const u32* __restrict__ kin, const u32* __restrict__ vin,
                                                            u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
                                                            const u64* __restrict__ n_dev, int drop, int shift,
-                                                           const u32* __restrict__ gbase, u32* __restrict__ status,
-                                                           u32* __restrict__ ticket) {
+                                                           const u32* __restrict__ offs, u64 tiles) {
+  __shared__ u32 kst[RS_TILE];
   __shared__ u32 skeys[RS_TILE];
-  __shared__ u32 svals[RS_TILE];
   __shared__ u32 whist[RS_WARPS][RS_BINS];
   __shared__ u32 tofs[RS_BINS];
   __shared__ u32 gstart[RS_BINS];
   __shared__ u32 wsum[RS_WARPS];
-  __shared__ u32 s_tile, s_kept;
+  __shared__ u32 s_kept;
 
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
-  if (t == 0) s_tile = atomicAdd(ticket, 1u);
   for (int i = t; i < RS_WARPS * RS_BINS; i += RS_THREADS) (&whist[0][0])[i] = 0;
   __syncthreads();
-  const u32 tile = s_tile;
+  const u32 tile = blockIdx.x;
   const u64 n = n_dev ? *n_dev : n_max;
   const u64 base = (u64)tile * RS_TILE;
-  if (base >= n) return;  // every later ticket is past the end too: nobody looks back at it
+  if (base >= n) return;
 
-  u32 k[RS_ITEMS], v[RS_ITEMS], rank[RS_ITEMS];
+  u32 rank[RS_ITEMS];  // (digit << 16) | rank in the warp's digit run, NONE = no item
+  {
+    u32 k[RS_ITEMS];
 #pragma unroll
-  for (int j = 0; j < RS_ITEMS; ++j) {
-    const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-    k[j] = idx < n ? kin[idx] : KEY_DROP;
-    v[j] = (vin && idx < n) ? vin[idx] : 0u;
+    for (int j = 0; j < RS_ITEMS; ++j) {
+      const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
+      k[j] = idx < n ? kin[idx] : KEY_DROP;
+    }
+    const u32 lt = lanemask_lt();
+#pragma unroll
+    for (int j = 0; j < RS_ITEMS; ++j) {
+      const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
+      const u32 d = (idx < n && !(drop && k[j] == KEY_DROP)) ? ((k[j] >> shift) & 0xFFu) : 256u;
+      const u32 peers = match9(d);
+      const u32 old = d < 256u ? whist[w][d] : 0u;
+      __syncwarp();
+      if (d < 256u && (peers & lt) == 0) whist[w][d] = old + __popc(peers);
+      __syncwarp();
+      rank[j] = d < 256u ? ((d << 16) | (old + __popc(peers & lt))) : NONE;
+      kst[w * (RS_ITEMS * 32) + j * 32 + l] = k[j];
+    }
   }
-  const u32 lt = lanemask_lt();
+  u32 v[RS_ITEMS];
 #pragma unroll
   for (int j = 0; j < RS_ITEMS; ++j) {
     const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-    const u32 d = (idx < n && !(drop && k[j] == KEY_DROP)) ? ((k[j] >> shift) & 0xFFu) : 256u;
-    const u32 peers = match9(d);
-    const u32 old = d < 256u ? whist[w][d] : 0u;
-    __syncwarp();
-    if (d < 256u && (peers & lt) == 0) whist[w][d] = old + __popc(peers);
-    __syncwarp();
-    rank[j] = d < 256u ? old + __popc(peers & lt) : NONE;
+    v[j] = (vin && rank[j] != NONE) ? vin[idx] : 0u;
   }
   __syncthreads();
   // per digit (thread t): prefix over warps, tile total
@@ -160,31 +247,7 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_pass(const u32* __restrict
     whist[ww][t] = total;
     total += c;
   }
-  // publish the tile aggregate, then look back for the exclusive prefix of this digit
-  volatile u32* vs = status;
-  u32 excl = 0;
-  if (tile == 0) {
-    vs[t] = ST_INC | total;
-  } else {
-    vs[(u64)tile * RS_BINS + t] = ST_AGG | total;
-    // walk back RS_LB predecessors per step with all their loads in flight (the first wave of
-    // co-resident tiles would otherwise walk up to ~300 tiles one L2 round trip at a time)
-    bool done = false;
-    for (u64 pt = tile; !done; pt = pt > RS_LB ? pt - RS_LB : 0) {
-      u32 s[RS_LB];
-#pragma unroll
-      for (int q = 0; q < RS_LB; ++q) s[q] = pt > (u64)q ? vs[(pt - 1 - q) * RS_BINS + t] : (u32)(2u << 30);
-#pragma unroll
-      for (int q = 0; q < RS_LB; ++q) {
-        if (done) break;
-        while ((s[q] & ~ST_VAL) == 0) s[q] = vs[(pt - 1 - q) * RS_BINS + t];
-        excl += s[q] & ST_VAL;
-        if (s[q] & ST_INC) done = true;
-      }
-    }
-    vs[(u64)tile * RS_BINS + t] = ST_INC | (excl + total);
-  }
-  gstart[t] = gbase[t] + excl;
+  gstart[t] = offs[(u64)t * tiles + tile];
   // tile-local exclusive scan of the digit totals
   {
     const u32 x = warp_incl_sum(total);
@@ -196,13 +259,13 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_pass(const u32* __restrict
     if (t == RS_BINS - 1) s_kept = off + x;
   }
   __syncthreads();
+  // keys: scatter into digit order, then write each digit run contiguously
 #pragma unroll
   for (int j = 0; j < RS_ITEMS; ++j) {
     if (rank[j] != NONE) {
-      const u32 d = (k[j] >> shift) & 0xFFu;
-      const u32 pos = tofs[d] + whist[w][d] + rank[j];
-      skeys[pos] = k[j];
-      svals[pos] = v[j];
+      const u32 d = rank[j] >> 16;
+      const u32 pos = tofs[d] + whist[w][d] + (rank[j] & 0xFFFFu);
+      skeys[pos] = kst[w * (RS_ITEMS * 32) + j * 32 + l];
     }
   }
   __syncthreads();
@@ -210,25 +273,80 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_pass(const u32* __restrict
   for (u32 q = t; q < tile_n; q += RS_THREADS) {
     const u32 kk = skeys[q];
     const u32 d = (kk >> shift) & 0xFFu;
-    const u64 op = (u64)gstart[d] + (q - tofs[d]);
-    kout[op] = kk;
-    if (vout) vout[op] = svals[q];
+    kout[(u64)gstart[d] + (q - tofs[d])] = kk;
+  }
+  if (!vout) return;
+  // values: the same permutation, staged in the (now free) input-order key buffer
+  u32* svals = kst;
+#pragma unroll
+  for (int j = 0; j < RS_ITEMS; ++j) {
+    if (rank[j] != NONE) {
+      const u32 d = rank[j] >> 16;
+      svals[tofs[d] + whist[w][d] + (rank[j] & 0xFFFFu)] = v[j];
+    }
+  }
+  __syncthreads();
+  for (u32 q = t; q < tile_n; q += RS_THREADS) {
+    const u32 d = (skeys[q] >> shift) & 0xFFu;
+    vout[(u64)gstart[d] + (q - tofs[d])] = svals[q];
   }
 }
 
 // ---------------------------------------------------------------------- scan
 constexpr int SC_THREADS = 256, SC_ITEMS = 8, SC_TILE = SC_THREADS * SC_ITEMS;
 
-__global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__ in, u32* __restrict__ out, u64 n,
-                                                         u64* status, u32* tile_counter, u64* total_out) {
-  __shared__ u32 s_tile;
+// reduce-then-scan: per-tile sums, one CTA scans the tile sums, then every tile scans itself
+__global__ void __launch_bounds__(SC_THREADS) k_scan_tsum(const u32* __restrict__ in, u64 n, u64* __restrict__ tsum) {
   __shared__ u64 wsum[SC_THREADS / 32];
-  __shared__ u64 s_excl;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
-  if (t == 0) s_tile = atomicAdd(tile_counter, 1u);
+  const u64 base = (u64)blockIdx.x * SC_TILE;
+  u64 sum = 0;
+#pragma unroll
+  for (int j = 0; j < SC_ITEMS; ++j) {
+    const u64 i = base + (u64)j * SC_THREADS + t;
+    sum += i < n ? in[i] : 0u;
+  }
+  const u64 x = warp_incl_sum(sum);
+  if (l == 31) wsum[w] = x;
   __syncthreads();
-  const u32 tile = s_tile;
-  const u64 base = (u64)tile * SC_TILE + (u64)t * SC_ITEMS;
+  if (t == 0) {
+    u64 tot = 0;
+    for (int ww = 0; ww < SC_THREADS / 32; ++ww) tot += wsum[ww];
+    tsum[blockIdx.x] = tot;
+  }
+}
+
+__global__ void __launch_bounds__(1024) k_scan_tiles(u64* __restrict__ tsum, u64 tiles, u64* __restrict__ total_out) {
+  __shared__ u64 wsum[32];
+  __shared__ u64 s_carry;
+  const int t = threadIdx.x, w = t >> 5, l = t & 31;
+  if (t == 0) s_carry = 0;
+  __syncthreads();
+  for (u64 c0 = 0; c0 < tiles; c0 += 1024) {
+    const u64 i = c0 + t;
+    const u64 v = i < tiles ? tsum[i] : 0ull;
+    const u64 x = warp_incl_sum(v);
+    if (l == 31) wsum[w] = x;
+    __syncthreads();
+    u64 off = 0, tot = 0;
+    for (int ww = 0; ww < 32; ++ww) {
+      if (ww < w) off += wsum[ww];
+      tot += wsum[ww];
+    }
+    const u64 carry = s_carry;
+    if (i < tiles) tsum[i] = carry + off + x - v;
+    __syncthreads();
+    if (t == 0) s_carry = carry + tot;
+    __syncthreads();
+  }
+  if (t == 0 && total_out) *total_out = s_carry;
+}
+
+__global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__ in, u32* __restrict__ out, u64 n,
+                                                         const u64* __restrict__ texcl) {
+  __shared__ u64 wsum[SC_THREADS / 32];
+  const int t = threadIdx.x, w = t >> 5, l = t & 31;
+  const u64 base = (u64)blockIdx.x * SC_TILE + (u64)t * SC_ITEMS;
   u32 v[SC_ITEMS];
   u64 sum = 0;
 #pragma unroll
@@ -236,27 +354,17 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__
     v[j] = base + j < n ? in[base + j] : 0u;
     sum += v[j];
   }
-  u64 x = warp_incl_sum(sum);
+  const u64 x = warp_incl_sum(sum);
   if (l == 31) wsum[w] = x;
   __syncthreads();
-  u64 off = 0, agg = 0;
-  for (int ww = 0; ww < SC_THREADS / 32; ++ww) {
-    if (ww < w) off += wsum[ww];
-    agg += wsum[ww];
-  }
-  if (w == 0) {
-    u64 e = lookback_u64_warp(status, tile, agg, l);
-    if (l == 0) s_excl = e;
-  }
-  __syncthreads();
-  u64 run = s_excl + off + x - sum;
+  u64 off = 0;
+  for (int ww = 0; ww < w; ++ww) off += wsum[ww];
+  u64 run = texcl[blockIdx.x] + off + x - sum;
 #pragma unroll
   for (int j = 0; j < SC_ITEMS; ++j) {
     if (base + j < n) out[base + j] = (u32)run;
     run += v[j];
   }
-  if (total_out && base < n && base + SC_ITEMS >= n) *total_out = run;
-  if (total_out && n == 0 && tile == 0 && t == 0) *total_out = 0;
 }
 
 }  // namespace
@@ -265,14 +373,16 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__
 size_t scan_temp_bytes(u64 n);
 size_t rs_temp_bytes(u64 n) {
   const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
-  // histograms + bases + tickets, then one status array per pass
-  return RS_HDR_BYTES + (size_t)RS_MAXP * ((tiles ? tiles : 1) * RS_BINS * sizeof(u32)) + 256;
+  // histograms + bases, then the (digit, tile) count / offset table of one pass
+  return RS_HDR_BYTES + (size_t)(tiles ? tiles : 1) * RS_BINS * sizeof(u32) + 256;
 }
 
-// Stable sort of (keys, vals) by key bits [bit_lo, bit_hi) (vals may be null: keys only).  Result is in (keys, vals) when the
-// function returns false, else in (keys_alt, vals_alt).  n is the (upper bound of the) item count;
-// with n_dev the exact count is read on the device.  drop: the first pass removes items whose key
-// is KEY_DROP and writes the number kept to *n_out_dev (at least one pass is run).
+// Stable sort of (keys, vals) by key bits [bit_lo, bit_hi) (vals may be null: keys only).  Result is
+// in (keys, vals) when the function returns false, else in (keys_alt, vals_alt).  n is the (upper
+// bound of the) item count; with n_dev the exact count is read on the device.  drop: the first pass
+// removes items whose key is KEY_DROP and writes the number kept to *n_out_dev (at least one pass
+// is run).  Per pass: k_rs_up (digit counts per tile) -> k_rs_rows (256 independent row scans) ->
+// k_rs_down (rank + scatter); one k_rs_hist read up front gives every pass's digit bases.
 bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi, void* temp,
                       cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop) {
   if (!drop && (n <= 1 || bit_hi <= bit_lo)) return false;
@@ -284,16 +394,15 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   if (passes > RS_MAXP) passes = RS_MAXP;
   if (passes < 1) passes = 1;
   const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
-  u32* ghist = (u32*)temp;                          // [RS_MAXP][256]
-  u32* gbase = ghist + RS_MAXP * RS_BINS;           // [RS_MAXP][256]
-  u32* tickets = gbase + RS_MAXP * RS_BINS;         // [RS_MAXP]
-  u32* status = (u32*)((char*)temp + RS_HDR_BYTES);         // [passes][tiles][256]
-  const size_t st_bytes = (size_t)tiles * RS_BINS * sizeof(u32);
-  cudaMemsetAsync(temp, 0, RS_HDR_BYTES + passes * st_bytes, st);
+  u32* ghist = (u32*)temp;                           // [RS_MAXP][256]
+  u32* gbase = ghist + RS_MAXP * RS_BINS;            // [RS_MAXP][256]
+  u32* counts = (u32*)((char*)temp + RS_HDR_BYTES);  // [256][tiles]
+  cudaMemsetAsync(ghist, 0, RS_MAXP * RS_BINS * sizeof(u32), st);
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const unsigned hgrid = (unsigned)std::min<u64>((n + RS_THREADS * RS_HIST_ITEMS - 1) / (RS_THREADS * RS_HIST_ITEMS), (u64)sms * 8);
+  const unsigned hgrid =
+      (unsigned)std::min<u64>((n + RS_THREADS * RS_HIST_ITEMS - 1) / (RS_THREADS * RS_HIST_ITEMS), (u64)sms * 8);
   k_rs_hist<<<hgrid, RS_THREADS, 0, st>>>(keys, n, n_dev, drop ? 1 : 0, bit_lo, passes, ghist); ++g_launches;
   k_rs_bins<<<passes, RS_BINS, 0, st>>>(ghist, gbase, drop ? n_out_dev : nullptr); ++g_launches;
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
@@ -301,8 +410,9 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   for (int p = 0; p < passes; ++p) {
     const int shift = bit_lo + 8 * p;
     const int dr = (drop && p == 0) ? 1 : 0;
-    k_rs_pass<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, nd, dr, shift, gbase + p * RS_BINS,
-                                                       (u32*)((char*)status + p * st_bytes), tickets + p);
+    k_rs_up<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles); ++g_launches;
+    k_rs_rows<<<RS_BINS, RS_THREADS, 0, st>>>(counts, tiles, gbase + p * RS_BINS); ++g_launches;
+    k_rs_down<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, nd, dr, shift, counts, tiles);
     ++g_launches;
     if (dr) nd = n_out_dev;
     u32* tk = ki; ki = ko; ko = tk;
@@ -311,16 +421,19 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   return (passes & 1) != 0;
 }
 
-size_t scan_temp_bytes(u64 n) { return 64 + ((n + SC_TILE - 1) / SC_TILE + 1) * sizeof(u64) + 64; }
+size_t scan_temp_bytes(u64 n) { return ((n + SC_TILE - 1) / SC_TILE + 1) * sizeof(u64) + 64; }
 
 // exclusive scan in -> out (out may alias in); total written to *total_dev if non-null
 void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_dev, cudaStream_t st) {
-  u64 tiles = (n + SC_TILE - 1) / SC_TILE;
-  if (tiles == 0) tiles = 1;
-  u32* counter = (u32*)temp;
-  u64* status = (u64*)((char*)temp + 64);
-  cudaMemsetAsync(temp, 0, 64 + tiles * sizeof(u64), st);
-  k_scan_u32<<<(unsigned)tiles, SC_THREADS, 0, st>>>(in, out, n, status, counter, total_dev); ++g_launches;
+  const u64 tiles = (n + SC_TILE - 1) / SC_TILE;
+  u64* tsum = (u64*)temp;
+  if (tiles == 0) {
+    if (total_dev) cudaMemsetAsync(total_dev, 0, 8, st);
+    return;
+  }
+  k_scan_tsum<<<(unsigned)tiles, SC_THREADS, 0, st>>>(in, n, tsum); ++g_launches;
+  k_scan_tiles<<<1, 1024, 0, st>>>(tsum, tiles, total_dev); ++g_launches;
+  k_scan_u32<<<(unsigned)tiles, SC_THREADS, 0, st>>>(in, out, n, tsum); ++g_launches;
 }
 
 }  // namespace bc

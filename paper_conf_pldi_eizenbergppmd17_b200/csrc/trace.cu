@@ -3,6 +3,8 @@
 //   k_replay   (a3)    K2 compressed clock replay: one analysis warp per traced warp walks its records
 //   k_barriers (a3)    block barrier completion labels (§4.3.2 block max)
 //   k_expand   (a5)    K4 lane expansion into (granule key | op, event) items in trace order
+#include <algorithm>
+
 #include "common.cuh"
 #include "kernels.cuh"
 
@@ -321,89 +323,121 @@ __global__ void __launch_bounds__(256) k_barriers(Geo g, const u32* __restrict__
 // granules (block, offset).  Accesses to never-written global pages cannot take
 // part in a race (every race needs a write): their slots get the sentinel key
 // KEY_DROP, which the first radix pass removes.  Also validates per-lane alignment / shared
-// bounds for every op <= AR_GLB.  One warp per EXP_RPW consecutive records; loads issued in three
-// waves (headers, address rows, page-table words) so each warp has them all in flight.
-constexpr int EXP_RPW = 8;
+// bounds for every op <= AR_GLB.
+//
+// Data movement (the trace is read once, at HBM rate): persistent CTAs stream chunks of EX_REC
+// consecutive records (EX_REC x 272 B, contiguous) into shared memory with 1-D TMA bulk copies
+// (cp.async.bulk ... mbarrier::complete_tx), EX_STAGES chunks in flight per CTA; the 8 warps then
+// expand the staged records (warp w: records w*EX_RPW ...; header = a broadcast shared-memory read,
+// lane l's address = addr[l]) while the next chunks land.
+constexpr int EX_REC = 32;
+constexpr int EX_STAGES = 4;
+constexpr int EX_THREADS = 256;
+constexpr int EX_RPW = EX_REC / (EX_THREADS / 32);  // records per warp per chunk
 
-__global__ void __launch_bounds__(256) k_expand(const bc_record* __restrict__ recs, Geo g,
-                                                const u32* __restrict__ page_bits,
-                                                const u32* __restrict__ page_rank, u32 shared_base,
-                                                const u32* __restrict__ ub_off, u32* __restrict__ okeys,
-                                                u32* __restrict__ oevs, u32* __restrict__ err) {
-  const int lane = threadIdx.x & 31;
-  const u64 r0 = (((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * EXP_RPW;
-  if (r0 >= g.n_recs) return;
-  // wave 1: headers and slot offsets (lane j < EXP_RPW holds record r0 + j)
-  uint4 hv = make_uint4(0, 0, 0xFFu, 0);  // op 0xFF: past the end
-  u32 uo = 0;
-  if (lane < EXP_RPW && r0 + lane < g.n_recs) {
-    hv = __ldg(reinterpret_cast<const uint4*>(recs + r0 + lane));
-    uo = __ldg(ub_off + r0 + lane);
+__device__ __forceinline__ u32 smem_u32(const void* p) { return (u32)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(u64* bar, u32 count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(u64* bar, u32 bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, u32 bytes, u64* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(u64* bar, u32 phase) {
+  u32 done = 0;
+  while (!done) {
+    asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+                 : "=r"(done) : "r"(smem_u32(bar)), "r"(phase) : "memory");
   }
-  u32 hwarp[EXP_RPW], hmask[EXP_RPW], hz[EXP_RPW];
-#pragma unroll
-  for (int j = 0; j < EXP_RPW; ++j) {
-    hwarp[j] = __shfl_sync(0xFFFFFFFFu, hv.x, j);
-    hmask[j] = __shfl_sync(0xFFFFFFFFu, hv.y, j);
-    hz[j] = __shfl_sync(0xFFFFFFFFu, hv.z, j);
+}
+
+__global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restrict__ recs, Geo g,
+                                                       const u32* __restrict__ page_bits,
+                                                       const u32* __restrict__ page_rank, u32 shared_base,
+                                                       const u32* __restrict__ ub_off, u32* __restrict__ okeys,
+                                                       u32* __restrict__ oevs, u32* __restrict__ err) {
+  extern __shared__ __align__(128) unsigned char ex_smem[];
+  bc_record* buf = reinterpret_cast<bc_record*>(ex_smem);                    // [EX_STAGES][EX_REC]
+  u64* bar = reinterpret_cast<u64*>(ex_smem + sizeof(bc_record) * EX_REC * EX_STAGES);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const u64 n = g.n_recs;
+  const u64 n_chunks = (n + EX_REC - 1) / EX_REC;
+  auto issue = [&](u64 chunk, int st) {
+    const u64 r0 = chunk * EX_REC;
+    const u32 cnt = (u32)(n - r0 < (u64)EX_REC ? n - r0 : (u64)EX_REC);
+    mbar_expect_tx(&bar[st], cnt * (u32)sizeof(bc_record));
+    bulk_g2s(&buf[st * EX_REC], recs + r0, cnt * (u32)sizeof(bc_record), &bar[st]);
+  };
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < EX_STAGES; ++s) mbar_init(&bar[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  // wave 2: address rows of memory / sync records
-  u64 a[EXP_RPW];
-#pragma unroll
-  for (int j = 0; j < EXP_RPW; ++j) {
-    const u32 op = hz[j] & 0xFFu;
-    a[j] = 0;
-    if (op <= BC_OP_AR_GLB && ((hmask[j] >> lane) & 1u)) a[j] = __ldg(&recs[r0 + j].addr[lane]);
-  }
-  // wave 3: page-table words of global memory accesses
-  u32 pw[EXP_RPW], pr[EXP_RPW];
-#pragma unroll
-  for (int j = 0; j < EXP_RPW; ++j) {
-    const u32 op = hz[j] & 0xFFu, space = (hz[j] >> 8) & 0xFFu;
-    pw[j] = 0;
-    pr[j] = 0;
-    const u64 p = a[j] >> 20;
-    if (op <= BC_OP_ATOM && space == BC_SPACE_GLOBAL && ((hmask[j] >> lane) & 1u) && p < (1ull << 28)) {
-      pw[j] = __ldg(&page_bits[p >> 5]);
-      pr[j] = __ldg(&page_rank[p >> 5]);
+  __syncthreads();
+  if (threadIdx.x == 0)
+    for (int s = 0; s < EX_STAGES; ++s) {
+      const u64 c = blockIdx.x + (u64)s * gridDim.x;
+      if (c < n_chunks) issue(c, s);
     }
-  }
   const u32 lt = lanemask_lt();
   bool bad = false, ovf = false;
+  u32 it = 0;
+  for (u64 c = blockIdx.x; c < n_chunks; c += gridDim.x, ++it) {
+    const int st = (int)(it % EX_STAGES);
+    const u32 phase = (it / EX_STAGES) & 1u;
+    const u64 rbase = c * EX_REC + (u64)wid * EX_RPW;
+    // slot offsets of this warp's records (independent of the staged bytes: load before waiting)
+    u32 uo[EX_RPW];
 #pragma unroll
-  for (int j = 0; j < EXP_RPW; ++j) {
-    const u32 op = hz[j] & 0xFFu, space = (hz[j] >> 8) & 0xFFu, sl = (hz[j] >> 16) & 0xFFu, fl = (hz[j] >> 24) & 0xFFu;
-    const u32 uoj = __shfl_sync(0xFFFFFFFFu, uo, j);
-    if (op <= BC_OP_AR_GLB && ((hmask[j] >> lane) & 1u) && sl <= 4 && space <= 1 && hwarp[j] < g.n_warps) {
+    for (int j = 0; j < EX_RPW; ++j) uo[j] = rbase + j < n ? __ldg(ub_off + rbase + j) : 0u;
+    mbar_wait(&bar[st], phase);
+    const bc_record* sr = &buf[st * EX_REC + wid * EX_RPW];
+#pragma unroll
+    for (int j = 0; j < EX_RPW; ++j) {
+      const u64 r = rbase + j;
+      if (r >= n) break;
+      const uint4 hv = *reinterpret_cast<const uint4*>(&sr[j]);
+      const u32 hwarp = hv.x, hmask = hv.y, op = hv.z & 0xFFu, space = (hv.z >> 8) & 0xFFu,
+                sl = (hv.z >> 16) & 0xFFu, fl = (hv.z >> 24) & 0xFFu;
+      if (!(op <= BC_OP_AR_GLB && ((hmask >> lane) & 1u) && sl <= 4 && space <= 1 && hwarp < g.n_warps)) continue;
+      const u64 a = sr[j].addr[lane];
       const u64 size = 1ull << sl;
-      if (a[j] & (size - 1)) bad = true;  // natural alignment
-      if (space == BC_SPACE_SHARED && a[j] + size > g.smem) bad = true;
-      if (op <= BC_OP_ATOM) {
-        u32 n = (u32)(size >> g.G);
-        if (n == 0) n = 1;
-        const u32 opc = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM
-                                                                 : ((fl & BC_REC_SAME_VALUE) ? IOP_ST_SV : IOP_ST);
-        u32 key0 = KEY_DROP;
-        if (bad) {
-        } else if (space == BC_SPACE_SHARED) {
-          key0 = shared_base + (hwarp[j] / g.wpb) * g.smem_gran + (u32)(a[j] >> g.G);
+      if (a & (size - 1)) bad = true;  // natural alignment
+      if (space == BC_SPACE_SHARED && a + size > g.smem) bad = true;
+      if (op > BC_OP_ATOM) continue;
+      u32 nk = (u32)(size >> g.G);
+      if (nk == 0) nk = 1;
+      const u32 opc = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM
+                                                               : ((fl & BC_REC_SAME_VALUE) ? IOP_ST_SV : IOP_ST);
+      u32 key0 = KEY_DROP;
+      if (bad) {
+      } else if (space == BC_SPACE_SHARED) {
+        key0 = shared_base + blk_of(g, hwarp) * g.smem_gran + (u32)(a >> g.G);
+      } else {
+        const u64 p = a >> 20;
+        if (p < (1ull << 28)) {
+          const u32 pw = __ldg(&page_bits[p >> 5]);
+          const u32 bit = (u32)(p & 31);
+          if ((pw >> bit) & 1u)
+            key0 = (__ldg(&page_rank[p >> 5]) + __popc(pw & ((1u << bit) - 1u))) << (20 - g.G) |
+                   (u32)((a & 0xFFFFFull) >> g.G);
         } else {
-          const u64 p = a[j] >> 20;
-          if (p < (1ull << 28)) {
-            const u32 bit = (u32)(p & 31);
-            if ((pw[j] >> bit) & 1u)
-              key0 = (pr[j] + __popc(pw[j] & ((1u << bit) - 1u))) << (20 - g.G) | (u32)((a[j] & 0xFFFFFull) >> g.G);
-          } else {
-            ovf = true;
-          }
-        }
-        const u64 o = (u64)uoj + (u64)__popc(hmask[j] & lt) * n;
-        const u32 ev = (u32)((r0 + j) << 5) | lane;
-        for (u32 k = 0; k < n; ++k) {
-          okeys[o + k] = key0 == KEY_DROP ? KEY_DROP : (((key0 + k) << 2) | opc);
-          oevs[o + k] = ev;
+          ovf = true;
         }
       }
+      const u64 o = (u64)uo[j] + (u64)__popc(hmask & lt) * nk;
+      const u32 ev = (u32)(r << 5) | (u32)lane;
+      for (u32 k = 0; k < nk; ++k) {
+        okeys[o + k] = key0 == KEY_DROP ? KEY_DROP : (((key0 + k) << 2) | opc);
+        oevs[o + k] = ev;
+      }
+    }
+    __syncthreads();  // every warp is done with stage st: refill it
+    if (threadIdx.x == 0) {
+      const u64 cn = c + (u64)EX_STAGES * gridDim.x;
+      if (cn < n_chunks) issue(cn, st);
     }
   }
   if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
@@ -544,10 +578,21 @@ void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStrea
 
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
                    const u32* ub_off, u32* keys, u32* evs, u32* err, cudaStream_t st) {
-  const u64 warps = (g.n_recs + EXP_RPW - 1) / EXP_RPW;
-  if (!warps) return;
-  k_expand<<<(unsigned)((warps * 32 + 255) / 256), 256, 0, st>>>(recs, g, page_bits, page_rank, shared_base, ub_off,
-                                                                  keys, evs, err); ++g_launches;
+  const u64 chunks = (g.n_recs + EX_REC - 1) / EX_REC;
+  if (!chunks) return;
+  const size_t smem = sizeof(bc_record) * EX_REC * EX_STAGES + 8 * EX_STAGES;
+  static int grid = 0;
+  if (!grid) {
+    int dev = 0, sms = 148, per = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_expand, EX_THREADS, smem);
+    grid = sms * (per > 0 ? per : 1);
+  }
+  const unsigned gr = (unsigned)std::min<u64>(chunks, (u64)grid);
+  k_expand<<<gr, EX_THREADS, smem, st>>>(recs, g, page_bits, page_rank, shared_base, ub_off, keys, evs, err);
+  ++g_launches;
 }
 
 }  // namespace bc
