@@ -105,7 +105,14 @@ typedef struct bc_config {
   uint32_t smem_bytes_per_block;      /* shared-memory shadow size per block      */
   uint32_t flags;                     /* BC_F_*                                                  */
   int32_t device;                     /* CUDA device ordinal                                     */
-  int32_t rank, world;                /* world = 1 single GPU (multi-GPU: DESIGN.md §"Multi-GPU")*/
+  int32_t rank, world;                /* address sharding: world = 0 or
+                                         1 checks every shadow granule.  world = W > 1 (W <= 1024,
+                                         0 <= rank < W): every rank is given the SAME trace, derives
+                                         the clocks (K1-K3) itself, and checks only the granules it
+                                         owns, owner(g) = hash(g) mod W; barrier-divergence findings
+                                         are reported by rank 0 only.  The W per-rank race lists are
+                                         disjoint and their canonical merge is the world = 1 list
+                                         (the caller gathers them, e.g. over torch.distributed). */
   void* stream;                       /* cudaStream_t (NULL = a stream owned by the context)     */
 } bc_config;
 

@@ -117,7 +117,10 @@ def _stats_dict(s: _Stats):
 class Context:
     """One traced launch geometry on one GPU (bc_init ... bc_destroy)."""
 
-    def __init__(self, geometry: dict, device: int = 0, flags: int = 0, stream=None):
+    def __init__(self, geometry: dict, device: int = 0, flags: int = 0, stream=None, rank: int = 0, world: int = 1):
+        """rank / world > 1: address-sharded check (bc.h bc_config.rank/world): every rank loads
+        the same trace and reports the races of the shadow granules it owns; merge the per-rank
+        lists with merge_races() or gather_races()."""
         L = lib()
         grid = tuple(geometry["grid"]) + (1,) * (3 - len(geometry["grid"]))
         block = tuple(geometry["block"]) + (1,) * (3 - len(geometry["block"]))
@@ -129,7 +132,7 @@ class Context:
         c.smem_bytes_per_block = geometry.get("smem_bytes", 0)
         c.flags = flags
         c.device = device
-        c.rank, c.world = 0, 1
+        c.rank, c.world = rank, world
         c.stream = stream
         h = ctypes.c_void_p()
         st = L.bc_init(ctypes.byref(c), ctypes.byref(h))
@@ -208,6 +211,36 @@ class Context:
         self.close()
 
 
+def merge_races(parts) -> np.ndarray:
+    """Canonical merge of disjoint per-rank race lists (bc.h bc_race order): findings first by
+    (block, record), then global races by address, then shared races by (block, offset); ties by
+    (cur_event, prior_event).  Host-side argument marshalling only (no race arithmetic)."""
+    parts = [np.asarray(p, dtype=RACE_DTYPE) for p in parts]
+    r = np.concatenate(parts) if parts else np.zeros(0, dtype=RACE_DTYPE)
+    if len(r) == 0:
+        return r
+    finding = r["cls"] == 4
+    shared = r["space"] == 1
+    k1 = np.where(finding, 0, 1)
+    k2 = np.where(finding, 0, r["space"].astype(np.int64))
+    k3 = np.where(finding | shared, r["block"].astype(np.int64), 0)
+    k4 = np.where(finding, 0, r["addr"]).astype(np.uint64)
+    order = np.lexsort((r["prior_event"], r["cur_event"], k4, k3, k2, k1))
+    return r[order]
+
+
+def gather_races(local: np.ndarray, group=None, dst: int = 0):
+    """Gather every rank's race list over torch.distributed (any backend) and return the canonical
+    merge on rank `dst` (None elsewhere)."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    objs = [None] * world if dist.get_rank(group) == dst else None
+    dist.gather_object(np.asarray(local, dtype=RACE_DTYPE).tobytes(), objs, dst=dst, group=group)
+    if objs is None:
+        return None
+    return merge_races([np.frombuffer(b, dtype=RACE_DTYPE) for b in objs])
+
+
 @dataclass
 class Result:
     status: int
@@ -215,11 +248,12 @@ class Result:
     stats: dict
 
 
-def detect(records, geometry: dict, device="cuda:0", flags: int = 0, stream=None) -> Result:
+def detect(records, geometry: dict, device="cuda:0", flags: int = 0, stream=None, rank: int = 0,
+           world: int = 1) -> Result:
     """One-shot bc_init/bc_load_trace/bc_detect/bc_races.  Infeasible traces return
     status -2 with no races (as the oracle does)."""
     dev = int(str(device).split(":")[-1]) if str(device).startswith("cuda") else int(device)
-    with Context(geometry, device=dev, flags=flags, stream=stream) as ctx:
+    with Context(geometry, device=dev, flags=flags, stream=stream, rank=rank, world=world) as ctx:
         ctx.load_trace(records)
         st, stats = ctx.detect(allow=(-2,))
         races = ctx.races() if st == OK else np.zeros(0, dtype=RACE_DTYPE)

@@ -84,7 +84,8 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   *out = nullptr;
   if (cfg->warp_size != 32 || cfg->granule_log2 > 4) return BC_ERR_INVALID_ARG;
   if (cfg->flags & ~(u32)(BC_F_NO_SAME_VALUE_FILTER)) return BC_ERR_INVALID_ARG;  // overwrite: not on GPU yet
-  if (cfg->world != 1 && cfg->world != 0) return BC_ERR_INVALID_ARG;
+  if (cfg->world < 0 || cfg->world > 1024) return BC_ERR_INVALID_ARG;
+  if (cfg->world > 1 && (cfg->rank < 0 || cfg->rank >= cfg->world)) return BC_ERR_INVALID_ARG;
   u64 nb = (u64)cfg->grid_dim[0] * cfg->grid_dim[1] * cfg->grid_dim[2];
   u64 tpb = (u64)cfg->block_dim[0] * cfg->block_dim[1] * cfg->block_dim[2];
   if (nb == 0 || tpb == 0 || tpb > 1024 || nb * tpb > 0xFFFFFFFFull) return BC_ERR_INVALID_ARG;
@@ -107,6 +108,8 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   g.wpb = (u32)wpb;
   g.n_warps = (u32)(nb * wpb);
   g.wpb_m = wpb == 1 ? 0u : (u32)(((1ull << 32) + wpb - 1) / wpb);
+  g.world = cfg->world > 1 ? (u32)cfg->world : 1u;
+  g.rank = cfg->world > 1 ? (u32)cfg->rank : 0u;
   g.G = cfg->granule_log2;
   g.smem = cfg->smem_bytes_per_block;
   g.smem_gran = (u32)(((u64)g.smem + (1u << g.G) - 1) >> g.G);
@@ -355,6 +358,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   sx.items = n_items;
   cudaEventRecord(c->ev[7], st);
   // ---- K8: finalize
+  if (g.world > 1 && g.rank != 0) nfind = 0;  // findings come from the replicated replay: rank 0 reports them
   u64 total = (u64)n_r + nfind;
   if (total > c->races_cap) {
     if (c->races) cudaFree(c->races);

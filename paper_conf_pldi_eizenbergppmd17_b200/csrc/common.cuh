@@ -42,12 +42,24 @@ constexpr u32 SYNC_LOOKUP_CAP = 1u << 16;  // step cap of one foreign lookup
 struct Geo {
   u32 n_blocks, tpb, wpb, n_warps;
   u32 wpb_m;       // ceil(2^32 / wpb), 0 when wpb == 1: block of warp w = umulhi(w, wpb_m) (exact: n_warps * wpb < 2^32)
+  u32 rank, world; // address sharding: this context checks the granules g with shard_of(g) == rank
   u32 G;           // granule_log2
   u32 smem;        // bytes per block
   u32 smem_gran;   // granules per block
   u32 flags;
   u64 n_recs;
 };
+
+// owner rank of dense shadow key k (every rank derives the same dense keys from the same trace):
+// a murmur3 finaliser spreads neighbouring granules, then a multiply-shift maps to [0, world)
+__device__ __forceinline__ u32 shard_of(u32 k, u32 world) {
+  k ^= k >> 16;
+  k *= 0x85EBCA6Bu;
+  k ^= k >> 13;
+  k *= 0xC2B2AE35u;
+  k ^= k >> 16;
+  return (u32)(((u64)k * world) >> 32);
+}
 
 // traced block of traced warp w without an integer division
 __device__ __forceinline__ u32 blk_of(const Geo& g, u32 w) { return g.wpb_m ? __umulhi(w, g.wpb_m) : w; }
@@ -286,59 +298,24 @@ __device__ __forceinline__ T warp_incl_sum(T v) {
   return v;
 }
 
-// decoupled look-back status words (u64): [63:62] flag, [61:0] value
-constexpr u64 LB_AGG = 1ull << 62, LB_INC = 2ull << 62, LB_MASK = (1ull << 62) - 1;
-
-// Warp-cooperative version: all 32 lanes call it; 32 predecessors are inspected per round.
-__device__ __forceinline__ u64 lookback_u64_warp(volatile u64* status, u32 tile, u64 agg, int lane) {
-  if (tile == 0) {
-    if (lane == 0) status[0] = LB_INC | agg;
-    return 0;
-  }
-  if (lane == 0) status[tile] = LB_AGG | agg;
-  u64 excl = 0;
-  int hi = (int)tile - 1;
-  while (true) {
-    int idx = hi - lane;
-    u64 s = idx >= 0 ? (u64)status[idx] : (u64)(2ull << 62);
-    while (__any_sync(0xFFFFFFFFu, (s & ~LB_MASK) == 0)) {
-      if ((s & ~LB_MASK) == 0) s = status[idx];
-    }
-    u32 incm = __ballot_sync(0xFFFFFFFFu, (s & ~LB_MASK) == LB_INC);
-    int last = incm ? __ffs(incm) - 1 : 31;  // nearest inclusive predecessor ends the walk
-    u64 v = lane <= last ? (s & LB_MASK) : 0;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, o);
-    excl += v;
-    if (incm) break;
-    hi -= 32;
-  }
-  __threadfence();
-  if (lane == 0) status[tile] = LB_INC | (excl + agg);
-  return excl;
+// ------------------------------------------------ TMA 1-D bulk copies + mbarriers (sm_90+)
+__device__ __forceinline__ u32 smem_u32(const void* p) { return (u32)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(u64* bar, u32 count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
-
-// exclusive prefix of `agg` for tile `tile` over u64 status words (single value per tile).
-// Called by one thread.
-__device__ __forceinline__ u64 lookback_u64(volatile u64* status, u32 tile, u64 agg) {
-  if (tile == 0) {
-    status[0] = LB_INC | agg;
-    return 0;
+__device__ __forceinline__ void mbar_expect_tx(u64* bar, u32 bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, u32 bytes, u64* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(u64* bar, u32 phase) {
+  u32 done = 0;
+  while (!done) {
+    asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+                 : "=r"(done) : "r"(smem_u32(bar)), "r"(phase) : "memory");
   }
-  status[tile] = LB_AGG | agg;
-  u64 excl = 0;
-  int t = (int)tile - 1;
-  while (true) {
-    u64 s = status[t];
-    u64 f = s & ~LB_MASK;
-    if (f == 0) continue;
-    excl += s & LB_MASK;
-    if (f == LB_INC) break;
-    --t;
-  }
-  __threadfence();
-  status[tile] = LB_INC | (excl + agg);
-  return excl;
 }
 
 }  // namespace bc

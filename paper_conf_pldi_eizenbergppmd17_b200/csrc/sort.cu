@@ -186,109 +186,133 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_rows(u32* __restrict__ counts
   }
 }
 
-// Downsweep of one pass (stable in-tile rank, scatter through shared memory so that each digit's
-// run is written contiguously).  Register diet for occupancy (3 CTAs / SM): keys are staged in
-// shared memory in input order while they are ranked, each item keeps only (digit << 16 | rank),
-// and values are loaded after ranking.
-__global__ void __launch_bounds__(RS_THREADS, 3) k_rs_down(const u32* __restrict__ kin, const u32* __restrict__ vin,
+// Downsweep of one pass: stable in-tile rank (ballot match + per-warp histograms), scatter through
+// shared memory so that each digit's run is written contiguously (8 B in, 8 B out per item).
+// Persistent CTAs; each tile's keys and values arrive in shared memory by 1-D TMA bulk copies issued
+// RS_DSTAGES tiles ahead (mbarrier ring), so the global-load latency that dominated a one-tile-per-CTA
+// kernel overlaps the ranking and scattering of the previous tile.  The staged keys are read in input
+// order for ranking; once scattered, the stage's key half holds the permuted values.
+constexpr int RS_DSTAGES = 2;
+constexpr size_t RS_DSMEM = (size_t)RS_DSTAGES * 2 * RS_TILE * sizeof(u32) + RS_TILE * sizeof(u32) +
+                            RS_WARPS * RS_BINS * sizeof(u32) + 3 * RS_BINS * sizeof(u32) + 64 + RS_DSTAGES * 8;
+
+__global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict__ kin, const u32* __restrict__ vin,
                                                            u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
                                                            const u64* __restrict__ n_dev, int drop, int shift,
                                                            const u32* __restrict__ offs, u64 tiles) {
-  __shared__ u32 kst[RS_TILE];
-  __shared__ u32 skeys[RS_TILE];
-  __shared__ u32 whist[RS_WARPS][RS_BINS];
-  __shared__ u32 tofs[RS_BINS];
-  __shared__ u32 gstart[RS_BINS];
-  __shared__ u32 wsum[RS_WARPS];
-  __shared__ u32 s_kept;
+  extern __shared__ __align__(128) unsigned char rs_smem[];
+  u32* stage = reinterpret_cast<u32*>(rs_smem);                 // [RS_DSTAGES][2][RS_TILE] (keys, vals)
+  u32* skeys = stage + RS_DSTAGES * 2 * RS_TILE;                // [RS_TILE]
+  u32(*whist)[RS_BINS] = reinterpret_cast<u32(*)[RS_BINS]>(skeys + RS_TILE);
+  u32* tofs = &whist[RS_WARPS][0];
+  u32* gstart = tofs + RS_BINS;
+  u32* wsum = gstart + RS_BINS;                                 // [RS_WARPS]
+  u32* s_kept = wsum + RS_WARPS;
+  u64* bar = reinterpret_cast<u64*>(rs_smem + RS_DSMEM - RS_DSTAGES * 8);
 
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
-  for (int i = t; i < RS_WARPS * RS_BINS; i += RS_THREADS) (&whist[0][0])[i] = 0;
-  __syncthreads();
-  const u32 tile = blockIdx.x;
   const u64 n = n_dev ? *n_dev : n_max;
-  const u64 base = (u64)tile * RS_TILE;
-  if (base >= n) return;
-
-  u32 rank[RS_ITEMS];  // (digit << 16) | rank in the warp's digit run, NONE = no item
-  {
-    u32 k[RS_ITEMS];
-#pragma unroll
-    for (int j = 0; j < RS_ITEMS; ++j) {
-      const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-      k[j] = idx < n ? kin[idx] : KEY_DROP;
+  const u64 n_tiles = (n + RS_TILE - 1) / RS_TILE;
+  auto issue = [&](u64 tile, int st) {
+    const u64 base = tile * RS_TILE;
+    const u64 cnt = n - base < (u64)RS_TILE ? n - base : (u64)RS_TILE;
+    const u32 bytes = (u32)(((cnt + 3) & ~3ull) * sizeof(u32));  // whole 16-B units (buffers are padded)
+    mbar_expect_tx(&bar[st], vin ? 2 * bytes : bytes);
+    bulk_g2s(stage + st * 2 * RS_TILE, kin + base, bytes, &bar[st]);
+    if (vin) bulk_g2s(stage + st * 2 * RS_TILE + RS_TILE, vin + base, bytes, &bar[st]);
+  };
+  if (t == 0) {
+    for (int q = 0; q < RS_DSTAGES; ++q) mbar_init(&bar[q], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (t == 0)
+    for (int q = 0; q < RS_DSTAGES; ++q) {
+      const u64 tl = blockIdx.x + (u64)q * gridDim.x;
+      if (tl < n_tiles) issue(tl, q);
     }
-    const u32 lt = lanemask_lt();
+  const u32 lt = lanemask_lt();
+  u32 it = 0;
+  for (u64 tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++it) {
+    const int st = (int)(it % RS_DSTAGES);
+    const u32 phase = (it / RS_DSTAGES) & 1u;
+    u32* sk = stage + st * 2 * RS_TILE;
+    u32* sv = sk + RS_TILE;
+    const u64 base = tile * RS_TILE;
+    for (int i = t; i < RS_WARPS * RS_BINS; i += RS_THREADS) (&whist[0][0])[i] = 0;
+    gstart[t] = offs[(u64)t * tiles + tile];
+    __syncthreads();
+    mbar_wait(&bar[st], phase);
+    u32 rank[RS_ITEMS];  // (digit << 16) | rank in the warp's digit run, NONE = no item
 #pragma unroll
     for (int j = 0; j < RS_ITEMS; ++j) {
-      const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-      const u32 d = (idx < n && !(drop && k[j] == KEY_DROP)) ? ((k[j] >> shift) & 0xFFu) : 256u;
+      const u32 li = w * (RS_ITEMS * 32) + j * 32 + l;
+      const u64 idx = base + li;
+      const u32 k = idx < n ? sk[li] : KEY_DROP;
+      const u32 d = (idx < n && !(drop && k == KEY_DROP)) ? ((k >> shift) & 0xFFu) : 256u;
       const u32 peers = match9(d);
       const u32 old = d < 256u ? whist[w][d] : 0u;
       __syncwarp();
       if (d < 256u && (peers & lt) == 0) whist[w][d] = old + __popc(peers);
       __syncwarp();
       rank[j] = d < 256u ? ((d << 16) | (old + __popc(peers & lt))) : NONE;
-      kst[w * (RS_ITEMS * 32) + j * 32 + l] = k[j];
     }
-  }
-  u32 v[RS_ITEMS];
-#pragma unroll
-  for (int j = 0; j < RS_ITEMS; ++j) {
-    const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
-    v[j] = (vin && rank[j] != NONE) ? vin[idx] : 0u;
-  }
-  __syncthreads();
-  // per digit (thread t): prefix over warps, tile total
-  u32 total = 0;
-#pragma unroll
-  for (int ww = 0; ww < RS_WARPS; ++ww) {
-    const u32 c = whist[ww][t];
-    whist[ww][t] = total;
-    total += c;
-  }
-  gstart[t] = offs[(u64)t * tiles + tile];
-  // tile-local exclusive scan of the digit totals
-  {
-    const u32 x = warp_incl_sum(total);
-    if (l == 31) wsum[w] = x;
     __syncthreads();
-    u32 off = 0;
-    for (int ww = 0; ww < w; ++ww) off += wsum[ww];
-    tofs[t] = off + x - total;
-    if (t == RS_BINS - 1) s_kept = off + x;
-  }
-  __syncthreads();
-  // keys: scatter into digit order, then write each digit run contiguously
+    // per digit (thread t): prefix over warps, tile total; tile-local exclusive scan of the totals
+    u32 total = 0;
 #pragma unroll
-  for (int j = 0; j < RS_ITEMS; ++j) {
-    if (rank[j] != NONE) {
-      const u32 d = rank[j] >> 16;
-      const u32 pos = tofs[d] + whist[w][d] + (rank[j] & 0xFFFFu);
-      skeys[pos] = kst[w * (RS_ITEMS * 32) + j * 32 + l];
+    for (int ww = 0; ww < RS_WARPS; ++ww) {
+      const u32 c = whist[ww][t];
+      whist[ww][t] = total;
+      total += c;
     }
-  }
-  __syncthreads();
-  const u32 tile_n = s_kept;
-  for (u32 q = t; q < tile_n; q += RS_THREADS) {
-    const u32 kk = skeys[q];
-    const u32 d = (kk >> shift) & 0xFFu;
-    kout[(u64)gstart[d] + (q - tofs[d])] = kk;
-  }
-  if (!vout) return;
-  // values: the same permutation, staged in the (now free) input-order key buffer
-  u32* svals = kst;
+    {
+      const u32 x = warp_incl_sum(total);
+      if (l == 31) wsum[w] = x;
+      __syncthreads();
+      u32 off = 0;
+      for (int ww = 0; ww < w; ++ww) off += wsum[ww];
+      tofs[t] = off + x - total;
+      if (t == RS_BINS - 1) *s_kept = off + x;
+    }
+    __syncthreads();
 #pragma unroll
-  for (int j = 0; j < RS_ITEMS; ++j) {
-    if (rank[j] != NONE) {
-      const u32 d = rank[j] >> 16;
-      svals[tofs[d] + whist[w][d] + (rank[j] & 0xFFFFu)] = v[j];
+    for (int j = 0; j < RS_ITEMS; ++j) {
+      if (rank[j] != NONE) {
+        const u32 d = rank[j] >> 16;
+        skeys[tofs[d] + whist[w][d] + (rank[j] & 0xFFFFu)] = sk[w * (RS_ITEMS * 32) + j * 32 + l];
+      }
     }
-  }
-  __syncthreads();
-  for (u32 q = t; q < tile_n; q += RS_THREADS) {
-    const u32 d = (skeys[q] >> shift) & 0xFFu;
-    vout[(u64)gstart[d] + (q - tofs[d])] = svals[q];
+    __syncthreads();
+    const u32 tile_n = *s_kept;
+    for (u32 q = t; q < tile_n; q += RS_THREADS) {
+      const u32 kk = skeys[q];
+      const u32 d = (kk >> shift) & 0xFFu;
+      kout[(u64)gstart[d] + (q - tofs[d])] = kk;
+    }
+    if (vout) {
+      // values: the same permutation, staged in the stage's (now consumed) key half
+#pragma unroll
+      for (int j = 0; j < RS_ITEMS; ++j) {
+        if (rank[j] != NONE) {
+          const u32 d = rank[j] >> 16;
+          sk[tofs[d] + whist[w][d] + (rank[j] & 0xFFFFu)] = sv[w * (RS_ITEMS * 32) + j * 32 + l];
+        }
+      }
+      __syncthreads();
+      for (u32 q = t; q < tile_n; q += RS_THREADS) {
+        const u32 d = (skeys[q] >> shift) & 0xFFu;
+        vout[(u64)gstart[d] + (q - tofs[d])] = sk[q];
+      }
+    }
+    __syncthreads();  // stage st and the per-tile tables are free: refill the stage
+    if (t == 0) {
+      const u64 tn = tile + (u64)RS_DSTAGES * gridDim.x;
+      if (tn < n_tiles) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        issue(tn, st);
+      }
+    }
   }
 }
 
@@ -401,6 +425,13 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  static int down_grid = 0;
+  if (!down_grid) {
+    int per = 1;
+    cudaFuncSetAttribute(k_rs_down, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)RS_DSMEM);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_rs_down, RS_THREADS, RS_DSMEM);
+    down_grid = sms * (per > 0 ? per : 1);
+  }
   const unsigned hgrid =
       (unsigned)std::min<u64>((n + RS_THREADS * RS_HIST_ITEMS - 1) / (RS_THREADS * RS_HIST_ITEMS), (u64)sms * 8);
   k_rs_hist<<<hgrid, RS_THREADS, 0, st>>>(keys, n, n_dev, drop ? 1 : 0, bit_lo, passes, ghist); ++g_launches;
@@ -412,7 +443,8 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
     const int dr = (drop && p == 0) ? 1 : 0;
     k_rs_up<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles); ++g_launches;
     k_rs_rows<<<RS_BINS, RS_THREADS, 0, st>>>(counts, tiles, gbase + p * RS_BINS); ++g_launches;
-    k_rs_down<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, vi, ko, vo, n, nd, dr, shift, counts, tiles);
+    k_rs_down<<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, RS_DSMEM, st>>>(ki, vi, ko, vo, n, nd, dr,
+                                                                                           shift, counts, tiles);
     ++g_launches;
     if (dr) nd = n_out_dev;
     u32* tk = ki; ki = ko; ko = tk;

@@ -335,25 +335,6 @@ constexpr int EX_STAGES = 4;
 constexpr int EX_THREADS = 256;
 constexpr int EX_RPW = EX_REC / (EX_THREADS / 32);  // records per warp per chunk
 
-__device__ __forceinline__ u32 smem_u32(const void* p) { return (u32)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(u64* bar, u32 count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(u64* bar, u32 bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, u32 bytes, u64* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(u64* bar, u32 phase) {
-  u32 done = 0;
-  while (!done) {
-    asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
-                 : "=r"(done) : "r"(smem_u32(bar)), "r"(phase) : "memory");
-  }
-}
-
 __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restrict__ recs, Geo g,
                                                        const u32* __restrict__ page_bits,
                                                        const u32* __restrict__ page_rank, u32 shared_base,
@@ -430,7 +411,8 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
       const u64 o = (u64)uo[j] + (u64)__popc(hmask & lt) * nk;
       const u32 ev = (u32)(r << 5) | (u32)lane;
       for (u32 k = 0; k < nk; ++k) {
-        okeys[o + k] = key0 == KEY_DROP ? KEY_DROP : (((key0 + k) << 2) | opc);
+        const bool mine = key0 != KEY_DROP && (g.world == 1 || shard_of(key0 + k, g.world) == g.rank);
+        okeys[o + k] = mine ? (((key0 + k) << 2) | opc) : KEY_DROP;
         oevs[o + k] = ev;
       }
     }

@@ -1,0 +1,5 @@
+#!/bin/bash
+python -c "import __graft_entry__ as g; g.build()" || exit 1
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:k_rs_pass -s 2 -c 1 -o gpurun_out/prof_pass_c2 python tools/prof_one.py c2 > gpurun_out/ncu_pass_c2.log 2>&1; echo n1=$?
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:k_expand -c 1 -o gpurun_out/prof_expand_c4 python tools/prof_one.py c4 > gpurun_out/ncu_exp_c4.log 2>&1; echo n2=$?
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:k_check -c 1 -o gpurun_out/prof_check_c2 python tools/prof_one.py c2 > gpurun_out/ncu_chk_c2.log 2>&1; echo n3=$?
