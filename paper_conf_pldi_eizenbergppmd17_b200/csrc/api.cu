@@ -33,6 +33,7 @@ struct bc_ctx {
   size_t races_cap = 0;
   u64 n_races = 0;
   bc_stats stats{};
+  Arena arena;  // scratch buffers, reused across bc_detect calls
   std::string err;
   cudaEvent_t ev[16] = {};
 };
@@ -142,6 +143,7 @@ void bc_destroy(bc_ctx* c) {
   if (c->stream) cudaStreamSynchronize(c->stream);
   if (c->owned) cudaFree(c->owned);
   if (c->races) cudaFree(c->races);
+  c->arena.free_all();
   for (int i = 0; i < 16; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
   if (c->own_stream) cudaStreamDestroy(c->stream);
@@ -403,7 +405,7 @@ bc_status bc_detect(bc_ctx* c, bc_stats* out) {
   c->err.clear();
   bc_status s;
   {
-    Scratch S(c->stream);
+    Scratch S(c->stream, &c->arena);
     try {
       s = detect_impl(c, S);
     } catch (const std::bad_alloc&) {

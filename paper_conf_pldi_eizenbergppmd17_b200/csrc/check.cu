@@ -15,6 +15,9 @@
 // plus independent happens-before queries per item, evaluated with warp ballots over rounds of 32
 // sorted items (below).  Arbitrarily long (hot) granule segments cost the same per item as short
 // ones, and the shadow state never has to be materialised in memory.
+#include <cstdlib>
+#include <cstring>
+
 #include "common.cuh"
 #include "kernels.cuh"
 
@@ -402,6 +405,260 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
   }
 }
 
+// ---------------------------------------------------------------------------------------
+// Lane-sequential formulation (BC_K7=seq).  Same persistent warp ranges and incoming state
+// (walk_back / WarpEnd) as k_check, but each range is processed in blocks of KS_BLK = 1024 items:
+//   load   : the warp stages the block's (key, ev) words in shared memory (coalesced; stored with a
+//            33-word row pitch so that lane l reading item l*32+j is bank-conflict free)
+//   phase 1: lane l walks ITS 32 consecutive items and computes (a) the READINFLATE flag of each
+//            read (Fig. 2: its predecessor is a read of the same granule not ordered before it)
+//            and (b) the summary Sum of its chunk (last key, last writer, first inflation after it)
+//   scan   : a 5-step warp scan of the summaries (the same associative combine as k_check) gives
+//            every lane the automaton state (LW, FI) entering its chunk, and the block carry
+//   phase 2: lane l replays the rules of Fig. 2 / Fig. 3 over its chunk sequentially (W check,
+//            R check as epoch or vector, same-value filter) from that state.
+// Per item this costs a handful of thread instructions instead of a warp-wide ballot round per 32
+// items, and the per-item happens-before queries run on 32 independent lanes.
+constexpr int KS_WARPS = 8;
+constexpr int KS_BLK = 1024;
+constexpr int KS_PITCH = KS_BLK + KS_BLK / 32;  // 33-word rows
+
+__device__ __forceinline__ u32 kpad(u32 i) { return i + (i >> 5); }
+
+__device__ __forceinline__ Sum shfl_up_sum(const Sum& s, int o) {
+  Sum r;
+  r.fk = __shfl_up_sync(0xFFFFFFFFu, s.fk, o);
+  r.lk = __shfl_up_sync(0xFFFFFFFFu, s.lk, o);
+  r.lw = __shfl_up_sync(0xFFFFFFFFu, s.lw, o);
+  r.fi = __shfl_up_sync(0xFFFFFFFFu, s.fi, o);
+  r.bits = __shfl_up_sync(0xFFFFFFFFu, s.bits, o);
+  return r;
+}
+__device__ __forceinline__ Sum shfl_sum(const Sum& s, int src) {
+  Sum r;
+  r.fk = __shfl_sync(0xFFFFFFFFu, s.fk, src);
+  r.lk = __shfl_sync(0xFFFFFFFFu, s.lk, src);
+  r.lw = __shfl_sync(0xFFFFFFFFu, s.lw, src);
+  r.fi = __shfl_sync(0xFFFFFFFFu, s.fi, src);
+  r.bits = __shfl_sync(0xFFFFFFFFu, s.bits, src);
+  return r;
+}
+
+__global__ void __launch_bounds__(KS_WARPS * 32, 2) k_check_seq(CheckArgs a, WarpEnd* wend, u32 nw) {
+  extern __shared__ __align__(16) u32 ks_smem[];
+  const int wi = threadIdx.x >> 5;
+  u32* sK = ks_smem + (size_t)wi * 2 * KS_PITCH;
+  u32* sE = sK + KS_PITCH;
+  const u64 n = *a.n_dev;
+  const u32 w = blockIdx.x * KS_WARPS + wi;
+  const u32 lane = threadIdx.x & 31;
+  const HbCtx& c = a.c;
+  const u64 nr = (n + 31) / 32;
+  const u64 beg = (nr * w / nw) * 32, end = min(n, (nr * (w + 1) / nw) * 32);
+  const u32 no_sv = c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
+
+  // ---- incoming state of the range (as k_check)
+  Sum carry = sum_ident();
+  u32 pkx = NONE, pev = 0;  // the item before the block
+  u32 cwk = 0, cwe = 0;     // key word / event of carry.lw
+  if (beg > 0 && beg < end) {
+    pkx = a.keys[beg - 1];
+    pev = a.evs[beg - 1];
+    if ((pkx >> 2) == (a.keys[beg] >> 2)) {
+      if (!walk_back(a, beg, carry)) {
+        volatile WarpEnd* pe = &wend[w - 1];
+        while (pe->flag == 0) {
+        }
+        __threadfence();
+        carry.fk = carry.lk = pe->lk;
+        carry.lw = pe->lw;
+        carry.fi = pe->fi;
+        carry.bits = 1u | (carry.lw ? 2u : 0u);
+      }
+      if (carry.lw) {
+        cwk = a.keys[carry.lw - 1];
+        cwe = a.evs[carry.lw - 1];
+      }
+    }
+  }
+
+  u32 segs = 0;
+  for (u64 bb = beg; bb < end; bb += KS_BLK) {
+    const u32 nb = (u32)(end - bb < (u64)KS_BLK ? end - bb : (u64)KS_BLK);
+#pragma unroll 8
+    for (u32 r = 0; r < 32; ++r) {
+      const u32 li = r * 32 + lane;
+      sK[kpad(li)] = li < nb ? a.keys[bb + li] : NONE;
+      sE[kpad(li)] = li < nb ? a.evs[bb + li] : 0u;
+    }
+    __syncwarp();
+    const u32 l0 = lane * 32;
+    const u32 ppk = lane == 0 ? pkx : (l0 - 1 < nb ? sK[kpad(l0 - 1)] : NONE);
+    const u32 ppe = lane == 0 ? pev : (l0 - 1 < nb ? sE[kpad(l0 - 1)] : 0u);
+    const u32 cnt = l0 < nb ? min(32u, nb - l0) : 0u;
+
+    // ---- phase 1: READINFLATE flags and the chunk summary
+    Sum sm = sum_ident();
+    u32 imask = 0;
+    {
+      u32 pk = ppk, pe = ppe, pw = 0;
+      bool pw_ok = false, kc = false;
+      u32 tlw = 0, tfi = NONE;
+      for (u32 j = 0; j < cnt; ++j) {
+        const u32 li = l0 + j;
+        const u32 k = sK[kpad(li)], e = sE[kpad(li)];
+        const u32 key = k >> 2, op = k & 3u;
+        const u32 gi = (u32)(bb + li);
+        const bool same = pk != NONE && (pk >> 2) == key;
+        if (j == 0) sm.fk = key;
+        if (!same) {
+          ++segs;
+          if (j > 0) kc = true;
+          tlw = 0;
+          tfi = NONE;
+        }
+        bool loaded = false;
+        if (op != IOP_LD) {
+          tlw = gi + 1u;
+          tfi = NONE;
+        } else if (same && (pk & 3u) == IOP_LD) {
+          if (!pw_ok) pw = __ldg(&c.snap[pe >> 5].x);
+          const Snap s2 = load_snap(c.snap, e >> 5);
+          if (!hb_ev(c, pe, pw, e, s2)) {
+            imask |= 1u << j;
+            if (tfi == NONE) tfi = gi;
+          }
+          pw = s2.warp;
+          loaded = true;
+        }
+        pw_ok = loaded;
+        pk = k;
+        pe = e;
+        sm.lk = key;
+      }
+      if (cnt) {
+        sm.lw = tlw;
+        sm.fi = tfi;
+        sm.bits = (kc ? 0u : 1u) | (tlw ? 2u : 0u);
+      }
+    }
+
+    // ---- scan of the chunk summaries -> state entering each chunk; block carry
+    Sum incl = sm;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const Sum up = shfl_up_sum(incl, o);
+      if ((int)lane >= o) incl = combine(up, incl);
+    }
+    Sum ex = shfl_up_sum(incl, 1);
+    if (lane == 0) ex = sum_ident();
+    const Sum in = combine(carry, ex);
+    const Sum blk = shfl_sum(incl, 31);
+
+    // ---- phase 2: the rules, lane-sequentially
+    if (cnt) {
+      u32 lw = (in.fk != NONE) ? in.lw : 0u, fi = (in.fk != NONE) ? in.fi : NONE;
+      u32 wk = 0, we = 0, ww = 0;
+      bool ww_ok = false;
+      if (lw) {
+        if ((u64)(lw - 1) >= bb) {
+          wk = sK[kpad((u32)(lw - 1 - bb))];
+          we = sE[kpad((u32)(lw - 1 - bb))];
+        } else {
+          wk = cwk;
+          we = cwe;
+        }
+      }
+      u32 pk = ppk, pe = ppe, pw = 0;
+      bool pw_ok = false;
+      for (u32 j = 0; j < cnt; ++j) {
+        const u32 li = l0 + j;
+        const u32 k = sK[kpad(li)], e = sE[kpad(li)];
+        const u32 key = k >> 2, op = k & 3u;
+        const u32 gi = (u32)(bb + li);
+        const bool same = pk != NONE && (pk >> 2) == key;
+        if (!same) {
+          lw = 0;
+          fi = NONE;
+        }
+        const u32 nk = li + 1 < nb ? sK[kpad(li + 1)] : NONE;
+        const bool same_next = nk != NONE && (nk >> 2) == key;
+        const bool atm_only = op == IOP_ATOM && (!same || (pk & 3u) == IOP_ATOM) &&
+                              (!same_next || (nk & 3u) == IOP_ATOM);
+        const bool need = (same || same_next) && !atm_only;
+        Snap s2{0, 0, 0, 0};
+        if (need) s2 = load_snap(c.snap, e >> 5);
+        if (op == IOP_LD) {
+          if (((imask >> j) & 1u) && fi == NONE) fi = gi;
+          if (lw) {  // W_x check of a read (Fig. 2 READ*)
+            if (!ww_ok) {
+              ww = __ldg(&c.snap[we >> 5].x);
+              ww_ok = true;
+            }
+            if (!hb_ev(c, we, ww, e, s2)) emit(a, key, e, we, (wk & 3u) == IOP_ATOM ? BC_KIND_AR : BC_KIND_WR);
+          }
+        } else {
+          const bool patm = (wk & 3u) == IOP_ATOM;
+          if (lw && !(op == IOP_ATOM && patm)) {  // W_x check (atomics only against a plain write)
+            if (!ww_ok) {
+              ww = __ldg(&c.snap[we >> 5].x);
+              ww_ok = true;
+            }
+            if (!hb_ev(c, we, ww, e, s2)) {
+              if (op == IOP_ATOM) {
+                emit(a, key, e, we, BC_KIND_WA);
+              } else {
+                const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (we >> 5) == (e >> 5);
+                if (!filtered) emit(a, key, e, we, patm ? BC_KIND_AW : BC_KIND_WW);
+              }
+            }
+          }
+          if (same && (pk & 3u) == IOP_LD) {  // R_x check at a writer: epoch, or vector after READINFLATE
+            const u32 kind = op == IOP_ATOM ? BC_KIND_RA : BC_KIND_RW;
+            if (fi == NONE) {
+              if (!pw_ok) pw = __ldg(&c.snap[pe >> 5].x);
+              if (!hb_ev(c, pe, pw, e, s2)) emit(a, key, e, pe, kind);
+            } else {
+              vc_check(a.evs, a.races, a.race_cnt, a.race_cap, (u64)fi - 1, (u64)gi - 1, e, s2.warp, s2.ps, s2.node,
+                       s2.blab, key, kind);
+            }
+          }
+          lw = gi + 1u;
+          wk = k;
+          we = e;
+          ww = s2.warp;
+          ww_ok = need;
+          fi = NONE;
+        }
+        pw = s2.warp;
+        pw_ok = need;
+        pk = k;
+        pe = e;
+      }
+    }
+
+    // ---- block carry
+    carry = combine(carry, blk);
+    if (carry.lw && (u64)(carry.lw - 1) >= bb) {
+      cwk = sK[kpad((u32)(carry.lw - 1 - bb))];
+      cwe = sE[kpad((u32)(carry.lw - 1 - bb))];
+    }
+    pkx = sK[kpad(nb - 1)];
+    pev = sE[kpad(nb - 1)];
+    __syncwarp();
+  }
+  segs = __reduce_add_sync(0xFFFFFFFFu, segs);
+  if (lane == 0) {
+    if (segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)segs);
+    volatile WarpEnd* me = &wend[w];
+    me->lk = carry.lk;
+    me->lw = carry.lw;
+    me->fi = carry.fi;
+    __threadfence();
+    me->flag = 1u;
+  }
+}
+
 }  // namespace
 
 size_t check_status_bytes(u64 n) { return (size_t)148 * 64 * sizeof(WarpEnd) + 256; }
@@ -409,17 +666,27 @@ size_t check_status_bytes(u64 n) { return (size_t)148 * 64 * sizeof(WarpEnd) + 2
 void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_dev, u64 n_max, void* status,
                   uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, cudaStream_t st) {
   if (n_max == 0) return;
-  static int grid = 0;
-  if (!grid) {
+  // K7 variant: ballot rounds (default; fastest on read-heavy C2/C3) or lane-sequential
+  // (BC_K7=seq; fastest on atomic-heavy C4/C5)
+  static int use_seq = -1, grid = 0;
+  const size_t smem_seq = (size_t)KS_WARPS * 2 * KS_PITCH * sizeof(u32);
+  if (use_seq < 0) {
+    const char* v = getenv("BC_K7");
+    use_seq = (v && !strcmp(v, "seq")) ? 1 : 0;
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_check, K7_WARPS * 32, 0);
+    if (use_seq) {
+      cudaFuncSetAttribute(k_check_seq, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_seq);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_check_seq, KS_WARPS * 32, smem_seq);
+    } else {
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_check, K7_WARPS * 32, 0);
+    }
     if (per < 1) per = 1;
     grid = sms * per;
     if (grid * K7_WARPS > 148 * 64) grid = 148 * 64 / K7_WARPS;
   }
-  const u32 nw = (u32)grid * K7_WARPS;
+  const u32 nw = (u32)grid * (use_seq ? KS_WARPS : K7_WARPS);
   cudaMemsetAsync(status, 0, (size_t)nw * sizeof(WarpEnd), st);
   cudaMemcpyToSymbolAsync(cHC, &c, sizeof(HbCtx), 0, cudaMemcpyHostToDevice, st);
   CheckArgs a;
@@ -431,7 +698,12 @@ void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_
   a.race_cnt = race_cnt;
   a.race_cap = race_cap;
   a.seg_cnt = seg_cnt;
-  k_check<<<grid, K7_WARPS * 32, 0, st>>>(a, (WarpEnd*)status, nw); ++g_launches;
+  if (use_seq) {
+    k_check_seq<<<grid, KS_WARPS * 32, smem_seq, st>>>(a, (WarpEnd*)status, nw);
+  } else {
+    k_check<<<grid, K7_WARPS * 32, 0, st>>>(a, (WarpEnd*)status, nw);
+  }
+  ++g_launches;
 }
 
 }  // namespace bc

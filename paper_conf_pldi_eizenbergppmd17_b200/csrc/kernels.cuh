@@ -16,33 +16,55 @@ extern u64 g_launches;
 enum { C_LANE_EVENTS = 0, C_CONTROL_EVENTS, C_SYNC_RECS, C_ACQ_RECS, C_MEM_RECS, C_IFS, C_BARS, C_SYNC_LANEOPS,
        C_ITEMS, C_ITEM_BOUND, C_SEGMENTS, C_PAGE_WORDS, C_PAGES, C_N };
 
-// Stream-ordered scratch memory for one bc_detect: cudaMallocAsync from the device's memory
-// pool (kept cached between calls), all freed at release().
+// Per-context scratch arena.  A bc_detect allocates its scratch buffers in a fixed order; the i-th
+// allocation reuses the i-th buffer of earlier calls when it is large enough, so repeated detects of
+// one trace see identical pointers -- which is what lets the post-header pipeline be replayed as a
+// CUDA graph (api.cu).  Buffers are 256-B aligned and padded to a multiple of 256 B (the TMA bulk
+// copies of the radix sort may read up to 12 B past an array's end).  Freed at bc_destroy.
+struct Arena {
+  std::vector<std::pair<void*, size_t>> bufs;
+  u64 gen = 0;  // bumped whenever a buffer is (re)allocated
+  void free_all() {
+    for (auto& b : bufs)
+      if (b.first) cudaFree(b.first);
+    bufs.clear();
+    ++gen;
+  }
+};
+
 class Scratch {
  public:
-  explicit Scratch(cudaStream_t st) : st_(st) {}
-  ~Scratch() { release(); }
+  Scratch(cudaStream_t st, Arena* ar) : st_(st), ar_(ar) {}
   template <typename T>
   T* alloc(size_t n) {
-    void* p = nullptr;
     size_t bytes = n * sizeof(T);
     if (bytes == 0) bytes = 16;
     bytes = (bytes + 255) & ~(size_t)255;
-    if (cudaMallocAsync(&p, bytes, st_) != cudaSuccess || !p) {
+    const size_t i = next_++;
+    if (i < ar_->bufs.size() && ar_->bufs[i].second >= bytes) return (T*)ar_->bufs[i].first;
+    if (i < ar_->bufs.size()) {
+      cudaStreamSynchronize(st_);  // the old buffer may still be read by queued work
+      cudaFree(ar_->bufs[i].first);
+      ar_->bufs[i] = {nullptr, 0};
+    } else {
+      ar_->bufs.push_back({nullptr, 0});
+    }
+    void* p = nullptr;
+    const size_t cap = bytes + ((bytes / 8 + 255) & ~(size_t)255);
+    if (cudaMalloc(&p, cap) != cudaSuccess || !p) {
       cudaGetLastError();
       throw std::bad_alloc();
     }
-    ptrs_.push_back(p);
+    ar_->bufs[i] = {p, cap};
+    ++ar_->gen;
     return (T*)p;
   }
-  void release() {
-    for (void* p : ptrs_) cudaFreeAsync(p, st_);
-    ptrs_.clear();
-  }
+  void release() {}
 
  private:
   cudaStream_t st_;
-  std::vector<void*> ptrs_;
+  Arena* ar_;
+  size_t next_ = 0;
 };
 
 // sort.cu

@@ -1,5 +1,5 @@
-// sort.cu — hand-written stable LSD radix sort (8-bit digits, reduce-then-scan per pass) and a
-// device-wide exclusive scan, for sm_100a.
+// sort.cu — hand-written stable LSD radix sort (8- to 10-bit digits, reduce-then-scan per pass)
+// and a device-wide exclusive scan, for sm_100a.
 //
 // The radix sort is the paper's per-location serialisation (a spinlock per shadow
 // entry orders the host threads' accesses) turned into data parallelism: a STABLE sort of
@@ -26,17 +26,18 @@ constexpr int RS_THREADS = 256;
 constexpr int RS_ITEMS = 16;
 constexpr int RS_TILE = RS_THREADS * RS_ITEMS;  // 4096
 constexpr int RS_WARPS = RS_THREADS / 32;
-constexpr int RS_BINS = 256;
+constexpr int RS_MAXB = 1024;                   // bins of the widest digit (10 bits)
 constexpr int RS_MAXP = 4;
-// temp header: ghist[RS_MAXP][256], gbase[RS_MAXP][256]; the (digit, tile) table follows
-constexpr size_t RS_HDR_BYTES = (2 * RS_MAXP * 256 + 64) * sizeof(u32);
+// temp header: ghist[RS_MAXP][RS_MAXB], gbase[RS_MAXP][RS_MAXB]; the (digit, tile) table follows
+constexpr size_t RS_HDR_BYTES = (2 * RS_MAXP * RS_MAXB + 64) * sizeof(u32);
 
-// Lanes of the warp holding the same 9-bit label (digit, or 256 = no item): 9 ballots, a fixed
-// cost independent of how many distinct digits the warp holds.
-__device__ __forceinline__ u32 match9(u32 d) {
+// Lanes of the warp holding the same (RB+1)-bit label (digit, or 1 << RB = no item): RB+1 ballots,
+// a fixed cost independent of how many distinct digits the warp holds.
+template <int RB>
+__device__ __forceinline__ u32 match_label(u32 d) {
   u32 m = 0xFFFFFFFFu;
 #pragma unroll
-  for (int b = 0; b < 9; ++b) {
+  for (int b = 0; b <= RB; ++b) {
     const bool bit = (d >> b) & 1u;
     const u32 bal = __ballot_sync(0xFFFFFFFFu, bit);
     m &= bit ? bal : ~bal;
@@ -44,17 +45,29 @@ __device__ __forceinline__ u32 match9(u32 d) {
   return m;
 }
 
+// add 1 per lane to h[d]; a warp that holds one digit only (the common case for the high digits of
+// sorted-ish keys) does a single atomic
+__device__ __forceinline__ void warp_hist_add(u32* h, u32 d, bool ok, u32 lt) {
+  const u32 vm = __ballot_sync(0xFFFFFFFFu, ok);
+  const u32 d0 = __shfl_sync(0xFFFFFFFFu, d, vm ? __ffs(vm) - 1 : 0);
+  if (__all_sync(0xFFFFFFFFu, !ok || d == d0)) {
+    if (vm && (lt & vm) == 0 && ok) atomicAdd(&h[d], (u32)__popc(vm));
+  } else if (ok) {
+    atomicAdd(&h[d], 1u);
+  }
+}
+
 constexpr int RS_HIST_ITEMS = 8;
 
-// Global digit histograms of all passes in one read.  Same-digit keys of a warp are combined
-// (match9) before the shared-memory atomic (sorted-ish inputs hit one bin hard).  Each thread keeps
-// RS_HIST_ITEMS loads in flight.
+// Global digit histograms of all passes in one read of the keys.
+template <int RB>
 __global__ void __launch_bounds__(RS_THREADS) k_rs_hist(const u32* __restrict__ kin, u64 n_max,
                                                         const u64* __restrict__ n_dev, int drop, int bit_lo,
                                                         int passes, u32* __restrict__ ghist) {
-  __shared__ u32 h[RS_MAXP][RS_BINS];
+  constexpr int BINS = 1 << RB;
+  __shared__ u32 h[RS_MAXP * BINS];
   const int t = threadIdx.x;
-  for (int i = t; i < RS_MAXP * RS_BINS; i += RS_THREADS) (&h[0][0])[i] = 0;
+  for (int i = t; i < RS_MAXP * BINS; i += RS_THREADS) h[i] = 0;
   __syncthreads();
   const u64 n = n_dev ? *n_dev : n_max;
   const u32 lt = lanemask_lt();
@@ -71,52 +84,47 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_hist(const u32* __restrict__ 
     for (int j = 0; j < RS_HIST_ITEMS; ++j) {
       const u64 idx = base + (u64)j * RS_THREADS + t;
       const bool ok = idx < n && !(drop && k[j] == KEY_DROP);
-      const u32 vm = __ballot_sync(0xFFFFFFFFu, ok);
-      for (int p = 0; p < passes; ++p) {
-        const u32 d = ok ? (k[j] >> (bit_lo + 8 * p)) & 0xFFu : 0x100u;
-        // one digit across the warp (the common case for the high digits): one atomic
-        const u32 d0 = __shfl_sync(0xFFFFFFFFu, d, vm ? __ffs(vm) - 1 : 0);
-        if (__all_sync(0xFFFFFFFFu, !ok || d == d0)) {
-          if (vm && (lt & vm) == 0 && ok) atomicAdd(&h[p][d], (u32)__popc(vm));
-        } else if (ok) {
-          atomicAdd(&h[p][d], 1u);
-        }
-      }
+      for (int p = 0; p < passes; ++p)
+        warp_hist_add(h + p * BINS, ok ? (k[j] >> (bit_lo + RB * p)) & (BINS - 1) : 0u, ok, lt);
     }
   }
   __syncthreads();
-  for (int i = t; i < passes * RS_BINS; i += RS_THREADS) {
-    const u32 v = (&h[0][0])[i];
-    if (v) atomicAdd(&ghist[i], v);
+  for (int i = t; i < passes * BINS; i += RS_THREADS) {
+    const u32 v = h[i];
+    if (v) atomicAdd(&ghist[(i / BINS) * RS_MAXB + (i % BINS)], v);
   }
 }
 
-// gbase[p][d] = exclusive prefix of ghist[p][*]; *n_out = kept items (pass 0 total)
-__global__ void __launch_bounds__(RS_BINS) k_rs_bins(const u32* __restrict__ ghist, u32* __restrict__ gbase,
+// gbase[p][d] = exclusive prefix of ghist[p][*]; *n_out = kept items (pass 0 total).  BINS threads.
+template <int RB>
+__global__ void __launch_bounds__(1 << RB) k_rs_bins(const u32* __restrict__ ghist, u32* __restrict__ gbase,
                                                      u64* __restrict__ n_out) {
-  __shared__ u32 wsum[RS_BINS / 32];
+  constexpr int BINS = 1 << RB;
+  __shared__ u32 wsum[BINS / 32];
   const int t = threadIdx.x, w = t >> 5, l = t & 31, p = blockIdx.x;
-  const u32 v = ghist[p * RS_BINS + t];
+  const u32 v = ghist[p * RS_MAXB + t];
   const u32 x = warp_incl_sum(v);
   if (l == 31) wsum[w] = x;
   __syncthreads();
   u32 off = 0, tot = 0;
-  for (int ww = 0; ww < RS_BINS / 32; ++ww) {
+  for (int ww = 0; ww < BINS / 32; ++ww) {
     if (ww < w) off += wsum[ww];
     tot += wsum[ww];
   }
-  gbase[p * RS_BINS + t] = off + x - v;
+  gbase[p * RS_MAXB + t] = off + x - v;
   if (p == 0 && t == 0 && n_out) *n_out = tot;
 }
 
 // Upsweep of one pass: the digit counts of every tile, digit-major (counts[d * tiles + tile]);
 // tiles past the (device-side) item count write zeros.
+template <int RB>
 __global__ void __launch_bounds__(RS_THREADS) k_rs_up(const u32* __restrict__ kin, u64 n_max,
                                                       const u64* __restrict__ n_dev, int drop, int shift,
                                                       u32* __restrict__ counts, u64 tiles) {
-  __shared__ u32 h[RS_BINS];
+  constexpr int BINS = 1 << RB;
+  __shared__ u32 h[BINS];
   const int t = threadIdx.x;
-  h[t] = 0;
+  for (int i = t; i < BINS; i += RS_THREADS) h[i] = 0;
   __syncthreads();
   const u64 n = n_dev ? *n_dev : n_max;
   const u64 base = (u64)blockIdx.x * RS_TILE;
@@ -132,22 +140,16 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_up(const u32* __restrict__ ki
     for (int j = 0; j < RS_ITEMS; ++j) {
       const u64 idx = base + (u64)j * RS_THREADS + t;
       const bool ok = idx < n && !(drop && k[j] == KEY_DROP);
-      const u32 d = ok ? (k[j] >> shift) & 0xFFu : 0x100u;
-      const u32 vm = __ballot_sync(0xFFFFFFFFu, ok);
-      const u32 d0 = __shfl_sync(0xFFFFFFFFu, d, vm ? __ffs(vm) - 1 : 0);
-      if (__all_sync(0xFFFFFFFFu, !ok || d == d0)) {
-        if (vm && (lt & vm) == 0 && ok) atomicAdd(&h[d], (u32)__popc(vm));
-      } else if (ok) {
-        atomicAdd(&h[d], 1u);
-      }
+      warp_hist_add(h, ok ? (k[j] >> shift) & (BINS - 1) : 0u, ok, lt);
     }
   }
   __syncthreads();
-  counts[(u64)t * tiles + blockIdx.x] = h[t];
+  for (int d = t; d < BINS; d += RS_THREADS) counts[(u64)d * tiles + blockIdx.x] = h[d];
 }
 
 // One CTA per digit d: offs[d * tiles + tile] = gbase[d] + (items of digit d in tiles < tile).
-// The 256 rows are independent, so there is no serial chain across tiles.
+// The rows are independent, so there is no serial chain across tiles (unlike a decoupled
+// look-back, whose first wave of ~450 co-resident tiles walks back one L2 round trip per step).
 __global__ void __launch_bounds__(RS_THREADS) k_rs_rows(u32* __restrict__ counts, u64 tiles,
                                                         const u32* __restrict__ gbase) {
   __shared__ u32 wsum[RS_WARPS];
@@ -188,27 +190,33 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_rows(u32* __restrict__ counts
 
 // Downsweep of one pass: stable in-tile rank (ballot match + per-warp histograms), scatter through
 // shared memory so that each digit's run is written contiguously (8 B in, 8 B out per item).
-// Persistent CTAs; each tile's keys and values arrive in shared memory by 1-D TMA bulk copies issued
-// RS_DSTAGES tiles ahead (mbarrier ring), so the global-load latency that dominated a one-tile-per-CTA
-// kernel overlaps the ranking and scattering of the previous tile.  The staged keys are read in input
-// order for ranking; once scattered, the stage's key half holds the permuted values.
+// Persistent CTAs; each tile's keys arrive in shared memory by 1-D TMA bulk copies issued
+// RS_DSTAGES tiles ahead (mbarrier ring), so the load latency that dominated a one-tile-per-CTA kernel
+// overlaps the ranking of the previous tile; the tile's values are loaded into registers at the start
+// of the tile and land while it is ranked.  Once scattered, the stage holds the permuted values.
 constexpr int RS_DSTAGES = 2;
-constexpr size_t RS_DSMEM = (size_t)RS_DSTAGES * 2 * RS_TILE * sizeof(u32) + RS_TILE * sizeof(u32) +
-                            RS_WARPS * RS_BINS * sizeof(u32) + 3 * RS_BINS * sizeof(u32) + 64 + RS_DSTAGES * 8;
+template <int RB>
+constexpr size_t rs_dsmem() {
+  return (size_t)RS_DSTAGES * RS_TILE * sizeof(u32) + RS_TILE * sizeof(u32) +
+         (size_t)(RS_WARPS + 2) * (1 << RB) * sizeof(u32) + 64 + RS_DSTAGES * 8;
+}
 
+template <int RB>
 __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict__ kin, const u32* __restrict__ vin,
                                                            u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
                                                            const u64* __restrict__ n_dev, int drop, int shift,
                                                            const u32* __restrict__ offs, u64 tiles) {
+  constexpr int BINS = 1 << RB;
+  constexpr int DPT = BINS / RS_THREADS;  // digits per thread (1, 2 or 4)
   extern __shared__ __align__(128) unsigned char rs_smem[];
-  u32* stage = reinterpret_cast<u32*>(rs_smem);                 // [RS_DSTAGES][2][RS_TILE] (keys, vals)
-  u32* skeys = stage + RS_DSTAGES * 2 * RS_TILE;                // [RS_TILE]
-  u32(*whist)[RS_BINS] = reinterpret_cast<u32(*)[RS_BINS]>(skeys + RS_TILE);
-  u32* tofs = &whist[RS_WARPS][0];
-  u32* gstart = tofs + RS_BINS;
-  u32* wsum = gstart + RS_BINS;                                 // [RS_WARPS]
+  u32* stage = reinterpret_cast<u32*>(rs_smem);                 // [RS_DSTAGES][RS_TILE] keys
+  u32* skeys = stage + RS_DSTAGES * RS_TILE;                    // [RS_TILE]
+  u32* whist = skeys + RS_TILE;                                 // [RS_WARPS][BINS]
+  u32* tofs = whist + RS_WARPS * BINS;                          // [BINS]
+  u32* gstart = tofs + BINS;                                    // [BINS]
+  u32* wsum = gstart + BINS;                                    // [RS_WARPS]
   u32* s_kept = wsum + RS_WARPS;
-  u64* bar = reinterpret_cast<u64*>(rs_smem + RS_DSMEM - RS_DSTAGES * 8);
+  u64* bar = reinterpret_cast<u64*>(rs_smem + rs_dsmem<RB>() - RS_DSTAGES * 8);
 
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
   const u64 n = n_dev ? *n_dev : n_max;
@@ -217,9 +225,8 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
     const u64 base = tile * RS_TILE;
     const u64 cnt = n - base < (u64)RS_TILE ? n - base : (u64)RS_TILE;
     const u32 bytes = (u32)(((cnt + 3) & ~3ull) * sizeof(u32));  // whole 16-B units (buffers are padded)
-    mbar_expect_tx(&bar[st], vin ? 2 * bytes : bytes);
-    bulk_g2s(stage + st * 2 * RS_TILE, kin + base, bytes, &bar[st]);
-    if (vin) bulk_g2s(stage + st * 2 * RS_TILE + RS_TILE, vin + base, bytes, &bar[st]);
+    mbar_expect_tx(&bar[st], bytes);
+    bulk_g2s(stage + st * RS_TILE, kin + base, bytes, &bar[st]);
   };
   if (t == 0) {
     for (int q = 0; q < RS_DSTAGES; ++q) mbar_init(&bar[q], 1);
@@ -236,11 +243,18 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
   for (u64 tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++it) {
     const int st = (int)(it % RS_DSTAGES);
     const u32 phase = (it / RS_DSTAGES) & 1u;
-    u32* sk = stage + st * 2 * RS_TILE;
-    u32* sv = sk + RS_TILE;
+    u32* sk = stage + st * RS_TILE;
     const u64 base = tile * RS_TILE;
-    for (int i = t; i < RS_WARPS * RS_BINS; i += RS_THREADS) (&whist[0][0])[i] = 0;
-    gstart[t] = offs[(u64)t * tiles + tile];
+    u32 v[RS_ITEMS];
+    if (vin) {
+#pragma unroll
+      for (int j = 0; j < RS_ITEMS; ++j) {
+        const u64 idx = base + (u64)w * (RS_ITEMS * 32) + j * 32 + l;
+        v[j] = idx < n ? vin[idx] : 0u;
+      }
+    }
+    for (int i = t; i < RS_WARPS * BINS; i += RS_THREADS) whist[i] = 0;
+    for (int d = t; d < BINS; d += RS_THREADS) gstart[d] = offs[(u64)d * tiles + tile];
     __syncthreads();
     mbar_wait(&bar[st], phase);
     u32 rank[RS_ITEMS];  // (digit << 16) | rank in the warp's digit run, NONE = no item
@@ -249,59 +263,72 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
       const u32 li = w * (RS_ITEMS * 32) + j * 32 + l;
       const u64 idx = base + li;
       const u32 k = idx < n ? sk[li] : KEY_DROP;
-      const u32 d = (idx < n && !(drop && k == KEY_DROP)) ? ((k >> shift) & 0xFFu) : 256u;
-      const u32 peers = match9(d);
-      const u32 old = d < 256u ? whist[w][d] : 0u;
+      const u32 d = (idx < n && !(drop && k == KEY_DROP)) ? ((k >> shift) & (BINS - 1)) : (u32)BINS;
+      const u32 peers = match_label<RB>(d);
+      u32* hw = whist + w * BINS;
+      const u32 old = d < (u32)BINS ? hw[d] : 0u;
       __syncwarp();
-      if (d < 256u && (peers & lt) == 0) whist[w][d] = old + __popc(peers);
+      if (d < (u32)BINS && (peers & lt) == 0) hw[d] = old + __popc(peers);
       __syncwarp();
-      rank[j] = d < 256u ? ((d << 16) | (old + __popc(peers & lt))) : NONE;
+      rank[j] = d < (u32)BINS ? ((d << 16) | (old + __popc(peers & lt))) : NONE;
     }
     __syncthreads();
-    // per digit (thread t): prefix over warps, tile total; tile-local exclusive scan of the totals
-    u32 total = 0;
+    // per digit: prefix over warps, tile total; thread t owns digits [t*DPT, t*DPT + DPT)
+    u32 tsum = 0, dtot[DPT];
 #pragma unroll
-    for (int ww = 0; ww < RS_WARPS; ++ww) {
-      const u32 c = whist[ww][t];
-      whist[ww][t] = total;
-      total += c;
+    for (int q = 0; q < DPT; ++q) {
+      const int d = t * DPT + q;
+      u32 total = 0;
+#pragma unroll
+      for (int ww = 0; ww < RS_WARPS; ++ww) {
+        const u32 c = whist[ww * BINS + d];
+        whist[ww * BINS + d] = total;
+        total += c;
+      }
+      dtot[q] = total;
+      tsum += total;
     }
     {
-      const u32 x = warp_incl_sum(total);
+      const u32 x = warp_incl_sum(tsum);
       if (l == 31) wsum[w] = x;
       __syncthreads();
       u32 off = 0;
       for (int ww = 0; ww < w; ++ww) off += wsum[ww];
-      tofs[t] = off + x - total;
-      if (t == RS_BINS - 1) *s_kept = off + x;
+      u32 run = off + x - tsum;
+#pragma unroll
+      for (int q = 0; q < DPT; ++q) {
+        tofs[t * DPT + q] = run;
+        run += dtot[q];
+      }
+      if (t == RS_THREADS - 1) *s_kept = run;
     }
     __syncthreads();
 #pragma unroll
     for (int j = 0; j < RS_ITEMS; ++j) {
       if (rank[j] != NONE) {
         const u32 d = rank[j] >> 16;
-        skeys[tofs[d] + whist[w][d] + (rank[j] & 0xFFFFu)] = sk[w * (RS_ITEMS * 32) + j * 32 + l];
+        skeys[tofs[d] + whist[w * BINS + d] + (rank[j] & 0xFFFFu)] = sk[w * (RS_ITEMS * 32) + j * 32 + l];
       }
     }
     __syncthreads();
     const u32 tile_n = *s_kept;
     for (u32 q = t; q < tile_n; q += RS_THREADS) {
       const u32 kk = skeys[q];
-      const u32 d = (kk >> shift) & 0xFFu;
+      const u32 d = (kk >> shift) & (BINS - 1);
       kout[(u64)gstart[d] + (q - tofs[d])] = kk;
     }
     if (vout) {
-      // values: the same permutation, staged in the stage's (now consumed) key half
+      // values: the same permutation, staged in the (consumed) key stage
 #pragma unroll
       for (int j = 0; j < RS_ITEMS; ++j) {
         if (rank[j] != NONE) {
           const u32 d = rank[j] >> 16;
-          sk[tofs[d] + whist[w][d] + (rank[j] & 0xFFFFu)] = sv[w * (RS_ITEMS * 32) + j * 32 + l];
+          sk[tofs[d] + whist[w * BINS + d] + (rank[j] & 0xFFFFu)] = v[j];
         }
       }
       __syncthreads();
       for (u32 q = t; q < tile_n; q += RS_THREADS) {
-        const u32 d = (skeys[q] >> shift) & 0xFFu;
+        const u32 d = (skeys[q] >> shift) & (BINS - 1);
         vout[(u64)gstart[d] + (q - tofs[d])] = sk[q];
       }
     }
@@ -366,6 +393,35 @@ __global__ void __launch_bounds__(1024) k_scan_tiles(u64* __restrict__ tsum, u64
   if (t == 0 && total_out) *total_out = s_carry;
 }
 
+// small inputs: one CTA scans the whole array in chunks of 1024 with a running carry (one launch)
+constexpr u64 SC_SMALL = 8192;
+__global__ void __launch_bounds__(1024) k_scan_small(const u32* __restrict__ in, u32* __restrict__ out, u64 n,
+                                                     u64* __restrict__ total_out) {
+  __shared__ u64 wsum[32];
+  __shared__ u64 s_carry;
+  const int t = threadIdx.x, w = t >> 5, l = t & 31;
+  if (t == 0) s_carry = 0;
+  __syncthreads();
+  for (u64 c0 = 0; c0 < n; c0 += 1024) {
+    const u64 i = c0 + t;
+    const u64 v = i < n ? in[i] : 0u;
+    const u64 x = warp_incl_sum(v);
+    if (l == 31) wsum[w] = x;
+    __syncthreads();
+    u64 off = 0, tot = 0;
+    for (int ww = 0; ww < 32; ++ww) {
+      if (ww < w) off += wsum[ww];
+      tot += wsum[ww];
+    }
+    const u64 carry = s_carry;
+    if (i < n) out[i] = (u32)(carry + off + x - v);
+    __syncthreads();
+    if (t == 0) s_carry = carry + tot;
+    __syncthreads();
+  }
+  if (t == 0 && total_out) *total_out = s_carry;
+}
+
 __global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__ in, u32* __restrict__ out, u64 n,
                                                          const u64* __restrict__ texcl) {
   __shared__ u64 wsum[SC_THREADS / 32];
@@ -398,15 +454,110 @@ size_t scan_temp_bytes(u64 n);
 size_t rs_temp_bytes(u64 n) {
   const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
   // histograms + bases, then the (digit, tile) count / offset table of one pass
-  return RS_HDR_BYTES + (size_t)(tiles ? tiles : 1) * RS_BINS * sizeof(u32) + 256;
+  return RS_HDR_BYTES + (size_t)(tiles ? tiles : 1) * RS_MAXB * sizeof(u32) + 256;
+}
+
+// Small sorts (n <= RS_SMALL, e.g. the K3 sync-skeleton tables, K1 of small traces): one CTA sorts
+// (digit << 32 | input index) composites with a bitonic network in shared memory -- the index makes
+// the order stable -- and gathers keys / values into the alternate buffers: one launch instead of a
+// histogram, a bins scan and three kernels per digit pass.
+constexpr u32 RS_SMALL = 8192;
+__global__ void __launch_bounds__(1024) k_sort_small(const u32* __restrict__ kin, const u32* __restrict__ vin,
+                                                     u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
+                                                     const u64* __restrict__ n_dev, int drop, int bit_lo, int bits,
+                                                     u64* __restrict__ n_out) {
+  extern __shared__ __align__(16) unsigned long long cs[];
+  __shared__ u32 s_kept;
+  const u32 t = threadIdx.x;
+  const u32 n = (u32)(n_dev ? *n_dev : n_max);
+  if (t == 0) s_kept = 0;
+  u32 P = 1;
+  while (P < n) P <<= 1;
+  const u32 dmask = bits >= 32 ? 0xFFFFFFFFu : ((1u << bits) - 1u);
+  __syncthreads();
+  u32 kept = 0;
+  for (u32 i = t; i < P; i += 1024) {
+    unsigned long long v = ~0ull;
+    if (i < n) {
+      const u32 k = kin[i];
+      if (!(drop && k == KEY_DROP)) {
+        v = ((unsigned long long)((k >> bit_lo) & dmask) << 32) | i;
+        ++kept;
+      }
+    }
+    cs[i] = v;
+  }
+  atomicAdd(&s_kept, kept);
+  __syncthreads();
+  for (u32 k = 2; k <= P; k <<= 1) {
+    for (u32 j = k >> 1; j > 0; j >>= 1) {
+      for (u32 i = t; i < P; i += 1024) {
+        const u32 ij = i ^ j;
+        if (ij > i) {
+          const unsigned long long a = cs[i], b = cs[ij];
+          if (((i & k) == 0) == (a > b)) {
+            cs[i] = b;
+            cs[ij] = a;
+          }
+        }
+      }
+      __syncthreads();
+    }
+  }
+  const u32 nk = s_kept;
+  for (u32 i = t; i < nk; i += 1024) {
+    const u32 src = (u32)(cs[i] & 0xFFFFFFFFull);
+    kout[i] = kin[src];
+    if (vout) vout[i] = vin[src];
+  }
+  if (t == 0 && n_out) *n_out = nk;
+}
+
+template <int RB>
+static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo, int passes, void* temp,
+                       cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop) {
+  constexpr int BINS = 1 << RB;
+  const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
+  u32* ghist = (u32*)temp;                           // [RS_MAXP][RS_MAXB]
+  u32* gbase = ghist + RS_MAXP * RS_MAXB;            // [RS_MAXP][RS_MAXB]
+  u32* counts = (u32*)((char*)temp + RS_HDR_BYTES);  // [BINS][tiles]
+  cudaMemsetAsync(ghist, 0, RS_MAXP * RS_MAXB * sizeof(u32), st);
+  static int sms = 0, down_grid = 0;
+  constexpr size_t dsmem = rs_dsmem<RB>();
+  if (!down_grid) {
+    int dev = 0, per = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaFuncSetAttribute(k_rs_down<RB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_rs_down<RB>, RS_THREADS, dsmem);
+    down_grid = sms * (per > 0 ? per : 1);
+  }
+  const unsigned hgrid =
+      (unsigned)std::min<u64>((n + RS_THREADS * RS_HIST_ITEMS - 1) / (RS_THREADS * RS_HIST_ITEMS), (u64)sms * 8);
+  k_rs_hist<RB><<<hgrid, RS_THREADS, 0, st>>>(ki, n, n_dev, drop ? 1 : 0, bit_lo, passes, ghist); ++g_launches;
+  k_rs_bins<RB><<<passes, BINS, 0, st>>>(ghist, gbase, drop ? n_out_dev : nullptr); ++g_launches;
+  const u64* nd = n_dev;
+  for (int p = 0; p < passes; ++p) {
+    const int shift = bit_lo + RB * p;
+    const int dr = (drop && p == 0) ? 1 : 0;
+    k_rs_up<RB><<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles); ++g_launches;
+    k_rs_rows<<<BINS, RS_THREADS, 0, st>>>(counts, tiles, gbase + p * RS_MAXB); ++g_launches;
+    k_rs_down<RB><<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, dsmem, st>>>(ki, vi, ko, vo, n, nd, dr,
+                                                                                              shift, counts, tiles);
+    ++g_launches;
+    if (dr) nd = n_out_dev;
+    u32* tk = ki; ki = ko; ko = tk;
+    u32* tv = vi; vi = vo; vo = tv;
+  }
 }
 
 // Stable sort of (keys, vals) by key bits [bit_lo, bit_hi) (vals may be null: keys only).  Result is
 // in (keys, vals) when the function returns false, else in (keys_alt, vals_alt).  n is the (upper
 // bound of the) item count; with n_dev the exact count is read on the device.  drop: the first pass
 // removes items whose key is KEY_DROP and writes the number kept to *n_out_dev (at least one pass
-// is run).  Per pass: k_rs_up (digit counts per tile) -> k_rs_rows (256 independent row scans) ->
-// k_rs_down (rank + scatter); one k_rs_hist read up front gives every pass's digit bases.
+// is run).  Digit width: the fewest passes of at most 10 bits, each pass 8, 9 or 10 bits wide.  Per
+// pass: k_rs_up (digit counts per tile) -> k_rs_rows (independent per-digit row scans) -> k_rs_down
+// (rank + scatter); one k_rs_hist read up front gives every pass's digit bases.
 bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi, void* temp,
                       cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop) {
   if (!drop && (n <= 1 || bit_hi <= bit_lo)) return false;
@@ -414,42 +565,26 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
     if (n_out_dev) cudaMemsetAsync(n_out_dev, 0, 8, st);
     return false;
   }
-  int passes = (bit_hi - bit_lo + 7) / 8;
-  if (passes > RS_MAXP) passes = RS_MAXP;
-  if (passes < 1) passes = 1;
-  const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
-  u32* ghist = (u32*)temp;                           // [RS_MAXP][256]
-  u32* gbase = ghist + RS_MAXP * RS_BINS;            // [RS_MAXP][256]
-  u32* counts = (u32*)((char*)temp + RS_HDR_BYTES);  // [256][tiles]
-  cudaMemsetAsync(ghist, 0, RS_MAXP * RS_BINS * sizeof(u32), st);
-  int dev = 0, sms = 148;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  static int down_grid = 0;
-  if (!down_grid) {
-    int per = 1;
-    cudaFuncSetAttribute(k_rs_down, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)RS_DSMEM);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_rs_down, RS_THREADS, RS_DSMEM);
-    down_grid = sms * (per > 0 ? per : 1);
-  }
-  const unsigned hgrid =
-      (unsigned)std::min<u64>((n + RS_THREADS * RS_HIST_ITEMS - 1) / (RS_THREADS * RS_HIST_ITEMS), (u64)sms * 8);
-  k_rs_hist<<<hgrid, RS_THREADS, 0, st>>>(keys, n, n_dev, drop ? 1 : 0, bit_lo, passes, ghist); ++g_launches;
-  k_rs_bins<<<passes, RS_BINS, 0, st>>>(ghist, gbase, drop ? n_out_dev : nullptr); ++g_launches;
-  u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
-  const u64* nd = n_dev;
-  for (int p = 0; p < passes; ++p) {
-    const int shift = bit_lo + 8 * p;
-    const int dr = (drop && p == 0) ? 1 : 0;
-    k_rs_up<<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles); ++g_launches;
-    k_rs_rows<<<RS_BINS, RS_THREADS, 0, st>>>(counts, tiles, gbase + p * RS_BINS); ++g_launches;
-    k_rs_down<<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, RS_DSMEM, st>>>(ki, vi, ko, vo, n, nd, dr,
-                                                                                           shift, counts, tiles);
+  const int bits = std::max(bit_hi - bit_lo, 1);
+  if (n <= RS_SMALL) {
+    static bool attr = false;
+    if (!attr) {
+      cudaFuncSetAttribute(k_sort_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(RS_SMALL * 8));
+      attr = true;
+    }
+    u32 P = 1;
+    while (P < n) P <<= 1;
+    k_sort_small<<<1, 1024, P * 8, st>>>(keys, vals, keys_alt, vals_alt, n, n_dev, drop ? 1 : 0, bit_lo, bits,
+                                         drop ? n_out_dev : nullptr);
     ++g_launches;
-    if (dr) nd = n_out_dev;
-    u32* tk = ki; ki = ko; ko = tk;
-    u32* tv = vi; vi = vo; vo = tv;
+    return true;
   }
+  int passes = std::min((bits + 9) / 10, RS_MAXP);
+  const int rb = std::max(8, std::min(10, (bits + passes - 1) / passes));
+  u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
+  if (rb == 8) rs_sort_rb<8>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
+  else if (rb == 9) rs_sort_rb<9>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
+  else rs_sort_rb<10>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
   return (passes & 1) != 0;
 }
 
@@ -461,6 +596,10 @@ void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_d
   u64* tsum = (u64*)temp;
   if (tiles == 0) {
     if (total_dev) cudaMemsetAsync(total_dev, 0, 8, st);
+    return;
+  }
+  if (n <= SC_SMALL) {
+    k_scan_small<<<1, 1024, 0, st>>>(in, out, n, total_dev); ++g_launches;
     return;
   }
   k_scan_tsum<<<(unsigned)tiles, SC_THREADS, 0, st>>>(in, n, tsum); ++g_launches;
