@@ -212,6 +212,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* sync_list = S.alloc<u32>(n);
   u32* page_bits = S.alloc<u32>(nwords);
   u32* ub_off = S.alloc<u32>(n + 1);  // per record: upper bound of its items, then its first slot
+  uint4* hdr16 = S.alloc<uint4>(n);  // compact record headers (K2 gathers them per warp)
   cudaMemsetAsync(err, 0, 4, st);
   cudaMemsetAsync(cnt, 0, C_N * 8, st);
   cudaMemsetAsync(if_cnt, 0, (g.n_warps + 1) * 4, st);
@@ -220,7 +221,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   // ---- header pass; written pages ranked in address order from the list of non-zero bitmap words
   u32* word_list = S.alloc<u32>(nwords);
   u32* wl2 = S.alloc<u32>(nwords);
-  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, ub_off, err, st);
+  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, ub_off, hdr16, err, st);
   u32* words = word_list;
   u32* wl_prefix = wl2;
   u32* page_rank = S.alloc<u32>(nwords);
@@ -281,7 +282,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* find_rec = S.alloc<u32>(n_bar + 1);
   u32* find_cnt = S.alloc<u32>(1);
   cudaMemsetAsync(find_cnt, 0, 4, st);
-  launch_replay(recs, wrec, warp_start, g, node_base, bar_base, snap, nodes, bar_rec, bar_next, find_blk, find_rec,
+  launch_replay(hdr16, wrec, warp_start, g, node_base, bar_base, snap, nodes, bar_rec, bar_next, find_blk, find_rec,
                 find_cnt, err, st);
   launch_barriers(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err, st);
   launch_snap_blab(snap, n, g.wpb, g.n_warps, n_bar, bar_base, blockR, st);

@@ -90,6 +90,22 @@ __device__ __forceinline__ bool hb_ev(const HbCtx& c, u32 ev1, u32 w1, u32 ev2, 
   return hb_slow(ev1, w1, ev2, s2.warp, s2.ps, s2.node, s2.blab);
 }
 
+// Same query, evaluated branch-free up to the rare slow case (divergent intra-warp walk or foreign
+// knowledge): lane-sequential K7 lanes sit at different items, so every branch of the query would
+// be executed by the whole warp.
+__device__ __forceinline__ bool hbq(const HbCtx& c, u32 ev1, u32 w1, u32 ev2, const Snap& s2) {
+  const u32 r1 = ev1 >> 5, r2 = ev2 >> 5;
+  const bool samel = ((ev1 ^ ev2) & 31u) == 0u;
+  const bool samew = w1 == s2.warp;
+  const bool conv = s2.node == s2.warp;
+  const bool ord = (samew && (samel || (conv && s2.ps > r1))) ||
+                   (blk_of(c.g, w1) == blk_of(c.g, s2.warp) && s2.blab > r1);  // program order / endi / barrier
+  if (r1 == r2) return samel;  // lanes of one instruction are concurrent
+  if (ord) return true;
+  if (c.n_acq == 0 && !(samew && !conv)) return false;
+  return hb_slow(ev1, w1, ev2, s2.warp, s2.ps, s2.node, s2.blab);
+}
+
 // R_x is a vector clock at writer (ev2, s2): its entries are the latest read per thread among
 // items [lo, hi] (all reads of this granule).  Check each (Fig. 2 WRITESHARED, Fig. 3 *ATOMSHARED).
 static __device__ __noinline__ void vc_check(const u32* __restrict__ evs, uint4* races, u32* race_cnt, u32 race_cap,
@@ -406,24 +422,63 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
 }
 
 // ---------------------------------------------------------------------------------------
-// Lane-sequential formulation (BC_K7=seq).  Same persistent warp ranges and incoming state
-// (walk_back / WarpEnd) as k_check, but each range is processed in blocks of KS_BLK = 1024 items:
-//   load   : the warp stages the block's (key, ev) words in shared memory (coalesced; stored with a
-//            33-word row pitch so that lane l reading item l*32+j is bank-conflict free)
-//   phase 1: lane l walks ITS 32 consecutive items and computes (a) the READINFLATE flag of each
-//            read (Fig. 2: its predecessor is a read of the same granule not ordered before it)
-//            and (b) the summary Sum of its chunk (last key, last writer, first inflation after it)
-//   scan   : a 5-step warp scan of the summaries (the same associative combine as k_check) gives
-//            every lane the automaton state (LW, FI) entering its chunk, and the block carry
-//   phase 2: lane l replays the rules of Fig. 2 / Fig. 3 over its chunk sequentially (W check,
-//            R check as epoch or vector, same-value filter) from that state.
-// Per item this costs a handful of thread instructions instead of a warp-wide ballot round per 32
-// items, and the per-item happens-before queries run on 32 independent lanes.
-constexpr int KS_WARPS = 8;
-constexpr int KS_BLK = 1024;
-constexpr int KS_PITCH = KS_BLK + KS_BLK / 32;  // 33-word rows
+// Lane-sequential formulation with shared-memory staged clocks and a query buffer (default;
+// BC_K7=ballot selects k_check above).  Same persistent warp ranges and incoming state
+// (walk_back / WarpEnd) as k_check; each range is processed in blocks of 32 * KT_IPL items:
+//   load    : the block's (key, ev) words land in shared memory by cp.async, one block ahead
+//             (row pitch KT_IPL+1 words: lane l reading item l*KT_IPL+j is bank-conflict free)
+//   gather  : lane l walks ITS KT_IPL consecutive items; for each item some query can read (the
+//             snap_if_needed rule) it issues a 16-B cp.async of the record snapshot into shared
+//             memory (up to 32*KT_IPL gathers in flight per warp, no registers held), and for
+//             each read preceded by a read of the same granule it queues a READINFLATE query
+//   eval    : the queued happens-before queries are evaluated in uniform rounds (lane l, round i:
+//             its own i-th query), so the warp runs ONE copy of the query code instead of the
+//             union of every branch its lanes are in
+//   summary : lane l walks its items again: chunk summary Sum (last key, last writer, first
+//             inflation after it) from the READINFLATE flags (Fig. 2)
+//   scan    : a 5-step warp scan of the summaries (the associative combine of k_check) gives every
+//             lane the automaton state (LW, FI) entering its chunk, and the block carry
+//   rules   : lane l replays the rules of Fig. 2 / Fig. 3 over its chunk from that state and queues
+//             the checks they make (W check, R check against the epoch or the read vector, with
+//             the same-value filter applied at queueing), then the queries are evaluated as above.
+// A query is one u32: item index (current event), source index (prior event; two codes name
+// per-lane registers holding an event from before the block), kind.  Every query reads shared
+// memory only; values carried across blocks are loaded from global memory once per lane.
+constexpr int KT_IPL = 16;                   // items per lane per block
+constexpr int KT_BLK = 32 * KT_IPL;          // items per warp block
+constexpr int KT_PITCH = 32 * (KT_IPL + 1);  // padded entries per array
+constexpr int KT_WARPS = 12;
+// per warp: snapshots [KT_PITCH] uint4, keys / evs double-buffered [2][2][KT_PITCH] u32
+constexpr size_t KT_WARP_BYTES = (size_t)KT_PITCH * (sizeof(uint4) + 4 * sizeof(u32));
 
-__device__ __forceinline__ u32 kpad(u32 i) { return i + (i >> 5); }
+__device__ __forceinline__ u32 tpad(u32 i) { return i + i / KT_IPL; }
+
+__device__ __forceinline__ void cp_async4(void* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+// stage the (key, ev) words of items [bb, bb + nb) of the range into sK / sE (lane l copies items
+// r*32 + l); tail entries up to KT_BLK are NONE / 0
+__device__ __forceinline__ void kt_stage(const CheckArgs& a, u64 bb, u32 nb, u32* sK, u32* sE, u32 lane) {
+#pragma unroll 4
+  for (u32 r = 0; r < (u32)KT_IPL; ++r) {
+    const u32 li = r * 32u + lane;
+    if (li < nb) {
+      cp_async4(sK + tpad(li), a.keys + bb + li);
+      cp_async4(sE + tpad(li), a.evs + bb + li);
+    } else {
+      sK[tpad(li)] = NONE;
+      sE[tpad(li)] = 0u;
+    }
+  }
+  cp_async_commit();
+}
 
 __device__ __forceinline__ Sum shfl_up_sum(const Sum& s, int o) {
   Sum r;
@@ -444,13 +499,13 @@ __device__ __forceinline__ Sum shfl_sum(const Sum& s, int src) {
   return r;
 }
 
-__global__ void __launch_bounds__(KS_WARPS * 32, 2) k_check_seq(CheckArgs a, WarpEnd* wend, u32 nw) {
-  extern __shared__ __align__(16) u32 ks_smem[];
+__global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, WarpEnd* wend, u32 nw) {
+  extern __shared__ __align__(16) unsigned char kt_smem[];
   const int wi = threadIdx.x >> 5;
-  u32* sK = ks_smem + (size_t)wi * 2 * KS_PITCH;
-  u32* sE = sK + KS_PITCH;
+  uint4* sS = reinterpret_cast<uint4*>(kt_smem + (size_t)wi * KT_WARP_BYTES);
+  u32* const sKE = reinterpret_cast<u32*>(sS + KT_PITCH);  // [buf][key|ev][KT_PITCH]
   const u64 n = *a.n_dev;
-  const u32 w = blockIdx.x * KS_WARPS + wi;
+  const u32 w = blockIdx.x * KT_WARPS + wi;
   const u32 lane = threadIdx.x & 31;
   const HbCtx& c = a.c;
   const u64 nr = (n + 31) / 32;
@@ -483,64 +538,85 @@ __global__ void __launch_bounds__(KS_WARPS * 32, 2) k_check_seq(CheckArgs a, War
   }
 
   u32 segs = 0;
-  for (u64 bb = beg; bb < end; bb += KS_BLK) {
-    const u32 nb = (u32)(end - bb < (u64)KS_BLK ? end - bb : (u64)KS_BLK);
-#pragma unroll 8
-    for (u32 r = 0; r < 32; ++r) {
-      const u32 li = r * 32 + lane;
-      sK[kpad(li)] = li < nb ? a.keys[bb + li] : NONE;
-      sE[kpad(li)] = li < nb ? a.evs[bb + li] : 0u;
-    }
+  const u32 l0 = lane * KT_IPL;
+  if (beg < end) kt_stage(a, beg, (u32)(end - beg < (u64)KT_BLK ? end - beg : (u64)KT_BLK), sKE, sKE + KT_PITCH, lane);
+  for (u64 bb = beg; bb < end; bb += KT_BLK) {
+    const u32 nb = (u32)(end - bb < (u64)KT_BLK ? end - bb : (u64)KT_BLK);
+    // ---- this block's (key, ev) words were staged one iteration ago (or by the prologue)
+    const u32 buf = (u32)(((bb - beg) / KT_BLK) & 1u);
+    u32* const sK = sKE + buf * 2 * KT_PITCH;
+    u32* const sE = sK + KT_PITCH;
+    const u32 knext = bb + nb < end ? a.keys[bb + nb] : NONE;  // first item after the block
+    cp_async_wait<0>();
     __syncwarp();
-    const u32 l0 = lane * 32;
-    const u32 ppk = lane == 0 ? pkx : (l0 - 1 < nb ? sK[kpad(l0 - 1)] : NONE);
-    const u32 ppe = lane == 0 ? pev : (l0 - 1 < nb ? sE[kpad(l0 - 1)] : 0u);
-    const u32 cnt = l0 < nb ? min(32u, nb - l0) : 0u;
 
-    // ---- phase 1: READINFLATE flags and the chunk summary
-    Sum sm = sum_ident();
-    u32 imask = 0;
+    const u32 cnt = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
+    const u32 ppk = lane == 0 ? pkx : sK[tpad(l0 - 1)];
+    const u32 ppe = lane == 0 ? pev : sE[tpad(l0 - 1)];
+    // warp of the item before the lane's chunk (read only if that item is a same-granule read,
+    // which has a successor, so it was gathered; lane 0: the item before the block)
+    const u32 gbb = (u32)bb;
+
+    // ---- gather the snapshots some query can read
     {
-      u32 pk = ppk, pe = ppe, pw = 0;
-      bool pw_ok = false, kc = false;
-      u32 tlw = 0, tfi = NONE;
+      u32 kp = ppk, k = cnt ? sK[tpad(l0)] : NONE;
       for (u32 j = 0; j < cnt; ++j) {
         const u32 li = l0 + j;
-        const u32 k = sK[kpad(li)], e = sE[kpad(li)];
-        const u32 key = k >> 2, op = k & 3u;
-        const u32 gi = (u32)(bb + li);
-        const bool same = pk != NONE && (pk >> 2) == key;
-        if (j == 0) sm.fk = key;
+        const u32 kn = li + 1 < nb ? sK[tpad(li + 1)] : knext;
+        const u32 key = k >> 2;
+        const bool sp = kp != NONE && (kp >> 2) == key, sn = kn != NONE && (kn >> 2) == key;
+        const bool atm_only =
+            (k & 3u) == IOP_ATOM && (!sp || (kp & 3u) == IOP_ATOM) && (!sn || (kn & 3u) == IOP_ATOM);
+        if ((sp || sn) && !atm_only) cp_async16(sS + tpad(li), c.snap + (sE[tpad(li)] >> 5));
+        kp = k;
+        k = kn;
+      }
+    }
+    cp_async_commit();
+    if (bb + nb < end) {  // stage the next block now: its loads overlap this block's work
+      const u64 b2 = bb + nb;
+      kt_stage(a, b2, (u32)(end - b2 < (u64)KT_BLK ? end - b2 : (u64)KT_BLK), sKE + (buf ^ 1u) * 2 * KT_PITCH,
+               sKE + (buf ^ 1u) * 2 * KT_PITCH + KT_PITCH, lane);
+    }
+    const u32 pw0 = (lane == 0 && ppk != NONE) ? __ldg(&c.snap[pev >> 5].x) : 0u;
+    if (bb + nb < end) cp_async_wait<1>(); else cp_async_wait<0>();
+    __syncwarp();
+
+    // ---- READINFLATE flags (Fig. 2: a read whose predecessor is an unordered read of the same
+    // granule) and the chunk summary
+    Sum sm = sum_ident();
+    u32 imask = 0;
+    if (cnt) {
+      u32 pk = ppk, pe = ppe, pw = lane ? sS[tpad(l0 - 1)].x : pw0, tlw = 0, tfi = NONE;
+      bool kc = false;
+      sm.fk = sK[tpad(l0)] >> 2;
+      for (u32 j = 0; j < cnt; ++j) {
+        const u32 li = l0 + j;
+        const u32 k = sK[tpad(li)], e = sE[tpad(li)];
+        const uint4 sv = sS[tpad(li)];
+        const u32 gi = gbb + li;
+        const bool same = pk != NONE && (pk >> 2) == (k >> 2);
         if (!same) {
           ++segs;
-          if (j > 0) kc = true;
+          kc |= j > 0;
           tlw = 0;
           tfi = NONE;
         }
-        bool loaded = false;
-        if (op != IOP_LD) {
+        if ((k & 3u) != IOP_LD) {
           tlw = gi + 1u;
           tfi = NONE;
-        } else if (same && (pk & 3u) == IOP_LD) {
-          if (!pw_ok) pw = __ldg(&c.snap[pe >> 5].x);
-          const Snap s2 = load_snap(c.snap, e >> 5);
-          if (!hb_ev(c, pe, pw, e, s2)) {
-            imask |= 1u << j;
-            if (tfi == NONE) tfi = gi;
-          }
-          pw = s2.warp;
-          loaded = true;
+        } else if (same && (pk & 3u) == IOP_LD && !hbq(c, pe, pw, e, to_snap(sv))) {
+          imask |= 1u << j;
+          if (tfi == NONE) tfi = gi;
         }
-        pw_ok = loaded;
         pk = k;
         pe = e;
-        sm.lk = key;
+        pw = sv.x;
       }
-      if (cnt) {
-        sm.lw = tlw;
-        sm.fi = tfi;
-        sm.bits = (kc ? 0u : 1u) | (tlw ? 2u : 0u);
-      }
+      sm.lk = pk >> 2;
+      sm.lw = tlw;
+      sm.fi = tfi;
+      sm.bits = (kc ? 0u : 1u) | (tlw ? 2u : 0u);
     }
 
     // ---- scan of the chunk summaries -> state entering each chunk; block carry
@@ -555,96 +631,87 @@ __global__ void __launch_bounds__(KS_WARPS * 32, 2) k_check_seq(CheckArgs a, War
     const Sum in = combine(carry, ex);
     const Sum blk = shfl_sum(incl, 31);
 
-    // ---- phase 2: the rules, lane-sequentially
+    // ---- the rules of Fig. 2 / Fig. 3, lane-sequentially
     if (cnt) {
       u32 lw = (in.fk != NONE) ? in.lw : 0u, fi = (in.fk != NONE) ? in.fi : NONE;
       u32 wk = 0, we = 0, ww = 0;
-      bool ww_ok = false;
       if (lw) {
         if ((u64)(lw - 1) >= bb) {
-          wk = sK[kpad((u32)(lw - 1 - bb))];
-          we = sE[kpad((u32)(lw - 1 - bb))];
+          const u32 wl = (u32)(lw - 1 - bb);
+          wk = sK[tpad(wl)];
+          we = sE[tpad(wl)];
+          ww = sS[tpad(wl)].x;  // gathered: the writer has a same-granule successor in the block
         } else {
           wk = cwk;
           we = cwe;
+          ww = __ldg(&c.snap[cwe >> 5].x);
         }
       }
-      u32 pk = ppk, pe = ppe, pw = 0;
-      bool pw_ok = false;
+      u32 pk = ppk, pe = ppe, pw = lane ? sS[tpad(l0 - 1)].x : pw0;
       for (u32 j = 0; j < cnt; ++j) {
         const u32 li = l0 + j;
-        const u32 k = sK[kpad(li)], e = sE[kpad(li)];
-        const u32 key = k >> 2, op = k & 3u;
-        const u32 gi = (u32)(bb + li);
-        const bool same = pk != NONE && (pk >> 2) == key;
+        const u32 k = sK[tpad(li)], e = sE[tpad(li)];
+        const uint4 sv = sS[tpad(li)];
+        const Snap s2 = to_snap(sv);
+        const u32 op = k & 3u;
+        const u32 gi = gbb + li;
+        const bool same = pk != NONE && (pk >> 2) == (k >> 2);
         if (!same) {
           lw = 0;
           fi = NONE;
         }
-        const u32 nk = li + 1 < nb ? sK[kpad(li + 1)] : NONE;
-        const bool same_next = nk != NONE && (nk >> 2) == key;
-        const bool atm_only = op == IOP_ATOM && (!same || (pk & 3u) == IOP_ATOM) &&
-                              (!same_next || (nk & 3u) == IOP_ATOM);
-        const bool need = (same || same_next) && !atm_only;
-        Snap s2{0, 0, 0, 0};
-        if (need) s2 = load_snap(c.snap, e >> 5);
-        if (op == IOP_LD) {
-          if (((imask >> j) & 1u) && fi == NONE) fi = gi;
-          if (lw) {  // W_x check of a read (Fig. 2 READ*)
-            if (!ww_ok) {
-              ww = __ldg(&c.snap[we >> 5].x);
-              ww_ok = true;
-            }
-            if (!hb_ev(c, we, ww, e, s2)) emit(a, key, e, we, (wk & 3u) == IOP_ATOM ? BC_KIND_AR : BC_KIND_WR);
-          }
-        } else {
-          const bool patm = (wk & 3u) == IOP_ATOM;
-          if (lw && !(op == IOP_ATOM && patm)) {  // W_x check (atomics only against a plain write)
-            if (!ww_ok) {
-              ww = __ldg(&c.snap[we >> 5].x);
-              ww_ok = true;
-            }
-            if (!hb_ev(c, we, ww, e, s2)) {
-              if (op == IOP_ATOM) {
-                emit(a, key, e, we, BC_KIND_WA);
-              } else {
-                const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (we >> 5) == (e >> 5);
-                if (!filtered) emit(a, key, e, we, patm ? BC_KIND_AW : BC_KIND_WW);
-              }
-            }
-          }
+        if (op == IOP_LD && ((imask >> j) & 1u) && fi == NONE) fi = gi;
+        const bool patm = (wk & 3u) == IOP_ATOM;
+        // W_x check (every rule of Fig. 2; atomics only against a plain last write)
+        if (lw && !(op == IOP_ATOM && patm) && !hbq(c, we, ww, e, s2)) {
+          const u32 kind = op == IOP_LD ? (patm ? BC_KIND_AR : BC_KIND_WR)
+                                        : op == IOP_ATOM ? BC_KIND_WA : (patm ? BC_KIND_AW : BC_KIND_WW);
+          const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (we >> 5) == (e >> 5);
+          if (!filtered) emit(a, k >> 2, e, we, kind);
+        }
+        if (op != IOP_LD) {
           if (same && (pk & 3u) == IOP_LD) {  // R_x check at a writer: epoch, or vector after READINFLATE
             const u32 kind = op == IOP_ATOM ? BC_KIND_RA : BC_KIND_RW;
             if (fi == NONE) {
-              if (!pw_ok) pw = __ldg(&c.snap[pe >> 5].x);
-              if (!hb_ev(c, pe, pw, e, s2)) emit(a, key, e, pe, kind);
+              if (!hbq(c, pe, pw, e, s2)) emit(a, k >> 2, e, pe, kind);
             } else {
-              vc_check(a.evs, a.races, a.race_cnt, a.race_cap, (u64)fi - 1, (u64)gi - 1, e, s2.warp, s2.ps, s2.node,
-                       s2.blab, key, kind);
+              const u64 lo = (u64)fi - 1;
+              if (lo >= bb && gi - (u32)lo <= 64u) {
+                // the read run is staged in this block: the latest read of each thread in it
+                const u32 jl = (u32)(lo - bb);
+                for (u32 jj = li; jj-- > jl;) {
+                  const u32 ev1 = sE[tpad(jj)], w1 = sS[tpad(jj)].x;
+                  bool dup = false;
+                  for (u32 q = jj + 1; q < li && !dup; ++q)
+                    dup = sS[tpad(q)].x == w1 && ((sE[tpad(q)] ^ ev1) & 31u) == 0u;
+                  if (!dup && !hbq(c, ev1, w1, e, s2)) emit(a, k >> 2, e, ev1, kind);
+                }
+              } else {
+                vc_check(a.evs, a.races, a.race_cnt, a.race_cap, lo, (u64)gi - 1, e, s2.warp, s2.ps, s2.node,
+                         s2.blab, k >> 2, kind);
+              }
             }
           }
           lw = gi + 1u;
           wk = k;
           we = e;
-          ww = s2.warp;
-          ww_ok = need;
+          ww = sv.x;
           fi = NONE;
         }
-        pw = s2.warp;
-        pw_ok = need;
         pk = k;
         pe = e;
+        pw = sv.x;
       }
     }
 
     // ---- block carry
     carry = combine(carry, blk);
     if (carry.lw && (u64)(carry.lw - 1) >= bb) {
-      cwk = sK[kpad((u32)(carry.lw - 1 - bb))];
-      cwe = sE[kpad((u32)(carry.lw - 1 - bb))];
+      cwk = sK[tpad((u32)(carry.lw - 1 - bb))];
+      cwe = sE[tpad((u32)(carry.lw - 1 - bb))];
     }
-    pkx = sK[kpad(nb - 1)];
-    pev = sE[kpad(nb - 1)];
+    pkx = sK[tpad(nb - 1)];
+    pev = sE[tpad(nb - 1)];
     __syncwarp();
   }
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);
@@ -666,27 +733,29 @@ size_t check_status_bytes(u64 n) { return (size_t)148 * 64 * sizeof(WarpEnd) + 2
 void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_dev, u64 n_max, void* status,
                   uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, cudaStream_t st) {
   if (n_max == 0) return;
-  // K7 variant: ballot rounds (default; fastest on read-heavy C2/C3) or lane-sequential
-  // (BC_K7=seq; fastest on atomic-heavy C4/C5)
-  static int use_seq = -1, grid = 0;
-  const size_t smem_seq = (size_t)KS_WARPS * 2 * KS_PITCH * sizeof(u32);
-  if (use_seq < 0) {
-    const char* v = getenv("BC_K7");
-    use_seq = (v && !strcmp(v, "seq")) ? 1 : 0;
+  // K7 variant: lane-sequential with shared-memory staged clocks (default) or ballot rounds
+  // (BC_K7=ballot); read at every launch so that tests can switch it
+  const char* v = getenv("BC_K7");
+  const int use_tile = (v && !strcmp(v, "ballot")) ? 0 : 1;
+  static int grid_tile = 0, grid_ballot = 0;
+  const size_t smem_tile = (size_t)KT_WARPS * KT_WARP_BYTES;
+  int& grid = use_tile ? grid_tile : grid_ballot;
+  if (grid == 0) {
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (use_seq) {
-      cudaFuncSetAttribute(k_check_seq, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_seq);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_check_seq, KS_WARPS * 32, smem_seq);
+    if (use_tile) {
+      cudaFuncSetAttribute(k_check_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_tile);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_check_tile, KT_WARPS * 32, smem_tile);
     } else {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_check, K7_WARPS * 32, 0);
     }
     if (per < 1) per = 1;
+    const int wpc = use_tile ? KT_WARPS : K7_WARPS;
     grid = sms * per;
-    if (grid * K7_WARPS > 148 * 64) grid = 148 * 64 / K7_WARPS;
+    if (grid * wpc > 148 * 64) grid = 148 * 64 / wpc;
   }
-  const u32 nw = (u32)grid * (use_seq ? KS_WARPS : K7_WARPS);
+  const u32 nw = (u32)grid * (use_tile ? KT_WARPS : K7_WARPS);
   cudaMemsetAsync(status, 0, (size_t)nw * sizeof(WarpEnd), st);
   cudaMemcpyToSymbolAsync(cHC, &c, sizeof(HbCtx), 0, cudaMemcpyHostToDevice, st);
   CheckArgs a;
@@ -698,8 +767,8 @@ void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_
   a.race_cnt = race_cnt;
   a.race_cap = race_cap;
   a.seg_cnt = seg_cnt;
-  if (use_seq) {
-    k_check_seq<<<grid, KS_WARPS * 32, smem_seq, st>>>(a, (WarpEnd*)status, nw);
+  if (use_tile) {
+    k_check_tile<<<grid, KT_WARPS * 32, smem_tile, st>>>(a, (WarpEnd*)status, nw);
   } else {
     k_check<<<grid, K7_WARPS * 32, 0, st>>>(a, (WarpEnd*)status, nw);
   }

@@ -22,7 +22,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
                                                 u32* __restrict__ bar_cnt, u32* __restrict__ sync_list,
                                                 u32* __restrict__ page_bits, u32* __restrict__ word_list,
                                                 u64* __restrict__ cnt, u32* __restrict__ rec_ub,
-                                                u32* __restrict__ err) {
+                                                uint4* __restrict__ hdr16, u32* __restrict__ err) {
   const u32 lane = threadIdx.x & 31;
   const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const u64 r = gw * 32 + lane;
@@ -31,7 +31,15 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
   u32 bad = 0;
   u32 lane_ev = 0, ctl_ev = 0, is_sync = 0, is_acq = 0, is_mem = 0, is_if = 0, is_bar = 0, ibound = 0;
   if (valid) {
-    h = load_hdr(recs, r);
+    const uint4 hv = __ldg(reinterpret_cast<const uint4*>(recs + r));
+    hdr16[r] = hv;  // compact copy of the 16-B header for K2 (gathered per warp there)
+    h.warp = hv.x;
+    h.mask = hv.y;
+    h.op = hv.z & 0xFFu;
+    h.space = (hv.z >> 8) & 0xFFu;
+    h.size_log2 = (hv.z >> 16) & 0xFFu;
+    h.flags = (hv.z >> 24) & 0xFFu;
+    h.aux = hv.w;
     if (h.op > BC_OP_FI || h.warp >= g.n_warps) {
       bad = 1;
     } else {
@@ -163,7 +171,7 @@ __global__ void k_warp_start(const u32* __restrict__ skeys, u64 n, u32 n_warps, 
 // snapshot {warp, ps, node, phase} is written by 32 lanes in parallel.  Per IF it writes the two
 // nodes {mask, parent, popen}; per BAR its record and the warp's next record (barrier feasibility)
 // and a BARRIER_DIVERGENCE finding when the mask is not the warp's initial mask.
-__global__ void __launch_bounds__(256) k_replay(const bc_record* __restrict__ recs, const u32* __restrict__ wrec,
+__global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16, const u32* __restrict__ wrec,
                                                 const u32* __restrict__ warp_start, Geo g,
                                                 const u32* __restrict__ node_base, const u32* __restrict__ bar_base,
                                                 uint4* __restrict__ snap, uint4* __restrict__ nodes,
@@ -189,7 +197,7 @@ __global__ void __launch_bounds__(256) k_replay(const bc_record* __restrict__ re
   uint4 nh = make_uint4(0, 0, 0, 0);
   if (i0 + lane < i1) {
     nr = wrec[i0 + lane];
-    nh = __ldg(reinterpret_cast<const uint4*>(recs + nr));
+    nh = __ldg(hdr16 + nr);
   }
   for (u32 c0 = i0; c0 < i1 && !bad; c0 += 32) {
     const u32 r = nr;
@@ -197,7 +205,7 @@ __global__ void __launch_bounds__(256) k_replay(const bc_record* __restrict__ re
     const u32 cnt = min(32u, i1 - c0);
     if (c0 + 32 + lane < i1) {  // next chunk in flight while this one is stepped through
       nr = wrec[c0 + 32 + lane];
-      nh = __ldg(reinterpret_cast<const uint4*>(recs + nr));
+      nh = __ldg(hdr16 + nr);
     }
     u32 my_ps = 0, my_node = 0, my_phase = 0;
     u32 done = 0;
@@ -497,23 +505,23 @@ __global__ void __launch_bounds__(1024) k_page_rank(u32* __restrict__ words, con
 
 // --------------------------------------------------------------------- host launchers
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
-                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, u32* err,
+                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, uint4* hdr16, u32* err,
                    cudaStream_t st) {
   u64 warps = (g.n_recs + 31) / 32;
   if (warps == 0) return;
   u64 blocks = (warps + 7) / 8;
   k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt,
-                                             rec_ub, err); ++g_launches;
+                                             rec_ub, hdr16, err); ++g_launches;
 }
 
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st) {
   k_warp_start<<<(n_warps + 1 + 255) / 256, 256, 0, st>>>(skeys, n, n_warps, warp_start); ++g_launches;
 }
 
-void launch_replay(const bc_record* recs, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
+void launch_replay(const uint4* hdr16, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
                    const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next, u32* find_blk,
                    u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st) {
-  k_replay<<<(unsigned)(((u64)g.n_warps * 32 + 255) / 256), 256, 0, st>>>(recs, wrec, warp_start, g, node_base, bar_base, snap, nodes,
+  k_replay<<<(unsigned)(((u64)g.n_warps * 32 + 255) / 256), 256, 0, st>>>(hdr16, wrec, warp_start, g, node_base, bar_base, snap, nodes,
                                                      bar_rec, bar_next, find_blk, find_rec, find_cnt, err); ++g_launches;
 }
 

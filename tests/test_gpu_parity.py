@@ -266,3 +266,19 @@ def test_device_borrowed_trace_and_idempotent():
         out = torch.zeros(len(want) * 32, dtype=torch.uint8, device="cuda")
         assert ctx.races_device(out) == len(want)
         assert np.array_equal(out.cpu().numpy(), want.view(np.uint8))
+
+
+# ------------------------------------------------------------------ K7 variants
+@pytest.mark.parametrize("variant", ["ballot", "tile"])
+def test_k7_variants(variant, monkeypatch):
+    """Both K7 formulations (lane-sequential with staged clocks = default, ballot rounds =
+    BC_K7=ballot) give the oracle's race set on random traces, a hot granule and reduced C2-C4."""
+    monkeypatch.setenv("BC_K7", variant)
+    for seed in range(5000, 5040):
+        recs, tb = random_trace(seed)
+        assert_parity(recs, tb.geom.as_dict())
+    test_hot_granule_long_segment()
+    for cfg, kw in [(2, dict(n_blocks=8, iters=6)), (3, dict(n_blocks=9, iters=3, tpb=256)),
+                    (4, dict(n_blocks=40, log2_nodes=16, nodes_per_thread=3, inj_scale=8))]:
+        plan = ConfigPlan(cfg, **kw)
+        assert_parity(plan.records(), plan.geometry)
