@@ -254,7 +254,11 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
       }
     }
     for (int i = t; i < RS_WARPS * BINS; i += RS_THREADS) whist[i] = 0;
-    for (int d = t; d < BINS; d += RS_THREADS) gstart[d] = offs[(u64)d * tiles + tile];
+    // this tile's digit offsets: loaded now, stored to shared memory after the ranking (their
+    // latency overlaps it instead of stalling the tile start)
+    u32 go[DPT];
+#pragma unroll
+    for (int q = 0; q < DPT; ++q) go[q] = __ldg(&offs[(u64)(t + q * RS_THREADS) * tiles + tile]);
     __syncthreads();
     mbar_wait(&bar[st], phase);
     u32 rank[RS_ITEMS];  // (digit << 16) | rank in the warp's digit run, NONE = no item
@@ -272,6 +276,8 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
       __syncwarp();
       rank[j] = d < (u32)BINS ? ((d << 16) | (old + __popc(peers & lt))) : NONE;
     }
+#pragma unroll
+    for (int q = 0; q < DPT; ++q) gstart[t + q * RS_THREADS] = go[q];
     __syncthreads();
     // per digit: prefix over warps, tile total; thread t owns digits [t*DPT, t*DPT + DPT)
     u32 tsum = 0, dtot[DPT];

@@ -165,10 +165,12 @@ __global__ void k_warp_start(const u32* __restrict__ skeys, u64 n, u32 n_warps, 
 // warp walks the traced warp's records in trace order with the SIMT stack of Fig. 2 (K_w,
 // P:L430-432).  Stack levels are branch-tree nodes: IF pushes the then-node (else-node
 // is its sibling, id+1, entered at ELSE); FI pops.  Every join-fork step (endi, if, else, fi, bar)
-// is labelled rec+1.  The 32 lanes load 32 consecutive records (index + header) at once, one chunk
-// ahead, and then step through them together: the stack update is uniform (every lane computes it,
-// operands broadcast by shuffles), and lane j keeps the state record j saw, so the per-record
-// snapshot {warp, ps, node, phase} is written by 32 lanes in parallel.  Per IF it writes the two
+// is labelled rec+1.  The 32 lanes load 32 consecutive records (index + compact 16-B header) at
+// once, one chunk ahead.  Runs of endi records (LD / ST / ATOM / ACQ / REL / AR: only ps changes)
+// are resolved in parallel (lane j: ps = rec[j-1] + 1); the control records between them (IF, ELSE,
+// FI, BAR, FENCE) are stepped one at a time, uniformly across the lanes (header = broadcast
+// shared-memory read, top of the SIMT stack in registers).  Lane j keeps the state record j saw,
+// so the per-record snapshot {warp, ps, node, phase} is written by 32 lanes in parallel.  Per IF it writes the two
 // nodes {mask, parent, popen}; per BAR its record and the warp's next record (barrier feasibility)
 // and a BARRIER_DIVERGENCE finding when the mask is not the warp's initial mask.
 __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16, const u32* __restrict__ wrec,
@@ -178,15 +180,16 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
                                                 u32* __restrict__ bar_rec, u32* __restrict__ bar_next,
                                                 u32* __restrict__ find_blk, u32* __restrict__ find_rec,
                                                 u32* __restrict__ find_cnt, u32* __restrict__ err) {
+  __shared__ uint4 s_hdr[8][32];  // the chunk's headers / record indices: broadcast reads in the
+  __shared__ u32 s_rec[8][32];    // serial steps instead of four shuffles each
   const u32 w = (u32)(((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
-  const u32 lane = threadIdx.x & 31;
+  const u32 lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   if (w >= g.n_warps) return;  // warp-uniform
   const u32 imask = init_mask(g, w);
-  u32 st_node[33], st_mask[33];
+  u32 st_node[33], st_mask[33];  // SIMT stack below the top (the top lives in cur_node / cur_mask)
+  u32 cur_node = w, cur_mask = imask;
   u64 then_bits = 0;  // bit d set: level d is a then-node
   int depth = 0;
-  st_node[0] = w;
-  st_mask[0] = imask;
   if (lane == 0) nodes[w] = make_uint4(imask, NONE, 0u, 0u);
   u32 ps = 0, phase = 0, nif = 0, nbar = 0;
   bool need_next = false;
@@ -207,24 +210,46 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
       nr = wrec[c0 + 32 + lane];
       nh = __ldg(hdr16 + nr);
     }
+    s_hdr[wib][lane] = hv;
+    s_rec[wib][lane] = r;
+    __syncwarp();
+    // control records (FENCE, BAR, IF, ELSE, FI) are stepped one by one; the runs of endi records
+    // between them (LD / ST / ATOM / ACQ / REL / AR: ps := rec + 1, stack unchanged) in parallel
+    const u32 ctl = __ballot_sync(0xFFFFFFFFu, lane < cnt && (hv.z & 0xFFu) >= BC_OP_FENCE);
+    const u32 rprev = __shfl_up_sync(0xFFFFFFFFu, r, 1);
     u32 my_ps = 0, my_node = 0, my_phase = 0;
-    u32 done = 0;
-    for (u32 j = 0; j < cnt; ++j) {
-      const u32 rj = __shfl_sync(0xFFFFFFFFu, r, j);
-      const u32 mask = __shfl_sync(0xFFFFFFFFu, hv.y, j);
-      const u32 op = __shfl_sync(0xFFFFFFFFu, hv.z, j) & 0xFFu;
-      const u32 aux = __shfl_sync(0xFFFFFFFFu, hv.w, j);
+    bool badl = false;
+    u32 sidx = 0;
+    while (sidx < cnt) {
+      const u32 rest = ctl & (~0u << sidx);
+      const u32 f = rest ? (u32)__ffs(rest) - 1u : cnt;
+      if (f > sidx) {  // endi run [sidx, f)
+        if (lane >= sidx && lane < f) {
+          my_ps = lane == sidx ? ps : rprev + 1u;
+          my_node = cur_node;
+          my_phase = phase;
+          badl |= hv.y != cur_mask;  // feasibility: record mask == K_w.peek()
+        }
+        if (need_next) {
+          if (lane == 0) bar_next[bb0 + nbar - 1] = s_rec[wib][sidx];
+          need_next = false;
+        }
+        ps = s_rec[wib][f - 1] + 1u;
+      }
+      if (f >= cnt) break;
+      // control record f
+      const uint4 hf = s_hdr[wib][f];
+      const u32 rj = s_rec[wib][f], mask = hf.y, op = hf.z & 0xFFu, aux = hf.w;
       if (need_next) {
         if (lane == 0) bar_next[bb0 + nbar - 1] = rj;
         need_next = false;
       }
-      if (lane == j) {
+      if (lane == f) {
         my_ps = ps;
-        my_node = st_node[depth];
+        my_node = cur_node;
         my_phase = phase;
       }
-      done = j + 1;
-      if (mask != st_mask[depth]) {  // feasibility: record mask == K_w.peek()
+      if (mask != cur_mask) {
         bad = true;
         break;
       }
@@ -237,20 +262,22 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
           const u32 nid = nb0 + 2 * nif;
           ++nif;
           if (lane == 0) {
-            nodes[nid] = make_uint4(then, st_node[depth], ps, 0u);
-            nodes[nid + 1] = make_uint4(mask & ~then, st_node[depth], ps, 0u);
+            nodes[nid] = make_uint4(then, cur_node, ps, 0u);
+            nodes[nid + 1] = make_uint4(mask & ~then, cur_node, ps, 0u);
           }
+          st_node[depth] = cur_node;
+          st_mask[depth] = cur_mask;
           ++depth;
-          st_node[depth] = nid;
-          st_mask[depth] = then;
+          cur_node = nid;
+          cur_mask = then;
           then_bits |= 1ull << depth;
           ps = rj + 1;
           break;
         }
         case BC_OP_ELSE: {
           if (depth == 0 || !((then_bits >> depth) & 1ull)) { bad = true; break; }
-          st_node[depth] += 1;
-          st_mask[depth] = st_mask[depth - 1] & ~st_mask[depth];
+          cur_node += 1;
+          cur_mask = st_mask[depth - 1] & ~cur_mask;
           then_bits &= ~(1ull << depth);
           ps = rj + 1;
           break;
@@ -258,10 +285,12 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
         case BC_OP_FI: {
           if (depth == 0 || ((then_bits >> depth) & 1ull)) { bad = true; break; }
           --depth;
+          cur_node = st_node[depth];
+          cur_mask = st_mask[depth];
           ps = rj + 1;
           break;
         }
-        case BC_OP_BAR: {
+        default: {  // BC_OP_BAR
           if (lane == 0) {
             if (mask != imask) {  // barrier divergence; the barrier still completes (R10)
               const u32 at = atomicAdd(find_cnt, 1u);
@@ -277,13 +306,13 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
           ps = rj + 1;
           break;
         }
-        default:  // LD/ST/ATOM and ACQ/REL/AR: the record's endi(w) step
-          ps = rj + 1;
-          break;
       }
       if (bad) break;
+      sidx = f + 1;
     }
-    if (lane < done) snap[r] = make_uint4(w, my_ps, my_node, my_phase);
+    bad |= __any_sync(0xFFFFFFFFu, badl);
+    if (lane < cnt) snap[r] = make_uint4(w, my_ps, my_node, my_phase);
+    __syncwarp();
   }
   if (bad && lane == 0) set_err(err, ERR_INFEASIBLE);
 }
