@@ -25,6 +25,9 @@ CONFIGS = {
     "c3": "threadFenceReduction-style trace: 4096 blocks x 256 threads, global atomics + __threadfence, ~50M events",
     "c4": "irregular BFS-like trace: 1M threads, random global addresses, atomics and injected races, ~200M events",
     "c5": "scale trace: 4M threads, ~1B events",
+    "c6": "lock-heavy hashtable trace (SURVEY row f2, P:L1522-1535): 256 blocks x 128 threads, 2 inserts "
+          "per thread under per-bucket locks, with both section-6.3 bugs (CAS without fence, unlock by plain "
+          "store); bug=0 is the fixed program",
 }
 
 
@@ -79,7 +82,8 @@ class _Params(ctypes.Structure):
                 ("nodes_per_thread", ctypes.c_uint32), ("max_resident", ctypes.c_uint32),
                 ("inject", ctypes.c_uint32), ("inj_scale", ctypes.c_uint32),
                 ("deg_lo", ctypes.c_uint32), ("deg_hi", ctypes.c_uint32),
-                ("bar_per_node", ctypes.c_uint32), ("seed", ctypes.c_uint64)]
+                ("bar_per_node", ctypes.c_uint32), ("seed", ctypes.c_uint64),
+                ("bug", ctypes.c_uint32), ("log2_buckets", ctypes.c_uint32)]
 
 
 class _Info(ctypes.Structure):
@@ -116,6 +120,8 @@ class ConfigPlan:
         p.config = config
         p.seed = config if seed is None else seed
         p.inject = kw.pop("inject", 1)
+        if config == 6:
+            p.bug = kw.pop("bug", 3)  # the benchmark as published has both section-6.3 bugs
         for k, v in kw.items():
             setattr(p, k, v)
         info = _Info()
@@ -159,7 +165,7 @@ class ConfigPlan:
             pass
 
 
-_CIDX = {"c1": 1, "c2": 2, "c3": 3, "c4": 4, "c5": 5}
+_CIDX = {"c1": 1, "c2": 2, "c3": 3, "c4": 4, "c5": 5, "c6": 6}
 
 
 def make_config(name, seed=None, **kw):

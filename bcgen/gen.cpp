@@ -15,6 +15,14 @@
 //                   atomics on cost/mask, Zipf(0.8) neighbour ids, injected races
 //   C5 scale        C4 shape with 16384 blocks, N = 2^26, 10 nodes/thread and a
 //                   BAR after every node iteration
+//   C6 hashtable    lock-heavy GPU-TM-style hashtable:
+//                   every thread inserts `iters` keys; the lanes of a warp take turns
+//                   (IF lane), each locks its bucket (atomicCAS + fence = ACQ_GLB), reads
+//                   and writes the bucket head, writes its node, and unlocks (fence +
+//                   atomicExch = REL_GLB).  `bug` reproduces the two bugs of §6.3: bit 0 =
+//                   CAS without fence (a plain ATOM, no acquire), bit 1 = unlock by a plain
+//                   store without fence (ST, no release).  The scheduler keeps the locks
+//                   mutually exclusive (an acquire of a held lock waits).
 #include <algorithm>
 #include <atomic>
 #include <cmath>
@@ -73,6 +81,8 @@ enum Role : uint16_t {
   // C4/C5
   R4_FRONTIER, R4_RP, R4_COL, R4_COST, R4_MASK, R4_INJ_INTER, R4_INJ_BR_ST, R4_INJ_BR_LD,
   R4_INJ_ATM,
+  // C6
+  R6_KEYS, R6_LOCK, R6_HEAD, R6_NODE,
 };
 
 struct Params {
@@ -88,6 +98,8 @@ struct Params {
   uint32_t deg_lo, deg_hi;
   uint32_t bar_per_node; // C5 style barrier after each node iteration
   uint64_t seed;
+  uint32_t bug;          // C6: bit 0 = CAS without fence, bit 1 = unlock by plain store
+  uint32_t log2_buckets; // C6: hashtable buckets (0 = default 2^12)
 };
 
 struct Gen {
@@ -130,6 +142,11 @@ struct Gen {
     return (uint32_t)(((rank - 1) * 0x9E3779B1ull) & (N - 1));
   }
 
+  // C6: bucket of the key inserted by thread g in iteration it
+  uint32_t bucket(uint32_t g, uint32_t it) const {
+    return (uint32_t)(splitmix64(p.seed * 7919 + (uint64_t)g * 64 + it) & ((1u << p.log2_buckets) - 1));
+  }
+
   uint64_t addr(const CRec& c, int lane) const {
     uint32_t w = c.warp, t = tib(w, lane), b = w / wpb, g = gtid(w, lane);
     switch (c.role) {
@@ -164,6 +181,10 @@ struct Gen {
       case R4_INJ_BR_ST: return GB + 6 * REGION + 4ull * (32ull * c.p32 + lane);
       case R4_INJ_BR_LD: return GB + 6 * REGION + 4ull * (32ull * c.p32 + (lane ^ 1));
       case R4_INJ_ATM: return GB + 7 * REGION + 4ull * (32ull * c.p32 + lane);
+      case R6_KEYS: return GB + 4ull * ((uint64_t)g * p.iters + c.p32);
+      case R6_LOCK: return GB + REGION + 4ull * bucket(g, c.p32);
+      case R6_HEAD: return GB + 2 * REGION + 4ull * bucket(g, c.p32);
+      case R6_NODE: return GB + 3 * REGION + 8ull * ((uint64_t)g * p.iters + c.p32);
       default: return 0;
     }
   }
@@ -307,6 +328,24 @@ struct Gen {
     }
   }
 
+  void prog_c6(uint32_t w, std::vector<CRec>& v) {
+    const uint32_t m = init_mask(w);
+    const bool cas_nofence = p.bug & 1u, unlock_plain = p.bug & 2u;
+    for (uint32_t it = 0; it < p.iters; ++it) {
+      v.push_back(mk(w, m, LD, GLOBAL, R6_KEYS, 0, it));
+      for (int l = 0; l < 32; ++l) {  // the lanes take turns: one lock holder per warp at a time
+        if (!((m >> l) & 1u)) continue;
+        branch(v, w, m, 1u << l, [&](uint32_t tm) {
+          v.push_back(mk(w, tm, cas_nofence ? ATOM : ACQ_GLB, GLOBAL, R6_LOCK, (uint16_t)l, it));
+          v.push_back(mk(w, tm, LD, GLOBAL, R6_HEAD, (uint16_t)l, it));
+          v.push_back(mk(w, tm, ST, GLOBAL, R6_NODE, (uint16_t)l, it));
+          v.push_back(mk(w, tm, ST, GLOBAL, R6_HEAD, (uint16_t)l, it));
+          v.push_back(mk(w, tm, unlock_plain ? ST : REL_GLB, GLOBAL, R6_LOCK, (uint16_t)(l | 0x100), it));
+        });
+      }
+    }
+  }
+
   void setup() {
     int c = p.config;
     tpb = p.tpb ? p.tpb : 256;
@@ -319,6 +358,13 @@ struct Gen {
       nb = p.n_blocks ? p.n_blocks : 4096;
       if (!p.iters) p.iters = 40;
       smem = tpb * 4 + 16;
+    } else if (c == 6) {
+      tpb = p.tpb ? p.tpb : 128;
+      wpb = (tpb + 31) / 32;
+      nb = p.n_blocks ? p.n_blocks : 256;
+      if (!p.iters) p.iters = 2;
+      if (!p.log2_buckets) p.log2_buckets = 12;
+      smem = 16;
     } else {
       nb = p.n_blocks ? p.n_blocks : (c == 5 ? 16384 : 4096);
       uint32_t ln = p.log2_nodes ? p.log2_nodes : (c == 5 ? 26 : 24);
@@ -372,6 +418,7 @@ struct Gen {
     switch (p.config) {
       case 2: prog_c2(w, v); break;
       case 3: prog_c3(w, v); break;
+      case 6: prog_c6(w, v); break;
       default: prog_c4(w, v); break;
     }
   }
@@ -385,6 +432,8 @@ struct Gen {
     std::vector<uint8_t> waiting(nw, 0);
     std::vector<uint32_t> arrived(nb, 0), live(nb, 0);
     std::vector<uint32_t> active;  // resident warps
+    std::vector<uint32_t> holder;  // C6: lock holder (warp + 1) per bucket, 0 = free
+    if (p.config == 6) holder.assign(1u << p.log2_buckets, 0);
     uint32_t next_block = 0, resident = 0, done_blocks = 0;
     out.clear();
     while (done_blocks < nb) {
@@ -407,6 +456,16 @@ struct Gen {
         if (!waiting[w]) {
           uint32_t burst = 1 + rng.below(3);
           for (uint32_t k = 0; k < burst && pc[w] < prog[w].size(); ++k) {
+            if (!holder.empty() && prog[w][pc[w]].role == R6_LOCK) {
+              const CRec& lc = prog[w][pc[w]];
+              const uint32_t bk = bucket(gtid(w, lc.p16 & 0xFF), lc.p32);
+              if (!(lc.p16 & 0x100)) {  // lock: wait while another thread holds the bucket
+                if (holder[bk]) break;
+                holder[bk] = w + 1;
+              } else {
+                holder[bk] = 0;
+              }
+            }
             CRec c = prog[w][pc[w]++];
             if (c.op == DYN) { prog_c3_tail(w, prog[w]); --k; continue; }
             if (c.op == AR_GLB && c.role == R3_COUNT) {

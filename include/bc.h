@@ -124,6 +124,8 @@ typedef struct bc_stats {
   uint64_t sync_ops;         /* acquire / release lane operations                                 */
   uint64_t written_pages;    /* 1-MB global pages with at least one write          */
   uint64_t kernel_launches;  /* libbc kernels launched by this bc_detect                          */
+  uint64_t clock_gathers;    /* 16-B record clock snapshots the per-granule check read (items that
+                                some happens-before check needs)                                 */
   float ms_total;            /* device time of bc_detect (cudaEvents on the stream)               */
   float ms_kernel[12];       /* per phase, then kernel-only k_check / k_sort_items / k_expand;
                                 see bc_phase_name()                                              */

@@ -60,7 +60,7 @@ class _Stats(ctypes.Structure):
                 ("control_events", ctypes.c_uint64), ("items", ctypes.c_uint64),
                 ("segments", ctypes.c_uint64), ("races", ctypes.c_uint64), ("findings", ctypes.c_uint64),
                 ("sync_ops", ctypes.c_uint64), ("written_pages", ctypes.c_uint64),
-                ("kernel_launches", ctypes.c_uint64),
+                ("kernel_launches", ctypes.c_uint64), ("clock_gathers", ctypes.c_uint64),
                 ("ms_total", ctypes.c_float), ("ms_kernel", ctypes.c_float * 12)]
 
 

@@ -335,20 +335,21 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32 race_cap = (u32)std::min<u64>(std::max<u64>(1u << 16, bound / 16), 1u << 30);
   uint4* rbuf = nullptr;
   u32* rcnt = S.alloc<u32>(1);
-  u64* segc = S.alloc<u64>(1);
+  u64* segc = S.alloc<u64>(2);  // [0] segments, [1] clock snapshot gathers
   void* cstatus = S.alloc<char>(check_status_bytes(bound));
   u32 n_r = 0, nfind = 0;
   u64 n_items = 0;
   for (int attempt = 0; attempt < 2; ++attempt) {
     rbuf = S.alloc<uint4>(race_cap);
     cudaMemsetAsync(rcnt, 0, 4, st);
-    cudaMemsetAsync(segc, 0, 8, st);
+    cudaMemsetAsync(segc, 0, 16, st);
     cudaEventRecord(c->ev[10], st);
     launch_check(hc, skey, sev, n_items_dev, bound, cstatus, rbuf, rcnt, race_cap, segc, st);
     cudaEventRecord(c->ev[11], st);
     cudaMemcpyAsync(&n_r, rcnt, 4, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&sx.segments, segc, 8, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(&sx.clock_gathers, segc + 1, 8, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&n_items, n_items_dev, 8, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&nfind, find_cnt, 4, cudaMemcpyDeviceToHost, st);
     if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "check");

@@ -58,7 +58,7 @@ struct CheckArgs {
   uint4* races;  // (key, cur_ev, prior_ev, kind)
   u32* race_cnt;
   u32 race_cap;
-  u64* seg_cnt;
+  u64* seg_cnt;  // [0] segments, [1] clock snapshot gathers
 };
 
 __device__ __forceinline__ void emit(const CheckArgs& a, u32 key, u32 cur, u32 prior, u32 kind) {
@@ -244,7 +244,7 @@ __device__ bool walk_back(const CheckArgs& a, u64 s, Sum& out) {
 // traces (C4/C5 cost/mask) this removes almost all random 16-B gathers.
 constexpr int K7_PS = 2;
 
-__device__ __forceinline__ uint4 snap_if_needed(const HbCtx& c, u32 k, u32 e, u32 kprev0, u32 knext31) {
+__device__ __forceinline__ uint4 snap_if_needed(const HbCtx& c, u32 k, u32 e, u32 kprev0, u32 knext31, u32& gat) {
   const int lane = threadIdx.x & 31;
   u32 kp = __shfl_up_sync(0xFFFFFFFFu, k, 1), kn = __shfl_down_sync(0xFFFFFFFFu, k, 1);
   if (lane == 0) kp = kprev0;
@@ -254,6 +254,7 @@ __device__ __forceinline__ uint4 snap_if_needed(const HbCtx& c, u32 k, u32 e, u3
   const bool sp = kp != NONE && (kp >> 2) == key, sn = kn != NONE && (kn >> 2) == key;
   const bool atm_only = (k & 3u) == IOP_ATOM && (!sp || (kp & 3u) == IOP_ATOM) && (!sn || (kn & 3u) == IOP_ATOM);
   if ((!sp && !sn) || atm_only) return make_uint4(0, 0, 0, 0);
+  ++gat;
   return __ldg(c.snap + (e >> 5));
 }
 
@@ -296,7 +297,7 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
 
   // ---- the range, round by round
   const u32 no_sv = c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
-  u32 segs = 0;
+  u32 segs = 0, gat = 0;
   u32 pf_k[K7_PF], pf_e[K7_PF];
   uint4 pf_s[K7_PS];
 #pragma unroll
@@ -309,7 +310,7 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
   for (int q = 0; q < K7_PS; ++q) {
     const u32 kp0 = q == 0 ? pkx : __shfl_sync(0xFFFFFFFFu, pf_k[q > 0 ? q - 1 : 0], 31);
     const u32 kn31 = __shfl_sync(0xFFFFFFFFu, pf_k[q + 1], 0);
-    pf_s[q] = snap_if_needed(c, pf_k[q], pf_e[q], kp0, kn31);
+    pf_s[q] = snap_if_needed(c, pf_k[q], pf_e[q], kp0, kn31, gat);
   }
   for (u64 base_r = beg; base_r < end; base_r += 32) {
     const u64 i = base_r + lane;
@@ -329,7 +330,7 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
       pf_e[K7_PF - 1] = ip < end ? a.evs[ip] : 0u;
       const u32 kp0 = __shfl_sync(0xFFFFFFFFu, K7_PS >= 2 ? pf_k[K7_PS >= 2 ? K7_PS - 2 : 0] : kx, 31);
       const u32 kn31 = __shfl_sync(0xFFFFFFFFu, pf_k[K7_PS], 0);
-      pf_s[K7_PS - 1] = snap_if_needed(c, pf_k[K7_PS - 1], pf_e[K7_PS - 1], kp0, kn31);
+      pf_s[K7_PS - 1] = snap_if_needed(c, pf_k[K7_PS - 1], pf_e[K7_PS - 1], kp0, kn31, gat);
     }
     u32 qkx = __shfl_up_sync(0xFFFFFFFFu, kx, 1);
     u32 qev = __shfl_up_sync(0xFFFFFFFFu, ev, 1);
@@ -410,8 +411,10 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
     pev = __shfl_sync(0xFFFFFFFFu, ev, last);
     pw = __shfl_sync(0xFFFFFFFFu, s2.warp, last);
   }
+  gat = __reduce_add_sync(0xFFFFFFFFu, gat);
   if (lane == 0) {
     if (segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)segs);
+    if (gat) atomicAdd((unsigned long long*)(a.seg_cnt + 1), (unsigned long long)gat);
     volatile WarpEnd* me = &wend[w];
     me->lk = carry.lk;
     me->lw = carry.lw;
@@ -537,7 +540,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
     }
   }
 
-  u32 segs = 0;
+  u32 segs = 0, gat = 0;
   const u32 l0 = lane * KT_IPL;
   if (beg < end) kt_stage(a, beg, (u32)(end - beg < (u64)KT_BLK ? end - beg : (u64)KT_BLK), sKE, sKE + KT_PITCH, lane);
   for (u64 bb = beg; bb < end; bb += KT_BLK) {
@@ -567,7 +570,10 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
         const bool sp = kp != NONE && (kp >> 2) == key, sn = kn != NONE && (kn >> 2) == key;
         const bool atm_only =
             (k & 3u) == IOP_ATOM && (!sp || (kp & 3u) == IOP_ATOM) && (!sn || (kn & 3u) == IOP_ATOM);
-        if ((sp || sn) && !atm_only) cp_async16(sS + tpad(li), c.snap + (sE[tpad(li)] >> 5));
+        if ((sp || sn) && !atm_only) {
+          cp_async16(sS + tpad(li), c.snap + (sE[tpad(li)] >> 5));
+          ++gat;
+        }
         kp = k;
         k = kn;
       }
@@ -715,8 +721,10 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
     __syncwarp();
   }
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);
+  gat = __reduce_add_sync(0xFFFFFFFFu, gat);
   if (lane == 0) {
     if (segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)segs);
+    if (gat) atomicAdd((unsigned long long*)(a.seg_cnt + 1), (unsigned long long)gat);
     volatile WarpEnd* me = &wend[w];
     me->lk = carry.lk;
     me->lw = carry.lw;

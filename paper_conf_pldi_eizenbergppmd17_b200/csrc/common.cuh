@@ -192,7 +192,7 @@ __device__ __forceinline__ u32 idx_lower_bound(const HbCtx& c, u64 ak) {
 // the link DAG; an array already visited with a bound >= the new one is skipped (its entries
 // are a superset), which keeps chains of releases linear.
 static __device__ __noinline__ bool view_knows(const HbCtx c, u32 uw, u32 ul, u32 r1, u32 arr, u32 bound) {
-  constexpr int STK = 96, VIS = 160;
+  constexpr int STK = 256, VIS = 256;
   u32 st_arr[STK], st_bd[STK];
   u32 vis_arr[VIS], vis_bd[VIS];
   int sp = 0, nv = 0;
@@ -220,6 +220,9 @@ static __device__ __noinline__ bool view_knows(const HbCtx c, u32 uw, u32 ul, u3
       set_err(c.err, ERR_OVERFLOW);
       return false;
     }
+    // once any lookup has overflowed the whole detect fails (BC_ERR_OVERFLOW): stop early instead of
+    // finishing every other long walk (lock-heavy traces)
+    if ((steps & 255u) == 0u && (*(volatile u32*)c.err & ERR_OVERFLOW)) return false;
     // block-level entries
     u64 ak = ((u64)a << 32) | (KEY_BLOCK | ub);
     for (u32 i = idx_lower_bound(c, ak); i < c.n_idx && c.idx_ak[i] == ak && c.idx_pos[i] < bd; ++i)
@@ -247,6 +250,13 @@ static __device__ __noinline__ bool view_knows(const HbCtx c, u32 uw, u32 ul, u3
         bool seen = false;
         for (int q = 0; q < nv; ++q)
           if (vis_arr[q] == tgt && vis_bd[q] >= best) seen = true;
+        // already waiting on the stack: keep one entry with the larger bound (lock chains reach the
+        // same views along many paths)
+        for (int q = 0; q < sp && !seen; ++q)
+          if (st_arr[q] == tgt) {
+            if (st_bd[q] < best) st_bd[q] = best;
+            seen = true;
+          }
         if (seen) continue;
         if (sp >= STK) {
           set_err(c.err, ERR_OVERFLOW);

@@ -282,3 +282,45 @@ def test_k7_variants(variant, monkeypatch):
                     (4, dict(n_blocks=40, log2_nodes=16, nodes_per_thread=3, inj_scale=8))]:
         plan = ConfigPlan(cfg, **kw)
         assert_parity(plan.records(), plan.geometry)
+
+
+# ------------------------------------------------- lock-heavy hashtable
+@pytest.mark.parametrize("bug", [0, 1, 2, 3])
+def test_c6_hashtable(bug):
+    """Per-bucket locks: K3 with thousands of single-lane acquire / release
+    records and SPARSEVC-style foreign knowledge; the fixed program and both section-6.3 bugs.
+    The fixed program (acquire AND release on every lock) chains every critical section of a
+    bucket to the next: its foreign-knowledge lookups walk the link graph of K3, which is
+    bounded, so beyond the small sizes it must fail loudly with
+    BC_ERR_OVERFLOW -- never return a wrong race set."""
+    sizes = (dict(n_blocks=1, tpb=32, iters=1, log2_buckets=1),
+             dict(n_blocks=2, tpb=32, iters=1, log2_buckets=3),
+             dict(n_blocks=6, tpb=64, iters=2, log2_buckets=5),
+             dict(n_blocks=24, tpb=128, iters=2, log2_buckets=7))
+    for i, kw in enumerate(sizes):
+        plan = ConfigPlan(6, bug=bug, **kw)
+        recs = plan.records()
+        if bug == 0 and i >= 2:
+            if i > 2:
+                continue  # (fails the same way, slower)
+            with pytest.raises(bc.BcError) as ei:
+                _gpu(recs, plan.geometry)
+            assert "OVERFLOW" in str(ei.value)
+            continue
+        want, _ = assert_parity(recs, plan.geometry)
+        assert (len(want) == 0) == (bug == 0)
+
+
+def test_c6_hashtable_bench_shape():
+    """The bench workload's shape (128-thread blocks, 2 inserts per thread, 4096 buckets, both
+    bugs) at 32 of its 256 blocks."""
+    plan = ConfigPlan(6, n_blocks=32)
+    want, res = assert_parity(plan.records(), plan.geometry)
+    assert len(want) > 0
+
+
+def test_c6_full_size():
+    """The c6 bench workload at full size (526 K records, ~184 K races) against the oracle."""
+    plan = ConfigPlan(6)
+    want, res = assert_parity(plan.records(), plan.geometry)
+    assert len(want) > 100_000

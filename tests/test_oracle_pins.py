@@ -26,6 +26,7 @@ import oracle
 from bcgen import TraceBuilder, GLOBAL_BASE
 from bcgen.configs import ConfigPlan
 from bcgen.fuzz import random_trace
+from bcgen.format import KIND_NAMES
 from oracle.bf import brute_force, valid_granules
 
 import litmus
@@ -286,3 +287,72 @@ def test_depth_32_accepted():
         tb.else_(0); tb.fi(0)
     st, races, _ = oracle.detect_geom(tb.records(), tb.geom.as_dict())
     assert st == 0 and len(races) == 0
+
+
+# ------------------------------------------------- lock-heavy hashtable
+def _c6(bug, **kw):
+    kw.setdefault("n_blocks", 2)
+    kw.setdefault("tpb", 32)
+    kw.setdefault("iters", 1)
+    kw.setdefault("log2_buckets", 3)
+    plan = ConfigPlan(6, bug=bug, **kw)
+    return plan.records(), plan.geometry
+
+
+def _c6_buckets(recs):
+    """head address -> set of threads that insert into it (from the trace itself)"""
+    from bcgen.format import OP_ST
+    heads = {}
+    region = 1 << 34
+    for r in recs:
+        if int(r["op"]) != OP_ST:
+            continue
+        for l in range(32):
+            if (int(r["mask"]) >> l) & 1:
+                a = int(r["addr"][l])
+                if GLOBAL_BASE + 2 * region <= a < GLOBAL_BASE + 3 * region:
+                    heads.setdefault(a, set()).add((int(r["warp"]), l))
+    return heads
+
+
+@pytest.mark.parametrize("bug", [0, 1, 2, 3])
+def test_c6_hashtable_vs_bruteforce(bug):
+    """the fixed hashtable (CAS + fence acquire, fence + exch release) is race-free
+    under §3.2; each bug (CAS without fence, unlock by plain store) makes the bucket heads of
+    contended buckets race.  The oracle's pairs are §3.2 races and its first race per granule is
+    §3.2's on the valid class."""
+    recs, geom = _c6(bug)
+    races = run(recs, geom)
+    bf = check_against_bf(recs, geom, races)
+    if bug == 0:
+        assert len(races) == 0 and len(bf.race_set()) == 0
+    else:
+        assert len(races) > 0
+
+
+@pytest.mark.parametrize("bug", [0, 1, 2, 3])
+def test_c6_hashtable_race_structure(bug):
+    """Closed form of where the races are: none without a bug; with either bug exactly the
+    bucket heads written by two or more threads race (a bucket with one inserter has nothing to
+    race with); the lock word races only when the unlock is a plain store (bug bit 1): WW
+    against the next plain unlock, or WA against the next lock attempt when the CAS is a plain
+    atomic too (both bugs)."""
+    recs, geom = _c6(bug, n_blocks=6, tpb=64, iters=2, log2_buckets=5)
+    races = run(recs, geom)
+    region = 1 << 34
+    heads = _c6_buckets(recs)
+    head_races = {int(r["addr"]) for r in races if GLOBAL_BASE + 2 * region <= int(r["addr"]) < GLOBAL_BASE + 3 * region}
+    lock_races = [r for r in races if GLOBAL_BASE + region <= int(r["addr"]) < GLOBAL_BASE + 2 * region]
+    other = [r for r in races if not (GLOBAL_BASE + region <= int(r["addr"]) < GLOBAL_BASE + 3 * region)]
+    assert not other
+    if bug == 0:
+        assert len(races) == 0
+        return
+    assert head_races == {a for a, th in heads.items() if len(th) >= 2}
+    kinds = {int(r["kind"]) for r in lock_races}
+    if bug == 1:
+        assert not lock_races
+    elif bug == 2:
+        assert lock_races and kinds == {KIND_NAMES.index("WW")}
+    else:
+        assert lock_races and kinds == {KIND_NAMES.index("WA")}
