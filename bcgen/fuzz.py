@@ -169,3 +169,21 @@ def random_trace(seed: int, *, max_blocks=3, max_tpb=72, ops_per_warp=(3, 14), n
         step(rng.choice(runnable))
     assert all(not waiting[w] for w in range(nw))
     return tb.records(), tb
+
+
+def random_values(records, seed: int, p_uniform: float = 0.4, n_distinct: int = 3):
+    """Per-lane store values [n_records, 32] (uint64) for SURVEY row f3: for each store record,
+    with probability p_uniform every lane stores one value, otherwise each lane draws from
+    n_distinct values (so some lane pairs agree and some do not).  Input fixture only."""
+    import numpy as np
+    from .format import OP_ST
+    rng = random.Random(seed * 7919 + 17)
+    vals = np.zeros((len(records), 32), dtype=np.uint64)
+    for i, r in enumerate(records):
+        if int(r["op"]) != OP_ST:
+            continue
+        if rng.random() < p_uniform:
+            vals[i, :] = rng.randrange(1 << 62)
+        else:
+            vals[i, :] = [rng.randrange(n_distinct) for _ in range(32)]
+    return vals

@@ -141,6 +141,18 @@ bc_status bc_init(const bc_config* cfg, struct bc_ctx** out);
  * must keep it alive and unmodified.  n_recs may be 0.  n_recs >= 2^27 -> BC_ERR_OVERFLOW. */
 bc_status bc_load_trace(struct bc_ctx* ctx, const bc_record* recs, uint64_t n_recs, int recs_on_device);
 
+/* Optional per-lane store values (reading R6b in DESIGN.md).
+ *   values[r * 32 + l] = the value lane l of store record r writes (8 B; a 64-bit digest for wider
+ *   vector stores); entries of other records / inactive lanes are ignored.
+ * With values loaded, the intra-warp same-value filter compares the two lanes' values (a
+ * write-write race between two lanes of ONE record is filtered iff they store the same value)
+ * instead of reading the BC_REC_SAME_VALUE flag.  n_recs must equal the loaded trace's record
+ * count.  Host pointer: copied (caller keeps ownership); device pointer (values_on_device = 1,
+ * 8-B aligned): borrowed until the next bc_load_trace / bc_load_values / bc_destroy.  values ==
+ * NULL clears them.  bc_load_trace clears them too.  Errors: BC_ERR_STATE (no trace loaded),
+ * BC_ERR_INVALID_ARG (count mismatch / misaligned device pointer), BC_ERR_OOM / BC_ERR_CUDA. */
+bc_status bc_load_values(bc_ctx* ctx, const uint64_t* values, uint64_t n_recs, int values_on_device);
+
 /* Run the race check on the loaded trace (all kernels on cfg.stream) and synchronize.
  * Infeasible trace -> BC_ERR_INFEASIBLE_TRACE (no races are kept).  `out` may be NULL.
  * Repeated calls on the same trace are idempotent. */

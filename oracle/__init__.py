@@ -53,14 +53,18 @@ def _load():
         lib.oracle_detect.restype = ctypes.c_int
         lib.oracle_detect.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.POINTER(_Geom),
                                       ctypes.POINTER(_Result)]
+        lib.oracle_detect_values.restype = ctypes.c_int
+        lib.oracle_detect_values.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.POINTER(_Geom),
+                                             ctypes.c_void_p, ctypes.POINTER(_Result)]
         lib.oracle_free.argtypes = [ctypes.c_void_p]
         _lib = lib
     return _lib
 
 
 def detect(records: np.ndarray, grid=(1, 1, 1), block=(32, 1, 1), smem_bytes=0, granule_log2=2,
-           flags=0, warp_size=32):
-    """Run the oracle.  Returns (status, races[RACE_DTYPE], stats dict)."""
+           flags=0, warp_size=32, values=None):
+    """Run the oracle.  Returns (status, races[RACE_DTYPE], stats dict).  values: optional uint64
+    array [n_records, 32] of per-lane store values (reading R6b)."""
     lib = _load()
     g = _Geom()
     grid = tuple(grid) + (1,) * (3 - len(grid))
@@ -70,8 +74,11 @@ def detect(records: np.ndarray, grid=(1, 1, 1), block=(32, 1, 1), smem_bytes=0, 
     g.warp_size, g.granule_log2, g.smem_bytes, g.flags = warp_size, granule_log2, smem_bytes, flags
     recs = np.ascontiguousarray(records)
     res = _Result()
-    st = lib.oracle_detect(recs.ctypes.data if len(recs) else None, len(recs), ctypes.byref(g),
-                           ctypes.byref(res))
+    vals = None if values is None else np.ascontiguousarray(values, dtype=np.uint64).reshape(-1)
+    if vals is not None and len(vals) != 32 * len(recs):
+        raise ValueError("values must hold 32 entries per record")
+    st = lib.oracle_detect_values(recs.ctypes.data if len(recs) else None, len(recs), ctypes.byref(g),
+                                  vals.ctypes.data if vals is not None and len(vals) else None, ctypes.byref(res))
     races = np.zeros(res.n_races, dtype=RACE_DTYPE)
     if res.n_races:
         ctypes.memmove(races.ctypes.data, res.races, res.n_races * 32)
@@ -79,6 +86,6 @@ def detect(records: np.ndarray, grid=(1, 1, 1), block=(32, 1, 1), smem_bytes=0, 
     return st, races, dict(lane_events=res.lane_events, control_events=res.control_events)
 
 
-def detect_geom(records, geom: dict, flags=0):
+def detect_geom(records, geom: dict, flags=0, values=None):
     return detect(records, grid=geom["grid"], block=geom["block"], smem_bytes=geom["smem_bytes"],
-                  granule_log2=geom.get("granule_log2", 2), flags=flags)
+                  granule_log2=geom.get("granule_log2", 2), flags=flags, values=values)

@@ -60,7 +60,10 @@ class BFResult:
 
 
 def brute_force(records: np.ndarray, grid=(1, 1, 1), block=(32, 1, 1), granule_log2=2,
-                same_value_filter=True):
+                same_value_filter=True, values=None):
+    """values: optional per-lane store values [n_records, 32] (reading R6b): two stores of one
+    record race only if they store different values (instead of the SAME_VALUE flag)."""
+    vals = None if values is None else np.asarray(values, dtype=np.uint64).reshape(-1)
     grid = tuple(grid) + (1,) * (3 - len(grid))
     block = tuple(block) + (1,) * (3 - len(block))
     nb = grid[0] * grid[1] * grid[2]
@@ -159,7 +162,8 @@ def brute_force(records: np.ndarray, grid=(1, 1, 1), block=(32, 1, 1), granule_l
                     continue
                 if (anc[nj] >> ni) & 1:
                     continue
-                if same_value_filter and ti == ST and tj == ST and ri == rj and svj:
+                sv = (vals[evi] == vals[evj]) if vals is not None else svj
+                if same_value_filter and ti == ST and tj == ST and ri == rj and sv:
                     continue
                 out.append((evi, evj, _KIND[(ti, tj)]))
         if out:

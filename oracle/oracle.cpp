@@ -22,7 +22,10 @@
 //   R5  lanes of a record are processed in ascending lane order, granules in
 //       ascending order; event id = (record index << 5) | lane.
 //   R6  SAME_VALUE record flag suppresses write-write races between two lanes
-//       of that same record.
+//       of that same record.  R6b: when per-lane
+//       store values are supplied (values[record * 32 + lane]), the filter
+//       compares them instead of the flag: a write-write race between two lanes
+//       of one record is filtered iff the two lanes store the same value.
 //   R7  an access of 2^k bytes at a (naturally aligned) address covers the
 //       granules [addr >> G, (addr + size - 1) >> G].
 //   R8  reported pairs are exactly the failed checks of the rules (FastTrack
@@ -162,6 +165,7 @@ enum EntryKind { ROOT, ELSE_ENTRY, THEN_ENTRY };
 
 struct Oracle {
   const Record* recs;
+  const uint64_t* values = nullptr;  // R6b: per-lane store values, nullable
   uint64_t n;
   Geom g;
   uint32_t flags;
@@ -243,7 +247,8 @@ struct Oracle {
     Shadow& s = shadow[x];
     if (!epoch_leq(s.W, C[t])) {
       uint8_t kind = s.W_atomic ? AW : WW;
-      bool filtered = kind == WW && same_value_rec && !(flags & F_NO_SAME_VALUE_FILTER) &&
+      const bool same_value = values ? values[s.W.ev] == values[ev] : same_value_rec;  // R6 / R6b
+      bool filtered = kind == WW && same_value && !(flags & F_NO_SAME_VALUE_FILTER) &&
                       (s.W.ev >> 5) == (ev >> 5);  // intra-warp same-value store
       if (!filtered) report(x, s.W, ev, kind);
     }
@@ -481,11 +486,21 @@ struct oracle_result {
   uint64_t n_races, lane_events, control_events;
 };
 
+int oracle_detect_values(const void* recs, uint64_t n_recs, const oracle_geom* gm, const uint64_t* values,
+                         oracle_result* res);
 int oracle_detect(const void* recs, uint64_t n_recs, const oracle_geom* gm, oracle_result* res) {
+  return oracle_detect_values(recs, n_recs, gm, nullptr, res);
+}
+
+// values: nullable, values[record * 32 + lane] = the value lane `lane` of store record `record`
+// writes (R6b); other entries are ignored
+int oracle_detect_values(const void* recs, uint64_t n_recs, const oracle_geom* gm, const uint64_t* values,
+                         oracle_result* res) {
   if (!gm || !res || (n_recs && !recs)) return -1;
   if (gm->warp_size != 32 || gm->granule_log2 > 4) return -1;
   Oracle o;
   o.recs = (const Record*)recs;
+  o.values = values;
   o.n = n_recs;
   o.flags = gm->flags;
   uint64_t nb = (uint64_t)gm->grid[0] * gm->grid[1] * gm->grid[2];

@@ -37,7 +37,7 @@ STATUS = {0: "OK", -1: "INVALID_ARG", -2: "INFEASIBLE_TRACE", -3: "OOM", -4: "CU
 F_RELEASE_OVERWRITE = 1
 F_NO_SAME_VALUE_FILTER = 2
 
-EXPORTS = ["bc_init", "bc_load_trace", "bc_detect", "bc_races", "bc_races_device", "bc_destroy",
+EXPORTS = ["bc_init", "bc_load_trace", "bc_load_values", "bc_detect", "bc_races", "bc_races_device", "bc_destroy",
            "bc_status_string", "bc_last_error", "bc_phase_name"]
 
 
@@ -79,6 +79,8 @@ def lib():
         L.bc_init.argtypes = [ctypes.POINTER(_Config), ctypes.POINTER(ctypes.c_void_p)]
         L.bc_load_trace.restype = ctypes.c_int
         L.bc_load_trace.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int]
+        L.bc_load_values.restype = ctypes.c_int
+        L.bc_load_values.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int]
         L.bc_detect.restype = ctypes.c_int
         L.bc_detect.argtypes = [ctypes.c_void_p, ctypes.POINTER(_Stats)]
         L.bc_races.restype = ctypes.c_int
@@ -165,6 +167,21 @@ class Context:
         self._keep = a
         return self._check(L.bc_load_trace(self._h, ctypes.c_void_p(a.ctypes.data if n else 0), n, 0))
 
+    def load_values(self, values):
+        """bc_load_values: per-lane store values [n_records, 32] (uint64) as a host
+        numpy array (copied) or a CUDA tensor (borrowed); None clears them."""
+        L = lib()
+        if values is None:
+            return self._check(L.bc_load_values(self._h, None, 0, 0))
+        if hasattr(values, "is_cuda") and values.is_cuda:
+            n = values.numel() // 32
+            self._keep_values = values
+            return self._check(L.bc_load_values(self._h, ctypes.c_void_p(values.data_ptr()), n, 1))
+        a = np.ascontiguousarray(values, dtype=np.uint64).reshape(-1)
+        self._keep_values = a
+        n = len(a) // 32
+        return self._check(L.bc_load_values(self._h, ctypes.c_void_p(a.ctypes.data if n else 0), n, 0))
+
     def detect(self, allow=()):
         """bc_detect; returns (status, stats dict)."""
         s = _Stats()
@@ -249,12 +266,14 @@ class Result:
 
 
 def detect(records, geometry: dict, device="cuda:0", flags: int = 0, stream=None, rank: int = 0,
-           world: int = 1) -> Result:
+           world: int = 1, values=None) -> Result:
     """One-shot bc_init/bc_load_trace/bc_detect/bc_races.  Infeasible traces return
     status -2 with no races (as the oracle does)."""
     dev = int(str(device).split(":")[-1]) if str(device).startswith("cuda") else int(device)
     with Context(geometry, device=dev, flags=flags, stream=stream, rank=rank, world=world) as ctx:
         ctx.load_trace(records)
+        if values is not None:
+            ctx.load_values(values)
         st, stats = ctx.detect(allow=(-2,))
         races = ctx.races() if st == OK else np.zeros(0, dtype=RACE_DTYPE)
         return Result(st, races, stats)

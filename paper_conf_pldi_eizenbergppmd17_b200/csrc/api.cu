@@ -29,6 +29,9 @@ struct bc_ctx {
   u64 n_recs = 0;
   bool loaded = false;
   bool detected = false;
+  const u64* values = nullptr;  // device, per-lane store values (row f3), nullable
+  u64* values_owned = nullptr;
+  size_t values_cap = 0;
   bc_race* races = nullptr;  // device, findings first
   size_t races_cap = 0;
   u64 n_races = 0;
@@ -142,6 +145,7 @@ void bc_destroy(bc_ctx* c) {
   cudaSetDevice(c->cfg.device);
   if (c->stream) cudaStreamSynchronize(c->stream);
   if (c->owned) cudaFree(c->owned);
+  if (c->values_owned) cudaFree(c->values_owned);
   if (c->races) cudaFree(c->races);
   c->arena.free_all();
   for (int i = 0; i < 16; ++i)
@@ -157,6 +161,7 @@ bc_status bc_load_trace(bc_ctx* c, const bc_record* recs, uint64_t n, int on_dev
   cudaSetDevice(c->cfg.device);
   c->loaded = false;
   c->detected = false;
+  c->values = nullptr;
   c->n_recs = n;
   c->g.n_recs = n;
   bool aligned = ((uintptr_t)recs & 15) == 0;
@@ -188,6 +193,7 @@ bc_status bc_load_trace(bc_ctx* c, const bc_record* recs, uint64_t n, int on_dev
 static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   cudaStream_t st = c->stream;
   Geo g = c->g;
+  if (c->values) g.flags |= GEO_F_VALUES;
   const u64 n = g.n_recs;
   const bc_record* recs = c->trace;
   bc_stats& sx = c->stats;
@@ -344,7 +350,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     cudaMemsetAsync(rcnt, 0, 4, st);
     cudaMemsetAsync(segc, 0, 16, st);
     cudaEventRecord(c->ev[10], st);
-    launch_check(hc, skey, sev, n_items_dev, bound, cstatus, rbuf, rcnt, race_cap, segc, st);
+    launch_check(hc, skey, sev, n_items_dev, bound, cstatus, rbuf, rcnt, race_cap, segc, c->values, st);
     cudaEventRecord(c->ev[11], st);
     cudaMemcpyAsync(&n_r, rcnt, 4, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
@@ -396,6 +402,37 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   }
   cudaEventElapsedTime(&sx.ms_kernel[PH_N + 2], c->ev[14], c->ev[15]);
   sx.kernel_launches = g_launches - launches0;
+  return BC_OK;
+}
+
+bc_status bc_load_values(bc_ctx* c, const uint64_t* values, uint64_t n, int on_device) {
+  if (!c) return BC_ERR_INVALID_ARG;
+  if (!c->loaded) return fail(c, BC_ERR_STATE, "bc_load_values before bc_load_trace");
+  c->detected = false;
+  c->values = nullptr;
+  if (!values) return BC_OK;
+  if (n != c->n_recs) return fail(c, BC_ERR_INVALID_ARG, "values: record count differs from the trace");
+  if (n == 0) return BC_OK;
+  cudaSetDevice(c->cfg.device);
+  if (on_device) {
+    if (((uintptr_t)values & 7) != 0) return fail(c, BC_ERR_INVALID_ARG, "values: misaligned device pointer");
+    c->values = (const u64*)values;
+    return BC_OK;
+  }
+  const size_t bytes = (size_t)n * 32 * sizeof(u64);
+  if (c->values_cap < bytes) {
+    if (c->values_owned) cudaFree(c->values_owned);
+    c->values_owned = nullptr;
+    c->values_cap = 0;
+    if (cudaMalloc(&c->values_owned, bytes) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(c, BC_ERR_OOM, "values buffer");
+    }
+    c->values_cap = bytes;
+  }
+  cudaMemcpyAsync(c->values_owned, values, bytes, cudaMemcpyHostToDevice, c->stream);
+  if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_check(c, "values copy");
+  c->values = c->values_owned;
   return BC_OK;
 }
 

@@ -59,7 +59,15 @@ struct CheckArgs {
   u32* race_cnt;
   u32 race_cap;
   u64* seg_cnt;  // [0] segments, [1] clock snapshot gathers
+  const u64* values;  // per-lane store values (row f3), nullable
 };
+
+// intra-warp same-value filter: two stores of one record; with per-lane values
+// (reading R6b) they must store the same value, else the record's SAME_VALUE flag decides
+// (the item op is IOP_ST_SV)
+__device__ __forceinline__ bool same_value(const CheckArgs& a, u32 ev_prior, u32 ev_cur) {
+  return (ev_prior >> 5) == (ev_cur >> 5) && (!a.values || a.values[ev_prior] == a.values[ev_cur]);
+}
 
 __device__ __forceinline__ void emit(const CheckArgs& a, u32 key, u32 cur, u32 prior, u32 kind) {
   u32 at = atomicAdd(a.race_cnt, 1u);
@@ -377,7 +385,7 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
         } else if (op == IOP_ATOM) {
           emit(a, key, ev, pev2, BC_KIND_WA);
         } else {
-          const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (pev2 >> 5) == (ev >> 5);
+          const bool filtered = !patm && op == IOP_ST_SV && !no_sv && same_value(a, pev2, ev);
           if (!filtered) emit(a, key, ev, pev2, patm ? BC_KIND_AW : BC_KIND_WW);
         }
       }
@@ -672,7 +680,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
         if (lw && !(op == IOP_ATOM && patm) && !hbq(c, we, ww, e, s2)) {
           const u32 kind = op == IOP_LD ? (patm ? BC_KIND_AR : BC_KIND_WR)
                                         : op == IOP_ATOM ? BC_KIND_WA : (patm ? BC_KIND_AW : BC_KIND_WW);
-          const bool filtered = !patm && op == IOP_ST_SV && !no_sv && (we >> 5) == (e >> 5);
+          const bool filtered = !patm && op == IOP_ST_SV && !no_sv && same_value(a, we, e);
           if (!filtered) emit(a, k >> 2, e, we, kind);
         }
         if (op != IOP_LD) {
@@ -739,7 +747,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
 size_t check_status_bytes(u64 n) { return (size_t)148 * 64 * sizeof(WarpEnd) + 256; }
 
 void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_dev, u64 n_max, void* status,
-                  uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, cudaStream_t st) {
+                  uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, const u64* values, cudaStream_t st) {
   if (n_max == 0) return;
   // K7 variant: lane-sequential with shared-memory staged clocks (default) or ballot rounds
   // (BC_K7=ballot); read at every launch so that tests can switch it
@@ -775,6 +783,7 @@ void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_
   a.race_cnt = race_cnt;
   a.race_cap = race_cap;
   a.seg_cnt = seg_cnt;
+  a.values = values;
   if (use_tile) {
     k_check_tile<<<grid, KT_WARPS * 32, smem_tile, st>>>(a, (WarpEnd*)status, nw);
   } else {

@@ -38,6 +38,9 @@ constexpr u32 KEY_DROP = 0xFFFFFFFFu;
 constexpr u32 KEY_BLOCK = 0x80000000u;  // block-level entry: key = KEY_BLOCK | block
 constexpr u32 KEY_LINK = 0xC0000000u;   // link entry:        key = KEY_LINK | target array
 constexpr u32 SYNC_LOOKUP_CAP = 1u << 16;  // step cap of one foreign lookup
+// internal Geo.flags bit: per-lane store values are loaded (row f3, reading R6b): every store item
+// is a same-value filter candidate and K7 compares the two lanes' values
+constexpr u32 GEO_F_VALUES = 0x80000000u;
 
 struct Geo {
   u32 n_blocks, tpb, wpb, n_warps;

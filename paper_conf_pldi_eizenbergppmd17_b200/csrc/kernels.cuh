@@ -102,7 +102,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
 // check.cu
 size_t check_status_bytes(u64 n);
 void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_dev, u64 n_max, void* status,
-                  uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, cudaStream_t st);
+                  uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, const u64* values, cudaStream_t st);
 
 // finalize.cu
 void launch_page_list(const u32* words, const u32* wl_prefix, const u32* page_bits, u64 n_words, u32* page_num,

@@ -428,7 +428,8 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
       u32 nk = (u32)(size >> g.G);
       if (nk == 0) nk = 1;
       const u32 opc = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM
-                                                               : ((fl & BC_REC_SAME_VALUE) ? IOP_ST_SV : IOP_ST);
+                                                               : (((fl & BC_REC_SAME_VALUE) || (g.flags & GEO_F_VALUES))
+                                                                      ? IOP_ST_SV : IOP_ST);
       u32 key0 = KEY_DROP;
       if (bad) {
       } else if (space == BC_SPACE_SHARED) {

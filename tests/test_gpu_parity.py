@@ -308,7 +308,8 @@ def test_c6_hashtable(bug):
             assert "OVERFLOW" in str(ei.value)
             continue
         want, _ = assert_parity(recs, plan.geometry)
-        assert (len(want) == 0) == (bug == 0)
+        if i > 0:  # (one warp alone: its lanes' turns are ordered by the FI joins anyway)
+            assert (len(want) == 0) == (bug == 0)
 
 
 def test_c6_hashtable_bench_shape():
@@ -324,3 +325,50 @@ def test_c6_full_size():
     plan = ConfigPlan(6)
     want, res = assert_parity(plan.records(), plan.geometry)
     assert len(want) > 100_000
+
+
+# ------------------------------------------- per-lane store values (reading R6b)
+def test_values_random_traces():
+    """bc_load_values: the same-value filter compares per-lane store values; parity with the
+    oracle on random traces (values partly uniform, partly colliding), host and device values."""
+    import torch
+    from bcgen.fuzz import random_values
+    for seed in range(8000, 8060):
+        recs, tb = random_trace(seed, same_value=True, n_glob=2)
+        geom = tb.geom.as_dict()
+        vals = random_values(recs, seed)
+        st_o, want, _ = oracle.detect_geom(recs, geom, values=vals)
+        res = bc.detect(recs, geom, device="cuda:0", values=vals)
+        assert res.status == st_o
+        if st_o == 0:
+            assert np.array_equal(res.races.view(np.uint8), want.view(np.uint8)), seed
+    recs, tb = random_trace(8100, same_value=True, n_glob=2)
+    geom = tb.geom.as_dict()
+    vals = random_values(recs, 8100)
+    st_o, want, _ = oracle.detect_geom(recs, geom, values=vals)
+    with bc.Context(geom, device=0) as ctx:
+        ctx.load_trace(recs)
+        ctx.load_values(torch.from_numpy(vals).cuda())
+        assert ctx.detect()[0] == 0
+        assert np.array_equal(ctx.races().view(np.uint8), want.view(np.uint8))
+        ctx.load_values(None)  # cleared: back to the record flags
+        assert ctx.detect()[0] == 0
+        st_f, want_f, _ = oracle.detect_geom(recs, geom)
+        assert np.array_equal(ctx.races().view(np.uint8), want_f.view(np.uint8))
+
+
+@pytest.mark.parametrize("variant", ["ballot", "tile"])
+def test_values_k7_variants_byte_granules(variant, monkeypatch):
+    """Values with byte granules (G = 0, the paper's default) and mixed access
+    sizes, through both K7 formulations."""
+    from bcgen.fuzz import random_values
+    monkeypatch.setenv("BC_K7", variant)
+    for seed in range(8200, 8240):
+        recs, tb = random_trace(seed, same_value=True, n_glob=2, granule_log2=0)
+        geom = tb.geom.as_dict()
+        vals = random_values(recs, seed)
+        st_o, want, _ = oracle.detect_geom(recs, geom, values=vals)
+        res = bc.detect(recs, geom, device="cuda:0", values=vals)
+        assert res.status == st_o
+        if st_o == 0:
+            assert np.array_equal(res.races.view(np.uint8), want.view(np.uint8)), seed

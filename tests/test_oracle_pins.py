@@ -47,10 +47,10 @@ def loc_of(r, G=2):
     return (sp, int(r["block"]) if sp == 1 else 0, int(r["addr"]) >> G)
 
 
-def check_against_bf(recs, geom, races, strict=True):
+def check_against_bf(recs, geom, races, strict=True, values=None):
     """Soundness always; first racy event + verdict per valid granule."""
     G = geom["granule_log2"]
-    bf = brute_force(recs, geom["grid"], geom["block"], G)
+    bf = brute_force(recs, geom["grid"], geom["block"], G, values=values)
     bfset = bf.race_set()
     orset = {(loc_of(r, G), int(r["prior_event"]), int(r["cur_event"])) for r in races if r["cls"] != 4}
     assert orset <= bfset, sorted(orset - bfset)[:5]
@@ -356,3 +356,56 @@ def test_c6_hashtable_race_structure(bug):
         assert lock_races and kinds == {KIND_NAMES.index("WW")}
     else:
         assert lock_races and kinds == {KIND_NAMES.index("WA")}
+
+
+# ------------------------------------------- per-lane store values (reading R6b)
+def test_values_worked_example():
+    """P:L577-581 with values: four lanes of ONE store record write one granule with values
+    (a, a, b, a).  Lanes run in ascending order (R5): lane 1 stores lane 0's value (filtered),
+    lane 2 differs from lane 1 (race), lane 3 differs from lane 2 (race): exactly two WW
+    SAME_INSN races, (l1, l2) and (l2, l3).  The SAME_VALUE flag alone would filter all three."""
+    tb = TraceBuilder(block=(32,))
+    r = tb.st(0, lambda l: GLOBAL_BASE if l < 4 else GLOBAL_BASE + 64 + 4 * l)
+    recs = tb.records()
+    vals = np.zeros((len(recs), 32), dtype=np.uint64)
+    vals[0, :4] = [7, 7, 9, 7]
+    st, races, _ = oracle.detect_geom(recs, tb.geom.as_dict(), values=vals)
+    assert st == 0
+    got = sorted((int(x["prior_event"]) & 31, int(x["cur_event"]) & 31, int(x["kind"]), int(x["cls"])) for x in races)
+    assert got == [(1, 2, KIND_NAMES.index("WW"), 0), (2, 3, KIND_NAMES.index("WW"), 0)]
+    # all equal -> no race; the flag gives the same answer as uniform values
+    vals[0, :4] = 5
+    assert len(oracle.detect_geom(recs, tb.geom.as_dict(), values=vals)[1]) == 0
+
+
+@pytest.mark.parametrize("chunk", range(3))
+def test_values_uniform_equals_flag(chunk):
+    """Special case that reduces to the flag: values that are uniform inside every SAME_VALUE
+    record and pairwise distinct elsewhere give exactly the flag's race set."""
+    from bcgen.format import OP_ST, FLAG_SAME_VALUE
+    for seed in range(6000 + 40 * chunk, 6040 + 40 * chunk):
+        recs, tb = random_trace(seed, same_value=True)
+        geom = tb.geom.as_dict()
+        vals = np.zeros((len(recs), 32), dtype=np.uint64)
+        for i, r in enumerate(recs):
+            if int(r["op"]) == OP_ST:
+                vals[i, :] = 1 if int(r["flags"]) & FLAG_SAME_VALUE else np.arange(32) + 100
+        st1, want, _ = oracle.detect_geom(recs, geom)
+        st2, got, _ = oracle.detect_geom(recs, geom, values=vals)
+        assert st1 == st2
+        assert np.array_equal(got.view(np.uint8), want.view(np.uint8))
+
+
+@pytest.mark.parametrize("chunk", range(3))
+def test_values_vs_bruteforce(chunk):
+    """With per-lane values the oracle's pairs are §3.2 pairs under the value filter, and its
+    first race per granule is brute force's on the valid class."""
+    from bcgen.fuzz import random_values
+    for seed in range(7000 + 40 * chunk, 7040 + 40 * chunk):
+        recs, tb = random_trace(seed, same_value=True, n_glob=2)
+        geom = tb.geom.as_dict()
+        vals = random_values(recs, seed)
+        st, races, _ = oracle.detect_geom(recs, geom, values=vals)
+        if st != 0:
+            continue
+        check_against_bf(recs, geom, races, values=vals)
