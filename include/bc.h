@@ -132,6 +132,8 @@ typedef struct bc_stats {
 } bc_stats;
 
 /* ------------------------------------------------------------------------- calls */
+typedef struct bc_ctx bc_ctx; /* opaque: one context per process / rank, not thread-safe          */
+
 /* Create a context for one traced launch geometry. */
 bc_status bc_init(const bc_config* cfg, struct bc_ctx** out);
 
