@@ -88,4 +88,5 @@ def detect(records: np.ndarray, grid=(1, 1, 1), block=(32, 1, 1), smem_bytes=0, 
 
 def detect_geom(records, geom: dict, flags=0, values=None):
     return detect(records, grid=geom["grid"], block=geom["block"], smem_bytes=geom["smem_bytes"],
-                  granule_log2=geom.get("granule_log2", 2), flags=flags, values=values)
+                  granule_log2=geom.get("granule_log2", 2), flags=flags, values=values,
+                  warp_size=geom.get("warp_size", 32))

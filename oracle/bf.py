@@ -60,7 +60,7 @@ class BFResult:
 
 
 def brute_force(records: np.ndarray, grid=(1, 1, 1), block=(32, 1, 1), granule_log2=2,
-                same_value_filter=True, values=None):
+                same_value_filter=True, values=None, warp_size=32):
     """values: optional per-lane store values [n_records, 32] (reading R6b): two stores of one
     record race only if they store different values (instead of the SAME_VALUE flag)."""
     vals = None if values is None else np.asarray(values, dtype=np.uint64).reshape(-1)
@@ -68,15 +68,16 @@ def brute_force(records: np.ndarray, grid=(1, 1, 1), block=(32, 1, 1), granule_l
     block = tuple(block) + (1,) * (3 - len(block))
     nb = grid[0] * grid[1] * grid[2]
     tpb = block[0] * block[1] * block[2]
-    wpb = (tpb + 31) // 32
+    ws = warp_size
+    wpb = (tpb + ws - 1) // ws
     G = granule_log2
 
     def init_mask(w):
-        lanes = min(32, tpb - (w % wpb) * 32)
+        lanes = min(ws, tpb - (w % wpb) * ws)
         return (1 << lanes) - 1
 
     def tid(w, l):
-        return (w // wpb) * tpb + (w % wpb) * 32 + l
+        return (w // wpb) * tpb + (w % wpb) * ws + l
 
     res = BFResult()
     anc = res.anc

@@ -151,14 +151,16 @@ struct LocHash {
   }
 };
 
+// ws = warp size: 32, or 4 / 8 / 16 when simulating smaller warps:
+// warp w of a block holds threads (w % wpb) * ws ... + ws - 1 of it in lanes 0 .. ws-1.
 struct Geom {
-  uint32_t n_blocks, tpb, wpb, n_warps, n_threads, G, smem;
+  uint32_t n_blocks, tpb, wpb, n_warps, n_threads, G, smem, ws;
   uint32_t init_mask(uint32_t w) const {
-    uint32_t lanes = std::min<uint32_t>(32, tpb - (w % wpb) * 32);
+    uint32_t lanes = std::min<uint32_t>(ws, tpb - (w % wpb) * ws);
     return lanes == 32 ? 0xFFFFFFFFu : ((1u << lanes) - 1);
   }
   uint32_t block_of_warp(uint32_t w) const { return w / wpb; }
-  uint32_t tid(uint32_t w, int lane) const { return (w / wpb) * tpb + (w % wpb) * 32 + lane; }
+  uint32_t tid(uint32_t w, int lane) const { return (w / wpb) * tpb + (w % wpb) * ws + lane; }
 };
 
 enum EntryKind { ROOT, ELSE_ENTRY, THEN_ENTRY };
@@ -497,7 +499,8 @@ int oracle_detect(const void* recs, uint64_t n_recs, const oracle_geom* gm, orac
 int oracle_detect_values(const void* recs, uint64_t n_recs, const oracle_geom* gm, const uint64_t* values,
                          oracle_result* res) {
   if (!gm || !res || (n_recs && !recs)) return -1;
-  if (gm->warp_size != 32 || gm->granule_log2 > 4) return -1;
+  const uint32_t ws = gm->warp_size;
+  if ((ws != 4 && ws != 8 && ws != 16 && ws != 32) || gm->granule_log2 > 4) return -1;
   Oracle o;
   o.recs = (const Record*)recs;
   o.values = values;
@@ -508,7 +511,8 @@ int oracle_detect_values(const void* recs, uint64_t n_recs, const oracle_geom* g
   if (nb == 0 || tpb == 0 || tpb > 1024 || nb * tpb > 0xFFFFFFFFull) return -1;
   o.g.n_blocks = (uint32_t)nb;
   o.g.tpb = (uint32_t)tpb;
-  o.g.wpb = (uint32_t)((tpb + 31) / 32);
+  o.g.ws = ws;
+  o.g.wpb = (uint32_t)((tpb + ws - 1) / ws);
   o.g.n_warps = o.g.n_blocks * o.g.wpb;
   o.g.n_threads = (uint32_t)(nb * tpb);
   o.g.G = gm->granule_log2;

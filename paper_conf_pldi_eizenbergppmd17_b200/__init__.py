@@ -129,7 +129,7 @@ class Context:
         c = _Config()
         for i in range(3):
             c.grid_dim[i], c.block_dim[i] = grid[i], block[i]
-        c.warp_size = 32
+        c.warp_size = geometry.get("warp_size", 32)  # 4 / 8 / 16: warp-size simulation (row f4)
         c.granule_log2 = geometry.get("granule_log2", 2)
         c.smem_bytes_per_block = geometry.get("smem_bytes", 0)
         c.flags = flags

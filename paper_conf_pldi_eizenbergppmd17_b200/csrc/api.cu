@@ -86,14 +86,15 @@ const char* bc_phase_name(int i) { return (i >= 0 && i < PH_N + 3) ? kPhase[i] :
 bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   if (!cfg || !out) return BC_ERR_INVALID_ARG;
   *out = nullptr;
-  if (cfg->warp_size != 32 || cfg->granule_log2 > 4) return BC_ERR_INVALID_ARG;
+  const u32 ws = cfg->warp_size;  // 32, or a simulated smaller warp
+  if ((ws != 4 && ws != 8 && ws != 16 && ws != 32) || cfg->granule_log2 > 4) return BC_ERR_INVALID_ARG;
   if (cfg->flags & ~(u32)(BC_F_NO_SAME_VALUE_FILTER)) return BC_ERR_INVALID_ARG;  // overwrite: not on GPU yet
   if (cfg->world < 0 || cfg->world > 1024) return BC_ERR_INVALID_ARG;
   if (cfg->world > 1 && (cfg->rank < 0 || cfg->rank >= cfg->world)) return BC_ERR_INVALID_ARG;
   u64 nb = (u64)cfg->grid_dim[0] * cfg->grid_dim[1] * cfg->grid_dim[2];
   u64 tpb = (u64)cfg->block_dim[0] * cfg->block_dim[1] * cfg->block_dim[2];
   if (nb == 0 || tpb == 0 || tpb > 1024 || nb * tpb > 0xFFFFFFFFull) return BC_ERR_INVALID_ARG;
-  u64 wpb = (tpb + 31) / 32;
+  u64 wpb = (tpb + ws - 1) / ws;
   if (nb * wpb >= (1ull << 30) || nb * wpb * wpb >= (1ull << 32)) return BC_ERR_INVALID_ARG;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
@@ -110,6 +111,7 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   g.n_blocks = (u32)nb;
   g.tpb = (u32)tpb;
   g.wpb = (u32)wpb;
+  g.ws = ws;
   g.n_warps = (u32)(nb * wpb);
   g.wpb_m = wpb == 1 ? 0u : (u32)(((1ull << 32) + wpb - 1) / wpb);
   g.world = cfg->world > 1 ? (u32)cfg->world : 1u;

@@ -44,6 +44,7 @@ constexpr u32 GEO_F_VALUES = 0x80000000u;
 
 struct Geo {
   u32 n_blocks, tpb, wpb, n_warps;
+  u32 ws;          // warp size: 32, or 4 / 8 / 16 for warp-size simulation
   u32 wpb_m;       // ceil(2^32 / wpb), 0 when wpb == 1: block of warp w = umulhi(w, wpb_m) (exact: n_warps * wpb < 2^32)
   u32 rank, world; // address sharding: this context checks the granules g with shard_of(g) == rank
   u32 G;           // granule_log2
@@ -69,7 +70,8 @@ __device__ __forceinline__ u32 blk_of(const Geo& g, u32 w) { return g.wpb_m ? __
 
 __host__ __device__ inline u32 init_mask(const Geo& g, u32 w) {
   u32 wib = w % g.wpb;
-  u32 lanes = g.tpb - wib * 32u;
+  u32 lanes = g.tpb - wib * g.ws;
+  if (lanes > g.ws) lanes = g.ws;
   return lanes >= 32u ? 0xFFFFFFFFu : ((1u << lanes) - 1u);
 }
 

@@ -322,7 +322,7 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
 // at the last arrival R_k = max over the block's warps of their k-th BAR record; its step is
 // labelled R_k + 1 for every thread of the block.  A warp whose next record after its k-th
 // BAR precedes R_k issued a record while waiting -> infeasible.  One warp per traced block; lane l
-// handles barriers l, l+32, ... (warps per block <= 32, so lane i also checks warp i's count).
+// handles barriers l, l+32, ... and checks the counts of warps l, l+32, ...
 __global__ void __launch_bounds__(256) k_barriers(Geo g, const u32* __restrict__ bar_cnt,
                                                   const u32* __restrict__ bar_base, const u32* __restrict__ bar_rec,
                                                   const u32* __restrict__ bar_next, u32* __restrict__ blockR,
@@ -332,7 +332,8 @@ __global__ void __launch_bounds__(256) k_barriers(Geo g, const u32* __restrict__
   if (b >= g.n_blocks) return;  // warp-uniform
   const u32 w0 = b * g.wpb;
   const u32 nb = bar_cnt[w0];
-  const bool diff = lane < g.wpb && bar_cnt[w0 + lane] != nb;
+  bool diff = false;
+  for (u32 i = lane; i < g.wpb; i += 32) diff |= bar_cnt[w0 + i] != nb;  // (wpb > 32: simulated small warps)
   if (__any_sync(0xFFFFFFFFu, diff)) {
     if (lane == 0) set_err(err, ERR_INFEASIBLE);
     return;

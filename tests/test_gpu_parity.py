@@ -372,3 +372,29 @@ def test_values_k7_variants_byte_granules(variant, monkeypatch):
         assert res.status == st_o
         if st_o == 0:
             assert np.array_equal(res.races.view(np.uint8), want.view(np.uint8)), seed
+
+
+# ------------------------------------------------ warp-size simulation
+@pytest.mark.parametrize("ws", [16, 8, 4])
+def test_warpsim_random_traces(ws):
+    """Traces re-split into virtual warps of ws lanes (bcgen.warpsim): bc_config.warp_size = ws;
+    bit-exact with the oracle (infeasible splits -- a BAR inside warp-divergent code -- must be
+    rejected by both)."""
+    from bcgen.warpsim import split_warps
+    for seed in range(9100, 9160):
+        recs, tb = random_trace(seed)
+        r2, g2, _ = split_warps(recs, tb.geom.as_dict(), ws)
+        assert_parity(r2, g2)
+
+
+@pytest.mark.parametrize("cfg,kw", [(2, dict(n_blocks=4, iters=3)), (3, dict(n_blocks=6, iters=2, tpb=64)),
+                                    (4, dict(n_blocks=8, log2_nodes=13, nodes_per_thread=2, inj_scale=4))])
+def test_warpsim_configs(cfg, kw):
+    """C2-C4 shapes with 16- and 8-lane virtual warps (block sizes up to 256 threads = 32 virtual
+    warps of 8)."""
+    from bcgen.warpsim import split_warps
+    plan = ConfigPlan(cfg, **kw)
+    recs = plan.records()
+    for ws in (16, 8):
+        r2, g2, _ = split_warps(recs, plan.geometry, ws)
+        assert_parity(r2, g2)

@@ -50,7 +50,7 @@ def loc_of(r, G=2):
 def check_against_bf(recs, geom, races, strict=True, values=None):
     """Soundness always; first racy event + verdict per valid granule."""
     G = geom["granule_log2"]
-    bf = brute_force(recs, geom["grid"], geom["block"], G, values=values)
+    bf = brute_force(recs, geom["grid"], geom["block"], G, values=values, warp_size=geom.get("warp_size", 32))
     bfset = bf.race_set()
     orset = {(loc_of(r, G), int(r["prior_event"]), int(r["cur_event"])) for r in races if r["cls"] != 4}
     assert orset <= bfset, sorted(orset - bfset)[:5]
@@ -409,3 +409,55 @@ def test_values_vs_bruteforce(chunk):
         if st != 0:
             continue
         check_against_bf(recs, geom, races, values=vals)
+
+
+# ------------------------------------------------ warp-size simulation
+def _exchange_trace():
+    """one 32-thread block: st.shared s[lane]; ld.shared s[lane ^ 16] (warp-synchronous exchange,
+    correct only because the 32 lanes execute in lock step)"""
+    tb = TraceBuilder(block=(32,), smem_bytes=256)
+    from bcgen import SPACE_SHARED
+    tb.st(0, lambda l: 4 * l, space=SPACE_SHARED)
+    tb.ld(0, lambda l: 4 * (l ^ 16), space=SPACE_SHARED)
+    return tb.records(), tb.geom.as_dict()
+
+
+def test_warpsim_identity_at_32():
+    from bcgen.warpsim import split_warps
+    recs, tb = random_trace(11)
+    r2, g2, org = split_warps(recs, tb.geom.as_dict(), 32)
+    assert np.array_equal(r2.view(np.uint8), recs.view(np.uint8))
+    assert np.array_equal(run(r2, g2).view(np.uint8), run(recs, tb.geom.as_dict()).view(np.uint8))
+
+
+@pytest.mark.parametrize("ws", [16, 8, 4])
+def test_warpsim_exchange_worked_example(ws):
+    """The exchange is race-free with 32-wide warps (the endi of the store orders every lane's
+    store before every lane's load) and has exactly 32 WR INTRA_BLOCK races with
+    virtual warps of 16, 8 or 4 lanes: every load reads a granule stored by a lane 16 away, which
+    is in another virtual warp, and nothing orders two warps of a block but a barrier."""
+    from bcgen.warpsim import split_warps
+    recs, geom = _exchange_trace()
+    assert len(run(recs, geom)) == 0
+    r2, g2, org = split_warps(recs, geom, ws)
+    races = run(r2, g2)
+    assert len(races) == 32
+    assert {(int(r["kind"]), int(r["cls"])) for r in races} == {(KIND_NAMES.index("WR"), 2)}
+    # reported against the recorded trace: prior = the store of lane l ^ 16, current = the load of lane l
+    for r in races:
+        pr, pl = org[int(r["prior_event"]) >> 5][0], org[int(r["prior_event"]) >> 5][1] + (int(r["prior_event"]) & 31)
+        cr, cl = org[int(r["cur_event"]) >> 5][0], org[int(r["cur_event"]) >> 5][1] + (int(r["cur_event"]) & 31)
+        assert (pr, cr) == (0, 1) and pl == cl ^ 16
+    check_against_bf(r2, g2, races)
+
+
+@pytest.mark.parametrize("ws", [16, 8])
+def test_warpsim_random_vs_bruteforce(ws):
+    from bcgen.warpsim import split_warps
+    for seed in range(9000, 9040):
+        recs, tb = random_trace(seed, p_bar=0.0, max_bars=0)
+        r2, g2, _ = split_warps(recs, tb.geom.as_dict(), ws)
+        st, races, _ = oracle.detect_geom(r2, g2)
+        if st != 0:
+            continue
+        check_against_bf(r2, g2, races)
