@@ -95,7 +95,8 @@ typedef struct bc_race {
 enum {
   BC_F_RELEASE_OVERWRITE = 1u,    /* printed S_x := C_t release (reading R1 uses join); not yet
                                      supported on the GPU path -> BC_ERR_INVALID_ARG            */
-  BC_F_NO_SAME_VALUE_FILTER = 2u  /* report intra-warp same-value WW races too (R6)           */
+  BC_F_NO_SAME_VALUE_FILTER = 2u, /* report intra-warp same-value WW races too (R6)           */
+  BC_F_COUNT_GATHERS = 4u         /* statistics: fill bc_stats.clock_gathers (one extra pass)  */
 };
 
 typedef struct bc_config {
@@ -124,8 +125,8 @@ typedef struct bc_stats {
   uint64_t sync_ops;         /* acquire / release lane operations                                 */
   uint64_t written_pages;    /* 1-MB global pages with at least one write          */
   uint64_t kernel_launches;  /* libbc kernels launched by this bc_detect                          */
-  uint64_t clock_gathers;    /* 16-B record clock snapshots the per-granule check read (items that
-                                some happens-before check needs)                                 */
+  uint64_t clock_gathers;    /* 16-B record clock snapshots the per-granule check reads (items that
+                                some happens-before check needs); 0 unless BC_F_COUNT_GATHERS    */
   float ms_total;            /* device time of bc_detect (cudaEvents on the stream)               */
   float ms_kernel[12];       /* per phase, then kernel-only k_check / k_sort_items / k_expand;
                                 see bc_phase_name()                                              */

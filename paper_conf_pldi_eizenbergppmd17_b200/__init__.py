@@ -36,6 +36,7 @@ STATUS = {0: "OK", -1: "INVALID_ARG", -2: "INFEASIBLE_TRACE", -3: "OOM", -4: "CU
           -6: "STATE", -7: "TRUNCATED", -8: "OVERFLOW"}
 F_RELEASE_OVERWRITE = 1
 F_NO_SAME_VALUE_FILTER = 2
+F_COUNT_GATHERS = 4  # statistics: fill stats["clock_gathers"] (one extra pass)
 
 EXPORTS = ["bc_init", "bc_load_trace", "bc_load_values", "bc_detect", "bc_races", "bc_races_device", "bc_destroy",
            "bc_status_string", "bc_last_error", "bc_phase_name"]

@@ -88,7 +88,7 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   *out = nullptr;
   const u32 ws = cfg->warp_size;  // 32, or a simulated smaller warp
   if ((ws != 4 && ws != 8 && ws != 16 && ws != 32) || cfg->granule_log2 > 4) return BC_ERR_INVALID_ARG;
-  if (cfg->flags & ~(u32)(BC_F_NO_SAME_VALUE_FILTER)) return BC_ERR_INVALID_ARG;  // overwrite: not on GPU yet
+  if (cfg->flags & ~(u32)(BC_F_NO_SAME_VALUE_FILTER | BC_F_COUNT_GATHERS)) return BC_ERR_INVALID_ARG;  // overwrite: not on GPU yet
   if (cfg->world < 0 || cfg->world > 1024) return BC_ERR_INVALID_ARG;
   if (cfg->world > 1 && (cfg->rank < 0 || cfg->rank >= cfg->world)) return BC_ERR_INVALID_ARG;
   u64 nb = (u64)cfg->grid_dim[0] * cfg->grid_dim[1] * cfg->grid_dim[2];
@@ -354,6 +354,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     cudaEventRecord(c->ev[10], st);
     launch_check(hc, skey, sev, n_items_dev, bound, cstatus, rbuf, rcnt, race_cap, segc, c->values, st);
     cudaEventRecord(c->ev[11], st);
+    if (g.flags & BC_F_COUNT_GATHERS) launch_count_gathers(skey, n_items_dev, segc + 1, st);
     cudaMemcpyAsync(&n_r, rcnt, 4, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
     cudaMemcpyAsync(&sx.segments, segc, 8, cudaMemcpyDeviceToHost, st);

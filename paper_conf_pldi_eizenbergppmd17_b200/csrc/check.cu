@@ -252,7 +252,7 @@ __device__ bool walk_back(const CheckArgs& a, u64 s, Sum& out) {
 // traces (C4/C5 cost/mask) this removes almost all random 16-B gathers.
 constexpr int K7_PS = 2;
 
-__device__ __forceinline__ uint4 snap_if_needed(const HbCtx& c, u32 k, u32 e, u32 kprev0, u32 knext31, u32& gat) {
+__device__ __forceinline__ uint4 snap_if_needed(const HbCtx& c, u32 k, u32 e, u32 kprev0, u32 knext31) {
   const int lane = threadIdx.x & 31;
   u32 kp = __shfl_up_sync(0xFFFFFFFFu, k, 1), kn = __shfl_down_sync(0xFFFFFFFFu, k, 1);
   if (lane == 0) kp = kprev0;
@@ -262,7 +262,6 @@ __device__ __forceinline__ uint4 snap_if_needed(const HbCtx& c, u32 k, u32 e, u3
   const bool sp = kp != NONE && (kp >> 2) == key, sn = kn != NONE && (kn >> 2) == key;
   const bool atm_only = (k & 3u) == IOP_ATOM && (!sp || (kp & 3u) == IOP_ATOM) && (!sn || (kn & 3u) == IOP_ATOM);
   if ((!sp && !sn) || atm_only) return make_uint4(0, 0, 0, 0);
-  ++gat;
   return __ldg(c.snap + (e >> 5));
 }
 
@@ -305,7 +304,7 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
 
   // ---- the range, round by round
   const u32 no_sv = c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
-  u32 segs = 0, gat = 0;
+  u32 segs = 0;
   u32 pf_k[K7_PF], pf_e[K7_PF];
   uint4 pf_s[K7_PS];
 #pragma unroll
@@ -318,7 +317,7 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
   for (int q = 0; q < K7_PS; ++q) {
     const u32 kp0 = q == 0 ? pkx : __shfl_sync(0xFFFFFFFFu, pf_k[q > 0 ? q - 1 : 0], 31);
     const u32 kn31 = __shfl_sync(0xFFFFFFFFu, pf_k[q + 1], 0);
-    pf_s[q] = snap_if_needed(c, pf_k[q], pf_e[q], kp0, kn31, gat);
+    pf_s[q] = snap_if_needed(c, pf_k[q], pf_e[q], kp0, kn31);
   }
   for (u64 base_r = beg; base_r < end; base_r += 32) {
     const u64 i = base_r + lane;
@@ -338,7 +337,7 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
       pf_e[K7_PF - 1] = ip < end ? a.evs[ip] : 0u;
       const u32 kp0 = __shfl_sync(0xFFFFFFFFu, K7_PS >= 2 ? pf_k[K7_PS >= 2 ? K7_PS - 2 : 0] : kx, 31);
       const u32 kn31 = __shfl_sync(0xFFFFFFFFu, pf_k[K7_PS], 0);
-      pf_s[K7_PS - 1] = snap_if_needed(c, pf_k[K7_PS - 1], pf_e[K7_PS - 1], kp0, kn31, gat);
+      pf_s[K7_PS - 1] = snap_if_needed(c, pf_k[K7_PS - 1], pf_e[K7_PS - 1], kp0, kn31);
     }
     u32 qkx = __shfl_up_sync(0xFFFFFFFFu, kx, 1);
     u32 qev = __shfl_up_sync(0xFFFFFFFFu, ev, 1);
@@ -419,10 +418,8 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
     pev = __shfl_sync(0xFFFFFFFFu, ev, last);
     pw = __shfl_sync(0xFFFFFFFFu, s2.warp, last);
   }
-  gat = __reduce_add_sync(0xFFFFFFFFu, gat);
   if (lane == 0) {
     if (segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)segs);
-    if (gat) atomicAdd((unsigned long long*)(a.seg_cnt + 1), (unsigned long long)gat);
     volatile WarpEnd* me = &wend[w];
     me->lk = carry.lk;
     me->lw = carry.lw;
@@ -548,7 +545,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
     }
   }
 
-  u32 segs = 0, gat = 0;
+  u32 segs = 0;
   const u32 l0 = lane * KT_IPL;
   if (beg < end) kt_stage(a, beg, (u32)(end - beg < (u64)KT_BLK ? end - beg : (u64)KT_BLK), sKE, sKE + KT_PITCH, lane);
   for (u64 bb = beg; bb < end; bb += KT_BLK) {
@@ -578,10 +575,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
         const bool sp = kp != NONE && (kp >> 2) == key, sn = kn != NONE && (kn >> 2) == key;
         const bool atm_only =
             (k & 3u) == IOP_ATOM && (!sp || (kp & 3u) == IOP_ATOM) && (!sn || (kn & 3u) == IOP_ATOM);
-        if ((sp || sn) && !atm_only) {
-          cp_async16(sS + tpad(li), c.snap + (sE[tpad(li)] >> 5));
-          ++gat;
-        }
+        if ((sp || sn) && !atm_only) cp_async16(sS + tpad(li), c.snap + (sE[tpad(li)] >> 5));
         kp = k;
         k = kn;
       }
@@ -729,10 +723,8 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
     __syncwarp();
   }
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);
-  gat = __reduce_add_sync(0xFFFFFFFFu, gat);
   if (lane == 0) {
     if (segs) atomicAdd((unsigned long long*)a.seg_cnt, (unsigned long long)segs);
-    if (gat) atomicAdd((unsigned long long*)(a.seg_cnt + 1), (unsigned long long)gat);
     volatile WarpEnd* me = &wend[w];
     me->lk = carry.lk;
     me->lw = carry.lw;
@@ -742,7 +734,29 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
   }
 }
 
+// Statistics only (bc_config.flags & BC_F_COUNT_GATHERS): the number of items whose record clock
+// snapshot K7 reads -- the snap_if_needed rule over the sorted items -- for the roofline's
+// algorithmic bytes.  A separate pass so that the hot kernels carry no counter.
+__global__ void k_count_gathers(const u32* __restrict__ keys, const u64* __restrict__ n_dev, u64* __restrict__ out) {
+  const u64 n = *n_dev;
+  u32 cnt = 0;
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) {
+    const u32 k = keys[i], kp = i ? keys[i - 1] : NONE, kn = i + 1 < n ? keys[i + 1] : NONE;
+    const u32 key = k >> 2;
+    const bool sp = kp != NONE && (kp >> 2) == key, sn = kn != NONE && (kn >> 2) == key;
+    const bool atm_only = (k & 3u) == IOP_ATOM && (!sp || (kp & 3u) == IOP_ATOM) && (!sn || (kn & 3u) == IOP_ATOM);
+    cnt += (sp || sn) && !atm_only;
+  }
+  cnt = __reduce_add_sync(0xFFFFFFFFu, cnt);
+  if ((threadIdx.x & 31) == 0 && cnt) atomicAdd((unsigned long long*)out, (unsigned long long)cnt);
+}
+
 }  // namespace
+
+void launch_count_gathers(const u32* keys, const u64* n_dev, u64* out, cudaStream_t st) {
+  k_count_gathers<<<148 * 8, 256, 0, st>>>(keys, n_dev, out);
+  ++g_launches;
+}
 
 size_t check_status_bytes(u64 n) { return (size_t)148 * 64 * sizeof(WarpEnd) + 256; }
 

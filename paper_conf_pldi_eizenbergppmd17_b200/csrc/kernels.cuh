@@ -104,6 +104,8 @@ size_t check_status_bytes(u64 n);
 void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_dev, u64 n_max, void* status,
                   uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, const u64* values, cudaStream_t st);
 
+void launch_count_gathers(const u32* keys, const u64* n_dev, u64* out, cudaStream_t st);
+
 // finalize.cu
 void launch_page_list(const u32* words, const u32* wl_prefix, const u32* page_bits, u64 n_words, u32* page_num,
                       cudaStream_t st);

@@ -28,6 +28,9 @@ constexpr int RS_TILE = RS_THREADS * RS_ITEMS;  // 4096
 constexpr int RS_WARPS = RS_THREADS / 32;
 constexpr int RS_MAXB = 1024;                   // bins of the widest digit (10 bits)
 constexpr int RS_MAXP = 4;
+#ifndef RS_MATCH_ANY
+#define RS_MATCH_ANY 1  // warp peers of a digit by one MATCH.ANY instead of RB+1 ballots
+#endif
 // temp header: ghist[RS_MAXP][RS_MAXB], gbase[RS_MAXP][RS_MAXB]; the (digit, tile) table follows
 constexpr size_t RS_HDR_BYTES = (2 * RS_MAXP * RS_MAXB + 64) * sizeof(u32);
 
@@ -268,7 +271,7 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
       const u64 idx = base + li;
       const u32 k = idx < n ? sk[li] : KEY_DROP;
       const u32 d = (idx < n && !(drop && k == KEY_DROP)) ? ((k >> shift) & (BINS - 1)) : (u32)BINS;
-      const u32 peers = match_label<RB>(d);
+      const u32 peers = RS_MATCH_ANY ? __match_any_sync(0xFFFFFFFFu, d) : match_label<RB>(d);
       u32* hw = whist + w * BINS;
       const u32 old = d < (u32)BINS ? hw[d] : 0u;
       __syncwarp();
