@@ -455,9 +455,15 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
 constexpr int KT_IPL = 16;                   // items per lane per block
 constexpr int KT_BLK = 32 * KT_IPL;          // items per warp block
 constexpr int KT_PITCH = 32 * (KT_IPL + 1);  // padded entries per array
-constexpr int KT_WARPS = 12;
+#ifndef KT_DB
+#define KT_DB 1  // keys / events of the next block staged during this one (double buffer)
+#endif
+#ifndef KT_NWARPS
+#define KT_NWARPS 12
+#endif
+constexpr int KT_WARPS = KT_NWARPS;
 // per warp: snapshots [KT_PITCH] uint4, keys / evs double-buffered [2][2][KT_PITCH] u32
-constexpr size_t KT_WARP_BYTES = (size_t)KT_PITCH * (sizeof(uint4) + 4 * sizeof(u32));
+constexpr size_t KT_WARP_BYTES = (size_t)KT_PITCH * (sizeof(uint4) + (KT_DB ? 4 : 2) * sizeof(u32));
 
 __device__ __forceinline__ u32 tpad(u32 i) { return i + i / KT_IPL; }
 
@@ -551,7 +557,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
   for (u64 bb = beg; bb < end; bb += KT_BLK) {
     const u32 nb = (u32)(end - bb < (u64)KT_BLK ? end - bb : (u64)KT_BLK);
     // ---- this block's (key, ev) words were staged one iteration ago (or by the prologue)
-    const u32 buf = (u32)(((bb - beg) / KT_BLK) & 1u);
+    const u32 buf = KT_DB ? (u32)(((bb - beg) / KT_BLK) & 1u) : 0u;
     u32* const sK = sKE + buf * 2 * KT_PITCH;
     u32* const sE = sK + KT_PITCH;
     const u32 knext = bb + nb < end ? a.keys[bb + nb] : NONE;  // first item after the block
@@ -581,13 +587,13 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
       }
     }
     cp_async_commit();
-    if (bb + nb < end) {  // stage the next block now: its loads overlap this block's work
+    if (KT_DB && bb + nb < end) {  // stage the next block now: its loads overlap this block's work
       const u64 b2 = bb + nb;
       kt_stage(a, b2, (u32)(end - b2 < (u64)KT_BLK ? end - b2 : (u64)KT_BLK), sKE + (buf ^ 1u) * 2 * KT_PITCH,
                sKE + (buf ^ 1u) * 2 * KT_PITCH + KT_PITCH, lane);
     }
     const u32 pw0 = (lane == 0 && ppk != NONE) ? __ldg(&c.snap[pev >> 5].x) : 0u;
-    if (bb + nb < end) cp_async_wait<1>(); else cp_async_wait<0>();
+    if (KT_DB && bb + nb < end) cp_async_wait<1>(); else cp_async_wait<0>();
     __syncwarp();
 
     // ---- READINFLATE flags (Fig. 2: a read whose predecessor is an unordered read of the same
@@ -721,6 +727,10 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, Wa
     pkx = sK[tpad(nb - 1)];
     pev = sE[tpad(nb - 1)];
     __syncwarp();
+    if (!KT_DB && bb + nb < end) {  // single buffer: stage the next block once this one is done
+      const u64 b2 = bb + nb;
+      kt_stage(a, b2, (u32)(end - b2 < (u64)KT_BLK ? end - b2 : (u64)KT_BLK), sKE, sKE + KT_PITCH, lane);
+    }
   }
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);
   if (lane == 0) {

@@ -14,6 +14,7 @@
 //   k_rs_down  : per tile: stable in-tile rank (ballot match + per-warp histograms), scatter through
 //                shared memory so that each digit's run is written contiguously (8 B in, 8 B out).
 #include <algorithm>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "kernels.cuh"
@@ -588,7 +589,12 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
     ++g_launches;
     return true;
   }
-  int passes = std::min((bits + 9) / 10, RS_MAXP);
+  static int maxb = 0;
+  if (!maxb) {
+    const char* e = getenv("BC_RS_MAXBITS");  // widest digit (8..10); experiments only
+    maxb = e ? std::max(8, std::min(10, atoi(e))) : 10;
+  }
+  int passes = std::min((bits + maxb - 1) / maxb, RS_MAXP);
   const int rb = std::max(8, std::min(10, (bits + passes - 1) / passes));
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
   if (rb == 8) rs_sort_rb<8>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
