@@ -452,14 +452,17 @@ __global__ void __launch_bounds__(K7_WARPS * 32, 2) k_check(CheckArgs a, WarpEnd
 // A query is one u32: item index (current event), source index (prior event; two codes name
 // per-lane registers holding an event from before the block), kind.  Every query reads shared
 // memory only; values carried across blocks are loaded from global memory once per lane.
-constexpr int KT_IPL = 16;                   // items per lane per block
+#ifndef KT_IPL_
+#define KT_IPL_ 16
+#endif
+constexpr int KT_IPL = KT_IPL_;              // items per lane per block
 constexpr int KT_BLK = 32 * KT_IPL;          // items per warp block
 constexpr int KT_PITCH = 32 * (KT_IPL + 1);  // padded entries per array
 #ifndef KT_DB
-#define KT_DB 1  // keys / events of the next block staged during this one (double buffer)
+#define KT_DB 0  // 1: keys / events of the next block staged during this one (double buffer)
 #endif
 #ifndef KT_NWARPS
-#define KT_NWARPS 12
+#define KT_NWARPS 16  // 16 x 128 registers fill the register file; the single-buffered stage fits 16
 #endif
 constexpr int KT_WARPS = KT_NWARPS;
 // per warp: snapshots [KT_PITCH] uint4, keys / evs double-buffered [2][2][KT_PITCH] u32
