@@ -39,6 +39,7 @@ struct bc_ctx {
   Arena arena;  // scratch buffers, reused across bc_detect calls
   std::string err;
   cudaEvent_t ev[16] = {};
+  u64* hcnt = nullptr;  // pinned host copy of the device counter array (one D2H copy per host sync)
 };
 
 static const char* kPhase[] = {"header", "partition", "replay", "sync", "expand", "sort", "check", "finalize",
@@ -134,6 +135,7 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
     cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
   }
   for (int i = 0; i < 16; ++i) cudaEventCreate(&c->ev[i]);
+  cudaMallocHost(&c->hcnt, C_N * sizeof(u64));
   if (cudaGetLastError() != cudaSuccess) {
     bc_destroy(c);
     return BC_ERR_CUDA;
@@ -150,6 +152,7 @@ void bc_destroy(bc_ctx* c) {
   if (c->values_owned) cudaFree(c->values_owned);
   if (c->races) cudaFree(c->races);
   c->arena.free_all();
+  if (c->hcnt) cudaFreeHost(c->hcnt);
   for (int i = 0; i < 16; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
   if (c->own_stream) cudaStreamDestroy(c->stream);
@@ -211,8 +214,8 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     return BC_OK;
   }
   const u64 nwords = 1ull << 23;  // page bitmap: 2^28 1-MB pages (48-bit addresses)
-  u32* err = S.alloc<u32>(1);
   u64* cnt = S.alloc<u64>(C_N);
+  u32* err = reinterpret_cast<u32*>(cnt + C_ERR);
   u32* wkey = S.alloc<u32>(n);
   u32* wval = S.alloc<u32>(n);
   u32* if_cnt = S.alloc<u32>(g.n_warps + 1);
@@ -221,7 +224,6 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* page_bits = S.alloc<u32>(nwords);
   u32* ub_off = S.alloc<u32>(n + 1);  // per record: upper bound of its items, then its first slot
   uint4* hdr16 = S.alloc<uint4>(n);  // compact record headers (K2 gathers them per warp)
-  cudaMemsetAsync(err, 0, 4, st);
   cudaMemsetAsync(cnt, 0, C_N * 8, st);
   cudaMemsetAsync(if_cnt, 0, (g.n_warps + 1) * 4, st);
   cudaMemsetAsync(bar_cnt, 0, (g.n_warps + 1) * 4, st);
@@ -233,16 +235,15 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* words = word_list;
   u32* wl_prefix = wl2;
   u32* page_rank = S.alloc<u32>(nwords);
-  u32* need_sort = S.alloc<u32>(1);
-  cudaMemsetAsync(need_sort, 0, 4, st);
+  u32* need_sort = reinterpret_cast<u32*>(cnt + C_NEED_SORT);
   launch_page_rank(words, cnt + C_PAGE_WORDS, page_bits, page_rank, wl_prefix, cnt + C_PAGES, need_sort, 0, st);
   cudaEventRecord(c->ev[1], st);
   u64 hc_cnt[C_N];
-  u32 herr = 0, h_need_sort = 0;
-  cudaMemcpyAsync(hc_cnt, cnt, sizeof(hc_cnt), cudaMemcpyDeviceToHost, st);
-  cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
-  cudaMemcpyAsync(&h_need_sort, need_sort, 4, cudaMemcpyDeviceToHost, st);
+  u64* const hcnt = c->hcnt;
+  cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
   if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "header");
+  memcpy(hc_cnt, hcnt, sizeof(hc_cnt));
+  u32 herr = (u32)hc_cnt[C_ERR], h_need_sort = (u32)hc_cnt[C_NEED_SORT];
   if (h_need_sort) {  // more non-zero page words than one CTA sorts: radix sort, then rank
     const u64 nwl = hc_cnt[C_PAGE_WORDS];
     if (radix_sort_pairs(word_list, nullptr, wl2, nullptr, nwl, 0, 23, S.alloc<char>(rs_temp_bytes(nwl)), st)) {
@@ -250,8 +251,9 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
       wl_prefix = word_list;
     }
     launch_page_rank(words, cnt + C_PAGE_WORDS, page_bits, page_rank, wl_prefix, cnt + C_PAGES, need_sort, 1, st);
-    cudaMemcpyAsync(hc_cnt, cnt, sizeof(hc_cnt), cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
     if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "page rank");
+    memcpy(hc_cnt, hcnt, sizeof(hc_cnt));
   }
   const u64 n_pages = hc_cnt[C_PAGES], n_words = hc_cnt[C_PAGE_WORDS];
   sx.lane_events = hc_cnt[C_LANE_EVENTS];
@@ -288,8 +290,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* blockR = S.alloc<u32>(n_bar + 1);
   u32* find_blk = S.alloc<u32>(n_bar + 1);
   u32* find_rec = S.alloc<u32>(n_bar + 1);
-  u32* find_cnt = S.alloc<u32>(1);
-  cudaMemsetAsync(find_cnt, 0, 4, st);
+  u32* find_cnt = reinterpret_cast<u32*>(cnt + C_FINDINGS);
   launch_replay(hdr16, wrec, warp_start, g, node_base, bar_base, snap, nodes, bar_rec, bar_next, find_blk, find_rec,
                 find_cnt, err, st);
   launch_barriers(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err, st);
@@ -298,8 +299,9 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   bc_status cs = cuda_check(c, "replay");
   if (cs) return cs;
   if (hc_cnt[C_SYNC_RECS]) {  // K3 walks snapshots: make sure the replay accepted the trace
-    cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
     if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "replay");
+    herr = (u32)hcnt[C_ERR];
     if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "SIMT stack / barrier feasibility");
   }
 
@@ -342,26 +344,26 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   // ---- K7: shadow check
   u32 race_cap = (u32)std::min<u64>(std::max<u64>(1u << 16, bound / 16), 1u << 30);
   uint4* rbuf = nullptr;
-  u32* rcnt = S.alloc<u32>(1);
-  u64* segc = S.alloc<u64>(2);  // [0] segments, [1] clock snapshot gathers
+  u32* rcnt = reinterpret_cast<u32*>(cnt + C_RACES);
+  u64* segc = cnt + C_SEGMENTS;  // [0] segments, [1] clock snapshot gathers (C_GATHERS)
   void* cstatus = S.alloc<char>(check_status_bytes(bound));
   u32 n_r = 0, nfind = 0;
   u64 n_items = 0;
   for (int attempt = 0; attempt < 2; ++attempt) {
     rbuf = S.alloc<uint4>(race_cap);
-    cudaMemsetAsync(rcnt, 0, 4, st);
-    cudaMemsetAsync(segc, 0, 16, st);
+    cudaMemsetAsync(cnt + C_RACES, 0, 3 * sizeof(u64), st);  // races, segments, gathers
     cudaEventRecord(c->ev[10], st);
     launch_check(hc, skey, sev, n_items_dev, bound, cstatus, rbuf, rcnt, race_cap, segc, c->values, st);
     cudaEventRecord(c->ev[11], st);
     if (g.flags & BC_F_COUNT_GATHERS) launch_count_gathers(skey, n_items_dev, segc + 1, st);
-    cudaMemcpyAsync(&n_r, rcnt, 4, cudaMemcpyDeviceToHost, st);
-    cudaMemcpyAsync(&herr, err, 4, cudaMemcpyDeviceToHost, st);
-    cudaMemcpyAsync(&sx.segments, segc, 8, cudaMemcpyDeviceToHost, st);
-    cudaMemcpyAsync(&sx.clock_gathers, segc + 1, 8, cudaMemcpyDeviceToHost, st);
-    cudaMemcpyAsync(&n_items, n_items_dev, 8, cudaMemcpyDeviceToHost, st);
-    cudaMemcpyAsync(&nfind, find_cnt, 4, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
     if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "check");
+    n_r = (u32)hcnt[C_RACES];
+    herr = (u32)hcnt[C_ERR];
+    sx.segments = hcnt[C_SEGMENTS];
+    sx.clock_gathers = hcnt[C_GATHERS];
+    n_items = hcnt[C_ITEMS];
+    nfind = (u32)hcnt[C_FINDINGS];
     if (herr) break;
     if (n_r <= race_cap) break;
     race_cap = n_r;

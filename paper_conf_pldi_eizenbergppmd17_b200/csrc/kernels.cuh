@@ -13,8 +13,11 @@ namespace bc {
 extern u64 g_launches;
 
 // counters written by the kernels (u64 device array)
+// (one u64 array, so that each host synchronisation reads every counter with ONE pinned copy; the u32
+// words err / need_sort / races / findings live in the low half of their slot)
 enum { C_LANE_EVENTS = 0, C_CONTROL_EVENTS, C_SYNC_RECS, C_ACQ_RECS, C_MEM_RECS, C_IFS, C_BARS, C_SYNC_LANEOPS,
-       C_ITEMS, C_ITEM_BOUND, C_SEGMENTS, C_PAGE_WORDS, C_PAGES, C_N };
+       C_ITEMS, C_ITEM_BOUND, C_SEGMENTS_UNUSED, C_PAGE_WORDS, C_PAGES, C_ERR, C_NEED_SORT, C_FINDINGS,
+       C_RACES, C_SEGMENTS, C_GATHERS, C_N };
 
 // Per-context scratch arena.  A bc_detect allocates its scratch buffers in a fixed order; the i-th
 // allocation reuses the i-th buffer of earlier calls when it is large enough, so repeated detects of
