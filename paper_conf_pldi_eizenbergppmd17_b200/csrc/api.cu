@@ -218,20 +218,22 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* err = reinterpret_cast<u32*>(cnt + C_ERR);
   u32* wkey = S.alloc<u32>(n);
   u32* wval = S.alloc<u32>(n);
-  u32* if_cnt = S.alloc<u32>(g.n_warps + 1);
-  u32* bar_cnt = S.alloc<u32>(g.n_warps + 1);
+  const bool small_w = g.n_warps <= WS_SMALL;
+  u32* wcnt = S.alloc<u32>(3 * (size_t)(g.n_warps + 1));  // IFs, BARs, records per warp
+  u32* if_cnt = wcnt;
+  u32* bar_cnt = wcnt + (g.n_warps + 1);
+  u32* rec_cnt = small_w ? wcnt + 2 * (size_t)(g.n_warps + 1) : nullptr;
   u32* sync_list = S.alloc<u32>(n);
   u32* page_bits = S.alloc<u32>(nwords);
   u32* ub_off = S.alloc<u32>(n + 1);  // per record: upper bound of its items, then its first slot
   uint4* hdr16 = S.alloc<uint4>(n);  // compact record headers (K2 gathers them per warp)
   cudaMemsetAsync(cnt, 0, C_N * 8, st);
-  cudaMemsetAsync(if_cnt, 0, (g.n_warps + 1) * 4, st);
-  cudaMemsetAsync(bar_cnt, 0, (g.n_warps + 1) * 4, st);
+  cudaMemsetAsync(wcnt, 0, 3 * (size_t)(g.n_warps + 1) * 4, st);
   cudaMemsetAsync(page_bits, 0, nwords * 4, st);
   // ---- header pass; written pages ranked in address order from the list of non-zero bitmap words
   u32* word_list = S.alloc<u32>(nwords);
   u32* wl2 = S.alloc<u32>(nwords);
-  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, ub_off, hdr16, err, st);
+  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, ub_off, hdr16, rec_cnt, err, st);
   u32* words = word_list;
   u32* wl_prefix = wl2;
   u32* page_rank = S.alloc<u32>(nwords);
@@ -273,13 +275,17 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* skeys = alt ? wk2 : wkey;
   u32* wrec = alt ? wv2 : wval;
   u32* warp_start = S.alloc<u32>(g.n_warps + 1);
-  launch_warp_start(skeys, n, g.n_warps, warp_start, st);
   const u64 n_if = hc_cnt[C_IFS], n_bar = hc_cnt[C_BARS];
   u32* node_base = S.alloc<u32>(g.n_warps + 1);
   u32* bar_base = S.alloc<u32>(g.n_warps + 1);
-  exclusive_scan_u32(if_cnt, node_base, g.n_warps, S.alloc<char>(scan_temp_bytes(g.n_warps)), nullptr, st);
-  launch_node_base(node_base, g.n_warps, node_base, st);
-  exclusive_scan_u32(bar_cnt, bar_base, g.n_warps, S.alloc<char>(scan_temp_bytes(g.n_warps)), nullptr, st);
+  if (small_w) {
+    launch_warp_scans(rec_cnt, if_cnt, bar_cnt, g.n_warps, warp_start, node_base, bar_base, st);
+  } else {
+    launch_warp_start(skeys, n, g.n_warps, warp_start, st);
+    exclusive_scan_u32(if_cnt, node_base, g.n_warps, S.alloc<char>(scan_temp_bytes(g.n_warps)), nullptr, st);
+    launch_node_base(node_base, g.n_warps, node_base, st);
+    exclusive_scan_u32(bar_cnt, bar_base, g.n_warps, S.alloc<char>(scan_temp_bytes(g.n_warps)), nullptr, st);
+  }
   cudaEventRecord(c->ev[2], st);
   // ---- K2: clock replay
   const u64 n_nodes = g.n_warps + 2 * n_if;

@@ -79,8 +79,11 @@ void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_d
 
 // trace.cu
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
-                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, uint4* hdr16, u32* err,
-                   cudaStream_t st);
+                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, uint4* hdr16,
+                   u32* rec_cnt, u32* err, cudaStream_t st);
+constexpr u32 WS_SMALL = 8192;  // n_warps up to which one CTA does the per-warp scans (launch_warp_scans)
+void launch_warp_scans(const u32* rec_cnt, const u32* if_cnt, const u32* bar_cnt, u32 n_warps, u32* warp_start,
+                       u32* node_base, u32* bar_base, cudaStream_t st);
 void launch_page_rank(u32* words, const u64* n_words_dev, const u32* page_bits, u32* page_rank, u32* wl_prefix,
                       u64* n_pages_dev, u32* need_sort, int presorted, cudaStream_t st);
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st);

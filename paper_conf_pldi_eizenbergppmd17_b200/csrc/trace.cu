@@ -22,7 +22,8 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
                                                 u32* __restrict__ bar_cnt, u32* __restrict__ sync_list,
                                                 u32* __restrict__ page_bits, u32* __restrict__ word_list,
                                                 u64* __restrict__ cnt, u32* __restrict__ rec_ub,
-                                                uint4* __restrict__ hdr16, u32* __restrict__ err) {
+                                                uint4* __restrict__ hdr16, u32* __restrict__ rec_cnt,
+                                                u32* __restrict__ err) {
   const u32 lane = threadIdx.x & 31;
   const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const u64 r = gw * 32 + lane;
@@ -69,6 +70,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
     wkey[r] = bad ? 0u : h.warp;
     wval[r] = (u32)r;
     if (!bad) {
+      if (rec_cnt) atomicAdd(&rec_cnt[h.warp], 1u);  // K1 CSR offsets by a scan (small grids)
       if (is_if) atomicAdd(&if_cnt[h.warp], 1u);
       if (is_bar) atomicAdd(&bar_cnt[h.warp], 1u);
       if (is_sync) {
@@ -536,13 +538,13 @@ __global__ void __launch_bounds__(1024) k_page_rank(u32* __restrict__ words, con
 
 // --------------------------------------------------------------------- host launchers
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
-                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, uint4* hdr16, u32* err,
-                   cudaStream_t st) {
+                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, uint4* hdr16,
+                   u32* rec_cnt, u32* err, cudaStream_t st) {
   u64 warps = (g.n_recs + 31) / 32;
   if (warps == 0) return;
   u64 blocks = (warps + 7) / 8;
   k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt,
-                                             rec_ub, hdr16, err); ++g_launches;
+                                             rec_ub, hdr16, rec_cnt, err); ++g_launches;
 }
 
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st) {
@@ -586,6 +588,59 @@ void launch_page_rank(u32* words, const u64* n_words_dev, const u32* page_bits, 
                       u64* n_pages_dev, u32* need_sort, int presorted, cudaStream_t st) {
   k_page_rank<<<1, 1024, 0, st>>>(words, n_words_dev, page_bits, page_rank, wl_prefix, n_pages_dev, need_sort,
                                   presorted);
+  ++g_launches;
+}
+
+// Small grids (n_warps <= WS_SMALL): one CTA turns the header's per-warp counters into K1's CSR offsets
+// (warp_start = exclusive scan of records per warp, + total), the SIMT-node bases (n_warps + 2 x
+// exclusive scan of IFs) and the barrier bases (exclusive scan of BARs) -- one launch instead of a
+// binary search per warp and two device-wide scans.
+__global__ void __launch_bounds__(1024) k_warp_scans(const u32* __restrict__ rec_cnt, const u32* __restrict__ if_cnt,
+                                                     const u32* __restrict__ bar_cnt, u32 n_warps,
+                                                     u32* __restrict__ warp_start, u32* __restrict__ node_base,
+                                                     u32* __restrict__ bar_base) {
+  __shared__ u32 wsum[3][32];
+  __shared__ u32 s_carry[3];
+  const u32 t = threadIdx.x, wi = t >> 5, l = t & 31;
+  if (t < 3) s_carry[t] = 0;
+  __syncthreads();
+  for (u32 c0 = 0; c0 < n_warps; c0 += 1024) {
+    const u32 w = c0 + t;
+    u32 v[3], x[3];
+    v[0] = w < n_warps ? rec_cnt[w] : 0u;
+    v[1] = w < n_warps ? if_cnt[w] : 0u;
+    v[2] = w < n_warps ? bar_cnt[w] : 0u;
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+      x[a] = warp_incl_sum(v[a]);
+      if (l == 31) wsum[a][wi] = x[a];
+    }
+    __syncthreads();
+    u32 off[3] = {0, 0, 0}, tot[3] = {0, 0, 0};
+    for (u32 q = 0; q < 32; ++q) {
+#pragma unroll
+      for (int a = 0; a < 3; ++a) {
+        if (q < wi) off[a] += wsum[a][q];
+        tot[a] += wsum[a][q];
+      }
+    }
+    u32 ex[3];
+#pragma unroll
+    for (int a = 0; a < 3; ++a) ex[a] = s_carry[a] + off[a] + x[a] - v[a];
+    if (w < n_warps) {
+      warp_start[w] = ex[0];
+      node_base[w] = n_warps + 2u * ex[1];
+      bar_base[w] = ex[2];
+    }
+    __syncthreads();
+    if (t < 3) s_carry[t] += tot[t];
+    __syncthreads();
+  }
+  if (t == 0) warp_start[n_warps] = s_carry[0];
+}
+void launch_warp_scans(const u32* rec_cnt, const u32* if_cnt, const u32* bar_cnt, u32 n_warps, u32* warp_start,
+                       u32* node_base, u32* bar_base, cudaStream_t st) {
+  k_warp_scans<<<1, 1024, 0, st>>>(rec_cnt, if_cnt, bar_cnt, n_warps, warp_start, node_base, bar_base);
   ++g_launches;
 }
 
