@@ -267,12 +267,20 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
     mbar_wait(&bar[st], phase);
     u32 rank[RS_ITEMS];  // (digit << 16) | rank in the warp's digit run, NONE = no item
 #pragma unroll
+    // digits and warp peers of all items first (independent MATCH.ANYs in flight together), then the
+    // per-warp running counts in item order
+    u32 dg[RS_ITEMS], pr[RS_ITEMS];
+#pragma unroll
     for (int j = 0; j < RS_ITEMS; ++j) {
       const u32 li = w * (RS_ITEMS * 32) + j * 32 + l;
       const u64 idx = base + li;
       const u32 k = idx < n ? sk[li] : KEY_DROP;
-      const u32 d = (idx < n && !(drop && k == KEY_DROP)) ? ((k >> shift) & (BINS - 1)) : (u32)BINS;
-      const u32 peers = RS_MATCH_ANY ? __match_any_sync(0xFFFFFFFFu, d) : match_label<RB>(d);
+      dg[j] = (idx < n && !(drop && k == KEY_DROP)) ? ((k >> shift) & (BINS - 1)) : (u32)BINS;
+      pr[j] = RS_MATCH_ANY ? __match_any_sync(0xFFFFFFFFu, dg[j]) : match_label<RB>(dg[j]);
+    }
+#pragma unroll
+    for (int j = 0; j < RS_ITEMS; ++j) {
+      const u32 d = dg[j], peers = pr[j];
       u32* hw = whist + w * BINS;
       const u32 old = d < (u32)BINS ? hw[d] : 0u;
       __syncwarp();
