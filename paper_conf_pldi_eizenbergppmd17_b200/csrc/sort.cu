@@ -330,13 +330,9 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
     }
     __syncthreads();
     const u32 tile_n = *s_kept;
-    for (u32 q = t; q < tile_n; q += RS_THREADS) {
-      const u32 kk = skeys[q];
-      const u32 d = (kk >> shift) & (BINS - 1);
-      kout[(u64)gstart[d] + (q - tofs[d])] = kk;
-    }
     if (vout) {
-      // values: the same permutation, staged in the (consumed) key stage
+      // values: the same permutation, staged in the (consumed) key stage; keys and values then leave
+      // in one pass over the tile
 #pragma unroll
       for (int j = 0; j < RS_ITEMS; ++j) {
         if (rank[j] != NONE) {
@@ -346,8 +342,17 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
       }
       __syncthreads();
       for (u32 q = t; q < tile_n; q += RS_THREADS) {
-        const u32 d = (skeys[q] >> shift) & (BINS - 1);
-        vout[(u64)gstart[d] + (q - tofs[d])] = sk[q];
+        const u32 kk = skeys[q];
+        const u32 d = (kk >> shift) & (BINS - 1);
+        const u64 o = (u64)gstart[d] + (q - tofs[d]);
+        kout[o] = kk;
+        vout[o] = sk[q];
+      }
+    } else {
+      for (u32 q = t; q < tile_n; q += RS_THREADS) {
+        const u32 kk = skeys[q];
+        const u32 d = (kk >> shift) & (BINS - 1);
+        kout[(u64)gstart[d] + (q - tofs[d])] = kk;
       }
     }
     __syncthreads();  // stage st and the per-tile tables are free: refill the stage
