@@ -5,13 +5,13 @@
 // entry orders the host threads' accesses) turned into data parallelism: a STABLE sort of
 // (location key, trace position) items groups each location's accesses into one contiguous
 // segment that is still in trace order.
-//   k_rs_hist  : one read of the keys -> the global 256-bin histogram of every digit pass
-//   k_rs_bins  : exclusive scan of each pass's histogram (digit start offsets); kept-item count
+// Per pass:
 //   k_rs_up    : per 4096-key tile, the digit counts (reads 4 B / item)
-//   k_rs_rows  : one CTA per digit scans that digit's counts over all tiles (256 independent rows:
-//                no serial chain across tiles, unlike a decoupled look-back whose first wave of
-//                ~450 co-resident tiles walks back one L2 round trip per step)
-//   k_rs_down  : per tile: stable in-tile rank (ballot match + per-warp histograms), scatter through
+//   k_rs_rows  : one CTA per digit scans that digit's counts over all tiles (independent rows: no
+//                serial chain across tiles, unlike a decoupled look-back whose first wave of ~450
+//                co-resident tiles walks back one L2 round trip per step), and its total
+//   k_rs_bins  : exclusive scan of the digit totals (digit start offsets); kept-item count
+//   k_rs_down  : per tile: stable in-tile rank (MATCH.ANY + per-warp histograms), scatter through
 //                shared memory so that each digit's run is written contiguously (8 B in, 8 B out).
 #include <algorithm>
 #include <cstdlib>
@@ -32,7 +32,7 @@ constexpr int RS_MAXP = 4;
 #ifndef RS_MATCH_ANY
 #define RS_MATCH_ANY 1  // warp peers of a digit by one MATCH.ANY instead of RB+1 ballots
 #endif
-// temp header: ghist[RS_MAXP][RS_MAXB], gbase[RS_MAXP][RS_MAXB]; the (digit, tile) table follows
+// temp header: digit totals [RS_MAXP][RS_MAXB], gbase[RS_MAXP][RS_MAXB]; the (digit, tile) table follows
 constexpr size_t RS_HDR_BYTES = (2 * RS_MAXP * RS_MAXB + 64) * sizeof(u32);
 
 // Lanes of the warp holding the same (RB+1)-bit label (digit, or 1 << RB = no item): RB+1 ballots,
@@ -61,45 +61,7 @@ __device__ __forceinline__ void warp_hist_add(u32* h, u32 d, bool ok, u32 lt) {
   }
 }
 
-constexpr int RS_HIST_ITEMS = 8;
-
-// Global digit histograms of all passes in one read of the keys.
-template <int RB>
-__global__ void __launch_bounds__(RS_THREADS) k_rs_hist(const u32* __restrict__ kin, u64 n_max,
-                                                        const u64* __restrict__ n_dev, int drop, int bit_lo,
-                                                        int passes, u32* __restrict__ ghist) {
-  constexpr int BINS = 1 << RB;
-  __shared__ u32 h[RS_MAXP * BINS];
-  const int t = threadIdx.x;
-  for (int i = t; i < RS_MAXP * BINS; i += RS_THREADS) h[i] = 0;
-  __syncthreads();
-  const u64 n = n_dev ? *n_dev : n_max;
-  const u32 lt = lanemask_lt();
-  constexpr int CH = RS_THREADS * RS_HIST_ITEMS;
-  const u64 stride = (u64)gridDim.x * CH;
-  for (u64 base = (u64)blockIdx.x * CH; base < n; base += stride) {
-    u32 k[RS_HIST_ITEMS];
-#pragma unroll
-    for (int j = 0; j < RS_HIST_ITEMS; ++j) {
-      const u64 idx = base + (u64)j * RS_THREADS + t;
-      k[j] = idx < n ? kin[idx] : KEY_DROP;
-    }
-#pragma unroll
-    for (int j = 0; j < RS_HIST_ITEMS; ++j) {
-      const u64 idx = base + (u64)j * RS_THREADS + t;
-      const bool ok = idx < n && !(drop && k[j] == KEY_DROP);
-      for (int p = 0; p < passes; ++p)
-        warp_hist_add(h + p * BINS, ok ? (k[j] >> (bit_lo + RB * p)) & (BINS - 1) : 0u, ok, lt);
-    }
-  }
-  __syncthreads();
-  for (int i = t; i < passes * BINS; i += RS_THREADS) {
-    const u32 v = h[i];
-    if (v) atomicAdd(&ghist[(i / BINS) * RS_MAXB + (i % BINS)], v);
-  }
-}
-
-// gbase[p][d] = exclusive prefix of ghist[p][*]; *n_out = kept items (pass 0 total).  BINS threads.
+// gbase[d] = exclusive prefix of the digit totals; *n_out = kept items (all digits).  BINS threads.
 template <int RB>
 __global__ void __launch_bounds__(1 << RB) k_rs_bins(const u32* __restrict__ ghist, u32* __restrict__ gbase,
                                                      u64* __restrict__ n_out) {
@@ -151,16 +113,17 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_up(const u32* __restrict__ ki
   for (int d = t; d < BINS; d += RS_THREADS) counts[(u64)d * tiles + blockIdx.x] = h[d];
 }
 
-// One CTA per digit d: offs[d * tiles + tile] = gbase[d] + (items of digit d in tiles < tile).
+// One CTA per digit d: offs[d * tiles + tile] = items of digit d in tiles < tile; rowtot[d] = all items
+// of digit d (their exclusive scan over the digits, k_rs_bins, is the digit's output base).
 // The rows are independent, so there is no serial chain across tiles (unlike a decoupled
 // look-back, whose first wave of ~450 co-resident tiles walks back one L2 round trip per step).
 __global__ void __launch_bounds__(RS_THREADS) k_rs_rows(u32* __restrict__ counts, u64 tiles,
-                                                        const u32* __restrict__ gbase) {
+                                                        u32* __restrict__ rowtot) {
   __shared__ u32 wsum[RS_WARPS];
   __shared__ u32 s_carry;
   const int t = threadIdx.x, w = t >> 5, l = t & 31, d = blockIdx.x;
   u32* row = counts + (u64)d * tiles;
-  if (t == 0) s_carry = gbase[d];
+  if (t == 0) s_carry = 0;
   __syncthreads();
   constexpr int PER = 8;
   for (u64 c0 = 0; c0 < tiles; c0 += RS_THREADS * PER) {
@@ -190,6 +153,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_rows(u32* __restrict__ counts
     if (t == 0) s_carry += tot;
     __syncthreads();
   }
+  if (t == 0) rowtot[d] = s_carry;
 }
 
 // Downsweep of one pass: stable in-tile rank (ballot match + per-warp histograms), scatter through
@@ -209,7 +173,8 @@ template <int RB>
 __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict__ kin, const u32* __restrict__ vin,
                                                            u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
                                                            const u64* __restrict__ n_dev, int drop, int shift,
-                                                           const u32* __restrict__ offs, u64 tiles) {
+                                                           const u32* __restrict__ offs, u64 tiles,
+                                                           const u32* __restrict__ gbase) {
   constexpr int BINS = 1 << RB;
   constexpr int DPT = BINS / RS_THREADS;  // digits per thread (1, 2 or 4)
   extern __shared__ __align__(128) unsigned char rs_smem[];
@@ -262,7 +227,8 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
     // latency overlaps it instead of stalling the tile start)
     u32 go[DPT];
 #pragma unroll
-    for (int q = 0; q < DPT; ++q) go[q] = __ldg(&offs[(u64)(t + q * RS_THREADS) * tiles + tile]);
+    for (int q = 0; q < DPT; ++q)
+      go[q] = __ldg(&gbase[t + q * RS_THREADS]) + __ldg(&offs[(u64)(t + q * RS_THREADS) * tiles + tile]);
     __syncthreads();
     mbar_wait(&bar[st], phase);
     u32 rank[RS_ITEMS];  // (digit << 16) | rank in the warp's digit run, NONE = no item
@@ -544,7 +510,6 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
   u32* ghist = (u32*)temp;                           // [RS_MAXP][RS_MAXB]
   u32* gbase = ghist + RS_MAXP * RS_MAXB;            // [RS_MAXP][RS_MAXB]
   u32* counts = (u32*)((char*)temp + RS_HDR_BYTES);  // [BINS][tiles]
-  cudaMemsetAsync(ghist, 0, RS_MAXP * RS_MAXB * sizeof(u32), st);
   static int sms = 0, down_grid = 0;
   constexpr size_t dsmem = rs_dsmem<RB>();
   if (!down_grid) {
@@ -555,18 +520,17 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_rs_down<RB>, RS_THREADS, dsmem);
     down_grid = sms * (per > 0 ? per : 1);
   }
-  const unsigned hgrid =
-      (unsigned)std::min<u64>((n + RS_THREADS * RS_HIST_ITEMS - 1) / (RS_THREADS * RS_HIST_ITEMS), (u64)sms * 8);
-  k_rs_hist<RB><<<hgrid, RS_THREADS, 0, st>>>(ki, n, n_dev, drop ? 1 : 0, bit_lo, passes, ghist); ++g_launches;
-  k_rs_bins<RB><<<passes, BINS, 0, st>>>(ghist, gbase, drop ? n_out_dev : nullptr); ++g_launches;
   const u64* nd = n_dev;
   for (int p = 0; p < passes; ++p) {
     const int shift = bit_lo + RB * p;
     const int dr = (drop && p == 0) ? 1 : 0;
     k_rs_up<RB><<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles); ++g_launches;
-    k_rs_rows<<<BINS, RS_THREADS, 0, st>>>(counts, tiles, gbase + p * RS_MAXB); ++g_launches;
+    k_rs_rows<<<BINS, RS_THREADS, 0, st>>>(counts, tiles, ghist + p * RS_MAXB); ++g_launches;
+    k_rs_bins<RB><<<1, BINS, 0, st>>>(ghist + p * RS_MAXB, gbase + p * RS_MAXB, dr ? n_out_dev : nullptr);
+    ++g_launches;
     k_rs_down<RB><<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, dsmem, st>>>(ki, vi, ko, vo, n, nd, dr,
-                                                                                              shift, counts, tiles);
+                                                                                              shift, counts, tiles,
+                                                                                              gbase + p * RS_MAXB);
     ++g_launches;
     if (dr) nd = n_out_dev;
     u32* tk = ki; ki = ko; ko = tk;
@@ -579,8 +543,8 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
 // bound of the) item count; with n_dev the exact count is read on the device.  drop: the first pass
 // removes items whose key is KEY_DROP and writes the number kept to *n_out_dev (at least one pass
 // is run).  Digit width: the fewest passes of at most 10 bits, each pass 8, 9 or 10 bits wide.  Per
-// pass: k_rs_up (digit counts per tile) -> k_rs_rows (independent per-digit row scans) -> k_rs_down
-// (rank + scatter); one k_rs_hist read up front gives every pass's digit bases.
+// pass: k_rs_up (digit counts per tile) -> k_rs_rows (independent per-digit row scans + totals) ->
+// k_rs_bins (digit bases from the totals) -> k_rs_down (rank + scatter).
 bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi, void* temp,
                       cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop) {
   if (!drop && (n <= 1 || bit_hi <= bit_lo)) return false;
