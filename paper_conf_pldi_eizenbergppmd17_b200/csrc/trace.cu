@@ -368,8 +368,8 @@ __global__ void __launch_bounds__(256) k_barriers(Geo g, const u32* __restrict__
 // Data movement (the trace is read once, at HBM rate): persistent CTAs stream chunks of EX_REC
 // consecutive records (EX_REC x 272 B, contiguous) into shared memory with 1-D TMA bulk copies
 // (cp.async.bulk ... mbarrier::complete_tx), EX_STAGES chunks in flight per CTA; the 8 warps then
-// expand the staged records (warp w: records w*EX_RPW ...; header = a broadcast shared-memory read,
-// lane l's address = addr[l]) while the next chunks land.
+// expand the staged records (warp w: records w, w+8, w+16, w+24; header = a broadcast shared-memory
+// read, lane l's address = addr[l]) while the next chunks land.
 constexpr int EX_REC = 32;
 constexpr int EX_STAGES = 4;
 constexpr int EX_THREADS = 256;
@@ -408,22 +408,25 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
   for (u64 c = blockIdx.x; c < n_chunks; c += gridDim.x, ++it) {
     const int st = (int)(it % EX_STAGES);
     const u32 phase = (it / EX_STAGES) & 1u;
-    const u64 rbase = c * EX_REC + (u64)wid * EX_RPW;
-    // slot offsets of this warp's records (independent of the staged bytes: load before waiting)
-    u32 uo[EX_RPW];
-#pragma unroll
-    for (int j = 0; j < EX_RPW; ++j) uo[j] = rbase + j < n ? __ldg(ub_off + rbase + j) : 0u;
+    const u64 cbase = c * EX_REC;
+    // warp wid expands records wid, wid + 8, ... of the chunk (interleaved: control and memory records
+    // alternate in most programs, so the warps of a CTA finish a chunk at about the same time); their
+    // slot offsets are independent of the staged bytes: one load per lane before waiting
+    const u64 rl = cbase + (u64)wid + (u64)(lane & (EX_RPW - 1)) * (EX_THREADS / 32);
+    const u32 uo_l = (lane < EX_RPW && rl < n) ? __ldg(ub_off + rl) : 0u;
     mbar_wait(&bar[st], phase);
-    const bc_record* sr = &buf[st * EX_REC + wid * EX_RPW];
 #pragma unroll
     for (int j = 0; j < EX_RPW; ++j) {
-      const u64 r = rbase + j;
+      const u32 jr = (u32)wid + (u32)j * (EX_THREADS / 32);  // record within the chunk
+      const u64 r = cbase + jr;
+      const u32 uoj = __shfl_sync(0xFFFFFFFFu, uo_l, j);
       if (r >= n) break;
-      const uint4 hv = *reinterpret_cast<const uint4*>(&sr[j]);
+      const bc_record* sr = &buf[st * EX_REC + jr];
+      const uint4 hv = *reinterpret_cast<const uint4*>(sr);
       const u32 hwarp = hv.x, hmask = hv.y, op = hv.z & 0xFFu, space = (hv.z >> 8) & 0xFFu,
                 sl = (hv.z >> 16) & 0xFFu, fl = (hv.z >> 24) & 0xFFu;
       if (!(op <= BC_OP_AR_GLB && ((hmask >> lane) & 1u) && sl <= 4 && space <= 1 && hwarp < g.n_warps)) continue;
-      const u64 a = sr[j].addr[lane];
+      const u64 a = sr->addr[lane];
       const u64 size = 1ull << sl;
       if (a & (size - 1)) bad = true;  // natural alignment
       if (space == BC_SPACE_SHARED && a + size > g.smem) bad = true;
@@ -449,8 +452,13 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
           ovf = true;
         }
       }
-      const u64 o = (u64)uo[j] + (u64)__popc(hmask & lt) * nk;
+      const u64 o = (u64)uoj + (u64)__popc(hmask & lt) * nk;
       const u32 ev = (u32)(r << 5) | (u32)lane;
+      if (nk == 1 && g.world == 1) {  // one granule, one shard: the common case
+        okeys[o] = key0 != KEY_DROP ? ((key0 << 2) | opc) : KEY_DROP;
+        oevs[o] = ev;
+        continue;
+      }
       for (u32 k = 0; k < nk; ++k) {
         const bool mine = key0 != KEY_DROP && (g.world == 1 || shard_of(key0 + k, g.world) == g.rank);
         okeys[o + k] = mine ? (((key0 + k) << 2) | opc) : KEY_DROP;
