@@ -27,7 +27,7 @@ constexpr int RS_THREADS = 256;
 constexpr int RS_ITEMS = 16;
 constexpr int RS_TILE = RS_THREADS * RS_ITEMS;  // 4096
 constexpr int RS_WARPS = RS_THREADS / 32;
-constexpr int RS_MAXB = 1024;                   // bins of the widest digit (10 bits)
+constexpr int RS_MAXB = 2048;                   // bins of the widest digit (11 bits)
 constexpr int RS_MAXP = 4;
 #ifndef RS_MATCH_ANY
 #define RS_MATCH_ANY 1  // warp peers of a digit by one MATCH.ANY instead of RB+1 ballots
@@ -63,22 +63,34 @@ __device__ __forceinline__ void warp_hist_add(u32* h, u32 d, bool ok, u32 lt) {
 
 // gbase[d] = exclusive prefix of the digit totals; *n_out = kept items (all digits).  BINS threads.
 template <int RB>
-__global__ void __launch_bounds__(1 << RB) k_rs_bins(const u32* __restrict__ ghist, u32* __restrict__ gbase,
-                                                     u64* __restrict__ n_out) {
+__global__ void __launch_bounds__((1 << RB) < 1024 ? (1 << RB) : 1024) k_rs_bins(const u32* __restrict__ ghist,
+                                                                               u32* __restrict__ gbase,
+                                                                               u64* __restrict__ n_out) {
   constexpr int BINS = 1 << RB;
-  __shared__ u32 wsum[BINS / 32];
-  const int t = threadIdx.x, w = t >> 5, l = t & 31, p = blockIdx.x;
-  const u32 v = ghist[p * RS_MAXB + t];
-  const u32 x = warp_incl_sum(v);
+  constexpr int T = BINS < 1024 ? BINS : 1024, PER = BINS / T;  // thread t: digits [t*PER, t*PER+PER)
+  __shared__ u32 wsum[T / 32];
+  const int t = threadIdx.x, w = t >> 5, l = t & 31;
+  u32 v[PER], sum = 0;
+#pragma unroll
+  for (int q = 0; q < PER; ++q) {
+    v[q] = ghist[t * PER + q];
+    sum += v[q];
+  }
+  const u32 x = warp_incl_sum(sum);
   if (l == 31) wsum[w] = x;
   __syncthreads();
   u32 off = 0, tot = 0;
-  for (int ww = 0; ww < BINS / 32; ++ww) {
+  for (int ww = 0; ww < T / 32; ++ww) {
     if (ww < w) off += wsum[ww];
     tot += wsum[ww];
   }
-  gbase[p * RS_MAXB + t] = off + x - v;
-  if (p == 0 && t == 0 && n_out) *n_out = tot;
+  u32 run = off + x - sum;
+#pragma unroll
+  for (int q = 0; q < PER; ++q) {
+    gbase[t * PER + q] = run;
+    run += v[q];
+  }
+  if (t == 0 && n_out) *n_out = tot;
 }
 
 // Upsweep of one pass: the digit counts of every tile, digit-major (counts[d * tiles + tile]);
@@ -526,7 +538,8 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
     const int dr = (drop && p == 0) ? 1 : 0;
     k_rs_up<RB><<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles); ++g_launches;
     k_rs_rows<<<BINS, RS_THREADS, 0, st>>>(counts, tiles, ghist + p * RS_MAXB); ++g_launches;
-    k_rs_bins<RB><<<1, BINS, 0, st>>>(ghist + p * RS_MAXB, gbase + p * RS_MAXB, dr ? n_out_dev : nullptr);
+    k_rs_bins<RB><<<1, BINS < 1024 ? BINS : 1024, 0, st>>>(ghist + p * RS_MAXB, gbase + p * RS_MAXB,
+                                                          dr ? n_out_dev : nullptr);
     ++g_launches;
     k_rs_down<RB><<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, dsmem, st>>>(ki, vi, ko, vo, n, nd, dr,
                                                                                               shift, counts, tiles,
@@ -568,15 +581,16 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   }
   static int maxb = 0;
   if (!maxb) {
-    const char* e = getenv("BC_RS_MAXBITS");  // widest digit (8..10); experiments only
-    maxb = e ? std::max(8, std::min(10, atoi(e))) : 10;
+    const char* e = getenv("BC_RS_MAXBITS");  // widest digit (8..11); experiments only
+    maxb = e ? std::max(8, std::min(11, atoi(e))) : 11;
   }
   int passes = std::min((bits + maxb - 1) / maxb, RS_MAXP);
-  const int rb = std::max(8, std::min(10, (bits + passes - 1) / passes));
+  const int rb = std::max(8, std::min(maxb, (bits + passes - 1) / passes));
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
   if (rb == 8) rs_sort_rb<8>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
   else if (rb == 9) rs_sort_rb<9>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
-  else rs_sort_rb<10>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
+  else if (rb == 10) rs_sort_rb<10>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
+  else rs_sort_rb<11>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
   return (passes & 1) != 0;
 }
 
