@@ -70,7 +70,6 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
     wkey[r] = bad ? 0u : h.warp;
     wval[r] = (u32)r;
     if (!bad) {
-      if (rec_cnt) atomicAdd(&rec_cnt[h.warp], 1u);  // K1 CSR offsets by a scan (small grids)
       if (is_if) atomicAdd(&if_cnt[h.warp], 1u);
       if (is_bar) atomicAdd(&bar_cnt[h.warp], 1u);
       if (is_sync) {
@@ -80,6 +79,11 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
     }
   }
   if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
+  if (rec_cnt) {  // records per traced warp (K1 CSR offsets by a scan, small grids): one atomic per warp id
+    const bool cnt_me = valid && !bad;
+    const u32 peers = __match_any_sync(0xFFFFFFFFu, cnt_me ? h.warp : 0xFFFFFFFFu);
+    if (cnt_me && (peers & lanemask_lt()) == 0) atomicAdd(&rec_cnt[h.warp], (u32)__popc(peers));
+  }
   // warp-reduced counters
   if (bad) ibound = 0;
   if (valid) rec_ub[r] = ibound;  // upper bound of the record's items (K4 writes at static slots)
