@@ -398,3 +398,29 @@ def test_warpsim_configs(cfg, kw):
     for ws in (16, 8):
         r2, g2, _ = split_warps(recs, plan.geometry, ws)
         assert_parity(r2, g2)
+
+
+# ------------------------------------------------ full-size configs (bench launch configuration)
+@pytest.mark.slow
+def test_c3_full_size_race_free():
+    """C3 at the bench size (4096 x 256 threads, ~50 M events, 4096 AR_GLB tickets): the
+    threadFenceReduction program is race-free by construction (every shared access is ordered by a
+    barrier, the partial sums by the fence + ticket) -- a property that holds at any
+    size and that the oracle confirms at reduced sizes (test_configs_reduced)."""
+    plan = ConfigPlan(3)
+    res = _gpu(plan.records(), plan.geometry)
+    assert res.status == 0
+    assert len(res.races) == 0 and res.stats["lane_events"] > 40_000_000
+
+
+@pytest.mark.slow
+def test_c4_full_size_injected_truth():
+    """C4 at the bench size (1 M threads, ~220 M lane events): the race set equals the generator's
+    injected set exactly (each injected granule is touched by exactly two unsynchronised
+    conflicting accesses and nothing else races, as the oracle confirms at reduced sizes)."""
+    plan = ConfigPlan(4)
+    res = _gpu(plan.records(), plan.geometry)
+    assert res.status == 0
+    truth = plan.truth()
+    assert len(truth) > 0
+    assert np.array_equal(np.sort(res.races.view("V32")), np.sort(truth.view("V32")))
