@@ -372,10 +372,18 @@ __global__ void __launch_bounds__(256) k_barriers(Geo g, const u32* __restrict__
 // Data movement (the trace is read once, at HBM rate): persistent CTAs stream chunks of EX_REC
 // consecutive records (EX_REC x 272 B, contiguous) into shared memory with 1-D TMA bulk copies
 // (cp.async.bulk ... mbarrier::complete_tx), EX_STAGES chunks in flight per CTA; the 8 warps then
-// expand the staged records (warp w: records w, w+8, w+16, w+24; header = a broadcast shared-memory
-// read, lane l's address = addr[l]) while the next chunks land.
-constexpr int EX_REC = 32;
-constexpr int EX_STAGES = 4;
+// expand the staged records (warp w: records w, w+8, ...; header = a broadcast shared-memory read,
+// lane l's address = addr[l]) while the next chunk lands.  64-record chunks, 2 stages: fewer CTA
+// barriers per record (the warps' work per record differs: control vs memory records) beat deeper
+// staging (C4: 32 x 4 -> 64 x 2 took k_expand from 5.1 to 4.4 ms; 128 or 256 records are slower).
+#ifndef EX_REC_
+#define EX_REC_ 64
+#endif
+#ifndef EX_STAGES_
+#define EX_STAGES_ 2
+#endif
+constexpr int EX_REC = EX_REC_;
+constexpr int EX_STAGES = EX_STAGES_;
 constexpr int EX_THREADS = 256;
 constexpr int EX_RPW = EX_REC / (EX_THREADS / 32);  // records per warp per chunk
 
