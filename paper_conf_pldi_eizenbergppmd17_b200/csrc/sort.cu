@@ -6,7 +6,7 @@
 // (location key, trace position) items groups each location's accesses into one contiguous
 // segment that is still in trace order.
 // Per pass:
-//   k_rs_up    : per 4096-key tile, the digit counts (reads 4 B / item)
+//   k_rs_up    : per 6144-key tile (24 keys / thread), the digit counts (reads 4 B / item)
 //   k_rs_rows  : one CTA per digit scans that digit's counts over all tiles (independent rows: no
 //                serial chain across tiles, unlike a decoupled look-back whose first wave of ~450
 //                co-resident tiles walks back one L2 round trip per step), and its total
@@ -24,8 +24,11 @@ namespace bc {
 namespace {
 
 constexpr int RS_THREADS = 256;
-constexpr int RS_ITEMS = 16;
-constexpr int RS_TILE = RS_THREADS * RS_ITEMS;  // 4096
+#ifndef RS_ITEMS_
+#define RS_ITEMS_ 24
+#endif
+constexpr int RS_ITEMS = RS_ITEMS_;  // keys per thread per tile
+constexpr int RS_TILE = RS_THREADS * RS_ITEMS;  // 6144 (A/B on C2 / C4: 24 keys per thread beat 8-32)
 constexpr int RS_WARPS = RS_THREADS / 32;
 constexpr int RS_MAXB = 2048;                   // bins of the widest digit (11 bits)
 constexpr int RS_MAXP = 4;
@@ -174,7 +177,10 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_rows(u32* __restrict__ counts
 // RS_DSTAGES tiles ahead (mbarrier ring), so the load latency that dominated a one-tile-per-CTA kernel
 // overlaps the ranking of the previous tile; the tile's values are loaded into registers at the start
 // of the tile and land while it is ranked.  Once scattered, the stage holds the permuted values.
-constexpr int RS_DSTAGES = 2;
+#ifndef RS_DSTAGES_
+#define RS_DSTAGES_ 2
+#endif
+constexpr int RS_DSTAGES = RS_DSTAGES_;
 template <int RB>
 constexpr size_t rs_dsmem() {
   return (size_t)RS_DSTAGES * RS_TILE * sizeof(u32) + RS_TILE * sizeof(u32) +
