@@ -13,6 +13,9 @@ namespace bc {
 // counters in `cnt` (u64)
 
 // ---------------------------------------------------------------------------- k_header
+#ifndef HDR_ROWS
+#define HDR_ROWS 8  // write records whose address rows one warp loads at once (page marking)
+#endif
 // One warp per 32 consecutive records.  Lane l validates record base+l's header (the checks of
 // P:L360-366 that need no state; stack / barrier checks are in k_replay / k_barriers), then the
 // warp marks the 1-MB pages written by the ST / ATOM global records among the 32 (the paper's
@@ -112,11 +115,11 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
   // page marking: ST / ATOM on global memory
   u32 wr = __ballot_sync(0xFFFFFFFFu, valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) &&
                                           h.space == BC_SPACE_GLOBAL);
-  while (wr) {  // 8 records' address rows in flight at a time
-    int js[8];
-    u64 a[8];
+  while (wr) {  // HDR_ROWS records' address rows in flight at a time
+    int js[HDR_ROWS];
+    u64 a[HDR_ROWS];
 #pragma unroll
-    for (int k = 0; k < 8; ++k) {
+    for (int k = 0; k < HDR_ROWS; ++k) {
       js[k] = -1;
       if (wr) {
         js[k] = __ffs(wr) - 1;
@@ -124,7 +127,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
       }
     }
 #pragma unroll
-    for (int k = 0; k < 8; ++k) {
+    for (int k = 0; k < HDR_ROWS; ++k) {
       a[k] = ~0ull;
       if (js[k] >= 0) {
         u32 m = __shfl_sync(0xFFFFFFFFu, h.mask, js[k]);
@@ -134,7 +137,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
       }
     }
 #pragma unroll
-    for (int k = 0; k < 8; ++k) {
+    for (int k = 0; k < HDR_ROWS; ++k) {
       if (a[k] == ~0ull) continue;
       u64 p = a[k] >> 20;
       if (p >= (1ull << 28)) {
