@@ -587,11 +587,14 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   }
   static int maxb = 0;
   if (!maxb) {
-    const char* e = getenv("BC_RS_MAXBITS");  // widest digit (8..11); experiments only
-    maxb = e ? std::max(8, std::min(11, atoi(e))) : 11;
+    const char* e = getenv("BC_RS_MAXBITS");  // widest digit of a multi-pass sort (8..10); experiments only
+    maxb = e ? std::max(8, std::min(10, atoi(e))) : 10;
   }
-  int passes = std::min((bits + maxb - 1) / maxb, RS_MAXP);
-  const int rb = std::max(8, std::min(maxb, (bits + passes - 1) / passes));
+  // an 11-bit digit only when it makes the sort single-pass (K1 of 2048-warp traces): the 2048-bin
+  // downsweep runs one CTA per SM, which loses to one more 8-10-bit pass when both need passes
+  const int mb = bits == 11 ? 11 : maxb;
+  int passes = std::min((bits + mb - 1) / mb, RS_MAXP);
+  const int rb = std::max(8, std::min(mb, (bits + passes - 1) / passes));
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
   if (rb == 8) rs_sort_rb<8>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
   else if (rb == 9) rs_sort_rb<9>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
