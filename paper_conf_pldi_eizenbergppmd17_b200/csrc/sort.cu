@@ -464,56 +464,116 @@ size_t rs_temp_bytes(u64 n) {
   return RS_HDR_BYTES + (size_t)(tiles ? tiles : 1) * RS_MAXB * sizeof(u32) + 256;
 }
 
-// Small sorts (n <= RS_SMALL, e.g. the K3 sync-skeleton tables, K1 of small traces): one CTA sorts
-// (digit << 32 | input index) composites with a bitonic network in shared memory -- the index makes
-// the order stable -- and gathers keys / values into the alternate buffers: one launch instead of a
-// histogram, a bins scan and three kernels per digit pass.
+// Small sorts (n <= RS_SMALL, e.g. the K3 sync-skeleton tables, K1 of small traces): one CTA sorts in
+// shared memory and gathers keys / values into the alternate buffers: one launch instead of four
+// kernels per digit pass.
 constexpr u32 RS_SMALL = 8192;
-__global__ void __launch_bounds__(1024) k_sort_small(const u32* __restrict__ kin, const u32* __restrict__ vin,
-                                                     u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
-                                                     const u64* __restrict__ n_dev, int drop, int bit_lo, int bits,
-                                                     u64* __restrict__ n_out) {
-  extern __shared__ __align__(16) unsigned long long cs[];
+// One CTA, 1024 threads, up to RS_SMALL keys resident in shared memory: LSD radix passes of 8 bits
+// over (digit, input index) pairs.  Per pass every warp ranks its 256 keys (32 consecutive keys per
+// step, MATCH.ANY peers + per-warp running digit counts, so equal digits keep their order), the CTA
+// turns the 32 x 256 warp counts into scatter bases (digit-major, warp-minor), and the pairs move to
+// the other buffer -- 8 barriers per pass instead of a bitonic network's ~90.  The input index
+// travels along, so the last step gathers keys / values from global memory in sorted order.
+constexpr int SS_THREADS = 1024, SS_WARPS = SS_THREADS / 32, SS_PER = RS_SMALL / SS_THREADS;  // 8
+constexpr size_t SS_SMEM = (size_t)RS_SMALL * 4 * sizeof(u32) + (size_t)SS_WARPS * 256 * sizeof(u32) + 64;
+__global__ void __launch_bounds__(SS_THREADS) k_sort_small(const u32* __restrict__ kin, const u32* __restrict__ vin,
+                                                           u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
+                                                           const u64* __restrict__ n_dev, int drop, int bit_lo,
+                                                           int bits, u64* __restrict__ n_out) {
+  extern __shared__ __align__(16) u32 ss[];
+  u32* dA = ss;                      // digits-source keys (already shifted / masked), buffer A
+  u32* iA = dA + RS_SMALL;           // input indices, buffer A
+  u32* dB = iA + RS_SMALL;           // buffer B
+  u32* iB = dB + RS_SMALL;
+  u32* wh = iB + RS_SMALL;           // [SS_WARPS][256] warp digit counts -> scatter bases
   __shared__ u32 s_kept;
-  const u32 t = threadIdx.x;
+  const u32 t = threadIdx.x, w = t >> 5, l = t & 31;
   const u32 n = (u32)(n_dev ? *n_dev : n_max);
-  if (t == 0) s_kept = 0;
-  u32 P = 1;
-  while (P < n) P <<= 1;
   const u32 dmask = bits >= 32 ? 0xFFFFFFFFu : ((1u << bits) - 1u);
+  // compact the kept keys (drop: KEY_DROP removed) in input order: one warp-aggregated pass
+  if (t == 0) s_kept = 0;
   __syncthreads();
-  u32 kept = 0;
-  for (u32 i = t; i < P; i += 1024) {
-    unsigned long long v = ~0ull;
-    if (i < n) {
-      const u32 k = kin[i];
-      if (!(drop && k == KEY_DROP)) {
-        v = ((unsigned long long)((k >> bit_lo) & dmask) << 32) | i;
-        ++kept;
+  for (u32 c0 = 0; c0 < n; c0 += SS_THREADS) {
+    const u32 i = c0 + t;
+    const u32 k = i < n ? kin[i] : KEY_DROP;
+    const bool keep = i < n && !(drop && k == KEY_DROP);
+    const u32 bal = __ballot_sync(0xFFFFFFFFu, keep);
+    __shared__ u32 s_wbase[SS_WARPS];
+    if (l == 0) s_wbase[w] = __popc(bal);
+    __syncthreads();
+    if (t == 0) {  // 32 warp counts -> bases (tiny serial scan)
+      u32 run = s_kept;
+      for (u32 q = 0; q < SS_WARPS; ++q) {
+        const u32 c = s_wbase[q];
+        s_wbase[q] = run;
+        run += c;
       }
+      s_kept = run;
     }
-    cs[i] = v;
-  }
-  atomicAdd(&s_kept, kept);
-  __syncthreads();
-  for (u32 k = 2; k <= P; k <<= 1) {
-    for (u32 j = k >> 1; j > 0; j >>= 1) {
-      for (u32 i = t; i < P; i += 1024) {
-        const u32 ij = i ^ j;
-        if (ij > i) {
-          const unsigned long long a = cs[i], b = cs[ij];
-          if (((i & k) == 0) == (a > b)) {
-            cs[i] = b;
-            cs[ij] = a;
-          }
-        }
-      }
-      __syncthreads();
+    __syncthreads();
+    if (keep) {
+      const u32 at = s_wbase[w] + __popc(bal & lanemask_lt());
+      dA[at] = (k >> bit_lo) & dmask;
+      iA[at] = i;
     }
+    __syncthreads();
   }
   const u32 nk = s_kept;
-  for (u32 i = t; i < nk; i += 1024) {
-    const u32 src = (u32)(cs[i] & 0xFFFFFFFFull);
+  const int passes = (bits + 7) / 8;
+  for (int p = 0; p < passes; ++p) {
+    const u32 sh = 8u * (u32)p;
+    for (u32 q = t; q < SS_WARPS * 256; q += SS_THREADS) wh[q] = 0;
+    __syncthreads();
+    u32 rk[SS_PER], dg[SS_PER];
+#pragma unroll
+    for (int j = 0; j < SS_PER; ++j) {  // warp w owns keys [w*256, w*256+256), 32 per step in order
+      const u32 i = (u32)w * 256u + (u32)j * 32u + l;
+      const u32 d = i < nk ? (dA[i] >> sh) & 255u : 256u;
+      const u32 peers = __match_any_sync(0xFFFFFFFFu, d);
+      u32 old = 0;
+      if (d < 256u) old = wh[w * 256 + d];
+      __syncwarp();
+      if (d < 256u && (peers & lanemask_lt()) == 0) wh[w * 256 + d] = old + __popc(peers);
+      __syncwarp();
+      dg[j] = d;
+      rk[j] = old + __popc(peers & lanemask_lt());
+    }
+    __syncthreads();
+    // scatter bases: digit-major, warp-minor exclusive prefix over the 32 x 256 counts
+    if (t < 256) {
+      u32 tot = 0;
+      for (u32 q = 0; q < SS_WARPS; ++q) {
+        const u32 c = wh[q * 256 + t];
+        wh[q * 256 + t] = tot;
+        tot += c;
+      }
+      // exclusive scan of the 256 digit totals (8 warps x 32)
+      const u32 x = warp_incl_sum(tot);
+      __shared__ u32 s_dsum[8];
+      if (l == 31) s_dsum[w] = x;
+      __syncwarp();
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      u32 off = 0;
+      for (u32 q = 0; q < w; ++q) off += s_dsum[q];
+      const u32 base = off + x - tot;
+      for (u32 q = 0; q < SS_WARPS; ++q) wh[q * 256 + t] += base;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < SS_PER; ++j) {
+      const u32 i = (u32)w * 256u + (u32)j * 32u + l;
+      if (dg[j] < 256u) {
+        const u32 at = wh[w * 256 + dg[j]] + rk[j];
+        dB[at] = dA[i];
+        iB[at] = iA[i];
+      }
+    }
+    __syncthreads();
+    u32* tmp = dA; dA = dB; dB = tmp;
+    tmp = iA; iA = iB; iB = tmp;
+  }
+  for (u32 i = t; i < nk; i += SS_THREADS) {
+    const u32 src = iA[i];
     kout[i] = kin[src];
     if (vout) vout[i] = vin[src];
   }
@@ -575,13 +635,11 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   if (n <= RS_SMALL) {
     static bool attr = false;
     if (!attr) {
-      cudaFuncSetAttribute(k_sort_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(RS_SMALL * 8));
+      cudaFuncSetAttribute(k_sort_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SS_SMEM);
       attr = true;
     }
-    u32 P = 1;
-    while (P < n) P <<= 1;
-    k_sort_small<<<1, 1024, P * 8, st>>>(keys, vals, keys_alt, vals_alt, n, n_dev, drop ? 1 : 0, bit_lo, bits,
-                                         drop ? n_out_dev : nullptr);
+    k_sort_small<<<1, SS_THREADS, SS_SMEM, st>>>(keys, vals, keys_alt, vals_alt, n, n_dev, drop ? 1 : 0, bit_lo,
+                                                 bits, drop ? n_out_dev : nullptr);
     ++g_launches;
     return true;
   }
