@@ -323,8 +323,8 @@ static int bits_for(u64 maxval) {
 }
 
 // Runs K3.  Fills the foreign-knowledge fields of `hc` (acq_*, idx_*).  Returns 0 or a bc_status.
-int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_lo, HbCtx& hc, Scratch& S,
-                      cudaStream_t st, u64* n_entries_out) {
+int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_lo, u32 n_acq, HbCtx& hc,
+                      Scratch& S, cudaStream_t st, u64* n_entries_out) {
   const Geo& g = hc.g;
   *n_entries_out = 0;
   if (n_srec == 0) return 0;
@@ -343,11 +343,8 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   u32* aex = S.alloc<u32>(n_srec);
   u64* tot = S.alloc<u64>(1);
   k_acq_flags<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, aflag); ++g_launches;
+  // (n_acq = the header's count of acquire records: no host round trip for it)
   exclusive_scan_u32(aflag, aex, n_srec, S.alloc<char>(scan_temp_bytes(n_srec)), tot, st);
-  u64 n_acq64 = 0;
-  cudaMemcpyAsync(&n_acq64, tot, 8, cudaMemcpyDeviceToHost, st);
-  if (cudaStreamSynchronize(st) != cudaSuccess) return BC_ERR_CUDA;
-  u32 n_acq = (u32)n_acq64;
   u32* acq_blk = S.alloc<u32>(n_acq + 1);
   u32* acq_rec = S.alloc<u32>(n_acq + 1);
   u32* acq_warp = S.alloc<u32>(n_acq + 1);
