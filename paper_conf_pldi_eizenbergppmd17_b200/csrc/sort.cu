@@ -11,6 +11,7 @@
 //                serial chain across tiles, unlike a decoupled look-back whose first wave of ~450
 //                co-resident tiles walks back one L2 round trip per step), and its total
 //   k_rs_bins  : exclusive scan of the digit totals (digit start offsets); kept-item count
+//                (default RS_FUSED_BINS: done by every k_rs_down CTA itself, no launch)
 //   k_rs_down  : per tile: stable in-tile rank (MATCH.ANY + per-warp histograms), scatter through
 //                shared memory so that each digit's run is written contiguously (8 B in, 8 B out).
 #include <algorithm>
@@ -177,6 +178,9 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_rows(u32* __restrict__ counts
 // RS_DSTAGES tiles ahead (mbarrier ring), so the load latency that dominated a one-tile-per-CTA kernel
 // overlaps the ranking of the previous tile; the tile's values are loaded into registers at the start
 // of the tile and land while it is ranked.  Once scattered, the stage holds the permuted values.
+#ifndef RS_FUSED_BINS
+#define RS_FUSED_BINS 1  // digit bases scanned inside k_rs_down (no k_rs_bins launch per pass)
+#endif
 #ifndef RS_DSTAGES_
 #define RS_DSTAGES_ 2
 #endif
@@ -192,7 +196,8 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
                                                            u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
                                                            const u64* __restrict__ n_dev, int drop, int shift,
                                                            const u32* __restrict__ offs, u64 tiles,
-                                                           const u32* __restrict__ gbase) {
+                                                           const u32* __restrict__ gbase,
+                                                           const u32* __restrict__ rowtot, u64* __restrict__ n_out) {
   constexpr int BINS = 1 << RB;
   constexpr int DPT = BINS / RS_THREADS;  // digits per thread (1, 2 or 4)
   extern __shared__ __align__(128) unsigned char rs_smem[];
@@ -226,6 +231,32 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
       if (tl < n_tiles) issue(tl, q);
     }
   const u32 lt = lanemask_lt();
+  // digit bases: with rowtot (RS_FUSED_BINS) every CTA scans the digit totals itself, once (thread t
+  // owns digits t + q * RS_THREADS, i.e. q-th block of RS_THREADS consecutive digits), instead of a
+  // separate one-CTA k_rs_bins launch per pass; CTA 0 publishes the kept-item count
+  u32 gb[DPT];
+  if (rowtot) {
+    u32 carry = 0;
+#pragma unroll
+    for (int q = 0; q < DPT; ++q) {
+      const u32 v0 = __ldg(&rowtot[t + q * RS_THREADS]);
+      const u32 x = warp_incl_sum(v0);
+      if (l == 31) wsum[w] = x;
+      __syncthreads();
+      u32 off = 0, tot = 0;
+      for (int ww = 0; ww < RS_WARPS; ++ww) {
+        if (ww < w) off += wsum[ww];
+        tot += wsum[ww];
+      }
+      gb[q] = carry + off + x - v0;
+      carry += tot;
+      __syncthreads();
+    }
+    if (n_out && blockIdx.x == 0 && t == 0) *n_out = carry;
+  } else {
+#pragma unroll
+    for (int q = 0; q < DPT; ++q) gb[q] = __ldg(&gbase[t + q * RS_THREADS]);
+  }
   u32 it = 0;
   for (u64 tile = blockIdx.x; tile < n_tiles; tile += gridDim.x, ++it) {
     const int st = (int)(it % RS_DSTAGES);
@@ -246,7 +277,7 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
     u32 go[DPT];
 #pragma unroll
     for (int q = 0; q < DPT; ++q)
-      go[q] = __ldg(&gbase[t + q * RS_THREADS]) + __ldg(&offs[(u64)(t + q * RS_THREADS) * tiles + tile]);
+      go[q] = gb[q] + __ldg(&offs[(u64)(t + q * RS_THREADS) * tiles + tile]);
     __syncthreads();
     mbar_wait(&bar[st], phase);
     u32 rank[RS_ITEMS];  // (digit << 16) | rank in the warp's digit run, NONE = no item
@@ -604,12 +635,17 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
     const int dr = (drop && p == 0) ? 1 : 0;
     k_rs_up<RB><<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles); ++g_launches;
     k_rs_rows<<<BINS, RS_THREADS, 0, st>>>(counts, tiles, ghist + p * RS_MAXB); ++g_launches;
-    k_rs_bins<RB><<<1, BINS < 1024 ? BINS : 1024, 0, st>>>(ghist + p * RS_MAXB, gbase + p * RS_MAXB,
-                                                          dr ? n_out_dev : nullptr);
-    ++g_launches;
-    k_rs_down<RB><<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, dsmem, st>>>(ki, vi, ko, vo, n, nd, dr,
-                                                                                              shift, counts, tiles,
-                                                                                              gbase + p * RS_MAXB);
+    // the digit bases come from the downsweep's own scan of the row totals, unless the kept count it
+    // publishes would overwrite the item count the same launch reads (n_dev == n_out_dev)
+    const bool fused = RS_FUSED_BINS && !(dr && nd == n_out_dev);
+    if (!fused) {
+      k_rs_bins<RB><<<1, BINS < 1024 ? BINS : 1024, 0, st>>>(ghist + p * RS_MAXB, gbase + p * RS_MAXB,
+                                                            dr ? n_out_dev : nullptr);
+      ++g_launches;
+    }
+    k_rs_down<RB><<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, dsmem, st>>>(
+        ki, vi, ko, vo, n, nd, dr, shift, counts, tiles, gbase + p * RS_MAXB, fused ? ghist + p * RS_MAXB : nullptr,
+        fused && dr ? n_out_dev : nullptr);
     ++g_launches;
     if (dr) nd = n_out_dev;
     u32* tk = ki; ki = ko; ko = tk;
