@@ -439,10 +439,18 @@ __global__ void __launch_bounds__(1024) k_scan_small(const u32* __restrict__ in,
   __shared__ u64 s_carry;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
   if (t == 0) s_carry = 0;
+  // every chunk's input is loaded before the first scan step: one memory round trip, not one per chunk
+  constexpr int CH = (int)(SC_SMALL / 1024);
+  u32 pre[CH];
+#pragma unroll
+  for (int j = 0; j < CH; ++j) pre[j] = (u64)j * 1024 + t < n ? in[(u64)j * 1024 + t] : 0u;
   __syncthreads();
-  for (u64 c0 = 0; c0 < n; c0 += 1024) {
+#pragma unroll
+  for (int j = 0; j < CH; ++j) {
+    const u64 c0 = (u64)j * 1024;
+    if (c0 >= n) break;
     const u64 i = c0 + t;
-    const u64 v = i < n ? in[i] : 0u;
+    const u64 v = pre[j];
     const u64 x = warp_incl_sum(v);
     if (l == 31) wsum[w] = x;
     __syncthreads();
