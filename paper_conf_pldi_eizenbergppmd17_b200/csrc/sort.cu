@@ -178,6 +178,10 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_rows(u32* __restrict__ counts
 // RS_DSTAGES tiles ahead (mbarrier ring), so the load latency that dominated a one-tile-per-CTA kernel
 // overlaps the ranking of the previous tile; the tile's values are loaded into registers at the start
 // of the tile and land while it is ranked.  Once scattered, the stage holds the permuted values.
+#ifndef RS_FASTRANK
+#define RS_FASTRANK 0  // shuffle + vote fast paths (all-distinct / all-equal digits) before MATCH.ANY:
+                       // A/B lost (C2 sort 0.279 -> 0.291 ms, C4 4.38 -> 4.69 ms; profiles/r1_ab_fastrank.txt)
+#endif
 #ifndef RS_FUSED_BINS
 #define RS_FUSED_BINS 1  // digit bases scanned inside k_rs_down (no k_rs_bins launch per pass)
 #endif
@@ -291,6 +295,16 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
       const u64 idx = base + li;
       const u32 k = idx < n ? sk[li] : KEY_DROP;
       dg[j] = (idx < n && !(drop && k == KEY_DROP)) ? ((k >> shift) & (BINS - 1)) : (u32)BINS;
+#if RS_FASTRANK
+      // warp-uniform fast paths before the (MIO-bound) MATCH.ANY: 32 strictly increasing digits are
+      // all distinct (low digits of consecutive granules), 32 equal digits are one run (high digits)
+      const u32 dprev = __shfl_up_sync(0xFFFFFFFFu, dg[j], 1);
+      if (__all_sync(0xFFFFFFFFu, l == 0 || dg[j] > dprev))
+        pr[j] = 1u << l;
+      else if (__all_sync(0xFFFFFFFFu, dg[j] == __shfl_sync(0xFFFFFFFFu, dg[j], 0)))
+        pr[j] = 0xFFFFFFFFu;
+      else
+#endif
       pr[j] = RS_MATCH_ANY ? __match_any_sync(0xFFFFFFFFu, dg[j]) : match_label<RB>(dg[j]);
     }
 #pragma unroll
