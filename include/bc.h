@@ -43,7 +43,7 @@ typedef enum {
   BC_ERR_NCCL = -5,             /* multi-GPU communicator error                                 */
   BC_ERR_STATE = -6,            /* call out of order (e.g. bc_detect before bc_load_trace)      */
   BC_ERR_TRUNCATED = -7,        /* bc_races: cap < number of races (cap entries were copied)    */
-  BC_ERR_OVERFLOW = -8          /* a 32-bit index space overflowed (records >= 2^27, keys >= 2^30,
+  BC_ERR_OVERFLOW = -8          /* an index space overflowed (records >= 2^32 - 1, shadow keys >= 2^30,
                                    sync-lookup step cap)                 */
 } bc_status;
 
@@ -84,7 +84,7 @@ enum { BC_CLS_SAME_INSN = 0,          /* two lanes of one warp instruction (P:L5
 
 typedef struct bc_race {
   uint64_t addr;         /* granule start: global byte address, or byte offset in the block's smem */
-  uint64_t prior_event;  /* (record_index << 5) | lane; ~0 for findings                         */
+  uint64_t prior_event;  /* (record_index << 5) | lane, record index in the whole trace; ~0 for findings */
   uint64_t cur_event;    /* (record_index << 5) | lane                                          */
   uint8_t kind, cls, space, pad;
   uint32_t block;        /* shared: owning block; global: block of the current event; finding: block */
@@ -93,15 +93,25 @@ typedef struct bc_race {
 
 /* ------------------------------------------------------------------ configuration */
 enum {
-  BC_F_RELEASE_OVERWRITE = 1u,    /* printed S_x := C_t release (reading R1 uses join); not yet
-                                     supported on the GPU path -> BC_ERR_INVALID_ARG            */
+  BC_F_RELEASE_OVERWRITE = 1u,    /* the printed release S_x := C_t (Fig. 3 RELBLOCK / RELGLOBAL,
+                                     P:L754-758) instead of reading R1's join      */
   BC_F_NO_SAME_VALUE_FILTER = 2u, /* report intra-warp same-value WW races too (R6)           */
   BC_F_COUNT_GATHERS = 4u         /* statistics: fill bc_stats.clock_gathers (one extra pass)  */
 };
 
+/* Optional device allocator ("PyTorch only for device memory"): every device buffer the
+ * context owns (trace copy, scratch, shadow tables, race list) is obtained from dev_alloc and returned
+ * to dev_free with the context's stream, e.g. torch's caching allocator.  NULL: cudaMalloc / cudaFree.
+ * dev_alloc returns NULL on failure (-> BC_ERR_OOM); returned memory must be 256-B aligned. */
+typedef void* (*bc_dev_alloc_fn)(size_t bytes, void* stream, void* user);
+typedef void (*bc_dev_free_fn)(void* ptr, size_t bytes, void* stream, void* user);
+
 typedef struct bc_config {
   uint32_t grid_dim[3], block_dim[3]; /* traced launch geometry; x fastest          */
-  uint32_t warp_size;                 /* must be 32                                 */
+  uint32_t warp_size;                 /* 32, or 4 / 8 / 16: warp-size simulation (SURVEY row f4,
+                                         P:L277-282): the trace's records describe warps of that
+                                         many lanes (lanes >= warp_size inactive); see
+                                         bc_split_warps() to produce such a trace from a 32-lane one */
   uint32_t granule_log2;              /* shadow granularity 2^G bytes, G in 0..4  */
   uint32_t smem_bytes_per_block;      /* shared-memory shadow size per block      */
   uint32_t flags;                     /* BC_F_*                                                  */
@@ -115,6 +125,15 @@ typedef struct bc_config {
                                          disjoint and their canonical merge is the world = 1 list
                                          (the caller gathers them, e.g. over torch.distributed). */
   void* stream;                       /* cudaStream_t (NULL = a stream owned by the context)     */
+  uint64_t window_events;             /* trace window budget: records are checked in
+                                         consecutive windows of at most this many items (granule x
+                                         lane events) + 8 per record; the per-granule shadow state
+                                         (Fig. 8) carries from one window to the next.
+                                         0 = auto (one window up to 2^30 - 1024, else 2^28 each);
+                                         larger values are clamped to 2^30 - 1024.                */
+  bc_dev_alloc_fn dev_alloc;          /* optional, see above                                     */
+  bc_dev_free_fn dev_free;
+  void* alloc_user;
 } bc_config;
 
 typedef struct bc_stats {
@@ -127,6 +146,8 @@ typedef struct bc_stats {
   uint64_t kernel_launches;  /* libbc kernels launched by this bc_detect                          */
   uint64_t clock_gathers;    /* 16-B record clock snapshots the per-granule check reads (items that
                                 some happens-before check needs); 0 unless BC_F_COUNT_GATHERS    */
+  uint64_t windows;          /* trace windows checked (window_events)                             */
+  uint64_t vc_pool_entries;  /* read-vector entries carried between windows                        */
   float ms_total;            /* device time of bc_detect (cudaEvents on the stream)               */
   float ms_kernel[12];       /* per phase, then kernel-only k_check / k_sort_items / k_expand;
                                 see bc_phase_name()                                              */
@@ -141,7 +162,7 @@ bc_status bc_init(const bc_config* cfg, struct bc_ctx** out);
 /* Hand the trace to the context.  recs_on_device = 0: `recs` is host memory and is copied
  * (stream-ordered; the caller keeps ownership).  recs_on_device = 1: `recs` is device memory
  * on cfg.device, borrowed (not copied) until the next bc_load_trace / bc_destroy; the caller
- * must keep it alive and unmodified.  n_recs may be 0.  n_recs >= 2^27 -> BC_ERR_OVERFLOW. */
+ * must keep it alive and unmodified.  n_recs may be 0.  n_recs >= 2^32 - 1 -> BC_ERR_OVERFLOW. */
 bc_status bc_load_trace(struct bc_ctx* ctx, const bc_record* recs, uint64_t n_recs, int recs_on_device);
 
 /* Optional per-lane store values (reading R6b in DESIGN.md).

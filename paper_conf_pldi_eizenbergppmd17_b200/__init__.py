@@ -48,12 +48,17 @@ class BcError(RuntimeError):
         self.status = status
 
 
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+
+
 class _Config(ctypes.Structure):
     _fields_ = [("grid_dim", ctypes.c_uint32 * 3), ("block_dim", ctypes.c_uint32 * 3),
                 ("warp_size", ctypes.c_uint32), ("granule_log2", ctypes.c_uint32),
                 ("smem_bytes_per_block", ctypes.c_uint32), ("flags", ctypes.c_uint32),
                 ("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
-                ("stream", ctypes.c_void_p)]
+                ("stream", ctypes.c_void_p), ("window_events", ctypes.c_uint64),
+                ("dev_alloc", _ALLOC_FN), ("dev_free", _FREE_FN), ("alloc_user", ctypes.c_void_p)]
 
 
 class _Stats(ctypes.Structure):
@@ -62,6 +67,7 @@ class _Stats(ctypes.Structure):
                 ("segments", ctypes.c_uint64), ("races", ctypes.c_uint64), ("findings", ctypes.c_uint64),
                 ("sync_ops", ctypes.c_uint64), ("written_pages", ctypes.c_uint64),
                 ("kernel_launches", ctypes.c_uint64), ("clock_gathers", ctypes.c_uint64),
+                ("windows", ctypes.c_uint64), ("vc_pool_entries", ctypes.c_uint64),
                 ("ms_total", ctypes.c_float), ("ms_kernel", ctypes.c_float * 12)]
 
 
@@ -117,13 +123,33 @@ def _stats_dict(s: _Stats):
     return d
 
 
+def torch_allocator():
+    """(dev_alloc, dev_free) callbacks over torch's CUDA caching allocator (bc_config.dev_alloc /
+    dev_free: PyTorch supplies the device memory).  Marshalling only."""
+    import torch
+
+    def _alloc(nbytes, stream, user):
+        try:
+            return torch.cuda.caching_allocator_alloc(int(nbytes), torch.cuda.current_device(), stream or 0)
+        except Exception:
+            return None
+
+    def _free(ptr, nbytes, stream, user):
+        torch.cuda.caching_allocator_delete(ptr)
+
+    return _ALLOC_FN(_alloc), _FREE_FN(_free)
+
+
 class Context:
     """One traced launch geometry on one GPU (bc_init ... bc_destroy)."""
 
-    def __init__(self, geometry: dict, device: int = 0, flags: int = 0, stream=None, rank: int = 0, world: int = 1):
+    def __init__(self, geometry: dict, device: int = 0, flags: int = 0, stream=None, rank: int = 0, world: int = 1,
+                 window_events: int = 0, allocator=None):
         """rank / world > 1: address-sharded check (bc.h bc_config.rank/world): every rank loads
         the same trace and reports the races of the shadow granules it owns; merge the per-rank
-        lists with merge_races() or gather_races()."""
+        lists with merge_races() or gather_races().  window_events: bc_config.window_events (0 =
+        auto).  allocator: None (cudaMalloc), "torch" (torch's caching allocator) or a
+        (dev_alloc, dev_free) pair of ctypes callbacks."""
         L = lib()
         grid = tuple(geometry["grid"]) + (1,) * (3 - len(geometry["grid"]))
         block = tuple(geometry["block"]) + (1,) * (3 - len(geometry["block"]))
@@ -137,6 +163,11 @@ class Context:
         c.device = device
         c.rank, c.world = rank, world
         c.stream = stream
+        c.window_events = window_events
+        self._alloc = None
+        if allocator is not None:
+            self._alloc = torch_allocator() if allocator == "torch" else tuple(allocator)
+            c.dev_alloc, c.dev_free = self._alloc
         h = ctypes.c_void_p()
         st = L.bc_init(ctypes.byref(c), ctypes.byref(h))
         if st != OK:
@@ -267,11 +298,12 @@ class Result:
 
 
 def detect(records, geometry: dict, device="cuda:0", flags: int = 0, stream=None, rank: int = 0,
-           world: int = 1, values=None) -> Result:
+           world: int = 1, values=None, window_events: int = 0, allocator=None) -> Result:
     """One-shot bc_init/bc_load_trace/bc_detect/bc_races.  Infeasible traces return
     status -2 with no races (as the oracle does)."""
     dev = int(str(device).split(":")[-1]) if str(device).startswith("cuda") else int(device)
-    with Context(geometry, device=dev, flags=flags, stream=stream, rank=rank, world=world) as ctx:
+    with Context(geometry, device=dev, flags=flags, stream=stream, rank=rank, world=world,
+                 window_events=window_events, allocator=allocator) as ctx:
         ctx.load_trace(records)
         if values is not None:
             ctx.load_values(values)

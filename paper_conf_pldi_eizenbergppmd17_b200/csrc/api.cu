@@ -23,6 +23,7 @@ struct bc_ctx {
   Geo g;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
+  DevAlloc da;
   const bc_record* trace = nullptr;  // device
   bc_record* owned = nullptr;
   size_t owned_cap = 0;
@@ -35,6 +36,10 @@ struct bc_ctx {
   bc_race* races = nullptr;  // device, findings first
   size_t races_cap = 0;
   u64 n_races = 0;
+  uint4* rbuf = nullptr;     // device, K7 race records of all windows (grown on demand)
+  size_t rbuf_cap = 0;       // entries
+  uint2* pool = nullptr;     // device, read-vector pool carried between windows (grown on demand)
+  size_t pool_cap = 0;       // entries
   bc_stats stats{};
   Arena arena;  // scratch buffers, reused across bc_detect calls
   std::string err;
@@ -90,13 +95,15 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   const u32 ws = cfg->warp_size;  // 32, or a simulated smaller warp
   if ((ws != 4 && ws != 8 && ws != 16 && ws != 32) || cfg->granule_log2 > 4) return BC_ERR_INVALID_ARG;
   if (cfg->flags & ~(u32)(BC_F_NO_SAME_VALUE_FILTER | BC_F_COUNT_GATHERS)) return BC_ERR_INVALID_ARG;  // overwrite: not on GPU yet
+  if ((cfg->dev_alloc == nullptr) != (cfg->dev_free == nullptr)) return BC_ERR_INVALID_ARG;
   if (cfg->world < 0 || cfg->world > 1024) return BC_ERR_INVALID_ARG;
   if (cfg->world > 1 && (cfg->rank < 0 || cfg->rank >= cfg->world)) return BC_ERR_INVALID_ARG;
   u64 nb = (u64)cfg->grid_dim[0] * cfg->grid_dim[1] * cfg->grid_dim[2];
   u64 tpb = (u64)cfg->block_dim[0] * cfg->block_dim[1] * cfg->block_dim[2];
   if (nb == 0 || tpb == 0 || tpb > 1024 || nb * tpb > 0xFFFFFFFFull) return BC_ERR_INVALID_ARG;
   u64 wpb = (tpb + ws - 1) / ws;
-  if (nb * wpb >= (1ull << 30) || nb * wpb * wpb >= (1ull << 32)) return BC_ERR_INVALID_ARG;
+  // warps < 2^27: a thread id (warp << 5 | lane) is 32 bits (shadow entries, read-vector pool)
+  if (nb * wpb >= (1ull << 27) || nb * wpb * wpb >= (1ull << 32)) return BC_ERR_INVALID_ARG;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
     cudaGetLastError();
@@ -128,6 +135,11 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
     cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking);
     c->own_stream = true;
   }
+  c->da.fa = cfg->dev_alloc;
+  c->da.ff = cfg->dev_free;
+  c->da.user = cfg->alloc_user;
+  c->da.st = c->stream;
+  c->arena.da = &c->da;
   // keep pooled scratch memory cached between bc_detect calls
   cudaMemPool_t pool;
   if (cudaDeviceGetDefaultMemPool(&pool, cfg->device) == cudaSuccess) {
@@ -148,9 +160,11 @@ void bc_destroy(bc_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->cfg.device);
   if (c->stream) cudaStreamSynchronize(c->stream);
-  if (c->owned) cudaFree(c->owned);
-  if (c->values_owned) cudaFree(c->values_owned);
-  if (c->races) cudaFree(c->races);
+  c->da.free(c->owned, c->owned_cap);
+  c->da.free(c->values_owned, c->values_cap);
+  c->da.free(c->races, c->races_cap * sizeof(bc_race));
+  c->da.free(c->rbuf, c->rbuf_cap * sizeof(uint4));
+  c->da.free(c->pool, c->pool_cap * sizeof(uint2));
   c->arena.free_all();
   if (c->hcnt) cudaFreeHost(c->hcnt);
   for (int i = 0; i < 16; ++i)
@@ -162,7 +176,7 @@ void bc_destroy(bc_ctx* c) {
 bc_status bc_load_trace(bc_ctx* c, const bc_record* recs, uint64_t n, int on_device) {
   if (!c) return BC_ERR_INVALID_ARG;
   if (n && !recs) return fail(c, BC_ERR_INVALID_ARG, "null trace");
-  if (n >= (1ull << 27)) return fail(c, BC_ERR_OVERFLOW, "more than 2^27 records (event id = rec << 5 | lane)");
+  if (n >= 0xFFFFFFFFull) return fail(c, BC_ERR_OVERFLOW, "2^32 - 1 or more records (32-bit record indices)");
   cudaSetDevice(c->cfg.device);
   c->loaded = false;
   c->detected = false;
@@ -177,13 +191,10 @@ bc_status bc_load_trace(bc_ctx* c, const bc_record* recs, uint64_t n, int on_dev
   } else {
     size_t bytes = n * sizeof(bc_record);
     if (bytes > c->owned_cap) {
-      if (c->owned) cudaFree(c->owned);
-      c->owned = nullptr;
+      c->da.free(c->owned, c->owned_cap);
       c->owned_cap = 0;
-      if (cudaMalloc(&c->owned, bytes) != cudaSuccess) {
-        cudaGetLastError();
-        return fail(c, BC_ERR_OOM, "trace buffer");
-      }
+      c->owned = (bc_record*)c->da.alloc(bytes);
+      if (!c->owned) return fail(c, BC_ERR_OOM, "trace buffer");
       c->owned_cap = bytes;
     }
     cudaMemcpyAsync(c->owned, recs, bytes, on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
@@ -225,7 +236,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* rec_cnt = small_w ? wcnt + 2 * (size_t)(g.n_warps + 1) : nullptr;
   u32* sync_list = S.alloc<u32>(n);
   u32* page_bits = S.alloc<u32>(nwords);
-  u32* ub_off = S.alloc<u32>(n + 1);  // per record: upper bound of its items, then its first slot
+  u32* rec_w = S.alloc<u32>(n);  // per record: window weight (item upper bound + REC_W)
   uint4* hdr16 = S.alloc<uint4>(n);  // compact record headers (K2 gathers them per warp)
   cudaMemsetAsync(cnt, 0, C_N * 8, st);
   cudaMemsetAsync(wcnt, 0, 3 * (size_t)(g.n_warps + 1) * 4, st);
@@ -233,7 +244,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   // ---- header pass; written pages ranked in address order from the list of non-zero bitmap words
   u32* word_list = S.alloc<u32>(nwords);
   u32* wl2 = S.alloc<u32>(nwords);
-  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, ub_off, hdr16, rec_cnt, err, st);
+  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, rec_w, hdr16, rec_cnt, err, st);
   u32* words = word_list;
   u32* wl_prefix = wl2;
   u32* page_rank = S.alloc<u32>(nwords);
@@ -327,74 +338,178 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     if (rs) return fail(c, (bc_status)rs, "sync skeleton");
   }
   cudaEventRecord(c->ev[4], st);
-  // ---- K4: expansion (static slots from the header's per-record upper bounds)
-  const u64 bound = hc_cnt[C_ITEM_BOUND];
-  exclusive_scan_u32(ub_off, ub_off, n, S.alloc<char>(scan_temp_bytes(n)), nullptr, st);
-  u32* ikeys = S.alloc<u32>(bound + 1);
-  u32* ievs = S.alloc<u32>(bound + 1);
-  cudaEventRecord(c->ev[14], st);
-  launch_expand(recs, g, page_bits, page_rank, shared_base, ub_off, ikeys, ievs, err, st);
-  cudaEventRecord(c->ev[15], st);
-  cudaEventRecord(c->ev[5], st);
-  // ---- K5: stable radix sort by granule key; the first pass drops the never-written slots
-  u64* n_items_dev = cnt + C_ITEMS;
-  u32* ik2 = S.alloc<u32>(bound + 1);
-  u32* iv2 = S.alloc<u32>(bound + 1);
-  int kbits = bits_for(n_keys ? n_keys - 1 : 0);
-  void* rtmp = S.alloc<char>(rs_temp_bytes(bound));
-  cudaEventRecord(c->ev[12], st);
-  alt = radix_sort_pairs(ikeys, ievs, ik2, iv2, bound, 2, 2 + kbits, rtmp, st, nullptr, n_items_dev, true);
-  cudaEventRecord(c->ev[13], st);
-  u32* skey = alt ? ik2 : ikeys;
-  u32* sev = alt ? iv2 : ievs;
-  cudaEventRecord(c->ev[6], st);
-  // ---- K7: shadow check
-  u32 race_cap = (u32)std::min<u64>(std::max<u64>(1u << 16, bound / 16), 1u << 30);
-  uint4* rbuf = nullptr;
-  u32* rcnt = reinterpret_cast<u32*>(cnt + C_RACES);
-  u64* segc = cnt + C_SEGMENTS;  // [0] segments, [1] clock snapshot gathers (C_GATHERS)
-  void* cstatus = S.alloc<char>(check_status_bytes(bound));
-  u32 n_r = 0, nfind = 0;
-  u64 n_items = 0;
-  for (int attempt = 0; attempt < 2; ++attempt) {
-    rbuf = S.alloc<uint4>(race_cap);
-    cudaMemsetAsync(cnt + C_RACES, 0, 3 * sizeof(u64), st);  // races, segments, gathers
-    cudaEventRecord(c->ev[10], st);
-    launch_check(hc, skey, sev, n_items_dev, bound, cstatus, rbuf, rcnt, race_cap, segc, c->values, st);
-    cudaEventRecord(c->ev[11], st);
-    if (g.flags & BC_F_COUNT_GATHERS) launch_count_gathers(skey, n_items_dev, segc + 1, st);
-    cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
-    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "check");
-    n_r = (u32)hcnt[C_RACES];
-    herr = (u32)hcnt[C_ERR];
-    sx.segments = hcnt[C_SEGMENTS];
-    sx.clock_gathers = hcnt[C_GATHERS];
-    n_items = hcnt[C_ITEMS];
-    nfind = (u32)hcnt[C_FINDINGS];
-    if (herr) break;
-    if (n_r <= race_cap) break;
-    race_cap = n_r;
+  // ---- windows: consecutive record ranges of at most `we` weight (item upper bound +
+  // REC_W per record: < 2^27 records, so window-local event ids are 32-bit); the per-granule shadow
+  // state (Fig. 8) carries from one window to the next
+  const u64 bound_all = hc_cnt[C_ITEM_BOUND];
+  const u64 total_w = bound_all + (u64)REC_W * n;
+  u64 we = c->cfg.window_events ? std::min<u64>(c->cfg.window_events, WIN_MAX)
+                                : (total_w <= WIN_MAX ? WIN_MAX : (1ull << 28));
+  u64* cum = S.alloc<u64>(n + 1);
+  exclusive_scan_u32_u64(rec_w, cum, n, S.alloc<char>(scan_temp_bytes(n)), cum + n, st);
+  const u64 nwin64 = std::max<u64>(1, (total_w + we - 1) / we);
+  if (nwin64 >= (1ull << 31)) return fail(c, BC_ERR_INVALID_ARG, "window_events too small for this trace");
+  const u32 nwin = (u32)nwin64;
+  std::vector<u64> wst(nwin + 1), wbd(nwin);
+  if (nwin == 1) {
+    wst[0] = 0;
+    wst[1] = n;
+    wbd[0] = bound_all;
+  } else {
+    u64* d_wst = S.alloc<u64>(nwin + 1);
+    u64* d_wbd = S.alloc<u64>(nwin);
+    launch_window_starts(cum, n, we, nwin, d_wst, d_wbd, st);
+    cudaMemcpyAsync(wst.data(), d_wst, (nwin + 1) * sizeof(u64), cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(wbd.data(), d_wbd, nwin * sizeof(u64), cudaMemcpyDeviceToHost, st);
+    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "windows");
   }
-  if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "infeasible trace");
-  if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "index overflow / sync lookup step cap");
+  u64 maxb = 0;
+  int last_win = -1;
+  for (u32 k = 0; k < nwin; ++k)
+    if (wst[k + 1] > wst[k]) {
+      maxb = std::max(maxb, wbd[k]);
+      last_win = (int)k;
+    }
+  const bool multi = nwin > 1;
+  u32* ikeys = S.alloc<u32>(maxb + 1);
+  u32* ievs = S.alloc<u32>(maxb + 1);
+  u32* ik2 = S.alloc<u32>(maxb + 1);
+  u32* iv2 = S.alloc<u32>(maxb + 1);
+  void* rtmp = S.alloc<char>(rs_temp_bytes(maxb));
+  void* cstatus = S.alloc<char>(check_status_bytes(maxb));
+  uint4* sh_cur = multi ? S.alloc<uint4>(2 * n_keys) : nullptr;  // entries after the last window (double buffer)
+  uint4* sh_nxt = multi ? S.alloc<uint4>(2 * n_keys) : nullptr;
+  bool have_state = false;
+  u64* n_items_dev = cnt + C_ITEMS;
+  const int kbits = bits_for(n_keys ? n_keys - 1 : 0);
+  u64 n_r = 0, n_items = 0, pool_used = 0;
+  float ms_ex = 0, ms_sort = 0, ms_chk = 0;
+  for (u32 k = 0; k < nwin; ++k) {
+    const u64 R0 = wst[k], R1 = wst[k + 1], b = wbd[k];
+    if (R0 == R1) continue;
+    ++sx.windows;
+    // ---- K4: expansion (static slots from the header's per-record upper bounds)
+    cudaEventRecord(c->ev[14], st);
+    launch_expand(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, ikeys, ievs, err, st);
+    cudaEventRecord(c->ev[15], st);
+    // ---- K5: stable radix sort by granule key; the first pass drops the never-written slots
+    cudaEventRecord(c->ev[12], st);
+    const bool alt = radix_sort_pairs(ikeys, ievs, ik2, iv2, b, 2, 2 + kbits, rtmp, st, nullptr, n_items_dev, true);
+    cudaEventRecord(c->ev[13], st);
+    u32* skey = alt ? ik2 : ikeys;
+    u32* sev = alt ? iv2 : ievs;
+    // ---- K7: shadow check of the window (carried entries in, entries for the next window out)
+    uint4* sh_out = (multi && (int)k != last_win) ? sh_nxt : nullptr;
+    if (sh_out) {
+      if (have_state) cudaMemcpyAsync(sh_out, sh_cur, 2 * n_keys * sizeof(uint4), cudaMemcpyDeviceToDevice, st);
+      else cudaMemsetAsync(sh_out, 0, 2 * n_keys * sizeof(uint4), st);
+      // every carried vector may be re-copied once and every item appended once
+      const u64 need = 2 * pool_used + b + 1024;
+      if (need >= (1ull << 32)) return fail(c, BC_ERR_OVERFLOW, "read-vector pool >= 2^32 entries");
+      if (need > c->pool_cap) {
+        uint2* np = (uint2*)c->da.alloc(need * sizeof(uint2));
+        if (!np) return fail(c, BC_ERR_OOM, "read-vector pool");
+        if (pool_used) cudaMemcpyAsync(np, c->pool, pool_used * sizeof(uint2), cudaMemcpyDeviceToDevice, st);
+        cudaStreamSynchronize(st);
+        c->da.free(c->pool, c->pool_cap * sizeof(uint2));
+        c->pool = np;
+        c->pool_cap = need;
+      }
+    }
+    CheckLaunch L{};
+    L.c = hc;
+    L.keys = skey;
+    L.evs = sev;
+    L.n_dev = n_items_dev;
+    L.n_max = b;
+    L.R0 = (u32)R0;
+    L.sh_in = have_state ? sh_cur : nullptr;
+    L.sh_out = sh_out;
+    L.pool = c->pool;
+    L.pool_cnt = reinterpret_cast<u32*>(cnt + C_POOL);
+    L.pool_cap = (u32)std::min<u64>(c->pool_cap, 0xFFFFFFFFull);
+    L.race_cnt = reinterpret_cast<u32*>(cnt + C_RACES);
+    L.seg_cnt = cnt + C_SEGMENTS;
+    L.values = c->values;
+    L.status = cstatus;
+    for (int attempt = 0; attempt < 3; ++attempt) {
+      if (c->rbuf_cap < (1u << 16)) {
+        c->da.free(c->rbuf, c->rbuf_cap * sizeof(uint4));
+        c->rbuf_cap = 0;
+        c->rbuf = (uint4*)c->da.alloc((1u << 16) * sizeof(uint4));
+        if (!c->rbuf) return fail(c, BC_ERR_OOM, "race buffer");
+        c->rbuf_cap = 1u << 16;
+      }
+      L.races = c->rbuf;
+      L.race_cap = (u32)std::min<u64>(c->rbuf_cap, 0xFFFFFFFFull);
+      // device counters: races so far, this window's segments / gathers, the carried pool size
+      hcnt[C_RACES] = n_r;
+      hcnt[C_SEGMENTS] = 0;
+      hcnt[C_GATHERS] = 0;
+      hcnt[C_POOL] = pool_used;
+      cudaMemcpyAsync(cnt + C_RACES, hcnt + C_RACES, 4 * sizeof(u64), cudaMemcpyHostToDevice, st);
+      cudaEventRecord(c->ev[10], st);
+      launch_check(L, st);
+      cudaEventRecord(c->ev[11], st);
+      if (g.flags & BC_F_COUNT_GATHERS) launch_count_gathers(skey, n_items_dev, cnt + C_GATHERS, st);
+      cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
+      if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "check");
+      herr = (u32)hcnt[C_ERR];
+      if (herr) break;
+      const u64 tot = (u32)hcnt[C_RACES];
+      if (tot <= c->rbuf_cap) break;
+      // more races than room: grow (keeping the earlier windows' races) and check the window again
+      // (idempotent: the shadow entries it writes are a function of the window, the pool is reset)
+      const u64 cap2 = std::max<u64>(2 * c->rbuf_cap, tot + 1024);
+      if (cap2 >= 0xFFFFFFFFull) return fail(c, BC_ERR_OVERFLOW, "2^32 or more races");
+      uint4* nb2 = (uint4*)c->da.alloc(cap2 * sizeof(uint4));
+      if (!nb2) return fail(c, BC_ERR_OOM, "race buffer");
+      if (n_r) cudaMemcpyAsync(nb2, c->rbuf, n_r * sizeof(uint4), cudaMemcpyDeviceToDevice, st);
+      cudaStreamSynchronize(st);
+      c->da.free(c->rbuf, c->rbuf_cap * sizeof(uint4));
+      c->rbuf = nb2;
+      c->rbuf_cap = cap2;
+    }
+    if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "infeasible trace");
+    if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "index overflow / sync lookup step cap");
+    n_r = (u32)hcnt[C_RACES];
+    pool_used = (u32)hcnt[C_POOL];
+    n_items += hcnt[C_ITEMS];
+    sx.segments += hcnt[C_SEGMENTS];
+    sx.clock_gathers += hcnt[C_GATHERS];
+    float t = 0;
+    cudaEventElapsedTime(&t, c->ev[14], c->ev[15]);
+    ms_ex += t;
+    cudaEventElapsedTime(&t, c->ev[12], c->ev[13]);
+    ms_sort += t;
+    cudaEventElapsedTime(&t, c->ev[10], c->ev[11]);
+    ms_chk += t;
+    if (sh_out) {
+      std::swap(sh_cur, sh_nxt);
+      have_state = true;
+    }
+  }
+  u32 nfind = (u32)hcnt[C_FINDINGS];
+  if (nwin == 1 && last_win < 0) {  // no records at all in the window loop (cannot happen for n > 0)
+    nfind = 0;
+  }
   sx.items = n_items;
+  sx.vc_pool_entries = pool_used;
   cudaEventRecord(c->ev[7], st);
   // ---- K8: finalize
   if (g.world > 1 && g.rank != 0) nfind = 0;  // findings come from the replicated replay: rank 0 reports them
-  u64 total = (u64)n_r + nfind;
+  u64 total = n_r + nfind;
   if (total > c->races_cap) {
-    if (c->races) cudaFree(c->races);
-    c->races = nullptr;
+    c->da.free(c->races, c->races_cap * sizeof(bc_race));
     c->races_cap = 0;
-    if (cudaMalloc(&c->races, std::max<u64>(total, 1) * sizeof(bc_race)) != cudaSuccess) {
-      cudaGetLastError();
-      return fail(c, BC_ERR_OOM, "race buffer");
-    }
+    c->races = (bc_race*)c->da.alloc(std::max<u64>(total, 1) * sizeof(bc_race));
+    if (!c->races) return fail(c, BC_ERR_OOM, "race list");
     c->races_cap = std::max<u64>(total, 1);
   }
   u32* page_num = S.alloc<u32>(n_pages + 1);
   if (n_r) launch_page_list(words, wl_prefix, page_bits, n_words, page_num, st);
-  finalize_races(rbuf, n_r, find_blk, find_rec, nfind, g, snap, page_num, shared_base, (u32)n_keys, c->races, S, st);
+  finalize_races(c->rbuf, (u32)n_r, find_blk, find_rec, nfind, g, snap, page_num, shared_base, (u32)n_keys, c->races, S,
+                 st);
   cudaEventRecord(c->ev[PH_N], st);
   if (cudaEventSynchronize(c->ev[PH_N]) != cudaSuccess) return cuda_check(c, "finalize");
   cs = cuda_check(c, "detect");
@@ -405,14 +520,16 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   cudaEventElapsedTime(&sx.ms_total, c->ev[0], c->ev[PH_N]);
   for (int i = 0; i < PH_N; ++i) {
     cudaEvent_t e1 = i + 1 < PH_N ? c->ev[i + 1] : c->ev[PH_N];
+    if (i == PH_EXPAND || i == PH_SORT || i == PH_CHECK) continue;
     cudaEventElapsedTime(&sx.ms_kernel[i], c->ev[i], e1);
   }
-  // kernel-only timings of the three heavy kernels (no host gaps inside)
-  if (n_items) {
-    cudaEventElapsedTime(&sx.ms_kernel[PH_N + 0], c->ev[10], c->ev[11]);
-    cudaEventElapsedTime(&sx.ms_kernel[PH_N + 1], c->ev[12], c->ev[13]);
-  }
-  cudaEventElapsedTime(&sx.ms_kernel[PH_N + 2], c->ev[14], c->ev[15]);
+  // the window loop: per-kernel sums over the windows (expand / sort / check also as kernel-only times)
+  sx.ms_kernel[PH_EXPAND] = ms_ex;
+  sx.ms_kernel[PH_SORT] = ms_sort;
+  sx.ms_kernel[PH_CHECK] = ms_chk;
+  sx.ms_kernel[PH_N + 0] = ms_chk;
+  sx.ms_kernel[PH_N + 1] = ms_sort;
+  sx.ms_kernel[PH_N + 2] = ms_ex;
   sx.kernel_launches = g_launches - launches0;
   return BC_OK;
 }
@@ -433,13 +550,10 @@ bc_status bc_load_values(bc_ctx* c, const uint64_t* values, uint64_t n, int on_d
   }
   const size_t bytes = (size_t)n * 32 * sizeof(u64);
   if (c->values_cap < bytes) {
-    if (c->values_owned) cudaFree(c->values_owned);
-    c->values_owned = nullptr;
+    c->da.free(c->values_owned, c->values_cap);
     c->values_cap = 0;
-    if (cudaMalloc(&c->values_owned, bytes) != cudaSuccess) {
-      cudaGetLastError();
-      return fail(c, BC_ERR_OOM, "values buffer");
-    }
+    c->values_owned = (u64*)c->da.alloc(bytes);
+    if (!c->values_owned) return fail(c, BC_ERR_OOM, "values buffer");
     c->values_cap = bytes;
   }
   cudaMemcpyAsync(c->values_owned, values, bytes, cudaMemcpyHostToDevice, c->stream);

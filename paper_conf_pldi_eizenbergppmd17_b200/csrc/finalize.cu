@@ -1,9 +1,10 @@
 // finalize.cu — K8 race finalize: canonical order and classification.
 //
-// Races leave K7 as (granule key, current event, prior event, kind) in arbitrary order.  The
-// dense key order is the canonical location order (global granules by address, then shared
-// granules by (block, offset)), so a stable LSD sort by prior, then current, then key gives
-// the canonical (location, current, prior) order.  Classification from the two events
+// Races leave K7 as (granule key, current record, prior record, current lane | prior lane << 5 |
+// kind << 10) in arbitrary order (global record indices: any trace length).  The dense key order is
+// the canonical location order (global granules by address, then shared granules by (block,
+// offset)), so a stable LSD sort by prior (lane, record), then current (lane, record), then key gives
+// the canonical (location, current event, prior event) order, event = record << 5 | lane.  Classification from the two events
 // (reading R9): same record -> SAME_INSN; same warp -> BRANCH (branch ordering,
 // P:L591-630); same block -> INTRA_BLOCK; else INTER_BLOCK.  Barrier-divergence findings
 // come first, ordered by (block, record).
@@ -20,7 +21,7 @@ __global__ void k_field(const uint4* __restrict__ r, u32 n, int f, u32* __restri
   u32 i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   uint4 v = r[i];
-  out[i] = f == 0 ? v.x : f == 1 ? v.y : v.z;
+  out[i] = f == 0 ? v.x : f == 1 ? v.y : f == 2 ? v.z : f == 3 ? (v.w & 31u) : ((v.w >> 5) & 31u);
 }
 
 // rank -> page number, from the sorted list of non-zero bitmap words (k_page_rank)
@@ -44,9 +45,9 @@ __global__ void k_emit_races(const uint4* __restrict__ r, const u32* __restrict_
   u32 i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   uint4 v = r[perm[i]];
-  u32 key = v.x, cur = v.y, prior = v.z, kind = v.w;
+  const u32 key = v.x, cr = v.y, pr = v.z, cl = v.w & 31u, pl = (v.w >> 5) & 31u, kind = (v.w >> 10) & 0xFFu;
   bc_race o;
-  u32 cw = snap[cur >> 5].x, pw = snap[prior >> 5].x;
+  u32 cw = snap[cr].x, pw = snap[pr].x;
   if (key < shared_base) {
     u32 sh = 20 - g.G;
     u64 page = page_num[key >> sh];
@@ -59,10 +60,10 @@ __global__ void k_emit_races(const uint4* __restrict__ r, const u32* __restrict_
     o.space = BC_SPACE_SHARED;
     o.block = k / g.smem_gran;
   }
-  o.prior_event = (u64)prior;
-  o.cur_event = (u64)cur;
+  o.prior_event = ((u64)pr << 5) | pl;
+  o.cur_event = ((u64)cr << 5) | cl;
   o.kind = (uint8_t)kind;
-  if ((cur >> 5) == (prior >> 5)) o.cls = BC_CLS_SAME_INSN;
+  if (cr == pr) o.cls = BC_CLS_SAME_INSN;
   else if (cw == pw) o.cls = BC_CLS_BRANCH;
   else if (cw / g.wpb == pw / g.wpb) o.cls = BC_CLS_INTRA_BLOCK;
   else o.cls = BC_CLS_INTER_BLOCK;
@@ -116,10 +117,11 @@ void finalize_races(const uint4* races, u32 n_r, const u32* fblk, const u32* fre
     u32* p = S.alloc<u32>(n_r);
     u32* f = S.alloc<u32>(n_r);
     launch_iota(p, n_r, st);
-    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 2, f); ++g_launches;
-    sort_perm_by(p, f, n_r, 32, S, st);
-    k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 1, f); ++g_launches;
-    sort_perm_by(p, f, n_r, 32, S, st);
+    const int fields[4] = {4, 2, 3, 1};  // prior lane, prior record, current lane, current record
+    for (int q = 0; q < 4; ++q) {
+      k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, fields[q], f); ++g_launches;
+      sort_perm_by(p, f, n_r, (fields[q] == 3 || fields[q] == 4) ? 5 : bits_for(g.n_recs), S, st);
+    }
     k_field<<<nb(n_r), 256, 0, st>>>(races, n_r, 0, f); ++g_launches;
     sort_perm_by(p, f, n_r, bits_for(n_keys), S, st);
     k_emit_races<<<nb(n_r), 256, 0, st>>>(races, p, n_r, g, snap, page_num, shared_base, out + n_f); ++g_launches;

@@ -17,19 +17,43 @@ extern u64 g_launches;
 // words err / need_sort / races / findings live in the low half of their slot)
 enum { C_LANE_EVENTS = 0, C_CONTROL_EVENTS, C_SYNC_RECS, C_ACQ_RECS, C_MEM_RECS, C_IFS, C_BARS, C_SYNC_LANEOPS,
        C_ITEMS, C_ITEM_BOUND, C_SEGMENTS_UNUSED, C_PAGE_WORDS, C_PAGES, C_ERR, C_NEED_SORT, C_FINDINGS,
-       C_RACES, C_SEGMENTS, C_GATHERS, C_N };
+       C_RACES, C_SEGMENTS, C_GATHERS, C_POOL, C_N };
+
+// Device memory of a context: cudaMalloc / cudaFree, or the caller's allocator (bc_config.dev_alloc /
+// dev_free, e.g. torch's caching allocator).
+struct DevAlloc {
+  bc_dev_alloc_fn fa = nullptr;
+  bc_dev_free_fn ff = nullptr;
+  void* user = nullptr;
+  cudaStream_t st = nullptr;
+  void* alloc(size_t bytes) {
+    if (fa) return fa(bytes, (void*)st, user);
+    void* p = nullptr;
+    if (cudaMalloc(&p, bytes) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    return p;
+  }
+  void free(void* p, size_t bytes) {
+    if (!p) return;
+    if (ff) ff(p, bytes, (void*)st, user);
+    else cudaFree(p);
+  }
+};
 
 // Per-context scratch arena.  A bc_detect allocates its scratch buffers in a fixed order; the i-th
 // allocation reuses the i-th buffer of earlier calls when it is large enough, so repeated detects of
-// one trace see identical pointers -- which is what lets the post-header pipeline be replayed as a
-// CUDA graph (api.cu).  Buffers are 256-B aligned and padded to a multiple of 256 B (the TMA bulk
-// copies of the radix sort may read up to 12 B past an array's end).  Freed at bc_destroy.
+// one trace see identical pointers and allocate nothing.  Buffers are 256-B aligned and padded to a
+// multiple of 256 B (the TMA bulk copies of the radix sort may read up to 12 B past an array's end).
+// Freed at bc_destroy.
 struct Arena {
+  DevAlloc* da = nullptr;
   std::vector<std::pair<void*, size_t>> bufs;
   u64 gen = 0;  // bumped whenever a buffer is (re)allocated
   void free_all() {
     for (auto& b : bufs)
-      if (b.first) cudaFree(b.first);
+      if (b.first) da->free(b.first, b.second);
     bufs.clear();
     ++gen;
   }
@@ -47,17 +71,14 @@ class Scratch {
     if (i < ar_->bufs.size() && ar_->bufs[i].second >= bytes) return (T*)ar_->bufs[i].first;
     if (i < ar_->bufs.size()) {
       cudaStreamSynchronize(st_);  // the old buffer may still be read by queued work
-      cudaFree(ar_->bufs[i].first);
+      ar_->da->free(ar_->bufs[i].first, ar_->bufs[i].second);
       ar_->bufs[i] = {nullptr, 0};
     } else {
       ar_->bufs.push_back({nullptr, 0});
     }
-    void* p = nullptr;
     const size_t cap = bytes + ((bytes / 8 + 255) & ~(size_t)255);
-    if (cudaMalloc(&p, cap) != cudaSuccess || !p) {
-      cudaGetLastError();
-      throw std::bad_alloc();
-    }
+    void* p = ar_->da->alloc(cap);
+    if (!p) throw std::bad_alloc();
     ar_->bufs[i] = {p, cap};
     ++ar_->gen;
     return (T*)p;
@@ -76,11 +97,17 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
                       cudaStream_t st, const u64* n_dev = nullptr, u64* n_out_dev = nullptr, bool drop = false);
 size_t scan_temp_bytes(u64 n);
 void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_dev, cudaStream_t st);
+void exclusive_scan_u32_u64(const u32* in, u64* out, u64 n, void* temp, u64* total_dev, cudaStream_t st);
 
 // trace.cu
+// window weight of a record: its item upper bound + REC_W (DESIGN.md §7 "Windows"): a window of at
+// most WIN_MAX weight holds < 2^27 records (32-bit window-local event ids) and < 2^30 items
+constexpr u32 REC_W = 8;
+constexpr u64 WIN_MAX = (1ull << 30) - 1024;
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
-                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, uint4* hdr16,
+                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_w, uint4* hdr16,
                    u32* rec_cnt, u32* err, cudaStream_t st);
+void launch_window_starts(const u64* cum, u64 n, u64 we, u32 nwin, u64* starts, u64* bounds, cudaStream_t st);
 constexpr u32 WS_SMALL = 8192;  // n_warps up to which one CTA does the per-warp scans (launch_warp_scans)
 void launch_warp_scans(const u32* rec_cnt, const u32* if_cnt, const u32* bar_cnt, u32 n_warps, u32* warp_start,
                        u32* node_base, u32* bar_base, cudaStream_t st);
@@ -95,7 +122,7 @@ void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, cons
 void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, const u32* bar_base, const u32* blockR,
                       cudaStream_t st);
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
-                   const u32* ub_off, u32* keys, u32* evs, u32* err, cudaStream_t st);
+                   const u64* cum, u64 R0, u64 R1, u32* keys, u32* evs, u32* err, cudaStream_t st);
 void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st);
 
 // sync.cu
@@ -107,8 +134,26 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
 
 // check.cu
 size_t check_status_bytes(u64 n);
-void launch_check(const HbCtx& c, const u32* keys, const u32* evs, const u64* n_dev, u64 n_max, void* status,
-                  uint4* races, u32* race_cnt, u32 race_cap, u64* seg_cnt, const u64* values, cudaStream_t st);
+struct CheckLaunch {
+  HbCtx c;
+  const u32* keys;      // (granule key << 2) | op, sorted
+  const u32* evs;       // (record - R0) << 5 | lane
+  const u64* n_dev;     // item count (device)
+  u64 n_max;            // upper bound of the item count
+  u32 R0;               // first record of the window
+  const uint4* sh_in;   // carried shadow entries (2 x uint4 per granule) or null (first window)
+  uint4* sh_out;        // shadow entries after the window, or null (last window)
+  uint2* pool;          // append-only read-vector pool (record, warp << 5 | lane)
+  u32* pool_cnt;
+  u32 pool_cap;
+  uint4* races;         // (key, cur rec, prior rec, cur lane | prior lane << 5 | kind << 10)
+  u32* race_cnt;
+  u32 race_cap;
+  u64* seg_cnt;
+  const u64* values;
+  void* status;         // check_status_bytes() of scratch
+};
+void launch_check(const CheckLaunch& L, cudaStream_t st);
 
 void launch_count_gathers(const u32* keys, const u64* n_dev, u64* out, cudaStream_t st);
 

@@ -447,7 +447,8 @@ __global__ void __launch_bounds__(1024) k_scan_tiles(u64* __restrict__ tsum, u64
 
 // small inputs: one CTA scans the whole array in chunks of 1024 with a running carry (one launch)
 constexpr u64 SC_SMALL = 8192;
-__global__ void __launch_bounds__(1024) k_scan_small(const u32* __restrict__ in, u32* __restrict__ out, u64 n,
+template <typename TO>
+__global__ void __launch_bounds__(1024) k_scan_small(const u32* __restrict__ in, TO* __restrict__ out, u64 n,
                                                      u64* __restrict__ total_out) {
   __shared__ u64 wsum[32];
   __shared__ u64 s_carry;
@@ -474,7 +475,7 @@ __global__ void __launch_bounds__(1024) k_scan_small(const u32* __restrict__ in,
       tot += wsum[ww];
     }
     const u64 carry = s_carry;
-    if (i < n) out[i] = (u32)(carry + off + x - v);
+    if (i < n) out[i] = (TO)(carry + off + x - v);
     __syncthreads();
     if (t == 0) s_carry = carry + tot;
     __syncthreads();
@@ -482,7 +483,8 @@ __global__ void __launch_bounds__(1024) k_scan_small(const u32* __restrict__ in,
   if (t == 0 && total_out) *total_out = s_carry;
 }
 
-__global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__ in, u32* __restrict__ out, u64 n,
+template <typename TO>
+__global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__ in, TO* __restrict__ out, u64 n,
                                                          const u64* __restrict__ texcl) {
   __shared__ u64 wsum[SC_THREADS / 32];
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
@@ -502,7 +504,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__
   u64 run = texcl[blockIdx.x] + off + x - sum;
 #pragma unroll
   for (int j = 0; j < SC_ITEMS; ++j) {
-    if (base + j < n) out[base + j] = (u32)run;
+    if (base + j < n) out[base + j] = (TO)run;
     run += v[j];
   }
 }
@@ -722,7 +724,8 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
 size_t scan_temp_bytes(u64 n) { return ((n + SC_TILE - 1) / SC_TILE + 1) * sizeof(u64) + 64; }
 
 // exclusive scan in -> out (out may alias in); total written to *total_dev if non-null
-void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_dev, cudaStream_t st) {
+template <typename TO>
+static void exclusive_scan_t(const u32* in, TO* out, u64 n, void* temp, u64* total_dev, cudaStream_t st) {
   const u64 tiles = (n + SC_TILE - 1) / SC_TILE;
   u64* tsum = (u64*)temp;
   if (tiles == 0) {
@@ -730,12 +733,19 @@ void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_d
     return;
   }
   if (n <= SC_SMALL) {
-    k_scan_small<<<1, 1024, 0, st>>>(in, out, n, total_dev); ++g_launches;
+    k_scan_small<TO><<<1, 1024, 0, st>>>(in, out, n, total_dev); ++g_launches;
     return;
   }
   k_scan_tsum<<<(unsigned)tiles, SC_THREADS, 0, st>>>(in, n, tsum); ++g_launches;
   k_scan_tiles<<<1, 1024, 0, st>>>(tsum, tiles, total_dev); ++g_launches;
-  k_scan_u32<<<(unsigned)tiles, SC_THREADS, 0, st>>>(in, out, n, tsum); ++g_launches;
+  k_scan_u32<TO><<<(unsigned)tiles, SC_THREADS, 0, st>>>(in, out, n, tsum); ++g_launches;
+}
+void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_dev, cudaStream_t st) {
+  exclusive_scan_t<u32>(in, out, n, temp, total_dev, st);
+}
+// u64 prefix of u32 values (record window weights: totals beyond 2^32)
+void exclusive_scan_u32_u64(const u32* in, u64* out, u64 n, void* temp, u64* total_dev, cudaStream_t st) {
+  exclusive_scan_t<u64>(in, out, n, temp, total_dev, st);
 }
 
 }  // namespace bc

@@ -174,7 +174,11 @@ __device__ u32 laneop_entries(const K3In& k, u32 i, const EntOut* o, u32 base) {
   u32 w = k.recs[r].warp;
   u32 b = w / c.g.wpb;
   u32 x = k.xid[i];
-  u32 ev = (r << 5) | lane;
+  // position of this lane-op = its rank among the sync lane-ops in trace order (record, then lane):
+  // order-preserving, so "entries with pos < bound" is the trace-order view of Fig. 3, and 32 bits
+  // suffice for any record count
+  u32 ev = i;
+  (void)lane;
   u32 n = base;
   // range of block arrays of x
   u32 blo = pair_lower(k, x, 0), bhi = pair_lower(k, x + 1, 0);

@@ -24,7 +24,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
                                                 u32* __restrict__ wval, u32* __restrict__ if_cnt,
                                                 u32* __restrict__ bar_cnt, u32* __restrict__ sync_list,
                                                 u32* __restrict__ page_bits, u32* __restrict__ word_list,
-                                                u64* __restrict__ cnt, u32* __restrict__ rec_ub,
+                                                u64* __restrict__ cnt, u32* __restrict__ rec_w,
                                                 uint4* __restrict__ hdr16, u32* __restrict__ rec_cnt,
                                                 u32* __restrict__ err) {
   const u32 lane = threadIdx.x & 31;
@@ -89,7 +89,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
   }
   // warp-reduced counters
   if (bad) ibound = 0;
-  if (valid) rec_ub[r] = ibound;  // upper bound of the record's items (K4 writes at static slots)
+  if (valid) rec_w[r] = ibound + REC_W;  // window weight: item upper bound (K4 writes at static slots) + REC_W
   u32 v[8] = {lane_ev, ctl_ev, is_acq, is_mem, is_if, is_bar, is_sync ? lane_ev : 0u, ibound};
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
@@ -360,11 +360,12 @@ __global__ void __launch_bounds__(256) k_barriers(Geo g, const u32* __restrict__
 }
 
 // ---------------------------------------------------------------------------- k_expand
-// K4: lowering of each LD / ST / ATOM warp record into one thread operation per active lane
-// and per shadow granule (R7), emitted as 8-byte items
-//   key = (dense granule key << 2) | op,   ev = event = (record << 5) | lane
-// at static slots: record r owns [ub_off[r], ub_off[r] + popc(mask) * granules) (upper bound
-// from k_header), lane l the popc(mask & lanemask_lt) * granules slots of it -- so items land in
+// K4: lowering of each LD / ST / ATOM warp record of one window [R0, R1) into one thread operation
+// per active lane and per shadow granule (R7), emitted as 8-byte items
+//   key = (dense granule key << 2) | op,   ev = window-local event = ((record - R0) << 5) | lane
+// at static slots: record r owns popc(mask) * granules slots (upper bound from k_header) starting
+// at its weight prefix within the window (cum[r] - cum[R0] - REC_W * (r - R0)), lane l the
+// popc(mask & lanemask_lt) * granules slots of it -- so items land in
 // trace order with no synchronisation at all.  Dense keys: global granules of written 1-MB
 // pages first (page rank from the write bitmap, so keys follow address order), then shared
 // granules (block, offset).  Accesses to never-written global pages cannot take
@@ -393,19 +394,21 @@ constexpr int EX_RPW = EX_REC / (EX_THREADS / 32);  // records per warp per chun
 __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restrict__ recs, Geo g,
                                                        const u32* __restrict__ page_bits,
                                                        const u32* __restrict__ page_rank, u32 shared_base,
-                                                       const u32* __restrict__ ub_off, u32* __restrict__ okeys,
-                                                       u32* __restrict__ oevs, u32* __restrict__ err) {
+                                                       const u64* __restrict__ cum, u64 R0, u64 R1,
+                                                       u32* __restrict__ okeys, u32* __restrict__ oevs,
+                                                       u32* __restrict__ err) {
   extern __shared__ __align__(128) unsigned char ex_smem[];
   bc_record* buf = reinterpret_cast<bc_record*>(ex_smem);                    // [EX_STAGES][EX_REC]
   u64* bar = reinterpret_cast<u64*>(ex_smem + sizeof(bc_record) * EX_REC * EX_STAGES);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const u64 n = g.n_recs;
+  const u64 n = R1 - R0;  // records of the window
   const u64 n_chunks = (n + EX_REC - 1) / EX_REC;
+  const u64 cum0 = __ldg(cum + R0);
   auto issue = [&](u64 chunk, int st) {
     const u64 r0 = chunk * EX_REC;
     const u32 cnt = (u32)(n - r0 < (u64)EX_REC ? n - r0 : (u64)EX_REC);
     mbar_expect_tx(&bar[st], cnt * (u32)sizeof(bc_record));
-    bulk_g2s(&buf[st * EX_REC], recs + r0, cnt * (u32)sizeof(bc_record), &bar[st]);
+    bulk_g2s(&buf[st * EX_REC], recs + R0 + r0, cnt * (u32)sizeof(bc_record), &bar[st]);
   };
   if (threadIdx.x == 0) {
     for (int s = 0; s < EX_STAGES; ++s) mbar_init(&bar[s], 1);
@@ -423,12 +426,13 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
   for (u64 c = blockIdx.x; c < n_chunks; c += gridDim.x, ++it) {
     const int st = (int)(it % EX_STAGES);
     const u32 phase = (it / EX_STAGES) & 1u;
-    const u64 cbase = c * EX_REC;
+    const u64 cbase = c * EX_REC;  // window-local record index of the chunk
     // warp wid expands records wid, wid + 8, ... of the chunk (interleaved: control and memory records
     // alternate in most programs, so the warps of a CTA finish a chunk at about the same time); their
-    // slot offsets are independent of the staged bytes: one load per lane before waiting
+    // slot offsets (window weight prefix minus REC_W per record) are independent of the staged bytes:
+    // one load per lane before waiting
     const u64 rl = cbase + (u64)wid + (u64)(lane & (EX_RPW - 1)) * (EX_THREADS / 32);
-    const u32 uo_l = (lane < EX_RPW && rl < n) ? __ldg(ub_off + rl) : 0u;
+    const u32 uo_l = (lane < EX_RPW && rl < n) ? (u32)(__ldg(cum + R0 + rl) - cum0 - (u64)REC_W * rl) : 0u;
     mbar_wait(&bar[st], phase);
 #pragma unroll
     for (int j = 0; j < EX_RPW; ++j) {
@@ -468,7 +472,7 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
         }
       }
       const u64 o = (u64)uoj + (u64)__popc(hmask & lt) * nk;
-      const u32 ev = (u32)(r << 5) | (u32)lane;
+      const u32 ev = (u32)(r << 5) | (u32)lane;  // window-local event id
       if (nk == 1 && g.world == 1) {  // one granule, one shard: the common case
         okeys[o] = key0 != KEY_DROP ? ((key0 << 2) | opc) : KEY_DROP;
         oevs[o] = ev;
@@ -488,6 +492,33 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
   }
   if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
   if (__any_sync(0xFFFFFFFFu, ovf) && lane == 0) set_err(err, ERR_OVERFLOW);
+}
+
+// Window k = the records whose weight prefix cum[r] (exclusive) lies in [k * we, (k + 1) * we):
+// starts[k] = lower bound of k * we in cum (n + 1 entries, cum[n] = total), starts[nwin] = n;
+// bounds[k] = the window's item upper bound (its weight minus REC_W per record).
+__global__ void k_window_starts(const u64* __restrict__ cum, u64 n, u64 we, u32 nwin, u64* __restrict__ starts,
+                                u64* __restrict__ bounds) {
+  const u32 k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k > nwin) return;
+  auto lb = [&](u64 v) {
+    u64 lo = 0, hi = n;
+    while (lo < hi) {
+      const u64 m = (lo + hi) >> 1;
+      if (cum[m] < v) lo = m + 1; else hi = m;
+    }
+    return lo;
+  };
+  const u64 s0 = k == 0 ? 0 : (k == nwin ? n : lb((u64)k * we));
+  starts[k] = s0;
+  if (k < nwin) {
+    const u64 s1 = k + 1 == nwin ? n : lb((u64)(k + 1) * we);
+    bounds[k] = (cum[s1] - cum[s0]) - (u64)REC_W * (s1 - s0);
+  }
+}
+void launch_window_starts(const u64* cum, u64 n, u64 we, u32 nwin, u64* starts, u64* bounds, cudaStream_t st) {
+  k_window_starts<<<(nwin + 1 + 255) / 256, 256, 0, st>>>(cum, n, we, nwin, starts, bounds);
+  ++g_launches;
 }
 
 // Ranks of the written 1-MB pages in address order (the dense global key space):
@@ -561,13 +592,13 @@ __global__ void __launch_bounds__(1024) k_page_rank(u32* __restrict__ words, con
 
 // --------------------------------------------------------------------- host launchers
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
-                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_ub, uint4* hdr16,
+                   u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_w, uint4* hdr16,
                    u32* rec_cnt, u32* err, cudaStream_t st) {
   u64 warps = (g.n_recs + 31) / 32;
   if (warps == 0) return;
   u64 blocks = (warps + 7) / 8;
   k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt,
-                                             rec_ub, hdr16, rec_cnt, err); ++g_launches;
+                                             rec_w, hdr16, rec_cnt, err); ++g_launches;
 }
 
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st) {
@@ -676,21 +707,23 @@ void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStrea
 }
 
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
-                   const u32* ub_off, u32* keys, u32* evs, u32* err, cudaStream_t st) {
-  const u64 chunks = (g.n_recs + EX_REC - 1) / EX_REC;
+                   const u64* cum, u64 R0, u64 R1, u32* keys, u32* evs, u32* err, cudaStream_t st) {
+  const u64 chunks = (R1 - R0 + EX_REC - 1) / EX_REC;
   if (!chunks) return;
   const size_t smem = sizeof(bc_record) * EX_REC * EX_STAGES + 8 * EX_STAGES;
-  static int grid = 0;
-  if (!grid) {
-    int dev = 0, sms = 148, per = 1;
-    cudaGetDevice(&dev);
+  static int grid[64] = {};  // per device: the shared-memory opt-in and the occupancy-derived grid
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  if (!grid[dev]) {
+    int sms = 148, per = 1;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_expand, EX_THREADS, smem);
-    grid = sms * (per > 0 ? per : 1);
+    grid[dev] = sms * (per > 0 ? per : 1);
   }
-  const unsigned gr = (unsigned)std::min<u64>(chunks, (u64)grid);
-  k_expand<<<gr, EX_THREADS, smem, st>>>(recs, g, page_bits, page_rank, shared_base, ub_off, keys, evs, err);
+  const unsigned gr = (unsigned)std::min<u64>(chunks, (u64)grid[dev]);
+  k_expand<<<gr, EX_THREADS, smem, st>>>(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, keys, evs, err);
   ++g_launches;
 }
 

@@ -26,13 +26,13 @@ import litmus
 pytestmark = pytest.mark.gpu
 
 
-def _gpu(recs, geom, flags=0):
-    return bc.detect(recs, geom, device="cuda:0", flags=flags)
+def _gpu(recs, geom, flags=0, window_events=0):
+    return bc.detect(recs, geom, device="cuda:0", flags=flags, window_events=window_events)
 
 
-def assert_parity(recs, geom, flags=0, expect_status=None):
+def assert_parity(recs, geom, flags=0, expect_status=None, window_events=0):
     st_o, want, stats_o = oracle.detect_geom(recs, geom, flags)
-    res = _gpu(recs, geom, flags)
+    res = _gpu(recs, geom, flags, window_events)
     assert res.status == st_o, (res.status, st_o)
     if expect_status is not None:
         assert st_o == expect_status
@@ -193,7 +193,11 @@ def test_depth_32():
 
 def test_hot_granule_long_segment():
     """One granule touched by thousands of reads and writes from many warps / blocks: the
-    segment spans many K7 tiles (look-back carries), with inflated read vectors."""
+    segment spans many K7 tiles (range-scan carries), with inflated read vectors."""
+    _hot_granule()
+
+
+def _hot_granule(window_events=0):
     tb = TraceBuilder(grid=(4,), block=(256,))
     hot = GLOBAL_BASE + 0x40
     import random
@@ -209,7 +213,7 @@ def test_hot_granule_long_segment():
                     tb.atom(w, hot)
                 else:
                     tb.st(w, lambda l: hot if l == rng.randrange(32) else GLOBAL_BASE + 0x1000 + 4 * l)
-    want, _ = assert_parity(tb.records(), tb.geom.as_dict())
+    want, _ = assert_parity(tb.records(), tb.geom.as_dict(), window_events=window_events)
     assert len(want) > 100
 
 
@@ -268,20 +272,66 @@ def test_device_borrowed_trace_and_idempotent():
         assert np.array_equal(out.cpu().numpy(), want.view(np.uint8))
 
 
-# ------------------------------------------------------------------ K7 variants
-@pytest.mark.parametrize("variant", ["ballot", "tile"])
-def test_k7_variants(variant, monkeypatch):
-    """Both K7 formulations (lane-sequential with staged clocks = default, ballot rounds =
-    BC_K7=ballot) give the oracle's race set on random traces, a hot granule and reduced C2-C4."""
-    monkeypatch.setenv("BC_K7", variant)
+# ------------------------------------------------------------------ windows (row a5)
+@pytest.mark.parametrize("we", [64, 700, 9000])
+def test_windows(we):
+    """The trace checked in windows of at most `we` weight (bc_config.window_events): every granule's
+    state (last writer, read epoch or read vector, atomic bit: the 32-B shadow entry of Fig. 8,
+    P:L1247-1268) is carried from window to window; the race set must not change.  Tiny windows
+    put window boundaries inside read runs, after inflations, between a writer and its readers."""
     for seed in range(5000, 5040):
         recs, tb = random_trace(seed)
-        assert_parity(recs, tb.geom.as_dict())
-    test_hot_granule_long_segment()
+        _, res = assert_parity(recs, tb.geom.as_dict(), window_events=we)
+        assert res.stats["windows"] >= 1
+    _hot_granule(window_events=we)
     for cfg, kw in [(2, dict(n_blocks=8, iters=6)), (3, dict(n_blocks=9, iters=3, tpb=256)),
                     (4, dict(n_blocks=40, log2_nodes=16, nodes_per_thread=3, inj_scale=8))]:
         plan = ConfigPlan(cfg, **kw)
-        assert_parity(plan.records(), plan.geometry)
+        _, res = assert_parity(plan.records(), plan.geometry, window_events=we * 50)
+        assert res.stats["windows"] > 1
+
+
+def test_windows_litmus_and_vectors():
+    """The 66 litmus traces and random traces with many readers (read vectors carried across windows)
+    in windows of one or two records."""
+    for name, build, _exp, _opts in litmus.SUITE:
+        tb = build()
+        assert_parity(tb.records(), tb.geom.as_dict(), window_events=16)
+    for seed in range(5100, 5130):
+        recs, tb = random_trace(seed, n_glob=2, tpb=128, ops_per_warp=(10, 30))
+        _, res = assert_parity(recs, tb.geom.as_dict(), window_events=40)
+        assert res.stats["windows"] > 5
+
+
+def test_long_read_run_after_write():
+    """One write, then ~20 K reads of one granule by ~20 K threads and few other items (the
+    reads span many K7 warp ranges: the state entering each comes from the range-tail scan, there is
+    no walk cap and no wait on another warp), then a plain write that races with every reader."""
+    tb = TraceBuilder(grid=(80,), block=(256,))
+    flag = GLOBAL_BASE + 0x80
+    tb.st(tb.warp(0, 0), lambda l: flag if l == 0 else GLOBAL_BASE + 0x1000 + 4 * l)
+    for b in range(80):
+        for wib in range(8):
+            tb.ld(tb.warp(b, wib), flag)
+    tb.st(tb.warp(79, 7), lambda l: flag if l == 3 else GLOBAL_BASE + 0x2000 + 4 * l)
+    want, res = assert_parity(tb.records(), tb.geom.as_dict())
+    assert len(want) > 20_000
+    assert_parity(tb.records(), tb.geom.as_dict(), window_events=2000)
+
+
+def test_torch_allocator():
+    """bc_config.dev_alloc / dev_free over torch's caching allocator."""
+    import torch
+    recs, tb = random_trace(77)
+    geom = tb.geom.as_dict()
+    st, want, _ = oracle.detect_geom(recs, geom)
+    before = torch.cuda.memory_allocated()
+    with bc.Context(geom, device=0, allocator="torch") as ctx:
+        ctx.load_trace(recs)
+        assert ctx.detect()[0] == 0
+        assert torch.cuda.memory_allocated() > before
+        assert np.array_equal(ctx.races().view(np.uint8), want.view(np.uint8))
+    assert torch.cuda.memory_allocated() == before
 
 
 # ------------------------------------------------- lock-heavy hashtable (SURVEY row f2)
@@ -357,18 +407,17 @@ def test_values_random_traces():
         assert np.array_equal(ctx.races().view(np.uint8), want_f.view(np.uint8))
 
 
-@pytest.mark.parametrize("variant", ["ballot", "tile"])
-def test_values_k7_variants_byte_granules(variant, monkeypatch):
+@pytest.mark.parametrize("we", [0, 100])
+def test_values_byte_granules(we):
     """Values with byte granules (G = 0, the paper's default) and mixed access
-    sizes, through both K7 formulations."""
+    sizes, in one window and in many."""
     from bcgen.fuzz import random_values
-    monkeypatch.setenv("BC_K7", variant)
     for seed in range(8200, 8240):
         recs, tb = random_trace(seed, same_value=True, n_glob=2, granule_log2=0)
         geom = tb.geom.as_dict()
         vals = random_values(recs, seed)
         st_o, want, _ = oracle.detect_geom(recs, geom, values=vals)
-        res = bc.detect(recs, geom, device="cuda:0", values=vals)
+        res = bc.detect(recs, geom, device="cuda:0", values=vals, window_events=we)
         assert res.status == st_o
         if st_o == 0:
             assert np.array_equal(res.races.view(np.uint8), want.view(np.uint8)), seed
