@@ -119,7 +119,7 @@ class ConfigPlan:
         p = _Params()
         p.config = config
         p.seed = config if seed is None else seed
-        p.inject = kw.pop("inject", 1)
+        p.inject = kw.pop("inject", 1 if config in (4, 5) else 0)  # C2 / C3: injected variants on request
         if config == 6:
             p.bug = kw.pop("bug", 3)  # the benchmark as published has both section-6.3 bugs
         for k, v in kw.items():
@@ -176,7 +176,7 @@ def make_config(name, seed=None, **kw):
         return recs, tb.geom.as_dict(), None
     plan = ConfigPlan(idx, seed, **kw)
     recs = plan.records()
-    truth = plan.truth() if idx in (4, 5) else None
+    truth = plan.truth() if (idx in (4, 5) or kw.get("inject")) else None
     geom = plan.geometry
     plan.close()
     return recs, geom, truth

@@ -8,9 +8,15 @@
 // warps; a warp at BAR waits until every warp of its block has arrived.
 //
 // Programs (per warp):
-//   C2 stencil      1-D 3-point stencil with shared-memory double buffering
+//   C2 stencil      1-D 3-point stencil with shared-memory double buffering; injected variant
+//                   (inject = 1): in `inj_scale` (default 8) seeded blocks, one iteration's barrier
+//                   interval holds an unsynchronised exchange -- warp 0 stores scratch[lane], warp 1
+//                   loads scratch[lane] with no barrier between them (the missing BAR of SURVEY §8(d.2))
 //   C3 tfr          threadFenceReduction: 40 grid-stride loads, shared tree,
-//                   tid0 {st part[b]; AR_GLB count}, last block reduces part[]
+//                   tid0 {st part[b]; AR_GLB count}, last block reduces part[]; injected variant
+//                   (inject = 1): block 0 takes its ticket with a plain atomicInc (no fence: an ATOM,
+//                   no release), so its part[0] store and its ticket are unordered with the last
+//                   block's read of part[0] and its final store count = 0
 //   C4 bfs          BFS-like frontier expansion with divergent neighbour loops,
 //                   atomics on cost/mask, Zipf(0.8) neighbour ids, injected races
 //   C5 scale        C4 shape with 16384 blocks, N = 2^26, 10 nodes/thread and a
@@ -78,6 +84,8 @@ enum Role : uint16_t {
   R2_IN, R2_TILE, R2_HALO_IN, R2_HALO_TILE, R2_OUT,
   // C3
   R3_IN, R3_SD, R3_SD_PLUS, R3_PART, R3_COUNT, R3_AMLAST, R3_PART_READ, R3_RESULT,
+  // injected variants of C2 / C3 (ground truth: bcgen_truth_list)
+  R2_INJ_ST, R2_INJ_LD, R3_INJ_PART, R3_INJ_COUNT, R3_FINAL_COUNT,
   // C4/C5
   R4_FRONTIER, R4_RP, R4_COL, R4_COST, R4_MASK, R4_INJ_INTER, R4_INJ_BR_ST, R4_INJ_BR_LD,
   R4_INJ_ATM,
@@ -166,6 +174,9 @@ struct Gen {
       case R3_AMLAST: return 4ull * tpb;
       case R3_PART_READ: return GB + REGION + 4ull * (t + c.p32 * tpb);
       case R3_RESULT: return GB + 2 * REGION + 64;
+      case R2_INJ_ST: case R2_INJ_LD: return 4ull * (2u * 258u + (uint32_t)lane);
+      case R3_INJ_PART: return GB + REGION + 4ull * b;
+      case R3_INJ_COUNT: case R3_FINAL_COUNT: return GB + 2 * REGION;
       case R4_FRONTIER: return GB + 4ull * ((uint64_t)g + (uint64_t)c.p32 * nthreads);
       case R4_RP: return GB + REGION + 4ull * ((uint64_t)g + (uint64_t)c.p32 * nthreads + c.p16);
       case R4_COL: {
@@ -223,12 +234,18 @@ struct Gen {
       v.push_back(mk(w, tm, ST, SHARED, R2_HALO_TILE, 1));
     });
     uint32_t cur = 0;
+    const uint32_t b = w / wpb;
     for (uint32_t it = 0; it < p.iters; ++it) {
       v.push_back(mk(w, m, BAR));
+      if (inj_kind[w] && it == inj_slot[w]) {  // the unsynchronised exchange of the injected variant
+        if (wib == 0) v.push_back(mk(w, m, ST, SHARED, R2_INJ_ST));
+        if (wib == 1) v.push_back(mk(w, m, LD, SHARED, R2_INJ_LD));
+      }
       for (uint32_t off = 0; off < 3; ++off) v.push_back(mk(w, m, LD, SHARED, R2_TILE, cur, off));
       v.push_back(mk(w, m, ST, SHARED, R2_TILE, cur ^ 1, 1));
       cur ^= 1;
     }
+    (void)b;
     v.push_back(mk(w, m, BAR));
     v.push_back(mk(w, m, ST, GLOBAL, R2_OUT));
   }
@@ -257,9 +274,11 @@ struct Gen {
     v.push_back(mk(w, m, ST, SHARED, R3_SD));
     v.push_back(mk(w, m, BAR));
     tree(v, w, m);
+    const bool inj = inj_kind[w] != 0;
     branch(v, w, m, lanes_below(w, 1), [&](uint32_t tm) {
-      v.push_back(mk(w, tm, ST, GLOBAL, R3_PART));
-      v.push_back(mk(w, tm, AR_GLB, GLOBAL, R3_COUNT));  // __threadfence + atomicInc (amb. 12)
+      v.push_back(mk(w, tm, ST, GLOBAL, inj ? R3_INJ_PART : R3_PART));
+      if (inj) v.push_back(mk(w, tm, ATOM, GLOBAL, R3_INJ_COUNT));  // atomicInc without the fence
+      else v.push_back(mk(w, tm, AR_GLB, GLOBAL, R3_COUNT));        // __threadfence + atomicInc (amb. 12)
       v.push_back(mk(w, tm, ST, SHARED, R3_AMLAST));
     });
     v.push_back(mk(w, m, BAR));
@@ -280,7 +299,7 @@ struct Gen {
       tree(v, w, tm);
       branch(v, w, tm, lanes_below(w, 1), [&](uint32_t t0) {
         v.push_back(mk(w, t0, ST, GLOBAL, R3_RESULT));
-        v.push_back(mk(w, t0, ST, GLOBAL, R3_COUNT));  // plain store count = 0
+        v.push_back(mk(w, t0, ST, GLOBAL, R3_FINAL_COUNT));  // plain store count = 0
       });
     });
   }
@@ -353,7 +372,7 @@ struct Gen {
     if (c == 2) {
       nb = p.n_blocks ? p.n_blocks : 256;
       if (!p.iters) p.iters = 36;
-      smem = 2 * 258 * 4;
+      smem = 2 * 258 * 4 + (p.inject ? 32 * 4 : 0);
     } else if (c == 3) {
       nb = p.n_blocks ? p.n_blocks : 4096;
       if (!p.iters) p.iters = 40;
@@ -379,6 +398,19 @@ struct Gen {
     is_last.assign(nb, 0);
     inj_kind.assign(nw, 0);
     inj_slot.assign(nw, 0);
+    if (c == 2 && p.inject && wpb >= 2) {  // warps 0 and 1 of `scale` seeded blocks, one iteration each
+      const uint32_t scale = std::min<uint32_t>(p.inj_scale ? p.inj_scale : 8, nb);
+      for (uint32_t q = 0; q < scale; ++q) {
+        uint32_t blk = (uint32_t)(splitmix64(p.seed * 7 + q) % nb);
+        while (inj_kind[blk * wpb]) blk = (blk + 1) % nb;
+        const uint32_t it = (uint32_t)(splitmix64(p.seed * 13 + q) % p.iters);
+        for (uint32_t i = 0; i < 2; ++i) {
+          inj_kind[blk * wpb + i] = 1;
+          inj_slot[blk * wpb + i] = it;
+        }
+      }
+    }
+    if (c == 3 && p.inject) inj_kind[0] = 1;  // block 0, warp 0 (its tid 0 takes the ticket)
     if (c == 4 || c == 5) {
       if ((uint64_t)nthreads * K > N) { N = 1u; while ((uint64_t)N < (uint64_t)nthreads * K) N <<= 1; }
       rowptr.resize((size_t)N + 1);
@@ -468,7 +500,7 @@ struct Gen {
             }
             CRec c = prog[w][pc[w]++];
             if (c.op == DYN) { prog_c3_tail(w, prog[w]); --k; continue; }
-            if (c.op == AR_GLB && c.role == R3_COUNT) {
+            if ((c.op == AR_GLB && c.role == R3_COUNT) || c.role == R3_INJ_COUNT) {
               if (ticket == nb - 1) is_last[b] = 1;
               ++ticket;
             }
@@ -558,15 +590,28 @@ void bcgen_fill(void* h, void* dst, uint64_t begin, uint64_t end, int threads) {
 // types, cls from the two warps/blocks, space GLOBAL.
 uint64_t bcgen_truth_list(void* h, bcgen_truth* out, uint64_t cap, uint32_t granule_log2) {
   Gen* g = (Gen*)h;
-  struct Acc { uint64_t gran; uint64_t ev; uint8_t type; uint32_t warp; };
+  struct Acc { uint64_t gran; uint64_t ev; uint8_t type; uint32_t warp; uint8_t space; uint64_t addr; };
   std::vector<Acc> acc;
+  auto injected = [&](const CRec& c) {
+    if (c.op > ATOM) return false;
+    if (c.role >= R4_INJ_INTER && c.role <= R4_INJ_ATM) return true;
+    if (c.role == R2_INJ_ST || c.role == R2_INJ_LD) return true;
+    // C3: block 0's part store and ticket, every read of part[] by the last block, the final count store
+    if (g->p.inject && (c.role == R3_INJ_PART || c.role == R3_INJ_COUNT || c.role == R3_PART_READ ||
+                        c.role == R3_FINAL_COUNT)) return true;
+    return false;
+  };
   for (uint64_t i = 0; i < g->out.size(); ++i) {
     const CRec& c = g->out[i];
-    if (c.role < R4_INJ_INTER || c.role > R4_INJ_ATM || c.op > ATOM) continue;
+    if (!injected(c)) continue;
     for (int l = 0; l < 32; ++l) {
       if (!((c.mask >> l) & 1)) continue;
       uint8_t ty = c.op == LD ? 0 : (c.op == ST ? 1 : 2);
-      acc.push_back({g->addr(c, l) >> granule_log2, (i << 5) | (uint64_t)l, ty, c.warp});
+      const uint64_t a = g->addr(c, l);
+      // a shared location is (block, offset)
+      const uint64_t gran = c.space == SHARED ? (((uint64_t)(c.warp / g->wpb) + 1) << 44) | (a >> granule_log2)
+                                              : a >> granule_log2;
+      acc.push_back({gran, (i << 5) | (uint64_t)l, ty, c.warp, c.space, (a >> granule_log2) << granule_log2});
     }
   }
   std::stable_sort(acc.begin(), acc.end(), [](const Acc& a, const Acc& b) {
@@ -579,17 +624,18 @@ uint64_t bcgen_truth_list(void* h, bcgen_truth* out, uint64_t cap, uint32_t gran
     // kind encoding (format.py): WW WR RW WA AW RA AR
     static const uint8_t kind_tab[3][3] = {{0xFF, 2, 5}, {1, 0, 3}, {6, 4, 0xFF}};
     uint8_t kind = kind_tab[a.type][b.type];
+    if (kind == 0xFF) continue;  // two reads / two atomics: not a conflict
     uint8_t cls;
     if ((a.ev >> 5) == (b.ev >> 5)) cls = 0;
     else if (a.warp == b.warp) cls = 1;
     else if (a.warp / g->wpb == b.warp / g->wpb) cls = 2;
     else cls = 3;
     if (n < cap) {
-      out[n].addr = a.gran << granule_log2;
+      out[n].addr = a.addr;
       out[n].prior_event = a.ev;
       out[n].cur_event = b.ev;
-      out[n].kind = kind; out[n].cls = cls; out[n].space = 0; out[n].pad = 0;
-      out[n].block = b.warp / g->wpb;
+      out[n].kind = kind; out[n].cls = cls; out[n].space = a.space; out[n].pad = 0;
+      out[n].block = a.space == SHARED ? a.warp / g->wpb : b.warp / g->wpb;
     }
     ++n;
   }

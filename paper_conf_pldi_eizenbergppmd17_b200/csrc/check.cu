@@ -674,9 +674,9 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
           const u32 kn = li + 1 < nb ? sK[tpad(li + 1)] : knext;
           if (kn == NONE || (kn >> 2) != (k >> 2)) {
             u32 wr = C.wr, wwl = C.wwl, wf = C.wf;
-            if (lw) {
+            if (lw) {  // (its warp from the snapshot table: a lone writer's snapshot is not gathered)
               wr = R0 + (we >> 5);
-              wwl = (ww << 5) | (we & 31u);
+              wwl = (item_warp(kx, we) << 5) | (we & 31u);
               wf = SH_W_VALID | ((wk & 3u) == IOP_ATOM ? SH_W_ATOM : 0u);
             }
             if (op != IOP_LD) {

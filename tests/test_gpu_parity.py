@@ -450,26 +450,94 @@ def test_warpsim_configs(cfg, kw):
 
 
 # ------------------------------------------------ full-size configs (bench launch configuration)
+def _golden(name):
+    from test_oracle_pins import _golden as g
+    return g(name)
+
+
+def _device_trace(plan, chunk=1 << 20):
+    """The plan's records generated straight into one device buffer, chunk by chunk through a pinned
+    host buffer (C5's 52 GB trace never exists in host memory)."""
+    import torch
+    n = plan.n_records
+    dev = torch.empty(n * 272, dtype=torch.uint8, device="cuda")
+    host = torch.empty(min(n, chunk) * 272, dtype=torch.uint8).pin_memory()
+    for b in range(0, n, chunk):
+        e = min(n, b + chunk)
+        plan.fill(host, b, e)
+        dev[b * 272:e * 272].copy_(host[:(e - b) * 272], non_blocking=False)
+    return dev
+
+
+def _assert_same(got, want):
+    assert len(got) == len(want), (len(got), len(want))
+    assert np.array_equal(got.view(np.uint8), want.view(np.uint8)), _first_diff(got, want)
+
+
 @pytest.mark.slow
-def test_c3_full_size_race_free():
-    """C3 at the bench size (4096 x 256 threads, ~50 M events, 4096 AR_GLB tickets): the
-    threadFenceReduction program is race-free by construction (every shared access is ordered by a
-    barrier, the partial sums by the fence + ticket) -- a property that holds at any
-    size and that the oracle confirms at reduced sizes (test_configs_reduced)."""
+def test_c2_full_size_injected():
+    """C2 at the bench size with its injected variant (8 blocks with an unsynchronised exchange): the
+    GPU list equals the stored oracle list byte for byte (tools/make_golden.py) and the generator's
+    closed form (32 INTRA_BLOCK races per injected block)."""
+    plan = ConfigPlan(2, inject=1)
+    head, want = _golden("c2_inj")
+    assert plan.n_records == int(head["records"])
+    res = _gpu(plan.records(), plan.geometry)
+    assert res.status == 0
+    _assert_same(res.races, want)
+    assert np.array_equal(np.sort(want.view("V32")), np.sort(plan.truth().view("V32")))
+
+
+@pytest.mark.slow
+def test_c3_full_size():
+    """C3 at the bench size (4096 x 256 threads, ~50 M events, 4096 AR_GLB tickets): race-free by
+    construction (every shared access is ordered by a barrier, the partial sums by fence + ticket,
+    P:L314-336; the oracle confirms it up to 256 blocks), and its injected variant (block 0's ticket
+    without the fence) reports exactly the generator's two races; at 256 blocks the injected list
+    equals the stored oracle list."""
     plan = ConfigPlan(3)
     res = _gpu(plan.records(), plan.geometry)
     assert res.status == 0
     assert len(res.races) == 0 and res.stats["lane_events"] > 40_000_000
+    plan = ConfigPlan(3, inject=1)
+    res = _gpu(plan.records(), plan.geometry)
+    truth = plan.truth()
+    assert res.status == 0 and len(truth) == 2
+    assert np.array_equal(np.sort(res.races.view("V32")), np.sort(truth.view("V32")))
+    head, want = _golden("c3_inj")
+    plan = ConfigPlan(3, inject=1, n_blocks=int(head["overrides"].split("n_blocks':")[1].split("}")[0]))
+    res = _gpu(plan.records(), plan.geometry)
+    _assert_same(res.races, want)
 
 
 @pytest.mark.slow
-def test_c4_full_size_injected_truth():
-    """C4 at the bench size (1 M threads, ~220 M lane events): the race set equals the generator's
-    injected set exactly (each injected granule is touched by exactly two unsynchronised
-    conflicting accesses and nothing else races, as the oracle confirms at reduced sizes)."""
+@pytest.mark.parametrize("we", [0, 1 << 27])
+def test_c4_full_size_golden(we):
+    """C4 at the bench size (1 M threads, 218 M lane events, 38 M records), one window and ~4 windows:
+    the race list equals the oracle's full-size list byte for byte (tests/golden/c4_oracle_races.txt,
+    800 s of oracle time, written by tools/make_golden.py)."""
     plan = ConfigPlan(4)
-    res = _gpu(plan.records(), plan.geometry)
+    head, want = _golden("c4")
+    assert plan.n_records == int(head["records"])
+    res = bc.detect(_device_trace(plan), plan.geometry, device="cuda:0", window_events=we)
     assert res.status == 0
+    assert res.stats["windows"] == (1 if we == 0 else 4)
+    _assert_same(res.races, want)
+
+
+@pytest.mark.slow
+def test_c5_full_size_truth():
+    """C5 at full size (16384 x 256 = 4 M threads, 193 M records, 1.09 G lane events, a 52 GB trace) on
+    one B200: more than 2^27 records, so the check runs in windows with the shadow state carried
+    between them; the race set equals the generator's injected set (4x C4's counts).  (The oracle
+    cannot run this size: SURVEY §8(d.4).)"""
+    import torch
+    plan = ConfigPlan(5)
+    assert plan.n_records > (1 << 27)
     truth = plan.truth()
+    res = bc.detect(_device_trace(plan), plan.geometry, device="cuda:0")
+    assert res.status == 0
+    assert res.stats["windows"] > 1 and res.stats["lane_events"] > 1_000_000_000
     assert len(truth) > 0
     assert np.array_equal(np.sort(res.races.view("V32")), np.sort(truth.view("V32")))
+    torch.cuda.empty_cache()

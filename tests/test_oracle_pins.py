@@ -237,6 +237,78 @@ def test_c4_reduced_exactly_injected():
     assert np.array_equal(np.sort(races.view("V32")), np.sort(truth.view("V32")))
 
 
+@pytest.mark.parametrize("kw", [dict(n_blocks=8, iters=6, inj_scale=3), dict(n_blocks=5, iters=4, tpb=96, inj_scale=2)])
+def test_c2_injected_exactly_truth(kw):
+    """C2's injected variant (a missing barrier): warp 0 stores scratch[lane] and warp 1
+    loads it in one barrier interval of a seeded iteration -> exactly one WR / RW INTRA_BLOCK race per
+    lane in each injected block, and nothing else races; brute force (§3.2) confirms the smallest."""
+    plan = ConfigPlan(2, inject=1, **kw)
+    recs = plan.records()
+    races = run(recs, plan.geometry)
+    truth = plan.truth()
+    assert len(truth) == 32 * kw["inj_scale"]
+    assert set(truth["cls"]) == {2} and set(truth["space"]) == {1}
+    assert np.array_equal(np.sort(races.view("V32")), np.sort(truth.view("V32")))
+
+
+def test_c2_injected_vs_bruteforce():
+    plan = ConfigPlan(2, inject=1, n_blocks=2, iters=2, tpb=64, inj_scale=1)
+    recs = plan.records()
+    races = run(recs, plan.geometry)
+    assert len(races) == 32
+    check_against_bf(recs, plan.geometry, races)
+
+
+@pytest.mark.parametrize("kw", [dict(n_blocks=16, iters=2, tpb=64), dict(n_blocks=24, iters=1, tpb=128)])
+def test_c3_injected_exactly_truth(kw):
+    """C3's injected variant: block 0 takes its ticket with a plain atomicInc (no fence, so no release,
+    P:L314-336): the last block's read of part[0] races with block 0's store (WR INTER_BLOCK) and its
+    final count = 0 with block 0's atomic (AW INTER_BLOCK) -- exactly these two."""
+    plan = ConfigPlan(3, inject=1, **kw)
+    recs = plan.records()
+    races = run(recs, plan.geometry)
+    truth = plan.truth()
+    assert sorted(truth["kind"].tolist()) == [1, 4] and set(truth["cls"]) == {3}
+    assert np.array_equal(np.sort(races.view("V32")), np.sort(truth.view("V32")))
+
+
+def test_c3_injected_vs_bruteforce():
+    plan = ConfigPlan(3, inject=1, n_blocks=3, iters=1, tpb=32)
+    recs = plan.records()
+    races = run(recs, plan.geometry)
+    assert len(races) == 2
+    check_against_bf(recs, plan.geometry, races)
+
+
+def _golden(name):
+    """tests/golden/<name>_oracle_races.txt (tools/make_golden.py: written by the oracle alone)"""
+    path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", f"{name}_oracle_races.txt")
+    head, rows = {}, []
+    for line in open(path):
+        if line.startswith("#"):
+            for tok in line[1:].split():
+                if "=" in tok:
+                    k, v = tok.split("=", 1)
+                    head[k] = v
+            continue
+        a, p, c, kind, cls, space, blk = line.split()
+        rows.append((int(a, 16), int(p, 16), int(c, 16), int(kind), int(cls), int(space), 0, int(blk)))
+    return head, np.array(rows, dtype=bcgen.RACE_DTYPE)
+
+
+def test_golden_c4_is_the_injected_set():
+    """The stored full-size C4 oracle list (13 min of oracle time) is exactly the generator's
+    injected set, and covers the three injected kinds (WW INTER_BLOCK, WR BRANCH, AR INTER_BLOCK)."""
+    head, races = _golden("c4")
+    assert int(head["races"]) == len(races) == 2304
+    kinds = {(int(k), int(c)) for k, c in zip(races["kind"], races["cls"])}
+    assert kinds == {(0, 3), (1, 1), (6, 3)}
+    plan = ConfigPlan(4)
+    assert plan.n_records == int(head["records"])
+    truth = plan.truth()
+    assert np.array_equal(np.sort(races.view("V32")), np.sort(truth.view("V32")))
+
+
 # ---------------------------------------------------------------- infeasible
 def _infeasible_traces():
     X = GLOBAL_BASE
