@@ -5,6 +5,7 @@
 //               -> K7 shadow check (a7) -> K8 finalize (a8/a9)
 // all on cfg.stream; every phase is bracketed by cudaEvents for bc_stats.ms_kernel.
 #include <algorithm>
+#include <atomic>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -15,7 +16,7 @@
 using namespace bc;
 
 namespace bc {
-u64 g_launches = 0;
+std::atomic<u64> g_launches{0};  // kernels launched by this process (per-detect delta in bc_stats)
 }
 
 struct bc_ctx {

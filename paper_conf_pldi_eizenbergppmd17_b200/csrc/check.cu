@@ -480,10 +480,84 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
 
   u32 segs = 0;
   const u32 l0 = lane * KT_IPL;
-  if (beg < end) kt_stage(a, beg, (u32)(end - beg < (u64)KT_BLK ? end - beg : (u64)KT_BLK), sK, sE, lane);
+  // fast path (one window, nothing carried in or out): a block none of whose items makes a check --
+  // every item alone in its granule, or an atomic between atomics (its W check is elided, P:L661-670,
+  // and no read follows it) -- only advances the automaton state: summarised from its key words
+  const bool fast_ok = !shadow && a.sh_out == nullptr;
   for (u64 bb = beg; bb < end; bb += KT_BLK) {
     const u32 nb = (u32)(end - bb < (u64)KT_BLK ? end - bb : (u64)KT_BLK);
     const u32 knext = bb + nb < n ? __ldg(a.keys + bb + nb) : NONE;  // first item after the block
+    if (fast_ok) {
+      u32 kr[KT_IPL];
+      const u32 cntf = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
+      if (cntf == (u32)KT_IPL) {
+        const uint4* kv = reinterpret_cast<const uint4*>(a.keys + bb + l0);  // 64-B aligned: bb, l0 are x16
+#pragma unroll
+        for (int q = 0; q < KT_IPL / 4; ++q) {
+          const uint4 v = __ldg(kv + q);
+          kr[4 * q] = v.x;
+          kr[4 * q + 1] = v.y;
+          kr[4 * q + 2] = v.z;
+          kr[4 * q + 3] = v.w;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < KT_IPL; ++j) kr[j] = (u32)j < cntf ? __ldg(a.keys + bb + l0 + j) : NONE;
+      }
+      u32 kp = __shfl_up_sync(0xFFFFFFFFu, kr[KT_IPL - 1], 1);
+      u32 knx = __shfl_down_sync(0xFFFFFFFFu, kr[0], 1);
+      if (lane == 0) kp = pkx;
+      if (lane == 31 || l0 + KT_IPL >= nb) knx = knext;
+      bool triv = true;
+      u32 fsegs = 0, tlw = 0, kl = kp;
+      bool kc = false;
+#pragma unroll
+      for (int j = 0; j < KT_IPL; ++j) {
+        if ((u32)j < cntf) {
+          const u32 k = kr[j], kpv = kl, knv = (u32)j + 1 < cntf ? kr[j + 1] : knx;
+          const u32 key = k >> 2;
+          const bool sp = kpv != NONE && (kpv >> 2) == key, sn = knv != NONE && (knv >> 2) == key;
+          const bool atm_only =
+              (k & 3u) == IOP_ATOM && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
+          triv &= (!sp && !sn) || atm_only;
+          if (!sp) {
+            ++fsegs;
+            kc |= j > 0;
+            tlw = 0;
+          }
+          if ((k & 3u) != IOP_LD) tlw = (u32)bb + l0 + (u32)j + 1u;
+          kl = k;
+        }
+      }
+      if (__all_sync(0xFFFFFFFFu, triv)) {
+        segs += fsegs;
+        // chunk summaries (no read has a same-granule read before it: no READINFLATE flags) and their
+        // warp combine = the block summary
+        Sum sm = sum_ident();
+        if (cntf) {
+          sm.fk = kr[0] >> 2;
+          sm.lk = kl >> 2;
+          sm.lw = tlw;
+          sm.fi = NONE;
+          sm.bits = (kc ? 0u : SB_ONE) | (tlw ? SB_W : 0u);
+        }
+        Sum incl = sm;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const Sum up = shfl_up_sum(incl, o);
+          if ((int)lane >= o) incl = combine(up, incl);
+        }
+        carry = combine(carry, shfl_sum(incl, 31));
+        if (carry.lw && (u64)(carry.lw - 1) >= bb) {
+          cwk = __ldg(a.keys + carry.lw - 1);
+          cwe = __ldg(a.evs + carry.lw - 1);
+        }
+        pkx = __ldg(a.keys + bb + nb - 1);
+        pev = __ldg(a.evs + bb + nb - 1);
+        continue;
+      }
+    }
+    kt_stage(a, bb, nb, sK, sE, lane);
     cp_async_wait0();
     __syncwarp();
 
@@ -705,10 +779,6 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
     pkx = sK[tpad(nb - 1)];
     pev = sE[tpad(nb - 1)];
     __syncwarp();
-    if (bb + nb < end) {  // stage the next block once this one is done
-      const u64 b2 = bb + nb;
-      kt_stage(a, b2, (u32)(end - b2 < (u64)KT_BLK ? end - b2 : (u64)KT_BLK), sK, sE, lane);
-    }
   }
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);
   if (lane == 0 && segs) atomicAdd((unsigned long long*)kx->seg_cnt, (unsigned long long)segs);

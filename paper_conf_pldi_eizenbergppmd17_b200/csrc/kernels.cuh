@@ -2,6 +2,7 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <new>
 #include <vector>
 
@@ -10,7 +11,7 @@
 namespace bc {
 
 // kernels launched by this process (bc_stats.kernel_launches is the delta over one bc_detect)
-extern u64 g_launches;
+extern std::atomic<u64> g_launches;
 
 // counters written by the kernels (u64 device array)
 // (one u64 array, so that each host synchronisation reads every counter with ONE pinned copy; the u32

@@ -314,10 +314,10 @@ void sort_perm_by(u32* perm, const u32* f, u32 n, int bits, Scratch& S, cudaStre
 }
 
 void launch_iota(u32* p, u32 n, cudaStream_t st) {
-  if (n) k_iota<<<nb(n), 256, 0, st>>>(p, n); ++g_launches;
+  if (n) { k_iota<<<nb(n), 256, 0, st>>>(p, n); ++g_launches; }
 }
 void launch_gather_u32(const u32* src, const u32* perm, u32 n, u32* dst, cudaStream_t st) {
-  if (n) k_gather_u32<<<nb(n), 256, 0, st>>>(src, perm, n, dst); ++g_launches;
+  if (n) { k_gather_u32<<<nb(n), 256, 0, st>>>(src, perm, n, dst); ++g_launches; }
 }
 
 static int bits_for(u64 maxval) {
@@ -429,7 +429,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   // arrF ids are nx + nB + acquire index; expose them for K7
   {
     u32* acq_arr = S.alloc<u32>(n_acq + 1);
-    if (n_acq) k_iota_add<<<nb(n_acq), 256, 0, st>>>(acq_arr, n_acq, nx + nB); ++g_launches;
+    if (n_acq) { k_iota_add<<<nb(n_acq), 256, 0, st>>>(acq_arr, n_acq, nx + nB); ++g_launches; }
     hc.acq_arr = acq_arr;
   }
   // 5. entries
@@ -473,7 +473,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   u32* ipos = S.alloc<u32>(ne + 1);
   u32* imask = S.alloc<u32>(ne + 1);
   u32* iclk = S.alloc<u32>(ne + 1);
-  if (ne) k_make_ak<<<nb(ne), 256, 0, st>>>(eo.arr, eo.key, eo.pos, eo.mask, eo.clk, ep, ne, ak, ipos, imask, iclk); ++g_launches;
+  if (ne) { k_make_ak<<<nb(ne), 256, 0, st>>>(eo.arr, eo.key, eo.pos, eo.mask, eo.clk, ep, ne, ak, ipos, imask, iclk); ++g_launches; }
   hc.n_idx = ne;
   hc.idx_ak = ak;
   hc.idx_pos = ipos;

@@ -287,7 +287,7 @@ def test_windows(we):
     for cfg, kw in [(2, dict(n_blocks=8, iters=6)), (3, dict(n_blocks=9, iters=3, tpb=256)),
                     (4, dict(n_blocks=40, log2_nodes=16, nodes_per_thread=3, inj_scale=8))]:
         plan = ConfigPlan(cfg, **kw)
-        _, res = assert_parity(plan.records(), plan.geometry, window_events=we * 50)
+        _, res = assert_parity(plan.records(), plan.geometry, window_events={64: 3000, 700: 12000}.get(we, 30000))
         assert res.stats["windows"] > 1
 
 
