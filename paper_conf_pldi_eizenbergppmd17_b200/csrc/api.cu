@@ -334,8 +334,11 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   // ---- K3: sync skeleton
   if (hc_cnt[C_SYNC_RECS]) {
     u64 ne = 0;
-    int rs = run_sync_skeleton(recs, sync_list, (u32)hc_cnt[C_SYNC_RECS], (u32)hc_cnt[C_SYNC_LANEOPS],
-                               (u32)hc_cnt[C_ACQ_RECS], hc, S, st, &ne);
+    const u32 n_srec = (u32)hc_cnt[C_SYNC_RECS];
+    bc_record* srecs = S.alloc<bc_record>(n_srec);
+    gather_sync_records(recs, sync_list, n_srec, n, srecs, S, st);
+    int rs = run_sync_skeleton(srecs, sync_list, n_srec, (u32)hc_cnt[C_SYNC_LANEOPS], (u32)hc_cnt[C_ACQ_RECS], hc, S, st,
+                               &ne);
     if (rs) return fail(c, (bc_status)rs, "sync skeleton");
   }
   cudaEventRecord(c->ev[4], st);

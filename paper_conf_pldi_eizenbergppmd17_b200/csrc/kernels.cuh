@@ -130,8 +130,10 @@ void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStrea
 void sort_perm_by(u32* perm, const u32* f, u32 n, int bits, Scratch& S, cudaStream_t st);
 void launch_iota(u32* p, u32 n, cudaStream_t st);
 void launch_gather_u32(const u32* src, const u32* perm, u32 n, u32* dst, cudaStream_t st);
-int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_lo, u32 n_acq, HbCtx& hc, Scratch& S,
-                      cudaStream_t st, u64* n_entries_out);
+int run_sync_skeleton(const bc_record* srecs, const u32* sgidx, u32 n_srec, u32 n_lo, u32 n_acq, HbCtx& hc,
+                      Scratch& S, cudaStream_t st, u64* n_entries_out);
+void gather_sync_records(const bc_record* recs, u32* sync_list, u32 n, u64 n_recs, bc_record* srecs, Scratch& S,
+                         cudaStream_t st);
 
 // check.cu
 size_t check_status_bytes(u64 n);

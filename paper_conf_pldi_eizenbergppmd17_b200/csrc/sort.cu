@@ -643,16 +643,19 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
   u32* ghist = (u32*)temp;                           // [RS_MAXP][RS_MAXB]
   u32* gbase = ghist + RS_MAXP * RS_MAXB;            // [RS_MAXP][RS_MAXB]
   u32* counts = (u32*)((char*)temp + RS_HDR_BYTES);  // [BINS][tiles]
-  static int sms = 0, down_grid = 0;
+  static int grid_of[64] = {};  // per device: shared-memory opt-in + occupancy-derived persistent grid
   constexpr size_t dsmem = rs_dsmem<RB>();
-  if (!down_grid) {
-    int dev = 0, per = 1;
-    cudaGetDevice(&dev);
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  if (!grid_of[dev]) {
+    int sms = 148, per = 1;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaFuncSetAttribute(k_rs_down<RB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_rs_down<RB>, RS_THREADS, dsmem);
-    down_grid = sms * (per > 0 ? per : 1);
+    grid_of[dev] = sms * (per > 0 ? per : 1);
   }
+  const int down_grid = grid_of[dev];
   const u64* nd = n_dev;
   for (int p = 0; p < passes; ++p) {
     const int shift = bit_lo + RB * p;
@@ -693,10 +696,13 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   }
   const int bits = std::max(bit_hi - bit_lo, 1);
   if (n <= RS_SMALL) {
-    static bool attr = false;
-    if (!attr) {
+    static bool attr[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (!attr[dev]) {
       cudaFuncSetAttribute(k_sort_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SS_SMEM);
-      attr = true;
+      attr[dev] = true;
     }
     k_sort_small<<<1, SS_THREADS, SS_SMEM, st>>>(keys, vals, keys_alt, vals_alt, n, n_dev, drop ? 1 : 0, bit_lo,
                                                  bits, drop ? n_out_dev : nullptr);

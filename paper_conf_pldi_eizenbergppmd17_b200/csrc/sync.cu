@@ -34,21 +34,20 @@ __device__ __forceinline__ bool is_glb_op(u32 op) {
   return op == BC_OP_ACQ_GLB || op == BC_OP_REL_GLB || op == BC_OP_AR_GLB;
 }
 
-__global__ void k_popc_recs(const bc_record* __restrict__ recs, const u32* __restrict__ srec, u32 n,
-                            u32* __restrict__ out) {
+__global__ void k_popc_recs(const bc_record* __restrict__ srecs, u32 n, u32* __restrict__ out) {
   u32 i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < n) out[i] = __popc(__ldg(&recs[srec[i]].mask));
+  if (i < n) out[i] = __popc(__ldg(&srecs[i].mask));
 }
 
-// lane-ops: rec, lane, 64-bit location key (split), index
-__global__ void k_laneops(const bc_record* __restrict__ recs, const u32* __restrict__ srec, u32 n,
+// lane-ops: global record, lane, sync position, 64-bit location key (split), index
+__global__ void k_laneops(const bc_record* __restrict__ srecs, const u32* __restrict__ sgidx, u32 n,
                           const u32* __restrict__ off, Geo g, u32* __restrict__ lo_rec, u32* __restrict__ lo_lane,
-                          u32* __restrict__ xk_lo, u32* __restrict__ xk_hi, u32* __restrict__ lo_idx,
-                          u32* __restrict__ err) {
+                          u32* __restrict__ lo_sp, u32* __restrict__ xk_lo, u32* __restrict__ xk_hi,
+                          u32* __restrict__ lo_idx, u32* __restrict__ err) {
   u32 i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  u32 r = srec[i];
-  const bc_record& rc = recs[r];
+  u32 r = sgidx[i];
+  const bc_record& rc = srecs[i];
   u32 m = rc.mask, o = off[i];
   u32 w = rc.warp;
   while (m) {
@@ -64,6 +63,7 @@ __global__ void k_laneops(const bc_record* __restrict__ recs, const u32* __restr
     }
     lo_rec[o] = r;
     lo_lane[o] = (u32)l;
+    lo_sp[o] = i;
     xk_lo[o] = (u32)xk;
     xk_hi[o] = (u32)(xk >> 32);
     lo_idx[o] = o;
@@ -94,16 +94,16 @@ __global__ void k_assign_ids(const u32* __restrict__ perm, const u32* __restrict
 }
 
 // candidate (xid, block) pairs of block-scope releases
-__global__ void k_bpairs(const bc_record* __restrict__ recs, const u32* __restrict__ lo_rec, const u32* __restrict__ xid,
+__global__ void k_bpairs(const bc_record* __restrict__ srecs, const u32* __restrict__ lo_sp, const u32* __restrict__ xid,
                          u32 n, Geo g, u32* __restrict__ pk_hi, u32* __restrict__ pk_lo, u32* __restrict__ cnt) {
   u32 i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  u32 r = lo_rec[i];
-  u32 op = recs[r].op;
+  const bc_record& rc = srecs[lo_sp[i]];
+  u32 op = rc.op;
   if (op == BC_OP_REL_BLK || op == BC_OP_AR_BLK) {
     u32 at = atomicAdd(cnt, 1u);
     pk_hi[at] = xid[i];
-    pk_lo[at] = recs[r].warp / g.wpb;
+    pk_lo[at] = rc.warp / g.wpb;
   }
 }
 
@@ -120,9 +120,9 @@ __global__ void k_compact_pairs(const u32* __restrict__ hi, const u32* __restric
 
 struct K3In {
   HbCtx hc;
-  const bc_record* recs;
+  const bc_record* srecs;  // sync records, trace order
   u32 n_lo;
-  const u32 *lo_rec, *lo_lane, *xid;
+  const u32 *lo_rec, *lo_lane, *lo_sp, *xid;
   u32 nx, nB;
   const u32 *bp_x, *bp_b;  // unique sorted (xid, block) pairs, bid = index
   const u32* acq_idx_of_rec_sorted;  // unused
@@ -170,8 +170,8 @@ __device__ __forceinline__ void put(const EntOut* o, u32& n, u32 arr, u32 key, u
 __device__ u32 laneop_entries(const K3In& k, u32 i, const EntOut* o, u32 base) {
   const HbCtx& c = k.hc;
   u32 r = k.lo_rec[i], lane = k.lo_lane[i];
-  u32 op = k.recs[r].op;
-  u32 w = k.recs[r].warp;
+  u32 op = k.srecs[k.lo_sp[i]].op;
+  u32 w = k.srecs[k.lo_sp[i]].warp;
   u32 b = w / c.g.wpb;
   u32 x = k.xid[i];
   // position of this lane-op = its rank among the sync lane-ops in trace order (record, then lane):
@@ -234,32 +234,32 @@ __global__ void k_ent_fill(K3In k, const u32* __restrict__ off, EntOut o) {
   if (i < k.n_lo) laneop_entries(k, i, &o, off[i]);
 }
 
-// acquire list: sync records (sorted by rec) that acquire -> keys = block, vals = rec
-__global__ void k_acq_collect(const bc_record* __restrict__ recs, const u32* __restrict__ srec, u32 n, Geo g,
-                              u32* __restrict__ akey, u32* __restrict__ aval, u32* __restrict__ cnt) {
+// acquire list: sync records (trace order) that acquire -> keys = block, vals = sync position
+__global__ void k_acq_collect(const bc_record* __restrict__ srecs, u32 n, Geo g, u32* __restrict__ akey,
+                              u32* __restrict__ aval, const u32* __restrict__ cnt) {
   u32 i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  u32 r = srec[i];
-  u32 op = recs[r].op;
-  // keep trace order: the slot is the rank among acquires, computed by a flag scan on the host side
+  u32 op = srecs[i].op;
+  // keep trace order: the slot is the rank among acquires (exclusive scan of the flags)
   if (is_acq_op(op)) {
     u32 at = cnt[i];
-    akey[at] = recs[r].warp / g.wpb;
-    aval[at] = r;
+    akey[at] = srecs[i].warp / g.wpb;
+    aval[at] = i;
   }
 }
-__global__ void k_acq_flags(const bc_record* __restrict__ recs, const u32* __restrict__ srec, u32 n,
-                            u32* __restrict__ flag) {
+__global__ void k_acq_flags(const bc_record* __restrict__ srecs, u32 n, u32* __restrict__ flag) {
   u32 i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < n) flag[i] = is_acq_op(recs[srec[i]].op) ? 1u : 0u;
+  if (i < n) flag[i] = is_acq_op(srecs[i].op) ? 1u : 0u;
 }
-__global__ void k_acq_info(const bc_record* __restrict__ recs, const u32* __restrict__ arec, u32 n,
-                           u32* __restrict__ awarp, u32* __restrict__ alane) {
+// acquire i (sorted by (block, record)): sync position -> global record, warp, a lane active in it
+__global__ void k_acq_info(const bc_record* __restrict__ srecs, const u32* __restrict__ sgidx, u32* __restrict__ arec,
+                           u32 n, u32* __restrict__ awarp, u32* __restrict__ alane) {
   u32 i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  u32 r = arec[i];
-  awarp[i] = recs[r].warp;
-  alane[i] = __ffs(recs[r].mask) - 1;
+  const u32 sp = arec[i];
+  awarp[i] = srecs[sp].warp;
+  alane[i] = __ffs(srecs[sp].mask) - 1;
+  arec[i] = sgidx[sp];
 }
 __global__ void k_block_start(const u32* __restrict__ sorted_blocks, u32 n, u32 n_blocks, u32* __restrict__ start) {
   u32 b = blockIdx.x * blockDim.x + threadIdx.x;
@@ -299,7 +299,31 @@ __global__ void k_make_ak(const u32* __restrict__ arr, const u32* __restrict__ k
 
 inline unsigned nb(u64 n) { return (unsigned)((n + 255) / 256); }
 
+// compact copy of the sync records: dst[i] = recs[idx[i]] (one warp per record, 272 B)
+__global__ void k_gather_records(const bc_record* __restrict__ recs, const u32* __restrict__ idx, u32 n,
+                                 bc_record* __restrict__ dst) {
+  const u32 i = (u32)(((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5), l = threadIdx.x & 31;
+  if (i >= n) return;
+  const u32* src = reinterpret_cast<const u32*>(recs + idx[i]);
+  u32* d = reinterpret_cast<u32*>(dst + i);
+  for (u32 q = l; q < sizeof(bc_record) / 4; q += 32) d[q] = src[q];
+}
+
 }  // namespace
+
+// sync_list[0, n) (record indices, any order) -> sorted in place, srecs[i] = recs[sync_list[i]]
+void gather_sync_records(const bc_record* recs, u32* sync_list, u32 n, u64 n_recs, bc_record* srecs, Scratch& S,
+                         cudaStream_t st) {
+  if (n == 0) return;
+  u32* k2 = S.alloc<u32>(n);
+  void* tmp = S.alloc<char>(rs_temp_bytes(n));
+  int b = 0;
+  while (b < 32 && (n_recs >> b)) ++b;
+  const bool alt = radix_sort_pairs(sync_list, nullptr, k2, nullptr, n, 0, b, tmp, st);
+  if (alt) cudaMemcpyAsync(sync_list, k2, (size_t)n * sizeof(u32), cudaMemcpyDeviceToDevice, st);
+  k_gather_records<<<(unsigned)(((u64)n * 32 + 255) / 256), 256, 0, st>>>(recs, sync_list, n, srecs);
+  ++g_launches;
+}
 
 // Sort a permutation `perm` (initially any order) stably by the 32-bit field `f` (bits [0, bits)).
 void sort_perm_by(u32* perm, const u32* f, u32 n, int bits, Scratch& S, cudaStream_t st) {
@@ -326,27 +350,19 @@ static int bits_for(u64 maxval) {
   return b;
 }
 
-// Runs K3.  Fills the foreign-knowledge fields of `hc` (acq_*, idx_*).  Returns 0 or a bc_status.
-int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_lo, u32 n_acq, HbCtx& hc,
+// Runs K3 over the sync records srecs[0, n_srec) (ACQ / REL / AR records, 272 B each, in trace order)
+// whose global record indices are sgidx[] (increasing).  Fills the foreign-knowledge fields of `hc`
+// (acq_*, idx_*).  Returns 0 or a bc_status.
+int run_sync_skeleton(const bc_record* srecs, const u32* sgidx, u32 n_srec, u32 n_lo, u32 n_acq, HbCtx& hc,
                       Scratch& S, cudaStream_t st, u64* n_entries_out) {
   const Geo& g = hc.g;
   *n_entries_out = 0;
   if (n_srec == 0) return 0;
-  // 1. sync records in trace order
-  {
-    u32* k2 = S.alloc<u32>(n_srec);
-    u32* v = S.alloc<u32>(n_srec);
-    u32* v2 = S.alloc<u32>(n_srec);
-    void* tmp = S.alloc<char>(rs_temp_bytes(n_srec));
-    launch_iota(v, n_srec, st);
-    bool alt = radix_sort_pairs(sync_list, v, k2, v2, n_srec, 0, bits_for(g.n_recs), tmp, st);
-    if (alt) cudaMemcpyAsync(sync_list, k2, n_srec * sizeof(u32), cudaMemcpyDeviceToDevice, st);
-  }
   // 2. acquire list sorted by (block, rec)
   u32* aflag = S.alloc<u32>(n_srec);
   u32* aex = S.alloc<u32>(n_srec);
   u64* tot = S.alloc<u64>(1);
-  k_acq_flags<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, aflag); ++g_launches;
+  k_acq_flags<<<nb(n_srec), 256, 0, st>>>(srecs, n_srec, aflag); ++g_launches;
   // (n_acq = the header's count of acquire records: no host round trip for it)
   exclusive_scan_u32(aflag, aex, n_srec, S.alloc<char>(scan_temp_bytes(n_srec)), tot, st);
   u32* acq_blk = S.alloc<u32>(n_acq + 1);
@@ -355,7 +371,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   u32* acq_lane = S.alloc<u32>(n_acq + 1);
   u32* acq_bstart = S.alloc<u32>(g.n_blocks + 1);
   if (n_acq) {
-    k_acq_collect<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, g, acq_blk, acq_rec, aex); ++g_launches;
+    k_acq_collect<<<nb(n_srec), 256, 0, st>>>(srecs, n_srec, g, acq_blk, acq_rec, aex); ++g_launches;
     u32* k2 = S.alloc<u32>(n_acq);
     u32* v2 = S.alloc<u32>(n_acq);
     void* tmp = S.alloc<char>(rs_temp_bytes(n_acq));
@@ -364,7 +380,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
       cudaMemcpyAsync(acq_blk, k2, n_acq * 4, cudaMemcpyDeviceToDevice, st);
       cudaMemcpyAsync(acq_rec, v2, n_acq * 4, cudaMemcpyDeviceToDevice, st);
     }
-    k_acq_info<<<nb(n_acq), 256, 0, st>>>(recs, acq_rec, n_acq, acq_warp, acq_lane); ++g_launches;
+    k_acq_info<<<nb(n_acq), 256, 0, st>>>(srecs, sgidx, acq_rec, n_acq, acq_warp, acq_lane); ++g_launches;
   }
   k_block_start<<<nb(g.n_blocks + 1), 256, 0, st>>>(acq_blk, n_acq, g.n_blocks, acq_bstart); ++g_launches;
   hc.n_acq = n_acq;
@@ -376,14 +392,17 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   // 3. lane-ops and dense sync-location ids
   u32* cnt = S.alloc<u32>(n_srec);
   u32* off = S.alloc<u32>(n_srec);
-  k_popc_recs<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, cnt); ++g_launches;
+  k_popc_recs<<<nb(n_srec), 256, 0, st>>>(srecs, n_srec, cnt); ++g_launches;
   exclusive_scan_u32(cnt, off, n_srec, S.alloc<char>(scan_temp_bytes(n_srec)), nullptr, st);
   u32* lo_rec = S.alloc<u32>(n_lo);
   u32* lo_lane = S.alloc<u32>(n_lo);
+  u32* lo_sp = S.alloc<u32>(n_lo);
   u32* xk_lo = S.alloc<u32>(n_lo);
   u32* xk_hi = S.alloc<u32>(n_lo);
   u32* perm = S.alloc<u32>(n_lo);
-  k_laneops<<<nb(n_srec), 256, 0, st>>>(recs, sync_list, n_srec, off, g, lo_rec, lo_lane, xk_lo, xk_hi, perm, hc.err); ++g_launches;
+  k_laneops<<<nb(n_srec), 256, 0, st>>>(srecs, sgidx, n_srec, off, g, lo_rec, lo_lane, lo_sp, xk_lo, xk_hi, perm,
+                                        hc.err);
+  ++g_launches;
   sort_perm_by(perm, xk_lo, n_lo, 32, S, st);
   sort_perm_by(perm, xk_hi, n_lo, 32, S, st);
   u32* flag = S.alloc<u32>(n_lo);
@@ -399,7 +418,7 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   u32* pk_lo = S.alloc<u32>(n_lo);
   u32* pcnt = S.alloc<u32>(1);
   cudaMemsetAsync(pcnt, 0, 4, st);
-  k_bpairs<<<nb(n_lo), 256, 0, st>>>(recs, lo_rec, xid, n_lo, g, pk_hi, pk_lo, pcnt); ++g_launches;
+  k_bpairs<<<nb(n_lo), 256, 0, st>>>(srecs, lo_sp, xid, n_lo, g, pk_hi, pk_lo, pcnt); ++g_launches;
   u32 np = 0;
   cudaMemcpyAsync(&np, pcnt, 4, cudaMemcpyDeviceToHost, st);
   if (cudaStreamSynchronize(st) != cudaSuccess) return BC_ERR_CUDA;
@@ -435,7 +454,8 @@ int run_sync_skeleton(const bc_record* recs, u32* sync_list, u32 n_srec, u32 n_l
   // 5. entries
   K3In k;
   k.hc = hc;
-  k.recs = recs;
+  k.srecs = srecs;
+  k.lo_sp = lo_sp;
   k.n_lo = n_lo;
   k.lo_rec = lo_rec;
   k.lo_lane = lo_lane;

@@ -505,7 +505,8 @@ def test_c3_full_size():
     assert res.status == 0 and len(truth) == 2
     assert np.array_equal(np.sort(res.races.view("V32")), np.sort(truth.view("V32")))
     head, want = _golden("c3_inj")
-    plan = ConfigPlan(3, inject=1, n_blocks=int(head["overrides"].split("n_blocks':")[1].split("}")[0]))
+    plan = ConfigPlan(3, inject=1, n_blocks=256)  # tools/make_golden.py GOLDEN["c3_inj"]
+    assert plan.n_records == int(head["records"])
     res = _gpu(plan.records(), plan.geometry)
     _assert_same(res.races, want)
 
