@@ -134,6 +134,15 @@ typedef struct bc_config {
   bc_dev_alloc_fn dev_alloc;          /* optional, see above                                     */
   bc_dev_free_fn dev_free;
   void* alloc_user;
+  /* Block-sharded multi-GPU: with world > 1 and a transport, every rank loads only the
+   * records of the blocks b with b % world == rank (bc_load_trace_shard) and the ranks exchange what
+   * the check needs (clock snapshots, sync records, per-window (granule, event) items to the granule's
+   * owner, races to rank 0) over the transport.  Exactly one of:                                    */
+  const void* nccl_unique_id;         /* 128 B from bc_nccl_unique_id() on rank 0, broadcast by the caller
+                                         (e.g. torch.distributed): NCCL over NVLink / NVSwitch, one
+                                         process per GPU; bc_init is collective                     */
+  struct bc_group* group;             /* in-process transport: the ranks are contexts of this process,
+                                         one host thread each (bc_group_create_local)              */
 } bc_config;
 
 typedef struct bc_stats {
@@ -164,6 +173,26 @@ bc_status bc_init(const bc_config* cfg, struct bc_ctx** out);
  * on cfg.device, borrowed (not copied) until the next bc_load_trace / bc_destroy; the caller
  * must keep it alive and unmodified.  n_recs may be 0.  n_recs >= 2^32 - 1 -> BC_ERR_OVERFLOW. */
 bc_status bc_load_trace(struct bc_ctx* ctx, const bc_record* recs, uint64_t n_recs, int recs_on_device);
+
+/* Block-sharded trace (per-block partitioning of P:L1072-1084): this rank's records --
+ * those of the traced blocks b with b % world == rank -- in trace order, with rec_index[i] = the
+ * global record index of recs[i] (strictly increasing, < n_global), n_global = records of the whole
+ * trace.  Ownership as bc_load_trace (recs_on_device applies to both arrays).  Needs a context with a
+ * transport (nccl_unique_id or group).  bc_detect is then collective: every rank calls it; race
+ * lists come back on rank 0 (bc_races on other ranks: 0 races).  Errors: BC_ERR_STATE (no transport),
+ * BC_ERR_INVALID_ARG, BC_ERR_OVERFLOW (n_global >= 2^32 - 1), BC_ERR_OOM / BC_ERR_CUDA. */
+bc_status bc_load_trace_shard(bc_ctx* ctx, const bc_record* recs, const uint32_t* rec_index, uint64_t n_local,
+                              uint64_t n_global, int recs_on_device);
+
+/* 128-byte NCCL unique id for bc_config.nccl_unique_id (call on rank 0 only).  BC_ERR_NCCL if no NCCL
+ * library can be loaded (libbc dlopens the libnccl.so.2 already in the process, else the system's). */
+bc_status bc_nccl_unique_id(void* out128);
+
+/* In-process group of `world` ranks for bc_config.group (tests, or several GPUs driven by one
+ * process); destroy after every context of the group. */
+typedef struct bc_group bc_group;
+bc_status bc_group_create_local(int world, bc_group** out);
+void bc_group_destroy(bc_group* group);
 
 /* Optional per-lane store values (reading R6b in DESIGN.md).
  *   values[r * 32 + l] = the value lane l of store record r writes (8 B; a 64-bit digest for wider

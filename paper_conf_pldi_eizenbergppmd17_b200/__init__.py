@@ -38,8 +38,9 @@ F_RELEASE_OVERWRITE = 1
 F_NO_SAME_VALUE_FILTER = 2
 F_COUNT_GATHERS = 4  # statistics: fill stats["clock_gathers"] (one extra pass)
 
-EXPORTS = ["bc_init", "bc_load_trace", "bc_load_values", "bc_detect", "bc_races", "bc_races_device", "bc_destroy",
-           "bc_status_string", "bc_last_error", "bc_phase_name"]
+EXPORTS = sorted(["bc_init", "bc_load_trace", "bc_load_values", "bc_detect", "bc_races", "bc_races_device",
+                  "bc_destroy", "bc_status_string", "bc_last_error", "bc_phase_name", "bc_load_trace_shard",
+                  "bc_nccl_unique_id", "bc_group_create_local", "bc_group_destroy"])
 
 
 class BcError(RuntimeError):
@@ -58,7 +59,8 @@ class _Config(ctypes.Structure):
                 ("smem_bytes_per_block", ctypes.c_uint32), ("flags", ctypes.c_uint32),
                 ("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("stream", ctypes.c_void_p), ("window_events", ctypes.c_uint64),
-                ("dev_alloc", _ALLOC_FN), ("dev_free", _FREE_FN), ("alloc_user", ctypes.c_void_p)]
+                ("dev_alloc", _ALLOC_FN), ("dev_free", _FREE_FN), ("alloc_user", ctypes.c_void_p),
+                ("nccl_unique_id", ctypes.c_void_p), ("group", ctypes.c_void_p)]
 
 
 class _Stats(ctypes.Structure):
@@ -102,6 +104,14 @@ def lib():
         L.bc_last_error.argtypes = [ctypes.c_void_p]
         L.bc_phase_name.restype = ctypes.c_char_p
         L.bc_phase_name.argtypes = [ctypes.c_int]
+        L.bc_load_trace_shard.restype = ctypes.c_int
+        L.bc_load_trace_shard.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                          ctypes.c_uint64, ctypes.c_int]
+        L.bc_nccl_unique_id.restype = ctypes.c_int
+        L.bc_nccl_unique_id.argtypes = [ctypes.c_void_p]
+        L.bc_group_create_local.restype = ctypes.c_int
+        L.bc_group_create_local.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_void_p)]
+        L.bc_group_destroy.argtypes = [ctypes.c_void_p]
         _lib = L
     return _lib
 
@@ -144,12 +154,13 @@ class Context:
     """One traced launch geometry on one GPU (bc_init ... bc_destroy)."""
 
     def __init__(self, geometry: dict, device: int = 0, flags: int = 0, stream=None, rank: int = 0, world: int = 1,
-                 window_events: int = 0, allocator=None):
+                 window_events: int = 0, allocator=None, nccl_id: bytes = None, group: "LocalGroup" = None):
         """rank / world > 1: address-sharded check (bc.h bc_config.rank/world): every rank loads
         the same trace and reports the races of the shadow granules it owns; merge the per-rank
         lists with merge_races() or gather_races().  window_events: bc_config.window_events (0 =
         auto).  allocator: None (cudaMalloc), "torch" (torch's caching allocator) or a
-        (dev_alloc, dev_free) pair of ctypes callbacks."""
+        (dev_alloc, dev_free) pair of ctypes callbacks.  nccl_id (128 bytes of nccl_unique_id() from
+        rank 0) or group (LocalGroup): the block-sharded multi-GPU check (load_trace_shard)."""
         L = lib()
         grid = tuple(geometry["grid"]) + (1,) * (3 - len(geometry["grid"]))
         block = tuple(geometry["block"]) + (1,) * (3 - len(geometry["block"]))
@@ -164,6 +175,12 @@ class Context:
         c.rank, c.world = rank, world
         c.stream = stream
         c.window_events = window_events
+        self._nccl_id = None
+        if nccl_id is not None:
+            self._nccl_id = ctypes.create_string_buffer(bytes(nccl_id), 128)
+            c.nccl_unique_id = ctypes.cast(self._nccl_id, ctypes.c_void_p)
+        if group is not None:
+            c.group = group.handle
         self._alloc = None
         if allocator is not None:
             self._alloc = torch_allocator() if allocator == "torch" else tuple(allocator)
@@ -198,6 +215,23 @@ class Context:
         n = a.nbytes // RECORD_BYTES
         self._keep = a
         return self._check(L.bc_load_trace(self._h, ctypes.c_void_p(a.ctypes.data if n else 0), n, 0))
+
+    def load_trace_shard(self, records, rec_index, n_global: int):
+        """bc_load_trace_shard: this rank's records (those of blocks b % world == rank, trace order) and
+        their global record indices (uint32, increasing); host arrays (copied) or CUDA tensors (borrowed)."""
+        L = lib()
+        if hasattr(records, "is_cuda") and records.is_cuda:
+            n = records.numel() * records.element_size() // RECORD_BYTES
+            self._keep, self._keep_idx = records, rec_index
+            return self._check(L.bc_load_trace_shard(self._h, ctypes.c_void_p(records.data_ptr()),
+                                                      ctypes.c_void_p(rec_index.data_ptr()), n, n_global, 1))
+        a = np.ascontiguousarray(records)
+        idx = np.ascontiguousarray(rec_index, dtype=np.uint32)
+        n = a.nbytes // RECORD_BYTES
+        assert len(idx) == n
+        self._keep, self._keep_idx = a, idx
+        return self._check(L.bc_load_trace_shard(self._h, ctypes.c_void_p(a.ctypes.data if n else 0),
+                                                  ctypes.c_void_p(idx.ctypes.data if n else 0), n, n_global, 0))
 
     def load_values(self, values):
         """bc_load_values: per-lane store values [n_records, 32] (uint64) as a host
@@ -258,6 +292,51 @@ class Context:
 
     def __exit__(self, *a):
         self.close()
+
+
+def nccl_unique_id() -> bytes:
+    """bc_nccl_unique_id: 128 bytes for Context(nccl_id=...) (rank 0 makes it, the caller broadcasts it)."""
+    buf = ctypes.create_string_buffer(128)
+    st = lib().bc_nccl_unique_id(buf)
+    if st != OK:
+        raise BcError(st, "no NCCL library")
+    return buf.raw
+
+
+class LocalGroup:
+    """bc_group_create_local: `world` ranks as contexts of this process, one host thread each."""
+
+    def __init__(self, world: int):
+        h = ctypes.c_void_p()
+        st = lib().bc_group_create_local(world, ctypes.byref(h))
+        if st != OK:
+            raise BcError(st, "group")
+        self.handle, self.world = h, world
+
+    def close(self):
+        if self.handle:
+            lib().bc_group_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def shard_trace(records, geometry: dict, rank: int, world: int):
+    """The block shard of rank `rank`: the records of the traced blocks b with
+    b % world == rank, in trace order, and their global record indices (marshalling only)."""
+    grid = tuple(geometry["grid"]) + (1,) * (3 - len(geometry["grid"]))
+    block = tuple(geometry["block"]) + (1,) * (3 - len(geometry["block"]))
+    tpb = block[0] * block[1] * block[2]
+    ws = geometry.get("warp_size", 32)
+    wpb = (tpb + ws - 1) // ws
+    recs = np.asarray(records)
+    blocks = recs["warp"].astype(np.int64) // wpb
+    idx = np.nonzero(blocks % world == rank)[0].astype(np.uint32)
+    return recs[idx], idx
 
 
 def merge_races(parts) -> np.ndarray:

@@ -10,6 +10,7 @@
 #include <cstring>
 #include <string>
 
+#include "comm.cuh"
 #include "common.cuh"
 #include "kernels.cuh"
 
@@ -19,54 +20,92 @@ namespace bc {
 std::atomic<u64> g_launches{0};  // kernels launched by this process (per-detect delta in bc_stats)
 }
 
-struct bc_ctx {
-  bc_config cfg;
-  Geo g;
-  cudaStream_t stream = nullptr;
-  bool own_stream = false;
-  DevAlloc da;
-  const bc_record* trace = nullptr;  // device
-  bc_record* owned = nullptr;
-  size_t owned_cap = 0;
-  u64 n_recs = 0;
-  bool loaded = false;
-  bool detected = false;
-  const u64* values = nullptr;  // device, per-lane store values (row f3), nullable
-  u64* values_owned = nullptr;
-  size_t values_cap = 0;
-  bc_race* races = nullptr;  // device, findings first
-  size_t races_cap = 0;
-  u64 n_races = 0;
-  uint4* rbuf = nullptr;     // device, K7 race records of all windows (grown on demand)
-  size_t rbuf_cap = 0;       // entries
-  uint2* pool = nullptr;     // device, read-vector pool carried between windows (grown on demand)
-  size_t pool_cap = 0;       // entries
-  bc_stats stats{};
-  Arena arena;  // scratch buffers, reused across bc_detect calls
-  std::string err;
-  cudaEvent_t ev[16] = {};
-  u64* hcnt = nullptr;  // pinned host copy of the device counter array (one D2H copy per host sync)
-};
+#include "ctx.cuh"
 
 static const char* kPhase[] = {"header", "partition", "replay", "sync", "expand", "sort", "check", "finalize",
                                "k_check", "k_sort_items", "k_expand", nullptr};
-enum { PH_HEADER = 0, PH_PARTITION, PH_REPLAY, PH_SYNC, PH_EXPAND, PH_SORT, PH_CHECK, PH_FINALIZE, PH_N };
 
-static bc_status fail(bc_ctx* c, bc_status s, const std::string& msg) {
-  if (c) c->err = msg;
-  return s;
+void* ctx_buffer(bc_ctx* c, int slot, size_t bytes) {
+  if (bytes <= c->xcap[slot]) return c->xbuf[slot];
+  cudaStreamSynchronize(c->stream);
+  c->da.free(c->xbuf[slot], c->xcap[slot]);
+  c->xcap[slot] = 0;
+  bytes = std::max<size_t>(bytes + bytes / 4, 4096);
+  c->xbuf[slot] = c->da.alloc(bytes);
+  if (c->xbuf[slot]) c->xcap[slot] = bytes;
+  return c->xbuf[slot];
 }
 
-static bc_status cuda_check(bc_ctx* c, const char* where) {
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return fail(c, BC_ERR_CUDA, std::string(where) + ": " + cudaGetErrorString(e));
+bc_status check_window(bc_ctx* c, CheckLaunch& L, u64 b, u64* cnt, u64& n_r, u64& pool_used, WindowOut& wo) {
+  cudaStream_t st = c->stream;
+  u64* const hcnt = c->hcnt;
+  if (L.sh_out) {
+    // every carried vector may be re-copied once and every item appended once
+    const u64 need = 2 * pool_used + b + 1024;
+    if (need >= (1ull << 32)) return fail(c, BC_ERR_OVERFLOW, "read-vector pool >= 2^32 entries");
+    if (need > c->pool_cap) {
+      uint2* np = (uint2*)c->da.alloc(need * sizeof(uint2));
+      if (!np) return fail(c, BC_ERR_OOM, "read-vector pool");
+      if (pool_used) cudaMemcpyAsync(np, c->pool, pool_used * sizeof(uint2), cudaMemcpyDeviceToDevice, st);
+      cudaStreamSynchronize(st);
+      c->da.free(c->pool, c->pool_cap * sizeof(uint2));
+      c->pool = np;
+      c->pool_cap = need;
+    }
+  }
+  L.pool = c->pool;
+  L.pool_cnt = reinterpret_cast<u32*>(cnt + C_POOL);
+  L.pool_cap = (u32)std::min<u64>(c->pool_cap, 0xFFFFFFFFull);
+  L.race_cnt = reinterpret_cast<u32*>(cnt + C_RACES);
+  L.seg_cnt = cnt + C_SEGMENTS;
+  u32 herr = 0;
+  for (int attempt = 0; attempt < 3; ++attempt) {
+    if (c->rbuf_cap < (1u << 16)) {
+      c->da.free(c->rbuf, c->rbuf_cap * sizeof(uint4));
+      c->rbuf_cap = 0;
+      c->rbuf = (uint4*)c->da.alloc((1u << 16) * sizeof(uint4));
+      if (!c->rbuf) return fail(c, BC_ERR_OOM, "race buffer");
+      c->rbuf_cap = 1u << 16;
+    }
+    L.races = c->rbuf;
+    L.race_cap = (u32)std::min<u64>(c->rbuf_cap, 0xFFFFFFFFull);
+    // device counters: races so far, this window's segments / gathers, the carried pool size
+    hcnt[C_RACES] = n_r;
+    hcnt[C_SEGMENTS] = 0;
+    hcnt[C_GATHERS] = 0;
+    hcnt[C_POOL] = pool_used;
+    cudaMemcpyAsync(cnt + C_RACES, hcnt + C_RACES, 4 * sizeof(u64), cudaMemcpyHostToDevice, st);
+    cudaEventRecord(c->ev[10], st);
+    launch_check(L, st);
+    cudaEventRecord(c->ev[11], st);
+    if (L.c.g.flags & BC_F_COUNT_GATHERS) launch_count_gathers(L.keys, L.n_dev, cnt + C_GATHERS, st);
+    cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
+    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "check");
+    herr = (u32)hcnt[C_ERR];
+    if (herr) break;
+    const u64 tot = (u32)hcnt[C_RACES];
+    if (tot <= c->rbuf_cap) break;
+    // more races than room: grow (keeping the earlier windows' races) and check the window again
+    // (idempotent: the shadow entries it writes are a function of the window, the pool is reset)
+    const u64 cap2 = std::max<u64>(2 * c->rbuf_cap, tot + 1024);
+    if (cap2 >= 0xFFFFFFFFull) return fail(c, BC_ERR_OVERFLOW, "2^32 or more races");
+    uint4* nb2 = (uint4*)c->da.alloc(cap2 * sizeof(uint4));
+    if (!nb2) return fail(c, BC_ERR_OOM, "race buffer");
+    if (n_r) cudaMemcpyAsync(nb2, c->rbuf, n_r * sizeof(uint4), cudaMemcpyDeviceToDevice, st);
+    cudaStreamSynchronize(st);
+    c->da.free(c->rbuf, c->rbuf_cap * sizeof(uint4));
+    c->rbuf = nb2;
+    c->rbuf_cap = cap2;
+  }
+  if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "infeasible trace");
+  if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "index overflow / sync lookup step cap");
+  n_r = (u32)hcnt[C_RACES];
+  pool_used = (u32)hcnt[C_POOL];
+  wo.items = hcnt[C_ITEMS];
+  wo.segments = hcnt[C_SEGMENTS];
+  wo.gathers = hcnt[C_GATHERS];
+  cudaEventElapsedTime(&wo.ms_check, c->ev[10], c->ev[11]);
   return BC_OK;
-}
-
-static int bits_for(u64 maxval) {
-  int b = 0;
-  while (b < 64 && (maxval >> b)) ++b;
-  return b;
 }
 
 extern "C" {
@@ -141,6 +180,19 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   c->da.user = cfg->alloc_user;
   c->da.st = c->stream;
   c->arena.da = &c->da;
+  if (cfg->world > 1 && (cfg->nccl_unique_id || cfg->group)) {
+    if (cfg->nccl_unique_id && cfg->group) {
+      bc_destroy(c);
+      return BC_ERR_INVALID_ARG;
+    }
+    int cs = BC_OK;
+    c->comm = cfg->group ? make_local_comm(reinterpret_cast<LocalGroup*>(cfg->group), cfg->rank, cfg->device)
+                         : make_nccl_comm(cfg->nccl_unique_id, cfg->rank, cfg->world, &cs);
+    if (!c->comm) {
+      bc_destroy(c);
+      return (bc_status)cs;
+    }
+  }
   // keep pooled scratch memory cached between bc_detect calls
   cudaMemPool_t pool;
   if (cudaDeviceGetDefaultMemPool(&pool, cfg->device) == cudaSuccess) {
@@ -166,7 +218,10 @@ void bc_destroy(bc_ctx* c) {
   c->da.free(c->races, c->races_cap * sizeof(bc_race));
   c->da.free(c->rbuf, c->rbuf_cap * sizeof(uint4));
   c->da.free(c->pool, c->pool_cap * sizeof(uint2));
+  c->da.free(c->gidx_owned, c->gidx_cap);
+  for (int i = 0; i < 5; ++i) c->da.free(c->xbuf[i], c->xcap[i]);
   c->arena.free_all();
+  delete c->comm;
   if (c->hcnt) cudaFreeHost(c->hcnt);
   for (int i = 0; i < 16; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
@@ -179,6 +234,7 @@ bc_status bc_load_trace(bc_ctx* c, const bc_record* recs, uint64_t n, int on_dev
   if (n && !recs) return fail(c, BC_ERR_INVALID_ARG, "null trace");
   if (n >= 0xFFFFFFFFull) return fail(c, BC_ERR_OVERFLOW, "2^32 - 1 or more records (32-bit record indices)");
   cudaSetDevice(c->cfg.device);
+  c->sharded = false;
   c->loaded = false;
   c->detected = false;
   c->values = nullptr;
@@ -309,8 +365,8 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* find_blk = S.alloc<u32>(n_bar + 1);
   u32* find_rec = S.alloc<u32>(n_bar + 1);
   u32* find_cnt = reinterpret_cast<u32*>(cnt + C_FINDINGS);
-  launch_replay(hdr16, wrec, warp_start, g, node_base, bar_base, snap, nodes, bar_rec, bar_next, find_blk, find_rec,
-                find_cnt, err, st);
+  launch_replay(hdr16, wrec, nullptr, warp_start, g, node_base, bar_base, snap, nodes, bar_rec, bar_next, find_blk,
+                find_rec, find_cnt, err, st);
   launch_barriers(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err, st);
   launch_snap_blab(snap, n, g.wpb, g.n_warps, n_bar, bar_base, blockR, st);
   cudaEventRecord(c->ev[3], st);
@@ -394,7 +450,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     ++sx.windows;
     // ---- K4: expansion (static slots from the header's per-record upper bounds)
     cudaEventRecord(c->ev[14], st);
-    launch_expand(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, ikeys, ievs, err, st);
+    launch_expand(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, nullptr, R0, ikeys, ievs, err, st);
     cudaEventRecord(c->ev[15], st);
     // ---- K5: stable radix sort by granule key; the first pass drops the never-written slots
     cudaEventRecord(c->ev[12], st);
@@ -407,18 +463,6 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     if (sh_out) {
       if (have_state) cudaMemcpyAsync(sh_out, sh_cur, 2 * n_keys * sizeof(uint4), cudaMemcpyDeviceToDevice, st);
       else cudaMemsetAsync(sh_out, 0, 2 * n_keys * sizeof(uint4), st);
-      // every carried vector may be re-copied once and every item appended once
-      const u64 need = 2 * pool_used + b + 1024;
-      if (need >= (1ull << 32)) return fail(c, BC_ERR_OVERFLOW, "read-vector pool >= 2^32 entries");
-      if (need > c->pool_cap) {
-        uint2* np = (uint2*)c->da.alloc(need * sizeof(uint2));
-        if (!np) return fail(c, BC_ERR_OOM, "read-vector pool");
-        if (pool_used) cudaMemcpyAsync(np, c->pool, pool_used * sizeof(uint2), cudaMemcpyDeviceToDevice, st);
-        cudaStreamSynchronize(st);
-        c->da.free(c->pool, c->pool_cap * sizeof(uint2));
-        c->pool = np;
-        c->pool_cap = need;
-      }
     }
     CheckLaunch L{};
     L.c = hc;
@@ -429,65 +473,20 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     L.R0 = (u32)R0;
     L.sh_in = have_state ? sh_cur : nullptr;
     L.sh_out = sh_out;
-    L.pool = c->pool;
-    L.pool_cnt = reinterpret_cast<u32*>(cnt + C_POOL);
-    L.pool_cap = (u32)std::min<u64>(c->pool_cap, 0xFFFFFFFFull);
-    L.race_cnt = reinterpret_cast<u32*>(cnt + C_RACES);
-    L.seg_cnt = cnt + C_SEGMENTS;
     L.values = c->values;
     L.status = cstatus;
-    for (int attempt = 0; attempt < 3; ++attempt) {
-      if (c->rbuf_cap < (1u << 16)) {
-        c->da.free(c->rbuf, c->rbuf_cap * sizeof(uint4));
-        c->rbuf_cap = 0;
-        c->rbuf = (uint4*)c->da.alloc((1u << 16) * sizeof(uint4));
-        if (!c->rbuf) return fail(c, BC_ERR_OOM, "race buffer");
-        c->rbuf_cap = 1u << 16;
-      }
-      L.races = c->rbuf;
-      L.race_cap = (u32)std::min<u64>(c->rbuf_cap, 0xFFFFFFFFull);
-      // device counters: races so far, this window's segments / gathers, the carried pool size
-      hcnt[C_RACES] = n_r;
-      hcnt[C_SEGMENTS] = 0;
-      hcnt[C_GATHERS] = 0;
-      hcnt[C_POOL] = pool_used;
-      cudaMemcpyAsync(cnt + C_RACES, hcnt + C_RACES, 4 * sizeof(u64), cudaMemcpyHostToDevice, st);
-      cudaEventRecord(c->ev[10], st);
-      launch_check(L, st);
-      cudaEventRecord(c->ev[11], st);
-      if (g.flags & BC_F_COUNT_GATHERS) launch_count_gathers(skey, n_items_dev, cnt + C_GATHERS, st);
-      cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
-      if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "check");
-      herr = (u32)hcnt[C_ERR];
-      if (herr) break;
-      const u64 tot = (u32)hcnt[C_RACES];
-      if (tot <= c->rbuf_cap) break;
-      // more races than room: grow (keeping the earlier windows' races) and check the window again
-      // (idempotent: the shadow entries it writes are a function of the window, the pool is reset)
-      const u64 cap2 = std::max<u64>(2 * c->rbuf_cap, tot + 1024);
-      if (cap2 >= 0xFFFFFFFFull) return fail(c, BC_ERR_OVERFLOW, "2^32 or more races");
-      uint4* nb2 = (uint4*)c->da.alloc(cap2 * sizeof(uint4));
-      if (!nb2) return fail(c, BC_ERR_OOM, "race buffer");
-      if (n_r) cudaMemcpyAsync(nb2, c->rbuf, n_r * sizeof(uint4), cudaMemcpyDeviceToDevice, st);
-      cudaStreamSynchronize(st);
-      c->da.free(c->rbuf, c->rbuf_cap * sizeof(uint4));
-      c->rbuf = nb2;
-      c->rbuf_cap = cap2;
-    }
-    if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "infeasible trace");
-    if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "index overflow / sync lookup step cap");
-    n_r = (u32)hcnt[C_RACES];
-    pool_used = (u32)hcnt[C_POOL];
-    n_items += hcnt[C_ITEMS];
-    sx.segments += hcnt[C_SEGMENTS];
-    sx.clock_gathers += hcnt[C_GATHERS];
+    WindowOut wo;
+    bc_status ws = check_window(c, L, b, cnt, n_r, pool_used, wo);
+    if (ws) return ws;
+    n_items += wo.items;
+    sx.segments += wo.segments;
+    sx.clock_gathers += wo.gathers;
     float t = 0;
     cudaEventElapsedTime(&t, c->ev[14], c->ev[15]);
     ms_ex += t;
     cudaEventElapsedTime(&t, c->ev[12], c->ev[13]);
     ms_sort += t;
-    cudaEventElapsedTime(&t, c->ev[10], c->ev[11]);
-    ms_chk += t;
+    ms_chk += wo.ms_check;
     if (sh_out) {
       std::swap(sh_cur, sh_nxt);
       have_state = true;
@@ -538,9 +537,58 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   return BC_OK;
 }
 
+bc_status bc_load_trace_shard(bc_ctx* c, const bc_record* recs, const uint32_t* rec_index, uint64_t n_local,
+                              uint64_t n_global, int on_device) {
+  if (!c) return BC_ERR_INVALID_ARG;
+  if (!c->comm) return fail(c, BC_ERR_STATE, "bc_load_trace_shard needs a transport (nccl_unique_id or group)");
+  if (n_global >= 0xFFFFFFFFull) return fail(c, BC_ERR_OVERFLOW, "2^32 - 1 or more records");
+  if (n_local > n_global || (n_local && !rec_index)) return fail(c, BC_ERR_INVALID_ARG, "shard indices");
+  if (!on_device)
+    for (u64 i = 0; i < n_local; ++i)
+      if (rec_index[i] >= n_global || (i && rec_index[i] <= rec_index[i - 1]))
+        return fail(c, BC_ERR_INVALID_ARG, "rec_index must increase and stay below n_global");
+  bc_status s = bc_load_trace(c, recs, n_local, on_device);
+  if (s) return s;
+  c->loaded = false;
+  if (n_local && (!on_device || ((uintptr_t)rec_index & 3))) {
+    const size_t bytes = n_local * sizeof(u32);
+    if (bytes > c->gidx_cap) {
+      c->da.free(c->gidx_owned, c->gidx_cap);
+      c->gidx_cap = 0;
+      c->gidx_owned = (u32*)c->da.alloc(bytes);
+      if (!c->gidx_owned) return fail(c, BC_ERR_OOM, "record index buffer");
+      c->gidx_cap = bytes;
+    }
+    cudaMemcpyAsync(c->gidx_owned, rec_index, bytes, on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
+                    c->stream);
+    if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_check(c, "record index copy");
+    c->gidx = c->gidx_owned;
+  } else {
+    c->gidx = rec_index;
+  }
+  c->sharded = true;
+  c->n_global = n_global;
+  c->loaded = true;
+  return BC_OK;
+}
+
+bc_status bc_nccl_unique_id(void* out128) {
+  if (!out128) return BC_ERR_INVALID_ARG;
+  return (bc_status)nccl_unique_id(out128);
+}
+
+bc_status bc_group_create_local(int world, bc_group** out) {
+  if (!out || world < 1 || world > 1024) return BC_ERR_INVALID_ARG;
+  *out = reinterpret_cast<bc_group*>(local_group_create(world));
+  return BC_OK;
+}
+
+void bc_group_destroy(bc_group* g) { local_group_destroy(reinterpret_cast<LocalGroup*>(g)); }
+
 bc_status bc_load_values(bc_ctx* c, const uint64_t* values, uint64_t n, int on_device) {
   if (!c) return BC_ERR_INVALID_ARG;
   if (!c->loaded) return fail(c, BC_ERR_STATE, "bc_load_values before bc_load_trace");
+  if (c->sharded && values) return fail(c, BC_ERR_INVALID_ARG, "store values with a sharded trace: not supported");
   c->detected = false;
   c->values = nullptr;
   if (!values) return BC_OK;
@@ -576,7 +624,7 @@ bc_status bc_detect(bc_ctx* c, bc_stats* out) {
   {
     Scratch S(c->stream, &c->arena);
     try {
-      s = detect_impl(c, S);
+      s = c->sharded ? detect_sharded(c, S) : detect_impl(c, S);
     } catch (const std::bad_alloc&) {
       s = fail(c, BC_ERR_OOM, "scratch allocation");
     }

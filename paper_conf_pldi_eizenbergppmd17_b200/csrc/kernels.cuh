@@ -115,15 +115,16 @@ void launch_warp_scans(const u32* rec_cnt, const u32* if_cnt, const u32* bar_cnt
 void launch_page_rank(u32* words, const u64* n_words_dev, const u32* page_bits, u32* page_rank, u32* wl_prefix,
                       u64* n_pages_dev, u32* need_sort, int presorted, cudaStream_t st);
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st);
-void launch_replay(const uint4* hdr16, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
-                   const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next, u32* find_blk,
-                   u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st);
+void launch_replay(const uint4* hdr16, const u32* wrec, const u32* gidx, const u32* warp_start, const Geo& g,
+                   const u32* node_base, const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next,
+                   u32* find_blk, u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st);
 void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, const u32* bar_rec, const u32* bar_next,
                      u32* blockR, u32* err, cudaStream_t st);
 void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, const u32* bar_base, const u32* blockR,
                       cudaStream_t st);
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
-                   const u64* cum, u64 R0, u64 R1, u32* keys, u32* evs, u32* err, cudaStream_t st);
+                   const u64* cum, u64 R0, u64 R1, const u32* gidx, u64 G0, u32* keys, u32* evs, u32* err,
+                   cudaStream_t st);
 void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st);
 
 // sync.cu

@@ -183,7 +183,7 @@ __global__ void k_warp_start(const u32* __restrict__ skeys, u64 n, u32 n_warps, 
 // nodes {mask, parent, popen}; per BAR its record and the warp's next record (barrier feasibility)
 // and a BARRIER_DIVERGENCE finding when the mask is not the warp's initial mask.
 __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16, const u32* __restrict__ wrec,
-                                                const u32* __restrict__ warp_start, Geo g,
+                                                const u32* __restrict__ gidx, const u32* __restrict__ warp_start, Geo g,
                                                 const u32* __restrict__ node_base, const u32* __restrict__ bar_base,
                                                 uint4* __restrict__ snap, uint4* __restrict__ nodes,
                                                 u32* __restrict__ bar_rec, u32* __restrict__ bar_next,
@@ -205,27 +205,31 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
   bool bad = false;
   const u32 nb0 = node_base[w], bb0 = bar_base[w];
   const u32 i0 = warp_start[w], i1 = warp_start[w + 1];
-  u32 nr = 0;
+  // local record index (hdr16 / snap position) and its global index (the step label is global index + 1;
+  // the same unless the context holds a block shard of the trace)
+  u32 nr = 0, ng = 0;
   uint4 nh = make_uint4(0, 0, 0, 0);
   if (i0 + lane < i1) {
     nr = wrec[i0 + lane];
     nh = __ldg(hdr16 + nr);
+    ng = gidx ? __ldg(gidx + nr) : nr;
   }
   for (u32 c0 = i0; c0 < i1 && !bad; c0 += 32) {
-    const u32 r = nr;
+    const u32 r = nr, rg = ng;
     const uint4 hv = nh;
     const u32 cnt = min(32u, i1 - c0);
     if (c0 + 32 + lane < i1) {  // next chunk in flight while this one is stepped through
       nr = wrec[c0 + 32 + lane];
       nh = __ldg(hdr16 + nr);
+      ng = gidx ? __ldg(gidx + nr) : nr;
     }
     s_hdr[wib][lane] = hv;
-    s_rec[wib][lane] = r;
+    s_rec[wib][lane] = rg;
     __syncwarp();
     // control records (FENCE, BAR, IF, ELSE, FI) are stepped one by one; the runs of endi records
     // between them (LD / ST / ATOM / ACQ / REL / AR: ps := rec + 1, stack unchanged) in parallel
     const u32 ctl = __ballot_sync(0xFFFFFFFFu, lane < cnt && (hv.z & 0xFFu) >= BC_OP_FENCE);
-    const u32 rprev = __shfl_up_sync(0xFFFFFFFFu, r, 1);
+    const u32 rprev = __shfl_up_sync(0xFFFFFFFFu, rg, 1);
     u32 my_ps = 0, my_node = 0, my_phase = 0;
     bool badl = false;
     u32 sidx = 0;
@@ -395,6 +399,7 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
                                                        const u32* __restrict__ page_bits,
                                                        const u32* __restrict__ page_rank, u32 shared_base,
                                                        const u64* __restrict__ cum, u64 R0, u64 R1,
+                                                       const u32* __restrict__ gidx, u64 G0,
                                                        u32* __restrict__ okeys, u32* __restrict__ oevs,
                                                        u32* __restrict__ err) {
   extern __shared__ __align__(128) unsigned char ex_smem[];
@@ -472,7 +477,8 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
         }
       }
       const u64 o = (u64)uoj + (u64)__popc(hmask & lt) * nk;
-      const u32 ev = (u32)(r << 5) | (u32)lane;  // window-local event id
+      // window-local event id: (global record - window start) << 5 | lane
+      const u32 ev = (u32)(((gidx ? (u64)__ldg(gidx + R0 + r) : R0 + r) - G0) << 5) | (u32)lane;
       if (nk == 1 && g.world == 1) {  // one granule, one shard: the common case
         okeys[o] = key0 != KEY_DROP ? ((key0 << 2) | opc) : KEY_DROP;
         oevs[o] = ev;
@@ -605,10 +611,10 @@ void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cu
   k_warp_start<<<(n_warps + 1 + 255) / 256, 256, 0, st>>>(skeys, n, n_warps, warp_start); ++g_launches;
 }
 
-void launch_replay(const uint4* hdr16, const u32* wrec, const u32* warp_start, const Geo& g, const u32* node_base,
-                   const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next, u32* find_blk,
-                   u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st) {
-  k_replay<<<(unsigned)(((u64)g.n_warps * 32 + 255) / 256), 256, 0, st>>>(hdr16, wrec, warp_start, g, node_base, bar_base, snap, nodes,
+void launch_replay(const uint4* hdr16, const u32* wrec, const u32* gidx, const u32* warp_start, const Geo& g,
+                   const u32* node_base, const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next,
+                   u32* find_blk, u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st) {
+  k_replay<<<(unsigned)(((u64)g.n_warps * 32 + 255) / 256), 256, 0, st>>>(hdr16, wrec, gidx, warp_start, g, node_base, bar_base, snap, nodes,
                                                      bar_rec, bar_next, find_blk, find_rec, find_cnt, err); ++g_launches;
 }
 
@@ -707,7 +713,8 @@ void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStrea
 }
 
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
-                   const u64* cum, u64 R0, u64 R1, u32* keys, u32* evs, u32* err, cudaStream_t st) {
+                   const u64* cum, u64 R0, u64 R1, const u32* gidx, u64 G0, u32* keys, u32* evs, u32* err,
+                   cudaStream_t st) {
   const u64 chunks = (R1 - R0 + EX_REC - 1) / EX_REC;
   if (!chunks) return;
   const size_t smem = sizeof(bc_record) * EX_REC * EX_STAGES + 8 * EX_STAGES;
@@ -723,7 +730,8 @@ void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, co
     grid[dev] = sms * (per > 0 ? per : 1);
   }
   const unsigned gr = (unsigned)std::min<u64>(chunks, (u64)grid[dev]);
-  k_expand<<<gr, EX_THREADS, smem, st>>>(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, keys, evs, err);
+  k_expand<<<gr, EX_THREADS, smem, st>>>(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, gidx, G0, keys, evs,
+                                         err);
   ++g_launches;
 }
 

@@ -1,8 +1,15 @@
-"""Address-sharded multi-GPU mode (bc.h bc_config.rank/world).
+"""Multi-GPU modes (bc.h bc_config.rank/world).
 
-Each rank gets the same trace, derives the same clocks, and checks only the shadow granules
-it owns; the per-rank race lists are disjoint and their canonical merge must equal the
-single-GPU list (and hence the oracle's).
+Block-sharded (bc_load_trace_shard + a transport): rank r holds the records of the blocks
+b % world == r, replays only those, exchanges clock snapshots / branch nodes / sync records, routes
+every (granule, event) item to the granule's owner per window, and rank 0 finalizes the gathered
+races; its list must equal the oracle's.  The GPU tests run the ranks as threads over the
+in-process transport (bc_group_create_local) on one B200 -- the same data plane as NCCL, whose
+calls are only the transport.
+
+Replicated-trace address sharding (bc_load_trace with world > 1, no transport): each rank gets the
+same trace, derives the same clocks, and checks only the shadow granules it owns; the per-rank race
+lists are disjoint and their canonical merge must equal the single-GPU list.
 
 * CPU (`-m "not gpu"`): the host-side merge (merge_races) restores the canonical order from
   any disjoint split of an oracle race list, and gather_races does it across a world-size-2
@@ -95,8 +102,140 @@ def test_gather_over_gloo(tmp_path):
     assert np.array_equal(got.view(np.uint8), want.view(np.uint8))
 
 
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+def test_shard_trace_partitions_blocks(world):
+    """bc.shard_trace: the shards are disjoint, cover every record, keep trace order, and hold whole
+    blocks (every record of block b on rank b % world)."""
+    recs, geom = _c4_small()
+    seen = np.zeros(len(recs), dtype=np.int64)
+    wpb = (geom["block"][0] + 31) // 32
+    for r in range(world):
+        loc, idx = bc.shard_trace(recs, geom, r, world)
+        assert np.all(np.diff(idx.astype(np.int64)) > 0)
+        assert np.array_equal(loc.view(np.uint8), recs[idx].view(np.uint8))
+        assert np.all((loc["warp"] // wpb) % world == r)
+        seen[idx] += 1
+    assert np.all(seen == 1)
+
+
+def _shard_worker(rank, world, port, path):
+    """one rank of a world-size-2 gloo group: shard the trace, all-gather the record indices, and
+    check that every global record is on exactly one rank (the loader side of the sharded path)"""
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    recs = np.load(path)
+    geom = dict(grid=(12, 1, 1), block=(256, 1, 1), smem_bytes=16)
+    loc, idx = bc.shard_trace(recs, geom, rank, world)
+    sizes = [torch.zeros(1, dtype=torch.int64) for _ in range(world)]
+    dist.all_gather(sizes, torch.tensor([len(idx)]))
+    mx = int(max(s.item() for s in sizes))
+    buf = torch.full((mx,), -1, dtype=torch.int64)
+    buf[:len(idx)] = torch.from_numpy(idx.astype(np.int64))
+    parts = [torch.zeros(mx, dtype=torch.int64) for _ in range(world)]
+    dist.all_gather(parts, buf)
+    allidx = torch.cat([p[p >= 0] for p in parts]).numpy()
+    assert sorted(allidx.tolist()) == list(range(len(recs)))
+    assert int(sum(s.item() for s in sizes)) == len(recs)
+    dist.destroy_process_group()
+
+
+def test_shard_loader_over_gloo(tmp_path):
+    import socket
+
+    import torch.multiprocessing as mp
+    recs, geom = _c4_small()
+    assert geom["grid"][0] == 12
+    path = str(tmp_path / "recs.npy")
+    np.save(path, recs)
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    mp.spawn(_shard_worker, args=(2, port, path), nprocs=2, join=True)
+
+
 # ----------------------------------------------------------------------------- GPU
-def _sharded(recs, geom, world):
+def sharded_detect(recs, geom, world, window_events=0, timeout=300):
+    """Block-sharded detect: `world` ranks = threads over one in-process group on cuda:0.  Returns
+    rank 0's (status, races, stats) and every rank's status."""
+    import threading
+    grp = bc.LocalGroup(world)
+    out, errs = [None] * world, [None] * world
+
+    def run(r):
+        try:
+            with bc.Context(geom, device=0, rank=r, world=world, group=grp, window_events=window_events) as ctx:
+                loc, idx = bc.shard_trace(recs, geom, r, world)
+                ctx.load_trace_shard(loc, idx, len(recs))
+                st, stats = ctx.detect(allow=(-2, -8))
+                out[r] = (st, ctx.races() if st == 0 else None, stats)
+        except Exception as e:  # pragma: no cover - reported below
+            errs[r] = e
+
+    ts = [threading.Thread(target=run, args=(r,), daemon=True) for r in range(world)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join(timeout)
+    assert not any(t.is_alive() for t in ts), "a rank hung"
+    grp.close()
+    for e in errs:
+        if e is not None:
+            raise e
+    sts = [o[0] for o in out]
+    assert len(set(sts)) == 1, sts  # every rank agrees on the status
+    for o in out[1:]:
+        assert o[0] != 0 or len(o[1]) == 0  # races come back on rank 0 only
+    return out[0]
+
+
+def assert_sharded(recs, geom, world, window_events=0):
+    st, want, stats_o = oracle.detect_geom(recs, geom)
+    st2, got, stats = sharded_detect(recs, geom, world, window_events)
+    assert st2 == st, (st2, st)
+    if st != 0:
+        return want, stats
+    assert len(got) == len(want), (len(got), len(want), got[:3], want[:3])
+    assert np.array_equal(got.view(np.uint8), want.view(np.uint8))
+    assert stats["lane_events"] == stats_o["lane_events"]
+    return want, stats
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("case", range(11), ids=lambda i: f"case{i}")
+def test_block_sharded_equals_oracle(case, world):
+    name, recs, geom = _cases()[case]
+    assert_sharded(recs, geom, world)
+
+
+@pytest.mark.gpu
+def test_block_sharded_litmus_and_random():
+    for name, build, _exp, _opts in litmus.SUITE:
+        tb = build()
+        assert_sharded(tb.records(), tb.geom.as_dict(), 2)
+    for seed in range(6000, 6040):
+        recs, tb = random_trace(seed)
+        assert_sharded(recs, tb.geom.as_dict(), 1 + seed % 4)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("we", [64, 3000])
+def test_block_sharded_windows(we):
+    """Sharded and windowed: per window the items go to their owners, whose 32-B shadow entries
+    carry the state to the next window."""
+    for seed in range(6100, 6120):
+        recs, tb = random_trace(seed)
+        assert_sharded(recs, tb.geom.as_dict(), 2, window_events=we)
+    plan = ConfigPlan(4, n_blocks=40, log2_nodes=16, nodes_per_thread=3, inj_scale=8)
+    want, stats = assert_sharded(plan.records(), plan.geometry, 3, window_events=we * 20)
+    assert stats["windows"] > 1
+
+
+def _replicated(recs, geom, world):
     parts, items = [], 0
     for r in range(world):
         res = bc.detect(recs, geom, device="cuda:0", rank=r, world=world)
@@ -128,7 +267,7 @@ def test_sharded_equals_oracle(case, world):
     st, want, _ = oracle.detect_geom(recs, geom)
     if st != 0:
         pytest.skip("infeasible trace")
-    got, items = _sharded(recs, geom, world)
+    got, items = _replicated(recs, geom, world)
     assert len(got) == len(want), (len(got), len(want))
     assert np.array_equal(got.view(np.uint8), want.view(np.uint8))
     single = bc.detect(recs, geom, device="cuda:0")
@@ -143,5 +282,5 @@ def test_sharded_litmus_suite():
         st, want, _ = oracle.detect_geom(recs, geom)
         if st != 0:
             continue
-        got, _ = _sharded(recs, geom, 4)
+        got, _ = _replicated(recs, geom, 4)
         assert np.array_equal(got.view(np.uint8), want.view(np.uint8)), name
