@@ -180,7 +180,7 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   c->da.user = cfg->alloc_user;
   c->da.st = c->stream;
   c->arena.da = &c->da;
-  if (cfg->world > 1 && (cfg->nccl_unique_id || cfg->group)) {
+  if (cfg->world >= 1 && (cfg->nccl_unique_id || cfg->group)) {
     if (cfg->nccl_unique_id && cfg->group) {
       bc_destroy(c);
       return BC_ERR_INVALID_ARG;
