@@ -106,6 +106,9 @@ def _load():
         lib.bcgen_truth_list.restype = ctypes.c_uint64
         lib.bcgen_truth_list.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32]
         lib.bcgen_free.argtypes = [ctypes.c_void_p]
+        lib.bcgen_fill_shard.restype = ctypes.c_uint64
+        lib.bcgen_fill_shard.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32,
+                                         ctypes.c_uint32, ctypes.c_int]
         _lib = lib
     return _lib
 
@@ -139,6 +142,27 @@ class ConfigPlan:
             ptr = buf.data_ptr()
         threads = threads or min(16, os.cpu_count() or 1)
         _load().bcgen_fill(self._h, ctypes.c_void_p(ptr), begin, end, threads)
+
+    def shard_count(self, rank, world):
+        """records in the block shard of `rank`"""
+        return int(_load().bcgen_fill_shard(self._h, None, None, rank, world, min(16, os.cpu_count() or 1)))
+
+    def shard(self, rank, world, out=None):
+        """The block shard (blocks b % world == rank): (records, global indices uint32).  `out`: an
+        optional writable uint8 buffer (e.g. pinned torch tensor) of >= count * 272 bytes."""
+        lib = _load()
+        threads = min(16, os.cpu_count() or 1)
+        n = int(lib.bcgen_fill_shard(self._h, None, None, rank, world, threads))
+        idx = np.empty(n, dtype=np.uint32)
+        if out is None:
+            recs = np.empty(n, dtype=RECORD_DTYPE)
+            ptr = recs.ctypes.data
+        else:
+            recs = out
+            ptr = out.ctypes.data if isinstance(out, np.ndarray) else out.data_ptr()
+        if n:
+            lib.bcgen_fill_shard(self._h, ctypes.c_void_p(ptr), idx.ctypes.data, rank, world, threads)
+        return recs, idx
 
     def records(self) -> np.ndarray:
         a = np.empty(self.n_records, dtype=RECORD_DTYPE)

@@ -529,7 +529,7 @@ struct Gen {
   void fill(Rec* dst, uint64_t begin, uint64_t end) const {
     for (uint64_t i = begin; i < end; ++i) {
       const CRec& c = out[i];
-      Rec& r = dst[i - begin];
+      Rec& r = dst[i - begin];  // (dst points at record `begin`)
       r.warp = c.warp; r.mask = c.mask; r.op = c.op; r.space = c.space;
       r.size_log2 = c.size_log2; r.flags = c.flags; r.aux = c.aux;
       bool has_addr = c.op <= AR_GLB;
@@ -581,6 +581,42 @@ void bcgen_fill(void* h, void* dst, uint64_t begin, uint64_t end, int threads) {
     ts.emplace_back([=] { g->fill((Rec*)dst + (b - begin), b, e); });
   }
   for (auto& t : ts) t.join();
+}
+
+// Block shard: the records of the traced blocks b with b % world == rank, in trace
+// order, and their global indices.  dst == NULL: only the count.
+uint64_t bcgen_fill_shard(void* h, void* dst, uint32_t* idx, uint32_t rank, uint32_t world, int threads) {
+  Gen* g = (Gen*)h;
+  const uint64_t n = g->out.size();
+  if (threads < 1) threads = 1;
+  const uint64_t chunk = (n + threads - 1) / threads;
+  std::vector<uint64_t> cnt(threads + 1, 0);
+  auto mine = [&](uint64_t i) { return (g->out[i].warp / g->wpb) % world == rank; };
+  {
+    std::vector<std::thread> ts;
+    for (int t = 0; t < threads; ++t)
+      ts.emplace_back([&, t] {
+        uint64_t c = 0;
+        for (uint64_t i = t * chunk; i < std::min(n, (t + 1) * chunk); ++i) c += mine(i);
+        cnt[t + 1] = c;
+      });
+    for (auto& t : ts) t.join();
+  }
+  for (int t = 0; t < threads; ++t) cnt[t + 1] += cnt[t];
+  if (!dst) return cnt[threads];
+  std::vector<std::thread> ts;
+  for (int t = 0; t < threads; ++t)
+    ts.emplace_back([&, t] {
+      uint64_t o = cnt[t];
+      for (uint64_t i = t * chunk; i < std::min(n, (t + 1) * chunk); ++i)
+        if (mine(i)) {
+          g->fill((Rec*)dst + o, i, i + 1);
+          idx[o] = (uint32_t)i;
+          ++o;
+        }
+    });
+  for (auto& t : ts) t.join();
+  return cnt[threads];
 }
 
 // Ground truth for the injected races (C4/C5): every injected granule is
