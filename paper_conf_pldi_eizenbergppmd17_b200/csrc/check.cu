@@ -467,16 +467,8 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
 
   // ---- state entering the range
   Sum carry = beg < end ? a.rin[w] : sum_ident();
-  u32 pkx = NONE, pev = 0;  // the item before the block
-  u32 cwk = 0, cwe = 0;     // key word / event of carry.lw
-  if (beg > 0 && beg < end) {
-    pkx = __ldg(a.keys + beg - 1);
-    pev = __ldg(a.evs + beg - 1);
-    if (carry.fk != NONE && carry.lw) {
-      cwk = __ldg(a.keys + carry.lw - 1);
-      cwe = __ldg(a.evs + carry.lw - 1);
-    }
-  }
+  u32 pkx = NONE;  // key word of the item before the block (its event: evs[bb - 1], loaded when needed)
+  if (beg > 0 && beg < end) pkx = __ldg(a.keys + beg - 1);
 
   u32 segs = 0;
   const u32 l0 = lane * KT_IPL;
@@ -548,12 +540,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
           if ((int)lane >= o) incl = combine(up, incl);
         }
         carry = combine(carry, shfl_sum(incl, 31));
-        if (carry.lw && (u64)(carry.lw - 1) >= bb) {
-          cwk = __ldg(a.keys + carry.lw - 1);
-          cwe = __ldg(a.evs + carry.lw - 1);
-        }
-        pkx = __ldg(a.keys + bb + nb - 1);
-        pev = __ldg(a.evs + bb + nb - 1);
+        pkx = __shfl_sync(0xFFFFFFFFu, kl, (nb - 1) / (u32)KT_IPL);  // the block's last item
         continue;
       }
     }
@@ -563,7 +550,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
 
     const u32 cnt = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
     const u32 ppk = lane == 0 ? pkx : sK[tpad(l0 - 1)];
-    const u32 ppe = lane == 0 ? pev : sE[tpad(l0 - 1)];
+    const u32 ppe = lane == 0 ? (bb > 0 ? __ldg(a.evs + bb - 1) : 0u) : sE[tpad(l0 - 1)];
     const u32 gbb = (u32)bb;
 
     // ---- gather the snapshots some query can read: an item with a same-granule neighbour (unless an
@@ -585,7 +572,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
       }
     }
     cp_async_commit();
-    const u32 pw0 = (lane == 0 && ppk != NONE) ? __ldg(&c.snap[R0 + (pev >> 5)].x) : 0u;
+    const u32 pw0 = (lane == 0 && ppk != NONE) ? __ldg(&c.snap[R0 + (ppe >> 5)].x) : 0u;
     cp_async_wait0();
     __syncwarp();
 
@@ -660,10 +647,10 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
           wk = sK[tpad(wl)];
           we = sE[tpad(wl)];
           ww = sS[tpad(wl)].x;  // gathered: the writer has a same-granule successor in the block
-        } else {
-          wk = cwk;
-          we = cwe;
-          ww = __ldg(&c.snap[R0 + (cwe >> 5)].x);
+        } else {  // the last writer lies before the block
+          wk = __ldg(a.keys + lw - 1);
+          we = __ldg(a.evs + lw - 1);
+          ww = __ldg(&c.snap[R0 + (we >> 5)].x);
         }
       }
       u32 pk = ppk, pe = ppe, pw = lane ? sS[tpad(l0 - 1)].x : pw0;
@@ -772,12 +759,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
 
     // ---- block carry
     carry = combine(carry, blk);
-    if (carry.lw && (u64)(carry.lw - 1) >= bb) {
-      cwk = sK[tpad((u32)(carry.lw - 1 - bb))];
-      cwe = sE[tpad((u32)(carry.lw - 1 - bb))];
-    }
     pkx = sK[tpad(nb - 1)];
-    pev = sE[tpad(nb - 1)];
     __syncwarp();
   }
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);

@@ -195,7 +195,10 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
   const u32 lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   if (w >= g.n_warps) return;  // warp-uniform
   const u32 imask = init_mask(g, w);
-  u32 st_node[33], st_mask[33];  // SIMT stack below the top (the top lives in cur_node / cur_mask)
+  // SIMT stack below the top (the top lives in cur_node / cur_mask): warp-uniform, so one copy per
+  // analysis warp in shared memory (a per-lane array would be spilled to local memory 32 times over)
+  __shared__ uint2 s_stack[8][33];
+  uint2* const stk = s_stack[threadIdx.x >> 5];
   u32 cur_node = w, cur_mask = imask;
   u64 then_bits = 0;  // bit d set: level d is a then-node
   int depth = 0;
@@ -278,8 +281,8 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
             nodes[nid] = make_uint4(then, cur_node, ps, 0u);
             nodes[nid + 1] = make_uint4(mask & ~then, cur_node, ps, 0u);
           }
-          st_node[depth] = cur_node;
-          st_mask[depth] = cur_mask;
+          if (lane == 0) stk[depth] = make_uint2(cur_node, cur_mask);
+          __syncwarp();
           ++depth;
           cur_node = nid;
           cur_mask = then;
@@ -290,7 +293,7 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
         case BC_OP_ELSE: {
           if (depth == 0 || !((then_bits >> depth) & 1ull)) { bad = true; break; }
           cur_node += 1;
-          cur_mask = st_mask[depth - 1] & ~cur_mask;
+          cur_mask = stk[depth - 1].y & ~cur_mask;
           then_bits &= ~(1ull << depth);
           ps = rj + 1;
           break;
@@ -298,8 +301,9 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
         case BC_OP_FI: {
           if (depth == 0 || ((then_bits >> depth) & 1ull)) { bad = true; break; }
           --depth;
-          cur_node = st_node[depth];
-          cur_mask = st_mask[depth];
+          const uint2 top = stk[depth];
+          cur_node = top.x;
+          cur_mask = top.y;
           ps = rj + 1;
           break;
         }
@@ -438,18 +442,30 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
     // one load per lane before waiting
     const u64 rl = cbase + (u64)wid + (u64)(lane & (EX_RPW - 1)) * (EX_THREADS / 32);
     const u32 uo_l = (lane < EX_RPW && rl < n) ? (u32)(__ldg(cum + R0 + rl) - cum0 - (u64)REC_W * rl) : 0u;
+    // the record's window-local event base ((global record - window start) << 5), one per lane as well
+    const u32 eb_l = (lane < EX_RPW && rl < n) ? (u32)(((gidx ? (u64)__ldg(gidx + R0 + rl) : R0 + rl) - G0) << 5) : 0u;
     mbar_wait(&bar[st], phase);
-#pragma unroll
-    for (int j = 0; j < EX_RPW; ++j) {
+    // lane j < EX_RPW classifies record wid + 8 j from its header: the warp then walks only the records
+    // that carry addresses (LD / ST / ATOM, and ACQ / REL / AR for the alignment check); control records
+    // (IF / ELSE / FI / BAR / FENCE: about half of a divergent program's records) cost one ballot
+    u32 mem = 0;
+    {
+      const u32 jr = (u32)wid + (u32)(lane & (EX_RPW - 1)) * (EX_THREADS / 32);
+      const bool have = lane < EX_RPW && cbase + jr < n;
+      const u32 hz = have ? reinterpret_cast<const uint4*>(&buf[st * EX_REC + jr])->z : 0xFFu;
+      mem = __ballot_sync(0xFFFFFFFFu, have && (hz & 0xFFu) <= BC_OP_AR_GLB);
+    }
+    while (mem) {
+      const int j = __ffs(mem) - 1;
+      mem &= mem - 1;
       const u32 jr = (u32)wid + (u32)j * (EX_THREADS / 32);  // record within the chunk
-      const u64 r = cbase + jr;
       const u32 uoj = __shfl_sync(0xFFFFFFFFu, uo_l, j);
-      if (r >= n) break;
+      const u32 evb = __shfl_sync(0xFFFFFFFFu, eb_l, j);
       const bc_record* sr = &buf[st * EX_REC + jr];
       const uint4 hv = *reinterpret_cast<const uint4*>(sr);
       const u32 hwarp = hv.x, hmask = hv.y, op = hv.z & 0xFFu, space = (hv.z >> 8) & 0xFFu,
                 sl = (hv.z >> 16) & 0xFFu, fl = (hv.z >> 24) & 0xFFu;
-      if (!(op <= BC_OP_AR_GLB && ((hmask >> lane) & 1u) && sl <= 4 && space <= 1 && hwarp < g.n_warps)) continue;
+      if (!(((hmask >> lane) & 1u) && sl <= 4 && space <= 1 && hwarp < g.n_warps)) continue;
       const u64 a = sr->addr[lane];
       const u64 size = 1ull << sl;
       if (a & (size - 1)) bad = true;  // natural alignment
@@ -476,9 +492,8 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
           ovf = true;
         }
       }
-      const u64 o = (u64)uoj + (u64)__popc(hmask & lt) * nk;
-      // window-local event id: (global record - window start) << 5 | lane
-      const u32 ev = (u32)(((gidx ? (u64)__ldg(gidx + R0 + r) : R0 + r) - G0) << 5) | (u32)lane;
+      const u32 o = uoj + (u32)__popc(hmask & lt) * nk;  // window slots < 2^30
+      const u32 ev = evb | (u32)lane;                    // window-local event id
       if (nk == 1 && g.world == 1) {  // one granule, one shard: the common case
         okeys[o] = key0 != KEY_DROP ? ((key0 << 2) | opc) : KEY_DROP;
         oevs[o] = ev;
