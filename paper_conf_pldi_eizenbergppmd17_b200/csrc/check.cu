@@ -286,87 +286,80 @@ __device__ __forceinline__ bool carried_infl(const CheckArgs& a, const Carry& C,
   return !hbq(a.k, a.c, C.rr, C.rwl & 31u, C.rwl >> 5, a.R0 + (ev_s >> 5), ev_s & 31u, s_s);
 }
 
-// ---------------------------------------------------------------------- K7a: range tail summaries
-// Summary (Sum) of warp range w: the tail granule run's last writer and first inflation after it,
-// found by walking back from the range end (usually a few items: a writer or the granule's start
-// ends the walk; never past the range start).  The exclusive combine of these summaries
-// (k_range_scan) is the automaton state entering every range: no warp ever waits for another.
-__global__ void __launch_bounds__(256) k_range_tail(CheckArgs a, u32 nw, Sum* __restrict__ out) {
-  const u32 w = (u32)(((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+// ---------------------------------------------------------------------- tail summary of an item range
+// Summary (Sum) of the items [beg, end): the tail granule run's last writer and first inflation after
+// it, found by walking back from the end (usually a few items: a writer or the granule's start ends
+// the walk; never past beg).  Warp-cooperative; uniform result.
+__device__ Sum tail_sum(const CheckArgs& a, u64 beg, u64 end) {
   const int lane = threadIdx.x & 31;
-  if (w >= nw) return;  // warp-uniform
   const HbCtx& c = a.c;
-  u64 beg, end;
-  warp_range(*a.n_dev, w, nw, beg, end);
   Sum s = sum_ident();
-  if (beg < end) {
-    const u32 k0 = __ldg(a.keys + end - 1) >> 2;
-    s.fk = __ldg(a.keys + beg) >> 2;
-    s.lk = k0;
-    u32 bits = s.fk == k0 ? SB_ONE : 0u, lw = 0, fi = NONE;
-    u64 hi = end - 1;
-    for (;;) {
-      const u64 lo = hi >= beg + 31 ? hi - 31 : beg;
-      const u64 i = lo + lane;
-      const bool in = i <= hi;
-      const u32 kx = in ? __ldg(a.keys + i) : NONE, ev = in ? __ldg(a.evs + i) : 0u;
-      const bool inkey = in && (kx >> 2) == k0;
-      const u32 W = __ballot_sync(0xFFFFFFFFu, inkey && (kx & 3u) != IOP_LD);
-      const u32 B = __ballot_sync(0xFFFFFFFFu, in && !inkey);  // other granules (below: keys sorted)
-      const int hw = W ? (int)hibit(W) : -1, hbk = B ? (int)hibit(B) : -1;
-      const int bnd = hw > hbk ? hw : hbk;  // the read run is (bnd, top]
-      u32 qkx = __shfl_up_sync(0xFFFFFFFFu, kx, 1), qev = __shfl_up_sync(0xFFFFFFFFu, ev, 1);
-      if (lane == 0) {
-        qkx = lo > 0 ? __ldg(a.keys + lo - 1) : NONE;
-        qev = lo > 0 ? __ldg(a.evs + lo - 1) : 0u;
-      }
-      const bool inrun = in && lane > bnd;
-      bool e = false;
-      if (inrun && qkx != NONE && (qkx >> 2) == k0 && (qkx & 3u) == IOP_LD) {
-        const Snap s2 = load_snap(c.snap, a.R0 + (ev >> 5));
-        const u32 qw = __ldg(&c.snap[a.R0 + (qev >> 5)].x);
-        e = !hbq(a.k, c, a.R0 + (qev >> 5), qev & 31u, qw, a.R0 + (ev >> 5), ev & 31u, s2);
-      }
-      const u32 I = __ballot_sync(0xFFFFFFFFu, e);
-      if (I) fi = (u32)(lo + __ffs(I) - 1);  // earlier rounds hold later items
-      bool seg_at = false;                   // the run starts at its granule's first item s
-      u64 sidx = 0;
-      bool done = false;
-      if (bnd >= 0) {
-        if (hw >= 0 && hw > hbk) {
-          lw = (u32)(lo + hw) + 1u;
-          bits |= SB_W;
-        } else {
-          seg_at = true;
-          sidx = lo + hbk + 1;
-        }
-        done = true;
-      } else if (lo == beg) {
-        seg_at = beg == 0 || (__ldg(a.keys + beg - 1) >> 2) != k0;
-        sidx = beg;
-        done = true;
-      }
-      if (done) {
-        if (seg_at && a.sh_in) {
-          const Carry C = load_carry(a.sh_in, k0);
-          const u32 evs_ = __ldg(a.evs + sidx);
-          const bool ci = carried_infl(a, C, evs_, load_snap(c.snap, a.R0 + (evs_ >> 5)));
-          if (ci) bits |= SB_CI;
-        }
-        break;
-      }
-      hi = lo - 1;
+  if (beg >= end) return s;
+  const u32 k0 = __ldg(a.keys + end - 1) >> 2;
+  s.fk = __ldg(a.keys + beg) >> 2;
+  s.lk = k0;
+  u32 bits = s.fk == k0 ? SB_ONE : 0u, lw = 0, fi = NONE;
+  u64 hi = end - 1;
+  for (;;) {
+    const u64 lo = hi >= beg + 31 ? hi - 31 : beg;
+    const u64 i = lo + lane;
+    const bool in = i <= hi;
+    const u32 kx = in ? __ldg(a.keys + i) : NONE, ev = in ? __ldg(a.evs + i) : 0u;
+    const bool inkey = in && (kx >> 2) == k0;
+    const u32 W = __ballot_sync(0xFFFFFFFFu, inkey && (kx & 3u) != IOP_LD);
+    const u32 B = __ballot_sync(0xFFFFFFFFu, in && !inkey);  // other granules (below: keys sorted)
+    const int hw = W ? (int)hibit(W) : -1, hbk = B ? (int)hibit(B) : -1;
+    const int bnd = hw > hbk ? hw : hbk;  // the read run is (bnd, top]
+    u32 qkx = __shfl_up_sync(0xFFFFFFFFu, kx, 1), qev = __shfl_up_sync(0xFFFFFFFFu, ev, 1);
+    if (lane == 0) {
+      qkx = lo > 0 ? __ldg(a.keys + lo - 1) : NONE;
+      qev = lo > 0 ? __ldg(a.evs + lo - 1) : 0u;
     }
-    s.lw = lw;
-    s.fi = fi;
-    s.bits = bits;
+    const bool inrun = in && lane > bnd;
+    bool e = false;
+    if (inrun && qkx != NONE && (qkx >> 2) == k0 && (qkx & 3u) == IOP_LD) {
+      const Snap s2 = load_snap(c.snap, a.R0 + (ev >> 5));
+      const u32 qw = __ldg(&c.snap[a.R0 + (qev >> 5)].x);
+      e = !hbq(a.k, c, a.R0 + (qev >> 5), qev & 31u, qw, a.R0 + (ev >> 5), ev & 31u, s2);
+    }
+    const u32 I = __ballot_sync(0xFFFFFFFFu, e);
+    if (I) fi = (u32)(lo + __ffs(I) - 1);  // earlier rounds hold later items
+    bool seg_at = false;                   // the run starts at its granule's first item s
+    u64 sidx = 0;
+    bool done = false;
+    if (bnd >= 0) {
+      if (hw >= 0 && hw > hbk) {
+        lw = (u32)(lo + hw) + 1u;
+        bits |= SB_W;
+      } else {
+        seg_at = true;
+        sidx = lo + hbk + 1;
+      }
+      done = true;
+    } else if (lo == beg) {
+      seg_at = beg == 0 || (__ldg(a.keys + beg - 1) >> 2) != k0;
+      sidx = beg;
+      done = true;
+    }
+    if (done) {
+      if (seg_at && a.sh_in) {
+        const Carry C = load_carry(a.sh_in, k0);
+        const u32 evs_ = __ldg(a.evs + sidx);
+        if (carried_infl(a, C, evs_, load_snap(c.snap, a.R0 + (evs_ >> 5)))) bits |= SB_CI;
+      }
+      break;
+    }
+    hi = lo - 1;
   }
-  if (lane == 0) out[w] = s;
+  s.lw = lw;
+  s.fi = fi;
+  s.bits = bits;
+  return s;
 }
 
-// ---------------------------------------------------------------------- K7s: exclusive scan of the range sums
-// One CTA: thread t combines ranges [t*P, t*P + P) sequentially, a Hillis-Steele scan over the
-// 1024 thread totals, then every thread writes the exclusive prefix of its ranges.
+// ---------------------------------------------------------------------- K7s: exclusive scan of summaries
+// One CTA: thread t combines entries [t*P, t*P + P) sequentially, a Hillis-Steele scan over the
+// 1024 thread totals, then every thread writes the exclusive prefix of its entries.
 __global__ void __launch_bounds__(1024) k_range_scan(const Sum* __restrict__ in, u32 nw, Sum* __restrict__ out) {
   __shared__ Sum sh[2][1024];
   const u32 t = threadIdx.x;
@@ -449,101 +442,144 @@ __device__ __forceinline__ void kt_stage(const CheckArgs& a, u64 bb, u32 nb, u32
   cp_async_commit();
 }
 
-__global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u32 nw) {
+// ---------------------------------------------------------------------- K7a: block summaries
+// One warp per block of KT_BLK sorted items (a CTA = KT_SWARPS consecutive blocks).  From the key
+// words alone (vector loads) it counts the granules starting in the block and decides whether any
+// item makes a check: with one window and nothing carried, an item alone in its granule or an atomic
+// between atomics (its W check is elided, and no read follows it) checks nothing.  Such a
+// block only advances the automaton state: its summary comes from the keys.  Any other block is
+// summarised by a bounded tail walk and listed for K7b.  The CTA's combined summary goes to ctot.
+constexpr int KT_SWARPS = 8;
+__global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_sum(CheckArgs a, u32 nblk, Sum* __restrict__ sums,
+                                                            Sum* __restrict__ ctot, u32* __restrict__ wl,
+                                                            u32* __restrict__ wl_cnt, u64* __restrict__ seg_cnt) {
+  __shared__ Sum s_sum[KT_SWARPS];
+  __shared__ u32 s_segs[KT_SWARPS];
+  const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const u32 blk = blockIdx.x * KT_SWARPS + wi;
+  const u64 n = *a.n_dev;
+  const bool fast_ok = a.sh_in == nullptr && a.sh_out == nullptr;
+  Sum bs = sum_ident();
+  u32 fsegs = 0;
+  const u64 bb = (u64)blk * KT_BLK;
+  if (blk < nblk && bb < n) {  // warp-uniform
+    const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
+    const u32 l0 = lane * KT_IPL;
+    const u32 cntf = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
+    u32 kr[KT_IPL];
+    if (cntf == (u32)KT_IPL) {
+      const uint4* kv = reinterpret_cast<const uint4*>(a.keys + bb + l0);  // 64-B aligned: bb, l0 are x16
+#pragma unroll
+      for (int q = 0; q < KT_IPL / 4; ++q) {
+        const uint4 v = __ldg(kv + q);
+        kr[4 * q] = v.x;
+        kr[4 * q + 1] = v.y;
+        kr[4 * q + 2] = v.z;
+        kr[4 * q + 3] = v.w;
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < KT_IPL; ++j) kr[j] = (u32)j < cntf ? __ldg(a.keys + bb + l0 + j) : NONE;
+    }
+    const u32 kprev = (lane == 0 && bb > 0) ? __ldg(a.keys + bb - 1) : NONE;
+    const u32 knext = (lane == 31 && bb + nb < n) ? __ldg(a.keys + bb + nb) : NONE;
+    u32 kp = __shfl_up_sync(0xFFFFFFFFu, kr[KT_IPL - 1], 1);
+    u32 knx = __shfl_down_sync(0xFFFFFFFFu, kr[0], 1);
+    const u32 kn_blk = __shfl_sync(0xFFFFFFFFu, knext, 31);
+    if (lane == 0) kp = kprev;
+    if (lane == 31 || l0 + KT_IPL >= nb) knx = kn_blk;
+    bool triv = true;
+    u32 tlw = 0, kl = kp;
+    bool kc = false;
+#pragma unroll
+    for (int j = 0; j < KT_IPL; ++j) {
+      if ((u32)j < cntf) {
+        const u32 k = kr[j], kpv = kl, knv = (u32)j + 1 < cntf ? kr[j + 1] : knx;
+        const u32 key = k >> 2;
+        const bool sp = kpv != NONE && (kpv >> 2) == key, sn = knv != NONE && (knv >> 2) == key;
+        const bool atm_only =
+            (k & 3u) == IOP_ATOM && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
+        triv &= (!sp && !sn) || atm_only;
+        if (!sp) {
+          ++fsegs;
+          kc |= j > 0;
+          tlw = 0;
+        }
+        if ((k & 3u) != IOP_LD) tlw = (u32)bb + l0 + (u32)j + 1u;
+        kl = k;
+      }
+    }
+    if (fast_ok && __all_sync(0xFFFFFFFFu, triv)) {
+      // chunk summaries (no read has a same-granule read before it: no READINFLATE flags) and their
+      // warp combine = the block summary
+      Sum sm = sum_ident();
+      if (cntf) {
+        sm.fk = kr[0] >> 2;
+        sm.lk = kl >> 2;
+        sm.lw = tlw;
+        sm.fi = NONE;
+        sm.bits = (kc ? 0u : SB_ONE) | (tlw ? SB_W : 0u);
+      }
+      Sum incl = sm;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const Sum up = shfl_up_sum(incl, o);
+        if ((int)lane >= o) incl = combine(up, incl);
+      }
+      bs = shfl_sum(incl, 31);
+    } else {
+      bs = tail_sum(a, bb, bb + nb);
+      if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = blk;
+    }
+  }
+  fsegs = __reduce_add_sync(0xFFFFFFFFu, fsegs);
+  if (lane == 0) {
+    s_sum[wi] = bs;
+    s_segs[wi] = fsegs;
+    if (blk < nblk) sums[blk] = bs;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    Sum t = sum_ident();
+    u32 sg = 0;
+    for (int q = 0; q < KT_SWARPS; ++q) {
+      t = combine(t, s_sum[q]);
+      sg += s_segs[q];
+    }
+    ctot[blockIdx.x] = t;
+    if (sg) atomicAdd((unsigned long long*)seg_cnt, (unsigned long long)sg);
+  }
+}
+
+// ---------------------------------------------------------------------- K7b: the listed blocks
+__global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, const u32* __restrict__ wl,
+                                                                 const u32* __restrict__ wl_cnt,
+                                                                 const Sum* __restrict__ sums,
+                                                                 const Sum* __restrict__ cpre) {
   extern __shared__ __align__(16) unsigned char kt_smem[];
   const int wi = threadIdx.x >> 5;
   uint4* sS = reinterpret_cast<uint4*>(kt_smem + (size_t)wi * KT_WARP_BYTES);
   u32* const sK = reinterpret_cast<u32*>(sS + KT_PITCH);
   u32* const sE = sK + KT_PITCH;
   const u64 n = *a.n_dev;
-  const u32 w = blockIdx.x * KT_WARPS + wi;
+  const u32 w = blockIdx.x * KT_WARPS + wi, nw = gridDim.x * KT_WARPS;
   const u32 lane = threadIdx.x & 31;
   const HbCtx& c = a.c;
   const K7Ctx* const kx = a.k;
   const u32 R0 = a.R0;
   const bool shadow = a.sh_in != nullptr;
-  u64 beg, end;
-  warp_range(n, w, nw, beg, end);
-
-  // ---- state entering the range
-  Sum carry = beg < end ? a.rin[w] : sum_ident();
-  u32 pkx = NONE;  // key word of the item before the block (its event: evs[bb - 1], loaded when needed)
-  if (beg > 0 && beg < end) pkx = __ldg(a.keys + beg - 1);
-
+  const u32 n_tasks = *wl_cnt;
   u32 segs = 0;
   const u32 l0 = lane * KT_IPL;
-  // fast path (one window, nothing carried in or out): a block none of whose items makes a check --
-  // every item alone in its granule, or an atomic between atomics (its W check is elided, P:L661-670,
-  // and no read follows it) -- only advances the automaton state: summarised from its key words
-  const bool fast_ok = !shadow && a.sh_out == nullptr;
-  for (u64 bb = beg; bb < end; bb += KT_BLK) {
-    const u32 nb = (u32)(end - bb < (u64)KT_BLK ? end - bb : (u64)KT_BLK);
+  for (u32 task = w; task < n_tasks; task += nw) {
+    const u32 blkid = wl[task];
+    const u64 bb = (u64)blkid * KT_BLK;
+    const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
+    // state entering the block: the CTA-group prefix (K7s), then the group's earlier blocks
+    Sum carry = cpre[blkid / KT_SWARPS];
+    for (u32 q = blkid & ~(u32)(KT_SWARPS - 1); q < blkid; ++q) carry = combine(carry, sums[q]);
+    const u32 pkx = bb > 0 ? __ldg(a.keys + bb - 1) : NONE;  // the item before the block
     const u32 knext = bb + nb < n ? __ldg(a.keys + bb + nb) : NONE;  // first item after the block
-    if (fast_ok) {
-      u32 kr[KT_IPL];
-      const u32 cntf = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
-      if (cntf == (u32)KT_IPL) {
-        const uint4* kv = reinterpret_cast<const uint4*>(a.keys + bb + l0);  // 64-B aligned: bb, l0 are x16
-#pragma unroll
-        for (int q = 0; q < KT_IPL / 4; ++q) {
-          const uint4 v = __ldg(kv + q);
-          kr[4 * q] = v.x;
-          kr[4 * q + 1] = v.y;
-          kr[4 * q + 2] = v.z;
-          kr[4 * q + 3] = v.w;
-        }
-      } else {
-#pragma unroll
-        for (int j = 0; j < KT_IPL; ++j) kr[j] = (u32)j < cntf ? __ldg(a.keys + bb + l0 + j) : NONE;
-      }
-      u32 kp = __shfl_up_sync(0xFFFFFFFFu, kr[KT_IPL - 1], 1);
-      u32 knx = __shfl_down_sync(0xFFFFFFFFu, kr[0], 1);
-      if (lane == 0) kp = pkx;
-      if (lane == 31 || l0 + KT_IPL >= nb) knx = knext;
-      bool triv = true;
-      u32 fsegs = 0, tlw = 0, kl = kp;
-      bool kc = false;
-#pragma unroll
-      for (int j = 0; j < KT_IPL; ++j) {
-        if ((u32)j < cntf) {
-          const u32 k = kr[j], kpv = kl, knv = (u32)j + 1 < cntf ? kr[j + 1] : knx;
-          const u32 key = k >> 2;
-          const bool sp = kpv != NONE && (kpv >> 2) == key, sn = knv != NONE && (knv >> 2) == key;
-          const bool atm_only =
-              (k & 3u) == IOP_ATOM && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
-          triv &= (!sp && !sn) || atm_only;
-          if (!sp) {
-            ++fsegs;
-            kc |= j > 0;
-            tlw = 0;
-          }
-          if ((k & 3u) != IOP_LD) tlw = (u32)bb + l0 + (u32)j + 1u;
-          kl = k;
-        }
-      }
-      if (__all_sync(0xFFFFFFFFu, triv)) {
-        segs += fsegs;
-        // chunk summaries (no read has a same-granule read before it: no READINFLATE flags) and their
-        // warp combine = the block summary
-        Sum sm = sum_ident();
-        if (cntf) {
-          sm.fk = kr[0] >> 2;
-          sm.lk = kl >> 2;
-          sm.lw = tlw;
-          sm.fi = NONE;
-          sm.bits = (kc ? 0u : SB_ONE) | (tlw ? SB_W : 0u);
-        }
-        Sum incl = sm;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const Sum up = shfl_up_sum(incl, o);
-          if ((int)lane >= o) incl = combine(up, incl);
-        }
-        carry = combine(carry, shfl_sum(incl, 31));
-        pkx = __shfl_sync(0xFFFFFFFFu, kl, (nb - 1) / (u32)KT_IPL);  // the block's last item
-        continue;
-      }
-    }
     kt_stage(a, bb, nb, sK, sE, lane);
     cp_async_wait0();
     __syncwarp();
@@ -590,7 +626,6 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
         const u32 gi = gbb + li;
         const bool same = pk != NONE && (pk >> 2) == (k >> 2);
         if (!same) {
-          ++segs;
           kc |= j > 0;
           tlw = 0;
           tfi = NONE;
@@ -757,13 +792,10 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, u3
       }
     }
 
-    // ---- block carry
-    carry = combine(carry, blk);
-    pkx = sK[tpad(nb - 1)];
+    (void)blk;
     __syncwarp();
   }
-  segs = __reduce_add_sync(0xFFFFFFFFu, segs);
-  if (lane == 0 && segs) atomicAdd((unsigned long long*)kx->seg_cnt, (unsigned long long)segs);
+  (void)segs;
 }
 
 // Statistics only (bc_config.flags & BC_F_COUNT_GATHERS): the number of items whose record clock
@@ -808,19 +840,26 @@ static int k7_grid(int dev) {
   return grid[dev];
 }
 
-size_t check_status_bytes(u64) { return (size_t)(148 * 64 * 2 + 64) * sizeof(Sum) + sizeof(K7Ctx) + 256; }
+// status scratch: [K7Ctx][Sum sums[nblk]][Sum ctot[nct]][Sum cpre[nct]][u32 wl[nblk]][u32 wl_cnt]
+size_t check_status_bytes(u64 n) {
+  const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1, nct = nblk / KT_SWARPS + 2;
+  return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (nblk + 2 * nct) * sizeof(Sum) + (nblk + 64) * sizeof(u32) + 512;
+}
 
 void launch_check(const CheckLaunch& L, cudaStream_t st) {
   if (L.n_max == 0) return;
   int dev = 0;
   cudaGetDevice(&dev);
   const int grid = k7_grid(dev);
-  const u32 nw = (u32)grid * KT_WARPS;
-  // status scratch: [K7Ctx][Sum tail[nw]][Sum rin[nw]]
+  const u64 nblk = (L.n_max + KT_BLK - 1) / KT_BLK;
+  const u64 nct = (nblk + KT_SWARPS - 1) / KT_SWARPS;
   char* base = (char*)L.status;
   K7Ctx* kdev = reinterpret_cast<K7Ctx*>(base);
-  Sum* tail = reinterpret_cast<Sum*>(base + ((sizeof(K7Ctx) + 255) & ~(size_t)255));
-  Sum* rin = tail + nw;
+  Sum* sums = reinterpret_cast<Sum*>(base + ((sizeof(K7Ctx) + 255) & ~(size_t)255));
+  Sum* ctot = sums + nblk + 1;
+  Sum* cpre = ctot + nct + 1;
+  u32* wl = reinterpret_cast<u32*>(cpre + nct + 1);
+  u32* wl_cnt = wl + nblk + 1;
   K7Ctx k{};
   k.c = L.c;
   k.keys = L.keys;
@@ -838,6 +877,7 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   k.values = L.values;
   k.n_dev = L.n_dev;
   cudaMemcpyAsync(kdev, &k, sizeof(K7Ctx), cudaMemcpyHostToDevice, st);
+  cudaMemsetAsync(wl_cnt, 0, sizeof(u32), st);
   CheckArgs a;
   a.k = kdev;
   a.c = L.c;
@@ -847,12 +887,12 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   a.R0 = L.R0;
   a.sh_in = L.sh_in;
   a.sh_out = L.sh_out;
-  a.rin = rin;
+  a.rin = nullptr;
   a.no_sv = L.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   a.values = L.values;
-  k_range_tail<<<(nw * 32 + 255) / 256, 256, 0, st>>>(a, nw, tail);
-  k_range_scan<<<1, 1024, 0, st>>>(tail, nw, rin);
-  k_check_tile<<<grid, KT_WARPS * 32, (size_t)KT_WARPS * KT_WARP_BYTES, st>>>(a, nw);
+  k_blk_sum<<<(unsigned)nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, sums, ctot, wl, wl_cnt, L.seg_cnt);
+  k_range_scan<<<1, 1024, 0, st>>>(ctot, (u32)nct, cpre);
+  k_check_tile<<<grid, KT_WARPS * 32, (size_t)KT_WARPS * KT_WARP_BYTES, st>>>(a, wl, wl_cnt, sums, cpre);
   g_launches += 3;
 }
 
