@@ -219,7 +219,7 @@ void bc_destroy(bc_ctx* c) {
   c->da.free(c->rbuf, c->rbuf_cap * sizeof(uint4));
   c->da.free(c->pool, c->pool_cap * sizeof(uint2));
   c->da.free(c->gidx_owned, c->gidx_cap);
-  for (int i = 0; i < 5; ++i) c->da.free(c->xbuf[i], c->xcap[i]);
+  for (int i = 0; i < 6; ++i) c->da.free(c->xbuf[i], c->xcap[i]);
   c->arena.free_all();
   delete c->comm;
   if (c->hcnt) cudaFreeHost(c->hcnt);

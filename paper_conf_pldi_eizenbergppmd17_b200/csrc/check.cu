@@ -360,32 +360,65 @@ __device__ Sum tail_sum(const CheckArgs& a, u64 beg, u64 end) {
 // ---------------------------------------------------------------------- K7s: exclusive scan of summaries
 // One CTA: thread t combines entries [t*P, t*P + P) sequentially, a Hillis-Steele scan over the
 // 1024 thread totals, then every thread writes the exclusive prefix of its entries.
-__global__ void __launch_bounds__(1024) k_range_scan(const Sum* __restrict__ in, u32 nw, Sum* __restrict__ out) {
-  __shared__ Sum sh[2][1024];
-  const u32 t = threadIdx.x;
-  const u32 P = (nw + 1023) / 1024;
-  Sum tot = sum_ident();
-  for (u32 q = 0; q < P; ++q) {
-    const u32 i = t * P + q;
-    if (i < nw) tot = combine(tot, in[i]);
-  }
-  int cur = 0;
-  sh[0][t] = tot;
-  __syncthreads();
-  for (u32 o = 1; o < 1024; o <<= 1) {
-    Sum v = sh[cur][t];
-    if (t >= o) v = combine(sh[cur][t - o], v);
-    sh[cur ^ 1][t] = v;
-    cur ^= 1;
+__global__ void __launch_bounds__(1024) k_range_scan(const Sum* __restrict__ in, u32 nw, Sum* __restrict__ out,
+                                                     const u32* __restrict__ segs, u64* __restrict__ seg_cnt) {
+  // chunks of 2048 entries: coalesced loads into shared memory, thread t combines entries 2t, 2t+1,
+  // warp shuffle scans of the thread totals and of the 32 warp totals, a running carry across chunks
+  constexpr int PER = 2;
+  __shared__ Sum sh[1024 * PER];
+  __shared__ Sum s_w[32];
+  __shared__ Sum s_carry;
+  const u32 t = threadIdx.x, lane = t & 31, wi = t >> 5;
+  u64 sg = 0;
+  if (t == 0) s_carry = sum_ident();
+  for (u32 c0 = 0; c0 < nw; c0 += 1024 * PER) {
+    for (u32 q = t; q < 1024 * PER; q += 1024) {
+      sh[q] = c0 + q < nw ? in[c0 + q] : sum_ident();
+      if (segs && c0 + q < nw) sg += segs[c0 + q];
+    }
+    __syncthreads();
+    Sum tot = sum_ident();
+#pragma unroll
+    for (int q = 0; q < PER; ++q) tot = combine(tot, sh[t * PER + q]);
+    Sum incl = tot;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const Sum up = shfl_up_sum(incl, o);
+      if ((int)lane >= o) incl = combine(up, incl);
+    }
+    if (lane == 31) s_w[wi] = incl;
+    Sum ex = shfl_up_sum(incl, 1);
+    if (lane == 0) ex = sum_ident();
+    __syncthreads();
+    if (wi == 0) {
+      Sum wv = s_w[lane], wincl = wv;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const Sum up = shfl_up_sum(wincl, o);
+        if ((int)lane >= o) wincl = combine(up, wincl);
+      }
+      Sum wex = shfl_up_sum(wincl, 1);
+      if (lane == 0) wex = sum_ident();
+      s_w[lane] = wex;
+    }
+    __syncthreads();
+    Sum run = combine(s_carry, combine(s_w[wi], ex));
+    const Sum chunk_end = combine(run, tot);
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const Sum v = sh[t * PER + q];
+      sh[t * PER + q] = run;  // exclusive prefix, written back coalesced below
+      run = combine(run, v);
+    }
+    __syncthreads();
+    for (u32 q = t; q < 1024 * PER; q += 1024)
+      if (c0 + q < nw) out[c0 + q] = sh[q];
+    if (t == 1023) s_carry = chunk_end;
     __syncthreads();
   }
-  Sum run = t ? sh[cur][t - 1] : sum_ident();
-  for (u32 q = 0; q < P; ++q) {
-    const u32 i = t * P + q;
-    if (i < nw) {
-      out[i] = run;
-      run = combine(run, in[i]);
-    }
+  if (segs) {
+    sg = __reduce_add_sync(0xFFFFFFFFu, (u32)sg);
+    if (lane == 0 && sg) atomicAdd((unsigned long long*)seg_cnt, (unsigned long long)sg);
   }
 }
 
@@ -449,10 +482,10 @@ __device__ __forceinline__ void kt_stage(const CheckArgs& a, u64 bb, u32 nb, u32
 // between atomics (its W check is elided, and no read follows it) checks nothing.  Such a
 // block only advances the automaton state: its summary comes from the keys.  Any other block is
 // summarised by a bounded tail walk and listed for K7b.  The CTA's combined summary goes to ctot.
-constexpr int KT_SWARPS = 8;
+constexpr int KT_SWARPS = 32;
 __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_sum(CheckArgs a, u32 nblk, Sum* __restrict__ sums,
                                                             Sum* __restrict__ ctot, u32* __restrict__ wl,
-                                                            u32* __restrict__ wl_cnt, u64* __restrict__ seg_cnt) {
+                                                            u32* __restrict__ wl_cnt, u32* __restrict__ csegs) {
   __shared__ Sum s_sum[KT_SWARPS];
   __shared__ u32 s_segs[KT_SWARPS];
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -547,7 +580,7 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_sum(CheckArgs a, u32 nbl
       sg += s_segs[q];
     }
     ctot[blockIdx.x] = t;
-    if (sg) atomicAdd((unsigned long long*)seg_cnt, (unsigned long long)sg);
+    csegs[blockIdx.x] = sg;  // summed by k_range_scan
   }
 }
 
@@ -840,10 +873,11 @@ static int k7_grid(int dev) {
   return grid[dev];
 }
 
-// status scratch: [K7Ctx][Sum sums[nblk]][Sum ctot[nct]][Sum cpre[nct]][u32 wl[nblk]][u32 wl_cnt]
+// status scratch: [K7Ctx][Sum sums[nblk]][Sum ctot[nct]][Sum cpre[nct]][u32 wl[nblk]][u32 wl_cnt][u32 csegs[nct]]
 size_t check_status_bytes(u64 n) {
   const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1, nct = nblk / KT_SWARPS + 2;
-  return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (nblk + 2 * nct) * sizeof(Sum) + (nblk + 64) * sizeof(u32) + 512;
+  return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (nblk + 2 * nct + 4) * sizeof(Sum) +
+         (nblk + nct + 64) * sizeof(u32) + 512;
 }
 
 void launch_check(const CheckLaunch& L, cudaStream_t st) {
@@ -860,6 +894,7 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   Sum* cpre = ctot + nct + 1;
   u32* wl = reinterpret_cast<u32*>(cpre + nct + 1);
   u32* wl_cnt = wl + nblk + 1;
+  u32* csegs = wl_cnt + 1;
   K7Ctx k{};
   k.c = L.c;
   k.keys = L.keys;
@@ -890,8 +925,8 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   a.rin = nullptr;
   a.no_sv = L.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   a.values = L.values;
-  k_blk_sum<<<(unsigned)nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, sums, ctot, wl, wl_cnt, L.seg_cnt);
-  k_range_scan<<<1, 1024, 0, st>>>(ctot, (u32)nct, cpre);
+  k_blk_sum<<<(unsigned)nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, sums, ctot, wl, wl_cnt, csegs);
+  k_range_scan<<<1, 1024, 0, st>>>(ctot, (u32)nct, cpre, csegs, L.seg_cnt);
   k_check_tile<<<grid, KT_WARPS * 32, (size_t)KT_WARPS * KT_WARP_BYTES, st>>>(a, wl, wl_cnt, sums, cpre);
   g_launches += 3;
 }

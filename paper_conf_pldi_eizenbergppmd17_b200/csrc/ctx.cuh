@@ -42,8 +42,8 @@ struct bc_ctx {
   u32* gidx_owned = nullptr;
   size_t gidx_cap = 0;
   u64 n_global = 0;           // records of the whole trace (sharded)
-  void* xbuf[5] = {};         // device exchange buffers (grown on demand)
-  size_t xcap[5] = {};
+  void* xbuf[6] = {};         // device exchange / scratch buffers (grown on demand)
+  size_t xcap[6] = {};
 };
 
 enum { PH_HEADER = 0, PH_PARTITION, PH_REPLAY, PH_SYNC, PH_EXPAND, PH_SORT, PH_CHECK, PH_FINALIZE, PH_N };

@@ -414,7 +414,6 @@ bc_status detect_sharded(bc_ctx* c, Scratch& S) {
   uint4* sh_cur = multi ? S.alloc<uint4>(2 * n_keys) : nullptr;
   uint4* sh_nxt = multi ? S.alloc<uint4>(2 * n_keys) : nullptr;
   bool have_state = false;
-  void* cstatus = S.alloc<char>(check_status_bytes(0));
   const int kbits = bits_for(n_keys ? n_keys - 1 : 0);
   u64* n_send_dev = cnt + C_ITEMS;
   u64 n_r = 0, n_items = 0, pool_used = 0;
@@ -492,7 +491,8 @@ bc_status detect_sharded(bc_ctx* c, Scratch& S) {
     L.sh_in = have_state ? sh_cur : nullptr;
     L.sh_out = sh_out;
     L.values = nullptr;
-    L.status = cstatus;
+    L.status = ctx_buffer(c, 5, check_status_bytes(n_recv));
+    if (!L.status) return fail(c, BC_ERR_OOM, "check scratch");
     WindowOut wo;
     bc_status ws = check_window(c, L, n_recv, cnt, n_r, pool_used, wo);
     if (bc_status a = agree(c, ws, dtmp)) return a;
