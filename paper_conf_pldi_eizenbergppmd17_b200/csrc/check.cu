@@ -25,6 +25,7 @@
 // window extend (a carried read vector counts as already inflated).  Read
 // vectors live in an append-only pool of (record, warp << 5 | lane) entries.  The entries are read
 // from one table and written to another (double buffer), so no lane ever sees a half-updated state.
+#include <algorithm>
 #include <cstdlib>
 #include <cstring>
 
@@ -476,110 +477,156 @@ __device__ __forceinline__ void kt_stage(const CheckArgs& a, u64 bb, u32 nb, u32
 }
 
 // ---------------------------------------------------------------------- K7a: block summaries
-// One warp per block of KT_BLK sorted items (a CTA = KT_SWARPS consecutive blocks).  From the key
-// words alone (vector loads) it counts the granules starting in the block and decides whether any
-// item makes a check: with one window and nothing carried, an item alone in its granule or an atomic
-// between atomics (its W check is elided, and no read follows it) checks nothing.  Such a
-// block only advances the automaton state: its summary comes from the keys.  Any other block is
-// summarised by a bounded tail walk and listed for K7b.  The CTA's combined summary goes to ctot.
-constexpr int KT_SWARPS = 32;
-__global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_sum(CheckArgs a, u32 nblk, Sum* __restrict__ sums,
-                                                            Sum* __restrict__ ctot, u32* __restrict__ wl,
-                                                            u32* __restrict__ wl_cnt, u32* __restrict__ csegs) {
-  __shared__ Sum s_sum[KT_SWARPS];
+// Persistent CTAs, CTA c owning the contiguous blocks [c * G, (c + 1) * G) of KT_BLK sorted items.
+// Phase 1, one warp per block (the next block's key words prefetched while this one is summarised):
+// from the key words alone (vector loads) it counts the granules starting in the block and decides
+// whether any item makes a check -- with one window and nothing carried, an item alone in its granule
+// or an atomic between atomics (its W check is elided, and no read follows it) checks
+// nothing.  Such a block only advances the automaton state: its summary comes from the keys.  Any other
+// block is summarised by a bounded tail walk and listed for K7b.  Phase 2: the CTA scans its blocks'
+// summaries (exclusive prefix within the CTA -> rin) and writes its total (ctot, scanned by K7s).
+constexpr int KT_SWARPS = 8;
+__device__ __forceinline__ void load_keys16(const u32* __restrict__ keys, u64 bb, u32 nb, u32 l0, u32 (&kr)[KT_IPL]) {
+  const u32 cntf = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
+  if (cntf == (u32)KT_IPL) {
+    const uint4* kv = reinterpret_cast<const uint4*>(keys + bb + l0);  // 64-B aligned: bb, l0 are x16
+#pragma unroll
+    for (int q = 0; q < KT_IPL / 4; ++q) {
+      const uint4 v = __ldg(kv + q);
+      kr[4 * q] = v.x;
+      kr[4 * q + 1] = v.y;
+      kr[4 * q + 2] = v.z;
+      kr[4 * q + 3] = v.w;
+    }
+  } else {
+#pragma unroll
+    for (int j = 0; j < KT_IPL; ++j) kr[j] = (u32)j < cntf ? __ldg(keys + bb + l0 + j) : NONE;
+  }
+}
+
+static __device__ __noinline__ Sum tail_sum_nl(const CheckArgs* a, u64 beg, u64 end) { return tail_sum(*a, beg, end); }
+
+__global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
+                                                            Sum* __restrict__ rin, Sum* __restrict__ ctot,
+                                                            u32* __restrict__ wl, u32* __restrict__ wl_cnt,
+                                                            u32* __restrict__ csegs) {
+  __shared__ Sum s_w[KT_SWARPS];
+  __shared__ Sum s_carry;
   __shared__ u32 s_segs[KT_SWARPS];
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const u32 blk = blockIdx.x * KT_SWARPS + wi;
   const u64 n = *a.n_dev;
   const bool fast_ok = a.sh_in == nullptr && a.sh_out == nullptr;
-  Sum bs = sum_ident();
-  u32 fsegs = 0;
-  const u64 bb = (u64)blk * KT_BLK;
-  if (blk < nblk && bb < n) {  // warp-uniform
-    const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
-    const u32 l0 = lane * KT_IPL;
-    const u32 cntf = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
-    u32 kr[KT_IPL];
-    if (cntf == (u32)KT_IPL) {
-      const uint4* kv = reinterpret_cast<const uint4*>(a.keys + bb + l0);  // 64-B aligned: bb, l0 are x16
-#pragma unroll
-      for (int q = 0; q < KT_IPL / 4; ++q) {
-        const uint4 v = __ldg(kv + q);
-        kr[4 * q] = v.x;
-        kr[4 * q + 1] = v.y;
-        kr[4 * q + 2] = v.z;
-        kr[4 * q + 3] = v.w;
-      }
-    } else {
-#pragma unroll
-      for (int j = 0; j < KT_IPL; ++j) kr[j] = (u32)j < cntf ? __ldg(a.keys + bb + l0 + j) : NONE;
+  const u32 b0 = blockIdx.x * G, b1 = min(nblk, b0 + G);
+  const u32 l0 = lane * KT_IPL;
+  u32 segs = 0;
+  // ---- phase 1
+  u32 kr[KT_IPL], kq[KT_IPL];
+  u32 blk = b0 + wi;
+  auto blk_n = [&](u32 b) -> u32 {
+    const u64 x = (u64)b * KT_BLK;
+    return x < n ? (u32)(n - x < (u64)KT_BLK ? n - x : (u64)KT_BLK) : 0u;
+  };
+  if (blk < b1) load_keys16(a.keys, (u64)blk * KT_BLK, blk_n(blk), l0, kr);
+  for (; blk < b1; blk += KT_SWARPS) {
+    const u64 bb = (u64)blk * KT_BLK;
+    const u32 nb = bb < n ? (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK) : 0u;
+    const u32 kprev = (lane == 0 && bb > 0 && nb) ? __ldg(a.keys + bb - 1) : NONE;
+    const u32 knext = (lane == 31 && nb && bb + nb < n) ? __ldg(a.keys + bb + nb) : NONE;
+    const u32 nxt = blk + KT_SWARPS;
+    if (nxt < b1) {  // prefetch the next block's keys
+      const u64 b2 = (u64)nxt * KT_BLK;
+      load_keys16(a.keys, b2, blk_n(nxt), l0, kq);
     }
-    const u32 kprev = (lane == 0 && bb > 0) ? __ldg(a.keys + bb - 1) : NONE;
-    const u32 knext = (lane == 31 && bb + nb < n) ? __ldg(a.keys + bb + nb) : NONE;
-    u32 kp = __shfl_up_sync(0xFFFFFFFFu, kr[KT_IPL - 1], 1);
-    u32 knx = __shfl_down_sync(0xFFFFFFFFu, kr[0], 1);
-    const u32 kn_blk = __shfl_sync(0xFFFFFFFFu, knext, 31);
-    if (lane == 0) kp = kprev;
-    if (lane == 31 || l0 + KT_IPL >= nb) knx = kn_blk;
-    bool triv = true;
-    u32 tlw = 0, kl = kp;
-    bool kc = false;
+    Sum bs = sum_ident();
+    if (nb) {
+      const u32 cntf = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
+      u32 kp = __shfl_up_sync(0xFFFFFFFFu, kr[KT_IPL - 1], 1);
+      u32 knx = __shfl_down_sync(0xFFFFFFFFu, kr[0], 1);
+      const u32 kn_blk = __shfl_sync(0xFFFFFFFFu, knext, 31);
+      if (lane == 0) kp = kprev;
+      if (lane == 31 || l0 + KT_IPL >= nb) knx = kn_blk;
+      bool triv = true;
+      u32 tlw = 0, kl = kp, fsegs = 0;
+      bool kc = false;
 #pragma unroll
-    for (int j = 0; j < KT_IPL; ++j) {
-      if ((u32)j < cntf) {
-        const u32 k = kr[j], kpv = kl, knv = (u32)j + 1 < cntf ? kr[j + 1] : knx;
-        const u32 key = k >> 2;
-        const bool sp = kpv != NONE && (kpv >> 2) == key, sn = knv != NONE && (knv >> 2) == key;
-        const bool atm_only =
-            (k & 3u) == IOP_ATOM && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
-        triv &= (!sp && !sn) || atm_only;
-        if (!sp) {
-          ++fsegs;
-          kc |= j > 0;
-          tlw = 0;
+      for (int j = 0; j < KT_IPL; ++j) {
+        if ((u32)j < cntf) {
+          const u32 k = kr[j], kpv = kl, knv = (u32)j + 1 < cntf ? kr[j + 1] : knx;
+          const u32 key = k >> 2;
+          const bool sp = kpv != NONE && (kpv >> 2) == key, sn = knv != NONE && (knv >> 2) == key;
+          const bool atm_only =
+              (k & 3u) == IOP_ATOM && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
+          triv &= (!sp && !sn) || atm_only;
+          if (!sp) {
+            ++fsegs;
+            kc |= j > 0;
+            tlw = 0;
+          }
+          if ((k & 3u) != IOP_LD) tlw = (u32)bb + l0 + (u32)j + 1u;
+          kl = k;
         }
-        if ((k & 3u) != IOP_LD) tlw = (u32)bb + l0 + (u32)j + 1u;
-        kl = k;
       }
-    }
-    if (fast_ok && __all_sync(0xFFFFFFFFu, triv)) {
-      // chunk summaries (no read has a same-granule read before it: no READINFLATE flags) and their
-      // warp combine = the block summary
-      Sum sm = sum_ident();
-      if (cntf) {
-        sm.fk = kr[0] >> 2;
-        sm.lk = kl >> 2;
-        sm.lw = tlw;
-        sm.fi = NONE;
-        sm.bits = (kc ? 0u : SB_ONE) | (tlw ? SB_W : 0u);
-      }
-      Sum incl = sm;
+      segs += fsegs;
+      if (fast_ok && __all_sync(0xFFFFFFFFu, triv)) {
+        // chunk summaries (no read has a same-granule read before it: no READINFLATE flags) and their
+        // warp combine = the block summary
+        Sum sm = sum_ident();
+        if (cntf) {
+          sm.fk = kr[0] >> 2;
+          sm.lk = kl >> 2;
+          sm.lw = tlw;
+          sm.fi = NONE;
+          sm.bits = (kc ? 0u : SB_ONE) | (tlw ? SB_W : 0u);
+        }
+        Sum incl = sm;
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const Sum up = shfl_up_sum(incl, o);
-        if ((int)lane >= o) incl = combine(up, incl);
+        for (int o = 1; o < 32; o <<= 1) {
+          const Sum up = shfl_up_sum(incl, o);
+          if ((int)lane >= o) incl = combine(up, incl);
+        }
+        bs = shfl_sum(incl, 31);
+      } else {
+        bs = tail_sum_nl(&a, bb, bb + nb);
+        if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = blk;
       }
-      bs = shfl_sum(incl, 31);
-    } else {
-      bs = tail_sum(a, bb, bb + nb);
-      if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = blk;
     }
+    if (lane == 0) sums[blk] = bs;
+#pragma unroll
+    for (int j = 0; j < KT_IPL; ++j) kr[j] = kq[j];
   }
-  fsegs = __reduce_add_sync(0xFFFFFFFFu, fsegs);
-  if (lane == 0) {
-    s_sum[wi] = bs;
-    s_segs[wi] = fsegs;
-    if (blk < nblk) sums[blk] = bs;
-  }
+  segs = __reduce_add_sync(0xFFFFFFFFu, segs);
+  if (lane == 0) s_segs[wi] = segs;
+  if (threadIdx.x == 0) s_carry = sum_ident();
   __syncthreads();
-  if (threadIdx.x == 0) {
-    Sum t = sum_ident();
-    u32 sg = 0;
-    for (int q = 0; q < KT_SWARPS; ++q) {
-      t = combine(t, s_sum[q]);
-      sg += s_segs[q];
+  // ---- phase 2: exclusive prefix of the CTA's block summaries, 256 at a time
+  for (u32 c0 = b0; c0 < b1; c0 += KT_SWARPS * 32) {
+    const u32 i = c0 + threadIdx.x;
+    const Sum v = i < b1 ? sums[i] : sum_ident();
+    Sum incl = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const Sum up = shfl_up_sum(incl, o);
+      if ((int)lane >= o) incl = combine(up, incl);
     }
-    ctot[blockIdx.x] = t;
+    Sum ex = shfl_up_sum(incl, 1);
+    if (lane == 0) ex = sum_ident();
+    if (lane == 31) s_w[wi] = incl;
+    __syncthreads();
+    Sum wpre = s_carry;
+    for (u32 q = 0; q < wi; ++q) wpre = combine(wpre, s_w[q]);
+    if (i < b1) rin[i] = combine(wpre, ex);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      Sum t = s_carry;
+      for (int q = 0; q < KT_SWARPS; ++q) t = combine(t, s_w[q]);
+      s_carry = t;
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    u32 sg = 0;
+    for (int q = 0; q < KT_SWARPS; ++q) sg += s_segs[q];
+    ctot[blockIdx.x] = s_carry;
     csegs[blockIdx.x] = sg;  // summed by k_range_scan
   }
 }
@@ -587,8 +634,8 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_sum(CheckArgs a, u32 nbl
 // ---------------------------------------------------------------------- K7b: the listed blocks
 __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, const u32* __restrict__ wl,
                                                                  const u32* __restrict__ wl_cnt,
-                                                                 const Sum* __restrict__ sums,
-                                                                 const Sum* __restrict__ cpre) {
+                                                                 const Sum* __restrict__ rin,
+                                                                 const Sum* __restrict__ cpre, u32 G) {
   extern __shared__ __align__(16) unsigned char kt_smem[];
   const int wi = threadIdx.x >> 5;
   uint4* sS = reinterpret_cast<uint4*>(kt_smem + (size_t)wi * KT_WARP_BYTES);
@@ -608,9 +655,8 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
     const u32 blkid = wl[task];
     const u64 bb = (u64)blkid * KT_BLK;
     const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
-    // state entering the block: the CTA-group prefix (K7s), then the group's earlier blocks
-    Sum carry = cpre[blkid / KT_SWARPS];
-    for (u32 q = blkid & ~(u32)(KT_SWARPS - 1); q < blkid; ++q) carry = combine(carry, sums[q]);
+    // state entering the block: its K7a CTA's prefix (K7s), then the prefix within that CTA
+    Sum carry = combine(cpre[blkid / G], rin[blkid]);
     const u32 pkx = bb > 0 ? __ldg(a.keys + bb - 1) : NONE;  // the item before the block
     const u32 knext = bb + nb < n ? __ldg(a.keys + bb + nb) : NONE;  // first item after the block
     kt_stage(a, bb, nb, sK, sE, lane);
@@ -873,10 +919,12 @@ static int k7_grid(int dev) {
   return grid[dev];
 }
 
-// status scratch: [K7Ctx][Sum sums[nblk]][Sum ctot[nct]][Sum cpre[nct]][u32 wl[nblk]][u32 wl_cnt][u32 csegs[nct]]
+// status scratch: [K7Ctx][Sum sums[nblk]][Sum rin[nblk]][Sum ctot[nct]][Sum cpre[nct]][u32 wl[nblk]][u32 wl_cnt]
+// [u32 csegs[nct]]
+constexpr u32 K7A_CTAS = 148 * 8;
 size_t check_status_bytes(u64 n) {
-  const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1, nct = nblk / KT_SWARPS + 2;
-  return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (nblk + 2 * nct + 4) * sizeof(Sum) +
+  const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1, nct = K7A_CTAS + 2;
+  return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (2 * nblk + 2 * nct + 4) * sizeof(Sum) +
          (nblk + nct + 64) * sizeof(u32) + 512;
 }
 
@@ -886,11 +934,13 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   cudaGetDevice(&dev);
   const int grid = k7_grid(dev);
   const u64 nblk = (L.n_max + KT_BLK - 1) / KT_BLK;
-  const u64 nct = (nblk + KT_SWARPS - 1) / KT_SWARPS;
+  const u32 G = (u32)std::max<u64>(1, (nblk + K7A_CTAS - 1) / K7A_CTAS);  // blocks per K7a CTA
+  const u32 nct = (u32)((nblk + G - 1) / G);
   char* base = (char*)L.status;
   K7Ctx* kdev = reinterpret_cast<K7Ctx*>(base);
   Sum* sums = reinterpret_cast<Sum*>(base + ((sizeof(K7Ctx) + 255) & ~(size_t)255));
-  Sum* ctot = sums + nblk + 1;
+  Sum* rin = sums + nblk + 1;
+  Sum* ctot = rin + nblk + 1;
   Sum* cpre = ctot + nct + 1;
   u32* wl = reinterpret_cast<u32*>(cpre + nct + 1);
   u32* wl_cnt = wl + nblk + 1;
@@ -925,9 +975,9 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   a.rin = nullptr;
   a.no_sv = L.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   a.values = L.values;
-  k_blk_sum<<<(unsigned)nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, sums, ctot, wl, wl_cnt, csegs);
-  k_range_scan<<<1, 1024, 0, st>>>(ctot, (u32)nct, cpre, csegs, L.seg_cnt);
-  k_check_tile<<<grid, KT_WARPS * 32, (size_t)KT_WARPS * KT_WARP_BYTES, st>>>(a, wl, wl_cnt, sums, cpre);
+  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, rin, ctot, wl, wl_cnt, csegs);
+  k_range_scan<<<1, 1024, 0, st>>>(ctot, nct, cpre, csegs, L.seg_cnt);
+  k_check_tile<<<grid, KT_WARPS * 32, (size_t)KT_WARPS * KT_WARP_BYTES, st>>>(a, wl, wl_cnt, rin, cpre, G);
   g_launches += 3;
 }
 
