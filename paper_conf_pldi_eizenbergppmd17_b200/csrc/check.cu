@@ -506,10 +506,17 @@ __device__ __forceinline__ void load_keys16(const u32* __restrict__ keys, u64 bb
 
 static __device__ __noinline__ Sum tail_sum_nl(const CheckArgs* a, u64 beg, u64 end) { return tail_sum(*a, beg, end); }
 
-__global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
+// key words stream through shared memory: one chunk = KT_SWARPS blocks (+ 4 words on each side for
+// the neighbours of the first / last item), KB_STAGES chunks in flight per CTA (1-D TMA bulk copies)
+constexpr int KB_STAGES = 2;
+constexpr int KB_CHUNK = KT_SWARPS * KT_BLK;     // items per chunk
+constexpr int KB_ROW = KB_CHUNK + 8;             // words per stage
+__global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
                                                             Sum* __restrict__ rin, Sum* __restrict__ ctot,
                                                             u32* __restrict__ wl, u32* __restrict__ wl_cnt,
                                                             u32* __restrict__ csegs) {
+  __shared__ __align__(128) u32 s_keys[KB_STAGES][KB_ROW];
+  __shared__ u64 s_bar[KB_STAGES];
   __shared__ Sum s_w[KT_SWARPS];
   __shared__ Sum s_carry;
   __shared__ u32 s_segs[KT_SWARPS];
@@ -518,31 +525,54 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_sum(CheckArgs a, u32 nbl
   const bool fast_ok = a.sh_in == nullptr && a.sh_out == nullptr;
   const u32 b0 = blockIdx.x * G, b1 = min(nblk, b0 + G);
   const u32 l0 = lane * KT_IPL;
-  u32 segs = 0;
-  // ---- phase 1
-  u32 kr[KT_IPL], kq[KT_IPL];
-  u32 blk = b0 + wi;
-  auto blk_n = [&](u32 b) -> u32 {
-    const u64 x = (u64)b * KT_BLK;
-    return x < n ? (u32)(n - x < (u64)KT_BLK ? n - x : (u64)KT_BLK) : 0u;
+  const u64 i0 = (u64)b0 * KT_BLK, i1 = min(n, (u64)b1 * KT_BLK);  // the CTA's items
+  const u32 n_chunks = i1 > i0 ? (u32)((i1 - i0 + KB_CHUNK - 1) / KB_CHUNK) : 0u;
+  // chunk c covers items [i0 + c * KB_CHUNK, ...); the stage holds words from item (c0 - 4) at index 0
+  auto issue = [&](u32 c, int st) {
+    const u64 c0 = i0 + (u64)c * KB_CHUNK;
+    const u64 lo = c0 >= 4 ? c0 - 4 : 0;                  // 16-B aligned: c0 is a multiple of 512
+    const u64 hi = min(n, c0 + KB_CHUNK + 4);
+    const u32 bytes = (u32)(((hi - lo) + 3) & ~3ull) * 4u;  // whole 16-B units (buffers are padded)
+    mbar_expect_tx(&s_bar[st], bytes);
+    bulk_g2s(&s_keys[st][c0 >= 4 ? 0 : 4], a.keys + lo, bytes, &s_bar[st]);
   };
-  if (blk < b1) load_keys16(a.keys, (u64)blk * KT_BLK, blk_n(blk), l0, kr);
-  for (; blk < b1; blk += KT_SWARPS) {
+  if (threadIdx.x == 0) {
+    for (int q = 0; q < KB_STAGES; ++q) mbar_init(&s_bar[q], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (threadIdx.x == 0)
+    for (int q = 0; q < KB_STAGES; ++q)
+      if ((u32)q < n_chunks) issue(q, q);
+  u32 segs = 0;
+  for (u32 c = 0; c < n_chunks; ++c) {
+    const int st = (int)(c % KB_STAGES);
+    mbar_wait(&s_bar[st], (c / KB_STAGES) & 1u);
+    const u64 c0 = i0 + (u64)c * KB_CHUNK;
+    const u32* sk = &s_keys[st][4];  // sk[j] = key word of item c0 + j (sk[-1]: the item before)
+    const u32 blk = b0 + c * KT_SWARPS + wi;
     const u64 bb = (u64)blk * KT_BLK;
-    const u32 nb = bb < n ? (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK) : 0u;
-    const u32 kprev = (lane == 0 && bb > 0 && nb) ? __ldg(a.keys + bb - 1) : NONE;
-    const u32 knext = (lane == 31 && nb && bb + nb < n) ? __ldg(a.keys + bb + nb) : NONE;
-    const u32 nxt = blk + KT_SWARPS;
-    if (nxt < b1) {  // prefetch the next block's keys
-      const u64 b2 = (u64)nxt * KT_BLK;
-      load_keys16(a.keys, b2, blk_n(nxt), l0, kq);
-    }
+    const u32 nb = (blk < b1 && bb < n) ? (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK) : 0u;
     Sum bs = sum_ident();
     if (nb) {
+      const u32 off = wi * KT_BLK;  // the block's first item in the chunk
       const u32 cntf = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
+      u32 kr[KT_IPL];
+#pragma unroll
+      for (int q = 0; q < KT_IPL / 4; ++q) {
+        const uint4 v = *reinterpret_cast<const uint4*>(sk + off + l0 + 4 * q);
+        kr[4 * q] = v.x;
+        kr[4 * q + 1] = v.y;
+        kr[4 * q + 2] = v.z;
+        kr[4 * q + 3] = v.w;
+      }
+#pragma unroll
+      for (int j = 0; j < KT_IPL; ++j)
+        if ((u32)j >= cntf) kr[j] = NONE;
+      const u32 kprev = bb > 0 ? sk[(int)off - 1] : NONE;
+      const u32 kn_blk = bb + nb < n ? sk[off + nb] : NONE;
       u32 kp = __shfl_up_sync(0xFFFFFFFFu, kr[KT_IPL - 1], 1);
       u32 knx = __shfl_down_sync(0xFFFFFFFFu, kr[0], 1);
-      const u32 kn_blk = __shfl_sync(0xFFFFFFFFu, knext, 31);
       if (lane == 0) kp = kprev;
       if (lane == 31 || l0 + KT_IPL >= nb) knx = kn_blk;
       bool triv = true;
@@ -589,10 +619,14 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_sum(CheckArgs a, u32 nbl
         bs = tail_sum_nl(&a, bb, bb + nb);
         if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = blk;
       }
+      if (lane == 0) sums[blk] = bs;
     }
-    if (lane == 0) sums[blk] = bs;
-#pragma unroll
-    for (int j = 0; j < KT_IPL; ++j) kr[j] = kq[j];
+    (void)c0;
+    __syncthreads();  // every warp is done with stage st: refill it
+    if (threadIdx.x == 0 && c + KB_STAGES < n_chunks) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      issue(c + KB_STAGES, st);
+    }
   }
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);
   if (lane == 0) s_segs[wi] = segs;
@@ -921,7 +955,7 @@ static int k7_grid(int dev) {
 
 // status scratch: [K7Ctx][Sum sums[nblk]][Sum rin[nblk]][Sum ctot[nct]][Sum cpre[nct]][u32 wl[nblk]][u32 wl_cnt]
 // [u32 csegs[nct]]
-constexpr u32 K7A_CTAS = 148 * 8;
+constexpr u32 K7A_CTAS = 148 * 4;
 size_t check_status_bytes(u64 n) {
   const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1, nct = K7A_CTAS + 2;
   return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (2 * nblk + 2 * nct + 4) * sizeof(Sum) +
@@ -934,7 +968,8 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   cudaGetDevice(&dev);
   const int grid = k7_grid(dev);
   const u64 nblk = (L.n_max + KT_BLK - 1) / KT_BLK;
-  const u32 G = (u32)std::max<u64>(1, (nblk + K7A_CTAS - 1) / K7A_CTAS);  // blocks per K7a CTA
+  u32 G = (u32)std::max<u64>(1, (nblk + K7A_CTAS - 1) / K7A_CTAS);  // blocks per K7a CTA, whole chunks
+  G = (G + KT_SWARPS - 1) / KT_SWARPS * KT_SWARPS;
   const u32 nct = (u32)((nblk + G - 1) / G);
   char* base = (char*)L.status;
   K7Ctx* kdev = reinterpret_cast<K7Ctx*>(base);
