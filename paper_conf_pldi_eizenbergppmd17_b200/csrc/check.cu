@@ -576,8 +576,7 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 
       if (lane == 0) kp = kprev;
       if (lane == 31 || l0 + KT_IPL >= nb) knx = kn_blk;
       bool triv = true;
-      u32 tlw = 0, kl = kp, fsegs = 0;
-      bool kc = false;
+      u32 kl = kp, fsegs = 0;
 #pragma unroll
       for (int j = 0; j < KT_IPL; ++j) {
         if ((u32)j < cntf) {
@@ -587,34 +586,27 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 
           const bool atm_only =
               (k & 3u) == IOP_ATOM && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
           triv &= (!sp && !sn) || atm_only;
-          if (!sp) {
-            ++fsegs;
-            kc |= j > 0;
-            tlw = 0;
-          }
-          if ((k & 3u) != IOP_LD) tlw = (u32)bb + l0 + (u32)j + 1u;
+          fsegs += !sp;
           kl = k;
         }
       }
       segs += fsegs;
       if (fast_ok && __all_sync(0xFFFFFFFFu, triv)) {
-        // chunk summaries (no read has a same-granule read before it: no READINFLATE flags) and their
-        // warp combine = the block summary
-        Sum sm = sum_ident();
-        if (cntf) {
-          sm.fk = kr[0] >> 2;
-          sm.lk = kl >> 2;
-          sm.lw = tlw;
-          sm.fi = NONE;
-          sm.bits = (kc ? 0u : SB_ONE) | (tlw ? SB_W : 0u);
-        }
-        Sum incl = sm;
+        // no read has a same-granule read before it (no READINFLATE flags), so the summary is closed-form:
+        // first and last granule, and the last writer of the last granule (keys are sorted: its items are
+        // the block's tail run)
+        const u32 lkw = __shfl_sync(0xFFFFFFFFu, kl, (nb - 1) / (u32)KT_IPL);
+        const u32 fkw = __shfl_sync(0xFFFFFFFFu, kr[0], 0);
+        u32 mlw = 0;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const Sum up = shfl_up_sum(incl, o);
-          if ((int)lane >= o) incl = combine(up, incl);
-        }
-        bs = shfl_sum(incl, 31);
+        for (int j = 0; j < KT_IPL; ++j)
+          if ((u32)j < cntf && (kr[j] >> 2) == (lkw >> 2) && (kr[j] & 3u) != IOP_LD) mlw = (u32)bb + l0 + (u32)j + 1u;
+        mlw = __reduce_max_sync(0xFFFFFFFFu, mlw);
+        bs.fk = fkw >> 2;
+        bs.lk = lkw >> 2;
+        bs.lw = mlw;
+        bs.fi = NONE;
+        bs.bits = (bs.fk == bs.lk ? SB_ONE : 0u) | (mlw ? SB_W : 0u);
       } else {
         bs = tail_sum_nl(&a, bb, bb + nb);
         if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = blk;
