@@ -511,10 +511,10 @@ static __device__ __noinline__ Sum tail_sum_nl(const CheckArgs* a, u64 beg, u64 
 constexpr int KB_STAGES = 2;
 constexpr int KB_CHUNK = KT_SWARPS * KT_BLK;     // items per chunk
 constexpr int KB_ROW = KB_CHUNK + 8;             // words per stage
-__global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
+__global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
                                                             Sum* __restrict__ rin, Sum* __restrict__ ctot,
                                                             u32* __restrict__ wl, u32* __restrict__ wl_cnt,
-                                                            u32* __restrict__ csegs) {
+                                                            u32* __restrict__ csegs, u32* __restrict__ bflag) {
   __shared__ __align__(128) u32 s_keys[KB_STAGES][KB_ROW];
   __shared__ u64 s_bar[KB_STAGES];
   __shared__ Sum s_w[KT_SWARPS];
@@ -556,38 +556,43 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 
     Sum bs = sum_ident();
     if (nb) {
       const u32 off = wi * KT_BLK;  // the block's first item in the chunk
-      const u32 cntf = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
-      u32 kr[KT_IPL];
-#pragma unroll
-      for (int q = 0; q < KT_IPL / 4; ++q) {
-        const uint4 v = *reinterpret_cast<const uint4*>(sk + off + l0 + 4 * q);
-        kr[4 * q] = v.x;
-        kr[4 * q + 1] = v.y;
-        kr[4 * q + 2] = v.z;
-        kr[4 * q + 3] = v.w;
-      }
-#pragma unroll
-      for (int j = 0; j < KT_IPL; ++j)
-        if ((u32)j >= cntf) kr[j] = NONE;
-      const u32 kprev = bb > 0 ? sk[(int)off - 1] : NONE;
-      const u32 kn_blk = bb + nb < n ? sk[off + nb] : NONE;
-      u32 kp = __shfl_up_sync(0xFFFFFFFFu, kr[KT_IPL - 1], 1);
-      u32 knx = __shfl_down_sync(0xFFFFFFFFu, kr[0], 1);
-      if (lane == 0) kp = kprev;
-      if (lane == 31 || l0 + KT_IPL >= nb) knx = kn_blk;
+      // 4 rounds of 128 items; in round q lane l holds items 128 q + 4 l .. + 3 (one conflict-free
+      // 16-B shared-memory read); neighbours across lanes / rounds by shuffles and broadcast reads
+      const u32 lkw = sk[off + nb - 1];                           // the block's last item
+      const u32 fkw = sk[off];
+      u32 pk_round = bb > 0 ? sk[(int)off - 1] : NONE;            // item before the round
       bool triv = true;
-      u32 kl = kp, fsegs = 0;
+      u32 fsegs = 0, mlw = 0;
 #pragma unroll
-      for (int j = 0; j < KT_IPL; ++j) {
-        if ((u32)j < cntf) {
-          const u32 k = kr[j], kpv = kl, knv = (u32)j + 1 < cntf ? kr[j + 1] : knx;
+      for (int q = 0; q < KT_BLK / 128; ++q) {
+        const u32 base = (u32)q * 128u + lane * 4u;  // item index within the block
+        const uint4 v = *reinterpret_cast<const uint4*>(sk + off + base);
+        u32 kk[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+        for (int t = 0; t < 4; ++t)
+          if (base + (u32)t >= nb) kk[t] = NONE;
+        u32 kprev = __shfl_up_sync(0xFFFFFFFFu, kk[3], 1);
+        if (lane == 0) kprev = pk_round;
+        u32 knext = __shfl_down_sync(0xFFFFFFFFu, kk[0], 1);
+        if (lane == 31) {
+          const u32 nx = (u32)q * 128u + 128u;
+          knext = nx < nb ? sk[off + nx] : (bb + nb < n ? sk[off + nb] : NONE);
+        }
+        pk_round = __shfl_sync(0xFFFFFFFFu, kk[3], 31);
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          const u32 k = kk[t];
+          if (k == NONE) continue;
+          const u32 kpv = t ? kk[t - 1] : kprev;
+          const u32 knv = t < 3 ? kk[t + 1] : knext;
           const u32 key = k >> 2;
-          const bool sp = kpv != NONE && (kpv >> 2) == key, sn = knv != NONE && (knv >> 2) == key;
-          const bool atm_only =
-              (k & 3u) == IOP_ATOM && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
+          const bool sp = kpv != NONE && (kpv >> 2) == key;
+          const bool sn = knv != NONE && (knv >> 2) == key;
+          const bool atm = (k & 3u) == IOP_ATOM;
+          const bool atm_only = atm && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
           triv &= (!sp && !sn) || atm_only;
           fsegs += !sp;
-          kl = k;
+          if (key == (lkw >> 2) && (k & 3u) != IOP_LD) mlw = (u32)bb + base + (u32)t + 1u;
         }
       }
       segs += fsegs;
@@ -595,23 +600,20 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 
         // no read has a same-granule read before it (no READINFLATE flags), so the summary is closed-form:
         // first and last granule, and the last writer of the last granule (keys are sorted: its items are
         // the block's tail run)
-        const u32 lkw = __shfl_sync(0xFFFFFFFFu, kl, (nb - 1) / (u32)KT_IPL);
-        const u32 fkw = __shfl_sync(0xFFFFFFFFu, kr[0], 0);
-        u32 mlw = 0;
-#pragma unroll
-        for (int j = 0; j < KT_IPL; ++j)
-          if ((u32)j < cntf && (kr[j] >> 2) == (lkw >> 2) && (kr[j] & 3u) != IOP_LD) mlw = (u32)bb + l0 + (u32)j + 1u;
         mlw = __reduce_max_sync(0xFFFFFFFFu, mlw);
         bs.fk = fkw >> 2;
         bs.lk = lkw >> 2;
         bs.lw = mlw;
         bs.fi = NONE;
         bs.bits = (bs.fk == bs.lk ? SB_ONE : 0u) | (mlw ? SB_W : 0u);
-      } else {
-        bs = tail_sum_nl(&a, bb, bb + nb);
-        if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = blk;
+        if (lane == 0) {
+          sums[blk] = bs;
+          bflag[blk] = 0;
+        }
+      } else if (lane == 0) {  // summarised after the stream (phase 1b), checked by K7b
+        bflag[blk] = 1;
+        wl[atomicAdd(wl_cnt, 1u)] = blk;
       }
-      if (lane == 0) sums[blk] = bs;
     }
     (void)c0;
     __syncthreads();  // every warp is done with stage st: refill it
@@ -623,6 +625,15 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);
   if (lane == 0) s_segs[wi] = segs;
   if (threadIdx.x == 0) s_carry = sum_ident();
+  __syncthreads();
+  // ---- phase 1b: the blocks with checks, summarised by a bounded tail walk
+  for (u32 blk = b0 + wi; blk < b1; blk += KT_SWARPS) {
+    if (!bflag[blk]) continue;  // warp-uniform
+    const u64 bb = (u64)blk * KT_BLK;
+    const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
+    const Sum bs = tail_sum_nl(&a, bb, bb + nb);
+    if (lane == 0) sums[blk] = bs;
+  }
   __syncthreads();
   // ---- phase 2: exclusive prefix of the CTA's block summaries, 256 at a time
   for (u32 c0 = b0; c0 < b1; c0 += KT_SWARPS * 32) {
@@ -951,7 +962,7 @@ constexpr u32 K7A_CTAS = 148 * 4;
 size_t check_status_bytes(u64 n) {
   const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1, nct = K7A_CTAS + 2;
   return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (2 * nblk + 2 * nct + 4) * sizeof(Sum) +
-         (nblk + nct + 64) * sizeof(u32) + 512;
+         (2 * nblk + nct + 64) * sizeof(u32) + 512;
 }
 
 void launch_check(const CheckLaunch& L, cudaStream_t st) {
@@ -972,6 +983,7 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   u32* wl = reinterpret_cast<u32*>(cpre + nct + 1);
   u32* wl_cnt = wl + nblk + 1;
   u32* csegs = wl_cnt + 1;
+  u32* bflag = csegs + nct + 1;
   K7Ctx k{};
   k.c = L.c;
   k.keys = L.keys;
@@ -1002,7 +1014,7 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   a.rin = nullptr;
   a.no_sv = L.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   a.values = L.values;
-  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, rin, ctot, wl, wl_cnt, csegs);
+  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, rin, ctot, wl, wl_cnt, csegs, bflag);
   k_range_scan<<<1, 1024, 0, st>>>(ctot, nct, cpre, csegs, L.seg_cnt);
   k_check_tile<<<grid, KT_WARPS * 32, (size_t)KT_WARPS * KT_WARP_BYTES, st>>>(a, wl, wl_cnt, rin, cpre, G);
   g_launches += 3;
