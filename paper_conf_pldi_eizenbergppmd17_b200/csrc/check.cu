@@ -574,25 +574,26 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
         u32 kprev = __shfl_up_sync(0xFFFFFFFFu, kk[3], 1);
         if (lane == 0) kprev = pk_round;
         u32 knext = __shfl_down_sync(0xFFFFFFFFu, kk[0], 1);
-        if (lane == 31) {
+        {  // lane 31: the next round's first item, or the item after the block (a broadcast read)
           const u32 nx = (u32)q * 128u + 128u;
-          knext = nx < nb ? sk[off + nx] : (bb + nb < n ? sk[off + nb] : NONE);
+          const u32 k31 = sk[off + (nx < nb ? nx : nb)];
+          const u32 kn31 = (nx < nb || bb + nb < n) ? k31 : NONE;
+          knext = lane == 31 ? kn31 : knext;
         }
         pk_round = __shfl_sync(0xFFFFFFFFu, kk[3], 31);
 #pragma unroll
-        for (int t = 0; t < 4; ++t) {
+        for (int t = 0; t < 4; ++t) {  // branch-free: predicates and selects only
           const u32 k = kk[t];
-          if (k == NONE) continue;
           const u32 kpv = t ? kk[t - 1] : kprev;
           const u32 knv = t < 3 ? kk[t + 1] : knext;
+          const bool valid = k != NONE;
           const u32 key = k >> 2;
-          const bool sp = kpv != NONE && (kpv >> 2) == key;
-          const bool sn = knv != NONE && (knv >> 2) == key;
-          const bool atm = (k & 3u) == IOP_ATOM;
-          const bool atm_only = atm && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
-          triv &= (!sp && !sn) || atm_only;
-          fsegs += !sp;
-          if (key == (lkw >> 2) && (k & 3u) != IOP_LD) mlw = (u32)bb + base + (u32)t + 1u;
+          const bool sp = valid && kpv != NONE && (kpv >> 2) == key;
+          const bool sn = valid && knv != NONE && (knv >> 2) == key;
+          const bool atm_only = (k & 3u) == IOP_ATOM && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
+          triv = triv && (!(sp || sn) || atm_only);
+          fsegs += (valid && !sp) ? 1u : 0u;
+          mlw = (valid && key == (lkw >> 2) && (k & 3u) != IOP_LD) ? (u32)bb + base + (u32)t + 1u : mlw;
         }
       }
       segs += fsegs;
@@ -626,13 +627,18 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
   if (lane == 0) s_segs[wi] = segs;
   if (threadIdx.x == 0) s_carry = sum_ident();
   __syncthreads();
-  // ---- phase 1b: the blocks with checks, summarised by a bounded tail walk
-  for (u32 blk = b0 + wi; blk < b1; blk += KT_SWARPS) {
-    if (!bflag[blk]) continue;  // warp-uniform
-    const u64 bb = (u64)blk * KT_BLK;
-    const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
-    const Sum bs = tail_sum_nl(&a, bb, bb + nb);
-    if (lane == 0) sums[blk] = bs;
+  // ---- phase 1b: the blocks with checks, summarised by a bounded tail walk (flags read 32 at a time)
+  for (u32 g0 = b0 + wi * 32; g0 < b1; g0 += KT_SWARPS * 32) {
+    const u32 bl = g0 + lane;
+    u32 fl = __ballot_sync(0xFFFFFFFFu, bl < b1 && bflag[bl]);
+    while (fl) {
+      const u32 blk = g0 + (u32)__ffs(fl) - 1u;
+      fl &= fl - 1;
+      const u64 bb = (u64)blk * KT_BLK;
+      const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
+      const Sum bs = tail_sum_nl(&a, bb, bb + nb);
+      if (lane == 0) sums[blk] = bs;
+    }
   }
   __syncthreads();
   // ---- phase 2: exclusive prefix of the CTA's block summaries, 256 at a time
