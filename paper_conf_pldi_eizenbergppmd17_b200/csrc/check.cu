@@ -561,18 +561,19 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
       const u32 lkw = sk[off + nb - 1];                           // the block's last item
       const u32 fkw = sk[off];
       u32 pk_round = bb > 0 ? sk[(int)off - 1] : NONE;            // item before the round
-      bool triv = true;
-      u32 fsegs = 0, mlw = 0;
+      // A block makes no check iff no two neighbouring items (including the items just before and
+      // after it) share a granule unless both are atomics.  Absent items are NONE: granule 0x3FFFFFFF
+      // (never a real key, keys < 2^30 - 1) with the atomic op bits, so they never form a bad pair.
+      u32 bad = 0, fsegs = 0, mlw = 0;
 #pragma unroll
       for (int q = 0; q < KT_BLK / 128; ++q) {
         const u32 base = (u32)q * 128u + lane * 4u;  // item index within the block
         const uint4 v = *reinterpret_cast<const uint4*>(sk + off + base);
         u32 kk[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
-        for (int t = 0; t < 4; ++t)
-          if (base + (u32)t >= nb) kk[t] = NONE;
+        for (int t = 0; t < 4; ++t) kk[t] = base + (u32)t < nb ? kk[t] : NONE;
         u32 kprev = __shfl_up_sync(0xFFFFFFFFu, kk[3], 1);
-        if (lane == 0) kprev = pk_round;
+        kprev = lane == 0 ? pk_round : kprev;
         u32 knext = __shfl_down_sync(0xFFFFFFFFu, kk[0], 1);
         {  // lane 31: the next round's first item, or the item after the block (a broadcast read)
           const u32 nx = (u32)q * 128u + 128u;
@@ -581,21 +582,19 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
           knext = lane == 31 ? kn31 : knext;
         }
         pk_round = __shfl_sync(0xFFFFFFFFu, kk[3], 31);
+        u32 kpv = kprev;
 #pragma unroll
-        for (int t = 0; t < 4; ++t) {  // branch-free: predicates and selects only
+        for (int t = 0; t < 4; ++t) {
           const u32 k = kk[t];
-          const u32 kpv = t ? kk[t - 1] : kprev;
-          const u32 knv = t < 3 ? kk[t + 1] : knext;
-          const bool valid = k != NONE;
-          const u32 key = k >> 2;
-          const bool sp = valid && kpv != NONE && (kpv >> 2) == key;
-          const bool sn = valid && knv != NONE && (knv >> 2) == key;
-          const bool atm_only = (k & 3u) == IOP_ATOM && (!sp || (kpv & 3u) == IOP_ATOM) && (!sn || (knv & 3u) == IOP_ATOM);
-          triv = triv && (!(sp || sn) || atm_only);
-          fsegs += (valid && !sp) ? 1u : 0u;
-          mlw = (valid && key == (lkw >> 2) && (k & 3u) != IOP_LD) ? (u32)bb + base + (u32)t + 1u : mlw;
+          const u32 x = k ^ kpv;
+          bad |= (x < 4u) & ((k & kpv & 3u) != 3u);
+          fsegs += (x >= 4u) & (k != NONE);
+          mlw = (((k ^ lkw) < 4u) & ((k & 3u) != IOP_LD)) ? (u32)bb + base + (u32)t + 1u : mlw;
+          kpv = k;
         }
+        bad |= ((kk[3] ^ knext) < 4u) & ((kk[3] & knext & 3u) != 3u);
       }
+      const bool triv = bad == 0u;
       segs += fsegs;
       if (fast_ok && __all_sync(0xFFFFFFFFu, triv)) {
         // no read has a same-granule read before it (no READINFLATE flags), so the summary is closed-form:
