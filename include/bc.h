@@ -184,6 +184,19 @@ bc_status bc_load_trace(struct bc_ctx* ctx, const bc_record* recs, uint64_t n_re
 bc_status bc_load_trace_shard(bc_ctx* ctx, const bc_record* recs, const uint32_t* rec_index, uint64_t n_local,
                               uint64_t n_global, int recs_on_device);
 
+/* Warp-size simulation (reading R17 in DESIGN.md): re-split a trace recorded
+ * with 32-lane warps (the geometry of ctx, whose warp_size must be 32) into virtual warps of ws lanes
+ * (4, 8, 16; 32 copies it).  Record (warp w, mask m) becomes, in trace order, one record per virtual
+ * warp j of w that executes it: warp (block, (w_in_block * 32 + j * ws) / ws), mask
+ * (m >> j*ws) & (2^ws - 1), addresses addr[j*ws ...]; an IF none of whose lanes are in virtual warp j is
+ * not executed by it, nor its ELSE / FI or anything nested.  recs, out, origin: DEVICE pointers on
+ * ctx's device; origin[i] = (source record << 5) | first lane of out[i].  *n_out = records of the
+ * split trace (out == NULL: count only); cap < *n_out -> cap records written, BC_ERR_TRUNCATED.  The
+ * result is checked with a context of warp_size = ws and the same grid / block.  Stream-ordered on
+ * ctx's stream, synchronizes before return. */
+bc_status bc_split_warps(bc_ctx* ctx, const bc_record* recs, uint64_t n_recs, uint32_t ws, bc_record* out,
+                         uint64_t* origin, uint64_t cap, uint64_t* n_out);
+
 /* 128-byte NCCL unique id for bc_config.nccl_unique_id (call on rank 0 only).  BC_ERR_NCCL if no NCCL
  * library can be loaded (libbc dlopens the libnccl.so.2 already in the process, else the system's). */
 bc_status bc_nccl_unique_id(void* out128);

@@ -40,7 +40,7 @@ F_COUNT_GATHERS = 4  # statistics: fill stats["clock_gathers"] (one extra pass)
 
 EXPORTS = sorted(["bc_init", "bc_load_trace", "bc_load_values", "bc_detect", "bc_races", "bc_races_device",
                   "bc_destroy", "bc_status_string", "bc_last_error", "bc_phase_name", "bc_load_trace_shard",
-                  "bc_nccl_unique_id", "bc_group_create_local", "bc_group_destroy"])
+                  "bc_nccl_unique_id", "bc_group_create_local", "bc_group_destroy", "bc_split_warps"])
 
 
 class BcError(RuntimeError):
@@ -112,6 +112,10 @@ def lib():
         L.bc_group_create_local.restype = ctypes.c_int
         L.bc_group_create_local.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_void_p)]
         L.bc_group_destroy.argtypes = [ctypes.c_void_p]
+        L.bc_split_warps.restype = ctypes.c_int
+        L.bc_split_warps.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32,
+                                     ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                     ctypes.POINTER(ctypes.c_uint64)]
         _lib = L
     return _lib
 
@@ -292,6 +296,35 @@ class Context:
 
     def __exit__(self, *a):
         self.close()
+
+
+def split_warps(records, geometry: dict, ws: int, device: int = 0):
+    """bc_split_warps (reading R17): the trace re-split into virtual warps of ws lanes,
+    on the GPU.  records: host array or CUDA uint8 tensor of the 32-lane trace.  Returns (CUDA uint8
+    tensor of the split records, geometry with warp_size = ws, CUDA int64 tensor of origins =
+    (source record << 5) | first lane).  Marshalling only."""
+    import torch
+    dev = torch.device("cuda", device)
+    if hasattr(records, "is_cuda") and records.is_cuda:
+        d_in = records
+    else:
+        d_in = torch.from_numpy(np.ascontiguousarray(records).view(np.uint8)).to(dev)
+    n = d_in.numel() // RECORD_BYTES
+    g32 = dict(geometry)
+    g32["warp_size"] = 32
+    with Context(g32, device=device) as ctx:
+        L = lib()
+        cnt = ctypes.c_uint64()
+        ctx._check(L.bc_split_warps(ctx._h, ctypes.c_void_p(d_in.data_ptr()), n, ws, None, None, 0,
+                                    ctypes.byref(cnt)))
+        m = int(cnt.value)
+        out = torch.empty(max(m, 1) * RECORD_BYTES, dtype=torch.uint8, device=dev)
+        org = torch.empty(max(m, 1), dtype=torch.int64, device=dev)
+        ctx._check(L.bc_split_warps(ctx._h, ctypes.c_void_p(d_in.data_ptr()), n, ws, ctypes.c_void_p(out.data_ptr()),
+                                    ctypes.c_void_p(org.data_ptr()), m, ctypes.byref(cnt)))
+    g2 = dict(geometry)
+    g2["warp_size"] = ws
+    return out[:m * RECORD_BYTES], g2, org[:m]
 
 
 def nccl_unique_id() -> bytes:

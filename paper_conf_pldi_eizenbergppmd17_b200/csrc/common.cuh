@@ -278,12 +278,20 @@ static __device__ __noinline__ bool view_knows(const HbCtx c, u32 uw, u32 ul, u3
 // foreign part of know_t(u) >= r1+1 for t executing record r2 (snapshot s2): through the
 // views of the acquires of t's block that t structurally knows (every release->acquire path
 // into t's block ends at one of them).
+// The acquires are tried newest first: in lock-based code the acquire that orders an access is almost
+// always the latest one t knows (the critical section it is in), and its view holds the previous
+// holder's release directly -- an oldest-first search would walk the views of every earlier critical
+// section of the block first (the lock-heavy programs of SURVEY row f2).
 static __device__ __noinline__ bool foreign_knows(const HbCtx c, u32 w1, u32 l1, u32 r1, u32 r2, const Snap s2) {
   u32 b2 = s2.warp / c.g.wpb;
   u32 lo = c.acq_block_start[b2], hi = c.acq_block_start[b2 + 1];
-  for (u32 i = lo; i < hi; ++i) {
-    u32 ra = c.acq_rec[i];
-    if (ra >= r2) break;
+  while (lo < hi) {  // first acquire of the block at or after r2
+    const u32 m = (lo + hi) >> 1;
+    if (c.acq_rec[m] < r2) lo = m + 1; else hi = m;
+  }
+  for (u32 i = lo; i-- > c.acq_block_start[b2];) {
+    const u32 ra = c.acq_rec[i];
+    if (ra < r1) break;  // an acquire before the access cannot order it (view entries are older than ra)
     if (!struct_knows(c, c.acq_warp[i], c.acq_lane[i], ra, s2)) continue;
     if (view_knows(c, w1, l1, r1, c.acq_arr[i], NONE)) return true;
   }
