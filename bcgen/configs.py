@@ -28,6 +28,8 @@ CONFIGS = {
     "c6": "lock-heavy hashtable trace (SURVEY row f2, P:L1522-1535): 256 blocks x 128 threads, 2 inserts "
           "per thread under per-bucket locks, with both section-6.3 bugs (CAS without fence, unlock by plain "
           "store); bug=0 is the fixed program",
+    "c6f": "lock-heavy hashtable trace, fixed program (every lock an atomicCAS + fence acquire and a fence + "
+           "atomicExch release; race-free): 256 blocks x 128 threads, 2 inserts per thread",
 }
 
 
