@@ -512,14 +512,11 @@ constexpr int KB_STAGES = 2;
 constexpr int KB_CHUNK = KT_SWARPS * KT_BLK;     // items per chunk
 constexpr int KB_ROW = KB_CHUNK + 8;             // words per stage
 __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
-                                                            Sum* __restrict__ rin, Sum* __restrict__ ctot,
-                                                            u32* __restrict__ wl, u32* __restrict__ wl_cnt,
-                                                            u32* __restrict__ csegs, u32* __restrict__ bflag) {
+                                                            u32* __restrict__ csegs, u32* __restrict__ bflag,
+                                                            u32* __restrict__ n_nontriv) {
   __shared__ __align__(128) u32 s_keys[KB_STAGES][KB_ROW];
   __shared__ u64 s_bar[KB_STAGES];
-  __shared__ Sum s_w[KT_SWARPS];
-  __shared__ Sum s_carry;
-  __shared__ u32 s_segs[KT_SWARPS];
+  __shared__ u32 s_segs[1];
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const u64 n = *a.n_dev;
   const bool fast_ok = a.sh_in == nullptr && a.sh_out == nullptr;
@@ -539,12 +536,13 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
   if (threadIdx.x == 0) {
     for (int q = 0; q < KB_STAGES; ++q) mbar_init(&s_bar[q], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    s_segs[0] = 0;
   }
   __syncthreads();
   if (threadIdx.x == 0)
     for (int q = 0; q < KB_STAGES; ++q)
       if ((u32)q < n_chunks) issue(q, q);
-  u32 segs = 0;
+  u32 segs = 0, nontriv = 0;
   for (u32 c = 0; c < n_chunks; ++c) {
     const int st = (int)(c % KB_STAGES);
     mbar_wait(&s_bar[st], (c / KB_STAGES) & 1u);
@@ -610,9 +608,9 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
           sums[blk] = bs;
           bflag[blk] = 0;
         }
-      } else if (lane == 0) {  // summarised after the stream (phase 1b), checked by K7b
-        bflag[blk] = 1;
-        wl[atomicAdd(wl_cnt, 1u)] = blk;
+      } else {  // summarised with its unit (k_blk_units), checked by K7b
+        if (lane == 0) bflag[blk] = 1;
+        ++nontriv;
       }
     }
     (void)c0;
@@ -623,24 +621,56 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
     }
   }
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);
-  if (lane == 0) s_segs[wi] = segs;
-  if (threadIdx.x == 0) s_carry = sum_ident();
+  if (lane == 0) {
+    if (segs) atomicAdd(&s_segs[0], segs);
+    if (nontriv) atomicAdd(n_nontriv, nontriv);
+  }
   __syncthreads();
-  // ---- phase 1b: the blocks with checks, summarised by a bounded tail walk (flags read 32 at a time)
-  for (u32 g0 = b0 + wi * 32; g0 < b1; g0 += KT_SWARPS * 32) {
-    const u32 bl = g0 + lane;
-    u32 fl = __ballot_sync(0xFFFFFFFFu, bl < b1 && bflag[bl]);
+  if (threadIdx.x == 0) csegs[blockIdx.x] = s_segs[0];  // summed by k_range_scan
+}
+
+// ---------------------------------------------------------------------- K7a2: units and CTA scans
+// The blocks with checks are processed by K7b in UNITS of U consecutive blocks (a power of two chosen
+// from the number of such blocks: about one unit per K7b warp on dense traces, single blocks on
+// sparse ones), one warp per unit carrying the automaton state from block to block.  Per unit with a
+// check: one bounded tail walk gives the unit's summary (placed at its last block, identity at the
+// others) and the unit is listed.  Then each CTA scans its blocks' summaries (rin) and writes its total.
+__global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
+                                                              Sum* __restrict__ rin, Sum* __restrict__ ctot,
+                                                              u32* __restrict__ wl, u32* __restrict__ wl_cnt,
+                                                              const u32* __restrict__ bflag,
+                                                              const u32* __restrict__ n_nontriv, u32 nw_b,
+                                                              u32* __restrict__ unit_out) {
+  __shared__ Sum s_w[KT_SWARPS];
+  __shared__ Sum s_carry;
+  const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const u64 n = *a.n_dev;
+  const u32 b0 = blockIdx.x * G, b1 = min(nblk, b0 + G);
+  // U: the smallest power of two with (non-trivial blocks / U) <= K7b warps, at most G (G is a power of two)
+  const u32 nt = *n_nontriv;
+  u32 U = 1;
+  while (U < G && (u64)U * nw_b < nt) U <<= 1;
+  if (blockIdx.x == 0 && threadIdx.x == 0) *unit_out = U;
+  if (threadIdx.x == 0) s_carry = sum_ident();
+  // ---- units with a check: one tail walk each (flags of 32 units' blocks read at once per warp)
+  for (u32 u0 = b0 / U + wi * 32; u0 * U < b1; u0 += KT_SWARPS * 32) {
+    const u32 uu = u0 + lane;
+    bool any = false;
+    if (uu * U < b1)
+      for (u32 q = 0; q < U && uu * U + q < b1; ++q) any |= bflag[uu * U + q] != 0u;
+    u32 fl = __ballot_sync(0xFFFFFFFFu, any);
     while (fl) {
-      const u32 blk = g0 + (u32)__ffs(fl) - 1u;
+      const u32 u = u0 + (u32)__ffs(fl) - 1u;
       fl &= fl - 1;
-      const u64 bb = (u64)blk * KT_BLK;
-      const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
-      const Sum bs = tail_sum_nl(&a, bb, bb + nb);
-      if (lane == 0) sums[blk] = bs;
+      const u32 ub0 = u * U, ub1 = min(b1, ub0 + U);
+      const u64 beg = (u64)ub0 * KT_BLK, end = min(n, (u64)ub1 * KT_BLK);
+      const Sum bs = tail_sum_nl(&a, beg, end);
+      for (u32 q = ub0 + lane; q < ub1; q += 32) sums[q] = q + 1 == ub1 ? bs : sum_ident();
+      if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = u;
     }
   }
   __syncthreads();
-  // ---- phase 2: exclusive prefix of the CTA's block summaries, 256 at a time
+  // ---- exclusive prefix of the CTA's block summaries, 256 at a time
   for (u32 c0 = b0; c0 < b1; c0 += KT_SWARPS * 32) {
     const u32 i = c0 + threadIdx.x;
     const Sum v = i < b1 ? sums[i] : sum_ident();
@@ -665,19 +695,15 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
     }
     __syncthreads();
   }
-  if (threadIdx.x == 0) {
-    u32 sg = 0;
-    for (int q = 0; q < KT_SWARPS; ++q) sg += s_segs[q];
-    ctot[blockIdx.x] = s_carry;
-    csegs[blockIdx.x] = sg;  // summed by k_range_scan
-  }
+  if (threadIdx.x == 0) ctot[blockIdx.x] = s_carry;
 }
 
 // ---------------------------------------------------------------------- K7b: the listed blocks
 __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, const u32* __restrict__ wl,
                                                                  const u32* __restrict__ wl_cnt,
                                                                  const Sum* __restrict__ rin,
-                                                                 const Sum* __restrict__ cpre, u32 G) {
+                                                                 const Sum* __restrict__ cpre, u32 G, u32 nblk,
+                                                                 const u32* __restrict__ unit_p) {
   extern __shared__ __align__(16) unsigned char kt_smem[];
   const int wi = threadIdx.x >> 5;
   uint4* sS = reinterpret_cast<uint4*>(kt_smem + (size_t)wi * KT_WARP_BYTES);
@@ -691,15 +717,20 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
   const u32 R0 = a.R0;
   const bool shadow = a.sh_in != nullptr;
   const u32 n_tasks = *wl_cnt;
+  const u32 U = *unit_p;  // blocks per unit (K7a)
   u32 segs = 0;
   const u32 l0 = lane * KT_IPL;
   for (u32 task = w; task < n_tasks; task += nw) {
-    const u32 blkid = wl[task];
-    const u64 bb = (u64)blkid * KT_BLK;
+    // a unit: U consecutive blocks, processed in order with the automaton state carried through
+    const u32 u = wl[task];
+    const u32 blk0 = u * U, blk1 = min(nblk, blk0 + U);
+    // state entering the unit: its K7a CTA's prefix (K7s), then the prefix within that CTA
+    Sum carry = combine(cpre[blk0 / G], rin[blk0]);
+    u32 pkx = blk0 > 0 ? __ldg(a.keys + (u64)blk0 * KT_BLK - 1) : NONE;  // the item before the block
+    for (u32 bi = blk0; bi < blk1; ++bi) {
+    const u64 bb = (u64)bi * KT_BLK;
+    if (bb >= n) break;
     const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
-    // state entering the block: its K7a CTA's prefix (K7s), then the prefix within that CTA
-    Sum carry = combine(cpre[blkid / G], rin[blkid]);
-    const u32 pkx = bb > 0 ? __ldg(a.keys + bb - 1) : NONE;  // the item before the block
     const u32 knext = bb + nb < n ? __ldg(a.keys + bb + nb) : NONE;  // first item after the block
     kt_stage(a, bb, nb, sK, sE, lane);
     cp_async_wait0();
@@ -913,8 +944,10 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
       }
     }
 
-    (void)blk;
+    carry = combine(carry, blk);
+    pkx = sK[tpad(nb - 1)];
     __syncwarp();
+    }
   }
   (void)segs;
 }
@@ -967,7 +1000,7 @@ constexpr u32 K7A_CTAS = 148 * 4;
 size_t check_status_bytes(u64 n) {
   const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1, nct = K7A_CTAS + 2;
   return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (2 * nblk + 2 * nct + 4) * sizeof(Sum) +
-         (2 * nblk + nct + 64) * sizeof(u32) + 512;
+         (2 * nblk + nct + 64) * sizeof(u32) + 1024;
 }
 
 void launch_check(const CheckLaunch& L, cudaStream_t st) {
@@ -976,8 +1009,8 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   cudaGetDevice(&dev);
   const int grid = k7_grid(dev);
   const u64 nblk = (L.n_max + KT_BLK - 1) / KT_BLK;
-  u32 G = (u32)std::max<u64>(1, (nblk + K7A_CTAS - 1) / K7A_CTAS);  // blocks per K7a CTA, whole chunks
-  G = (G + KT_SWARPS - 1) / KT_SWARPS * KT_SWARPS;
+  u32 G = KT_SWARPS;  // blocks per K7a CTA: a power of two >= KT_SWARPS (whole chunks, whole units)
+  while ((u64)G * K7A_CTAS < nblk) G <<= 1;
   const u32 nct = (u32)((nblk + G - 1) / G);
   char* base = (char*)L.status;
   K7Ctx* kdev = reinterpret_cast<K7Ctx*>(base);
@@ -989,6 +1022,8 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   u32* wl_cnt = wl + nblk + 1;
   u32* csegs = wl_cnt + 1;
   u32* bflag = csegs + nct + 1;
+  u32* n_nontriv = bflag + nblk + 1;
+  u32* unit_p = n_nontriv + 1;
   K7Ctx k{};
   k.c = L.c;
   k.keys = L.keys;
@@ -1007,6 +1042,7 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   k.n_dev = L.n_dev;
   cudaMemcpyAsync(kdev, &k, sizeof(K7Ctx), cudaMemcpyHostToDevice, st);
   cudaMemsetAsync(wl_cnt, 0, sizeof(u32), st);
+  cudaMemsetAsync(n_nontriv, 0, sizeof(u32), st);
   CheckArgs a;
   a.k = kdev;
   a.c = L.c;
@@ -1019,10 +1055,13 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   a.rin = nullptr;
   a.no_sv = L.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   a.values = L.values;
-  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, rin, ctot, wl, wl_cnt, csegs, bflag);
+  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, csegs, bflag, n_nontriv);
+  k_blk_units<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, rin, ctot, wl, wl_cnt, bflag, n_nontriv,
+                                              (u32)grid * KT_WARPS, unit_p);
   k_range_scan<<<1, 1024, 0, st>>>(ctot, nct, cpre, csegs, L.seg_cnt);
-  k_check_tile<<<grid, KT_WARPS * 32, (size_t)KT_WARPS * KT_WARP_BYTES, st>>>(a, wl, wl_cnt, rin, cpre, G);
-  g_launches += 3;
+  k_check_tile<<<grid, KT_WARPS * 32, (size_t)KT_WARPS * KT_WARP_BYTES, st>>>(a, wl, wl_cnt, rin, cpre, G, (u32)nblk,
+                                                                            unit_p);
+  g_launches += 4;
 }
 
 }  // namespace bc
