@@ -631,7 +631,7 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
 
 // ---------------------------------------------------------------------- K7a2: units and CTA scans
 // The blocks with checks are processed by K7b in UNITS of U consecutive blocks (a power of two chosen
-// from the number of such blocks: about one unit per K7b warp on dense traces, single blocks on
+// from the number of such blocks: about two units per K7b warp on dense traces, single blocks on
 // sparse ones), one warp per unit carrying the automaton state from block to block.  Per unit with a
 // check: one bounded tail walk gives the unit's summary (placed at its last block, identity at the
 // others) and the unit is listed.  Then each CTA scans its blocks' summaries (rin) and writes its total.
@@ -646,10 +646,11 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, u32 n
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const u64 n = *a.n_dev;
   const u32 b0 = blockIdx.x * G, b1 = min(nblk, b0 + G);
-  // U: the smallest power of two with (non-trivial blocks / U) <= K7b warps, at most G (G is a power of two)
+  // U: the largest power of two with at least two units per K7b warp (load balance), at most G (a power
+  // of two); 1 on sparse traces
   const u32 nt = *n_nontriv;
   u32 U = 1;
-  while (U < G && (u64)U * nw_b < nt) U <<= 1;
+  while (U * 2 <= G && (u64)U * 2 * 2 * nw_b <= nt) U <<= 1;
   if (blockIdx.x == 0 && threadIdx.x == 0) *unit_out = U;
   if (threadIdx.x == 0) s_carry = sum_ident();
   // ---- units with a check: one tail walk each (flags of 32 units' blocks read at once per warp)
