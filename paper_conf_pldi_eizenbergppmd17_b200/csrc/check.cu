@@ -281,23 +281,26 @@ __device__ __forceinline__ void warp_range(u64 n, u32 w, u32 nw, u64& beg, u64& 
 
 // Carried inflation of a read run that starts at the granule's first item s of the window (a read):
 // the carried read state is a vector, or an epoch the read at s does not know (READINFLATE).
-__device__ __forceinline__ bool carried_infl(const CheckArgs& a, const Carry& C, u32 ev_s, const Snap& s_s) {
+__device__ __forceinline__ bool carried_infl(const K7Ctx* k, const Carry& C, u32 ev_s, const Snap& s_s) {
   if (C.rm == SH_R_VC) return true;
   if (C.rm != SH_R_EPOCH) return false;
-  return !hbq(a.k, a.c, C.rr, C.rwl & 31u, C.rwl >> 5, a.R0 + (ev_s >> 5), ev_s & 31u, s_s);
+  return !hbq(k, k->c, C.rr, C.rwl & 31u, C.rwl >> 5, k->R0 + (ev_s >> 5), ev_s & 31u, s_s);
 }
 
 // ---------------------------------------------------------------------- tail summary of an item range
 // Summary (Sum) of the items [beg, end): the tail granule run's last writer and first inflation after
 // it, found by walking back from the end (usually a few items: a writer or the granule's start ends
 // the walk; never past beg).  Warp-cooperative; uniform result.
-__device__ Sum tail_sum(const CheckArgs& a, u64 beg, u64 end) {
+__device__ Sum tail_sum(const K7Ctx* kc, u64 beg, u64 end) {
   const int lane = threadIdx.x & 31;
-  const HbCtx& c = a.c;
+  const HbCtx& c = kc->c;
+  const u32* const keys = kc->keys;
+  const u32* const evs = kc->evs;
+  const u32 R0 = kc->R0;
   Sum s = sum_ident();
   if (beg >= end) return s;
-  const u32 k0 = __ldg(a.keys + end - 1) >> 2;
-  s.fk = __ldg(a.keys + beg) >> 2;
+  const u32 k0 = __ldg(keys + end - 1) >> 2;
+  s.fk = __ldg(keys + beg) >> 2;
   s.lk = k0;
   u32 bits = s.fk == k0 ? SB_ONE : 0u, lw = 0, fi = NONE;
   u64 hi = end - 1;
@@ -305,7 +308,7 @@ __device__ Sum tail_sum(const CheckArgs& a, u64 beg, u64 end) {
     const u64 lo = hi >= beg + 31 ? hi - 31 : beg;
     const u64 i = lo + lane;
     const bool in = i <= hi;
-    const u32 kx = in ? __ldg(a.keys + i) : NONE, ev = in ? __ldg(a.evs + i) : 0u;
+    const u32 kx = in ? __ldg(keys + i) : NONE, ev = in ? __ldg(evs + i) : 0u;
     const bool inkey = in && (kx >> 2) == k0;
     const u32 W = __ballot_sync(0xFFFFFFFFu, inkey && (kx & 3u) != IOP_LD);
     const u32 B = __ballot_sync(0xFFFFFFFFu, in && !inkey);  // other granules (below: keys sorted)
@@ -313,15 +316,15 @@ __device__ Sum tail_sum(const CheckArgs& a, u64 beg, u64 end) {
     const int bnd = hw > hbk ? hw : hbk;  // the read run is (bnd, top]
     u32 qkx = __shfl_up_sync(0xFFFFFFFFu, kx, 1), qev = __shfl_up_sync(0xFFFFFFFFu, ev, 1);
     if (lane == 0) {
-      qkx = lo > 0 ? __ldg(a.keys + lo - 1) : NONE;
-      qev = lo > 0 ? __ldg(a.evs + lo - 1) : 0u;
+      qkx = lo > 0 ? __ldg(keys + lo - 1) : NONE;
+      qev = lo > 0 ? __ldg(evs + lo - 1) : 0u;
     }
     const bool inrun = in && lane > bnd;
     bool e = false;
     if (inrun && qkx != NONE && (qkx >> 2) == k0 && (qkx & 3u) == IOP_LD) {
-      const Snap s2 = load_snap(c.snap, a.R0 + (ev >> 5));
-      const u32 qw = __ldg(&c.snap[a.R0 + (qev >> 5)].x);
-      e = !hbq(a.k, c, a.R0 + (qev >> 5), qev & 31u, qw, a.R0 + (ev >> 5), ev & 31u, s2);
+      const Snap s2 = load_snap(c.snap, R0 + (ev >> 5));
+      const u32 qw = __ldg(&c.snap[R0 + (qev >> 5)].x);
+      e = !hbq(kc, c, R0 + (qev >> 5), qev & 31u, qw, R0 + (ev >> 5), ev & 31u, s2);
     }
     const u32 I = __ballot_sync(0xFFFFFFFFu, e);
     if (I) fi = (u32)(lo + __ffs(I) - 1);  // earlier rounds hold later items
@@ -338,15 +341,15 @@ __device__ Sum tail_sum(const CheckArgs& a, u64 beg, u64 end) {
       }
       done = true;
     } else if (lo == beg) {
-      seg_at = beg == 0 || (__ldg(a.keys + beg - 1) >> 2) != k0;
+      seg_at = beg == 0 || (__ldg(keys + beg - 1) >> 2) != k0;
       sidx = beg;
       done = true;
     }
     if (done) {
-      if (seg_at && a.sh_in) {
-        const Carry C = load_carry(a.sh_in, k0);
-        const u32 evs_ = __ldg(a.evs + sidx);
-        if (carried_infl(a, C, evs_, load_snap(c.snap, a.R0 + (evs_ >> 5)))) bits |= SB_CI;
+      if (seg_at && kc->sh_in) {
+        const Carry C = load_carry(kc->sh_in, k0);
+        const u32 evs_ = __ldg(evs + sidx);
+        if (carried_infl(kc, C, evs_, load_snap(c.snap, R0 + (evs_ >> 5)))) bits |= SB_CI;
       }
       break;
     }
@@ -504,7 +507,7 @@ __device__ __forceinline__ void load_keys16(const u32* __restrict__ keys, u64 bb
   }
 }
 
-static __device__ __noinline__ Sum tail_sum_nl(const CheckArgs* a, u64 beg, u64 end) { return tail_sum(*a, beg, end); }
+static __device__ __noinline__ Sum tail_sum_nl(const K7Ctx* k, u64 beg, u64 end) { return tail_sum(k, beg, end); }
 
 // key words stream through shared memory: one chunk = KT_SWARPS blocks (+ 4 words on each side for
 // the neighbours of the first / last item), KB_STAGES chunks in flight per CTA (1-D TMA bulk copies)
@@ -665,7 +668,7 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, u32 n
       fl &= fl - 1;
       const u32 ub0 = u * U, ub1 = min(b1, ub0 + U);
       const u64 beg = (u64)ub0 * KT_BLK, end = min(n, (u64)ub1 * KT_BLK);
-      const Sum bs = tail_sum_nl(&a, beg, end);
+      const Sum bs = tail_sum_nl(a.k, beg, end);
       for (u32 q = ub0 + lane; q < ub1; q += 32) sums[q] = q + 1 == ub1 ? bs : sum_ident();
       if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = u;
     }
@@ -783,7 +786,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
           tlw = 0;
           tfi = NONE;
           tci = false;
-          if (shadow && (k & 3u) == IOP_LD && carried_infl(a, load_carry(a.sh_in, k >> 2), e, to_snap(sv))) {
+          if (shadow && (k & 3u) == IOP_LD && carried_infl(kx, load_carry(a.sh_in, k >> 2), e, to_snap(sv))) {
             tci = true;
             cmask |= 1u << j;
           }
