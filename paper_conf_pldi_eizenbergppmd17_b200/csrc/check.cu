@@ -656,22 +656,17 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, u32 n
   while (U * 2 <= G && (u64)U * 2 * 2 * nw_b <= nt) U <<= 1;
   if (blockIdx.x == 0 && threadIdx.x == 0) *unit_out = U;
   if (threadIdx.x == 0) s_carry = sum_ident();
-  // ---- units with a check: one tail walk each (flags of 32 units' blocks read at once per warp)
-  for (u32 u0 = b0 / U + wi * 32; u0 * U < b1; u0 += KT_SWARPS * 32) {
-    const u32 uu = u0 + lane;
+  // ---- units with a check: one tail walk each; units dealt to the warps round-robin, a unit's block
+  // flags read by the warp's lanes together
+  for (u32 u = b0 / U + wi; u * U < b1; u += KT_SWARPS) {
+    const u32 ub0 = u * U, ub1 = min(b1, ub0 + U);
     bool any = false;
-    if (uu * U < b1)
-      for (u32 q = 0; q < U && uu * U + q < b1; ++q) any |= bflag[uu * U + q] != 0u;
-    u32 fl = __ballot_sync(0xFFFFFFFFu, any);
-    while (fl) {
-      const u32 u = u0 + (u32)__ffs(fl) - 1u;
-      fl &= fl - 1;
-      const u32 ub0 = u * U, ub1 = min(b1, ub0 + U);
-      const u64 beg = (u64)ub0 * KT_BLK, end = min(n, (u64)ub1 * KT_BLK);
-      const Sum bs = tail_sum_nl(a.k, beg, end);
-      for (u32 q = ub0 + lane; q < ub1; q += 32) sums[q] = q + 1 == ub1 ? bs : sum_ident();
-      if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = u;
-    }
+    for (u32 q = ub0 + lane; q < ub1; q += 32) any |= bflag[q] != 0u;
+    if (!__any_sync(0xFFFFFFFFu, any)) continue;
+    const u64 beg = (u64)ub0 * KT_BLK, end = min(n, (u64)ub1 * KT_BLK);
+    const Sum bs = tail_sum_nl(a.k, beg, end);
+    for (u32 q = ub0 + lane; q < ub1; q += 32) sums[q] = q + 1 == ub1 ? bs : sum_ident();
+    if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = u;
   }
   __syncthreads();
   // ---- exclusive prefix of the CTA's block summaries, 256 at a time
