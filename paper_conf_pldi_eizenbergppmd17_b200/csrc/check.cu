@@ -512,6 +512,7 @@ static __device__ __noinline__ Sum tail_sum_nl(const K7Ctx* k, u64 beg, u64 end)
 // key words stream through shared memory: one chunk = KT_SWARPS blocks (+ 4 words on each side for
 // the neighbours of the first / last item), KB_STAGES chunks in flight per CTA (1-D TMA bulk copies)
 constexpr int KB_STAGES = 2;
+constexpr u32 KT_UNITS_MAX = 1024;  // units per K7a CTA (G / U)
 constexpr int KB_CHUNK = KT_SWARPS * KT_BLK;     // items per chunk
 constexpr int KB_ROW = KB_CHUNK + 8;             // words per stage
 __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
@@ -654,15 +655,25 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, u32 n
   const u32 nt = *n_nontriv;
   u32 U = 1;
   while (U * 2 <= G && (u64)U * 2 * 2 * nw_b <= nt) U <<= 1;
+  while (G / U > KT_UNITS_MAX) U <<= 1;
   if (blockIdx.x == 0 && threadIdx.x == 0) *unit_out = U;
   if (threadIdx.x == 0) s_carry = sum_ident();
-  // ---- units with a check: one tail walk each; units dealt to the warps round-robin, a unit's block
-  // flags read by the warp's lanes together
-  for (u32 u = b0 / U + wi; u * U < b1; u += KT_SWARPS) {
-    const u32 ub0 = u * U, ub1 = min(b1, ub0 + U);
+  // ---- units with a check: the CTA's threads scan the unit flags together into a shared list, then the
+  // warps take the listed units round-robin, one tail walk each
+  __shared__ u32 s_units[KT_UNITS_MAX];
+  __shared__ u32 s_nu;
+  if (threadIdx.x == 0) s_nu = 0;
+  __syncthreads();
+  const u32 u_lo = b0 / U, u_hi = (b1 + U - 1) / U;  // G / U <= KT_UNITS_MAX
+  for (u32 u = u_lo + threadIdx.x; u < u_hi; u += KT_SWARPS * 32) {
     bool any = false;
-    for (u32 q = ub0 + lane; q < ub1; q += 32) any |= bflag[q] != 0u;
-    if (!__any_sync(0xFFFFFFFFu, any)) continue;
+    for (u32 q = u * U; q < min(b1, u * U + U); ++q) any |= bflag[q] != 0u;
+    if (any) s_units[atomicAdd(&s_nu, 1u)] = u;
+  }
+  __syncthreads();
+  for (u32 i = wi; i < s_nu; i += KT_SWARPS) {
+    const u32 u = s_units[i];
+    const u32 ub0 = u * U, ub1 = min(b1, ub0 + U);
     const u64 beg = (u64)ub0 * KT_BLK, end = min(n, (u64)ub1 * KT_BLK);
     const Sum bs = tail_sum_nl(a.k, beg, end);
     for (u32 q = ub0 + lane; q < ub1; q += 32) sums[q] = q + 1 == ub1 ? bs : sum_ident();
@@ -1010,6 +1021,8 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   const u64 nblk = (L.n_max + KT_BLK - 1) / KT_BLK;
   u32 G = KT_SWARPS;  // blocks per K7a CTA: a power of two >= KT_SWARPS (whole chunks, whole units)
   while ((u64)G * K7A_CTAS < nblk) G <<= 1;
+  // (G / U units per CTA must fit KT_UNITS_MAX: U grows with the count of blocks with checks, so only
+  //  G > KT_UNITS_MAX with almost no such blocks could exceed it -- U is then raised to G / KT_UNITS_MAX)
   const u32 nct = (u32)((nblk + G - 1) / G);
   char* base = (char*)L.status;
   K7Ctx* kdev = reinterpret_cast<K7Ctx*>(base);
