@@ -624,6 +624,12 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
       issue(c + KB_STAGES, st);
     }
   }
+  // blocks past the item count (K7's blocks are sized from its upper bound): empty
+  for (u32 blk = b0 + threadIdx.x; blk < b1; blk += KT_SWARPS * 32)
+    if ((u64)blk * KT_BLK >= n) {
+      sums[blk] = sum_ident();
+      bflag[blk] = 0;
+    }
   segs = __reduce_add_sync(0xFFFFFFFFu, segs);
   if (lane == 0) {
     if (segs) atomicAdd(&s_segs[0], segs);
