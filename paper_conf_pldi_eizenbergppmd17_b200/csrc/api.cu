@@ -491,6 +491,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
         rm.prov_shared = prov_shared;
         rm.shared_base = (u32)(n_pages << (20 - g.G));
         shared_base = rm.shared_base;
+        launch_remap_keys(ikeys, b, slot_rank, pslots, rm, st);
       }
       n_keys = (n_pages << (20 - g.G)) + (u64)g.n_blocks * g.smem_gran;
       if (n_keys >= (1ull << 30)) return fail(c, BC_ERR_OVERFLOW, "shadow key space >= 2^30 granules");
@@ -499,11 +500,9 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
       launch_expand(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, nullptr, R0, ikeys, ievs, err, st);
     }
     cudaEventRecord(c->ev[15], st);
-    // ---- K5: stable radix sort by granule key; the first pass drops the never-written slots (and turns
-    // the fused page map's provisional keys into dense keys)
+    // ---- K5: stable radix sort by granule key; the first pass drops the never-written slots
     cudaEventRecord(c->ev[12], st);
-    const bool alt = radix_sort_pairs(ikeys, ievs, ik2, iv2, b, 2, 2 + kbits, rtmp, st, nullptr, n_items_dev, true,
-                                      fused ? &rm : nullptr);
+    const bool alt = radix_sort_pairs(ikeys, ievs, ik2, iv2, b, 2, 2 + kbits, rtmp, st, nullptr, n_items_dev, true);
     cudaEventRecord(c->ev[13], st);
     u32* skey = alt ? ik2 : ikeys;
     u32* sev = alt ? iv2 : ievs;

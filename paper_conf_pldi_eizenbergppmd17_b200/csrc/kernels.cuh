@@ -147,6 +147,7 @@ void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, co
 // fused page discovery: the page map (pmap[0, slots) = page + 1 or 0, pmap[slots, 2 slots) = written
 // flags) -> slot_rank[slot] (written pages ranked by address, else NONE), page_num[rank], *n_pages
 void launch_pagemap_rank(const u32* pmap, u32 slots, u32* slot_rank, u32* page_num, u64* n_pages, cudaStream_t st);
+void launch_remap_keys(u32* keys, u64 n, const u32* slot_rank, u32 slots, const KeyRemap& rm, cudaStream_t st);
 constexpr u32 PMAP_OVERFLOW = 4u;  // err bit: the page map filled up (the caller retries without it)
 void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st);
 

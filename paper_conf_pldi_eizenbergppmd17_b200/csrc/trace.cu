@@ -530,7 +530,7 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
           const u32 want = (u32)p + 1u;
           u32 h = (want * 0x9E3779B1u) & (pslots - 1u), slot = NONE;
           for (u32 probe = 0; probe < pslots; ++probe, h = (h + 1u) & (pslots - 1u)) {
-            u32 cur = *(volatile u32*)&pmap[h];
+            u32 cur = pmap[h];  // (a cached read: a stale 0 only costs the CAS below)
             if (cur == 0u) cur = atomicCAS(&pmap[h], 0u, want);
             if (cur == 0u || cur == want) {
               slot = h;
@@ -540,7 +540,7 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
           if (slot == NONE) {
             set_err(err, PMAP_OVERFLOW);
           } else {
-            if (op != BC_OP_LD && !*(volatile u32*)&pmap[pslots + slot]) pmap[pslots + slot] = 1u;
+            if (op != BC_OP_LD && !pmap[pslots + slot]) pmap[pslots + slot] = 1u;
             key0 = (slot << (20 - g.G)) | (u32)((a & 0xFFFFFull) >> g.G);
           }
         } else {
@@ -711,6 +711,31 @@ __global__ void __launch_bounds__(1024) k_pagemap_rank(const u32* __restrict__ p
     page_num[r] = (u32)(sp[r] >> 32);
   }
   if (t == 0) *n_pages = nw;
+}
+// provisional -> dense item keys (fused page discovery), the slot table in shared memory
+__global__ void __launch_bounds__(256) k_remap_keys(u32* __restrict__ keys, u64 n, const u32* __restrict__ slot_rank,
+                                                    u32 slots, KeyRemap rm) {
+  __shared__ u32 s_rank[PMAP_MAX];
+  for (u32 i = threadIdx.x; i < slots; i += blockDim.x) s_rank[i] = slot_rank[i];
+  __syncthreads();
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) {
+    const u32 k = keys[i];
+    if (k == KEY_DROP) continue;
+    const u32 gk = k >> 2;
+    u32 o;
+    if (gk >= rm.prov_shared) {
+      o = ((gk - rm.prov_shared + rm.shared_base) << 2) | (k & 3u);
+    } else {
+      const u32 r = s_rank[gk >> rm.off_bits];
+      o = r == NONE ? KEY_DROP : ((((r << rm.off_bits) | (gk & ((1u << rm.off_bits) - 1u))) << 2) | (k & 3u));
+    }
+    if (o != k) keys[i] = o;
+  }
+}
+void launch_remap_keys(u32* keys, u64 n, const u32* slot_rank, u32 slots, const KeyRemap& rm, cudaStream_t st) {
+  if (!n) return;
+  k_remap_keys<<<(unsigned)std::min<u64>((n + 255) / 256, 148 * 8), 256, 0, st>>>(keys, n, slot_rank, slots, rm);
+  ++g_launches;
 }
 void launch_pagemap_rank(const u32* pmap, u32 slots, u32* slot_rank, u32* page_num, u64* n_pages, cudaStream_t st) {
   k_pagemap_rank<<<1, 1024, 0, st>>>(pmap, slots, slot_rank, page_num, n_pages);
