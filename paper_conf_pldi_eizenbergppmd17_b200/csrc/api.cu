@@ -297,63 +297,43 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   uint4* hdr16 = S.alloc<uint4>(n);  // compact record headers (K2 gathers them per warp)
   cudaMemsetAsync(cnt, 0, C_N * 8, st);
   cudaMemsetAsync(wcnt, 0, 3 * (size_t)(g.n_warps + 1) * 4, st);
-  // ---- header pass (validation, counters, K1 keys, window weights)
+  cudaMemsetAsync(page_bits, 0, nwords * 4, st);
+  // ---- header pass; written pages ranked in address order from the list of non-zero bitmap words
   u32* word_list = S.alloc<u32>(nwords);
   u32* wl2 = S.alloc<u32>(nwords);
-  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, rec_w, hdr16, rec_cnt, err, st,
-                false);
+  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, rec_w, hdr16, rec_cnt, err, st);
   u32* words = word_list;
   u32* wl_prefix = wl2;
   u32* page_rank = S.alloc<u32>(nwords);
   u32* need_sort = reinterpret_cast<u32*>(cnt + C_NEED_SORT);
+  launch_page_rank(words, cnt + C_PAGE_WORDS, page_bits, page_rank, wl_prefix, cnt + C_PAGES, need_sort, 0, st);
+  cudaEventRecord(c->ev[1], st);
   u64 hc_cnt[C_N];
   u64* const hcnt = c->hcnt;
   cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
   if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "header");
   memcpy(hc_cnt, hcnt, sizeof(hc_cnt));
-  u32 herr = (u32)hc_cnt[C_ERR];
+  u32 herr = (u32)hc_cnt[C_ERR], h_need_sort = (u32)hc_cnt[C_NEED_SORT];
+  if (h_need_sort) {  // more non-zero page words than one CTA sorts: radix sort, then rank
+    const u64 nwl = hc_cnt[C_PAGE_WORDS];
+    if (radix_sort_pairs(word_list, nullptr, wl2, nullptr, nwl, 0, 23, S.alloc<char>(rs_temp_bytes(nwl)), st)) {
+      words = wl2;
+      wl_prefix = word_list;
+    }
+    launch_page_rank(words, cnt + C_PAGE_WORDS, page_bits, page_rank, wl_prefix, cnt + C_PAGES, need_sort, 1, st);
+    cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
+    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "page rank");
+    memcpy(hc_cnt, hcnt, sizeof(hc_cnt));
+  }
+  const u64 n_pages = hc_cnt[C_PAGES], n_words = hc_cnt[C_PAGE_WORDS];
   sx.lane_events = hc_cnt[C_LANE_EVENTS];
   sx.control_events = hc_cnt[C_CONTROL_EVENTS];
   sx.sync_ops = hc_cnt[C_SYNC_LANEOPS];
+  sx.written_pages = n_pages;
   if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "record header violates feasibility");
-  // Written 1-MB pages give the dense global granule keys.  One window: K4 discovers them
-  // itself while it reads the addresses (fused page map, the trace is read once); several windows (a
-  // page written in a later window must not drop an earlier window's accesses) or a full page map:
-  // a marking pass over the address rows of the written records first.
-  const u64 bound_all = hc_cnt[C_ITEM_BOUND];
-  const u64 total_w = bound_all + (u64)REC_W * n;
-  const u64 we = c->cfg.window_events ? std::min<u64>(c->cfg.window_events, WIN_MAX) : WIN_MAX;
-  const u32 pslots = std::min<u32>(PMAP_SLOTS_MAX, 1u << (29 - (20 - g.G)));
-  const u32 prov_shared = pslots << (20 - g.G);
-  bool fused = total_w <= we && g.world == 1 && (u64)g.n_blocks * g.smem_gran < (1ull << 30) - prov_shared;
-  u64 n_pages = 0, n_words = 0;
-  auto mark_and_rank = [&]() -> bc_status {
-    cudaMemsetAsync(page_bits, 0, nwords * 4, st);
-    launch_mark_pages(recs, hdr16, n, g.n_warps, page_bits, word_list, cnt, err, st);
-    launch_page_rank(words, cnt + C_PAGE_WORDS, page_bits, page_rank, wl_prefix, cnt + C_PAGES, need_sort, 0, st);
-    cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
-    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "pages");
-    if ((u32)hcnt[C_NEED_SORT]) {  // more non-zero page words than one CTA sorts: radix sort, then rank
-      const u64 nwl = hcnt[C_PAGE_WORDS];
-      if (radix_sort_pairs(word_list, nullptr, wl2, nullptr, nwl, 0, 23, S.alloc<char>(rs_temp_bytes(nwl)), st)) {
-        words = wl2;
-        wl_prefix = word_list;
-      }
-      launch_page_rank(words, cnt + C_PAGE_WORDS, page_bits, page_rank, wl_prefix, cnt + C_PAGES, need_sort, 1, st);
-      cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
-      if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "page rank");
-    }
-    if ((u32)hcnt[C_ERR] & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "global address >= 2^48");
-    n_pages = hcnt[C_PAGES];
-    n_words = hcnt[C_PAGE_WORDS];
-    return BC_OK;
-  };
-  if (!fused)
-    if (bc_status ps = mark_and_rank()) return ps;
-  cudaEventRecord(c->ev[1], st);
-  // (fused: n_pages and the keys below are known after K4)
-  u32 shared_base = fused ? prov_shared : (u32)std::min<u64>(n_pages << (20 - g.G), 0xFFFFFFFFull);
-  u64 n_keys = (n_pages << (20 - g.G)) + (u64)g.n_blocks * g.smem_gran;
+  if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "global address >= 2^48");
+  const u32 shared_base = (u32)std::min<u64>(n_pages << (20 - g.G), 0xFFFFFFFFull);
+  const u64 n_keys = (n_pages << (20 - g.G)) + (u64)g.n_blocks * g.smem_gran;
   if (n_keys >= (1ull << 30)) return fail(c, BC_ERR_OVERFLOW, "shadow key space >= 2^30 granules");
 
   // ---- K1: records grouped by warp (stable -> trace order within a warp)
@@ -421,6 +401,10 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   // ---- windows: consecutive record ranges of at most `we` weight (item upper bound +
   // REC_W per record: < 2^27 records, so window-local event ids are 32-bit); the per-granule shadow
   // state (Fig. 8) carries from one window to the next
+  const u64 bound_all = hc_cnt[C_ITEM_BOUND];
+  const u64 total_w = bound_all + (u64)REC_W * n;
+  u64 we = c->cfg.window_events ? std::min<u64>(c->cfg.window_events, WIN_MAX)
+                                : (total_w <= WIN_MAX ? WIN_MAX : (1ull << 28));
   u64* cum = S.alloc<u64>(n + 1);
   exclusive_scan_u32_u64(rec_w, cum, n, S.alloc<char>(scan_temp_bytes(n)), cum + n, st);
   const u64 nwin64 = std::max<u64>(1, (total_w + we - 1) / we);
@@ -457,10 +441,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   uint4* sh_nxt = multi ? S.alloc<uint4>(2 * n_keys) : nullptr;
   bool have_state = false;
   u64* n_items_dev = cnt + C_ITEMS;
-  int kbits = bits_for(n_keys ? n_keys - 1 : 0);
-  u32* pmap = S.alloc<u32>(2 * (size_t)pslots);
-  u32* slot_rank = S.alloc<u32>(pslots);
-  u32* pmap_pages = S.alloc<u32>(pslots);
+  const int kbits = bits_for(n_keys ? n_keys - 1 : 0);
   u64 n_r = 0, n_items = 0, pool_used = 0;
   float ms_ex = 0, ms_sort = 0, ms_chk = 0;
   for (u32 k = 0; k < nwin; ++k) {
@@ -469,36 +450,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     ++sx.windows;
     // ---- K4: expansion (static slots from the header's per-record upper bounds)
     cudaEventRecord(c->ev[14], st);
-    KeyRemap rm{};
-    if (fused) {
-      cudaMemsetAsync(pmap, 0, 2 * (size_t)pslots * sizeof(u32), st);
-      launch_expand(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, nullptr, R0, ikeys, ievs, err, st, pmap,
-                    pslots);
-      launch_pagemap_rank(pmap, pslots, slot_rank, pmap_pages, cnt + C_PAGES, st);
-      cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
-      if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "expand");
-      if ((u32)hcnt[C_ERR] & PMAP_OVERFLOW) {  // more touched pages than the map holds: mark pages, expand again
-        fused = false;
-        const u32 keep = (u32)hcnt[C_ERR] & ~PMAP_OVERFLOW;
-        cudaMemcpyAsync(err, &keep, sizeof(u32), cudaMemcpyHostToDevice, st);
-        if (bc_status ps = mark_and_rank()) return ps;
-        shared_base = (u32)std::min<u64>(n_pages << (20 - g.G), 0xFFFFFFFFull);
-        launch_expand(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, nullptr, R0, ikeys, ievs, err, st);
-      } else {
-        n_pages = hcnt[C_PAGES];
-        rm.slot_rank = slot_rank;
-        rm.off_bits = 20 - g.G;
-        rm.prov_shared = prov_shared;
-        rm.shared_base = (u32)(n_pages << (20 - g.G));
-        shared_base = rm.shared_base;
-        launch_remap_keys(ikeys, b, slot_rank, pslots, rm, st);
-      }
-      n_keys = (n_pages << (20 - g.G)) + (u64)g.n_blocks * g.smem_gran;
-      if (n_keys >= (1ull << 30)) return fail(c, BC_ERR_OVERFLOW, "shadow key space >= 2^30 granules");
-      kbits = bits_for(n_keys ? n_keys - 1 : 0);
-    } else {
-      launch_expand(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, nullptr, R0, ikeys, ievs, err, st);
-    }
+    launch_expand(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, nullptr, R0, ikeys, ievs, err, st);
     cudaEventRecord(c->ev[15], st);
     // ---- K5: stable radix sort by granule key; the first pass drops the never-written slots
     cudaEventRecord(c->ev[12], st);
@@ -557,9 +509,8 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     if (!c->races) return fail(c, BC_ERR_OOM, "race list");
     c->races_cap = std::max<u64>(total, 1);
   }
-  sx.written_pages = n_pages;
-  u32* page_num = fused ? pmap_pages : S.alloc<u32>(n_pages + 1);
-  if (n_r && !fused) launch_page_list(words, wl_prefix, page_bits, n_words, page_num, st);
+  u32* page_num = S.alloc<u32>(n_pages + 1);
+  if (n_r) launch_page_list(words, wl_prefix, page_bits, n_words, page_num, st);
   finalize_races(c->rbuf, (u32)n_r, find_blk, find_rec, nfind, g, snap, page_num, shared_base, (u32)n_keys, c->races, S,
                  st);
   cudaEventRecord(c->ev[PH_N], st);

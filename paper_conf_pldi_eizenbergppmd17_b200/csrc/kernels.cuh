@@ -93,25 +93,9 @@ class Scratch {
 };
 
 // sort.cu
-// Provisional item keys of the fused page discovery (K4 with a page map): global granule =
-// page slot << off_bits | offset, shared granule = prov_shared + block * smem_gran + offset.  The first
-// radix pass maps them to dense keys (written pages by rank in address order, then shared granules
-// from shared_base); slots of never-written pages map to KEY_DROP.
-struct KeyRemap {
-  const u32* slot_rank = nullptr;  // [slots] rank of the slot's page among the written pages, or NONE
-  u32 off_bits = 0, prov_shared = 0, shared_base = 0;
-};
-__device__ __forceinline__ u32 remap_key(const KeyRemap& m, u32 k) {
-  if (k == KEY_DROP || !m.slot_rank) return k;
-  const u32 g = k >> 2;
-  if (g >= m.prov_shared) return ((g - m.prov_shared + m.shared_base) << 2) | (k & 3u);
-  const u32 r = __ldg(m.slot_rank + (g >> m.off_bits));
-  return r == NONE ? KEY_DROP : ((((r << m.off_bits) | (g & ((1u << m.off_bits) - 1u))) << 2) | (k & 3u));
-}
 size_t rs_temp_bytes(u64 n);
 bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi, void* temp,
-                      cudaStream_t st, const u64* n_dev = nullptr, u64* n_out_dev = nullptr, bool drop = false,
-                      const KeyRemap* remap = nullptr);
+                      cudaStream_t st, const u64* n_dev = nullptr, u64* n_out_dev = nullptr, bool drop = false);
 size_t scan_temp_bytes(u64 n);
 void exclusive_scan_u32(const u32* in, u32* out, u64 n, void* temp, u64* total_dev, cudaStream_t st);
 void exclusive_scan_u32_u64(const u32* in, u64* out, u64 n, void* temp, u64* total_dev, cudaStream_t st);
@@ -123,11 +107,8 @@ constexpr u32 REC_W = 8;
 constexpr u64 WIN_MAX = (1ull << 30) - 1024;
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
                    u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_w, uint4* hdr16,
-                   u32* rec_cnt, u32* err, cudaStream_t st, bool mark_pages = true);
+                   u32* rec_cnt, u32* err, cudaStream_t st);
 void launch_window_starts(const u64* cum, u64 n, u64 we, u32 nwin, u64* starts, u64* bounds, cudaStream_t st);
-void launch_mark_pages(const bc_record* recs, const uint4* hdr16, u64 n, u32 n_warps, u32* page_bits, u32* word_list,
-                       u64* cnt, u32* err, cudaStream_t st);
-constexpr u32 PMAP_SLOTS_MAX = 4096;
 constexpr u32 WS_SMALL = 8192;  // n_warps up to which one CTA does the per-warp scans (launch_warp_scans)
 void launch_warp_scans(const u32* rec_cnt, const u32* if_cnt, const u32* bar_cnt, u32 n_warps, u32* warp_start,
                        u32* node_base, u32* bar_base, cudaStream_t st);
@@ -143,12 +124,7 @@ void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, cons
                       cudaStream_t st);
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
                    const u64* cum, u64 R0, u64 R1, const u32* gidx, u64 G0, u32* keys, u32* evs, u32* err,
-                   cudaStream_t st, u32* pmap = nullptr, u32 pmap_slots = 0);
-// fused page discovery: the page map (pmap[0, slots) = page + 1 or 0, pmap[slots, 2 slots) = written
-// flags) -> slot_rank[slot] (written pages ranked by address, else NONE), page_num[rank], *n_pages
-void launch_pagemap_rank(const u32* pmap, u32 slots, u32* slot_rank, u32* page_num, u64* n_pages, cudaStream_t st);
-void launch_remap_keys(u32* keys, u64 n, const u32* slot_rank, u32 slots, const KeyRemap& rm, cudaStream_t st);
-constexpr u32 PMAP_OVERFLOW = 4u;  // err bit: the page map filled up (the caller retries without it)
+                   cudaStream_t st);
 void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st);
 
 // sync.cu

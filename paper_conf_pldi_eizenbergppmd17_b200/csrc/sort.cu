@@ -102,7 +102,7 @@ __global__ void __launch_bounds__((1 << RB) < 1024 ? (1 << RB) : 1024) k_rs_bins
 template <int RB>
 __global__ void __launch_bounds__(RS_THREADS) k_rs_up(const u32* __restrict__ kin, u64 n_max,
                                                       const u64* __restrict__ n_dev, int drop, int shift,
-                                                      u32* __restrict__ counts, u64 tiles, KeyRemap rm) {
+                                                      u32* __restrict__ counts, u64 tiles) {
   constexpr int BINS = 1 << RB;
   __shared__ u32 h[BINS];
   const int t = threadIdx.x;
@@ -116,7 +116,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_up(const u32* __restrict__ ki
 #pragma unroll
     for (int j = 0; j < RS_ITEMS; ++j) {
       const u64 idx = base + (u64)j * RS_THREADS + t;
-      k[j] = idx < n ? remap_key(rm, kin[idx]) : KEY_DROP;
+      k[j] = idx < n ? kin[idx] : KEY_DROP;
     }
 #pragma unroll
     for (int j = 0; j < RS_ITEMS; ++j) {
@@ -201,8 +201,7 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
                                                            const u64* __restrict__ n_dev, int drop, int shift,
                                                            const u32* __restrict__ offs, u64 tiles,
                                                            const u32* __restrict__ gbase,
-                                                           const u32* __restrict__ rowtot, u64* __restrict__ n_out,
-                                                           KeyRemap rm) {
+                                                           const u32* __restrict__ rowtot, u64* __restrict__ n_out) {
   constexpr int BINS = 1 << RB;
   constexpr int DPT = BINS / RS_THREADS;  // digits per thread (1, 2 or 4)
   extern __shared__ __align__(128) unsigned char rs_smem[];
@@ -294,11 +293,7 @@ __global__ void __launch_bounds__(RS_THREADS, 2) k_rs_down(const u32* __restrict
     for (int j = 0; j < RS_ITEMS; ++j) {
       const u32 li = w * (RS_ITEMS * 32) + j * 32 + l;
       const u64 idx = base + li;
-      u32 k = idx < n ? sk[li] : KEY_DROP;
-      if (rm.slot_rank && idx < n) {  // first pass of a fused-page sort: provisional -> dense key, in place
-        k = remap_key(rm, k);
-        sk[li] = k;
-      }
+      const u32 k = idx < n ? sk[li] : KEY_DROP;
       dg[j] = (idx < n && !(drop && k == KEY_DROP)) ? ((k >> shift) & (BINS - 1)) : (u32)BINS;
 #if RS_FASTRANK
       // warp-uniform fast paths before the (MIO-bound) MATCH.ANY: 32 strictly increasing digits are
@@ -539,7 +534,7 @@ constexpr size_t SS_SMEM = (size_t)RS_SMALL * 4 * sizeof(u32) + (size_t)SS_WARPS
 __global__ void __launch_bounds__(SS_THREADS) k_sort_small(const u32* __restrict__ kin, const u32* __restrict__ vin,
                                                            u32* __restrict__ kout, u32* __restrict__ vout, u64 n_max,
                                                            const u64* __restrict__ n_dev, int drop, int bit_lo,
-                                                           int bits, u64* __restrict__ n_out, KeyRemap rm) {
+                                                           int bits, u64* __restrict__ n_out) {
   extern __shared__ __align__(16) u32 ss[];
   u32* dA = ss;                      // digits-source keys (already shifted / masked), buffer A
   u32* iA = dA + RS_SMALL;           // input indices, buffer A
@@ -555,7 +550,7 @@ __global__ void __launch_bounds__(SS_THREADS) k_sort_small(const u32* __restrict
   __syncthreads();
   for (u32 c0 = 0; c0 < n; c0 += SS_THREADS) {
     const u32 i = c0 + t;
-    const u32 k = i < n ? remap_key(rm, kin[i]) : KEY_DROP;
+    const u32 k = i < n ? kin[i] : KEY_DROP;
     const bool keep = i < n && !(drop && k == KEY_DROP);
     const u32 bal = __ballot_sync(0xFFFFFFFFu, keep);
     __shared__ u32 s_wbase[SS_WARPS];
@@ -634,7 +629,7 @@ __global__ void __launch_bounds__(SS_THREADS) k_sort_small(const u32* __restrict
   }
   for (u32 i = t; i < nk; i += SS_THREADS) {
     const u32 src = iA[i];
-    kout[i] = remap_key(rm, kin[src]);
+    kout[i] = kin[src];
     if (vout) vout[i] = vin[src];
   }
   if (t == 0 && n_out) *n_out = nk;
@@ -642,7 +637,7 @@ __global__ void __launch_bounds__(SS_THREADS) k_sort_small(const u32* __restrict
 
 template <int RB>
 static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo, int passes, void* temp,
-                       cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop, const KeyRemap& rm0) {
+                       cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop) {
   constexpr int BINS = 1 << RB;
   const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
   u32* ghist = (u32*)temp;                           // [RS_MAXP][RS_MAXB]
@@ -665,8 +660,7 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
   for (int p = 0; p < passes; ++p) {
     const int shift = bit_lo + RB * p;
     const int dr = (drop && p == 0) ? 1 : 0;
-    const KeyRemap rm = p == 0 ? rm0 : KeyRemap{};
-    k_rs_up<RB><<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles, rm); ++g_launches;
+    k_rs_up<RB><<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles); ++g_launches;
     k_rs_rows<<<BINS, RS_THREADS, 0, st>>>(counts, tiles, ghist + p * RS_MAXB); ++g_launches;
     // the digit bases come from the downsweep's own scan of the row totals, unless the kept count it
     // publishes would overwrite the item count the same launch reads (n_dev == n_out_dev)
@@ -678,7 +672,7 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
     }
     k_rs_down<RB><<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, dsmem, st>>>(
         ki, vi, ko, vo, n, nd, dr, shift, counts, tiles, gbase + p * RS_MAXB, fused ? ghist + p * RS_MAXB : nullptr,
-        fused && dr ? n_out_dev : nullptr, rm);
+        fused && dr ? n_out_dev : nullptr);
     ++g_launches;
     if (dr) nd = n_out_dev;
     u32* tk = ki; ki = ko; ko = tk;
@@ -694,8 +688,7 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
 // pass: k_rs_up (digit counts per tile) -> k_rs_rows (independent per-digit row scans + totals) ->
 // k_rs_bins (digit bases from the totals) -> k_rs_down (rank + scatter).
 bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n, int bit_lo, int bit_hi, void* temp,
-                      cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop, const KeyRemap* remap) {
-  const KeyRemap rm = remap ? *remap : KeyRemap{};
+                      cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop) {
   if (!drop && (n <= 1 || bit_hi <= bit_lo)) return false;
   if (n == 0) {
     if (n_out_dev) cudaMemsetAsync(n_out_dev, 0, 8, st);
@@ -712,7 +705,7 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
       attr[dev] = true;
     }
     k_sort_small<<<1, SS_THREADS, SS_SMEM, st>>>(keys, vals, keys_alt, vals_alt, n, n_dev, drop ? 1 : 0, bit_lo,
-                                                 bits, drop ? n_out_dev : nullptr, rm);
+                                                 bits, drop ? n_out_dev : nullptr);
     ++g_launches;
     return true;
   }
@@ -727,10 +720,10 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   int passes = std::min((bits + mb - 1) / mb, RS_MAXP);
   const int rb = std::max(8, std::min(mb, (bits + passes - 1) / passes));
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
-  if (rb == 8) rs_sort_rb<8>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop, rm);
-  else if (rb == 9) rs_sort_rb<9>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop, rm);
-  else if (rb == 10) rs_sort_rb<10>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop, rm);
-  else rs_sort_rb<11>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop, rm);
+  if (rb == 8) rs_sort_rb<8>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
+  else if (rb == 9) rs_sort_rb<9>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
+  else if (rb == 10) rs_sort_rb<10>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
+  else rs_sort_rb<11>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
   return (passes & 1) != 0;
 }
 

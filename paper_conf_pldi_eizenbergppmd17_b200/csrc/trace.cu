@@ -26,7 +26,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
                                                 u32* __restrict__ page_bits, u32* __restrict__ word_list,
                                                 u64* __restrict__ cnt, u32* __restrict__ rec_w,
                                                 uint4* __restrict__ hdr16, u32* __restrict__ rec_cnt,
-                                                u32* __restrict__ err, int mark_pages) {
+                                                u32* __restrict__ err) {
   const u32 lane = threadIdx.x & 31;
   const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const u64 r = gw * 32 + lane;
@@ -113,7 +113,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
     }
   }
   // page marking: ST / ATOM on global memory
-  u32 wr = __ballot_sync(0xFFFFFFFFu, mark_pages && valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) &&
+  u32 wr = __ballot_sync(0xFFFFFFFFu, valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) &&
                                           h.space == BC_SPACE_GLOBAL);
   while (wr) {  // HDR_ROWS records' address rows in flight at a time
     int js[HDR_ROWS];
@@ -155,45 +155,6 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
       }
     }
   }
-}
-
-// Page marking on its own (windowed runs, and the fallback of the fused page map): one warp per 32
-// records, headers from the compact copies, address rows of the global ST / ATOM records
-__global__ void __launch_bounds__(256) k_mark_pages(const bc_record* __restrict__ recs, const uint4* __restrict__ hdr16,
-                                                    u64 n, u32 n_warps, u32* __restrict__ page_bits,
-                                                    u32* __restrict__ word_list, u64* __restrict__ cnt,
-                                                    u32* __restrict__ err) {
-  const u32 lane = threadIdx.x & 31;
-  const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const u64 r = gw * 32 + lane;
-  uint4 hv = make_uint4(0, 0, 0xFFu, 0);
-  if (r < n) hv = __ldg(hdr16 + r);
-  const u32 op = hv.z & 0xFFu, space = (hv.z >> 8) & 0xFFu;
-  u32 wr = __ballot_sync(0xFFFFFFFFu, r < n && hv.x < n_warps && (op == BC_OP_ST || op == BC_OP_ATOM) &&
-                                          space == BC_SPACE_GLOBAL);
-  while (wr) {
-    const int j = __ffs(wr) - 1;
-    wr &= wr - 1;
-    const u32 m = __shfl_sync(0xFFFFFFFFu, hv.y, j);
-    if (!((m >> lane) & 1u)) continue;
-    const u64 p = __ldg(&recs[gw * 32 + j].addr[lane]) >> 20;
-    if (p >= (1ull << 28)) {
-      set_err(err, ERR_OVERFLOW);
-      continue;
-    }
-    const u32 bit = 1u << (p & 31);
-    u32* wp = &page_bits[p >> 5];
-    if (!(*(volatile u32*)wp & bit) && atomicOr(wp, bit) == 0u) {
-      const u64 at = atomicAdd((unsigned long long*)&cnt[C_PAGE_WORDS], 1ull);
-      word_list[at] = (u32)(p >> 5);
-    }
-  }
-}
-void launch_mark_pages(const bc_record* recs, const uint4* hdr16, u64 n, u32 n_warps, u32* page_bits, u32* word_list,
-                       u64* cnt, u32* err, cudaStream_t st) {
-  if (!n) return;
-  k_mark_pages<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(recs, hdr16, n, n_warps, page_bits, word_list, cnt, err);
-  ++g_launches;
 }
 
 // warp_start[w] = first index of warp w in the warp-sorted record list (lower bound)
@@ -445,7 +406,7 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
                                                        const u64* __restrict__ cum, u64 R0, u64 R1,
                                                        const u32* __restrict__ gidx, u64 G0,
                                                        u32* __restrict__ okeys, u32* __restrict__ oevs,
-                                                       u32* __restrict__ err, u32* __restrict__ pmap, u32 pslots) {
+                                                       u32* __restrict__ err) {
   extern __shared__ __align__(128) unsigned char ex_smem[];
   bc_record* buf = reinterpret_cast<bc_record*>(ex_smem);                    // [EX_STAGES][EX_REC]
   u64* bar = reinterpret_cast<u64*>(ex_smem + sizeof(bc_record) * EX_REC * EX_STAGES);
@@ -522,33 +483,14 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
         key0 = shared_base + blk_of(g, hwarp) * g.smem_gran + (u32)(a >> g.G);
       } else {
         const u64 p = a >> 20;
-        if (p >= (1ull << 28)) {
-          ovf = true;
-        } else if (pmap) {
-          // fused page discovery: the page's slot in the map (claimed on first touch, linear probing);
-          // writes mark the slot; the first radix pass turns slot keys into dense keys
-          const u32 want = (u32)p + 1u;
-          u32 h = (want * 0x9E3779B1u) & (pslots - 1u), slot = NONE;
-          for (u32 probe = 0; probe < pslots; ++probe, h = (h + 1u) & (pslots - 1u)) {
-            u32 cur = pmap[h];  // (a cached read: a stale 0 only costs the CAS below)
-            if (cur == 0u) cur = atomicCAS(&pmap[h], 0u, want);
-            if (cur == 0u || cur == want) {
-              slot = h;
-              break;
-            }
-          }
-          if (slot == NONE) {
-            set_err(err, PMAP_OVERFLOW);
-          } else {
-            if (op != BC_OP_LD && !pmap[pslots + slot]) pmap[pslots + slot] = 1u;
-            key0 = (slot << (20 - g.G)) | (u32)((a & 0xFFFFFull) >> g.G);
-          }
-        } else {
+        if (p < (1ull << 28)) {
           const u32 pw = __ldg(&page_bits[p >> 5]);
           const u32 bit = (u32)(p & 31);
           if ((pw >> bit) & 1u)
             key0 = (__ldg(&page_rank[p >> 5]) + __popc(pw & ((1u << bit) - 1u))) << (20 - g.G) |
                    (u32)((a & 0xFFFFFull) >> g.G);
+        } else {
+          ovf = true;
         }
       }
       const u32 o = uoj + (u32)__popc(hmask & lt) * nk;  // window slots < 2^30
@@ -670,87 +612,15 @@ __global__ void __launch_bounds__(1024) k_page_rank(u32* __restrict__ words, con
   if (t == 0) *n_pages_dev = s_carry;
 }
 
-// Fused page discovery: one CTA ranks the written pages of the page map in address order
-// (bitonic sort of (page, slot) in shared memory) -> slot_rank[slot] = rank or NONE (never written),
-// page_num[rank] = page, *n_pages.
-constexpr u32 PMAP_MAX = 4096;
-__global__ void __launch_bounds__(1024) k_pagemap_rank(const u32* __restrict__ pmap, u32 slots, u32* __restrict__ slot_rank,
-                                                       u32* __restrict__ page_num, u64* __restrict__ n_pages) {
-  __shared__ unsigned long long sp[PMAP_MAX];
-  __shared__ u32 s_n;
-  const u32 t = threadIdx.x;
-  if (t == 0) s_n = 0;
-  __syncthreads();
-  for (u32 i = t; i < slots; i += 1024) {
-    slot_rank[i] = NONE;
-    const u32 pg = pmap[i];
-    if (pg && pmap[slots + i]) sp[atomicAdd(&s_n, 1u)] = ((unsigned long long)(pg - 1u) << 32) | i;
-  }
-  __syncthreads();
-  const u32 nw = s_n;
-  u32 P = 1;
-  while (P < nw) P <<= 1;
-  for (u32 i = nw + t; i < P; i += 1024) sp[i] = ~0ull;
-  __syncthreads();
-  for (u32 k = 2; k <= P; k <<= 1)
-    for (u32 j = k >> 1; j > 0; j >>= 1) {
-      for (u32 i = t; i < P; i += 1024) {
-        const u32 ij = i ^ j;
-        if (ij > i) {
-          const unsigned long long a = sp[i], b = sp[ij];
-          if (((i & k) == 0) == (a > b)) {
-            sp[i] = b;
-            sp[ij] = a;
-          }
-        }
-      }
-      __syncthreads();
-    }
-  for (u32 r = t; r < nw; r += 1024) {
-    slot_rank[(u32)sp[r]] = r;
-    page_num[r] = (u32)(sp[r] >> 32);
-  }
-  if (t == 0) *n_pages = nw;
-}
-// provisional -> dense item keys (fused page discovery), the slot table in shared memory
-__global__ void __launch_bounds__(256) k_remap_keys(u32* __restrict__ keys, u64 n, const u32* __restrict__ slot_rank,
-                                                    u32 slots, KeyRemap rm) {
-  __shared__ u32 s_rank[PMAP_MAX];
-  for (u32 i = threadIdx.x; i < slots; i += blockDim.x) s_rank[i] = slot_rank[i];
-  __syncthreads();
-  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) {
-    const u32 k = keys[i];
-    if (k == KEY_DROP) continue;
-    const u32 gk = k >> 2;
-    u32 o;
-    if (gk >= rm.prov_shared) {
-      o = ((gk - rm.prov_shared + rm.shared_base) << 2) | (k & 3u);
-    } else {
-      const u32 r = s_rank[gk >> rm.off_bits];
-      o = r == NONE ? KEY_DROP : ((((r << rm.off_bits) | (gk & ((1u << rm.off_bits) - 1u))) << 2) | (k & 3u));
-    }
-    if (o != k) keys[i] = o;
-  }
-}
-void launch_remap_keys(u32* keys, u64 n, const u32* slot_rank, u32 slots, const KeyRemap& rm, cudaStream_t st) {
-  if (!n) return;
-  k_remap_keys<<<(unsigned)std::min<u64>((n + 255) / 256, 148 * 8), 256, 0, st>>>(keys, n, slot_rank, slots, rm);
-  ++g_launches;
-}
-void launch_pagemap_rank(const u32* pmap, u32 slots, u32* slot_rank, u32* page_num, u64* n_pages, cudaStream_t st) {
-  k_pagemap_rank<<<1, 1024, 0, st>>>(pmap, slots, slot_rank, page_num, n_pages);
-  ++g_launches;
-}
-
 // --------------------------------------------------------------------- host launchers
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
                    u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_w, uint4* hdr16,
-                   u32* rec_cnt, u32* err, cudaStream_t st, bool mark_pages) {
+                   u32* rec_cnt, u32* err, cudaStream_t st) {
   u64 warps = (g.n_recs + 31) / 32;
   if (warps == 0) return;
   u64 blocks = (warps + 7) / 8;
   k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt,
-                                             rec_w, hdr16, rec_cnt, err, mark_pages ? 1 : 0); ++g_launches;
+                                             rec_w, hdr16, rec_cnt, err); ++g_launches;
 }
 
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st) {
@@ -861,7 +731,7 @@ void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStrea
 
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
                    const u64* cum, u64 R0, u64 R1, const u32* gidx, u64 G0, u32* keys, u32* evs, u32* err,
-                   cudaStream_t st, u32* pmap, u32 pmap_slots) {
+                   cudaStream_t st) {
   const u64 chunks = (R1 - R0 + EX_REC - 1) / EX_REC;
   if (!chunks) return;
   const size_t smem = sizeof(bc_record) * EX_REC * EX_STAGES + 8 * EX_STAGES;
@@ -878,7 +748,7 @@ void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, co
   }
   const unsigned gr = (unsigned)std::min<u64>(chunks, (u64)grid[dev]);
   k_expand<<<gr, EX_THREADS, smem, st>>>(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, gidx, G0, keys, evs,
-                                         err, pmap, pmap_slots);
+                                         err);
   ++g_launches;
 }
 
