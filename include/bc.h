@@ -143,6 +143,12 @@ typedef struct bc_config {
                                          process per GPU; bc_init is collective                     */
   struct bc_group* group;             /* in-process transport: the ranks are contexts of this process,
                                          one host thread each (bc_group_create_local)              */
+  /* Declared global allocations (the paper's global shadow page table):
+   * (base, size) byte ranges.  Required for streaming (bc_stream_open): the page set, and with it every
+   * shadow key, is then fixed before the first record arrives; a global access outside the ranges fails
+   * the detect with BC_ERR_INVALID_ARG.  Ignored otherwise. */
+  uint64_t global_ranges[2 * 64];
+  uint32_t n_global_ranges;
 } bc_config;
 
 typedef struct bc_stats {
@@ -196,6 +202,41 @@ bc_status bc_load_trace_shard(bc_ctx* ctx, const bc_record* recs, const uint32_t
  * ctx's stream, synchronizes before return. */
 bc_status bc_split_warps(bc_ctx* ctx, const bc_record* recs, uint64_t n_recs, uint32_t ws, bc_record* out,
                          uint64_t* origin, uint64_t cap, uint64_t* n_out);
+
+/* ---- streaming ingest (the device queue of Fig. 6) ----
+ * The traced program pushes its records into a lock-free device queue while it runs; the context
+ * consumes committed ranges as trace windows (row a5) while the producer keeps going, carrying every
+ * granule's 32-B shadow state from window to window.  Queue layout (device memory, 8-B aligned):
+ *   uint64_t write_head;   reservations: a producer takes ticket t = the record's trace position
+ *   uint64_t commit_head;  records [0, commit_head) are complete; a producer commits ticket t (stores
+ *                          t + 1) after writing its record, once commit_head == t (in ticket order)
+ *   uint64_t read_head;    records [0, read_head) have been consumed; a producer waits while
+ *                          t >= read_head + capacity (ring full)
+ *   uint64_t capacity;     ring slots
+ *   uint64_t error;        non-zero: a producer gave up (waited > ~10 s for room or its turn)
+ *   uint64_t pad[3];
+ *   bc_record ring[capacity];   record t lives in ring[t % capacity]
+ * bc_stream_open: allocate the queue (queue_records slots; *queue_dev = its device address) and room for
+ *   max_records records of trace; needs bc_config.global_ranges.  Starts the session's drain thread,
+ *   which moves committed records from the ring into the trace and advances read_head with copy-engine
+ *   transfers on its own (highest-priority) stream: the ring is served even while a window check waits
+ *   for SMs the producer holds.  The trace so far is the context's loaded trace (bc_load_trace is not
+ *   used in a streaming session).  Preloads every kernel a poll launches (CUDA lazy loading would
+ *   otherwise make a first launch wait for the running producer).
+ * bc_stream_poll: once at least min_window drained records are new (or finish = 1) check them as one
+ *   window; returns BC_OK with nothing checked when too few are new.  finish = 1 is called after the
+ *   producer has finished (e.g. its stream synchronised): it waits for the drain thread to take
+ *   everything committed, checks the rest and makes the race list available to bc_races (the session
+ *   ends).  Errors: as bc_detect, BC_ERR_STATE (no session / the producer reserved records it never
+ *   committed), BC_ERR_TRUNCATED (more records than max_records), BC_ERR_INVALID_ARG (producer error,
+ *   undeclared global access).  Any error ends the session.
+ * bc_queue_push: a stand-in producer (the instrumented kernel of the paper): pushes records recs[0, n)
+ *   (device memory, trace order) with tickets 0 .. n-1 through the protocol above, on `stream`
+ *   (cudaStream_t), asynchronously; run it concurrently with bc_stream_poll. */
+bc_status bc_stream_open(bc_ctx* ctx, uint64_t queue_records, uint64_t max_records, uint64_t min_window,
+                         void** queue_dev);
+bc_status bc_stream_poll(bc_ctx* ctx, int finish, bc_stats* out);
+bc_status bc_queue_push(void* queue_dev, const bc_record* recs, uint64_t n_recs, void* stream);
 
 /* 128-byte NCCL unique id for bc_config.nccl_unique_id (call on rank 0 only).  BC_ERR_NCCL if no NCCL
  * library can be loaded (libbc dlopens the libnccl.so.2 already in the process, else the system's). */

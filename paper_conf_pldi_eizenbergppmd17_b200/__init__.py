@@ -40,7 +40,8 @@ F_COUNT_GATHERS = 4  # statistics: fill stats["clock_gathers"] (one extra pass)
 
 EXPORTS = sorted(["bc_init", "bc_load_trace", "bc_load_values", "bc_detect", "bc_races", "bc_races_device",
                   "bc_destroy", "bc_status_string", "bc_last_error", "bc_phase_name", "bc_load_trace_shard",
-                  "bc_nccl_unique_id", "bc_group_create_local", "bc_group_destroy", "bc_split_warps"])
+                  "bc_nccl_unique_id", "bc_group_create_local", "bc_group_destroy", "bc_split_warps",
+                  "bc_stream_open", "bc_stream_poll", "bc_queue_push"])
 
 
 class BcError(RuntimeError):
@@ -60,7 +61,8 @@ class _Config(ctypes.Structure):
                 ("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("stream", ctypes.c_void_p), ("window_events", ctypes.c_uint64),
                 ("dev_alloc", _ALLOC_FN), ("dev_free", _FREE_FN), ("alloc_user", ctypes.c_void_p),
-                ("nccl_unique_id", ctypes.c_void_p), ("group", ctypes.c_void_p)]
+                ("nccl_unique_id", ctypes.c_void_p), ("group", ctypes.c_void_p),
+                ("global_ranges", ctypes.c_uint64 * 128), ("n_global_ranges", ctypes.c_uint32)]
 
 
 class _Stats(ctypes.Structure):
@@ -112,6 +114,13 @@ def lib():
         L.bc_group_create_local.restype = ctypes.c_int
         L.bc_group_create_local.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_void_p)]
         L.bc_group_destroy.argtypes = [ctypes.c_void_p]
+        L.bc_stream_open.restype = ctypes.c_int
+        L.bc_stream_open.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64,
+                                     ctypes.POINTER(ctypes.c_void_p)]
+        L.bc_stream_poll.restype = ctypes.c_int
+        L.bc_stream_poll.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.POINTER(_Stats)]
+        L.bc_queue_push.restype = ctypes.c_int
+        L.bc_queue_push.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p]
         L.bc_split_warps.restype = ctypes.c_int
         L.bc_split_warps.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32,
                                      ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
@@ -158,13 +167,15 @@ class Context:
     """One traced launch geometry on one GPU (bc_init ... bc_destroy)."""
 
     def __init__(self, geometry: dict, device: int = 0, flags: int = 0, stream=None, rank: int = 0, world: int = 1,
-                 window_events: int = 0, allocator=None, nccl_id: bytes = None, group: "LocalGroup" = None):
+                 window_events: int = 0, allocator=None, nccl_id: bytes = None, group: "LocalGroup" = None,
+                 global_ranges=None):
         """rank / world > 1: address-sharded check (bc.h bc_config.rank/world): every rank loads
         the same trace and reports the races of the shadow granules it owns; merge the per-rank
         lists with merge_races() or gather_races().  window_events: bc_config.window_events (0 =
         auto).  allocator: None (cudaMalloc), "torch" (torch's caching allocator) or a
         (dev_alloc, dev_free) pair of ctypes callbacks.  nccl_id (128 bytes of nccl_unique_id() from
-        rank 0) or group (LocalGroup): the block-sharded multi-GPU check (load_trace_shard)."""
+        rank 0) or group (LocalGroup): the block-sharded multi-GPU check (load_trace_shard).
+        global_ranges: [(base, size), ...] declared global allocations (required for streaming)."""
         L = lib()
         grid = tuple(geometry["grid"]) + (1,) * (3 - len(geometry["grid"]))
         block = tuple(geometry["block"]) + (1,) * (3 - len(geometry["block"]))
@@ -185,6 +196,12 @@ class Context:
             c.nccl_unique_id = ctypes.cast(self._nccl_id, ctypes.c_void_p)
         if group is not None:
             c.group = group.handle
+        if global_ranges:
+            if len(global_ranges) > 64:
+                raise ValueError("at most 64 global ranges")
+            for i, (base, size) in enumerate(global_ranges):
+                c.global_ranges[2 * i], c.global_ranges[2 * i + 1] = int(base), int(size)
+            c.n_global_ranges = len(global_ranges)
         self._alloc = None
         if allocator is not None:
             self._alloc = torch_allocator() if allocator == "torch" else tuple(allocator)
@@ -236,6 +253,19 @@ class Context:
         self._keep, self._keep_idx = a, idx
         return self._check(L.bc_load_trace_shard(self._h, ctypes.c_void_p(a.ctypes.data if n else 0),
                                                   ctypes.c_void_p(idx.ctypes.data if n else 0), n, n_global, 0))
+
+    def stream_open(self, queue_records: int, max_records: int, min_window: int = 1):
+        """bc_stream_open: returns the device address of the record queue (bc.h layout)."""
+        q = ctypes.c_void_p()
+        self._check(lib().bc_stream_open(self._h, queue_records, max_records, min_window, ctypes.byref(q)))
+        return q.value
+
+    def stream_poll(self, finish: bool = False, allow=()):
+        """bc_stream_poll: consume committed records, check a window when enough are new; finish=True
+        drains the queue and finalises the race list.  Returns (status, stats)."""
+        s = _Stats()
+        st = self._check(lib().bc_stream_poll(self._h, 1 if finish else 0, ctypes.byref(s)), allow)
+        return st, _stats_dict(s)
 
     def load_values(self, values):
         """bc_load_values: per-lane store values [n_records, 32] (uint64) as a host
@@ -325,6 +355,16 @@ def split_warps(records, geometry: dict, ws: int, device: int = 0):
     g2 = dict(geometry)
     g2["warp_size"] = ws
     return out[:m * RECORD_BYTES], g2, org[:m]
+
+
+def queue_push(queue: int, records, stream=None):
+    """bc_queue_push: the stand-in producer pushes a CUDA uint8 tensor of records through the queue on
+    `stream` (a torch.cuda.Stream or raw handle), asynchronously.  Marshalling only."""
+    n = records.numel() // RECORD_BYTES
+    h = stream.cuda_stream if hasattr(stream, "cuda_stream") else (stream or 0)
+    st = lib().bc_queue_push(ctypes.c_void_p(queue), ctypes.c_void_p(records.data_ptr()), n, ctypes.c_void_p(h))
+    if st != OK:
+        raise BcError(st, "queue push")
 
 
 def nccl_unique_id() -> bytes:

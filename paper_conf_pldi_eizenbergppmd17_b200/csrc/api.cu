@@ -6,6 +6,7 @@
 // all on cfg.stream; every phase is bracketed by cudaEvents for bc_stats.ms_kernel.
 #include <algorithm>
 #include <atomic>
+#include <chrono>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -99,6 +100,7 @@ bc_status check_window(bc_ctx* c, CheckLaunch& L, u64 b, u64* cnt, u64& n_r, u64
   }
   if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "infeasible trace");
   if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "index overflow / sync lookup step cap");
+  if (herr & ERR_UNDECLARED) return fail(c, BC_ERR_INVALID_ARG, "global access outside bc_config.global_ranges");
   n_r = (u32)hcnt[C_RACES];
   pool_used = (u32)hcnt[C_POOL];
   wo.items = hcnt[C_ITEMS];
@@ -106,6 +108,112 @@ bc_status check_window(bc_ctx* c, CheckLaunch& L, u64 b, u64* cnt, u64& n_r, u64
   wo.gathers = hcnt[C_GATHERS];
   cudaEventElapsedTime(&wo.ms_check, c->ev[10], c->ev[11]);
   return BC_OK;
+}
+
+// ---------------------------------------------------------------- streaming ingest (row f1)
+// Queue header (bc.h): write_head, commit_head, read_head, capacity, error, pad[3]; ring after 64 B.
+enum { Q_WRITE = 0, Q_COMMIT, Q_READ, Q_CAP, Q_ERROR, Q_HDR = 8 };
+
+// Stand-in producer: one warp per record, persistent warps taking records in increasing order (so the
+// warp that must commit before another is always resident).  Ticket t = the record's trace position:
+// wait for ring room (read_head), write the 272-B record, fence, wait for commit_head == t, commit.
+__global__ void __launch_bounds__(256) k_queue_push(u64* __restrict__ q, const bc_record* __restrict__ recs, u64 n) {
+  const u64 w = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = ((u64)gridDim.x * blockDim.x) >> 5;
+  const u32 lane = threadIdx.x & 31;
+  volatile u64* vq = q;
+  const u64 cap = vq[Q_CAP];
+  bc_record* ring = reinterpret_cast<bc_record*>(q + Q_HDR);
+  for (u64 t = w; t < n; t += nw) {
+    if (lane == 0) atomicMax((unsigned long long*)&q[Q_WRITE], (unsigned long long)(t + 1));  // reservation
+    const long long t0 = clock64();
+    bool ok = true;
+    while (t >= vq[Q_READ] + cap) {  // ring full: wait for the consumer
+      if (vq[Q_ERROR] || clock64() - t0 > 20000000000ll) { ok = false; break; }
+    }
+    if (__any_sync(0xFFFFFFFFu, !ok)) {
+      if (lane == 0) vq[Q_ERROR] = 1;
+      return;
+    }
+    const u32* src = reinterpret_cast<const u32*>(recs + t);
+    u32* dst = reinterpret_cast<u32*>(ring + t % cap);
+    for (u32 i = lane; i < sizeof(bc_record) / 4; i += 32) dst[i] = __ldg(src + i);
+    __threadfence();
+    __syncwarp();
+    if (lane == 0) {
+      const long long t1 = clock64();
+      while (vq[Q_COMMIT] != t) {  // commits in ticket order
+        if (vq[Q_ERROR] || clock64() - t1 > 20000000000ll) {
+          vq[Q_ERROR] = 1;
+          break;
+        }
+      }
+      __threadfence();
+      vq[Q_COMMIT] = t + 1;
+    }
+    __syncwarp();
+    if (vq[Q_ERROR]) return;
+  }
+}
+
+// The session's drain thread (the consumer half of Fig. 6's queue).  It reads the heads, copies the
+// newly committed records out of the ring into the trace buffer and then publishes the new read head,
+// all with copy-engine transfers on its own stream: no SM is needed, so a producer that fills the GPU
+// and waits on a full ring is always served, whatever the window checks are waiting for.
+static void drain_loop(bc_ctx* c) {
+  cudaSetDevice(c->cfg.device);
+  cudaStream_t ds = c->dstream;
+  u64* h = c->dhdr;
+  const bc_record* ring = reinterpret_cast<const bc_record*>(c->queue + Q_HDR);
+  const u64 cap = c->queue_cap;
+  u64 done = 0;
+  int idle = 0;
+  while (!c->drain_stop.load(std::memory_order_acquire)) {
+    cudaMemcpyAsync(h, c->queue, Q_HDR * sizeof(u64), cudaMemcpyDeviceToHost, ds);
+    if (cudaStreamSynchronize(ds) != cudaSuccess) {
+      c->drain_err.store(BC_ERR_CUDA);
+      return;
+    }
+    if (h[Q_ERROR]) {
+      c->drain_err.store(BC_ERR_INVALID_ARG);
+      return;
+    }
+    const u64 committed = h[Q_COMMIT], w = h[Q_WRITE];
+    if (committed > c->sbuf_cap) {
+      c->drain_err.store(BC_ERR_TRUNCATED);
+      h[Q_ERROR] = 1;  // stop the producer
+      cudaMemcpyAsync(c->queue + Q_ERROR, h + Q_ERROR, sizeof(u64), cudaMemcpyHostToDevice, ds);
+      cudaStreamSynchronize(ds);
+      return;
+    }
+    if (committed > done) {
+      for (u64 t = done; t < committed;) {  // two copies across the wrap
+        const u64 slot = t % cap;
+        const u64 m = std::min<u64>(committed - t, cap - slot);
+        cudaMemcpyAsync(c->sbuf + t, ring + slot, m * sizeof(bc_record), cudaMemcpyDeviceToDevice, ds);
+        t += m;
+      }
+      h[Q_HDR] = committed;  // the slots are free once the copies are done (stream order)
+      cudaMemcpyAsync(c->queue + Q_READ, h + Q_HDR, sizeof(u64), cudaMemcpyHostToDevice, ds);
+      if (cudaStreamSynchronize(ds) != cudaSuccess) {
+        c->drain_err.store(BC_ERR_CUDA);
+        return;
+      }
+      done = committed;
+      c->drained.store(done, std::memory_order_release);
+      idle = 0;
+    } else if (++idle > 64) {
+      std::this_thread::sleep_for(std::chrono::microseconds(50));
+    }
+    c->wseen.store(w, std::memory_order_release);
+    c->dgen.fetch_add(1, std::memory_order_acq_rel);
+  }
+}
+
+static void drain_stop(bc_ctx* c) {
+  if (c->drainer.joinable()) {
+    c->drain_stop.store(true, std::memory_order_release);
+    c->drainer.join();
+  }
 }
 
 extern "C" {
@@ -212,6 +320,7 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
 void bc_destroy(bc_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->cfg.device);
+  drain_stop(c);
   if (c->stream) cudaStreamSynchronize(c->stream);
   c->da.free(c->owned, c->owned_cap);
   c->da.free(c->values_owned, c->values_cap);
@@ -220,9 +329,16 @@ void bc_destroy(bc_ctx* c) {
   c->da.free(c->pool, c->pool_cap * sizeof(uint2));
   c->da.free(c->gidx_owned, c->gidx_cap);
   for (int i = 0; i < 6; ++i) c->da.free(c->xbuf[i], c->xcap[i]);
+  c->da.free(c->queue, c->queue_bytes);
+  c->da.free(c->sbuf, c->sbuf_cap * sizeof(bc_record));
+  c->da.free(c->granges, 2 * 64 * sizeof(u64));
+  for (int q = 0; q < 2; ++q) c->da.free(c->sh[q], c->sh_bytes);
   c->arena.free_all();
+  if (c->stream) cudaStreamSynchronize(c->stream);  // the stream-ordered frees
   delete c->comm;
   if (c->hcnt) cudaFreeHost(c->hcnt);
+  if (c->dhdr) cudaFreeHost(c->dhdr);
+  if (c->dstream) cudaStreamDestroy(c->dstream);
   for (int i = 0; i < 16; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
   if (c->own_stream) cudaStreamDestroy(c->stream);
@@ -263,10 +379,11 @@ bc_status bc_load_trace(bc_ctx* c, const bc_record* recs, uint64_t n, int on_dev
   return BC_OK;
 }
 
-static bc_status detect_impl(bc_ctx* c, Scratch& S) {
+static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
   cudaStream_t st = c->stream;
   Geo g = c->g;
   if (c->values) g.flags |= GEO_F_VALUES;
+  if (sw) g.flags |= GEO_F_DECLARED;  // streaming: the page set is the declared allocations
   const u64 n = g.n_recs;
   const bc_record* recs = c->trace;
   bc_stats& sx = c->stats;
@@ -301,7 +418,9 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   // ---- header pass; written pages ranked in address order from the list of non-zero bitmap words
   u32* word_list = S.alloc<u32>(nwords);
   u32* wl2 = S.alloc<u32>(nwords);
-  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, rec_w, hdr16, rec_cnt, err, st);
+  launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, rec_w, hdr16, rec_cnt, err, st,
+                sw == nullptr);
+  if (sw) launch_mark_ranges(c->granges, c->cfg.n_global_ranges, page_bits, word_list, cnt, err, st);
   u32* words = word_list;
   u32* wl_prefix = wl2;
   u32* page_rank = S.alloc<u32>(nwords);
@@ -367,7 +486,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   u32* find_cnt = reinterpret_cast<u32*>(cnt + C_FINDINGS);
   launch_replay(hdr16, wrec, nullptr, warp_start, g, node_base, bar_base, snap, nodes, bar_rec, bar_next, find_blk,
                 find_rec, find_cnt, err, st);
-  launch_barriers(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err, st);
+  launch_barriers(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err, st, sw && !sw->final);
   launch_snap_blab(snap, n, g.wpb, g.n_warps, n_bar, bar_base, blockR, st);
   cudaEventRecord(c->ev[3], st);
   bc_status cs = cuda_check(c, "replay");
@@ -403,15 +522,24 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   // state (Fig. 8) carries from one window to the next
   const u64 bound_all = hc_cnt[C_ITEM_BOUND];
   const u64 total_w = bound_all + (u64)REC_W * n;
-  u64 we = c->cfg.window_events ? std::min<u64>(c->cfg.window_events, WIN_MAX)
-                                : (total_w <= WIN_MAX ? WIN_MAX : (1ull << 28));
+  const u64 we = c->cfg.window_events ? std::min<u64>(c->cfg.window_events, WIN_MAX) : WIN_MAX;
   u64* cum = S.alloc<u64>(n + 1);
   exclusive_scan_u32_u64(rec_w, cum, n, S.alloc<char>(scan_temp_bytes(n)), cum + n, st);
-  const u64 nwin64 = std::max<u64>(1, (total_w + we - 1) / we);
+  const u64 nwin64 = sw ? 1 : std::max<u64>(1, (total_w + we - 1) / we);
   if (nwin64 >= (1ull << 31)) return fail(c, BC_ERR_INVALID_ARG, "window_events too small for this trace");
   const u32 nwin = (u32)nwin64;
   std::vector<u64> wst(nwin + 1), wbd(nwin);
-  if (nwin == 1) {
+  if (sw) {  // streaming: the new records [R0, n) are the window
+    u64 c01[2] = {0, 0};
+    cudaMemcpyAsync(&c01[0], cum + sw->R0, 8, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(&c01[1], cum + n, 8, cudaMemcpyDeviceToHost, st);
+    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "windows");
+    wst[0] = sw->R0;
+    wst[1] = n;
+    wbd[0] = (c01[1] - c01[0]) - (u64)REC_W * (n - sw->R0);
+    if (n - sw->R0 >= (1ull << 27) || c01[1] - c01[0] > WIN_MAX)
+      return fail(c, BC_ERR_OVERFLOW, "stream window too large: poll more often");
+  } else if (nwin == 1) {
     wst[0] = 0;
     wst[1] = n;
     wbd[0] = bound_all;
@@ -430,19 +558,38 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
       maxb = std::max(maxb, wbd[k]);
       last_win = (int)k;
     }
-  const bool multi = nwin > 1;
+  const bool multi = nwin > 1 || sw;
   u32* ikeys = S.alloc<u32>(maxb + 1);
   u32* ievs = S.alloc<u32>(maxb + 1);
   u32* ik2 = S.alloc<u32>(maxb + 1);
   u32* iv2 = S.alloc<u32>(maxb + 1);
   void* rtmp = S.alloc<char>(rs_temp_bytes(maxb));
   void* cstatus = S.alloc<char>(check_status_bytes(maxb));
-  uint4* sh_cur = multi ? S.alloc<uint4>(2 * n_keys) : nullptr;  // entries after the last window (double buffer)
-  uint4* sh_nxt = multi ? S.alloc<uint4>(2 * n_keys) : nullptr;
+  uint4* sh_cur = nullptr;  // entries after the last window (double buffer)
+  uint4* sh_nxt = nullptr;
   bool have_state = false;
+  if (sw) {  // a streaming session keeps its tables across polls (the declared page set fixes n_keys)
+    const size_t bytes = 2 * n_keys * sizeof(uint4);
+    if (!c->sh[0] || c->sh_bytes != bytes) {
+      for (int q = 0; q < 2; ++q) {
+        c->da.free(c->sh[q], c->sh_bytes);
+        c->sh[q] = (uint4*)c->da.alloc(bytes);
+        if (!c->sh[q]) return fail(c, BC_ERR_OOM, "stream shadow tables");
+      }
+      c->sh_bytes = bytes;
+    }
+    sh_cur = c->sh[c->sh_cur];
+    sh_nxt = c->sh[c->sh_cur ^ 1];
+    have_state = c->have_state;
+    if (sw->final) last_win = 0;
+    else last_win = -2;  // the window writes entries for the next poll
+  } else if (multi) {
+    sh_cur = S.alloc<uint4>(2 * n_keys);
+    sh_nxt = S.alloc<uint4>(2 * n_keys);
+  }
   u64* n_items_dev = cnt + C_ITEMS;
   const int kbits = bits_for(n_keys ? n_keys - 1 : 0);
-  u64 n_r = 0, n_items = 0, pool_used = 0;
+  u64 n_r = sw ? c->s_nr : 0, n_items = 0, pool_used = sw ? c->s_pool : 0;
   float ms_ex = 0, ms_sort = 0, ms_chk = 0;
   for (u32 k = 0; k < nwin; ++k) {
     const u64 R0 = wst[k], R1 = wst[k + 1], b = wbd[k];
@@ -490,7 +637,19 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
     if (sh_out) {
       std::swap(sh_cur, sh_nxt);
       have_state = true;
+      if (sw) c->sh_cur ^= 1;
     }
+  }
+  if (sw) {  // the session's running totals
+    c->have_state = have_state;
+    c->s_nr = n_r;
+    c->s_pool = pool_used;
+    c->s_items += n_items;
+    c->s_segs += sx.segments;
+    c->s_windows += sx.windows;
+    n_items = c->s_items;
+    sx.segments = c->s_segs;
+    sx.windows = c->s_windows;
   }
   u32 nfind = (u32)hcnt[C_FINDINGS];
   if (nwin == 1 && last_win < 0) {  // no records at all in the window loop (cannot happen for n > 0)
@@ -499,6 +658,12 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S) {
   sx.items = n_items;
   sx.vc_pool_entries = pool_used;
   cudaEventRecord(c->ev[7], st);
+  if (sw && !sw->final) {  // more windows follow: no race list yet
+    if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "stream window");
+    sx.races = n_r;
+    sx.kernel_launches = g_launches - launches0;
+    return BC_OK;
+  }
   // ---- K8: finalize
   if (g.world > 1 && g.rank != 0) nfind = 0;  // findings come from the replicated replay: rank 0 reports them
   u64 total = n_r + nfind;
@@ -624,7 +789,7 @@ bc_status bc_detect(bc_ctx* c, bc_stats* out) {
   {
     Scratch S(c->stream, &c->arena);
     try {
-      s = c->sharded ? detect_sharded(c, S) : detect_impl(c, S);
+      s = c->sharded ? detect_sharded(c, S) : detect_impl(c, S, nullptr);
     } catch (const std::bad_alloc&) {
       s = fail(c, BC_ERR_OOM, "scratch allocation");
     }
@@ -638,6 +803,144 @@ bc_status bc_detect(bc_ctx* c, bc_stats* out) {
   }
   if (out) *out = c->stats;
   return s;
+}
+
+bc_status bc_stream_open(bc_ctx* c, uint64_t queue_records, uint64_t max_records, uint64_t min_window,
+                         void** queue_dev) {
+  if (!c || !queue_dev || queue_records == 0 || max_records == 0) return BC_ERR_INVALID_ARG;
+  if (c->comm || c->cfg.world > 1) return fail(c, BC_ERR_INVALID_ARG, "streaming is single-GPU");
+  if (c->cfg.n_global_ranges > 64) return fail(c, BC_ERR_INVALID_ARG, "at most 64 global ranges");
+  if (max_records >= 0xFFFFFFFFull) return fail(c, BC_ERR_OVERFLOW, "2^32 - 1 or more records");
+  cudaSetDevice(c->cfg.device);
+  drain_stop(c);
+  // every kernel a poll may launch is loaded now: under lazy loading a first launch waits for the
+  // running kernels, i.e. for a producer that may be waiting for the queue to drain
+  preload_sort();
+  preload_check();
+  preload_trace();
+  preload_sync();
+  preload_finalize();
+  cudaStream_t st = c->stream;
+  c->da.free(c->queue, c->queue_bytes);
+  c->da.free(c->sbuf, c->sbuf_cap * sizeof(bc_record));
+  c->queue = nullptr;
+  c->sbuf = nullptr;
+  c->queue_bytes = Q_HDR * sizeof(u64) + queue_records * sizeof(bc_record);
+  c->queue = (u64*)c->da.alloc(c->queue_bytes);
+  c->sbuf = (bc_record*)c->da.alloc(max_records * sizeof(bc_record));
+  if (!c->granges) c->granges = (u64*)c->da.alloc(2 * 64 * sizeof(u64));
+  if (!c->dstream) {  // highest priority: its copies are dispatched ahead of queued check kernels
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    cudaStreamCreateWithPriority(&c->dstream, cudaStreamNonBlocking, hi);
+  }
+  if (!c->dhdr) cudaMallocHost(&c->dhdr, (Q_HDR + 1) * sizeof(u64));
+  if (!c->queue || !c->sbuf || !c->granges || !c->dstream || !c->dhdr) return fail(c, BC_ERR_OOM, "stream buffers");
+  c->queue_cap = queue_records;
+  c->sbuf_cap = max_records;
+  u64* hdr = c->dhdr;
+  memset(hdr, 0, Q_HDR * sizeof(u64));
+  hdr[Q_CAP] = queue_records;
+  cudaMemcpyAsync(c->queue, hdr, Q_HDR * sizeof(u64), cudaMemcpyHostToDevice, st);
+  cudaMemcpyAsync(c->granges, c->cfg.global_ranges, 2 * 64 * sizeof(u64), cudaMemcpyHostToDevice, st);
+  if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "stream open");
+  c->checked = 0;
+  c->drained.store(0);
+  c->wseen.store(0);
+  c->dgen.store(0);
+  c->drain_err.store(0);
+  c->drain_stop.store(false);
+  c->min_window = std::max<u64>(min_window, 1);
+  c->have_state = false;
+  c->sh_cur = 0;
+  c->s_nr = c->s_pool = c->s_items = c->s_segs = c->s_windows = 0;
+  c->loaded = false;
+  c->detected = false;
+  c->values = nullptr;
+  c->drainer = std::thread(drain_loop, c);
+  c->streaming = true;
+  *queue_dev = c->queue;
+  return BC_OK;
+}
+
+bc_status bc_stream_poll(bc_ctx* c, int finish, bc_stats* out) {
+  if (!c) return BC_ERR_INVALID_ARG;
+  if (!c->streaming) return fail(c, BC_ERR_STATE, "bc_stream_poll without bc_stream_open");
+  cudaSetDevice(c->cfg.device);
+  cudaStream_t st = c->stream;
+  auto stop_with = [&](bc_status s, const char* why) {
+    drain_stop(c);
+    c->streaming = false;
+    return fail(c, s, why);
+  };
+  u64 avail = c->drained.load(std::memory_order_acquire);
+  if (finish) {  // the producer has finished: one full drainer pass that began after this call sees the final heads
+    const u64 g0 = c->dgen.load(std::memory_order_acquire);
+    const auto t0 = std::chrono::steady_clock::now();
+    while (!c->drain_err.load() && c->dgen.load(std::memory_order_acquire) < g0 + 2) {
+      if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(30))
+        return stop_with(BC_ERR_CUDA, "the drain thread stalled");
+      std::this_thread::sleep_for(std::chrono::microseconds(20));
+    }
+    drain_stop(c);
+    avail = c->drained.load(std::memory_order_acquire);
+    if (!c->drain_err.load() && avail != c->wseen.load())
+      return stop_with(BC_ERR_STATE, "finish before the producer committed everything");
+  }
+  if (int e = c->drain_err.load()) {
+    return stop_with((bc_status)e, e == BC_ERR_TRUNCATED ? "more records than bc_stream_open's max_records"
+                                                         : "the producer gave up (queue error flag)");
+  }
+  if (!finish && avail - c->checked < c->min_window) {
+    if (out) *out = c->stats;
+    return BC_OK;
+  }
+  // check the drained records as one window (clocks from the whole prefix)
+  c->trace = c->sbuf;
+  c->n_recs = avail;
+  c->g.n_recs = avail;
+  c->err.clear();
+  StreamWin sw;
+  sw.R0 = c->checked;
+  sw.final = finish != 0;
+  bc_status s;
+  {
+    Scratch S(st, &c->arena);
+    try {
+      s = detect_impl(c, S, &sw);
+    } catch (const std::bad_alloc&) {
+      s = fail(c, BC_ERR_OOM, "scratch allocation");
+    }
+  }
+  cudaStreamSynchronize(st);
+  if (out) *out = c->stats;
+  if (s != BC_OK) {
+    drain_stop(c);
+    c->streaming = false;
+    return s;
+  }
+  c->checked = avail;
+  if (finish) {
+    c->streaming = false;
+    c->loaded = true;
+    c->detected = true;
+  }
+  return BC_OK;
+}
+
+bc_status bc_queue_push(void* queue_dev, const bc_record* recs, uint64_t n, void* stream) {
+  if (!queue_dev || (n && !recs)) return BC_ERR_INVALID_ARG;
+  if (!n) return BC_OK;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  // persistent and co-resident (a warp may wait for an earlier ticket's warp): at most 2 CTAs per SM
+  const u64 blocks = std::min<u64>((n + 7) / 8, (u64)sms * 2);
+  // its SMs keep the full shared-memory split, so the session's check kernels can share them
+  cudaFuncSetAttribute(k_queue_push, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  k_queue_push<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((u64*)queue_dev, recs, n);
+  ++g_launches;
+  return cudaGetLastError() == cudaSuccess ? BC_OK : BC_ERR_CUDA;
 }
 
 static bc_status races_copy(bc_ctx* c, bc_race* out, uint64_t cap, uint64_t* n_total, cudaMemcpyKind kind) {

@@ -1082,4 +1082,8 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   g_launches += 4;
 }
 
+void preload_check() {
+  preload(k_blk_sum, k_blk_units, k_check_tile, k_count_gathers, k_range_scan);
+}
+
 }  // namespace bc

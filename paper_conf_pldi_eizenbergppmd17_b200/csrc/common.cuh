@@ -28,6 +28,7 @@ constexpr int WARP = 32;
 // error flags (device word) -> bc_status
 constexpr u32 ERR_INFEASIBLE = 1u;
 constexpr u32 ERR_OVERFLOW = 2u;
+constexpr u32 ERR_UNDECLARED = 8u;  // streaming: a global access outside the declared allocations
 
 // item op codes (2 low bits of an item's key word)
 constexpr u32 IOP_LD = 0, IOP_ST = 1, IOP_ST_SV = 2, IOP_ATOM = 3;
@@ -41,6 +42,8 @@ constexpr u32 SYNC_LOOKUP_CAP = 1u << 16;  // step cap of one foreign lookup
 // internal Geo.flags bit: per-lane store values are loaded (row f3, reading R6b): every store item
 // is a same-value filter candidate and K7 compares the two lanes' values
 constexpr u32 GEO_F_VALUES = 0x80000000u;
+// internal Geo.flags bit: the global page set is the declared allocations (streaming, row f1)
+constexpr u32 GEO_F_DECLARED = 0x40000000u;
 
 struct Geo {
   u32 n_blocks, tpb, wpb, n_warps;

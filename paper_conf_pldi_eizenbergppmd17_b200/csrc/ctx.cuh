@@ -1,6 +1,8 @@
 // ctx.cuh — the context behind the opaque bc_ctx handle of include/bc.h (api.cu, shard.cu).
 #pragma once
+#include <atomic>
 #include <string>
+#include <thread>
 
 #include "comm.cuh"
 #include "common.cuh"
@@ -44,6 +46,37 @@ struct bc_ctx {
   u64 n_global = 0;           // records of the whole trace (sharded)
   void* xbuf[6] = {};         // device exchange / scratch buffers (grown on demand)
   size_t xcap[6] = {};
+  // streaming session (bc_stream_open)
+  bool streaming = false;
+  u64* queue = nullptr;       // device: 8 u64 header + ring
+  size_t queue_bytes = 0;
+  u64 queue_cap = 0;
+  bc_record* sbuf = nullptr;  // device: the trace so far
+  u64 sbuf_cap = 0;
+  // the drain thread: copy-engine copies ring -> sbuf on its own stream, then the new read head; it
+  // needs no SM, so a producer waiting on a full ring never waits for a window check
+  std::thread drainer;
+  std::atomic<bool> drain_stop{false};
+  std::atomic<u64> drained{0};  // records in sbuf (published after the copies completed)
+  std::atomic<u64> wseen{0};    // the write head the drainer last saw
+  std::atomic<u64> dgen{0};     // completed drainer passes (header read, copies, publish)
+  std::atomic<int> drain_err{0};
+  cudaStream_t dstream = nullptr;
+  u64* dhdr = nullptr;          // pinned: the header as last read, [Q_HDR] = the read head to write
+  u64 checked = 0;            // records checked (the next window starts here)
+  u64 min_window = 0;
+  u64* granges = nullptr;     // device copy of bc_config.global_ranges
+  uint4* sh[2] = {};          // shadow tables carried between polls
+  size_t sh_bytes = 0;
+  int sh_cur = 0;
+  bool have_state = false;
+  u64 s_nr = 0, s_pool = 0, s_items = 0, s_segs = 0, s_windows = 0;
+};
+
+// one window of a streaming session: records [R0, n) are new; earlier ones only feed the clocks
+struct StreamWin {
+  u64 R0 = 0;
+  bool final = false;
 };
 
 enum { PH_HEADER = 0, PH_PARTITION, PH_REPLAY, PH_SYNC, PH_EXPAND, PH_SORT, PH_CHECK, PH_FINALIZE, PH_N };

@@ -128,4 +128,8 @@ void finalize_races(const uint4* races, u32 n_r, const u32* fblk, const u32* fre
   }
 }
 
+void preload_finalize() {
+  preload(k_emit_findings, k_emit_races, k_field, k_page_list);
+}
+
 }  // namespace bc

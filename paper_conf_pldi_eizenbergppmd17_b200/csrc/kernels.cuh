@@ -20,8 +20,21 @@ enum { C_LANE_EVENTS = 0, C_CONTROL_EVENTS, C_SYNC_RECS, C_ACQ_RECS, C_MEM_RECS,
        C_ITEMS, C_ITEM_BOUND, C_SEGMENTS_UNUSED, C_PAGE_WORDS, C_PAGES, C_ERR, C_NEED_SORT, C_FINDINGS,
        C_RACES, C_SEGMENTS, C_GATHERS, C_POOL, C_N };
 
-// Device memory of a context: cudaMalloc / cudaFree, or the caller's allocator (bc_config.dev_alloc /
+// Device memory of a context: cudaMallocAsync / cudaFreeAsync on the context's stream, or the caller's allocator (bc_config.dev_alloc /
 // dev_free, e.g. torch's caching allocator).
+// Force-load kernels (CUDA lazy loading otherwise loads a kernel at its first launch, and that load
+// waits for running kernels: a streaming session's consumer would wait for its spinning producer).
+template <typename... K>
+inline void preload(K... k) {
+  cudaFuncAttributes a;
+  (cudaFuncGetAttributes(&a, (const void*)k), ...);
+}
+void preload_sort();
+void preload_check();
+void preload_trace();
+void preload_sync();
+void preload_finalize();
+
 struct DevAlloc {
   bc_dev_alloc_fn fa = nullptr;
   bc_dev_free_fn ff = nullptr;
@@ -29,8 +42,10 @@ struct DevAlloc {
   cudaStream_t st = nullptr;
   void* alloc(size_t bytes) {
     if (fa) return fa(bytes, (void*)st, user);
+    // stream-ordered: cudaFree would synchronise the whole device, which deadlocks a streaming
+    // session whose producer kernel (another stream) waits for this context to drain the queue
     void* p = nullptr;
-    if (cudaMalloc(&p, bytes) != cudaSuccess) {
+    if (cudaMallocAsync(&p, bytes ? bytes : 256, st) != cudaSuccess) {
       cudaGetLastError();
       return nullptr;
     }
@@ -39,7 +54,7 @@ struct DevAlloc {
   void free(void* p, size_t bytes) {
     if (!p) return;
     if (ff) ff(p, bytes, (void*)st, user);
-    else cudaFree(p);
+    else cudaFreeAsync(p, st);
   }
 };
 
@@ -107,7 +122,9 @@ constexpr u32 REC_W = 8;
 constexpr u64 WIN_MAX = (1ull << 30) - 1024;
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
                    u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_w, uint4* hdr16,
-                   u32* rec_cnt, u32* err, cudaStream_t st);
+                   u32* rec_cnt, u32* err, cudaStream_t st, bool mark_pages = true);
+void launch_mark_ranges(const u64* ranges, u32 n_ranges, u32* page_bits, u32* word_list, u64* cnt, u32* err,
+                        cudaStream_t st);
 void launch_window_starts(const u64* cum, u64 n, u64 we, u32 nwin, u64* starts, u64* bounds, cudaStream_t st);
 constexpr u32 WS_SMALL = 8192;  // n_warps up to which one CTA does the per-warp scans (launch_warp_scans)
 void launch_warp_scans(const u32* rec_cnt, const u32* if_cnt, const u32* bar_cnt, u32 n_warps, u32* warp_start,
@@ -119,7 +136,7 @@ void launch_replay(const uint4* hdr16, const u32* wrec, const u32* gidx, const u
                    const u32* node_base, const u32* bar_base, uint4* snap, uint4* nodes, u32* bar_rec, u32* bar_next,
                    u32* find_blk, u32* find_rec, u32* find_cnt, u32* err, cudaStream_t st);
 void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, const u32* bar_rec, const u32* bar_next,
-                     u32* blockR, u32* err, cudaStream_t st);
+                     u32* blockR, u32* err, cudaStream_t st, bool allow_pending = false);
 void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, const u32* bar_base, const u32* blockR,
                       cudaStream_t st);
 void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,

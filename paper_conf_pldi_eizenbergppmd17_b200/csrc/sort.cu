@@ -754,4 +754,10 @@ void exclusive_scan_u32_u64(const u32* in, u64* out, u64 n, void* temp, u64* tot
   exclusive_scan_t<u64>(in, out, n, temp, total_dev, st);
 }
 
+void preload_sort() {
+  preload(k_rs_bins<8>, k_rs_bins<9>, k_rs_bins<10>, k_rs_bins<11>, k_rs_up<8>, k_rs_up<9>, k_rs_up<10>, k_rs_up<11>,
+          k_rs_down<8>, k_rs_down<9>, k_rs_down<10>, k_rs_down<11>, k_rs_rows, k_sort_small, k_scan_small<u32>,
+          k_scan_small<u64>, k_scan_u32<u32>, k_scan_u32<u64>, k_scan_tiles, k_scan_tsum);
+}
+
 }  // namespace bc

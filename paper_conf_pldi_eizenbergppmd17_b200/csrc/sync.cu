@@ -502,4 +502,10 @@ int run_sync_skeleton(const bc_record* srecs, const u32* sgidx, u32 n_srec, u32 
   return 0;
 }
 
+void preload_sync() {
+  preload(k_acq_collect, k_acq_flags, k_acq_info, k_assign_ids, k_block_start, k_bpairs, k_compact_pairs,
+          k_ent_count, k_ent_fill, k_gather_records, k_gather_u32, k_iota, k_iota_add, k_laneops, k_make_ak, k_popc_recs,
+          k_uniq_flags2);
+}
+
 }  // namespace bc

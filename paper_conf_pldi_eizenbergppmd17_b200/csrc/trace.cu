@@ -26,7 +26,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
                                                 u32* __restrict__ page_bits, u32* __restrict__ word_list,
                                                 u64* __restrict__ cnt, u32* __restrict__ rec_w,
                                                 uint4* __restrict__ hdr16, u32* __restrict__ rec_cnt,
-                                                u32* __restrict__ err) {
+                                                u32* __restrict__ err, int mark_pages) {
   const u32 lane = threadIdx.x & 31;
   const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const u64 r = gw * 32 + lane;
@@ -113,7 +113,7 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
     }
   }
   // page marking: ST / ATOM on global memory
-  u32 wr = __ballot_sync(0xFFFFFFFFu, valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) &&
+  u32 wr = __ballot_sync(0xFFFFFFFFu, mark_pages && valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) &&
                                           h.space == BC_SPACE_GLOBAL);
   while (wr) {  // HDR_ROWS records' address rows in flight at a time
     int js[HDR_ROWS];
@@ -155,6 +155,34 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
       }
     }
   }
+}
+
+// Streaming (declared allocations, bc_config.global_ranges): mark every 1-MB page of the ranges; a
+// word that turns non-zero is listed for k_page_rank
+__global__ void k_mark_ranges(const u64* __restrict__ ranges, u32 n_ranges, u32* __restrict__ page_bits,
+                              u32* __restrict__ word_list, u64* __restrict__ cnt, u32* __restrict__ err) {
+  for (u32 q = 0; q < n_ranges; ++q) {
+    const u64 base = ranges[2 * q], size = ranges[2 * q + 1];
+    if (!size) continue;
+    const u64 p0 = base >> 20, p1 = (base + size - 1) >> 20;
+    if (p1 >= (1ull << 28)) {
+      if (threadIdx.x == 0 && blockIdx.x == 0) set_err(err, ERR_OVERFLOW);
+      continue;
+    }
+    for (u64 p = p0 + (u64)blockIdx.x * blockDim.x + threadIdx.x; p <= p1; p += (u64)gridDim.x * blockDim.x) {
+      const u32 bit = 1u << (p & 31);
+      if (atomicOr(&page_bits[p >> 5], bit) == 0u) {
+        const u64 at = atomicAdd((unsigned long long*)&cnt[C_PAGE_WORDS], 1ull);
+        word_list[at] = (u32)(p >> 5);
+      }
+    }
+  }
+}
+void launch_mark_ranges(const u64* ranges, u32 n_ranges, u32* page_bits, u32* word_list, u64* cnt, u32* err,
+                        cudaStream_t st) {
+  if (!n_ranges) return;
+  k_mark_ranges<<<64, 256, 0, st>>>(ranges, n_ranges, page_bits, word_list, cnt, err);
+  ++g_launches;
 }
 
 // warp_start[w] = first index of warp w in the warp-sorted record list (lower bound)
@@ -344,28 +372,38 @@ __global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16,
 __global__ void __launch_bounds__(256) k_barriers(Geo g, const u32* __restrict__ bar_cnt,
                                                   const u32* __restrict__ bar_base, const u32* __restrict__ bar_rec,
                                                   const u32* __restrict__ bar_next, u32* __restrict__ blockR,
-                                                  u32* __restrict__ err) {
+                                                  u32* __restrict__ err, int allow_pending) {
   const u32 b = (u32)(((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
   const u32 lane = threadIdx.x & 31;
   if (b >= g.n_blocks) return;  // warp-uniform
   const u32 w0 = b * g.wpb;
-  const u32 nb = bar_cnt[w0];
-  bool diff = false;
-  for (u32 i = lane; i < g.wpb; i += 32) diff |= bar_cnt[w0 + i] != nb;  // (wpb > 32: simulated small warps)
-  if (__any_sync(0xFFFFFFFFu, diff)) {
+  // barriers [0, nb) completed (every warp arrived); a prefix of a streamed trace (allow_pending) may end
+  // with barrier nb pending: some warps arrived (and may issue nothing more), the others not yet
+  u32 mn = NONE, mx = 0;
+  for (u32 i = lane; i < g.wpb; i += 32) {  // (wpb > 32: simulated small warps)
+    mn = min(mn, bar_cnt[w0 + i]);
+    mx = max(mx, bar_cnt[w0 + i]);
+  }
+  mn = __reduce_min_sync(0xFFFFFFFFu, mn);
+  mx = __reduce_max_sync(0xFFFFFFFFu, mx);
+  if (mx != mn && !(allow_pending && mx == mn + 1)) {
     if (lane == 0) set_err(err, ERR_INFEASIBLE);
     return;
   }
+  const u32 nb = mn;
   for (u32 k = lane; k < nb; k += 32) {
-    u32 R = 0, mn = NONE;
+    u32 R = 0, mnx = NONE;
     for (u32 i = 0; i < g.wpb; ++i) {
       u32 bi = bar_base[w0 + i] + k;
       R = max(R, bar_rec[bi]);
-      mn = min(mn, bar_next[bi]);
+      mnx = min(mnx, bar_next[bi]);
     }
-    if (mn != NONE && mn < R) set_err(err, ERR_INFEASIBLE);
+    if (mnx != NONE && mnx < R) set_err(err, ERR_INFEASIBLE);
     blockR[bar_base[w0] + k] = R + 1;
   }
+  if (mx > nb)  // the pending barrier: a warp that arrived issues nothing until it completes
+    for (u32 i = lane; i < g.wpb; i += 32)
+      if (bar_cnt[w0 + i] > nb && bar_next[bar_base[w0 + i] + nb] != NONE) set_err(err, ERR_INFEASIBLE);
 }
 
 // ---------------------------------------------------------------------------- k_expand
@@ -431,7 +469,7 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
       if (c < n_chunks) issue(c, s);
     }
   const u32 lt = lanemask_lt();
-  bool bad = false, ovf = false;
+  bool bad = false, ovf = false, undecl = false;
   u32 it = 0;
   for (u64 c = blockIdx.x; c < n_chunks; c += gridDim.x, ++it) {
     const int st = (int)(it % EX_STAGES);
@@ -489,6 +527,8 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
           if ((pw >> bit) & 1u)
             key0 = (__ldg(&page_rank[p >> 5]) + __popc(pw & ((1u << bit) - 1u))) << (20 - g.G) |
                    (u32)((a & 0xFFFFFull) >> g.G);
+          else if (g.flags & GEO_F_DECLARED)
+            undecl = true;  // streaming: the page set is the declared allocations, nothing may fall outside
         } else {
           ovf = true;
         }
@@ -514,6 +554,7 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
   }
   if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
   if (__any_sync(0xFFFFFFFFu, ovf) && lane == 0) set_err(err, ERR_OVERFLOW);
+  if (__any_sync(0xFFFFFFFFu, undecl) && lane == 0) set_err(err, ERR_UNDECLARED);
 }
 
 // Window k = the records whose weight prefix cum[r] (exclusive) lies in [k * we, (k + 1) * we):
@@ -615,12 +656,12 @@ __global__ void __launch_bounds__(1024) k_page_rank(u32* __restrict__ words, con
 // --------------------------------------------------------------------- host launchers
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
                    u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_w, uint4* hdr16,
-                   u32* rec_cnt, u32* err, cudaStream_t st) {
+                   u32* rec_cnt, u32* err, cudaStream_t st, bool mark_pages) {
   u64 warps = (g.n_recs + 31) / 32;
   if (warps == 0) return;
   u64 blocks = (warps + 7) / 8;
   k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt,
-                                             rec_w, hdr16, rec_cnt, err); ++g_launches;
+                                             rec_w, hdr16, rec_cnt, err, mark_pages ? 1 : 0); ++g_launches;
 }
 
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st) {
@@ -635,8 +676,10 @@ void launch_replay(const uint4* hdr16, const u32* wrec, const u32* gidx, const u
 }
 
 void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, const u32* bar_rec, const u32* bar_next,
-                     u32* blockR, u32* err, cudaStream_t st) {
-  k_barriers<<<(unsigned)(((u64)g.n_blocks * 32 + 255) / 256), 256, 0, st>>>(g, bar_cnt, bar_base, bar_rec, bar_next, blockR, err); ++g_launches;
+                     u32* blockR, u32* err, cudaStream_t st, bool allow_pending) {
+  k_barriers<<<(unsigned)(((u64)g.n_blocks * 32 + 255) / 256), 256, 0, st>>>(g, bar_cnt, bar_base, bar_rec, bar_next,
+                                                                             blockR, err, allow_pending ? 1 : 0);
+  ++g_launches;
 }
 
 // snapshot .w: barrier phase -> label of the block's last completed barrier (0 = none)
@@ -750,6 +793,11 @@ void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, co
   k_expand<<<gr, EX_THREADS, smem, st>>>(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, gidx, G0, keys, evs,
                                          err);
   ++g_launches;
+}
+
+void preload_trace() {
+  preload(k_barriers, k_expand, k_header, k_mark_ranges, k_node_base, k_page_rank, k_replay, k_snap_blab,
+          k_warp_scans, k_warp_start, k_window_starts);
 }
 
 }  // namespace bc
