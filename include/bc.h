@@ -94,14 +94,15 @@ typedef struct bc_race {
 /* ------------------------------------------------------------------ configuration */
 enum {
   BC_F_RELEASE_OVERWRITE = 1u,    /* the printed release S_x := C_t (Fig. 3 RELBLOCK / RELGLOBAL,
-                                     P:L754-758) instead of reading R1's join      */
+                                     P:L754-758; ACQREL joins the slot before it
+                                     writes it) instead of reading R1's join       */
   BC_F_NO_SAME_VALUE_FILTER = 2u, /* report intra-warp same-value WW races too (R6)           */
   BC_F_COUNT_GATHERS = 4u         /* statistics: fill bc_stats.clock_gathers (one extra pass)  */
 };
 
 /* Optional device allocator ("PyTorch only for device memory"): every device buffer the
  * context owns (trace copy, scratch, shadow tables, race list) is obtained from dev_alloc and returned
- * to dev_free with the context's stream, e.g. torch's caching allocator.  NULL: cudaMalloc / cudaFree.
+ * to dev_free with the context's stream, e.g. torch's caching allocator.  NULL: cudaMallocAsync / cudaFreeAsync on the context stream.
  * dev_alloc returns NULL on failure (-> BC_ERR_OOM); returned memory must be 256-B aligned. */
 typedef void* (*bc_dev_alloc_fn)(size_t bytes, void* stream, void* user);
 typedef void (*bc_dev_free_fn)(void* ptr, size_t bytes, void* stream, void* user);

@@ -242,7 +242,8 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
   *out = nullptr;
   const u32 ws = cfg->warp_size;  // 32, or a simulated smaller warp
   if ((ws != 4 && ws != 8 && ws != 16 && ws != 32) || cfg->granule_log2 > 4) return BC_ERR_INVALID_ARG;
-  if (cfg->flags & ~(u32)(BC_F_NO_SAME_VALUE_FILTER | BC_F_COUNT_GATHERS)) return BC_ERR_INVALID_ARG;  // overwrite: not on GPU yet
+  if (cfg->flags & ~(u32)(BC_F_RELEASE_OVERWRITE | BC_F_NO_SAME_VALUE_FILTER | BC_F_COUNT_GATHERS))
+    return BC_ERR_INVALID_ARG;
   if ((cfg->dev_alloc == nullptr) != (cfg->dev_free == nullptr)) return BC_ERR_INVALID_ARG;
   if (cfg->world < 0 || cfg->world > 1024) return BC_ERR_INVALID_ARG;
   if (cfg->world > 1 && (cfg->rank < 0 || cfg->rank >= cfg->world)) return BC_ERR_INVALID_ARG;
@@ -506,6 +507,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
   hc.err = err;
   hc.n_acq = 0;
   hc.n_idx = 0;
+  hc.e_off = hc.e_cnt = hc.e_arr = hc.e_key = hc.e_mask = hc.e_clk = nullptr;
   // ---- K3: sync skeleton
   if (hc_cnt[C_SYNC_RECS]) {
     u64 ne = 0;

@@ -146,6 +146,16 @@ struct HbCtx {
   const u32* idx_pos;
   const u32* idx_mask;
   const u32* idx_clk;
+  // BC_F_RELEASE_OVERWRITE (the printed S_x := C_t): the K3 entries in emission order, lane-op p's at
+  // [e_off[p], e_off[p] + e_cnt[p]) -- a window link names one writer lane-op of G_x / B_{x,b}
+  const u32* e_off;
+  const u32* e_cnt;
+  const u32* e_arr;
+  const u32* e_key;
+  const u32* e_mask;
+  const u32* e_clk;
+  const u32* lo_rec;  // lane-op -> global record
+  u32 f_base;         // acquire views F_a have array ids f_base + a
   u32* err;
 };
 
@@ -278,6 +288,111 @@ static __device__ __noinline__ bool view_knows(const HbCtx c, u32 uw, u32 ul, u3
   return false;
 }
 
+// The same question under BC_F_RELEASE_OVERWRITE.  There, S_x[b] holds only what its latest writer
+// put there (an ACQREL writer joins the previous content first, Fig. 3), so K3 links an
+// acquire (and an ACQREL's release) to a *window*: the entries of exactly one writer lane-op p
+// (link mask LINK_WIN, clk = p), read in emission order.  An acquire's own view F_a is still reached
+// as a prefix (entries with pos < bound).  Stack items: (array | WIN_BIT, lane-op) or (array, bound).
+constexpr u32 LINK_WIN = 1u;
+constexpr u32 WIN_BIT = 0x80000000u;
+static __device__ __noinline__ bool view_knows_ow(const HbCtx c, u32 uw, u32 ul, u32 r1, u32 arr, u32 bound) {
+  constexpr int STK = 256, VIS = 256;
+  u32 st_a[STK], st_v[STK];
+  u32 vis_a[VIS], vis_v[VIS];
+  int sp = 0, nv = 0;
+  st_a[sp] = arr;
+  st_v[sp++] = bound;
+  u32 steps = 0;
+  const u32 need = r1 + 1u;
+  const u32 kb = KEY_BLOCK | (uw / c.g.wpb);
+  bool ovf = false;
+  // push a link target unless an item that sees at least as much is already visited or waiting
+  auto push = [&](u32 a, u32 v) {
+    const bool win = a & WIN_BIT;
+    for (int q = 0; q < nv; ++q)
+      if (vis_a[q] == a && (win ? vis_v[q] == v : vis_v[q] >= v)) return;
+    for (int q = 0; q < sp; ++q)
+      if (st_a[q] == a) {
+        if (win) {
+          if (st_v[q] == v) return;
+        } else {
+          if (st_v[q] < v) st_v[q] = v;
+          return;
+        }
+      }
+    if (sp >= STK) {
+      ovf = true;
+      return;
+    }
+    st_a[sp] = a;
+    st_v[sp++] = v;
+  };
+  // Everything reachable from a writer window or an acquire view happened before that writer's /
+  // acquirer's record, so one older than r1 cannot know the step at r1: not pushed.
+  auto link = [&](u32 key, u32 mask, u32 clk, u32 cap) {
+    const u32 tgt = key & 0x3FFFFFFFu;
+    if (mask == LINK_WIN) {
+      if (c.lo_rec[clk] > r1) push(tgt | WIN_BIT, clk);
+    } else if (tgt < c.f_base || c.acq_rec[tgt - c.f_base] > r1) {
+      push(tgt, clk < cap ? clk : cap);
+    }
+  };
+  while (sp > 0) {
+    --sp;
+    const u32 a = st_a[sp], v = st_v[sp];
+    const bool win = a & WIN_BIT;
+    bool skip = false, found = false;
+    for (int q = 0; q < nv; ++q) {
+      if (vis_a[q] != a) continue;
+      if (win) {
+        if (vis_v[q] == v) {
+          skip = true;
+          break;
+        }
+      } else {  // one visited record per prefix array, with the largest bound walked so far
+        found = true;
+        if (vis_v[q] >= v) skip = true;
+        else vis_v[q] = v;
+        break;
+      }
+    }
+    if (skip) continue;
+    if (!found && nv < VIS) {
+      vis_a[nv] = a;
+      vis_v[nv++] = v;
+    }
+    if (++steps > SYNC_LOOKUP_CAP || ovf) {
+      set_err(c.err, ERR_OVERFLOW);
+      return false;
+    }
+    if (win) {  // the entries writer lane-op v put into array a
+      const u32 aid = a & ~WIN_BIT, e0 = c.e_off[v], e1 = e0 + c.e_cnt[v];
+      for (u32 e = e0; e < e1; ++e) {
+        if (c.e_arr[e] != aid) continue;
+        const u32 key = c.e_key[e], top = key & KEY_LINK;
+        if (top == KEY_LINK) link(key, c.e_mask[e], c.e_clk[e], NONE);
+        else if (key == kb) {
+          if (c.e_clk[e] >= need) return true;
+        } else if (top == 0 && key == uw) {
+          if (((c.e_mask[e] >> ul) & 1u) && c.e_clk[e] >= need) return true;
+        }
+      }
+    } else {  // prefix view of array a: entries with pos < v
+      u64 ak = ((u64)a << 32) | kb;
+      for (u32 i = idx_lower_bound(c, ak); i < c.n_idx && c.idx_ak[i] == ak && c.idx_pos[i] < v; ++i)
+        if (c.idx_clk[i] >= need) return true;
+      ak = ((u64)a << 32) | uw;
+      for (u32 i = idx_lower_bound(c, ak); i < c.n_idx && c.idx_ak[i] == ak && c.idx_pos[i] < v; ++i)
+        if (((c.idx_mask[i] >> ul) & 1u) && c.idx_clk[i] >= need) return true;
+      const u64 end = ((u64)a << 32) | 0xFFFFFFFFull;
+      for (u32 i = idx_lower_bound(c, ((u64)a << 32) | KEY_LINK); i < c.n_idx && c.idx_ak[i] <= end; ++i)
+        if (c.idx_pos[i] < v) link((u32)c.idx_ak[i], c.idx_mask[i], c.idx_clk[i], v);
+    }
+  }
+  if (ovf) set_err(c.err, ERR_OVERFLOW);
+  return false;
+}
+
 // foreign part of know_t(u) >= r1+1 for t executing record r2 (snapshot s2): through the
 // views of the acquires of t's block that t structurally knows (every release->acquire path
 // into t's block ends at one of them).
@@ -296,7 +411,9 @@ static __device__ __noinline__ bool foreign_knows(const HbCtx c, u32 w1, u32 l1,
     const u32 ra = c.acq_rec[i];
     if (ra < r1) break;  // an acquire before the access cannot order it (view entries are older than ra)
     if (!struct_knows(c, c.acq_warp[i], c.acq_lane[i], ra, s2)) continue;
-    if (view_knows(c, w1, l1, r1, c.acq_arr[i], NONE)) return true;
+    if ((c.g.flags & BC_F_RELEASE_OVERWRITE) ? view_knows_ow(c, w1, l1, r1, c.acq_arr[i], NONE)
+                                             : view_knows(c, w1, l1, r1, c.acq_arr[i], NONE))
+      return true;
   }
   return false;
 }

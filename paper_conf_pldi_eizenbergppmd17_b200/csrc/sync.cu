@@ -126,6 +126,10 @@ struct K3In {
   u32 nx, nB;
   const u32 *bp_x, *bp_b;  // unique sorted (xid, block) pairs, bid = index
   const u32* acq_idx_of_rec_sorted;  // unused
+  // BC_F_RELEASE_OVERWRITE: the writer lane-ops of each array G_x / B_{x,b}, ascending
+  bool ow;
+  const u32* wr_pos;    // lane-op indices grouped by array
+  const u32* wr_start;  // [nx + nB + 1]
 };
 
 __device__ __forceinline__ u32 pair_lower(const K3In& k, u32 x, u32 b) {
@@ -151,6 +155,17 @@ __device__ __forceinline__ u32 acq_index(const HbCtx& c, u32 b, u32 r) {
   return lo;
 }
 
+// the latest writer lane-op of array a before lane-op ev (NONE: none)
+__device__ __forceinline__ u32 last_writer(const K3In& k, u32 a, u32 ev) {
+  u32 lo = k.wr_start[a], hi = k.wr_start[a + 1];
+  const u32 base = lo;
+  while (lo < hi) {
+    u32 m = (lo + hi) >> 1;
+    if (k.wr_pos[m] < ev) lo = m + 1; else hi = m;
+  }
+  return lo > base ? k.wr_pos[lo - 1] : NONE;
+}
+
 // Emit (or count, when out == nullptr) the entries of lane-op i.
 struct EntOut {
   u32 *arr, *key, *pos, *mask, *clk;
@@ -165,6 +180,26 @@ __device__ __forceinline__ void put(const EntOut* o, u32& n, u32 arr, u32 key, u
     o->clk[n] = clk;
   }
   ++n;
+}
+
+// Overwrite reading (the printed Fig. 3): what lane-op ev acquires from S_x is the content of its slot(s)
+// as the latest writers left it -- window links to those writer lane-ops.  S_x[b] was last written by
+// the later of G_x's and B_{x,b}'s latest writers; ⊔_b S_x[b] is G_x's latest writer plus every block
+// writer after it.
+__device__ void prev_links(const K3In& k, const EntOut* o, u32& n, u32 arr, u32 op, u32 x, u32 my_bid, u32 blo, u32 bhi,
+                           u32 ev) {
+  const u32 gp = last_writer(k, x, ev);
+  if (is_glb_op(op)) {
+    if (gp != NONE) put(o, n, arr, KEY_LINK | x, ev, LINK_WIN, gp);
+    for (u32 j = blo; j < bhi; ++j) {
+      const u32 p = last_writer(k, k.nx + j, ev);
+      if (p != NONE && (gp == NONE || p > gp)) put(o, n, arr, KEY_LINK | (k.nx + j), ev, LINK_WIN, p);
+    }
+  } else {
+    const u32 bp = my_bid != NONE ? last_writer(k, k.nx + my_bid, ev) : NONE;
+    if (bp != NONE && (gp == NONE || bp > gp)) put(o, n, arr, KEY_LINK | (k.nx + my_bid), ev, LINK_WIN, bp);
+    else if (gp != NONE) put(o, n, arr, KEY_LINK | x, ev, LINK_WIN, gp);
+  }
 }
 
 __device__ u32 laneop_entries(const K3In& k, u32 i, const EntOut* o, u32 base) {
@@ -186,11 +221,15 @@ __device__ u32 laneop_entries(const K3In& k, u32 i, const EntOut* o, u32 base) {
   if (is_acq_op(op)) {
     u32 ai = acq_index(c, b, r);
     u32 farr = k.nx + k.nB + ai;
-    put(o, n, farr, KEY_LINK | x, ev, 0u, ev);  // S_x global part
-    if (is_glb_op(op)) {
-      for (u32 j = blo; j < bhi; ++j) put(o, n, farr, KEY_LINK | (k.nx + j), ev, 0u, ev);
-    } else if (my_bid != NONE) {
-      put(o, n, farr, KEY_LINK | (k.nx + my_bid), ev, 0u, ev);
+    if (k.ow) {
+      prev_links(k, o, n, farr, op, x, my_bid, blo, bhi, ev);
+    } else {
+      put(o, n, farr, KEY_LINK | x, ev, 0u, ev);  // S_x global part
+      if (is_glb_op(op)) {
+        for (u32 j = blo; j < bhi; ++j) put(o, n, farr, KEY_LINK | (k.nx + j), ev, 0u, ev);
+      } else if (my_bid != NONE) {
+        put(o, n, farr, KEY_LINK | (k.nx + my_bid), ev, 0u, ev);
+      }
     }
   }
   if (is_rel_op(op)) {
@@ -214,14 +253,29 @@ __device__ u32 laneop_entries(const K3In& k, u32 i, const EntOut* o, u32 base) {
       if (ra >= r) break;
       if (struct_knows(c, c.acq_warp[j], c.acq_lane[j], ra, s)) put(o, n, tarr, KEY_LINK | (k.nx + k.nB + j), ev, 0u, ev);
     }
-    // ACQREL: the part of S_x it acquired that lives in another array
-    if (op == BC_OP_AR_BLK) {
+    // ACQREL: the part of S_x it acquired that lives in another array (overwrite: the slot content
+    // it joined before writing, since its own window shows only its own entries)
+    if (k.ow) {
+      if (op == BC_OP_AR_BLK || op == BC_OP_AR_GLB) prev_links(k, o, n, tarr, op, x, my_bid, blo, bhi, ev);
+    } else if (op == BC_OP_AR_BLK) {
       put(o, n, tarr, KEY_LINK | x, ev, 0u, ev);
     } else if (op == BC_OP_AR_GLB) {
       for (u32 j = blo; j < bhi; ++j) put(o, n, tarr, KEY_LINK | (k.nx + j), ev, 0u, ev);
     }
   }
   return n - base;
+}
+
+// writer lists (overwrite reading): key = the array a release lane-op writes, or nx + nB for the rest
+__global__ void k_wr_keys(K3In k, u32* __restrict__ key, u32* __restrict__ val) {
+  u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= k.n_lo) return;
+  const bc_record& rc = k.srecs[k.lo_sp[i]];
+  const u32 op = rc.op;
+  u32 a = k.nx + k.nB;
+  if (is_rel_op(op)) a = is_glb_op(op) ? k.xid[i] : k.nx + find_bid(k, k.xid[i], rc.warp / k.hc.g.wpb);
+  key[i] = a;
+  val[i] = i;
 }
 
 __global__ void k_ent_count(K3In k, u32* __restrict__ out) {
@@ -465,6 +519,23 @@ int run_sync_skeleton(const bc_record* srecs, const u32* sgidx, u32 n_srec, u32 
   k.bp_x = bp_x;
   k.bp_b = bp_b;
   k.acq_idx_of_rec_sorted = nullptr;
+  k.ow = (g.flags & BC_F_RELEASE_OVERWRITE) != 0;
+  k.wr_pos = nullptr;
+  k.wr_start = nullptr;
+  if (k.ow) {  // writer lane-ops per array, ascending (stable sort of lane-op order by array)
+    u32* wk = S.alloc<u32>(n_lo);
+    u32* wv = S.alloc<u32>(n_lo);
+    u32* wk2 = S.alloc<u32>(n_lo);
+    u32* wv2 = S.alloc<u32>(n_lo);
+    u32* wstart = S.alloc<u32>((size_t)nx + nB + 2);
+    k_wr_keys<<<nb(n_lo), 256, 0, st>>>(k, wk, wv); ++g_launches;
+    const bool alt = radix_sort_pairs(wk, wv, wk2, wv2, n_lo, 0, bits_for((u64)nx + nB), S.alloc<char>(rs_temp_bytes(n_lo)),
+                                      st);
+    const u32* sk = alt ? wk2 : wk;
+    k.wr_pos = alt ? wv2 : wv;
+    k_block_start<<<nb((u64)nx + nB + 1), 256, 0, st>>>(sk, n_lo, nx + nB, wstart); ++g_launches;
+    k.wr_start = wstart;
+  }
   u32* ecnt = S.alloc<u32>(n_lo);
   u32* eoff = S.alloc<u32>(n_lo);
   k_ent_count<<<nb(n_lo), 256, 0, st>>>(k, ecnt); ++g_launches;
@@ -495,6 +566,14 @@ int run_sync_skeleton(const bc_record* srecs, const u32* sgidx, u32 n_srec, u32 
   u32* iclk = S.alloc<u32>(ne + 1);
   if (ne) { k_make_ak<<<nb(ne), 256, 0, st>>>(eo.arr, eo.key, eo.pos, eo.mask, eo.clk, ep, ne, ak, ipos, imask, iclk); ++g_launches; }
   hc.n_idx = ne;
+  hc.e_off = eoff;
+  hc.e_cnt = ecnt;
+  hc.e_arr = eo.arr;
+  hc.e_key = eo.key;
+  hc.e_mask = eo.mask;
+  hc.e_clk = eo.clk;
+  hc.lo_rec = lo_rec;
+  hc.f_base = nx + nB;
   hc.idx_ak = ak;
   hc.idx_pos = ipos;
   hc.idx_mask = imask;
@@ -505,7 +584,7 @@ int run_sync_skeleton(const bc_record* srecs, const u32* sgidx, u32 n_srec, u32 
 void preload_sync() {
   preload(k_acq_collect, k_acq_flags, k_acq_info, k_assign_ids, k_block_start, k_bpairs, k_compact_pairs,
           k_ent_count, k_ent_fill, k_gather_records, k_gather_u32, k_iota, k_iota_add, k_laneops, k_make_ak, k_popc_recs,
-          k_uniq_flags2);
+          k_uniq_flags2, k_wr_keys);
 }
 
 }  // namespace bc

@@ -482,3 +482,90 @@ def build(entry):
     name, fn, expected, opts = entry
     tb = fn()
     return tb.records(), tb.geom.as_dict()
+
+
+# ---------------------------------------------------------------------------
+# Release join (reading R1) vs the printed overwrite S_x := C_t (Fig. 3 RELBLOCK / RELGLOBAL,
+# P:L754-758; ACQREL joins the slot before writing it).  Not part of the
+# 66: these separate the two readings.  Each entry: (name, build, expected_join, expected_overwrite);
+# each warp uses 32 lanes on distinct granules, so a racing warp pair is 32 races.
+OVERWRITE_SUITE = []
+
+
+def lit_ow(name, join, overwrite):
+    def deco(fn):
+        OVERWRITE_SUITE.append((name, fn, sorted(join), sorted(overwrite)))
+        return fn
+    return deco
+
+
+@lit_ow("ow_second_release_erases", [], [(WR, INTRA, G)] * 32)
+def _b():
+    # one block, warps 0-2: w1's release replaces w0's in S_F[0]; w2 acquires only C_w1
+    tb = TraceBuilder(block=(96,))
+    tb.st(0, own(G)); tb.rel(0, F, scope="blk")
+    tb.rel(1, F, scope="blk")
+    tb.acq(2, F, scope="blk"); tb.ld(2, own(G))
+    return tb
+
+
+@lit_ow("ow_acqrel_keeps_slot", [], [])
+def _b():
+    # w1's ACQREL writes C_w1 ⊔ S_F[0] (which holds C_w0): w2 still learns w0's stores
+    tb = TraceBuilder(block=(96,))
+    tb.st(0, own(G)); tb.rel(0, F, scope="blk")
+    tb.ar(1, F, scope="blk")
+    tb.acq(2, F, scope="blk"); tb.ld(2, own(G))
+    return tb
+
+
+@lit_ow("ow_block_release_after_global", [], [(WR, INTER, G)] * 32)
+def _b():
+    # blocks 0 (warps 0, 1) and 1 (warps 2, 3): w0's global release fills every slot, w2's block
+    # release then replaces slot 1 only -- w3 (block 1) misses w0's stores, w1 (block 0) does not
+    tb = TraceBuilder(grid=(2,), block=(64,))
+    tb.st(0, own(G)); tb.rel(0, F, scope="glb")
+    tb.rel(2, F, scope="blk")
+    tb.acq(3, F, scope="blk"); tb.ld(3, own(G))
+    tb.acq(1, F, scope="blk"); tb.ld(1, own(G))
+    return tb
+
+
+@lit_ow("ow_global_release_overrides_block", [], [(WR, INTRA, G)] * 32)
+def _b():
+    # w0's block release fills slot 0; w2's (block 1) global release overwrites every slot
+    tb = TraceBuilder(grid=(2,), block=(64,))
+    tb.st(0, own(G)); tb.rel(0, F, scope="blk")
+    tb.rel(2, F, scope="glb")
+    tb.acq(1, F, scope="blk"); tb.ld(1, own(G))
+    return tb
+
+
+@lit_ow("ow_global_acquire_joins_slots", [], [])
+def _b():
+    # ⊔_b S_F[b]: slot 0 and 2 hold w0's global release, slot 1 w1's block release
+    tb = TraceBuilder(grid=(3,), block=(32,))
+    tb.st(0, own(G)); tb.rel(0, F, scope="glb")
+    tb.rel(1, F, scope="blk")
+    tb.acq(2, F, scope="glb"); tb.ld(2, own(G))
+    return tb
+
+
+@lit_ow("ow_global_acquire_after_global_release", [], [(WR, INTER, G)] * 32)
+def _b():
+    # w1's global release overwrites slot 0 (w0's block release): no slot holds C_w0 any more
+    tb = TraceBuilder(grid=(3,), block=(32,))
+    tb.st(0, own(G)); tb.rel(0, F, scope="blk")
+    tb.rel(1, F, scope="glb")
+    tb.acq(2, F, scope="glb"); tb.ld(2, own(G))
+    return tb
+
+
+@lit_ow("ow_global_acqrel_chain", [], [])
+def _b():
+    # w1's global ACQREL joins every slot (slot 0 = C_w0) and writes the join everywhere
+    tb = TraceBuilder(grid=(3,), block=(32,))
+    tb.st(0, own(G)); tb.rel(0, F, scope="blk")
+    tb.ar(1, F, scope="glb")
+    tb.acq(2, F, scope="blk"); tb.ld(2, own(G))
+    return tb

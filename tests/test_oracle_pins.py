@@ -533,3 +533,17 @@ def test_warpsim_random_vs_bruteforce(ws):
         if st != 0:
             continue
         check_against_bf(r2, g2, races)
+
+
+@pytest.mark.parametrize("entry", litmus.OVERWRITE_SUITE, ids=[e[0] for e in litmus.OVERWRITE_SUITE])
+def test_release_readings(entry):
+    """Hand-derived races under both readings of the release rule (litmus.OVERWRITE_SUITE); the join
+    results also match the brute-force §3.2 definition."""
+    name, fn, want_join, want_ow = entry
+    tb = fn()
+    recs, geom = tb.records(), tb.geom.as_dict()
+    races = run(recs, geom, oracle.F_CHECK_INVARIANT)
+    assert sorted((int(r["kind"]), int(r["cls"]), int(r["space"])) for r in races) == want_join
+    check_against_bf(recs, geom, races, strict=True)
+    races_o = run(recs, geom, oracle.F_RELEASE_OVERWRITE)
+    assert sorted((int(r["kind"]), int(r["cls"]), int(r["space"])) for r in races_o) == want_ow
