@@ -97,7 +97,7 @@ enum {
                                      P:L754-758; ACQREL joins the slot before it
                                      writes it) instead of reading R1's join       */
   BC_F_NO_SAME_VALUE_FILTER = 2u, /* report intra-warp same-value WW races too (R6)           */
-  BC_F_COUNT_GATHERS = 4u         /* statistics: fill bc_stats.clock_gathers (one extra pass)  */
+  BC_F_COUNT_GATHERS = 4u         /* statistics: fill bc_stats.clock_gathers and .segments (one extra pass) */
 };
 
 /* Optional device allocator ("PyTorch only for device memory"): every device buffer the
@@ -155,7 +155,8 @@ typedef struct bc_config {
 typedef struct bc_stats {
   uint64_t records, lane_events, control_events; /* SURVEY §8(d.1) units                         */
   uint64_t items;            /* (granule, lane event) pairs checked after the write-page filter   */
-  uint64_t segments;         /* distinct shadow granules checked                                  */
+  uint64_t segments;         /* granule segments checked (summed over windows); 0 unless          
+                                BC_F_COUNT_GATHERS                                                */
   uint64_t races, findings;  /* race records / barrier-divergence findings                       */
   uint64_t sync_ops;         /* acquire / release lane operations                                 */
   uint64_t written_pages;    /* 1-MB global pages with at least one write          */

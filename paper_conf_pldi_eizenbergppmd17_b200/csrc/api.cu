@@ -79,7 +79,7 @@ bc_status check_window(bc_ctx* c, CheckLaunch& L, u64 b, u64* cnt, u64& n_r, u64
     cudaEventRecord(c->ev[10], st);
     launch_check(L, st);
     cudaEventRecord(c->ev[11], st);
-    if (L.c.g.flags & BC_F_COUNT_GATHERS) launch_count_gathers(L.keys, L.n_dev, cnt + C_GATHERS, st);
+    if (L.c.g.flags & BC_F_COUNT_GATHERS) launch_count_gathers(L.keys, L.n_dev, cnt + C_GATHERS, cnt + C_SEGMENTS, st);
     cudaMemcpyAsync(hcnt, cnt, C_N * sizeof(u64), cudaMemcpyDeviceToHost, st);
     if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_check(c, "check");
     herr = (u32)hcnt[C_ERR];
@@ -567,8 +567,8 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
   u32* iv2 = S.alloc<u32>(maxb + 1);
   void* rtmp = S.alloc<char>(rs_temp_bytes(maxb));
   void* cstatus = S.alloc<char>(check_status_bytes(maxb));
-  uint4* sh_cur = nullptr;  // entries after the last window (double buffer)
-  uint4* sh_nxt = nullptr;
+  uint4* sh_cur = nullptr;  // the carried entries (current after every window)
+  uint4* sh_nxt = nullptr;  // K7's output entries of the touched granules, committed into sh_cur
   bool have_state = false;
   if (sw) {  // a streaming session keeps its tables across polls (the declared page set fixes n_keys)
     const size_t bytes = 2 * n_keys * sizeof(uint4);
@@ -580,8 +580,8 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
       }
       c->sh_bytes = bytes;
     }
-    sh_cur = c->sh[c->sh_cur];
-    sh_nxt = c->sh[c->sh_cur ^ 1];
+    sh_cur = c->sh[0];
+    sh_nxt = c->sh[1];
     have_state = c->have_state;
     if (sw->final) last_win = 0;
     else last_win = -2;  // the window writes entries for the next poll
@@ -609,10 +609,9 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
     u32* sev = alt ? iv2 : ievs;
     // ---- K7: shadow check of the window (carried entries in, entries for the next window out)
     uint4* sh_out = (multi && (int)k != last_win) ? sh_nxt : nullptr;
-    if (sh_out) {
-      if (have_state) cudaMemcpyAsync(sh_out, sh_cur, 2 * n_keys * sizeof(uint4), cudaMemcpyDeviceToDevice, st);
-      else cudaMemsetAsync(sh_out, 0, 2 * n_keys * sizeof(uint4), st);
-    }
+    // the first window that carries state: every entry starts empty (later windows update only the
+    // entries of the granules they touch, k_shadow_commit)
+    if (sh_out && !have_state) cudaMemsetAsync(sh_cur, 0, 2 * n_keys * sizeof(uint4), st);
     CheckLaunch L{};
     L.c = hc;
     L.keys = skey;
@@ -637,9 +636,8 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
     ms_sort += t;
     ms_chk += wo.ms_check;
     if (sh_out) {
-      std::swap(sh_cur, sh_nxt);
+      launch_shadow_commit(skey, n_items_dev, b, sh_nxt, sh_cur, st);
       have_state = true;
-      if (sw) c->sh_cur ^= 1;
     }
   }
   if (sw) {  // the session's running totals

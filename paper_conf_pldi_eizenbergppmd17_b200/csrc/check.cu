@@ -18,8 +18,10 @@
 //
 // Across windows the granule's state is carried in the paper's per-location shadow entry
 // (Fig. 8; shadow memory §4.3.3), 32 B per granule:
-//   e0 = {W rec, W (warp << 5 | lane), W flags (valid | atomic), R mode (none | epoch | vector)}
-//   e1 = {R rec | vector offset, R (warp << 5 | lane) | vector length, 0, 0}
+//   e0 = {W rec, W lane, W flags (valid | atomic), R mode (none | epoch | vector)}
+//   e1 = {R rec | vector offset, R lane | vector length, key, 0}
+// (a thread is (record, lane): its warp is snap[record].warp, looked up only when a check against the
+// carried access is made, so writing an entry never needs the record's clock snapshot)
 // The entry of granule k acts as virtual items in front of k's first item of the window: its W is
 // the last writer until the first writer of the window, its R the read state the first reads of the
 // window extend (a carried read vector counts as already inflated).  Read
@@ -72,8 +74,8 @@ constexpr u32 SH_W_VALID = 1u, SH_W_ATOM = 2u;
 constexpr u32 SH_R_NONE = 0u, SH_R_EPOCH = 1u, SH_R_VC = 2u;
 
 struct Carry {
-  u32 wr, wwl, wf;   // carried writer: record, warp << 5 | lane, flags
-  u32 rm, rr, rwl;   // carried read state: mode; epoch (record, warp << 5 | lane) or vector (offset, length)
+  u32 wr, wwl, wf;   // carried writer: record, lane, flags
+  u32 rm, rr, rwl;   // carried read state: mode; epoch (record, lane) or vector (offset, length)
 };
 __device__ __forceinline__ Carry no_carry() { return Carry{0u, 0u, 0u, SH_R_NONE, 0u, 0u}; }
 
@@ -155,6 +157,8 @@ __device__ __forceinline__ bool hbq(const K7Ctx* k, const HbCtx& c, u32 r1, u32 
 }
 
 __device__ __forceinline__ u32 item_warp(const K7Ctx* k, u32 ev) { return __ldg(&k->c.snap[k->R0 + (ev >> 5)].x); }
+// warp of a carried access (global record index)
+__device__ __forceinline__ u32 rec_warp(const HbCtx& c, u32 rec) { return __ldg(&c.snap[rec].x); }
 
 // first item of item i's granule in the window (keys sorted): lower bound of its key
 static __device__ __noinline__ u64 seg_start(const K7Ctx* k, u64 i) {
@@ -204,7 +208,7 @@ static __device__ __noinline__ void vc_check(const K7Ctx* k, u64 lo, u64 hi, u32
   }
   const u32 nc = cm == SH_R_VC ? crwl : (cm == SH_R_EPOCH ? 1u : 0u);
   for (u32 q = nc; q-- > 0;) {
-    const uint2 e = cm == SH_R_VC ? k->pool[crr + q] : make_uint2(crr, crwl);
+    const uint2 e = cm == SH_R_VC ? k->pool[crr + q] : make_uint2(crr, (rec_warp(c, crr) << 5) | crwl);
     const u32 tid = e.y;
     if (dup_of(tid, lo, q + 1)) continue;
     if (ns < 32) seen[ns++] = tid;
@@ -221,7 +225,7 @@ static __device__ __noinline__ void put_state(const K7Ctx* k, u32 key, u32 wr, u
   if (mode == SH_R_EPOCH) {
     const u32 ev = __ldg(k->evs + hi);
     e1.x = k->R0 + (ev >> 5);
-    e1.y = (item_warp(k, ev) << 5) | (ev & 31u);
+    e1.y = ev & 31u;
   } else if (mode == SH_R_VC) {
     const u32 nc = cm == SH_R_VC ? crwl : (cm == SH_R_EPOCH ? 1u : 0u);
     const u32 m = nc + (u32)(hi + 1 - lo);
@@ -230,7 +234,8 @@ static __device__ __noinline__ void put_state(const K7Ctx* k, u32 key, u32 wr, u
       set_err(k->c.err, ERR_OVERFLOW);  // cannot happen: the host sizes the pool for the worst case
       return;
     }
-    for (u32 q = 0; q < nc; ++q) k->pool[off + q] = cm == SH_R_VC ? k->pool[crr + q] : make_uint2(crr, crwl);
+    for (u32 q = 0; q < nc; ++q)
+      k->pool[off + q] = cm == SH_R_VC ? k->pool[crr + q] : make_uint2(crr, (rec_warp(k->c, crr) << 5) | crwl);
     for (u64 j = lo; j <= hi; ++j) {
       const u32 ev = __ldg(k->evs + j);
       k->pool[off + nc + (u32)(j - lo)] = make_uint2(k->R0 + (ev >> 5), (item_warp(k, ev) << 5) | (ev & 31u));
@@ -284,7 +289,7 @@ __device__ __forceinline__ void warp_range(u64 n, u32 w, u32 nw, u64& beg, u64& 
 __device__ __forceinline__ bool carried_infl(const K7Ctx* k, const Carry& C, u32 ev_s, const Snap& s_s) {
   if (C.rm == SH_R_VC) return true;
   if (C.rm != SH_R_EPOCH) return false;
-  return !hbq(k, k->c, C.rr, C.rwl & 31u, C.rwl >> 5, k->R0 + (ev_s >> 5), ev_s & 31u, s_s);
+  return !hbq(k, k->c, C.rr, C.rwl, rec_warp(k->c, C.rr), k->R0 + (ev_s >> 5), ev_s & 31u, s_s);
 }
 
 // ---------------------------------------------------------------------- tail summary of an item range
@@ -515,12 +520,11 @@ constexpr int KB_STAGES = 2;
 constexpr u32 KT_UNITS_MAX = 1024;  // units per K7a CTA (G / U)
 constexpr int KB_CHUNK = KT_SWARPS * KT_BLK;     // items per chunk
 constexpr int KB_ROW = KB_CHUNK + 8;             // words per stage
-__global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
-                                                            u32* __restrict__ csegs, u32* __restrict__ bflag,
+__global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
+                                                            u32* __restrict__ bflag,
                                                             u32* __restrict__ n_nontriv) {
   __shared__ __align__(128) u32 s_keys[KB_STAGES][KB_ROW];
   __shared__ u64 s_bar[KB_STAGES];
-  __shared__ u32 s_segs[1];
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const u64 n = *a.n_dev;
   const bool fast_ok = a.sh_in == nullptr && a.sh_out == nullptr;
@@ -540,13 +544,12 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
   if (threadIdx.x == 0) {
     for (int q = 0; q < KB_STAGES; ++q) mbar_init(&s_bar[q], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    s_segs[0] = 0;
   }
   __syncthreads();
   if (threadIdx.x == 0)
     for (int q = 0; q < KB_STAGES; ++q)
       if ((u32)q < n_chunks) issue(q, q);
-  u32 segs = 0, nontriv = 0;
+  u32 nontriv = 0;
   for (u32 c = 0; c < n_chunks; ++c) {
     const int st = (int)(c % KB_STAGES);
     mbar_wait(&s_bar[st], (c / KB_STAGES) & 1u);
@@ -566,14 +569,17 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
       // A block makes no check iff no two neighbouring items (including the items just before and
       // after it) share a granule unless both are atomics.  Absent items are NONE: granule 0x3FFFFFFF
       // (never a real key, keys < 2^30 - 1) with the atomic op bits, so they never form a bad pair.
-      u32 bad = 0, fsegs = 0, mlw = 0;
+      u32 bad = 0;
+      const bool full = nb == (u32)KT_BLK;
 #pragma unroll
       for (int q = 0; q < KT_BLK / 128; ++q) {
         const u32 base = (u32)q * 128u + lane * 4u;  // item index within the block
         const uint4 v = *reinterpret_cast<const uint4*>(sk + off + base);
         u32 kk[4] = {v.x, v.y, v.z, v.w};
+        if (!full) {
 #pragma unroll
-        for (int t = 0; t < 4; ++t) kk[t] = base + (u32)t < nb ? kk[t] : NONE;
+          for (int t = 0; t < 4; ++t) kk[t] = base + (u32)t < nb ? kk[t] : NONE;
+        }
         u32 kprev = __shfl_up_sync(0xFFFFFFFFu, kk[3], 1);
         kprev = lane == 0 ? pk_round : kprev;
         u32 knext = __shfl_down_sync(0xFFFFFFFFu, kk[0], 1);
@@ -588,21 +594,19 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
           const u32 k = kk[t];
-          const u32 x = k ^ kpv;
-          bad |= (x < 4u) & ((k & kpv & 3u) != 3u);
-          fsegs += (x >= 4u) & (k != NONE);
-          mlw = (((k ^ lkw) < 4u) & ((k & 3u) != IOP_LD)) ? (u32)bb + base + (u32)t + 1u : mlw;
+          bad |= ((k ^ kpv) < 4u) & ((k & kpv & 3u) != 3u);
           kpv = k;
         }
         bad |= ((kk[3] ^ knext) < 4u) & ((kk[3] & knext & 3u) != 3u);
       }
       const bool triv = bad == 0u;
-      segs += fsegs;
       if (fast_ok && __all_sync(0xFFFFFFFFu, triv)) {
         // no read has a same-granule read before it (no READINFLATE flags), so the summary is closed-form:
-        // first and last granule, and the last writer of the last granule (keys are sorted: its items are
-        // the block's tail run)
-        mlw = __reduce_max_sync(0xFFFFFFFFu, mlw);
+        // first and last granule, and the last writer of the last granule.  Keys are sorted, so the last
+        // granule's items are the block's tail run, and in a block without bad pairs that run is a single
+        // item or a run of atomics: its last writer is the block's last item unless that is a read (then
+        // the run is that read alone and holds no writer).
+        const u32 mlw = (lkw & 3u) != IOP_LD ? (u32)bb + nb : 0u;
         bs.fk = fkw >> 2;
         bs.lk = lkw >> 2;
         bs.lw = mlw;
@@ -630,13 +634,7 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 3) k_blk_sum(CheckArgs a, u32 
       sums[blk] = sum_ident();
       bflag[blk] = 0;
     }
-  segs = __reduce_add_sync(0xFFFFFFFFu, segs);
-  if (lane == 0) {
-    if (segs) atomicAdd(&s_segs[0], segs);
-    if (nontriv) atomicAdd(n_nontriv, nontriv);
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) csegs[blockIdx.x] = s_segs[0];  // summed by k_range_scan
+  if (lane == 0 && nontriv) atomicAdd(n_nontriv, nontriv);
 }
 
 // ---------------------------------------------------------------------- K7a2: units and CTA scans
@@ -715,18 +713,41 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, u32 n
 }
 
 // ---------------------------------------------------------------------- K7b: the listed blocks
-__global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, const u32* __restrict__ wl,
-                                                                 const u32* __restrict__ wl_cnt,
-                                                                 const Sum* __restrict__ rin,
-                                                                 const Sum* __restrict__ cpre, u32 G, u32 nblk,
-                                                                 const u32* __restrict__ unit_p) {
+// SH (several windows: carried entries in and / or entries out): half the warps per CTA, and per warp
+// the carried entries of the block's granule-first items staged in shared memory with the snapshots
+// (cp.async, all of a lane's loads in flight together), so the lane-sequential rules never wait on a
+// dependent global load per granule.
+template <bool SH>
+struct KtCfg {
+  static constexpr int WARPS = SH ? KT_WARPS / 2 : KT_WARPS;
+  static constexpr size_t WARP_BYTES =
+      KT_WARP_BYTES + (SH ? (size_t)KT_PITCH * (sizeof(uint4) + sizeof(uint2)) : 0);
+};
+
+__device__ __forceinline__ void cp_async8(void* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+
+__device__ __forceinline__ Carry carry_of(const uint4& e0, const uint2& e1) {
+  return Carry{e0.x, e0.y, e0.z, e0.w, e1.x, e1.y};
+}
+
+template <bool SH>
+__global__ void __launch_bounds__(KtCfg<SH>::WARPS * 32, 1) k_check_tile(CheckArgs a, const u32* __restrict__ wl,
+                                                                         const u32* __restrict__ wl_cnt,
+                                                                         const Sum* __restrict__ rin,
+                                                                         const Sum* __restrict__ cpre, u32 G, u32 nblk,
+                                                                         const u32* __restrict__ unit_p) {
+  constexpr int NWARP = KtCfg<SH>::WARPS;
   extern __shared__ __align__(16) unsigned char kt_smem[];
   const int wi = threadIdx.x >> 5;
-  uint4* sS = reinterpret_cast<uint4*>(kt_smem + (size_t)wi * KT_WARP_BYTES);
+  uint4* sS = reinterpret_cast<uint4*>(kt_smem + (size_t)wi * KtCfg<SH>::WARP_BYTES);
   u32* const sK = reinterpret_cast<u32*>(sS + KT_PITCH);
   u32* const sE = sK + KT_PITCH;
+  uint4* const sC0 = reinterpret_cast<uint4*>(sE + KT_PITCH);  // SH: carried e0 of granule-first items
+  uint2* const sC1 = reinterpret_cast<uint2*>(sC0 + KT_PITCH);  // SH: carried (e1.x, e1.y)
   const u64 n = *a.n_dev;
-  const u32 w = blockIdx.x * KT_WARPS + wi, nw = gridDim.x * KT_WARPS;
+  const u32 w = blockIdx.x * NWARP + wi, nw = gridDim.x * NWARP;
   const u32 lane = threadIdx.x & 31;
   const HbCtx& c = a.c;
   const K7Ctx* const kx = a.k;
@@ -760,6 +781,22 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
     // ---- gather the snapshots some query can read: an item with a same-granule neighbour (unless an
     // atomic among atomics: its W check is elided and no read follows it), and with carried
     // state every granule's first item (it checks against the carried entry)
+    if (SH && shadow) {  // first the carried entries of the granule-first items (they decide which
+                         // of those items make a check at all)
+      u32 kp = ppk;
+      for (u32 j = 0; j < cnt; ++j) {
+        const u32 li = l0 + j;
+        const u32 k = sK[tpad(li)];
+        if (kp == NONE || (kp >> 2) != (k >> 2)) {
+          cp_async16(sC0 + tpad(li), a.sh_in + 2 * (u64)(k >> 2));
+          cp_async8(sC1 + tpad(li), a.sh_in + 2 * (u64)(k >> 2) + 1);
+        }
+        kp = k;
+      }
+      cp_async_commit();
+      cp_async_wait0();
+      __syncwarp();
+    }
     {
       u32 kp = ppk, k = cnt ? sK[tpad(l0)] : NONE;
       for (u32 j = 0; j < cnt; ++j) {
@@ -769,8 +806,15 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
         const bool sp = kp != NONE && (kp >> 2) == key, sn = kn != NONE && (kn >> 2) == key;
         const bool atm_only =
             (k & 3u) == IOP_ATOM && (!sp || (kp & 3u) == IOP_ATOM) && (!sn || (kn & 3u) == IOP_ATOM);
-        if (((sp || sn) && !atm_only) || (shadow && !sp))
-          cp_async16(sS + tpad(li), c.snap + R0 + (sE[tpad(li)] >> 5));
+        // a granule-first item checks against the carried entry iff it holds a read state, or a writer
+        // the item's W check is not elided for (an atomic after an atomic)
+        bool need = (sp || sn) && !atm_only;
+        if (SH && shadow && !sp) {
+          const uint4 e0 = sC0[tpad(li)];
+          need |= e0.w != SH_R_NONE ||
+                  ((e0.z & SH_W_VALID) && !((k & 3u) == IOP_ATOM && (e0.z & SH_W_ATOM)));
+        }
+        if (need) cp_async16(sS + tpad(li), c.snap + R0 + (sE[tpad(li)] >> 5));
         kp = k;
         k = kn;
       }
@@ -798,7 +842,9 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
           tlw = 0;
           tfi = NONE;
           tci = false;
-          if (shadow && (k & 3u) == IOP_LD && carried_infl(kx, load_carry(a.sh_in, k >> 2), e, to_snap(sv))) {
+          if (shadow && (k & 3u) == IOP_LD &&
+              carried_infl(kx, SH ? carry_of(sC0[tpad(li)], sC1[tpad(li)]) : load_carry(a.sh_in, k >> 2), e,
+                           to_snap(sv))) {
             tci = true;
             cmask |= 1u << j;
           }
@@ -872,7 +918,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
           lw = 0;
           fi = NONE;
           ci = (cmask >> j) & 1u;
-          C = shadow ? load_carry(a.sh_in, k >> 2) : no_carry();
+          C = shadow ? (SH ? carry_of(sC0[tpad(li)], sC1[tpad(li)]) : load_carry(a.sh_in, k >> 2)) : no_carry();
         }
         if (op == IOP_LD && ((imask >> j) & 1u) && fi == NONE) fi = gi;
         // W_x check (every rule of Fig. 2; atomics only against a plain last write)
@@ -886,10 +932,10 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
           }
         } else if (C.wf & SH_W_VALID) {  // the carried writer (an earlier window: never the same record)
           const bool patm = (C.wf & SH_W_ATOM) != 0;
-          if (!(op == IOP_ATOM && patm) && !hbq(kx, c, C.wr, C.wwl & 31u, C.wwl >> 5, r2, l2, s2)) {
+          if (!(op == IOP_ATOM && patm) && !hbq(kx, c, C.wr, C.wwl, rec_warp(c, C.wr), r2, l2, s2)) {
             const u32 kind = op == IOP_LD ? (patm ? BC_KIND_AR : BC_KIND_WR)
                                           : op == IOP_ATOM ? BC_KIND_WA : (patm ? BC_KIND_AW : BC_KIND_WW);
-            emit(kx, k >> 2, r2, l2, C.wr, C.wwl & 31u, kind);
+            emit(kx, k >> 2, r2, l2, C.wr, C.wwl, kind);
           }
         }
         if (op != IOP_LD) {
@@ -921,7 +967,7 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
             }
           } else if (!same && C.rm != SH_R_NONE) {  // the granule's first item: the carried read state
             if (C.rm == SH_R_EPOCH) {
-              if (!hbq(kx, c, C.rr, C.rwl & 31u, C.rwl >> 5, r2, l2, s2)) emit(kx, k >> 2, r2, l2, C.rr, C.rwl & 31u, kind);
+              if (!hbq(kx, c, C.rr, C.rwl, rec_warp(c, C.rr), r2, l2, s2)) emit(kx, k >> 2, r2, l2, C.rr, C.rwl, kind);
             } else {
               vc_check(kx, 1, 0, r2, l2, s2.warp, s2.ps, s2.node, s2.blab, k >> 2, kind, C.rm, C.rr, C.rwl);
             }
@@ -934,23 +980,26 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
           ci = false;
         }
         // ---- the granule's last item of the window: its shadow entry for the next window
-        if (a.sh_out) {
+        if (SH && a.sh_out) {
           const u32 kn = li + 1 < nb ? sK[tpad(li + 1)] : knext;
           if (kn == NONE || (kn >> 2) != (k >> 2)) {
             u32 wr = C.wr, wwl = C.wwl, wf = C.wf;
-            if (lw) {  // (its warp from the snapshot table: a lone writer's snapshot is not gathered)
+            if (lw) {
               wr = R0 + (we >> 5);
-              wwl = (item_warp(kx, we) << 5) | (we & 31u);
+              wwl = we & 31u;
               wf = SH_W_VALID | ((wk & 3u) == IOP_ATOM ? SH_W_ATOM : 0u);
             }
-            if (op != IOP_LD) {
-              put_state(kx, k >> 2, wr, wwl, wf, SH_R_NONE, 1, 0, SH_R_NONE, 0, 0);
+            // no read state (a writer ends the window's run) or an epoch (the last read, gathered): two
+            // stores inline; a read vector (pool append) out of line
+            if (op != IOP_LD || (!(lw == 0 && ci) && fi == NONE)) {
+              uint4* const o = a.sh_out + 2 * (u64)(k >> 2);
+              const bool ep = op == IOP_LD;
+              o[0] = make_uint4(wr, wwl, wf, ep ? SH_R_EPOCH : SH_R_NONE);
+              o[1] = make_uint4(ep ? R0 + (e >> 5) : 0u, ep ? e & 31u : 0u, k >> 2, 0u);
             } else if (lw == 0 && ci) {
               put_state(kx, k >> 2, wr, wwl, wf, SH_R_VC, seg_start(kx, gi), gi, C.rm, C.rr, C.rwl);
-            } else if (fi != NONE) {
-              put_state(kx, k >> 2, wr, wwl, wf, SH_R_VC, (u64)fi - 1, gi, SH_R_NONE, 0, 0);
             } else {
-              put_state(kx, k >> 2, wr, wwl, wf, SH_R_EPOCH, gi, gi, SH_R_NONE, 0, 0);
+              put_state(kx, k >> 2, wr, wwl, wf, SH_R_VC, (u64)fi - 1, gi, SH_R_NONE, 0, 0);
             }
           }
         }
@@ -971,40 +1020,71 @@ __global__ void __launch_bounds__(KT_WARPS * 32, 1) k_check_tile(CheckArgs a, co
 // Statistics only (bc_config.flags & BC_F_COUNT_GATHERS): the number of items whose record clock
 // snapshot K7 reads -- the gather rule over the sorted items -- for the roofline's algorithmic
 // bytes.  A separate pass so that the hot kernel carries no counter.
-__global__ void k_count_gathers(const u32* __restrict__ keys, const u64* __restrict__ n_dev, u64* __restrict__ out) {
+__global__ void k_count_gathers(const u32* __restrict__ keys, const u64* __restrict__ n_dev, u64* __restrict__ out,
+                                u64* __restrict__ segs) {
   const u64 n = *n_dev;
-  u32 cnt = 0;
+  u32 cnt = 0, sg = 0;
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) {
     const u32 k = keys[i], kp = i ? keys[i - 1] : NONE, kn = i + 1 < n ? keys[i + 1] : NONE;
     const u32 key = k >> 2;
     const bool sp = kp != NONE && (kp >> 2) == key, sn = kn != NONE && (kn >> 2) == key;
     const bool atm_only = (k & 3u) == IOP_ATOM && (!sp || (kp & 3u) == IOP_ATOM) && (!sn || (kn & 3u) == IOP_ATOM);
     cnt += (sp || sn) && !atm_only;
+    sg += !sp;  // the granule's first item of the window
   }
   cnt = __reduce_add_sync(0xFFFFFFFFu, cnt);
+  sg = __reduce_add_sync(0xFFFFFFFFu, sg);
   if ((threadIdx.x & 31) == 0 && cnt) atomicAdd((unsigned long long*)out, (unsigned long long)cnt);
+  if ((threadIdx.x & 31) == 0 && sg) atomicAdd((unsigned long long*)segs, (unsigned long long)sg);
+}
+
+// Shadow commit after a window: K7 read the carried entries from `tab` and wrote the entry of every
+// granule the window touched into `out` (at the granule's last item), so `tab` could not be updated in
+// place while K7 ran.  Now copy exactly the touched entries back: one per granule segment of the sorted
+// items (its last item).  Untouched entries are already current in `tab`, so a window costs 4 B per item
+// + 64 B per touched granule instead of a copy of the whole table (32 B x every granule key).
+__global__ void k_shadow_commit(const u32* __restrict__ keys, const u64* __restrict__ n_dev,
+                                const uint4* __restrict__ out, uint4* __restrict__ tab) {
+  const u64 n = *n_dev;
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) {
+    const u32 k = __ldg(keys + i) >> 2;
+    if (i + 1 < n && (__ldg(keys + i + 1) >> 2) == k) continue;
+    const uint4 e0 = __ldg(out + 2 * (u64)k), e1 = __ldg(out + 2 * (u64)k + 1);
+    tab[2 * (u64)k] = e0;
+    tab[2 * (u64)k + 1] = e1;
+  }
 }
 
 }  // namespace
 
-void launch_count_gathers(const u32* keys, const u64* n_dev, u64* out, cudaStream_t st) {
-  k_count_gathers<<<148 * 8, 256, 0, st>>>(keys, n_dev, out);
+void launch_shadow_commit(const u32* keys, const u64* n_dev, u64 n_max, const uint4* out, uint4* tab,
+                          cudaStream_t st) {
+  if (n_max == 0) return;
+  const u64 want = (n_max + 255) / 256;
+  k_shadow_commit<<<(unsigned)std::min<u64>(want, 148 * 16), 256, 0, st>>>(keys, n_dev, out, tab);
+  ++g_launches;
+}
+
+void launch_count_gathers(const u32* keys, const u64* n_dev, u64* out, u64* segs, cudaStream_t st) {
+  k_count_gathers<<<148 * 8, 256, 0, st>>>(keys, n_dev, out, segs);
   ++g_launches;
 }
 
 // per device: K7b grid (fully co-resident persistent CTAs) and its shared-memory opt-in
+template <bool SH>
 static int k7_grid(int dev) {
   static int grid[64] = {};
   if (dev < 0 || dev >= 64) dev = 0;
   if (!grid[dev]) {
-    const size_t smem_tile = (size_t)KT_WARPS * KT_WARP_BYTES;
+    constexpr int NW = KtCfg<SH>::WARPS;
+    const size_t smem_tile = (size_t)NW * KtCfg<SH>::WARP_BYTES;
     int sms = 0, per = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(k_check_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_tile);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_check_tile, KT_WARPS * 32, smem_tile);
+    cudaFuncSetAttribute(k_check_tile<SH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_tile);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_check_tile<SH>, NW * 32, smem_tile);
     if (per < 1) per = 1;
     int g = sms * per;
-    if (g * KT_WARPS > 148 * 64) g = 148 * 64 / KT_WARPS;
+    if (g * NW > 148 * 64) g = 148 * 64 / NW;
     grid[dev] = g;
   }
   return grid[dev];
@@ -1023,7 +1103,9 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   if (L.n_max == 0) return;
   int dev = 0;
   cudaGetDevice(&dev);
-  const int grid = k7_grid(dev);
+  const bool SH = L.sh_in || L.sh_out;
+  const int grid = SH ? k7_grid<true>(dev) : k7_grid<false>(dev);
+  const int k7b_warps = SH ? KtCfg<true>::WARPS : KtCfg<false>::WARPS;
   const u64 nblk = (L.n_max + KT_BLK - 1) / KT_BLK;
   u32 G = KT_SWARPS;  // blocks per K7a CTA: a power of two >= KT_SWARPS (whole chunks, whole units)
   while ((u64)G * K7A_CTAS < nblk) G <<= 1;
@@ -1073,17 +1155,22 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   a.rin = nullptr;
   a.no_sv = L.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   a.values = L.values;
-  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, csegs, bflag, n_nontriv);
+  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, bflag, n_nontriv);
   k_blk_units<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, rin, ctot, wl, wl_cnt, bflag, n_nontriv,
-                                              (u32)grid * KT_WARPS, unit_p);
-  k_range_scan<<<1, 1024, 0, st>>>(ctot, nct, cpre, csegs, L.seg_cnt);
-  k_check_tile<<<grid, KT_WARPS * 32, (size_t)KT_WARPS * KT_WARP_BYTES, st>>>(a, wl, wl_cnt, rin, cpre, G, (u32)nblk,
-                                                                            unit_p);
+                                              (u32)grid * k7b_warps, unit_p);
+  k_range_scan<<<1, 1024, 0, st>>>(ctot, nct, cpre, nullptr, nullptr);  // segments: stats pass
+  if (SH)
+    k_check_tile<true><<<grid, KtCfg<true>::WARPS * 32, (size_t)KtCfg<true>::WARPS * KtCfg<true>::WARP_BYTES, st>>>(
+        a, wl, wl_cnt, rin, cpre, G, (u32)nblk, unit_p);
+  else
+    k_check_tile<false><<<grid, KtCfg<false>::WARPS * 32, (size_t)KtCfg<false>::WARPS * KtCfg<false>::WARP_BYTES,
+                          st>>>(a, wl, wl_cnt, rin, cpre, G, (u32)nblk, unit_p);
   g_launches += 4;
 }
 
 void preload_check() {
-  preload(k_blk_sum, k_blk_units, k_check_tile, k_count_gathers, k_range_scan);
+  preload(k_blk_sum, k_blk_units, k_check_tile<false>, k_check_tile<true>, k_count_gathers, k_range_scan,
+          k_shadow_commit);
 }
 
 }  // namespace bc

@@ -163,7 +163,7 @@ struct CheckLaunch {
   u64 n_max;            // upper bound of the item count
   u32 R0;               // first record of the window
   const uint4* sh_in;   // carried shadow entries (2 x uint4 per granule) or null (first window)
-  uint4* sh_out;        // shadow entries after the window, or null (last window)
+  uint4* sh_out;        // entries of the granules the window touches (others untouched), or null (last window)
   uint2* pool;          // append-only read-vector pool (record, warp << 5 | lane)
   u32* pool_cnt;
   u32 pool_cap;
@@ -176,7 +176,10 @@ struct CheckLaunch {
 };
 void launch_check(const CheckLaunch& L, cudaStream_t st);
 
-void launch_count_gathers(const u32* keys, const u64* n_dev, u64* out, cudaStream_t st);
+void launch_count_gathers(const u32* keys, const u64* n_dev, u64* out, u64* segs, cudaStream_t st);
+// after K7 of a window: tab[k] = out[k] for every granule k the sorted items touch
+void launch_shadow_commit(const u32* keys, const u64* n_dev, u64 n_max, const uint4* out, uint4* tab,
+                          cudaStream_t st);
 
 // finalize.cu
 void launch_page_list(const u32* words, const u32* wl_prefix, const u32* page_bits, u64 n_words, u32* page_num,

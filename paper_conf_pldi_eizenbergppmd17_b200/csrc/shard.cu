@@ -477,10 +477,7 @@ bc_status detect_sharded(bc_ctx* c, Scratch& S) {
     ++g_launches;
     // ---- K7 on the owned granules
     uint4* sh_out = (multi && k + 1 < nwin) ? sh_nxt : nullptr;
-    if (sh_out) {
-      if (have_state) cudaMemcpyAsync(sh_out, sh_cur, 2 * n_keys * sizeof(uint4), cudaMemcpyDeviceToDevice, st);
-      else cudaMemsetAsync(sh_out, 0, 2 * n_keys * sizeof(uint4), st);
-    }
+    if (sh_out && !have_state) cudaMemsetAsync(sh_cur, 0, 2 * n_keys * sizeof(uint4), st);
     CheckLaunch L{};
     L.c = hc;
     L.keys = fk;
@@ -500,7 +497,7 @@ bc_status detect_sharded(bc_ctx* c, Scratch& S) {
     sx.segments += wo.segments;
     ms_chk += wo.ms_check;
     if (sh_out) {
-      std::swap(sh_cur, sh_nxt);
+      launch_shadow_commit(fk, cnt + C_ITEMS, n_recv, sh_nxt, sh_cur, st);
       have_state = true;
     }
   }

@@ -210,7 +210,7 @@ __global__ void k_warp_start(const u32* __restrict__ skeys, u64 n, u32 n_warps, 
 // so the per-record snapshot {warp, ps, node, phase} is written by 32 lanes in parallel.  Per IF it writes the two
 // nodes {mask, parent, popen}; per BAR its record and the warp's next record (barrier feasibility)
 // and a BARRIER_DIVERGENCE finding when the mask is not the warp's initial mask.
-__global__ void __launch_bounds__(256) k_replay(const uint4* __restrict__ hdr16, const u32* __restrict__ wrec,
+__global__ void __launch_bounds__(256, 4) k_replay(const uint4* __restrict__ hdr16, const u32* __restrict__ wrec,
                                                 const u32* __restrict__ gidx, const u32* __restrict__ warp_start, Geo g,
                                                 const u32* __restrict__ node_base, const u32* __restrict__ bar_base,
                                                 uint4* __restrict__ snap, uint4* __restrict__ nodes,
