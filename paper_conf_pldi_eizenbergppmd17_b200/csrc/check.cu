@@ -514,6 +514,69 @@ __device__ __forceinline__ void load_keys16(const u32* __restrict__ keys, u64 bb
 
 static __device__ __noinline__ Sum tail_sum_nl(const K7Ctx* k, u64 beg, u64 end) { return tail_sum(k, beg, end); }
 
+// A block with no bad pair (see k_blk_sum) in a run of several windows.  Its granule-first items are
+// checked against the carried entries: the block stays trivial iff no entry holds a read state and no
+// entry holds a writer the item's W check would see (only an atomic after an atomic is elided,
+// P:L661-670) -- then no item makes a check at all.  A trivial block then writes the entry of each of
+// its granule-last items for the next window: a writer (ST / ATOM) is the new W with no read state; a
+// read is alone in its granule in the window (no bad pair), found no carried writer or read state, so
+// its entry is no writer and the read's epoch (Fig. 8).  sk: the block's key words in
+// shared memory (sk[-1]: the item before, sk[nb]: the item after).  Warp-uniform result.
+static __device__ __forceinline__ bool sh_block(const CheckArgs& a, const u32* sk, u64 bb, u32 nb, u64 n, u32 lane) {
+  const u32 kb = bb > 0 ? sk[-1] : NONE, ka = bb + nb < n ? sk[nb] : NONE;
+  if (a.sh_in) {
+    bool need = false;
+#pragma unroll
+    for (int q = 0; q < KT_BLK / 128; ++q) {
+#pragma unroll
+      for (int t = 0; t < 4; ++t) {
+        const u32 i = (u32)q * 128u + lane * 4u + (u32)t;
+        if (i < nb) {
+          const u32 k = sk[i], kp = i ? sk[i - 1] : kb;
+          if (kp == NONE || (kp >> 2) != (k >> 2)) {
+            const uint4 e0 = __ldg(a.sh_in + 2 * (u64)(k >> 2));
+            need |= e0.w != SH_R_NONE || ((e0.z & SH_W_VALID) && !((k & 3u) == IOP_ATOM && (e0.z & SH_W_ATOM)));
+          }
+        }
+      }
+    }
+    if (__any_sync(0xFFFFFFFFu, need)) return false;
+  }
+  if (a.sh_out) {
+#pragma unroll
+    for (int q = 0; q < KT_BLK / 128; ++q) {
+      const u32 i0 = (u32)q * 128u + lane * 4u;
+      u32 ev[4];
+      if (i0 + 4 <= nb) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4*>(a.evs + bb + i0));
+        ev[0] = v.x; ev[1] = v.y; ev[2] = v.z; ev[3] = v.w;
+      } else {
+#pragma unroll
+        for (int t = 0; t < 4; ++t) ev[t] = i0 + t < nb ? __ldg(a.evs + bb + i0 + t) : 0u;
+      }
+#pragma unroll
+      for (int t = 0; t < 4; ++t) {
+        const u32 i = i0 + (u32)t;
+        if (i < nb) {
+          const u32 k = sk[i], kn = i + 1 < nb ? sk[i + 1] : ka;
+          if (kn == NONE || (kn >> 2) != (k >> 2)) {
+            const u32 op = k & 3u, rec = a.R0 + (ev[t] >> 5), ln = ev[t] & 31u;
+            uint4* const o = a.sh_out + 2 * (u64)(k >> 2);
+            if (op != IOP_LD) {
+              o[0] = make_uint4(rec, ln, SH_W_VALID | (op == IOP_ATOM ? SH_W_ATOM : 0u), SH_R_NONE);
+              o[1] = make_uint4(0u, 0u, k >> 2, 0u);
+            } else {
+              o[0] = make_uint4(0u, 0u, 0u, SH_R_EPOCH);
+              o[1] = make_uint4(rec, ln, k >> 2, 0u);
+            }
+          }
+        }
+      }
+    }
+  }
+  return true;
+}
+
 // key words stream through shared memory: one chunk = KT_SWARPS blocks (+ 4 words on each side for
 // the neighbours of the first / last item), KB_STAGES chunks in flight per CTA (1-D TMA bulk copies)
 constexpr int KB_STAGES = 2;
@@ -599,8 +662,11 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 
         }
         bad |= ((kk[3] ^ knext) < 4u) & ((kk[3] & knext & 3u) != 3u);
       }
-      const bool triv = bad == 0u;
-      if (fast_ok && __all_sync(0xFFFFFFFFu, triv)) {
+      bool triv = __all_sync(0xFFFFFFFFu, bad == 0u);
+      // several windows: the carried entries decide too, and a trivial block writes its granules'
+      // entries for the next window here instead of in K7b
+      if (!fast_ok && triv) triv = sh_block(a, sk + off, bb, nb, n, lane);
+      if (triv) {
         // no read has a same-granule read before it (no READINFLATE flags), so the summary is closed-form:
         // first and last granule, and the last writer of the last granule.  Keys are sorted, so the last
         // granule's items are the block's tail run, and in a block without bad pairs that run is a single

@@ -9,6 +9,8 @@ timeout 900 python bench.py --steps 5 --no-cpu-baseline > $O/bench_c4.json 2> $O
 timeout 1200 python bench.py --config c5 --steps 3 --no-cpu-baseline --no-ncu > $O/bench_c5.json 2> $O/bench_c5.err; echo c5=$?
 for c in c4 c5; do timeout 20 python -c "
 import json; d=json.load(open('$O/bench_$c.json')); print('$c', round(d['value']/1e9,3), 'Gev/s', round(d['ms_per_step'],4), 'ms', 'K7', round(d['roofline']['frac'],4), d['roofline']['kernel_ms'], d['roofline']['traffic'], d.get('phases_ms'), d['config']['windows'])"; done
+timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv -k regex:"k_blk|k_check|k_range|k_shadow" --log-file $O/launches_c4_k7.csv python tools/prof_one.py c4 > $O/l4.log 2>&1; echo l4=$?
+python tools/launches.py $O/launches_c4_k7.csv > $O/launches_c4_k7.txt 2>&1; cat $O/launches_c4_k7.txt
 if [ -z "$NO_NCU" ]; then
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv -k regex:"k_blk|k_check|k_range|k_shadow" --log-file $O/launches_c5_k7.csv python tools/prof_one.py c5 > $O/l5.log 2>&1; echo l5=$?
 python tools/launches.py $O/launches_c5_k7.csv > $O/launches_c5_k7.txt 2>&1; cat $O/launches_c5_k7.txt
