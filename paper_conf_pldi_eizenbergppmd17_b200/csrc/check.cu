@@ -366,11 +366,42 @@ __device__ Sum tail_sum(const K7Ctx* kc, u64 beg, u64 end) {
   return s;
 }
 
+#ifndef KT_IPL_
+#define KT_IPL_ 16
+#endif
+constexpr int KT_IPL = KT_IPL_;              // items per lane per block
+constexpr int KT_BLK = 32 * KT_IPL;          // items per warp block
+constexpr int KT_PITCH = 32 * (KT_IPL + 1);  // padded entries per array
+#ifndef KT_NWARPS
+#define KT_NWARPS 16
+#endif
+constexpr int KT_WARPS = KT_NWARPS;
+constexpr size_t KT_WARP_BYTES = (size_t)KT_PITCH * (sizeof(uint4) + 2 * sizeof(u32));
+
+// Partition of a window's items among K7a's persistent CTAs, from the device-side item count (the host
+// knows only the window's upper bound, which can be far larger: C4's never-written pages drop 38 % of
+// the slots): CTA c owns the blocks [c * G, (c + 1) * G), G a multiple of 64 (whole K7a chunks, and
+// every power-of-two unit size up to 64 divides it), nct <= K7A_CTAS CTAs with blocks.
+constexpr u32 K7A_CTAS = 148 * 4;
+struct K7Part {
+  u32 nblk, G, nct;
+};
+__device__ __forceinline__ K7Part k7_part(u64 n) {
+  K7Part p;
+  p.nblk = (u32)((n + KT_BLK - 1) / KT_BLK);
+  u32 G = (p.nblk + K7A_CTAS - 1) / K7A_CTAS;
+  p.G = G < 64u ? 64u : (G + 63u) & ~63u;
+  p.nct = (p.nblk + p.G - 1) / p.G;
+  return p;
+}
+
 // ---------------------------------------------------------------------- K7s: exclusive scan of summaries
 // One CTA: thread t combines entries [t*P, t*P + P) sequentially, a Hillis-Steele scan over the
 // 1024 thread totals, then every thread writes the exclusive prefix of its entries.
-__global__ void __launch_bounds__(1024) k_range_scan(const Sum* __restrict__ in, u32 nw, Sum* __restrict__ out,
-                                                     const u32* __restrict__ segs, u64* __restrict__ seg_cnt) {
+__global__ void __launch_bounds__(1024) k_range_scan(const Sum* __restrict__ in, const u64* __restrict__ n_dev,
+                                                     Sum* __restrict__ out, const u32* __restrict__ segs,
+                                                     u64* __restrict__ seg_cnt) {
+  const u32 nw = k7_part(*n_dev).nct;  // the K7a CTA totals
   // chunks of 2048 entries: coalesced loads into shared memory, thread t combines entries 2t, 2t+1,
   // warp shuffle scans of the thread totals and of the 32 warp totals, a running carry across chunks
   constexpr int PER = 2;
@@ -446,17 +477,6 @@ __global__ void __launch_bounds__(1024) k_range_scan(const Sum* __restrict__ in,
 //             check against the epoch or the read vector, same-value filter), with the carried
 //             entry as the state before a granule's first item; at a granule's last item it writes
 //             the granule's entry for the next window
-#ifndef KT_IPL_
-#define KT_IPL_ 16
-#endif
-constexpr int KT_IPL = KT_IPL_;              // items per lane per block
-constexpr int KT_BLK = 32 * KT_IPL;          // items per warp block
-constexpr int KT_PITCH = 32 * (KT_IPL + 1);  // padded entries per array
-#ifndef KT_NWARPS
-#define KT_NWARPS 16
-#endif
-constexpr int KT_WARPS = KT_NWARPS;
-constexpr size_t KT_WARP_BYTES = (size_t)KT_PITCH * (sizeof(uint4) + 2 * sizeof(u32));
 
 __device__ __forceinline__ u32 tpad(u32 i) { return i + i / KT_IPL; }
 
@@ -583,13 +603,16 @@ constexpr int KB_STAGES = 2;
 constexpr u32 KT_UNITS_MAX = 1024;  // units per K7a CTA (G / U)
 constexpr int KB_CHUNK = KT_SWARPS * KT_BLK;     // items per chunk
 constexpr int KB_ROW = KB_CHUNK + 8;             // words per stage
-__global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
+__global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum* __restrict__ sums,
                                                             u32* __restrict__ bflag,
                                                             u32* __restrict__ n_nontriv) {
   __shared__ __align__(128) u32 s_keys[KB_STAGES][KB_ROW];
   __shared__ u64 s_bar[KB_STAGES];
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const u64 n = *a.n_dev;
+  const K7Part P = k7_part(n);
+  const u32 nblk = P.nblk, G = P.G;
+  if (blockIdx.x >= P.nct) return;  // CTA-uniform
   const bool fast_ok = a.sh_in == nullptr && a.sh_out == nullptr;
   const u32 b0 = blockIdx.x * G, b1 = min(nblk, b0 + G);
   const u32 l0 = lane * KT_IPL;
@@ -694,12 +717,6 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 
       issue(c + KB_STAGES, st);
     }
   }
-  // blocks past the item count (K7's blocks are sized from its upper bound): empty
-  for (u32 blk = b0 + threadIdx.x; blk < b1; blk += KT_SWARPS * 32)
-    if ((u64)blk * KT_BLK >= n) {
-      sums[blk] = sum_ident();
-      bflag[blk] = 0;
-    }
   if (lane == 0 && nontriv) atomicAdd(n_nontriv, nontriv);
 }
 
@@ -709,7 +726,7 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, u32 
 // sparse ones), one warp per unit carrying the automaton state from block to block.  Per unit with a
 // check: one bounded tail walk gives the unit's summary (placed at its last block, identity at the
 // others) and the unit is listed.  Then each CTA scans its blocks' summaries (rin) and writes its total.
-__global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, u32 nblk, u32 G, Sum* __restrict__ sums,
+__global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, Sum* __restrict__ sums,
                                                               Sum* __restrict__ rin, Sum* __restrict__ ctot,
                                                               u32* __restrict__ wl, u32* __restrict__ wl_cnt,
                                                               const u32* __restrict__ bflag,
@@ -719,12 +736,14 @@ __global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, u32 n
   __shared__ Sum s_carry;
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const u64 n = *a.n_dev;
+  const K7Part P = k7_part(n);
+  const u32 nblk = P.nblk, G = P.G;
   const u32 b0 = blockIdx.x * G, b1 = min(nblk, b0 + G);
   // U: the largest power of two with at least two units per K7b warp (load balance), at most G (a power
   // of two); 1 on sparse traces
   const u32 nt = *n_nontriv;
   u32 U = 1;
-  while (U * 2 <= G && (u64)U * 2 * 2 * nw_b <= nt) U <<= 1;
+  while (U * 2 <= 64u && U * 2 <= G && (u64)U * 2 * 2 * nw_b <= nt) U <<= 1;  // U | G (G: a multiple of 64)
   while (G / U > KT_UNITS_MAX) U <<= 1;
   if (blockIdx.x == 0 && threadIdx.x == 0) *unit_out = U;
   if (threadIdx.x == 0) s_carry = sum_ident();
@@ -802,7 +821,7 @@ template <bool SH>
 __global__ void __launch_bounds__(KtCfg<SH>::WARPS * 32, 1) k_check_tile(CheckArgs a, const u32* __restrict__ wl,
                                                                          const u32* __restrict__ wl_cnt,
                                                                          const Sum* __restrict__ rin,
-                                                                         const Sum* __restrict__ cpre, u32 G, u32 nblk,
+                                                                         const Sum* __restrict__ cpre, u32 nblk,
                                                                          const u32* __restrict__ unit_p) {
   constexpr int NWARP = KtCfg<SH>::WARPS;
   extern __shared__ __align__(16) unsigned char kt_smem[];
@@ -828,7 +847,7 @@ __global__ void __launch_bounds__(KtCfg<SH>::WARPS * 32, 1) k_check_tile(CheckAr
     const u32 u = wl[task];
     const u32 blk0 = u * U, blk1 = min(nblk, blk0 + U);
     // state entering the unit: its K7a CTA's prefix (K7s), then the prefix within that CTA
-    Sum carry = combine(cpre[blk0 / G], rin[blk0]);
+    Sum carry = combine(cpre[blk0 / k7_part(n).G], rin[blk0]);
     u32 pkx = blk0 > 0 ? __ldg(a.keys + (u64)blk0 * KT_BLK - 1) : NONE;  // the item before the block
     for (u32 bi = blk0; bi < blk1; ++bi) {
     const u64 bb = (u64)bi * KT_BLK;
@@ -1158,7 +1177,6 @@ static int k7_grid(int dev) {
 
 // status scratch: [K7Ctx][Sum sums[nblk]][Sum rin[nblk]][Sum ctot[nct]][Sum cpre[nct]][u32 wl[nblk]][u32 wl_cnt]
 // [u32 csegs[nct]]
-constexpr u32 K7A_CTAS = 148 * 4;
 size_t check_status_bytes(u64 n) {
   const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1, nct = K7A_CTAS + 2;
   return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (2 * nblk + 2 * nct + 4) * sizeof(Sum) +
@@ -1172,12 +1190,8 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   const bool SH = L.sh_in || L.sh_out;
   const int grid = SH ? k7_grid<true>(dev) : k7_grid<false>(dev);
   const int k7b_warps = SH ? KtCfg<true>::WARPS : KtCfg<false>::WARPS;
-  const u64 nblk = (L.n_max + KT_BLK - 1) / KT_BLK;
-  u32 G = KT_SWARPS;  // blocks per K7a CTA: a power of two >= KT_SWARPS (whole chunks, whole units)
-  while ((u64)G * K7A_CTAS < nblk) G <<= 1;
-  // (G / U units per CTA must fit KT_UNITS_MAX: U grows with the count of blocks with checks, so only
-  //  G > KT_UNITS_MAX with almost no such blocks could exceed it -- U is then raised to G / KT_UNITS_MAX)
-  const u32 nct = (u32)((nblk + G - 1) / G);
+  const u64 nblk = (L.n_max + KT_BLK - 1) / KT_BLK;  // upper bound (array sizes); the kernels partition the
+  const u32 nct = K7A_CTAS;                           // device-side item count (k7_part)
   char* base = (char*)L.status;
   K7Ctx* kdev = reinterpret_cast<K7Ctx*>(base);
   Sum* sums = reinterpret_cast<Sum*>(base + ((sizeof(K7Ctx) + 255) & ~(size_t)255));
@@ -1221,16 +1235,16 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   a.rin = nullptr;
   a.no_sv = L.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   a.values = L.values;
-  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, bflag, n_nontriv);
-  k_blk_units<<<nct, KT_SWARPS * 32, 0, st>>>(a, (u32)nblk, G, sums, rin, ctot, wl, wl_cnt, bflag, n_nontriv,
+  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, sums, bflag, n_nontriv);
+  k_blk_units<<<nct, KT_SWARPS * 32, 0, st>>>(a, sums, rin, ctot, wl, wl_cnt, bflag, n_nontriv,
                                               (u32)grid * k7b_warps, unit_p);
-  k_range_scan<<<1, 1024, 0, st>>>(ctot, nct, cpre, nullptr, nullptr);  // segments: stats pass
+  k_range_scan<<<1, 1024, 0, st>>>(ctot, L.n_dev, cpre, nullptr, nullptr);  // segments: stats pass
   if (SH)
     k_check_tile<true><<<grid, KtCfg<true>::WARPS * 32, (size_t)KtCfg<true>::WARPS * KtCfg<true>::WARP_BYTES, st>>>(
-        a, wl, wl_cnt, rin, cpre, G, (u32)nblk, unit_p);
+        a, wl, wl_cnt, rin, cpre, (u32)nblk, unit_p);
   else
     k_check_tile<false><<<grid, KtCfg<false>::WARPS * 32, (size_t)KtCfg<false>::WARPS * KtCfg<false>::WARP_BYTES,
-                          st>>>(a, wl, wl_cnt, rin, cpre, G, (u32)nblk, unit_p);
+                          st>>>(a, wl, wl_cnt, rin, cpre, (u32)nblk, unit_p);
   g_launches += 4;
 }
 
