@@ -308,7 +308,7 @@ bc_status bc_init(const bc_config* cfg, bc_ctx** out) {
     uint64_t thr = ~0ull;
     cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
   }
-  for (int i = 0; i < 16; ++i) cudaEventCreate(&c->ev[i]);
+  for (int i = 0; i < 18; ++i) cudaEventCreate(&c->ev[i]);
   cudaMallocHost(&c->hcnt, C_N * sizeof(u64));
   if (cudaGetLastError() != cudaSuccess) {
     bc_destroy(c);
@@ -340,7 +340,7 @@ void bc_destroy(bc_ctx* c) {
   if (c->hcnt) cudaFreeHost(c->hcnt);
   if (c->dhdr) cudaFreeHost(c->dhdr);
   if (c->dstream) cudaStreamDestroy(c->dstream);
-  for (int i = 0; i < 16; ++i)
+  for (int i = 0; i < 18; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
   if (c->own_stream) cudaStreamDestroy(c->stream);
   delete c;
@@ -593,13 +593,14 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
   const int kbits = bits_for(n_keys ? n_keys - 1 : 0);
   u64 n_r = sw ? c->s_nr : 0, n_items = 0, pool_used = sw ? c->s_pool : 0;
   float ms_ex = 0, ms_sort = 0, ms_chk = 0;
+  bool commit_pending = false;
   for (u32 k = 0; k < nwin; ++k) {
     const u64 R0 = wst[k], R1 = wst[k + 1], b = wbd[k];
     if (R0 == R1) continue;
     ++sx.windows;
     // ---- K4: expansion (static slots from the header's per-record upper bounds)
     cudaEventRecord(c->ev[14], st);
-    launch_expand(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, nullptr, R0, ikeys, ievs, err, st);
+    launch_expand(recs, hdr16, g, page_bits, page_rank, shared_base, cum, R0, R1, nullptr, R0, ikeys, ievs, err, st);
     cudaEventRecord(c->ev[15], st);
     // ---- K5: stable radix sort by granule key; the first pass drops the never-written slots
     cudaEventRecord(c->ev[12], st);
@@ -626,6 +627,12 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
     WindowOut wo;
     bc_status ws = check_window(c, L, b, cnt, n_r, pool_used, wo);
     if (ws) return ws;
+    if (commit_pending) {  // the previous window's shadow commit is part of K7's time (the stream is synced)
+      float tc = 0;
+      cudaEventElapsedTime(&tc, c->ev[16], c->ev[17]);
+      ms_chk += tc;
+      commit_pending = false;
+    }
     n_items += wo.items;
     sx.segments += wo.segments;
     sx.clock_gathers += wo.gathers;
@@ -636,7 +643,10 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
     ms_sort += t;
     ms_chk += wo.ms_check;
     if (sh_out) {
+      cudaEventRecord(c->ev[16], st);
       launch_shadow_commit(skey, n_items_dev, b, sh_nxt, sh_cur, st);
+      cudaEventRecord(c->ev[17], st);
+      commit_pending = true;
       have_state = true;
     }
   }

@@ -108,7 +108,6 @@ struct CheckArgs {
   u32 R0;
   const uint4* sh_in;
   uint4* sh_out;
-  const Sum* rin;       // state entering each warp range (k_range_tail + k_range_scan)
   u32 no_sv;
   const u64* values;
 };
@@ -367,7 +366,7 @@ __device__ Sum tail_sum(const K7Ctx* kc, u64 beg, u64 end) {
 }
 
 #ifndef KT_IPL_
-#define KT_IPL_ 16
+#define KT_IPL_ 8  // A/B (K7b on C2 / C3 / C4): 16 -> 8 took 699 / 375 / 53 us to 369 / 223 / 25 us
 #endif
 constexpr int KT_IPL = KT_IPL_;              // items per lane per block
 constexpr int KT_BLK = 32 * KT_IPL;          // items per warp block
@@ -381,7 +380,7 @@ constexpr size_t KT_WARP_BYTES = (size_t)KT_PITCH * (sizeof(uint4) + 2 * sizeof(
 // Partition of a window's items among K7a's persistent CTAs, from the device-side item count (the host
 // knows only the window's upper bound, which can be far larger: C4's never-written pages drop 38 % of
 // the slots): CTA c owns the blocks [c * G, (c + 1) * G), G a multiple of 64 (whole K7a chunks, and
-// every power-of-two unit size up to 64 divides it), nct <= K7A_CTAS CTAs with blocks.
+// whole 8-block chunks), nct <= K7A_CTAS CTAs with blocks.
 constexpr u32 K7A_CTAS = 148 * 4;
 struct K7Part {
   u32 nblk, G, nct;
@@ -395,76 +394,35 @@ __device__ __forceinline__ K7Part k7_part(u64 n) {
   return p;
 }
 
-// ---------------------------------------------------------------------- K7s: exclusive scan of summaries
-// One CTA: thread t combines entries [t*P, t*P + P) sequentially, a Hillis-Steele scan over the
-// 1024 thread totals, then every thread writes the exclusive prefix of its entries.
-__global__ void __launch_bounds__(1024) k_range_scan(const Sum* __restrict__ in, const u64* __restrict__ n_dev,
-                                                     Sum* __restrict__ out, const u32* __restrict__ segs,
-                                                     u64* __restrict__ seg_cnt) {
-  const u32 nw = k7_part(*n_dev).nct;  // the K7a CTA totals
-  // chunks of 2048 entries: coalesced loads into shared memory, thread t combines entries 2t, 2t+1,
-  // warp shuffle scans of the thread totals and of the 32 warp totals, a running carry across chunks
-  constexpr int PER = 2;
-  __shared__ Sum sh[1024 * PER];
-  __shared__ Sum s_w[32];
-  __shared__ Sum s_carry;
-  const u32 t = threadIdx.x, lane = t & 31, wi = t >> 5;
-  u64 sg = 0;
-  if (t == 0) s_carry = sum_ident();
-  for (u32 c0 = 0; c0 < nw; c0 += 1024 * PER) {
-    for (u32 q = t; q < 1024 * PER; q += 1024) {
-      sh[q] = c0 + q < nw ? in[c0 + q] : sum_ident();
-      if (segs && c0 + q < nw) sg += segs[c0 + q];
-    }
-    __syncthreads();
-    Sum tot = sum_ident();
-#pragma unroll
-    for (int q = 0; q < PER; ++q) tot = combine(tot, sh[t * PER + q]);
-    Sum incl = tot;
+// ---------------------------------------------------------------------- state entering a block
+// The automaton state entering block b = the exclusive prefix of the block summaries, of which only
+// the tail matters (the last granule's last writer, first inflation, carried inflation).  A summary
+// whose tail granule starts inside its block, or that holds a writer, fixes that tail whatever lies
+// before it (see combine), so the walk back over the summaries stops there: usually at block b - 1,
+// a run of one read-only granule over many blocks takes one step per 32 blocks.  Warp-cooperative.
+__device__ Sum enter_state(const Sum* __restrict__ sums, u32 b) {
+  const u32 lane = threadIdx.x & 31;
+  Sum acc = sum_ident();
+  u32 j = b;
+  while (j > 0) {
+    const u32 lo = j >= 32 ? j - 32 : 0;
+    const u32 i = lo + lane;
+    Sum incl = i < j ? sums[i] : sum_ident();  // identities after the range keep the order
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
       const Sum up = shfl_up_sum(incl, o);
       if ((int)lane >= o) incl = combine(up, incl);
     }
-    if (lane == 31) s_w[wi] = incl;
-    Sum ex = shfl_up_sum(incl, 1);
-    if (lane == 0) ex = sum_ident();
-    __syncthreads();
-    if (wi == 0) {
-      Sum wv = s_w[lane], wincl = wv;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const Sum up = shfl_up_sum(wincl, o);
-        if ((int)lane >= o) wincl = combine(up, wincl);
-      }
-      Sum wex = shfl_up_sum(wincl, 1);
-      if (lane == 0) wex = sum_ident();
-      s_w[lane] = wex;
-    }
-    __syncthreads();
-    Sum run = combine(s_carry, combine(s_w[wi], ex));
-    const Sum chunk_end = combine(run, tot);
-#pragma unroll
-    for (int q = 0; q < PER; ++q) {
-      const Sum v = sh[t * PER + q];
-      sh[t * PER + q] = run;  // exclusive prefix, written back coalesced below
-      run = combine(run, v);
-    }
-    __syncthreads();
-    for (u32 q = t; q < 1024 * PER; q += 1024)
-      if (c0 + q < nw) out[c0 + q] = sh[q];
-    if (t == 1023) s_carry = chunk_end;
-    __syncthreads();
+    acc = combine(shfl_sum(incl, 31), acc);
+    j = lo;
+    if (acc.fk != NONE && (!(acc.bits & SB_ONE) || (acc.bits & SB_W))) break;
   }
-  if (segs) {
-    sg = __reduce_add_sync(0xFFFFFFFFu, (u32)sg);
-    if (lane == 0 && sg) atomicAdd((unsigned long long*)seg_cnt, (unsigned long long)sg);
-  }
+  return acc;
 }
 
 // ---------------------------------------------------------------------------------------
 // K7b: lane-sequential check with shared-memory staged clocks.  Persistent warp ranges (state
-// entering each from K7a/K7s); each range is processed in blocks of 32 * KT_IPL items:
+// entering each from enter_state); each listed block of 32 * KT_IPL items is processed as:
 //   load    : the block's (key, ev) words land in shared memory by cp.async
 //             (row pitch KT_IPL+1 words: lane l reading item l*KT_IPL+j is bank-conflict free)
 //   gather  : lane l walks ITS KT_IPL consecutive items; for each item some query can read it issues
@@ -511,8 +469,8 @@ __device__ __forceinline__ void kt_stage(const CheckArgs& a, u64 bb, u32 nb, u32
 // whether any item makes a check -- with one window and nothing carried, an item alone in its granule
 // or an atomic between atomics (its W check is elided, and no read follows it) checks
 // nothing.  Such a block only advances the automaton state: its summary comes from the keys.  Any other
-// block is summarised by a bounded tail walk and listed for K7b.  Phase 2: the CTA scans its blocks'
-// summaries (exclusive prefix within the CTA -> rin) and writes its total (ctot, scanned by K7s).
+// block is summarised by a bounded tail walk (never past the block start) and listed for K7b, which
+// finds the state entering it by walking back over the summaries (enter_state).
 constexpr int KT_SWARPS = 8;
 __device__ __forceinline__ void load_keys16(const u32* __restrict__ keys, u64 bb, u32 nb, u32 l0, u32 (&kr)[KT_IPL]) {
   const u32 cntf = l0 < nb ? min((u32)KT_IPL, nb - l0) : 0u;
@@ -597,15 +555,24 @@ static __device__ __forceinline__ bool sh_block(const CheckArgs& a, const u32* s
   return true;
 }
 
-// key words stream through shared memory: one chunk = KT_SWARPS blocks (+ 4 words on each side for
+// key words stream through shared memory: one chunk = KT_SWARPS warp tiles of KA_TILE items, each
+// KA_BPT blocks (+ 4 words on each side for
 // the neighbours of the first / last item), KB_STAGES chunks in flight per CTA (1-D TMA bulk copies)
-constexpr int KB_STAGES = 2;
-constexpr u32 KT_UNITS_MAX = 1024;  // units per K7a CTA (G / U)
-constexpr int KB_CHUNK = KT_SWARPS * KT_BLK;     // items per chunk
+#ifndef KB_STAGES_
+#define KB_STAGES_ 2
+#endif
+constexpr int KB_STAGES = KB_STAGES_;
+#ifndef KA_UNROLL
+#define KA_UNROLL 1
+#endif
+constexpr int KA_UNR = KA_UNROLL;
+constexpr int KA_TILE = 512;                     // items per K7a warp per chunk (independent of the block size:
+constexpr int KA_BPT = KA_TILE / KT_BLK;         //  K7b's blocks are shorter, K7a's tiles stay long)
+static_assert(KA_TILE % KT_BLK == 0 && KT_BLK % 128 == 0, "K7a tiles hold whole blocks of whole 128-item rounds");
+constexpr int KB_CHUNK = KT_SWARPS * KA_TILE;    // items per chunk
 constexpr int KB_ROW = KB_CHUNK + 8;             // words per stage
 __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum* __restrict__ sums,
-                                                            u32* __restrict__ bflag,
-                                                            u32* __restrict__ n_nontriv) {
+                                                            u32* __restrict__ wl, u32* __restrict__ wl_cnt) {
   __shared__ __align__(128) u32 s_keys[KB_STAGES][KB_ROW];
   __shared__ u64 s_bar[KB_STAGES];
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -635,19 +602,20 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum*
   if (threadIdx.x == 0)
     for (int q = 0; q < KB_STAGES; ++q)
       if ((u32)q < n_chunks) issue(q, q);
-  u32 nontriv = 0;
   for (u32 c = 0; c < n_chunks; ++c) {
     const int st = (int)(c % KB_STAGES);
     mbar_wait(&s_bar[st], (c / KB_STAGES) & 1u);
     const u64 c0 = i0 + (u64)c * KB_CHUNK;
     const u32* sk = &s_keys[st][4];  // sk[j] = key word of item c0 + j (sk[-1]: the item before)
-    const u32 blk = b0 + c * KT_SWARPS + wi;
+#pragma unroll (KA_UNR)
+    for (int sb = 0; sb < KA_BPT; ++sb) {  // the warp's tile: KA_BPT consecutive blocks
+    const u32 blk = b0 + (c * KT_SWARPS + wi) * KA_BPT + sb;
     const u64 bb = (u64)blk * KT_BLK;
     const u32 nb = (blk < b1 && bb < n) ? (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK) : 0u;
     Sum bs = sum_ident();
     if (nb) {
-      const u32 off = wi * KT_BLK;  // the block's first item in the chunk
-      // 4 rounds of 128 items; in round q lane l holds items 128 q + 4 l .. + 3 (one conflict-free
+      const u32 off = (wi * KA_BPT + sb) * KT_BLK;  // the block's first item in the chunk
+      // KT_BLK / 128 rounds of 128 items; in round q lane l holds items 128 q + 4 l .. + 3 (one conflict-free
       // 16-B shared-memory read); neighbours across lanes / rounds by shuffles and broadcast reads
       const u32 lkw = sk[off + nb - 1];                           // the block's last item
       const u32 fkw = sk[off];
@@ -701,14 +669,15 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum*
         bs.lw = mlw;
         bs.fi = NONE;
         bs.bits = (bs.fk == bs.lk ? SB_ONE : 0u) | (mlw ? SB_W : 0u);
+        if (lane == 0) sums[blk] = bs;
+      } else {  // summarised by a bounded tail walk (its key and event words are in L2), listed for K7b
+        bs = tail_sum_nl(a.k, bb, bb + nb);
         if (lane == 0) {
           sums[blk] = bs;
-          bflag[blk] = 0;
+          wl[atomicAdd(wl_cnt, 1u)] = blk;
         }
-      } else {  // summarised with its unit (k_blk_units), checked by K7b
-        if (lane == 0) bflag[blk] = 1;
-        ++nontriv;
       }
+    }
     }
     (void)c0;
     __syncthreads();  // every warp is done with stage st: refill it
@@ -717,84 +686,6 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum*
       issue(c + KB_STAGES, st);
     }
   }
-  if (lane == 0 && nontriv) atomicAdd(n_nontriv, nontriv);
-}
-
-// ---------------------------------------------------------------------- K7a2: units and CTA scans
-// The blocks with checks are processed by K7b in UNITS of U consecutive blocks (a power of two chosen
-// from the number of such blocks: about two units per K7b warp on dense traces, single blocks on
-// sparse ones), one warp per unit carrying the automaton state from block to block.  Per unit with a
-// check: one bounded tail walk gives the unit's summary (placed at its last block, identity at the
-// others) and the unit is listed.  Then each CTA scans its blocks' summaries (rin) and writes its total.
-__global__ void __launch_bounds__(KT_SWARPS * 32) k_blk_units(CheckArgs a, Sum* __restrict__ sums,
-                                                              Sum* __restrict__ rin, Sum* __restrict__ ctot,
-                                                              u32* __restrict__ wl, u32* __restrict__ wl_cnt,
-                                                              const u32* __restrict__ bflag,
-                                                              const u32* __restrict__ n_nontriv, u32 nw_b,
-                                                              u32* __restrict__ unit_out) {
-  __shared__ Sum s_w[KT_SWARPS];
-  __shared__ Sum s_carry;
-  const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const u64 n = *a.n_dev;
-  const K7Part P = k7_part(n);
-  const u32 nblk = P.nblk, G = P.G;
-  const u32 b0 = blockIdx.x * G, b1 = min(nblk, b0 + G);
-  // U: the largest power of two with at least two units per K7b warp (load balance), at most G (a power
-  // of two); 1 on sparse traces
-  const u32 nt = *n_nontriv;
-  u32 U = 1;
-  while (U * 2 <= 64u && U * 2 <= G && (u64)U * 2 * 2 * nw_b <= nt) U <<= 1;  // U | G (G: a multiple of 64)
-  while (G / U > KT_UNITS_MAX) U <<= 1;
-  if (blockIdx.x == 0 && threadIdx.x == 0) *unit_out = U;
-  if (threadIdx.x == 0) s_carry = sum_ident();
-  // ---- units with a check: the CTA's threads scan the unit flags together into a shared list, then the
-  // warps take the listed units round-robin, one tail walk each
-  __shared__ u32 s_units[KT_UNITS_MAX];
-  __shared__ u32 s_nu;
-  if (threadIdx.x == 0) s_nu = 0;
-  __syncthreads();
-  const u32 u_lo = b0 / U, u_hi = (b1 + U - 1) / U;  // G / U <= KT_UNITS_MAX
-  for (u32 u = u_lo + threadIdx.x; u < u_hi; u += KT_SWARPS * 32) {
-    bool any = false;
-    for (u32 q = u * U; q < min(b1, u * U + U); ++q) any |= bflag[q] != 0u;
-    if (any) s_units[atomicAdd(&s_nu, 1u)] = u;
-  }
-  __syncthreads();
-  for (u32 i = wi; i < s_nu; i += KT_SWARPS) {
-    const u32 u = s_units[i];
-    const u32 ub0 = u * U, ub1 = min(b1, ub0 + U);
-    const u64 beg = (u64)ub0 * KT_BLK, end = min(n, (u64)ub1 * KT_BLK);
-    const Sum bs = tail_sum_nl(a.k, beg, end);
-    for (u32 q = ub0 + lane; q < ub1; q += 32) sums[q] = q + 1 == ub1 ? bs : sum_ident();
-    if (lane == 0) wl[atomicAdd(wl_cnt, 1u)] = u;
-  }
-  __syncthreads();
-  // ---- exclusive prefix of the CTA's block summaries, 256 at a time
-  for (u32 c0 = b0; c0 < b1; c0 += KT_SWARPS * 32) {
-    const u32 i = c0 + threadIdx.x;
-    const Sum v = i < b1 ? sums[i] : sum_ident();
-    Sum incl = v;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const Sum up = shfl_up_sum(incl, o);
-      if ((int)lane >= o) incl = combine(up, incl);
-    }
-    Sum ex = shfl_up_sum(incl, 1);
-    if (lane == 0) ex = sum_ident();
-    if (lane == 31) s_w[wi] = incl;
-    __syncthreads();
-    Sum wpre = s_carry;
-    for (u32 q = 0; q < wi; ++q) wpre = combine(wpre, s_w[q]);
-    if (i < b1) rin[i] = combine(wpre, ex);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      Sum t = s_carry;
-      for (int q = 0; q < KT_SWARPS; ++q) t = combine(t, s_w[q]);
-      s_carry = t;
-    }
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) ctot[blockIdx.x] = s_carry;
 }
 
 // ---------------------------------------------------------------------- K7b: the listed blocks
@@ -820,9 +711,7 @@ __device__ __forceinline__ Carry carry_of(const uint4& e0, const uint2& e1) {
 template <bool SH>
 __global__ void __launch_bounds__(KtCfg<SH>::WARPS * 32, 1) k_check_tile(CheckArgs a, const u32* __restrict__ wl,
                                                                          const u32* __restrict__ wl_cnt,
-                                                                         const Sum* __restrict__ rin,
-                                                                         const Sum* __restrict__ cpre, u32 nblk,
-                                                                         const u32* __restrict__ unit_p) {
+                                                                         const Sum* __restrict__ sums, u32 nblk) {
   constexpr int NWARP = KtCfg<SH>::WARPS;
   extern __shared__ __align__(16) unsigned char kt_smem[];
   const int wi = threadIdx.x >> 5;
@@ -839,15 +728,12 @@ __global__ void __launch_bounds__(KtCfg<SH>::WARPS * 32, 1) k_check_tile(CheckAr
   const u32 R0 = a.R0;
   const bool shadow = a.sh_in != nullptr;
   const u32 n_tasks = *wl_cnt;
-  const u32 U = *unit_p;  // blocks per unit (K7a)
   u32 segs = 0;
   const u32 l0 = lane * KT_IPL;
   for (u32 task = w; task < n_tasks; task += nw) {
-    // a unit: U consecutive blocks, processed in order with the automaton state carried through
-    const u32 u = wl[task];
-    const u32 blk0 = u * U, blk1 = min(nblk, blk0 + U);
-    // state entering the unit: its K7a CTA's prefix (K7s), then the prefix within that CTA
-    Sum carry = combine(cpre[blk0 / k7_part(n).G], rin[blk0]);
+    // a listed block (the loop below also serves runs of blocks carrying the state through)
+    const u32 blk0 = wl[task], blk1 = min(nblk, blk0 + 1);
+    Sum carry = enter_state(sums, blk0);
     u32 pkx = blk0 > 0 ? __ldg(a.keys + (u64)blk0 * KT_BLK - 1) : NONE;  // the item before the block
     for (u32 bi = blk0; bi < blk1; ++bi) {
     const u64 bb = (u64)bi * KT_BLK;
@@ -1175,12 +1061,11 @@ static int k7_grid(int dev) {
   return grid[dev];
 }
 
-// status scratch: [K7Ctx][Sum sums[nblk]][Sum rin[nblk]][Sum ctot[nct]][Sum cpre[nct]][u32 wl[nblk]][u32 wl_cnt]
-// [u32 csegs[nct]]
+// status scratch: [K7Ctx][Sum sums[nblk]][u32 wl[nblk]][u32 wl_cnt]
 size_t check_status_bytes(u64 n) {
-  const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1, nct = K7A_CTAS + 2;
-  return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (2 * nblk + 2 * nct + 4) * sizeof(Sum) +
-         (2 * nblk + nct + 64) * sizeof(u32) + 1024;
+  const u64 nblk = (n + KT_BLK - 1) / KT_BLK + 1;
+  return 256 + ((sizeof(K7Ctx) + 255) & ~(size_t)255) + (nblk + 4) * sizeof(Sum) + (nblk + 64) * sizeof(u32) +
+         1024;
 }
 
 void launch_check(const CheckLaunch& L, cudaStream_t st) {
@@ -1189,21 +1074,13 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   cudaGetDevice(&dev);
   const bool SH = L.sh_in || L.sh_out;
   const int grid = SH ? k7_grid<true>(dev) : k7_grid<false>(dev);
-  const int k7b_warps = SH ? KtCfg<true>::WARPS : KtCfg<false>::WARPS;
   const u64 nblk = (L.n_max + KT_BLK - 1) / KT_BLK;  // upper bound (array sizes); the kernels partition the
-  const u32 nct = K7A_CTAS;                           // device-side item count (k7_part)
+                                                      // device-side item count (k7_part)
   char* base = (char*)L.status;
   K7Ctx* kdev = reinterpret_cast<K7Ctx*>(base);
   Sum* sums = reinterpret_cast<Sum*>(base + ((sizeof(K7Ctx) + 255) & ~(size_t)255));
-  Sum* rin = sums + nblk + 1;
-  Sum* ctot = rin + nblk + 1;
-  Sum* cpre = ctot + nct + 1;
-  u32* wl = reinterpret_cast<u32*>(cpre + nct + 1);
+  u32* wl = reinterpret_cast<u32*>(sums + nblk + 1);
   u32* wl_cnt = wl + nblk + 1;
-  u32* csegs = wl_cnt + 1;
-  u32* bflag = csegs + nct + 1;
-  u32* n_nontriv = bflag + nblk + 1;
-  u32* unit_p = n_nontriv + 1;
   K7Ctx k{};
   k.c = L.c;
   k.keys = L.keys;
@@ -1222,7 +1099,6 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   k.n_dev = L.n_dev;
   cudaMemcpyAsync(kdev, &k, sizeof(K7Ctx), cudaMemcpyHostToDevice, st);
   cudaMemsetAsync(wl_cnt, 0, sizeof(u32), st);
-  cudaMemsetAsync(n_nontriv, 0, sizeof(u32), st);
   CheckArgs a;
   a.k = kdev;
   a.c = L.c;
@@ -1232,24 +1108,20 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   a.R0 = L.R0;
   a.sh_in = L.sh_in;
   a.sh_out = L.sh_out;
-  a.rin = nullptr;
   a.no_sv = L.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   a.values = L.values;
-  k_blk_sum<<<nct, KT_SWARPS * 32, 0, st>>>(a, sums, bflag, n_nontriv);
-  k_blk_units<<<nct, KT_SWARPS * 32, 0, st>>>(a, sums, rin, ctot, wl, wl_cnt, bflag, n_nontriv,
-                                              (u32)grid * k7b_warps, unit_p);
-  k_range_scan<<<1, 1024, 0, st>>>(ctot, L.n_dev, cpre, nullptr, nullptr);  // segments: stats pass
+  k_blk_sum<<<K7A_CTAS, KT_SWARPS * 32, 0, st>>>(a, sums, wl, wl_cnt);
   if (SH)
     k_check_tile<true><<<grid, KtCfg<true>::WARPS * 32, (size_t)KtCfg<true>::WARPS * KtCfg<true>::WARP_BYTES, st>>>(
-        a, wl, wl_cnt, rin, cpre, (u32)nblk, unit_p);
+        a, wl, wl_cnt, sums, (u32)nblk);
   else
     k_check_tile<false><<<grid, KtCfg<false>::WARPS * 32, (size_t)KtCfg<false>::WARPS * KtCfg<false>::WARP_BYTES,
-                          st>>>(a, wl, wl_cnt, rin, cpre, (u32)nblk, unit_p);
-  g_launches += 4;
+                          st>>>(a, wl, wl_cnt, sums, (u32)nblk);
+  g_launches += 2;
 }
 
 void preload_check() {
-  preload(k_blk_sum, k_blk_units, k_check_tile<false>, k_check_tile<true>, k_count_gathers, k_range_scan,
+  preload(k_blk_sum, k_check_tile<false>, k_check_tile<true>, k_count_gathers,
           k_shadow_commit);
 }
 

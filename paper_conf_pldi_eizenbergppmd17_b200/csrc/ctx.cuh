@@ -35,7 +35,7 @@ struct bc_ctx {
   bc_stats stats{};
   Arena arena;  // scratch buffers, reused across bc_detect calls
   std::string err;
-  cudaEvent_t ev[16] = {};
+  cudaEvent_t ev[18] = {};
   u64* hcnt = nullptr;  // pinned host copy of the device counter array (one D2H copy per host sync)
   // block-sharded multi-GPU: this rank holds the records of blocks b % world == rank
   Comm* comm = nullptr;       // NCCL or in-process transport, null: single GPU / replicated trace

@@ -139,7 +139,7 @@ void launch_barriers(const Geo& g, const u32* bar_cnt, const u32* bar_base, cons
                      u32* blockR, u32* err, cudaStream_t st, bool allow_pending = false);
 void launch_snap_blab(uint4* snap, u64 n, u32 wpb, u32 n_warps, u64 n_bars, const u32* bar_base, const u32* blockR,
                       cudaStream_t st);
-void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
+void launch_expand(const bc_record* recs, const uint4* hdr16, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
                    const u64* cum, u64 R0, u64 R1, const u32* gidx, u64 G0, u32* keys, u32* evs, u32* err,
                    cudaStream_t st);
 void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStream_t st);

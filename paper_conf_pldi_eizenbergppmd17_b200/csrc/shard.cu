@@ -423,7 +423,7 @@ bc_status detect_sharded(bc_ctx* c, Scratch& S) {
     const u64 p0 = pst[k], p1 = pst[k + 1], b = pbd[k];
     ++sx.windows;
     // ---- K4 over the local records of the window, then route each item to its granule's owner
-    launch_expand(recs, gl, page_bits, page_rank, shared_base, cum, p0, p1, gidx, R0, ikeys, ievs, err, st);
+    launch_expand(recs, hdr16, gl, page_bits, page_rank, shared_base, cum, p0, p1, gidx, R0, ikeys, ievs, err, st);
     if (b) { k_dest<<<nb(b), 256, 0, st>>>(ikeys, b, shared_base, (u32)W, (u32)me, dkeys, didx); ++g_launches; }
     const bool a4 = radix_sort_pairs(dkeys, didx, dk2, di2, b, 0, std::max(1, bits_for((u64)W - 1)), rtmp, st,
                                      nullptr, n_send_dev, true);

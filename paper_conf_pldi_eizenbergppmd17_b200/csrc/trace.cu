@@ -420,25 +420,23 @@ __global__ void __launch_bounds__(256) k_barriers(Geo g, const u32* __restrict__
 // KEY_DROP, which the first radix pass removes.  Also validates per-lane alignment / shared
 // bounds for every op <= AR_GLB.
 //
-// Data movement (the trace is read once, at HBM rate): persistent CTAs stream chunks of EX_REC
-// consecutive records (EX_REC x 272 B, contiguous) into shared memory with 1-D TMA bulk copies
-// (cp.async.bulk ... mbarrier::complete_tx), EX_STAGES chunks in flight per CTA; the 8 warps then
-// expand the staged records (warp w: records w, w+8, ...; header = a broadcast shared-memory read,
-// lane l's address = addr[l]) while the next chunk lands.  64-record chunks, 2 stages: fewer CTA
-// barriers per record (the warps' work per record differs: control vs memory records) beat deeper
-// staging (C4: 32 x 4 -> 64 x 2 took k_expand from 5.1 to 4.4 ms; 128 or 256 records are slower).
-#ifndef EX_REC_
-#define EX_REC_ 64
-#endif
-#ifndef EX_STAGES_
-#define EX_STAGES_ 2
-#endif
-constexpr int EX_REC = EX_REC_;
-constexpr int EX_STAGES = EX_STAGES_;
+// Data movement (each address-carrying record is read once, at HBM rate): every warp owns chunks of
+// EX_RPW consecutive records (warp-strided over the window) and stages only the 256-B address rows of
+// the records that carry addresses (LD / ST / ATOM / ACQ / REL / AR; the headers come from k_header's
+// compact copy hdr16), so the rows of control records (IF / ELSE / FI / BAR / FENCE: half of C4's
+// records) never leave HBM.  Rows land in the warp's own shared-memory buffer by cp.async (16 B per
+// lane: one warp instruction moves two rows), the next chunk in flight while this one is expanded
+// (two stages); no CTA-wide barrier, so a warp never waits for another warp's records.  (Round 1-2:
+// 64-record chunks by one TMA bulk copy per CTA and stage, 2 stages, whole records: 3.8 ms on C4,
+// barrier-stall bound; a bulk copy per run of address-carrying records was slower still: 5.0 ms.)
 constexpr int EX_THREADS = 256;
-constexpr int EX_RPW = EX_REC / (EX_THREADS / 32);  // records per warp per chunk
+constexpr int EX_WARPS = EX_THREADS / 32;
+constexpr int EX_RPW = 8;                          // records per warp chunk
+constexpr size_t EX_ROW = 32 * sizeof(u64);        // 256 B: one record's address row
+constexpr size_t EX_SMEM = (size_t)EX_WARPS * 2 * EX_RPW * EX_ROW;  // 32 KB per CTA
 
-__global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restrict__ recs, Geo g,
+__global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restrict__ recs,
+                                                       const uint4* __restrict__ hdr16, Geo g,
                                                        const u32* __restrict__ page_bits,
                                                        const u32* __restrict__ page_rank, u32 shared_base,
                                                        const u64* __restrict__ cum, u64 R0, u64 R1,
@@ -446,66 +444,68 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
                                                        u32* __restrict__ okeys, u32* __restrict__ oevs,
                                                        u32* __restrict__ err) {
   extern __shared__ __align__(128) unsigned char ex_smem[];
-  bc_record* buf = reinterpret_cast<bc_record*>(ex_smem);                    // [EX_STAGES][EX_REC]
-  u64* bar = reinterpret_cast<u64*>(ex_smem + sizeof(bc_record) * EX_REC * EX_STAGES);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  u64* const rows = reinterpret_cast<u64*>(ex_smem + (size_t)wid * 2 * EX_RPW * EX_ROW);  // [2][EX_RPW][32]
   const u64 n = R1 - R0;  // records of the window
-  const u64 n_chunks = (n + EX_REC - 1) / EX_REC;
+  const u64 n_chunks = (n + EX_RPW - 1) / EX_RPW;
+  const u64 nw = (u64)gridDim.x * EX_WARPS;
   const u64 cum0 = __ldg(cum + R0);
-  auto issue = [&](u64 chunk, int st) {
-    const u64 r0 = chunk * EX_REC;
-    const u32 cnt = (u32)(n - r0 < (u64)EX_REC ? n - r0 : (u64)EX_REC);
-    mbar_expect_tx(&bar[st], cnt * (u32)sizeof(bc_record));
-    bulk_g2s(&buf[st * EX_REC], recs + R0 + r0, cnt * (u32)sizeof(bc_record), &bar[st]);
-  };
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < EX_STAGES; ++s) mbar_init(&bar[s], 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  if (threadIdx.x == 0)
-    for (int s = 0; s < EX_STAGES; ++s) {
-      const u64 c = blockIdx.x + (u64)s * gridDim.x;
-      if (c < n_chunks) issue(c, s);
-    }
   const u32 lt = lanemask_lt();
   bool bad = false, ovf = false, undecl = false;
-  u32 it = 0;
-  for (u64 c = blockIdx.x; c < n_chunks; c += gridDim.x, ++it) {
-    const int st = (int)(it % EX_STAGES);
-    const u32 phase = (it / EX_STAGES) & 1u;
-    const u64 cbase = c * EX_REC;  // window-local record index of the chunk
-    // warp wid expands records wid, wid + 8, ... of the chunk (interleaved: control and memory records
-    // alternate in most programs, so the warps of a CTA finish a chunk at about the same time); their
-    // slot offsets (window weight prefix minus REC_W per record) are independent of the staged bytes:
-    // one load per lane before waiting
-    const u64 rl = cbase + (u64)wid + (u64)(lane & (EX_RPW - 1)) * (EX_THREADS / 32);
-    const u32 uo_l = (lane < EX_RPW && rl < n) ? (u32)(__ldg(cum + R0 + rl) - cum0 - (u64)REC_W * rl) : 0u;
-    // the record's window-local event base ((global record - window start) << 5), one per lane as well
-    const u32 eb_l = (lane < EX_RPW && rl < n) ? (u32)(((gidx ? (u64)__ldg(gidx + R0 + rl) : R0 + rl) - G0) << 5) : 0u;
-    mbar_wait(&bar[st], phase);
-    // lane j < EX_RPW classifies record wid + 8 j from its header: the warp then walks only the records
-    // that carry addresses (LD / ST / ATOM, and ACQ / REL / AR for the alignment check); control records
-    // (IF / ELSE / FI / BAR / FENCE: about half of a divergent program's records) cost one ballot
-    u32 mem = 0;
-    {
-      const u32 jr = (u32)wid + (u32)(lane & (EX_RPW - 1)) * (EX_THREADS / 32);
-      const bool have = lane < EX_RPW && cbase + jr < n;
-      const u32 hz = have ? reinterpret_cast<const uint4*>(&buf[st * EX_REC + jr])->z : 0xFFu;
-      mem = __ballot_sync(0xFFFFFFFFu, have && (hz & 0xFFu) <= BC_OP_AR_GLB);
+  // per chunk, lane j < EX_RPW holds record j's header, slot offset and event base
+  struct Ch {
+    uint4 h;
+    u32 uo, eb, sel;
+  };
+  // load a chunk's headers / offsets and start copying the address rows of its selected records
+  auto issue = [&](u64 chunk, int stg) -> Ch {
+    Ch c;
+    const u64 r0 = chunk * EX_RPW;
+    const u64 rl = r0 + (u64)(lane & (EX_RPW - 1));
+    const bool have = lane < EX_RPW && rl < n;
+    c.h = have ? __ldg(hdr16 + R0 + rl) : make_uint4(0, 0, 0xFFu, 0);
+    c.uo = have ? (u32)(__ldg(cum + R0 + rl) - cum0 - (u64)REC_W * rl) : 0u;
+    c.eb = have ? (u32)(((gidx ? (u64)__ldg(gidx + R0 + rl) : R0 + rl) - G0) << 5) : 0u;
+    c.sel = __ballot_sync(0xFFFFFFFFu, have && (c.h.z & 0xFFu) <= BC_OP_AR_GLB);
+    // two rows per instruction: lanes 0-15 the k-th selected record, lanes 16-31 the (k+1)-th
+    u32 m = c.sel;
+    while (m) {
+      const int ja = __ffs(m) - 1;
+      m &= m - 1;
+      const int jb = m ? __ffs(m) - 1 : -1;
+      if (m) m &= m - 1;
+      const int j = lane < 16 ? ja : jb;
+      if (j >= 0) {
+        const int q = lane & 15;  // 16-B piece of the row
+        const char* src = reinterpret_cast<const char*>(&recs[R0 + r0 + j].addr[0]) + q * 16;
+        char* dst = reinterpret_cast<char*>(rows + ((size_t)stg * EX_RPW + j) * 32) + q * 16;
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+      }
     }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    return c;
+  };
+  u64 chunk = (u64)blockIdx.x * EX_WARPS + wid;
+  int stg = 0;
+  Ch cur = chunk < n_chunks ? issue(chunk, 0) : Ch{};
+  for (; chunk < n_chunks; chunk += nw, stg ^= 1) {
+    Ch nxt{};
+    if (chunk + nw < n_chunks) nxt = issue(chunk + nw, stg ^ 1);
+    else asm volatile("cp.async.commit_group;" ::: "memory");  // (keeps the group count: wait 1 = current)
+    asm volatile("cp.async.wait_group 1;" ::: "memory");
+    __syncwarp();
+    const u64* const crow = rows + (size_t)stg * EX_RPW * 32;
+    u32 mem = cur.sel;
     while (mem) {
       const int j = __ffs(mem) - 1;
       mem &= mem - 1;
-      const u32 jr = (u32)wid + (u32)j * (EX_THREADS / 32);  // record within the chunk
-      const u32 uoj = __shfl_sync(0xFFFFFFFFu, uo_l, j);
-      const u32 evb = __shfl_sync(0xFFFFFFFFu, eb_l, j);
-      const bc_record* sr = &buf[st * EX_REC + jr];
-      const uint4 hv = *reinterpret_cast<const uint4*>(sr);
-      const u32 hwarp = hv.x, hmask = hv.y, op = hv.z & 0xFFu, space = (hv.z >> 8) & 0xFFu,
-                sl = (hv.z >> 16) & 0xFFu, fl = (hv.z >> 24) & 0xFFu;
+      const u32 uoj = __shfl_sync(0xFFFFFFFFu, cur.uo, j);
+      const u32 evb = __shfl_sync(0xFFFFFFFFu, cur.eb, j);
+      const u32 hwarp = __shfl_sync(0xFFFFFFFFu, cur.h.x, j), hmask = __shfl_sync(0xFFFFFFFFu, cur.h.y, j);
+      const u32 hz = __shfl_sync(0xFFFFFFFFu, cur.h.z, j);
+      const u32 op = hz & 0xFFu, space = (hz >> 8) & 0xFFu, sl = (hz >> 16) & 0xFFu, fl = (hz >> 24) & 0xFFu;
       if (!(((hmask >> lane) & 1u) && sl <= 4 && space <= 1 && hwarp < g.n_warps)) continue;
-      const u64 a = sr->addr[lane];
+      const u64 a = crow[j * 32 + lane];
       const u64 size = 1ull << sl;
       if (a & (size - 1)) bad = true;  // natural alignment
       if (space == BC_SPACE_SHARED && a + size > g.smem) bad = true;
@@ -546,12 +546,10 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
         oevs[o + k] = ev;
       }
     }
-    __syncthreads();  // every warp is done with stage st: refill it
-    if (threadIdx.x == 0) {
-      const u64 cn = c + (u64)EX_STAGES * gridDim.x;
-      if (cn < n_chunks) issue(cn, st);
-    }
+    __syncwarp();  // every lane is done with this stage: the next issue may refill it
+    cur = nxt;
   }
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
   if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
   if (__any_sync(0xFFFFFFFFu, ovf) && lane == 0) set_err(err, ERR_OVERFLOW);
   if (__any_sync(0xFFFFFFFFu, undecl) && lane == 0) set_err(err, ERR_UNDECLARED);
@@ -772,12 +770,11 @@ void launch_node_base(const u32* if_excl, u32 n_warps, u32* node_base, cudaStrea
   k_node_base<<<(n_warps + 255) / 256, 256, 0, st>>>(if_excl, n_warps, node_base); ++g_launches;
 }
 
-void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, const u32* page_rank, u32 shared_base,
-                   const u64* cum, u64 R0, u64 R1, const u32* gidx, u64 G0, u32* keys, u32* evs, u32* err,
-                   cudaStream_t st) {
-  const u64 chunks = (R1 - R0 + EX_REC - 1) / EX_REC;
+void launch_expand(const bc_record* recs, const uint4* hdr16, const Geo& g, const u32* page_bits, const u32* page_rank,
+                   u32 shared_base, const u64* cum, u64 R0, u64 R1, const u32* gidx, u64 G0, u32* keys, u32* evs,
+                   u32* err, cudaStream_t st) {
+  const u64 chunks = (R1 - R0 + EX_RPW - 1) / EX_RPW;
   if (!chunks) return;
-  const size_t smem = sizeof(bc_record) * EX_REC * EX_STAGES + 8 * EX_STAGES;
   static int grid[64] = {};  // per device: the shared-memory opt-in and the occupancy-derived grid
   int dev = 0;
   cudaGetDevice(&dev);
@@ -785,13 +782,13 @@ void launch_expand(const bc_record* recs, const Geo& g, const u32* page_bits, co
   if (!grid[dev]) {
     int sms = 148, per = 1;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_expand, EX_THREADS, smem);
+    cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)EX_SMEM);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_expand, EX_THREADS, EX_SMEM);
     grid[dev] = sms * (per > 0 ? per : 1);
   }
-  const unsigned gr = (unsigned)std::min<u64>(chunks, (u64)grid[dev]);
-  k_expand<<<gr, EX_THREADS, smem, st>>>(recs, g, page_bits, page_rank, shared_base, cum, R0, R1, gidx, G0, keys, evs,
-                                         err);
+  const unsigned gr = (unsigned)std::min<u64>((chunks + EX_WARPS - 1) / EX_WARPS, (u64)grid[dev]);
+  k_expand<<<gr, EX_THREADS, EX_SMEM, st>>>(recs, hdr16, g, page_bits, page_rank, shared_base, cum, R0, R1, gidx, G0,
+                                            keys, evs, err);
   ++g_launches;
 }
 
