@@ -98,6 +98,7 @@ bc_status check_window(bc_ctx* c, CheckLaunch& L, u64 b, u64* cnt, u64& n_r, u64
     c->rbuf = nb2;
     c->rbuf_cap = cap2;
   }
+  if (herr & ERR_PAGES) return BC_RETRY_FULL_PAGES;  // the sampled page set missed a written page
   if (herr & ERR_INFEASIBLE) return fail(c, BC_ERR_INFEASIBLE_TRACE, "infeasible trace");
   if (herr & ERR_OVERFLOW) return fail(c, BC_ERR_OVERFLOW, "index overflow / sync lookup step cap");
   if (herr & ERR_UNDECLARED) return fail(c, BC_ERR_INVALID_ARG, "global access outside bc_config.global_ranges");
@@ -380,7 +381,9 @@ bc_status bc_load_trace(bc_ctx* c, const bc_record* recs, uint64_t n, int on_dev
   return BC_OK;
 }
 
-static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
+// full_pages: k_header marks the page of every write address instead of a sample (the re-run after
+// K4 found a write outside the sampled set, BC_RETRY_FULL_PAGES)
+static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw, bool full_pages = false) {
   cudaStream_t st = c->stream;
   Geo g = c->g;
   if (c->values) g.flags |= GEO_F_VALUES;
@@ -420,7 +423,7 @@ static bc_status detect_impl(bc_ctx* c, Scratch& S, const StreamWin* sw) {
   u32* word_list = S.alloc<u32>(nwords);
   u32* wl2 = S.alloc<u32>(nwords);
   launch_header(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt, rec_w, hdr16, rec_cnt, err, st,
-                sw == nullptr);
+                sw ? 0 : (full_pages ? 1 : 2));
   if (sw) launch_mark_ranges(c->granges, c->cfg.n_global_ranges, page_bits, word_list, cnt, err, st);
   u32* words = word_list;
   u32* wl_prefix = wl2;
@@ -800,6 +803,11 @@ bc_status bc_detect(bc_ctx* c, bc_stats* out) {
     Scratch S(c->stream, &c->arena);
     try {
       s = c->sharded ? detect_sharded(c, S) : detect_impl(c, S, nullptr);
+      if (s == BC_RETRY_FULL_PAGES) {  // (internal) the sampled page set was incomplete: again, exactly
+        c->err.clear();
+        Scratch S2(c->stream, &c->arena);  // the same arena buffers, from the first again
+        s = detect_impl(c, S2, nullptr, true);
+      }
     } catch (const std::bad_alloc&) {
       s = fail(c, BC_ERR_OOM, "scratch allocation");
     }

@@ -563,7 +563,7 @@ static __device__ __forceinline__ bool sh_block(const CheckArgs& a, const u32* s
 #endif
 constexpr int KB_STAGES = KB_STAGES_;
 #ifndef KA_UNROLL
-#define KA_UNROLL 1
+#define KA_UNROLL 2  // the tile's blocks interleaved (A/B on C4: 159 -> 150 us)
 #endif
 constexpr int KA_UNR = KA_UNROLL;
 constexpr int KA_TILE = 512;                     // items per K7a warp per chunk (independent of the block size:
@@ -571,9 +571,11 @@ constexpr int KA_BPT = KA_TILE / KT_BLK;         //  K7b's blocks are shorter, K
 static_assert(KA_TILE % KT_BLK == 0 && KT_BLK % 128 == 0, "K7a tiles hold whole blocks of whole 128-item rounds");
 constexpr int KB_CHUNK = KT_SWARPS * KA_TILE;    // items per chunk
 constexpr int KB_ROW = KB_CHUNK + 8;             // words per stage
+constexpr size_t KB_SMEM = (size_t)KB_STAGES * KB_ROW * sizeof(u32);
 __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum* __restrict__ sums,
                                                             u32* __restrict__ wl, u32* __restrict__ wl_cnt) {
-  __shared__ __align__(128) u32 s_keys[KB_STAGES][KB_ROW];
+  extern __shared__ __align__(128) u32 kb_smem[];  // [KB_STAGES][KB_ROW] key words
+  u32 (*const s_keys)[KB_ROW] = reinterpret_cast<u32 (*)[KB_ROW]>(kb_smem);
   __shared__ u64 s_bar[KB_STAGES];
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const u64 n = *a.n_dev;
@@ -1110,7 +1112,12 @@ void launch_check(const CheckLaunch& L, cudaStream_t st) {
   a.sh_out = L.sh_out;
   a.no_sv = L.c.g.flags & BC_F_NO_SAME_VALUE_FILTER;
   a.values = L.values;
-  k_blk_sum<<<K7A_CTAS, KT_SWARPS * 32, 0, st>>>(a, sums, wl, wl_cnt);
+  static bool kb_attr[64] = {};
+  if (dev >= 0 && dev < 64 && !kb_attr[dev]) {
+    cudaFuncSetAttribute(k_blk_sum, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)KB_SMEM);
+    kb_attr[dev] = true;
+  }
+  k_blk_sum<<<K7A_CTAS, KT_SWARPS * 32, KB_SMEM, st>>>(a, sums, wl, wl_cnt);
   if (SH)
     k_check_tile<true><<<grid, KtCfg<true>::WARPS * 32, (size_t)KtCfg<true>::WARPS * KtCfg<true>::WARP_BYTES, st>>>(
         a, wl, wl_cnt, sums, (u32)nblk);

@@ -29,6 +29,7 @@ constexpr int WARP = 32;
 constexpr u32 ERR_INFEASIBLE = 1u;
 constexpr u32 ERR_OVERFLOW = 2u;
 constexpr u32 ERR_UNDECLARED = 8u;  // streaming: a global access outside the declared allocations
+constexpr u32 ERR_PAGES = 16u;      // K4 met a global write whose page the sampled page set lacks (re-run)
 
 // item op codes (2 low bits of an item's key word)
 constexpr u32 IOP_LD = 0, IOP_ST = 1, IOP_ST_SV = 2, IOP_ATOM = 3;

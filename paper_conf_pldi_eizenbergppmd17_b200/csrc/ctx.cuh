@@ -74,6 +74,9 @@ struct bc_ctx {
 };
 
 // one window of a streaming session: records [R0, n) are new; earlier ones only feed the clocks
+// internal status of detect_impl (never returned by the C ABI): re-run with every write page marked
+constexpr bc_status BC_RETRY_FULL_PAGES = (bc_status)-100;
+
 struct StreamWin {
   u64 R0 = 0;
   bool final = false;

@@ -122,7 +122,7 @@ constexpr u32 REC_W = 8;
 constexpr u64 WIN_MAX = (1ull << 30) - 1024;
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
                    u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_w, uint4* hdr16,
-                   u32* rec_cnt, u32* err, cudaStream_t st, bool mark_pages = true);
+                   u32* rec_cnt, u32* err, cudaStream_t st, int mark_pages = 1);  // 0 none, 1 every write address, 2 sampled
 void launch_mark_ranges(const u64* ranges, u32 n_ranges, u32* page_bits, u32* word_list, u64* cnt, u32* err,
                         cudaStream_t st);
 void launch_window_starts(const u64* cum, u64 n, u64 we, u32 nwin, u64* starts, u64* bounds, cudaStream_t st);

@@ -112,9 +112,30 @@ __global__ void __launch_bounds__(256) k_header(const bc_record* __restrict__ re
       if (s_cnt[threadIdx.x]) atomicAdd((unsigned long long*)&cnt[slot[threadIdx.x]], s_cnt[threadIdx.x]);
     }
   }
-  // page marking: ST / ATOM on global memory
-  u32 wr = __ballot_sync(0xFFFFFFFFu, mark_pages && valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) &&
-                                          h.space == BC_SPACE_GLOBAL);
+  // page marking: ST / ATOM on global memory.  mark_pages == 2 (sampled): only the first and last active
+  // lanes' addresses of each write record -- one or two 8-B loads instead of its 256-B row; K4 checks every
+  // write address against the set and flags a missing page (ERR_PAGES), and the host then re-runs the
+  // detect with every address marked (mark_pages == 1), so the page set K4-K7 use is always complete.
+  const bool wrec = valid && !bad && (h.op == BC_OP_ST || h.op == BC_OP_ATOM) && h.space == BC_SPACE_GLOBAL;
+  if (mark_pages == 2 && wrec) {
+    const int la = __ffs(h.mask) - 1, lb = 31 - __clz(h.mask);
+    const u64 a0 = __ldg(&recs[r].addr[la]), a1 = __ldg(&recs[r].addr[lb]);
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+      const u64 p = (k ? a1 : a0) >> 20;
+      if (p >= (1ull << 28)) {
+        set_err(err, ERR_OVERFLOW);
+      } else {
+        const u32 bit = 1u << (p & 31);
+        u32* wp = &page_bits[p >> 5];
+        if (!(*(volatile u32*)wp & bit) && atomicOr(wp, bit) == 0u) {
+          const u64 at = atomicAdd((unsigned long long*)&cnt[C_PAGE_WORDS], 1ull);
+          word_list[at] = (u32)(p >> 5);
+        }
+      }
+    }
+  }
+  u32 wr = __ballot_sync(0xFFFFFFFFu, mark_pages == 1 && wrec);
   while (wr) {  // HDR_ROWS records' address rows in flight at a time
     int js[HDR_ROWS];
     u64 a[HDR_ROWS];
@@ -451,7 +472,7 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
   const u64 nw = (u64)gridDim.x * EX_WARPS;
   const u64 cum0 = __ldg(cum + R0);
   const u32 lt = lanemask_lt();
-  bool bad = false, ovf = false, undecl = false;
+  bool bad = false, ovf = false, undecl = false, pmiss = false;
   // per chunk, lane j < EX_RPW holds record j's header, slot offset and event base
   struct Ch {
     uint4 h;
@@ -529,6 +550,8 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
                    (u32)((a & 0xFFFFFull) >> g.G);
           else if (g.flags & GEO_F_DECLARED)
             undecl = true;  // streaming: the page set is the declared allocations, nothing may fall outside
+          else if (op != BC_OP_LD)
+            pmiss = true;   // a write outside the (sampled) page set: the set is incomplete
         } else {
           ovf = true;
         }
@@ -553,6 +576,7 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
   if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) set_err(err, ERR_INFEASIBLE);
   if (__any_sync(0xFFFFFFFFu, ovf) && lane == 0) set_err(err, ERR_OVERFLOW);
   if (__any_sync(0xFFFFFFFFu, undecl) && lane == 0) set_err(err, ERR_UNDECLARED);
+  if (__any_sync(0xFFFFFFFFu, pmiss) && lane == 0) set_err(err, ERR_PAGES);
 }
 
 // Window k = the records whose weight prefix cum[r] (exclusive) lies in [k * we, (k + 1) * we):
@@ -654,12 +678,12 @@ __global__ void __launch_bounds__(1024) k_page_rank(u32* __restrict__ words, con
 // --------------------------------------------------------------------- host launchers
 void launch_header(const bc_record* recs, const Geo& g, u32* wkey, u32* wval, u32* if_cnt, u32* bar_cnt,
                    u32* sync_list, u32* page_bits, u32* word_list, u64* cnt, u32* rec_w, uint4* hdr16,
-                   u32* rec_cnt, u32* err, cudaStream_t st, bool mark_pages) {
+                   u32* rec_cnt, u32* err, cudaStream_t st, int mark_pages) {
   u64 warps = (g.n_recs + 31) / 32;
   if (warps == 0) return;
   u64 blocks = (warps + 7) / 8;
   k_header<<<(unsigned)blocks, 256, 0, st>>>(recs, g, wkey, wval, if_cnt, bar_cnt, sync_list, page_bits, word_list, cnt,
-                                             rec_w, hdr16, rec_cnt, err, mark_pages ? 1 : 0); ++g_launches;
+                                             rec_w, hdr16, rec_cnt, err, mark_pages); ++g_launches;
 }
 
 void launch_warp_start(const u32* skeys, u64 n, u32 n_warps, u32* warp_start, cudaStream_t st) {

@@ -574,3 +574,23 @@ def test_c5_full_size_truth():
     assert len(truth) > 0
     assert np.array_equal(np.sort(res.races.view("V32")), np.sort(truth.view("V32")))
     torch.cuda.empty_cache()
+
+
+# ------------------------------------------------------------------ sampled page set (k_header)
+def test_sampled_page_set_miss_reruns_exactly():
+    """k_header marks written pages from each write record's first and last active lanes only; a page
+    written solely by middle lanes is missing from the sample.  K4 sees the write, flags it and the
+    detect re-runs with every write address marked: the races on that page (a write by block 0's middle
+    lanes, read and rewritten by block 1) must all be found, bit-identical to the oracle."""
+    MB = 1 << 20
+    tb = TraceBuilder(grid=(2, 1, 1), block=(32, 1, 1))
+    w0, w1 = tb.warp(0), tb.warp(1)
+    # lanes 0 and 31 write page 0, lanes 1..30 write page 5 (never sampled)
+    tb.st(w0, lambda l: GLOBAL_BASE + (0 if l in (0, 31) else 5 * MB) + 4 * l)
+    tb.ld(w1, lambda l: GLOBAL_BASE + 5 * MB + 4 * l)
+    tb.st(w1, lambda l: GLOBAL_BASE + 5 * MB + 4 * l)
+    recs = tb.records()
+    want, res = assert_parity(recs, tb.geom.as_dict())
+    assert len(want) == 2 * 30  # WR then WW on each of the 30 middle granules
+    # the same with several windows (the miss is found in the first one)
+    assert_parity(recs, tb.geom.as_dict(), window_events=40)
