@@ -36,4 +36,10 @@ d, g2, org = bc.split_warps(recs, tb.geom.as_dict(), 8)
 from test_shard import assert_sharded
 p = ConfigPlan(4, n_blocks=12, log2_nodes=14, nodes_per_thread=2, inj_scale=4)
 assert_sharded(p.records(), p.geometry, 2)
+# the sampled page set misses a page written by middle lanes only: K4 flags it, the detect re-runs
+from bcgen import GLOBAL_BASE, TraceBuilder
+tb = TraceBuilder(grid=(2, 1, 1), block=(32, 1, 1))
+tb.st(tb.warp(0), lambda l: GLOBAL_BASE + (0 if l in (0, 31) else 5 << 20) + 4 * l)
+tb.ld(tb.warp(1), lambda l: GLOBAL_BASE + (5 << 20) + 4 * l)
+same(tb.records(), tb.geom.as_dict())
 print("sanitize workload ok")
