@@ -474,9 +474,10 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
   const u32 lt = lanemask_lt();
   bool bad = false, ovf = false, undecl = false, pmiss = false;
   // per chunk, lane j < EX_RPW holds record j's header, slot offset and event base
+  // meta: valid (1) | LD/ST/ATOM (2) | shared (4) | op code << 3 | size_log2 << 5 | (granules - 1) << 8 |
+  // writer << 13 -- decoded once per chunk, in parallel over its records
   struct Ch {
-    uint4 h;
-    u32 uo, eb, sel;
+    u32 mask, meta, sb, uo, eb, sel;
   };
   // load a chunk's headers / offsets and start copying the address rows of its selected records
   auto issue = [&](u64 chunk, int stg) -> Ch {
@@ -484,10 +485,20 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
     const u64 r0 = chunk * EX_RPW;
     const u64 rl = r0 + (u64)(lane & (EX_RPW - 1));
     const bool have = lane < EX_RPW && rl < n;
-    c.h = have ? __ldg(hdr16 + R0 + rl) : make_uint4(0, 0, 0xFFu, 0);
+    const uint4 h = have ? __ldg(hdr16 + R0 + rl) : make_uint4(0, 0, 0xFFu, 0);
     c.uo = have ? (u32)(__ldg(cum + R0 + rl) - cum0 - (u64)REC_W * rl) : 0u;
     c.eb = have ? (u32)(((gidx ? (u64)__ldg(gidx + R0 + rl) : R0 + rl) - G0) << 5) : 0u;
-    c.sel = __ballot_sync(0xFFFFFFFFu, have && (c.h.z & 0xFFu) <= BC_OP_AR_GLB);
+    const u32 op = h.z & 0xFFu, space = (h.z >> 8) & 0xFFu, sl = (h.z >> 16) & 0xFFu, fl = (h.z >> 24) & 0xFFu;
+    c.sel = __ballot_sync(0xFFFFFFFFu, have && op <= BC_OP_AR_GLB);
+    const bool rv = have && op <= BC_OP_AR_GLB && sl <= 4 && space <= 1 && h.x < g.n_warps;
+    const u32 nk = rv ? max(1u, (1u << sl) >> g.G) : 1u;
+    const u32 opc = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM
+                                                             : (((fl & BC_REC_SAME_VALUE) || (g.flags & GEO_F_VALUES))
+                                                                    ? IOP_ST_SV : IOP_ST);
+    c.mask = h.y;
+    c.meta = (u32)rv | ((u32)(op <= BC_OP_ATOM) << 1) | ((u32)(space == BC_SPACE_SHARED) << 2) | (opc << 3) |
+             ((sl & 7u) << 5) | ((nk - 1u) << 8) | ((u32)(op != BC_OP_LD) << 13);
+    c.sb = (rv && space == BC_SPACE_SHARED) ? shared_base + blk_of(g, h.x) * g.smem_gran : 0u;
     // two rows per instruction: lanes 0-15 the k-th selected record, lanes 16-31 the (k+1)-th
     u32 m = c.sel;
     while (m) {
@@ -522,39 +533,33 @@ __global__ void __launch_bounds__(EX_THREADS) k_expand(const bc_record* __restri
       mem &= mem - 1;
       const u32 uoj = __shfl_sync(0xFFFFFFFFu, cur.uo, j);
       const u32 evb = __shfl_sync(0xFFFFFFFFu, cur.eb, j);
-      const u32 hwarp = __shfl_sync(0xFFFFFFFFu, cur.h.x, j), hmask = __shfl_sync(0xFFFFFFFFu, cur.h.y, j);
-      const u32 hz = __shfl_sync(0xFFFFFFFFu, cur.h.z, j);
-      const u32 op = hz & 0xFFu, space = (hz >> 8) & 0xFFu, sl = (hz >> 16) & 0xFFu, fl = (hz >> 24) & 0xFFu;
-      if (!(((hmask >> lane) & 1u) && sl <= 4 && space <= 1 && hwarp < g.n_warps)) continue;
+      const u32 hmask = __shfl_sync(0xFFFFFFFFu, cur.mask, j), meta = __shfl_sync(0xFFFFFFFFu, cur.meta, j);
+      const u32 sb = __shfl_sync(0xFFFFFFFFu, cur.sb, j);
+      if (!((meta & 1u) && ((hmask >> lane) & 1u))) continue;
       const u64 a = crow[j * 32 + lane];
-      const u64 size = 1ull << sl;
-      if (a & (size - 1)) bad = true;  // natural alignment
-      if (space == BC_SPACE_SHARED && a + size > g.smem) bad = true;
-      if (op > BC_OP_ATOM) continue;
-      u32 nk = (u32)(size >> g.G);
-      if (nk == 0) nk = 1;
-      const u32 opc = op == BC_OP_LD ? IOP_LD : op == BC_OP_ATOM ? IOP_ATOM
-                                                               : (((fl & BC_REC_SAME_VALUE) || (g.flags & GEO_F_VALUES))
-                                                                      ? IOP_ST_SV : IOP_ST);
+      const u32 alo = (u32)a, ahi = (u32)(a >> 32);
+      const u32 sl = (meta >> 5) & 7u;
+      if (alo & ((1u << sl) - 1u)) bad = true;  // natural alignment
+      if ((meta & 4u) && a + (1ull << sl) > g.smem) bad = true;
+      if (!(meta & 2u)) continue;  // ACQ / REL / AR: alignment only
+      const u32 nk = ((meta >> 8) & 31u) + 1u;
+      const u32 opc = (meta >> 3) & 3u;
       u32 key0 = KEY_DROP;
       if (bad) {
-      } else if (space == BC_SPACE_SHARED) {
-        key0 = shared_base + blk_of(g, hwarp) * g.smem_gran + (u32)(a >> g.G);
+      } else if (meta & 4u) {
+        key0 = sb + (alo >> g.G);  // shared: a < smem_bytes
+      } else if (ahi < (1u << 16)) {  // < 2^48: 2^28 1-MB pages
+        const u32 p = (ahi << 12) | (alo >> 20);
+        const u32 pw = __ldg(&page_bits[p >> 5]);
+        const u32 bit = p & 31u;
+        if ((pw >> bit) & 1u)
+          key0 = (__ldg(&page_rank[p >> 5]) + __popc(pw & ((1u << bit) - 1u))) << (20 - g.G) | ((alo & 0xFFFFFu) >> g.G);
+        else if (g.flags & GEO_F_DECLARED)
+          undecl = true;  // streaming: the page set is the declared allocations, nothing may fall outside
+        else if (meta & (1u << 13))
+          pmiss = true;   // a write outside the (sampled) page set: the set is incomplete
       } else {
-        const u64 p = a >> 20;
-        if (p < (1ull << 28)) {
-          const u32 pw = __ldg(&page_bits[p >> 5]);
-          const u32 bit = (u32)(p & 31);
-          if ((pw >> bit) & 1u)
-            key0 = (__ldg(&page_rank[p >> 5]) + __popc(pw & ((1u << bit) - 1u))) << (20 - g.G) |
-                   (u32)((a & 0xFFFFFull) >> g.G);
-          else if (g.flags & GEO_F_DECLARED)
-            undecl = true;  // streaming: the page set is the declared allocations, nothing may fall outside
-          else if (op != BC_OP_LD)
-            pmiss = true;   // a write outside the (sampled) page set: the set is incomplete
-        } else {
-          ovf = true;
-        }
+        ovf = true;
       }
       const u32 o = uoj + (u32)__popc(hmask & lt) * nk;  // window slots < 2^30
       const u32 ev = evb | (u32)lane;                    // window-local event id
