@@ -381,7 +381,10 @@ constexpr size_t KT_WARP_BYTES = (size_t)KT_PITCH * (sizeof(uint4) + 2 * sizeof(
 // knows only the window's upper bound, which can be far larger: C4's never-written pages drop 38 % of
 // the slots): CTA c owns the blocks [c * G, (c + 1) * G), G a multiple of 64 (whole K7a chunks, and
 // whole 8-block chunks), nct <= K7A_CTAS CTAs with blocks.
-constexpr u32 K7A_CTAS = 148 * 4;
+#ifndef KA_MINB
+#define KA_MINB 4  // K7a CTAs per SM
+#endif
+constexpr u32 K7A_CTAS = 148 * KA_MINB;
 struct K7Part {
   u32 nblk, G, nct;
 };
@@ -566,17 +569,19 @@ constexpr int KB_STAGES = KB_STAGES_;
 #define KA_UNROLL 2  // the tile's blocks interleaved (A/B on C4: 159 -> 150 us)
 #endif
 constexpr int KA_UNR = KA_UNROLL;
-constexpr int KA_TILE = 512;                     // items per K7a warp per chunk (independent of the block size:
+constexpr int KA_TILE = 512;
+constexpr u32 KA_MAXG = 8192;  // blocks per K7a CTA: a window holds < 2^30 items, so G <= 7104                     // items per K7a warp per chunk (independent of the block size:
 constexpr int KA_BPT = KA_TILE / KT_BLK;         //  K7b's blocks are shorter, K7a's tiles stay long)
 static_assert(KA_TILE % KT_BLK == 0 && KT_BLK % 128 == 0, "K7a tiles hold whole blocks of whole 128-item rounds");
 constexpr int KB_CHUNK = KT_SWARPS * KA_TILE;    // items per chunk
 constexpr int KB_ROW = KB_CHUNK + 8;             // words per stage
 constexpr size_t KB_SMEM = (size_t)KB_STAGES * KB_ROW * sizeof(u32);
-__global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum* __restrict__ sums,
+__global__ void __launch_bounds__(KT_SWARPS * 32, KA_MINB) k_blk_sum(CheckArgs a, Sum* __restrict__ sums,
                                                             u32* __restrict__ wl, u32* __restrict__ wl_cnt) {
   extern __shared__ __align__(128) u32 kb_smem[];  // [KB_STAGES][KB_ROW] key words
   u32 (*const s_keys)[KB_ROW] = reinterpret_cast<u32 (*)[KB_ROW]>(kb_smem);
   __shared__ u64 s_bar[KB_STAGES];
+  __shared__ u32 s_nt[KA_MAXG / 32];  // the CTA's blocks with a check (bitmap)
   const u32 wi = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const u64 n = *a.n_dev;
   const K7Part P = k7_part(n);
@@ -600,6 +605,7 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum*
     for (int q = 0; q < KB_STAGES; ++q) mbar_init(&s_bar[q], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  for (u32 q = threadIdx.x; q < KA_MAXG / 32; q += KT_SWARPS * 32) s_nt[q] = 0;
   __syncthreads();
   if (threadIdx.x == 0)
     for (int q = 0; q < KB_STAGES; ++q)
@@ -672,12 +678,8 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum*
         bs.fi = NONE;
         bs.bits = (bs.fk == bs.lk ? SB_ONE : 0u) | (mlw ? SB_W : 0u);
         if (lane == 0) sums[blk] = bs;
-      } else {  // summarised by a bounded tail walk (its key and event words are in L2), listed for K7b
-        bs = tail_sum_nl(a.k, bb, bb + nb);
-        if (lane == 0) {
-          sums[blk] = bs;
-          wl[atomicAdd(wl_cnt, 1u)] = blk;
-        }
+      } else if (lane == 0) {  // tail-walked after the stream (no call in the hot loop), listed for K7b
+        atomicOr(&s_nt[(blk - b0) >> 5], 1u << ((blk - b0) & 31));
       }
     }
     }
@@ -686,6 +688,21 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, 4) k_blk_sum(CheckArgs a, Sum*
     if (threadIdx.x == 0 && c + KB_STAGES < n_chunks) {
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       issue(c + KB_STAGES, st);
+    }
+  }
+  // the blocks with a check: a bounded tail walk each (their words are L2-hot), then listed for K7b
+  for (u32 wd = wi; wd < (b1 - b0 + 31) / 32; wd += KT_SWARPS) {
+    u32 m = s_nt[wd];
+    while (m) {
+      const u32 blk = b0 + wd * 32 + (u32)(__ffs(m) - 1);
+      m &= m - 1;
+      const u64 bb = (u64)blk * KT_BLK;
+      const u32 nb = (u32)(n - bb < (u64)KT_BLK ? n - bb : (u64)KT_BLK);
+      const Sum bs = tail_sum_nl(a.k, bb, bb + nb);
+      if (lane == 0) {
+        sums[blk] = bs;
+        wl[atomicAdd(wl_cnt, 1u)] = blk;
+      }
     }
   }
 }
