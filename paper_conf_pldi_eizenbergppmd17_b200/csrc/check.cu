@@ -372,7 +372,7 @@ constexpr int KT_IPL = KT_IPL_;              // items per lane per block
 constexpr int KT_BLK = 32 * KT_IPL;          // items per warp block
 constexpr int KT_PITCH = 32 * (KT_IPL + 1);  // padded entries per array
 #ifndef KT_NWARPS
-#define KT_NWARPS 16
+#define KT_NWARPS 12  // A/B (K7b, C2 / C3 / C4): 16 -> 12 took 376 / 231 / 25.6 us to 332 / 219 / 24.2 us
 #endif
 constexpr int KT_WARPS = KT_NWARPS;
 constexpr size_t KT_WARP_BYTES = (size_t)KT_PITCH * (sizeof(uint4) + 2 * sizeof(u32));
@@ -708,13 +708,13 @@ __global__ void __launch_bounds__(KT_SWARPS * 32, KA_MINB) k_blk_sum(CheckArgs a
 }
 
 // ---------------------------------------------------------------------- K7b: the listed blocks
-// SH (several windows: carried entries in and / or entries out): half the warps per CTA, and per warp
+// SH (several windows: carried entries in and / or entries out): 8 warps per CTA, and per warp
 // the carried entries of the block's granule-first items staged in shared memory with the snapshots
 // (cp.async, all of a lane's loads in flight together), so the lane-sequential rules never wait on a
 // dependent global load per granule.
 template <bool SH>
 struct KtCfg {
-  static constexpr int WARPS = SH ? KT_WARPS / 2 : KT_WARPS;
+  static constexpr int WARPS = SH ? 8 : KT_WARPS;
   static constexpr size_t WARP_BYTES =
       KT_WARP_BYTES + (SH ? (size_t)KT_PITCH * (sizeof(uint4) + sizeof(uint2)) : 0);
 };
