@@ -635,9 +635,10 @@ __global__ void __launch_bounds__(SS_THREADS) k_sort_small(const u32* __restrict
   if (t == 0 && n_out) *n_out = nk;
 }
 
+// One pass of RB-bit digits at `shift` (pass index p: its row of the digit-total tables).
 template <int RB>
-static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo, int passes, void* temp,
-                       cudaStream_t st, const u64* n_dev, u64* n_out_dev, bool drop) {
+static void rs_pass(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, const u64*& nd, int shift, int p, bool dr,
+                    void* temp, cudaStream_t st, u64* n_out_dev) {
   constexpr int BINS = 1 << RB;
   const u64 tiles = (n + RS_TILE - 1) / RS_TILE;
   u32* ghist = (u32*)temp;                           // [RS_MAXP][RS_MAXB]
@@ -656,28 +657,31 @@ static void rs_sort_rb(u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, int bit_lo
     grid_of[dev] = sms * (per > 0 ? per : 1);
   }
   const int down_grid = grid_of[dev];
-  const u64* nd = n_dev;
-  for (int p = 0; p < passes; ++p) {
-    const int shift = bit_lo + RB * p;
-    const int dr = (drop && p == 0) ? 1 : 0;
-    k_rs_up<RB><<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr, shift, counts, tiles); ++g_launches;
-    k_rs_rows<<<BINS, RS_THREADS, 0, st>>>(counts, tiles, ghist + p * RS_MAXB); ++g_launches;
-    // the digit bases come from the downsweep's own scan of the row totals, unless the kept count it
-    // publishes would overwrite the item count the same launch reads (n_dev == n_out_dev)
-    const bool fused = RS_FUSED_BINS && !(dr && nd == n_out_dev);
-    if (!fused) {
-      k_rs_bins<RB><<<1, BINS < 1024 ? BINS : 1024, 0, st>>>(ghist + p * RS_MAXB, gbase + p * RS_MAXB,
-                                                            dr ? n_out_dev : nullptr);
-      ++g_launches;
-    }
-    k_rs_down<RB><<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, dsmem, st>>>(
-        ki, vi, ko, vo, n, nd, dr, shift, counts, tiles, gbase + p * RS_MAXB, fused ? ghist + p * RS_MAXB : nullptr,
-        fused && dr ? n_out_dev : nullptr);
+  k_rs_up<RB><<<(unsigned)tiles, RS_THREADS, 0, st>>>(ki, n, nd, dr ? 1 : 0, shift, counts, tiles); ++g_launches;
+  k_rs_rows<<<BINS, RS_THREADS, 0, st>>>(counts, tiles, ghist + p * RS_MAXB); ++g_launches;
+  // the digit bases come from the downsweep's own scan of the row totals, unless the kept count it
+  // publishes would overwrite the item count the same launch reads (n_dev == n_out_dev)
+  const bool fused = RS_FUSED_BINS && !(dr && nd == n_out_dev);
+  if (!fused) {
+    k_rs_bins<RB><<<1, BINS < 1024 ? BINS : 1024, 0, st>>>(ghist + p * RS_MAXB, gbase + p * RS_MAXB,
+                                                          dr ? n_out_dev : nullptr);
     ++g_launches;
-    if (dr) nd = n_out_dev;
-    u32* tk = ki; ki = ko; ko = tk;
-    u32* tv = vi; vi = vo; vo = tv;
   }
+  k_rs_down<RB><<<(unsigned)std::min<u64>(tiles, (u64)down_grid), RS_THREADS, dsmem, st>>>(
+      ki, vi, ko, vo, n, nd, dr ? 1 : 0, shift, counts, tiles, gbase + p * RS_MAXB,
+      fused ? ghist + p * RS_MAXB : nullptr, fused && dr ? n_out_dev : nullptr);
+  ++g_launches;
+  if (dr) nd = n_out_dev;
+  u32* tk = ki; ki = ko; ko = tk;
+  u32* tv = vi; vi = vo; vo = tv;
+}
+
+static void rs_pass_any(int rb, u32*& ki, u32*& vi, u32*& ko, u32*& vo, u64 n, const u64*& nd, int shift, int p,
+                        bool dr, void* temp, cudaStream_t st, u64* n_out_dev) {
+  if (rb == 8) rs_pass<8>(ki, vi, ko, vo, n, nd, shift, p, dr, temp, st, n_out_dev);
+  else if (rb == 9) rs_pass<9>(ki, vi, ko, vo, n, nd, shift, p, dr, temp, st, n_out_dev);
+  else if (rb == 10) rs_pass<10>(ki, vi, ko, vo, n, nd, shift, p, dr, temp, st, n_out_dev);
+  else rs_pass<11>(ki, vi, ko, vo, n, nd, shift, p, dr, temp, st, n_out_dev);
 }
 
 // Stable sort of (keys, vals) by key bits [bit_lo, bit_hi) (vals may be null: keys only).  Result is
@@ -717,13 +721,20 @@ bool radix_sort_pairs(u32* keys, u32* vals, u32* keys_alt, u32* vals_alt, u64 n,
   // an 11-bit digit only when it makes the sort single-pass (K1 of 2048-warp traces): the 2048-bin
   // downsweep runs one CTA per SM, which loses to one more 8-10-bit pass when both need passes
   const int mb = bits == 11 ? 11 : maxb;
-  int passes = std::min((bits + mb - 1) / mb, RS_MAXP);
-  const int rb = std::max(8, std::min(mb, (bits + passes - 1) / passes));
+  const int passes = std::min((bits + mb - 1) / mb, RS_MAXP);
+  // digit widths: the fewest passes; the extra bits of a uniform split go to the first passes only
+  // (bits - 8 * passes of them): the other passes run 8-bit digits (256 bins: longer digit runs per
+  // tile, better-coalesced scatter) -- e.g. 25 bits as 9 + 8 + 8 rather than 9 + 9 + 9
   u32 *ki = keys, *vi = vals, *ko = keys_alt, *vo = vals_alt;
-  if (rb == 8) rs_sort_rb<8>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
-  else if (rb == 9) rs_sort_rb<9>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
-  else if (rb == 10) rs_sort_rb<10>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
-  else rs_sort_rb<11>(ki, vi, ko, vo, n, bit_lo, passes, temp, st, n_dev, n_out_dev, drop);
+  const u64* nd = n_dev;
+  int shift = bit_lo, left = bits;
+  for (int p = 0; p < passes; ++p) {
+    const int rem = passes - p;
+    const int rb = std::max(8, std::min(mb, (left + rem - 1) / rem));
+    rs_pass_any(rb, ki, vi, ko, vo, n, nd, shift, p, drop && p == 0, temp, st, n_out_dev);
+    shift += rb;
+    left -= rb;
+  }
   return (passes & 1) != 0;
 }
 
