@@ -266,15 +266,19 @@ __global__ void __launch_bounds__(256, 4) k_replay(const uint4* __restrict__ hdr
     nh = __ldg(hdr16 + nr);
     ng = gidx ? __ldg(gidx + nr) : nr;
   }
+  u32 nr2 = i0 + 32 + lane < i1 ? wrec[i0 + 32 + lane] : 0u;
   for (u32 c0 = i0; c0 < i1 && !bad; c0 += 32) {
     const u32 r = nr, rg = ng;
     const uint4 hv = nh;
     const u32 cnt = min(32u, i1 - c0);
-    if (c0 + 32 + lane < i1) {  // next chunk in flight while this one is stepped through
-      nr = wrec[c0 + 32 + lane];
+    // the next chunk's headers in flight while this one is stepped through (their record indices were
+    // loaded one chunk earlier, so the gather does not wait on them), and the indices of the one after
+    if (c0 + 32 + lane < i1) {
+      nr = nr2;
       nh = __ldg(hdr16 + nr);
       ng = gidx ? __ldg(gidx + nr) : nr;
     }
+    if (c0 + 64 + lane < i1) nr2 = wrec[c0 + 64 + lane];
     s_hdr[wib][lane] = hv;
     s_rec[wib][lane] = rg;
     __syncwarp();
