@@ -88,6 +88,52 @@ __global__ void k_emit_findings(const u32* __restrict__ fblk, const u32* __restr
   out[i] = o;
 }
 
+// Few races (n <= FR_SMALL): one CTA sorts the permutation in shared memory by the canonical key
+// (granule key, current record, current lane, prior record, prior lane) -- a bitonic sort over the race
+// records themselves (they are distinct: one per failed check) -- instead of five LSD passes of
+// (field extraction + radix sort + gather) launches.
+constexpr u32 FR_SMALL = 4096;
+__device__ __forceinline__ bool race_less(const uint4& a, const uint4& b) {
+  if (a.x != b.x) return a.x < b.x;
+  if (a.y != b.y) return a.y < b.y;
+  if ((a.w & 31u) != (b.w & 31u)) return (a.w & 31u) < (b.w & 31u);
+  if (a.z != b.z) return a.z < b.z;
+  return ((a.w >> 5) & 31u) < ((b.w >> 5) & 31u);
+}
+__global__ void __launch_bounds__(1024) k_sort_races_small(const uint4* __restrict__ r, u32 n,
+                                                           u32* __restrict__ perm) {
+  extern __shared__ __align__(16) unsigned char fr_smem[];
+  uint4* const sr = reinterpret_cast<uint4*>(fr_smem);                        // [FR_SMALL]
+  unsigned short* const si = reinterpret_cast<unsigned short*>(sr + FR_SMALL);  // [FR_SMALL]
+  u32 m = 1;
+  while (m < n) m <<= 1;
+  for (u32 i = threadIdx.x; i < m; i += blockDim.x) {
+    sr[i] = i < n ? r[i] : make_uint4(0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu);
+    si[i] = (unsigned short)i;
+  }
+  __syncthreads();
+  for (u32 k = 2; k <= m; k <<= 1) {
+    for (u32 j = k >> 1; j > 0; j >>= 1) {
+      for (u32 i = threadIdx.x; i < m; i += blockDim.x) {
+        const u32 l = i ^ j;
+        if (l > i) {
+          const bool up = (i & k) == 0;
+          const uint4 a = sr[i], b = sr[l];
+          if (race_less(b, a) == up) {  // out of order for this half: swap
+            sr[i] = b;
+            sr[l] = a;
+            const unsigned short t = si[i];
+            si[i] = si[l];
+            si[l] = t;
+          }
+        }
+      }
+      __syncthreads();
+    }
+  }
+  for (u32 i = threadIdx.x; i < n; i += blockDim.x) perm[i] = si[i];
+}
+
 int bits_for(u64 maxval) {
   int b = 0;
   while (b < 32 && (maxval >> b)) ++b;
@@ -113,7 +159,19 @@ void finalize_races(const uint4* races, u32 n_r, const u32* fblk, const u32* fre
     sort_perm_by(p, fblk, n_f, bits_for(g.n_blocks), S, st);
     k_emit_findings<<<nb(n_f), 256, 0, st>>>(fblk, frec, p, n_f, out); ++g_launches;
   }
-  if (n_r) {
+  if (n_r && n_r <= FR_SMALL) {
+    u32* p = S.alloc<u32>(n_r);
+    constexpr size_t smem = FR_SMALL * (sizeof(uint4) + sizeof(unsigned short));
+    static bool attr[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev >= 0 && dev < 64 && !attr[dev]) {
+      cudaFuncSetAttribute(k_sort_races_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      attr[dev] = true;
+    }
+    k_sort_races_small<<<1, 1024, smem, st>>>(races, n_r, p); ++g_launches;
+    k_emit_races<<<nb(n_r), 256, 0, st>>>(races, p, n_r, g, snap, page_num, shared_base, out + n_f); ++g_launches;
+  } else if (n_r) {
     u32* p = S.alloc<u32>(n_r);
     u32* f = S.alloc<u32>(n_r);
     launch_iota(p, n_r, st);
@@ -129,7 +187,7 @@ void finalize_races(const uint4* races, u32 n_r, const u32* fblk, const u32* fre
 }
 
 void preload_finalize() {
-  preload(k_emit_findings, k_emit_races, k_field, k_page_list);
+  preload(k_emit_findings, k_emit_races, k_field, k_page_list, k_sort_races_small);
 }
 
 }  // namespace bc
