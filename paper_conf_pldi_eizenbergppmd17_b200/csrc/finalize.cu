@@ -4,7 +4,8 @@
 // kind << 10) in arbitrary order (global record indices: any trace length).  The dense key order is
 // the canonical location order (global granules by address, then shared granules by (block,
 // offset)), so a stable LSD sort by prior (lane, record), then current (lane, record), then key gives
-// the canonical (location, current event, prior event) order, event = record << 5 | lane.  Classification from the two events
+// the canonical (location, current event, prior event) order, event = record << 5 | lane (up to
+// FR_SMALL races: one CTA bitonic-sorts by that composite key directly; the records are distinct).  Classification from the two events
 // (reading R9): same record -> SAME_INSN; same warp -> BRANCH (branch ordering,
 // P:L591-630); same block -> INTRA_BLOCK; else INTER_BLOCK.  Barrier-divergence findings
 // come first, ordered by (block, record).

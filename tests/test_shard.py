@@ -284,3 +284,99 @@ def test_sharded_litmus_suite():
             continue
         got, _ = _replicated(recs, geom, 4)
         assert np.array_equal(got.view(np.uint8), want.view(np.uint8)), name
+
+
+# ----------------------------------------------------------------------------- item exchange (row e)
+def _mix_owner(g: np.ndarray, world: int) -> np.ndarray:
+    """Test model of the owner rule of the sharded data plane (shard.cu k_dest / common.cuh shard_of):
+    a murmur3 finaliser of the granule, then a multiply-shift to [0, world)."""
+    k = g.astype(np.uint64) & np.uint64(0xFFFFFFFF)
+    k ^= k >> np.uint64(16)
+    k = (k * np.uint64(0x85EBCA6B)) & np.uint64(0xFFFFFFFF)
+    k ^= k >> np.uint64(13)
+    k = (k * np.uint64(0xC2B2AE35)) & np.uint64(0xFFFFFFFF)
+    k ^= k >> np.uint64(16)
+    return ((k * np.uint64(world)) >> np.uint64(32)).astype(np.int64)
+
+
+def _items(recs, idx, geom):
+    """(granule id, global event) of every memory lane op of the records, in trace order (a model of
+    K4 for the exchange test: global granules by address, shared granules tagged by block)"""
+    G = geom.get("granule_log2", 2)
+    wpb = (geom["block"][0] + 31) // 32
+    out_g, out_e = [], []
+    for rec, gi in zip(recs, idx):
+        if rec["op"] > 2:  # LD / ST / ATOM only
+            continue
+        for l in range(32):
+            if (int(rec["mask"]) >> l) & 1:
+                a = int(rec["addr"][l])
+                if rec["space"] == 1:  # shared: (block, offset), never leaves its block's rank
+                    g = (1 << 62) | ((int(rec["warp"]) // wpb) << 32) | (a >> G)
+                else:
+                    g = a >> G
+                out_g.append(g)
+                out_e.append((int(gi) << 5) | l)
+    return np.array(out_g, dtype=np.uint64), np.array(out_e, dtype=np.int64)
+
+
+def _exchange_worker(rank, world, port, path):
+    """One rank of the per-window item exchange over gloo: expand the rank's block shard, route each
+    item to its granule's owner (shared granules stay; global ones by the owner rule) with a stable
+    partition, all-to-all the (granule, event) pairs, then sort by event and stably by granule."""
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    recs = np.load(path)
+    geom = dict(grid=(12, 1, 1), block=(256, 1, 1), smem_bytes=16, granule_log2=2)
+    loc, idx = bc.shard_trace(recs, geom, rank, world)
+    g, e = _items(loc, idx, geom)
+    shared = (g >> np.uint64(62)) == 1
+    dest = np.where(shared, rank, _mix_owner(g, world))
+    order = np.argsort(dest, kind="stable")
+    counts = np.bincount(dest, minlength=world).astype(np.int64)
+    rc = torch.zeros(world, dtype=torch.int64)
+    dist.all_to_all_single(rc, torch.from_numpy(counts))
+    rc = rc.numpy()
+    payload = torch.from_numpy(np.stack([g[order].astype(np.int64), e[order]], axis=1).reshape(-1))
+    recv = torch.zeros(int(rc.sum()) * 2, dtype=torch.int64)
+    dist.all_to_all_single(recv, payload, [int(c) * 2 for c in rc], [int(c) * 2 for c in counts])
+    got = recv.numpy().reshape(-1, 2)
+    got = got[np.argsort(got[:, 1], kind="stable")]        # trace order
+    got = got[np.argsort(got[:, 0], kind="stable")]        # then grouped by granule
+    np.save(f"{path}.{rank}.npy", got)
+    dist.destroy_process_group()
+
+
+def test_item_exchange_over_gloo(tmp_path):
+    """Row e's per-window data plane over a world-size-2 gloo group: after the all-to-all every granule
+    lives on exactly one rank, each rank's items are grouped by granule in global trace order, and the
+    union equals the single-rank expansion of the whole trace."""
+    import socket
+
+    import torch.multiprocessing as mp
+    recs, geom = _c4_small()
+    path = str(tmp_path / "trace.npy")
+    np.save(path, recs)
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    mp.spawn(_exchange_worker, args=(2, port, path), nprocs=2, join=True)
+    parts = [np.load(f"{path}.{r}.npy") for r in range(2)]
+    g_all, e_all = _items(recs, np.arange(len(recs)), dict(geom, granule_log2=2))
+    want = np.stack([g_all.astype(np.int64), e_all], axis=1)
+    want = want[np.argsort(want[:, 0], kind="stable")]
+    assert sum(len(p) for p in parts) == len(want)
+    owners = {}
+    for r, p in enumerate(parts):
+        assert np.all(np.diff(p[:, 0]) >= 0)
+        same = p[1:, 0] == p[:-1, 0]
+        assert np.all(np.diff(p[:, 1])[same] > 0)  # trace order inside a granule
+        for gk in np.unique(p[:, 0]):
+            assert owners.setdefault(int(gk), r) == r  # one owner per granule
+    merged = np.concatenate(parts)
+    merged = merged[np.lexsort((merged[:, 1], merged[:, 0]))]
+    assert np.array_equal(merged, want)
