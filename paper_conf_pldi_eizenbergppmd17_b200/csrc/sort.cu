@@ -489,23 +489,48 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_u32(const u32* __restrict__
   __shared__ u64 wsum[SC_THREADS / 32];
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
   const u64 base = (u64)blockIdx.x * SC_TILE + (u64)t * SC_ITEMS;
+  static_assert(SC_ITEMS == 8, "two 16-B loads per thread");
   u32 v[SC_ITEMS];
   u64 sum = 0;
+  // vector path: a whole 8-word group and 16-B aligned arrays (base is a multiple of 8 words; callers may
+  // pass arrays that start inside a buffer, e.g. the barrier counts after the IF counts)
+  const bool full = base + SC_ITEMS <= n && (((uintptr_t)in | (uintptr_t)out) & 15u) == 0;
+  if (full) {
+    const uint4 a = __ldg(reinterpret_cast<const uint4*>(in + base));
+    const uint4 b = __ldg(reinterpret_cast<const uint4*>(in + base) + 1);
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+  } else {
 #pragma unroll
-  for (int j = 0; j < SC_ITEMS; ++j) {
-    v[j] = base + j < n ? in[base + j] : 0u;
-    sum += v[j];
+    for (int j = 0; j < SC_ITEMS; ++j) v[j] = base + j < n ? in[base + j] : 0u;
   }
+#pragma unroll
+  for (int j = 0; j < SC_ITEMS; ++j) sum += v[j];
   const u64 x = warp_incl_sum(sum);
   if (l == 31) wsum[w] = x;
   __syncthreads();
   u64 off = 0;
   for (int ww = 0; ww < w; ++ww) off += wsum[ww];
   u64 run = texcl[blockIdx.x] + off + x - sum;
+  TO o[SC_ITEMS];
 #pragma unroll
   for (int j = 0; j < SC_ITEMS; ++j) {
-    if (base + j < n) out[base + j] = (TO)run;
+    o[j] = (TO)run;
     run += v[j];
+  }
+  if (full) {  // 16-B stores (out + base is 32-B / 64-B aligned)
+    constexpr int PER16 = 16 / (int)sizeof(TO);
+#pragma unroll
+    for (int j = 0; j < SC_ITEMS; j += PER16) {
+      if constexpr (sizeof(TO) == 8) {
+        *reinterpret_cast<ulonglong2*>(out + base + j) = make_ulonglong2(o[j], o[j + 1]);
+      } else {
+        *reinterpret_cast<uint4*>(out + base + j) = make_uint4(o[j], o[j + 1], o[j + 2], o[j + 3]);
+      }
+    }
+  } else {
+#pragma unroll
+    for (int j = 0; j < SC_ITEMS; ++j)
+      if (base + j < n) out[base + j] = o[j];
   }
 }
 
